@@ -1,0 +1,36 @@
+-- TPC-H Q1, Q3, Q5, Q6 with validation parameters (BASELINE config 4; the paper
+-- runs TPC-H, PAPER.md:305, :595).  Texts: SURVEY.md App. A.2, rewritten for the
+-- stored representation ONLY as the DESIGN.md readings require:
+--   O5  decimals are scale-2 integers: (1 - l_discount) -> (100 - l_discount),
+--       (1 + l_tax) -> (100 + l_tax); 0.05..0.07 -> 5..7; quantity < 24 -> < 2400.
+--       Results are therefore scaled integers (scale 2, 4 or 6).
+--   O11 dates are int yyyymmdd and date arithmetic is folded:
+--       date '1998-12-01' - interval '90' day = 19980902,
+--       date '1994-01-01' + interval '1' year = 19950101.
+--   avg(x) is reported as sum(x) and count(*) (O10: the average is a double
+--   computed at finalisation).  Q1's avg_disc uses sum(l_discount).
+--   LIMIT 10 of Q3 is dropped here so the whole pre-LIMIT group set is compared (O9).
+-- Used by tests/test_oracle_sqlite.py (SQLite 3.45) to pin the oracle.
+-- @tpch1
+select l_returnflag, l_linestatus, sum(l_quantity), sum(l_extendedprice),
+       sum(l_extendedprice*(100-l_discount)), sum(l_extendedprice*(100-l_discount)*(100+l_tax)),
+       sum(l_discount), count(*)
+  from lineitem where l_shipdate <= 19980902
+ group by l_returnflag, l_linestatus order by l_returnflag, l_linestatus;
+-- @tpch3
+select l_orderkey, o_orderdate, o_shippriority, sum(l_extendedprice*(100-l_discount)) as revenue
+  from customer, orders, lineitem
+ where c_mktsegment = 'BUILDING' and c_custkey = o_custkey and l_orderkey = o_orderkey
+   and o_orderdate < 19950315 and l_shipdate > 19950315
+ group by l_orderkey, o_orderdate, o_shippriority order by revenue desc, o_orderdate;
+-- @tpch5
+select n_name, sum(l_extendedprice*(100-l_discount)) as revenue
+  from customer, orders, lineitem, supplier, nation, region
+ where c_custkey = o_custkey and l_orderkey = o_orderkey and l_suppkey = s_suppkey
+   and c_nationkey = s_nationkey and s_nationkey = n_nationkey and n_regionkey = r_regionkey
+   and r_name = 'ASIA' and o_orderdate >= 19940101 and o_orderdate < 19950101
+ group by n_name order by revenue desc;
+-- @tpch6
+select sum(l_extendedprice*l_discount) as revenue, count(*) from lineitem
+ where l_shipdate >= 19940101 and l_shipdate < 19950101
+   and l_discount between 5 and 7 and l_quantity < 2400;
