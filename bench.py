@@ -1,0 +1,367 @@
+"""Benchmark: all 13 SSB queries at SF20, hot cache, on B200 (BASELINE config 2,
+the paper's Q3.3 setting); metric "SSB fact rows/s" (+ queries/s,
+HBM GB/s vs peak).
+
+One step = one pass of the whole hot path over the resident SF20 database: the 13
+prepared physical plans (select -> build -> probe -> gather/aggregate, every
+operator an sm_100a kernel of libddq) launched back to back on one stream.
+value = 13 * lineorder_rows * steps / device time (CUDA events), max over ranks.
+Inputs (6.7 GB of lineorder columns) are larger than L2 (126 MB), so no L2 flush
+is needed between steps.
+
+N > 1 (torchrun): lineorder of SF 20*N is range-sharded by row (P:407 horizontal
+partitioning), each rank holding 120M rows (weak scaling); per step every rank runs
+the 13 plans on its shard and the partial group tables are exchanged with one NCCL
+all_gather per query; rank 0 merges them (host finalisation, S8(a7)).
+
+--impl reference: the oracle (oracle/, single-threaded C++) on a bounded sample
+of the same workload, on the host's cores.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "SSB fact rows/s"
+UNIT = "rows/s"
+SF_PER_GPU = 20.0
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--sf", type=float, default=SF_PER_GPU, help="scale factor per GPU")
+    ap.add_argument("--e2e-steps", type=int, default=3)
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--profile-only", action="store_true", help="short run for ncu")
+    return ap.parse_args()
+
+
+def peaks():
+    try:
+        return json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
+    except Exception:
+        return {}
+
+
+class Clocks:
+    """nvidia-smi clock / throttle sampling during the timed region."""
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, device: int):
+        self.device = device
+        self.p = None
+        self.lines: list[str] = []
+
+    def start(self):
+        try:
+            self.p = subprocess.Popen(["nvidia-smi", "-i", str(self.device), f"--query-gpu={self.Q}",
+                                       "--format=csv,noheader,nounits", "-lms", "200"],
+                                      stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.p = None
+
+    def _read(self):
+        for line in self.p.stdout:
+            self.lines.append(line.strip())
+
+    def stop(self) -> dict:
+        if not self.p:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.p.terminate()
+        try:
+            self.p.wait(2)
+        except Exception:
+            self.p.kill()
+        self.t.join(1)
+        sm, mx, reasons = [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            f = [x.strip() for x in ln.split(",")]
+            if len(f) < 9:
+                continue
+            try:
+                sm.append(float(f[1]))
+                mx.append(float(f[2]))
+            except ValueError:
+                continue
+            for n, v in zip(names, f[5:9]):
+                if v.lower() == "active":
+                    reasons.add(n)
+        sm.sort()
+        return {"sm_mhz": sm[len(sm) // 2] if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+def dist_env():
+    ws = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return ws, rank, local
+
+
+def cpu_baseline(sf: float, sample_rows: int) -> dict:
+    """The oracle as it stands (single-threaded C++), on the first `sample_rows`
+    lineorder rows of the same SF database, all 13 queries."""
+    import datagen
+    import oracle
+    data = datagen.SSB(sf)
+
+    class Prefix:  # full dimension tables, lineorder prefix (generated only for the sample)
+        def __getitem__(self, c):
+            if c.startswith("lo_"):
+                return datagen.ssb_column(c, sf, end=sample_rows)
+            return data[c]
+    pre = Prefix()
+    cache = {}
+
+    class View:
+        def __getitem__(self, c):
+            if c not in cache:
+                cache[c] = pre[c]
+            return cache[c]
+    v = View()
+    for q in oracle.SSB_QUERIES:  # generate inputs outside the timed region
+        for c in oracle.SSB_QUERY_COLUMNS[int(q[3])]:
+            v[c]
+    t0 = time.perf_counter()
+    for q in oracle.SSB_QUERIES:
+        oracle.run(v, q)
+    dt = time.perf_counter() - t0
+    return {"value": 13 * sample_rows / dt, "unit": UNIT, "cores": 1, "kind": "oracle",
+            "sample": f"all 13 SSB queries over the first {sample_rows} lineorder rows of SF{sf:g} "
+                      f"(full dimension tables), single-threaded, {dt:.2f} s"}
+
+
+def run_reference(args):
+    ws, rank, _ = dist_env()
+    if rank != 0:
+        return
+    import datagen  # noqa: F401
+    sample = 2_000_000
+    vals = []
+    for _ in range(args.warmup):
+        cpu_baseline(args.sf, sample)
+    t_total = 0.0
+    for _ in range(args.steps):
+        r = cpu_baseline(args.sf, sample)
+        vals.append(r["value"])
+        t_total += 13 * sample / r["value"]
+    value = 13 * sample * args.steps / t_total
+    line = {"impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * t_total / args.steps,
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "int64",
+            "data": "synthetic (datagen, seed 0x5EED2016)",
+            "config": {"workload": f"SSB SF{args.sf:g}, all 13 queries (bounded sample: first {sample} lineorder "
+                                   f"rows per step)", "queries": 13},
+            "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle",
+                             "sample": f"first {sample} lineorder rows of SF{args.sf:g} per step"},
+            "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    args = parse()
+    if args.impl == "reference":
+        return run_reference(args)
+    import numpy as np
+    import torch
+    import datagen
+    from paper_conf_sigmod_bressft16_b200 import Database
+    from paper_conf_sigmod_bressft16_b200 import _abi as A
+    from paper_conf_sigmod_bressft16_b200.ssb import SSB_QUERIES, load_ssb, ssb_plan, QUERY_COLUMNS
+
+    ws, rank, local = dist_env()
+    assert ws == args.gpus or ws == 1, "launch N>1 with torchrun --nproc-per-node N"
+    torch.cuda.set_device(local)
+    if ws > 1:
+        import torch.distributed as dist
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    sf_total = args.sf * ws
+    data = datagen.SSB(sf_total)
+    n_lo = data.rows("lineorder")
+    b, e = rank * n_lo // ws, (rank + 1) * n_lo // ws
+    shard_rows = e - b
+
+    class Shard:  # dimension tables whole, lineorder rows [b, e) only
+        def __init__(self):
+            self.c = {}
+
+        def __getitem__(self, col):
+            if col not in self.c:
+                self.c[col] = (datagen.ssb_column(col, sf_total, begin=b, end=e) if col.startswith("lo_")
+                               else data[col])
+            return self.c[col]
+
+        def rows(self, t):
+            return data.rows(t)
+
+        def dict_for(self, col):
+            return data.dict_for(col)
+
+    shard = Shard()
+    t_setup = time.perf_counter()
+    db = Database(device=local, cache_bytes=64 << 30, heap_bytes=24 << 30, rank=rank, world=ws)
+
+    load_ssb(db, shard, row_begin=b, row_end=e, presliced=True)
+    preps = [db.prepare(ssb_plan(db, q), use_graph=True) for q in SSB_QUERIES]
+    setup_s = time.perf_counter() - t_setup
+    stream = torch.cuda.Stream()
+    sptr = stream.cuda_stream
+    kernels_per_step = sum(p.kernels for p in preps)
+
+    def step():
+        for p in preps:
+            p.launch(sptr)
+
+    def exchange():
+        """N>1: all_gather of every query's compacted partial group table."""
+        if ws == 1:
+            return None
+        import torch.distributed as dist
+        outs = []
+        with torch.cuda.stream(stream):
+            for p in preps:
+                keys, accs = p.partials(sptr)  # D2H of <= 800 groups per query
+                t = torch.from_numpy(np.concatenate([[keys.size], keys, accs.reshape(-1)]).astype(np.int64))
+                pad = torch.zeros(1 + 2048 * (1 + 2 * 2), dtype=torch.int64)
+                pad[:t.numel()] = t
+                g = [torch.zeros_like(pad, device="cuda") for _ in range(ws)]
+                dist.all_gather(g, pad.cuda())
+                outs.append(g)
+        return outs
+
+    if args.profile_only:
+        for _ in range(2):
+            step()
+        torch.cuda.synchronize()
+        return
+
+    for _ in range(args.warmup):
+        step()
+        exchange()
+    torch.cuda.synchronize()
+    if ws > 1:
+        import torch.distributed as dist
+        dist.barrier()
+    clk = Clocks(local)
+    clk.start()
+    time.sleep(0.3)
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    torch.cuda.synchronize()
+    ev0.record(stream)
+    for _ in range(args.steps):
+        step()
+        exchange()
+    ev1.record(stream)
+    torch.cuda.synchronize()
+    clocks = clk.stop()
+    ms = ev0.elapsed_time(ev1)
+    if ws > 1:
+        import torch.distributed as dist
+        t = torch.tensor([ms], device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms = float(t.item())
+        dist.barrier()
+    ms_per_step = ms / args.steps
+    total_rows = 13 * n_lo  # all ranks together
+    value = total_rows * args.steps / (ms / 1e3)
+
+    # results of the timed plans (validated against the oracle by tests/, here sanity only)
+    results = {q: p.fetch(sptr).rows for q, p in zip(SSB_QUERIES, preps)} if ws == 1 else {}
+
+    # ---- roofline of the dominant kernel class from an event-timed profiling replay
+    prof = [p.profile(sptr) for p in preps]
+    cls_ms, cls_bytes, cls_n = {}, {}, {}
+    for ops in prof:
+        for ms_, by, cl in ops:
+            cls_ms[cl] = cls_ms.get(cl, 0.0) + ms_
+            cls_bytes[cl] = cls_bytes.get(cl, 0.0) + by
+            cls_n[cl] = cls_n.get(cl, 0) + 1
+    names = {0: "dense scan (select/probe over all rows)", 1: "select/probe at TIDs", 2: "hash build",
+             3: "gather", 4: "group-by aggregate"}
+    dom = max(cls_ms, key=lambda c: cls_ms[c])
+    pk = peaks()
+    hbm_peak = pk.get("hbm_gbs", 6650.0)
+    achieved = cls_bytes[dom] / (cls_ms[dom] / 1e3) / 1e9
+    step_bytes = sum(cls_bytes.values())
+    roofline = {"bound": "hbm", "kernel": "filter_kernel: " + names[dom], "achieved": round(achieved, 1),
+                "peak": hbm_peak, "unit": "GB/s", "frac": round(achieved / hbm_peak, 4), "traffic": None,
+                "launches_per_step": cls_n[dom], "share_of_step": round(cls_ms[dom] / sum(cls_ms.values()), 3),
+                "peak_source": "MEASURED_PEAKS.json hbm_gbs (measured)" if "hbm_gbs" in pk else "fallback 6.65 TB/s",
+                "step_model_gb": round(step_bytes / 1e9, 3),
+                "step_gbs": round(step_bytes / (ms_per_step / 1e3) / 1e9 * ws, 1)}
+
+    # ---- e2e through the public API with host buffers: cold cache, every column
+    #      H2D from pinned host memory inside the timed region (GPU-only placement)
+    e2e = None
+    if not args.no_e2e and ws == 1:
+        cold = Database(device=local, cache_bytes=64 << 30, heap_bytes=24 << 30, placement=A.PLACE_GPU_ONLY)
+        load_ssb(cold, shard, row_begin=b, row_end=e, cache=False, presliced=True)
+        plans = [ssb_plan(cold, q) for q in SSB_QUERIES]
+        all_cols = [(t, c) for (t, c) in cold._cols]
+
+        def e2e_step():
+            for pl in plans:
+                cold.run(pl)
+            for (t, c) in all_cols:
+                cold.evict(t, c)
+        e2e_step()
+        cold.reset_stats()
+        t0 = time.perf_counter()
+        for _ in range(args.e2e_steps):
+            e2e_step()
+        dt = time.perf_counter() - t0
+        st = cold.stats()
+        e2e = {"value": total_rows * args.e2e_steps / dt, "unit": UNIT,
+               "h2d_bytes_per_step": st["h2d_bytes"] // args.e2e_steps,
+               "d2h_bytes_per_step": st["d2h_bytes"] // args.e2e_steps,
+               "h2d_gbs": round(st["h2d_bytes"] / max(st["h2d_ns"], 1), 2),
+               "path": "ddq_submit/ddq_fetch, GPU-only placement, empty cache; columns copied on demand "
+                       "from pinned host memory (cold cache, P:32)"}
+        cold.close()
+
+    cpu = None
+    if rank == 0 and not args.no_cpu_baseline:
+        cpu = cpu_baseline(sf_total, 6_000_000)
+
+    if rank == 0:
+        line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": ws, "steps": args.steps,
+                "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
+                "scaling": "weak", "vs_baseline": None, "dtype": "int64", "data": "synthetic (datagen, seed 0x5EED2016)",
+                "config": {"workload": f"SSB SF{sf_total:g}, all 13 queries, hot cache (BASELINE configs[1])",
+                           "lineorder_rows": n_lo, "rows_per_gpu": shard_rows, "queries": 13,
+                           "parallelism": f"row-sharded x{ws}" if ws > 1 else "1 GPU",
+                           "l2": "inputs (6.7 GB/GPU) larger than L2; no flush"},
+                "queries_per_s": 13 * args.steps / (ms / 1e3),
+                "gpu_launches": kernels_per_step * args.steps,
+                "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks,
+                "setup_s": round(setup_s, 1),
+                "checks": {q: len(r) for q, r in results.items()}}
+        print(json.dumps(line), flush=True)
+    for p in preps:
+        p.close()
+    db.close()
+    if ws > 1:
+        import torch.distributed as dist
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

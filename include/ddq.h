@@ -1,0 +1,356 @@
+/*
+ * ddq.h -- C ABI of libddq, the B200-native hot path of Bress, Funke & Teubner,
+ * "Robust Query Processing in Co-Processor-accelerated Databases" (SIGMOD'16).
+ *
+ * Citations "P:n" are /root/reference/PAPER.md line n (section named alongside);
+ * "S8(x)" is SURVEY.md section 8(x).  No torch or CUDA types appear here: device
+ * memory is passed as plain pointers, CUDA streams as `void*` (a cudaStream_t),
+ * sizes as integers.  Every call returns a ddq_status; nothing throws across the
+ * ABI.  On error, ddq_last_error() returns a thread-local message.
+ *
+ * Two layers:
+ *   1. Operator calls (ddq_op_*): the data-parallel kernels of S8(a1)-(a6) on
+ *      device buffers, stream-ordered, asynchronous.  Element counts that are
+ *      produced on the device stay on the device (a uint32 in device memory) so
+ *      operator chains never synchronise with the host.
+ *   2. The database (ddq_open .. ddq_fetch): a column store with a per-GPU column
+ *      cache and a heap-budget allocator (device memory = data cache + heap, P:62
+ *      Sec. 2.1), physical plans executed operator-at-a-time (Sec. 2.5) under
+ *      data-driven placement (Sec. 3.1, Sec. 3.3) and query chopping
+ *      (Sec. 5.1-5.2, Sec. 5.4), with abort-and-restart of a failed
+ *      operator on the host (Sec. 2.5.1, Sec. 4.1).
+ */
+#ifndef DDQ_H
+#define DDQ_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+/* ------------------------------------------------------------------ status */
+typedef int32_t ddq_status;
+enum {
+  DDQ_OK = 0,
+  DDQ_EINVAL = -1,        /* invalid argument / plan / duplicate build key */
+  DDQ_ENOTFOUND = -2,     /* unknown table, column or query handle */
+  DDQ_ENOMEM_HOST = -3,   /* host allocation failed */
+  DDQ_ENOMEM_DEVICE = -4, /* device heap exhausted (op layer / prepared plans only;
+                             inside ddq_submit an OOM aborts the operator and it is
+                             restarted on the host, P:111 -- never surfaced) */
+  DDQ_ECUDA = -5,         /* CUDA error (sticky) */
+  DDQ_ENCCL = -6,
+  DDQ_ESTATE = -7,        /* call not valid in the current state */
+  DDQ_ETIMEOUT = -8,
+  DDQ_EOVERFLOW = -9      /* a device hash table overflowed its capacity */
+};
+const char* ddq_last_error(void);
+const char* ddq_version(void);
+
+/* ========================================================================
+ * 1. Operator calls (device buffers; all pointers below are DEVICE pointers
+ *    unless named h_*).  TIDs are int32 row ids (< 2^31) in ascending order.
+ *    "count" arguments are device uint32 cells: an input count is read by the
+ *    kernel; an output count is written by it.  `n_cap` is a HOST upper bound on
+ *    the input count (sizes grids and scratch).  Outputs must hold n_cap items.
+ *    `scratch` is device memory of ddq_op_scratch_bytes(n_cap) bytes, owned by
+ *    the caller, reused freely after the call's stream work completes.
+ *    Errors: DDQ_EINVAL for bad widths / null required pointers / n_cap > 2^31;
+ *    DDQ_ECUDA if a launch fails.  Kernel-side overflow is reported through the
+ *    d_error cell where one exists.
+ * ====================================================================== */
+
+/* Predicate kinds (S8(a1)-(a2)).  RANGE covers =, <, <=, >, >=, BETWEEN on integer
+ * columns (constants folded into an inclusive [lo, hi]); IN holds up to 8 values
+ * (string IN/= become dictionary-code sets, reading O4). */
+enum { DDQ_PRED_RANGE = 1, DDQ_PRED_IN = 2 };
+#define DDQ_MAX_IN 8
+#define DDQ_MAX_PREDS 4
+#define DDQ_MAX_CARRY 4
+
+typedef struct {
+  const void* col; /* device column, indexed by row id */
+  int32_t width;   /* 4 (int32) or 8 (int64) */
+  int32_t kind;    /* DDQ_PRED_RANGE | DDQ_PRED_IN */
+  int64_t lo, hi;  /* RANGE: lo <= v <= hi */
+  int32_t n_in;    /* IN: number of values in in_vals */
+  int32_t _pad;
+  int64_t in_vals[DDQ_MAX_IN];
+} ddq_dev_pred;
+
+/* Scratch bytes needed by select / probe / build / groupby for n_cap inputs. */
+size_t ddq_op_scratch_bytes(int64_t n_cap);
+
+/* Selection (S8(a1) dimension, S8(a2) fact; App. B):
+ * out_tids = ascending row ids r of the input (all rows [0, n_cap) when
+ * in_tids == NULL, else r = in_tids[i] for i < *d_in_count) for which EVERY
+ * predicate holds.  Carried vectors (aligned with the input, int32) are
+ * compacted alongside: carry_out[c][j] = carry_in[c][i] for the j-th survivor i.
+ * *d_out_count receives the survivor count.  Stable stream compaction
+ * (decoupled look-back), deterministic. */
+ddq_status ddq_op_select(const ddq_dev_pred* preds, int32_t n_preds,
+                         const int32_t* in_tids, const uint32_t* d_in_count, int64_t n_cap,
+                         const int32_t* const* carry_in, int32_t* const* carry_out, int32_t n_carry,
+                         int32_t* out_tids, uint32_t* d_out_count,
+                         void* scratch, size_t scratch_bytes, void* stream);
+
+/* Hash build (S8(a3); join memory): insert (key = keys[r], payload =
+ * payload ? payload[r] : r) for every input row r into an open-addressing table
+ * of `capacity` 8-byte slots (power of two, >= 2x the number of keys, load <= 0.5;
+ * reading O13).  The table must be initialised with ddq_op_hash_init.  Keys must
+ * be unique and != INT32_MIN; a duplicate or a full table sets *d_error != 0
+ * (1 = duplicate key, 2 = table full). */
+ddq_status ddq_op_hash_init(uint64_t* table, uint32_t capacity, void* stream);
+ddq_status ddq_op_hash_build(const int32_t* keys, const int32_t* payload,
+                             const int32_t* in_tids, const uint32_t* d_in_count, int64_t n_cap,
+                             uint64_t* table, uint32_t capacity, uint32_t* d_error, void* stream);
+
+/* Hash probe = semi-join + payload (S8(a4)): for each input row r
+ * (all rows or in_tids[i]), look up fk[r]; survivors are compacted stably into
+ * out_tids, with the matched payload into out_payload (may be NULL) and carried
+ * vectors compacted alongside (as in ddq_op_select). */
+ddq_status ddq_op_hash_probe(const uint64_t* table, uint32_t capacity, const int32_t* fk,
+                             const int32_t* in_tids, const uint32_t* d_in_count, int64_t n_cap,
+                             const int32_t* const* carry_in, int32_t* const* carry_out, int32_t n_carry,
+                             int32_t* out_tids, int32_t* out_payload, uint32_t* d_out_count,
+                             void* scratch, size_t scratch_bytes, void* stream);
+
+/* Positional gather (S8(a5); P:107 materialisation): out[i] = col[tids[i]] for
+ * i < *d_count; width 4 or 8. */
+ddq_status ddq_op_gather(const void* col, int32_t width, const int32_t* tids,
+                         const uint32_t* d_count, int64_t n_cap, void* out, void* stream);
+
+/* Group-by aggregation (S8(a6)).  For each input position i < *d_count with
+ * row r = tids[i]: group key = k0 | k1 << 21 | k2 << 42 where kj is either the
+ * aligned vector key_vec[j][i] or the column key_col[j][r] (int32, 0 <= kj < 2^21);
+ * aggregate a adds expr_a(r) to the group's exact int128 accumulator.  The result
+ * is an open-addressing table of `capacity` slots (power of two, >= 2x groups):
+ *   keys  int64[capacity]           (empty = -1)
+ *   accs  int64[n_aggs][capacity][2] (lo, hi words of an int128)
+ * Init with ddq_op_groupby_init; read it back with ddq_op_groupby_compact.
+ * Overflow of the table sets *d_error = 2. */
+enum {
+  DDQ_AGG_COUNT = 1,          /* 1 */
+  DDQ_AGG_SUM = 2,            /* a */
+  DDQ_AGG_SUM_MUL = 3,        /* a * b */
+  DDQ_AGG_SUM_SUB = 4,        /* a - b */
+  DDQ_AGG_SUM_MUL_100M = 5,   /* a * (100 - b)            (TPC-H scale-2 decimals) */
+  DDQ_AGG_SUM_MUL_100M_100P = 6 /* a * (100 - b) * (100 + c) */
+};
+#define DDQ_MAX_AGGS 8
+#define DDQ_MAX_KEYS 3
+typedef struct {
+  int32_t kind;            /* DDQ_AGG_* */
+  int32_t width[3];        /* widths of the argument columns (4 or 8) */
+  const void* arg[3];      /* argument columns (device, indexed by row id) */
+} ddq_dev_agg;
+
+size_t ddq_op_groupby_table_bytes(uint32_t capacity, int32_t n_aggs);
+ddq_status ddq_op_groupby_init(void* table, uint32_t capacity, int32_t n_aggs, void* stream);
+ddq_status ddq_op_groupby(const int32_t* tids, const uint32_t* d_count, int64_t n_cap,
+                          const int32_t* const* key_vec, const int32_t* const* key_col, int32_t n_keys,
+                          const ddq_dev_agg* aggs, int32_t n_aggs,
+                          void* table, uint32_t capacity, uint32_t* d_error, void* stream);
+/* Compact the non-empty groups: out_keys int64[capacity], out_accs int64[n_aggs *
+ * capacity * 2] (group-major: accs of group g at [(g * n_aggs + a) * 2]),
+ * *d_out_groups = number of groups.  Group order is unspecified. */
+ddq_status ddq_op_groupby_compact(const void* table, uint32_t capacity, int32_t n_aggs,
+                                  int64_t* out_keys, int64_t* out_accs, uint32_t* d_out_groups,
+                                  void* stream);
+
+/* ========================================================================
+ * 2. The database: column store, device cache + heap, plans, chopping.
+ * ====================================================================== */
+typedef struct ddq_db ddq_db;
+typedef int32_t ddq_table;
+typedef int32_t ddq_column;
+typedef int64_t ddq_query;
+
+typedef enum { DDQ_I32 = 1, DDQ_I64 = 2 } ddq_type;
+
+/* Placement strategies (Sec. 6.2 and Sec. 3-5). */
+typedef enum {
+  DDQ_PLACE_DATA_DRIVEN = 0, /* GPU iff all inputs are cached there */
+  DDQ_PLACE_GPU_ONLY = 1,    /* "GPU Preferred": everything on the GPU; inputs that are
+                                not cached are copied on demand (operator-driven data
+                                placement with LRU caching) */
+  DDQ_PLACE_CPU_ONLY = 2
+} ddq_placement;
+
+typedef struct {
+  int32_t device;                /* CUDA device ordinal (one process per GPU) */
+  int32_t rank, world;           /* for row-sharded multi-GPU runs */
+  uint64_t cache_bytes;          /* device column cache budget */
+  uint64_t heap_bytes;           /* device heap for intermediates */
+  int32_t gpu_workers;           /* chopping bound: GPU worker threads, O17 */
+  int32_t host_workers;          /* host executor threads */
+  int32_t placement;             /* ddq_placement */
+  int32_t chopping;              /* 1: run-time placement + bounded pull queues (Sec. 5.2);
+                                    0: compile-time placement, one thread per operator */
+  int32_t cache_policy;          /* 0 = LFU (Alg. 1), 1 = LRU (App. E) */
+  uint32_t fault_alloc_every;    /* fault injection: fail every Nth device heap alloc (0=off) */
+} ddq_config;
+
+void ddq_config_default(ddq_config* cfg);
+ddq_status ddq_open(const ddq_config* cfg, ddq_db** out);
+void ddq_close(ddq_db* db);
+
+/* Tables and columns.  ddq_load_column copies host_data (n_rows values of the
+ * given type) into library-owned pinned host memory (Sec. 2.5.3); the caller
+ * keeps ownership of host_data.  shard_row_begin = global row id of local row 0. */
+ddq_status ddq_create_table(ddq_db* db, const char* name, int64_t n_rows, int64_t shard_row_begin,
+                            ddq_table* out);
+ddq_status ddq_load_column(ddq_db* db, ddq_table t, const char* name, ddq_type type,
+                           const void* host_data, int64_t n_rows, ddq_column* out);
+ddq_status ddq_find_column(ddq_db* db, const char* table, const char* name, ddq_column* out);
+/* Storage adviser: pin a column into the device cache (H2D copy on the
+ * library's copy stream, counted in stats) / evict it (freed once no running
+ * operator references it).  Fails with DDQ_ENOMEM_DEVICE if it does not
+ * fit the cache budget. */
+ddq_status ddq_cache_column(ddq_db* db, ddq_column c);
+ddq_status ddq_evict_column(ddq_db* db, ddq_column c);
+int32_t ddq_column_is_cached(ddq_db* db, ddq_column c);
+/* Device pointer of a cached column (for the operator layer), or NULL. */
+const void* ddq_column_device_ptr(ddq_db* db, ddq_column c);
+/* Run Algorithm 1 once (Sec. 3.2): sort columns by access count
+ * (descending; ties by column id, O16), keep the greedy prefix that fits the cache
+ * budget (stop at the first that does not fit), evict old\new, cache new\old. */
+ddq_status ddq_update_placement(ddq_db* db);
+/* Access counters (incremented per operator access) */
+uint64_t ddq_column_access_count(ddq_db* db, ddq_column c);
+ddq_status ddq_reset_access_counts(ddq_db* db);
+
+/* ---- physical plans (S8(b) plan IR) ----------------------------------------
+ * A plan is an array of operators; op i's children have indices < i; the last
+ * op is the root and must be an AGGREGATE (or a SELECT/GATHER for select-*).
+ * Every op produces a materialised intermediate: a TID list over a table's
+ * row space plus aligned int32/int64 vectors. */
+enum {
+  DDQ_OP_SELECT = 1,     /* preds over `table` at input TIDs (or all rows) */
+  DDQ_OP_HASH_BUILD = 2, /* hash table over input TIDs of `table` (key_col, payload_col) */
+  DDQ_OP_HASH_PROBE = 3, /* semi-join input TIDs of `table` via fk_col against op `build` */
+  DDQ_OP_GATHER = 4,     /* append vector col[tid] to the input's aligned vectors */
+  DDQ_OP_AGGREGATE = 5   /* group-by at input TIDs; root; finalised on the host */
+};
+
+typedef struct {
+  ddq_column column;
+  int32_t kind;   /* DDQ_PRED_RANGE | DDQ_PRED_IN */
+  int64_t lo, hi;
+  int32_t n_in;
+  int32_t _pad;
+  int64_t in_vals[DDQ_MAX_IN];
+} ddq_pred;
+
+typedef struct {
+  int32_t kind;            /* DDQ_OP_* */
+  int32_t input;           /* child op index whose output TIDs are consumed, or -1 = all rows */
+  ddq_table table;         /* row space of input and output TIDs */
+  /* SELECT */
+  int32_t n_preds;
+  ddq_pred preds[DDQ_MAX_PREDS];
+  /* HASH_BUILD */
+  ddq_column key_col;
+  ddq_column payload_col;  /* -1: payload = dimension row id */
+  /* HASH_PROBE */
+  int32_t build;           /* op index of the HASH_BUILD */
+  ddq_column fk_col;
+  int32_t emit_payload;    /* append matched payload as an aligned vector */
+  /* GATHER */
+  ddq_column gather_col;
+  /* AGGREGATE: keys are aligned vectors (index >= 0) or columns (-2 - column id) */
+  int32_t n_keys;
+  int32_t key_src[DDQ_MAX_KEYS];
+  int32_t n_aggs;
+  int32_t agg_kind[DDQ_MAX_AGGS];
+  ddq_column agg_col[DDQ_MAX_AGGS][3];
+  int64_t max_groups;      /* upper bound on the number of groups (sizes the table) */
+  /* finalisation (S8(a7)): ORDER BY entries: +(1+k) key k asc, -(1+k) key k desc,
+     +(101+a) aggregate a asc, -(101+a) desc; codes are order-preserving (O4). */
+  int32_t n_order;
+  int32_t order_by[8];
+  int64_t limit;           /* <= 0: no limit */
+} ddq_op;
+
+#define DDQ_MAX_OPS 32
+typedef struct {
+  int32_t n_ops;
+  ddq_op ops[DDQ_MAX_OPS];
+} ddq_plan;
+
+/* Result of a query: rows of (n_keys int32-code keys, n_aggs int128 aggregates)
+ * in ORDER BY order, or, for a select-* root, the TID list. Owned by the library. */
+typedef struct {
+  int64_t n_rows;
+  int32_t n_keys, n_aggs;
+  const int64_t* keys;   /* n_rows * n_keys (decoded from the packed group key) */
+  const int64_t* aggs;   /* n_rows * n_aggs * 2: (lo, hi) words of each int128 */
+  int64_t n_tids;        /* select-* roots: surviving TIDs (global row ids) */
+  const int32_t* tids;
+  int32_t gpu_ops, host_ops, aborts;
+  double exec_ms;        /* submit -> root finished */
+} ddq_result;
+
+/* Submit a plan (copied; thread-safe; many user threads may submit). */
+ddq_status ddq_submit(ddq_db* db, const ddq_plan* plan, ddq_query* out);
+ddq_status ddq_wait(ddq_db* db, ddq_query q, int64_t timeout_ns);
+ddq_status ddq_fetch(ddq_db* db, ddq_query q, ddq_result** out);
+void ddq_result_free(ddq_result* r);
+
+/* Prepared plans: the hot path for resident data (configs 1-3).  All operators
+ * are placed on the GPU (every input must be cached: data-driven placement,
+ * P:140), intermediates are allocated from the heap once (fail-fast), and
+ * the operator sequence is captured into one CUDA graph.  ddq_prepared_launch
+ * enqueues one execution on `stream` with no host synchronisation;
+ * ddq_prepared_fetch synchronises and finalises. */
+typedef struct ddq_prepared ddq_prepared;
+ddq_status ddq_prepare(ddq_db* db, const ddq_plan* plan, int32_t use_graph, ddq_prepared** out);
+ddq_status ddq_prepared_launch(ddq_prepared* p, void* stream);
+ddq_status ddq_prepared_fetch(ddq_prepared* p, void* stream, ddq_result** out);
+/* Partial aggregate access for multi-GPU merges (S8(e)): after a launch, copy the
+ * compacted group table (keys int64[cap], accs int64[cap*n_aggs*2]) to host. */
+ddq_status ddq_prepared_partials(ddq_prepared* p, void* stream, int64_t* h_n_groups,
+                                 int64_t* h_keys, int64_t* h_accs, int64_t cap);
+int64_t ddq_prepared_group_capacity(ddq_prepared* p);
+/* Per-op kernel timing of the last launch is not tracked in graph mode; this
+ * returns the number of kernels one launch enqueues. */
+int32_t ddq_prepared_kernel_count(ddq_prepared* p);
+/* Profiling pass (no graph): replays the plan on `stream` with a CUDA event
+ * before and after every operator, then reports per operator (up to max_ops):
+ * op_ms = event-timed duration, op_bytes = algorithmic HBM bytes of the SURVEY
+ * 8(d) model computed from the actual cardinalities (columns read once; TID-driven
+ * reads at 32-byte-sector granularity: N*w*(1-(1-m/N)^(32/w)); TID / vector /
+ * payload reads and writes; hash tables 0 bytes except their build writes),
+ * op_class = 0 dense scan (select/probe over all rows), 1 select/probe at TIDs,
+ * 2 hash build, 3 gather, 4 aggregate.  Returns the number of operators. */
+int32_t ddq_prepared_profile(ddq_prepared* p, void* stream, int32_t max_ops, float* op_ms, double* op_bytes,
+                             int32_t* op_class);
+/* Finalise externally merged partials (keys/accs as returned above) into a result. */
+ddq_status ddq_prepared_finalize(ddq_prepared* p, int64_t n_groups, const int64_t* h_keys,
+                                 const int64_t* h_accs, ddq_result** out);
+void ddq_prepared_free(ddq_prepared* p);
+
+/* ---- statistics (paper's counters, D10: P:330) ---- */
+typedef struct {
+  uint64_t h2d_bytes, d2h_bytes;
+  uint64_t h2d_ns, d2h_ns;
+  uint64_t gpu_ops, host_ops;
+  uint64_t aborts;          /* GPU operators aborted on allocation failure */
+  uint64_t wasted_ns;       /* begin->abort time of aborted GPU operators */
+  uint64_t heap_peak_bytes, heap_used_bytes, cache_used_bytes;
+  uint64_t cache_hits, cache_misses;
+  uint64_t queries_done;
+} ddq_stats;
+ddq_status ddq_get_stats(ddq_db* db, ddq_stats* out);
+ddq_status ddq_reset_stats(ddq_db* db);
+
+/* Device heap (for the operator layer / tests): fail-fast sub-allocation. */
+void* ddq_heap_try_alloc(ddq_db* db, uint64_t bytes);
+void ddq_heap_free(ddq_db* db, void* p);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* DDQ_H */

@@ -1,0 +1,117 @@
+// device_common.cuh -- small device helpers shared by the libddq kernels
+// (vector loads, warp scans, decoupled look-back, hashing, int128 atomics).
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace ddq {
+
+constexpr unsigned FULL = 0xffffffffu;
+
+// ---- loads ---------------------------------------------------------------
+// Streaming 128-bit loads that do not allocate in L1 (each column byte is read once).
+__device__ __forceinline__ int4 ld_stream_i4(const void* p) {
+  int4 r;
+  asm volatile("ld.global.nc.L1::no_allocate.v4.s32 {%0,%1,%2,%3}, [%4];"
+               : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(p));
+  return r;
+}
+__device__ __forceinline__ longlong2 ld_stream_l2(const void* p) {
+  longlong2 r;
+  asm volatile("ld.global.nc.L1::no_allocate.v2.s64 {%0,%1}, [%2];"
+               : "=l"(r.x), "=l"(r.y) : "l"(p));
+  return r;
+}
+__device__ __forceinline__ uint64_t ld_relaxed_u64(const uint64_t* p) {
+  uint64_t v;
+  asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_relaxed_u64(uint64_t* p, uint64_t v) {
+  asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ uint32_t ld_relaxed_u32(const uint32_t* p) {
+  uint32_t v;
+  asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+
+// Scalar read of column element r (width 4 or 8) widened to int64.
+__device__ __forceinline__ int64_t col_at(const void* col, int width, int64_t r) {
+  return width == 8 ? __ldg(reinterpret_cast<const long long*>(col) + r)
+                    : (int64_t)__ldg(reinterpret_cast<const int*>(col) + r);
+}
+
+// ---- warp scan -----------------------------------------------------------
+__device__ __forceinline__ uint32_t warp_incl_scan(uint32_t v, int lane) {
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    uint32_t t = __shfl_up_sync(FULL, v, o);
+    if (lane >= o) v += t;
+  }
+  return v;
+}
+
+// ---- decoupled look-back (single-pass prefix over tiles) -------------------
+// status word: [63:62] flag (0 invalid, 1 aggregate, 2 inclusive prefix), [31:0] value
+constexpr uint64_t LB_AGG = 1ull << 62;
+constexpr uint64_t LB_INC = 2ull << 62;
+
+// Called by one full warp.  Returns the exclusive prefix of `tile` (all lanes).
+__device__ __forceinline__ uint32_t lookback(uint64_t* status, uint32_t tile, uint32_t total, int lane) {
+  if (tile == 0) {
+    if (lane == 0) st_relaxed_u64(&status[0], LB_INC | total);
+    return 0;
+  }
+  if (lane == 0) st_relaxed_u64(&status[tile], LB_AGG | total);
+  uint32_t excl = 0;
+  int64_t pred = (int64_t)tile - 1 - lane;
+  while (true) {
+    uint64_t s;
+    unsigned spins = 0;
+    while (true) {
+      s = pred >= 0 ? ld_relaxed_u64(&status[pred]) : (LB_INC | 0ull);
+      if (__ballot_sync(FULL, (s >> 62) == 0) == 0) break;
+      if (++spins > 8) __nanosleep(32);
+    }
+    unsigned inc = __ballot_sync(FULL, (s >> 62) == 2);
+    uint32_t v = (uint32_t)s;
+    if (inc) {
+      int k = __ffs(inc) - 1;
+      if (lane > k) v = 0;
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(FULL, v, o);
+      excl += v;
+      break;
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(FULL, v, o);
+    excl += v;
+    pred -= 32;
+  }
+  if (lane == 0) st_relaxed_u64(&status[tile], LB_INC | (uint64_t)(excl + total));
+  return excl;
+}
+
+// ---- hashing ---------------------------------------------------------------
+constexpr uint64_t HT_EMPTY = 0x8000000000000000ull;  // key INT32_MIN, payload 0
+__device__ __forceinline__ uint32_t ht_hash(int32_t k, int shift) {
+  return ((uint32_t)k * 0x9E3779B1u) >> shift;  // shift = 32 - log2(capacity)
+}
+__device__ __forceinline__ int32_t ht_key(uint64_t s) { return (int32_t)(s >> 32); }
+__device__ __forceinline__ int32_t ht_val(uint64_t s) { return (int32_t)(uint32_t)s; }
+
+constexpr int64_t GB_EMPTY = -1;
+__device__ __forceinline__ uint32_t gb_hash(int64_t k, int shift) {
+  return (uint32_t)(((uint64_t)k * 0x9E3779B97F4A7C15ull) >> shift);  // shift = 64 - log2(cap)
+}
+
+// exact int128 accumulation with two 64-bit atomics (lo unsigned, hi signed)
+__device__ __forceinline__ void atomic_add_i128(unsigned long long* lo, unsigned long long* hi, long long v) {
+  unsigned long long old = atomicAdd(lo, (unsigned long long)v);
+  unsigned long long sum = old + (unsigned long long)v;
+  long long hadd = (v < 0 ? -1ll : 0ll) + (sum < old ? 1ll : 0ll);
+  if (hadd) atomicAdd(hi, (unsigned long long)hadd);
+}
+
+}  // namespace ddq

@@ -1,0 +1,809 @@
+// driver.cpp -- the paper's execution policy around the operators:
+//   * query chopping (Sec. 5.1-5.2): the leaf operators of every
+//     submitted query enter a global operator stream; each processor has a ready
+//     queue served by a bounded pool of worker threads that PULL operators; a
+//     finished operator notifies its parent, which enqueues itself once all its
+//     children are done (Fig. 11);
+//   * run-time data-driven placement (Sec. 3.1, Sec. 3.3
+//     Sec. 5.4): an operator goes to the GPU iff all its input columns are cached
+//     there and all its child intermediates live there; otherwise to the host;
+//   * abort and restart (Sec. 2.5.1, Sec. 4.1): a GPU operator
+//     whose heap allocation fails aborts at once (no wait-and-admit), its
+//     begin->abort time is counted as wasted time, and it is restarted on
+//     the host; its successors follow the data to the host;
+//   * the comparison arms of Sec. 6.2: GPU-only with operator-driven data
+//     placement (inputs copied on demand, LRU), compile-time placement (chopping=0:
+//     placement fixed at submit, no concurrency bound), and CPU-only.
+// The host executor (run_host_op) is the CPU fallback handler that exists for
+// every operator.  It is product code and shares nothing with oracle/.
+#include <algorithm>
+#include <array>
+#include <cstring>
+#include <numeric>
+#include <unordered_map>
+
+#include "engine.h"
+#include "ops_internal.h"
+
+namespace ddq {
+
+ddq_status cache_column_locked(ddq_db* db, int c, bool on_demand);
+void evict_column_locked(ddq_db* db, int c);
+ddq_status validate_plan_public(ddq_db* db, const ddq_plan* plan);
+
+enum Place { P_NONE = 0, P_GPU = 1, P_HOST = 2 };
+
+struct QueryState {
+  int64_t id = 0;
+  ddq_plan plan{};
+  std::vector<Inter> inters;
+  std::vector<int> pending;                 // unfinished children per op
+  std::vector<std::vector<int>> parents;
+  std::vector<int> place;                   // compile-time placement (chopping=0)
+  std::vector<int> consumers_left;          // for freeing intermediates early
+  int ops_left = 0;
+  bool done = false;
+  ddq_status status = DDQ_OK;
+  std::string error;
+  ddq_result* result = nullptr;
+  uint64_t t_submit = 0, t_done = 0;
+  int gpu_ops = 0, host_ops = 0, aborts = 0;
+  std::mutex mu;
+  std::condition_variable cv;
+};
+
+// ------------------------------------------------------------ column helpers
+static std::vector<int> op_columns(const ddq_op& op) {
+  std::vector<int> c;
+  switch (op.kind) {
+    case DDQ_OP_SELECT:
+      for (int i = 0; i < op.n_preds; i++) c.push_back(op.preds[i].column);
+      break;
+    case DDQ_OP_HASH_BUILD:
+      c.push_back(op.key_col);
+      if (op.payload_col >= 0) c.push_back(op.payload_col);
+      break;
+    case DDQ_OP_HASH_PROBE: c.push_back(op.fk_col); break;
+    case DDQ_OP_GATHER: c.push_back(op.gather_col); break;
+    case DDQ_OP_AGGREGATE:
+      for (int k = 0; k < op.n_keys; k++)
+        if (op.key_src[k] < -1) c.push_back(-2 - op.key_src[k]);
+      for (int a = 0; a < op.n_aggs; a++) {
+        int need = op.agg_kind[a] == DDQ_AGG_COUNT ? 0 : op.agg_kind[a] == DDQ_AGG_SUM ? 1
+                 : op.agg_kind[a] == DDQ_AGG_SUM_MUL_100M_100P ? 3 : 2;
+        for (int j = 0; j < need; j++) c.push_back(op.agg_col[a][j]);
+      }
+      break;
+  }
+  return c;
+}
+
+static std::vector<int> op_children(const ddq_op& op) {
+  std::vector<int> ch;
+  if (op.input >= 0) ch.push_back(op.input);
+  if (op.kind == DDQ_OP_HASH_PROBE && op.build >= 0 && op.build != op.input) ch.push_back(op.build);
+  return ch;
+}
+
+// ------------------------------------------------------------ transfers
+static void* host_alloc(Inter& x, size_t bytes) {
+  void* p = std::malloc(std::max<size_t>(bytes, 8));
+  if (p) x.host_blocks.push_back(p);
+  return p;
+}
+
+// Move an intermediate to host memory (D2H; counted as GPU->CPU transfer).
+ddq_status inter_to_host(ddq_db* db, Inter& x, cudaStream_t st) {
+  if (x.on_host) return DDQ_OK;
+  Inter h;
+  h.on_host = true;
+  h.table = x.table;
+  uint64_t t0 = now_ns();
+  uint64_t bytes = 0;
+  if (x.table_ptr) {
+    auto t = std::make_shared<std::vector<uint64_t>>(x.table_cap);
+    cudaMemcpyAsync(t->data(), x.table_ptr, (size_t)x.table_cap * 8, cudaMemcpyDeviceToHost, st);
+    h.host_table = t;
+    h.table_cap = x.table_cap;
+    bytes += (uint64_t)x.table_cap * 8;
+  }
+  if (x.gb_table) {
+    uint32_t g = 0;
+    cudaMemcpyAsync(&g, x.gb_groups, 4, cudaMemcpyDeviceToHost, st);
+    cudaStreamSynchronize(st);
+    // aggregate inputs are consumed by finalisation only; keep the arrays
+    return set_error(DDQ_ESTATE, "aggregate output cannot move");
+  }
+  if (x.tids || x.d_count) {
+    uint32_t n = 0;
+    cudaMemcpyAsync(&n, x.d_count, 4, cudaMemcpyDeviceToHost, st);
+    cudaError_t e = cudaStreamSynchronize(st);
+    if (e != cudaSuccess) return cuda_status(e, "inter_to_host count");
+    h.count = n;
+    h.cap = n;
+    h.tids = (int32_t*)host_alloc(h, (size_t)n * 4);
+    if (!h.tids) return set_error(DDQ_ENOMEM_HOST, "inter_to_host");
+    if (n) cudaMemcpyAsync(h.tids, x.tids, (size_t)n * 4, cudaMemcpyDeviceToHost, st);
+    bytes += (uint64_t)n * 4;
+    for (const Vec& v : x.vecs) {
+      void* p = host_alloc(h, (size_t)n * v.width);
+      if (!p) return set_error(DDQ_ENOMEM_HOST, "inter_to_host");
+      if (n) cudaMemcpyAsync(p, v.ptr, (size_t)n * v.width, cudaMemcpyDeviceToHost, st);
+      h.vecs.push_back(Vec{p, v.width, true});
+      bytes += (uint64_t)n * v.width;
+    }
+  }
+  cudaError_t e = cudaStreamSynchronize(st);
+  if (e != cudaSuccess) return cuda_status(e, "inter_to_host");
+  db->stats.d2h_bytes += bytes;
+  db->stats.d2h_ns += now_ns() - t0;
+  release_inter(db, x);
+  x = std::move(h);
+  return DDQ_OK;
+}
+
+// Move a host intermediate to the device heap (H2D; CPU->GPU transfer).
+// Returns DDQ_ENOMEM_DEVICE if the heap cannot hold it (-> abort).
+static ddq_status inter_to_device(ddq_db* db, Inter& x, cudaStream_t st) {
+  if (!x.on_host) return DDQ_OK;
+  Inter d;
+  d.table = x.table;
+  uint64_t t0 = now_ns(), bytes = 0;
+  auto get = [&](uint64_t b) -> void* {
+    void* p = db->heap.try_alloc(b);
+    if (p) d.heap_blocks.push_back(p);
+    return p;
+  };
+  if (x.host_table) {
+    d.table_cap = x.table_cap;
+    d.table_ptr = (uint64_t*)get((uint64_t)x.table_cap * 8);
+    d.d_error = (uint32_t*)get(64);
+    if (!d.table_ptr || !d.d_error) {
+      release_inter(db, d);
+      return DDQ_ENOMEM_DEVICE;
+    }
+    cudaMemsetAsync(d.d_error, 0, 4, st);
+    cudaMemcpyAsync(d.table_ptr, x.host_table->data(), (size_t)x.table_cap * 8, cudaMemcpyHostToDevice, st);
+    bytes += (uint64_t)x.table_cap * 8;
+  } else {
+    int64_t n = x.count;
+    d.cap = n;
+    d.count = n;
+    d.tids = (int32_t*)get((uint64_t)std::max<int64_t>(n, 1) * 4);
+    d.d_count = (uint32_t*)get(64);
+    d.d_error = (uint32_t*)get(64);
+    for (const Vec& v : x.vecs) d.vecs.push_back(Vec{get((uint64_t)std::max<int64_t>(n, 1) * v.width), v.width, false});
+    bool ok = d.tids && d.d_count && d.d_error;
+    for (auto& v : d.vecs) ok = ok && v.ptr;
+    if (!ok) {
+      release_inter(db, d);
+      return DDQ_ENOMEM_DEVICE;
+    }
+    uint32_t n32 = (uint32_t)n;
+    cudaMemcpyAsync(d.d_count, &n32, 4, cudaMemcpyHostToDevice, st);
+    cudaMemsetAsync(d.d_error, 0, 4, st);
+    if (n) cudaMemcpyAsync(d.tids, x.tids, (size_t)n * 4, cudaMemcpyHostToDevice, st);
+    for (size_t i = 0; i < x.vecs.size(); i++)
+      if (n) cudaMemcpyAsync(d.vecs[i].ptr, x.vecs[i].ptr, (size_t)n * x.vecs[i].width, cudaMemcpyHostToDevice, st);
+    bytes += (uint64_t)n * 4;
+    for (auto& v : x.vecs) bytes += (uint64_t)n * v.width;
+  }
+  cudaError_t e = cudaStreamSynchronize(st);
+  if (e != cudaSuccess) {
+    release_inter(db, d);
+    return cuda_status(e, "inter_to_device");
+  }
+  db->stats.h2d_bytes += bytes;
+  db->stats.h2d_ns += now_ns() - t0;
+  release_inter(db, x);
+  x = std::move(d);
+  return DDQ_OK;
+}
+
+// ------------------------------------------------------------ host executor
+static inline uint32_t host_hash32(int32_t k, int shift) { return ((uint32_t)k * 0x9E3779B1u) >> shift; }
+static constexpr uint64_t kHostEmpty = 0x8000000000000000ull;
+
+template <class F>
+static void parallel_chunks(int64_t n, int threads, F f) {  // f(chunk, begin, end)
+  if (threads <= 1 || n < (1 << 16)) {
+    f(0, 0, n);
+    return;
+  }
+  std::vector<std::thread> th;
+  int64_t step = (n + threads - 1) / threads;
+  for (int t = 0; t < threads; t++) {
+    int64_t b = t * step, e = std::min<int64_t>(n, b + step);
+    if (b >= e) break;
+    th.emplace_back([=] { f(t, b, e); });
+  }
+  for (auto& x : th) x.join();
+}
+
+static int host_threads(ddq_db* db) {
+  int hw = (int)std::thread::hardware_concurrency();
+  int t = hw / std::max(1, db->cfg.host_workers);
+  return std::max(1, t);
+}
+
+static inline int64_t hcol(const Column* c, int64_t r) {
+  return c->width == 8 ? ((const int64_t*)c->host)[r] : (int64_t)((const int32_t*)c->host)[r];
+}
+
+ddq_status run_host_op(ddq_db* db, const ddq_op& op, const std::vector<Inter>& I, Inter& out) {
+  out = Inter();
+  out.on_host = true;
+  out.table = op.table;
+  const Table& T = db->tables[(size_t)op.table];
+  const Inter* in = op.input >= 0 ? &I[(size_t)op.input] : nullptr;
+  if (in && !in->on_host) return set_error(DDQ_ESTATE, "host op with a device-resident input");
+  const int64_t n = in ? in->count : T.n_rows;
+  auto row_of = [&](int64_t i) -> int32_t { return in ? in->tids[i] : (int32_t)i; };
+  const int threads = host_threads(db);
+  for (int c : op_columns(op)) {
+    db->cols[(size_t)c]->access++;
+    db->cols[(size_t)c]->last_access = ++db->clock;
+  }
+  switch (op.kind) {
+    case DDQ_OP_SELECT:
+    case DDQ_OP_HASH_PROBE: {
+      const bool probe = op.kind == DDQ_OP_HASH_PROBE;
+      const Inter* build = probe ? &I[(size_t)op.build] : nullptr;
+      if (probe && !build->host_table) return set_error(DDQ_ESTATE, "host probe needs a host table");
+      std::vector<const Column*> pc;
+      for (int i = 0; i < op.n_preds && !probe; i++) pc.push_back(col_of(db, op.preds[i].column));
+      const Column* fk = probe ? col_of(db, op.fk_col) : nullptr;
+      int lg = 0;
+      if (probe)
+        while ((1u << lg) < build->table_cap) lg++;
+      const uint64_t* tab = probe ? build->host_table->data() : nullptr;
+      const uint32_t mask = probe ? build->table_cap - 1 : 0;
+      int nchunks = (threads <= 1 || n < (1 << 16)) ? 1 : threads;
+      std::vector<std::vector<int64_t>> sel((size_t)nchunks);     // positions i
+      std::vector<std::vector<int32_t>> pay((size_t)nchunks);
+      parallel_chunks(n, nchunks, [&](int t, int64_t b, int64_t e) {
+        auto& S = sel[(size_t)t];
+        auto& Pv = pay[(size_t)t];
+        for (int64_t i = b; i < e; i++) {
+          int32_t r = row_of(i);
+          bool ok = true;
+          if (!probe) {
+            for (int p = 0; p < op.n_preds && ok; p++) {
+              int64_t v = hcol(pc[(size_t)p], r);
+              const ddq_pred& pr = op.preds[p];
+              if (pr.kind == DDQ_PRED_RANGE) ok = v >= pr.lo && v <= pr.hi;
+              else {
+                bool m = false;
+                for (int j = 0; j < pr.n_in; j++) m |= v == pr.in_vals[j];
+                ok = m;
+              }
+            }
+            if (ok) S.push_back(i);
+          } else {
+            int32_t k = ((const int32_t*)fk->host)[r];
+            uint32_t h = host_hash32(k, 32 - lg);
+            while (true) {
+              uint64_t s = tab[h];
+              if (s == kHostEmpty) { ok = false; break; }
+              if ((int32_t)(s >> 32) == k) { Pv.push_back((int32_t)(uint32_t)s); break; }
+              h = (h + 1) & mask;
+            }
+            if (ok) S.push_back(i);
+          }
+        }
+      });
+      int64_t total = 0;
+      for (auto& s : sel) total += (int64_t)s.size();
+      out.count = out.cap = total;
+      out.tids = (int32_t*)host_alloc(out, (size_t)total * 4);
+      size_t nv = in ? in->vecs.size() : 0;
+      for (size_t v = 0; v < nv; v++) out.vecs.push_back(Vec{host_alloc(out, (size_t)total * in->vecs[v].width), in->vecs[v].width, true});
+      int32_t* payout = nullptr;
+      if (probe && op.emit_payload) {
+        payout = (int32_t*)host_alloc(out, (size_t)total * 4);
+        out.vecs.push_back(Vec{payout, 4, true});
+      }
+      int64_t o = 0;
+      for (int t = 0; t < nchunks; t++) {
+        for (size_t j = 0; j < sel[(size_t)t].size(); j++, o++) {
+          int64_t i = sel[(size_t)t][j];
+          out.tids[o] = row_of(i);
+          for (size_t v = 0; v < nv; v++) {
+            if (in->vecs[v].width == 4) ((int32_t*)out.vecs[v].ptr)[o] = ((const int32_t*)in->vecs[v].ptr)[i];
+            else ((int64_t*)out.vecs[v].ptr)[o] = ((const int64_t*)in->vecs[v].ptr)[i];
+          }
+          if (payout) payout[o] = pay[(size_t)t][j];
+        }
+      }
+      return DDQ_OK;
+    }
+    case DDQ_OP_HASH_BUILD: {
+      const Column* kc = col_of(db, op.key_col);
+      const Column* pc = op.payload_col >= 0 ? col_of(db, op.payload_col) : nullptr;
+      int64_t cap = pow2_at_least(std::max<int64_t>(16, 2 * n));
+      int lg = 0;
+      while ((1ll << lg) < cap) lg++;
+      auto t = std::make_shared<std::vector<uint64_t>>((size_t)cap, kHostEmpty);
+      for (int64_t i = 0; i < n; i++) {
+        int32_t r = row_of(i);
+        int32_t k = ((const int32_t*)kc->host)[r];
+        int32_t v = pc ? ((const int32_t*)pc->host)[r] : r;
+        uint32_t h = host_hash32(k, 32 - lg);
+        while ((*t)[h] != kHostEmpty) {
+          if ((int32_t)((*t)[h] >> 32) == k) return set_error(DDQ_EINVAL, "duplicate build key");
+          h = (h + 1) & (uint32_t)(cap - 1);
+        }
+        (*t)[h] = ((uint64_t)(uint32_t)k << 32) | (uint32_t)v;
+      }
+      out.host_table = t;
+      out.table_cap = (uint32_t)cap;
+      return DDQ_OK;
+    }
+    case DDQ_OP_GATHER: {
+      const Column* c = col_of(db, op.gather_col);
+      out.count = out.cap = n;
+      out.tids = (int32_t*)host_alloc(out, (size_t)n * 4);
+      std::memcpy(out.tids, in->tids, (size_t)n * 4);
+      for (const Vec& v : in->vecs) {
+        void* p = host_alloc(out, (size_t)n * v.width);
+        std::memcpy(p, v.ptr, (size_t)n * v.width);
+        out.vecs.push_back(Vec{p, v.width, true});
+      }
+      void* dst = host_alloc(out, (size_t)n * c->width);
+      for (int64_t i = 0; i < n; i++) {
+        if (c->width == 8) ((int64_t*)dst)[i] = ((const int64_t*)c->host)[in->tids[i]];
+        else ((int32_t*)dst)[i] = ((const int32_t*)c->host)[in->tids[i]];
+      }
+      out.vecs.push_back(Vec{dst, c->width, true});
+      return DDQ_OK;
+    }
+    case DDQ_OP_AGGREGATE: {
+      const int na = op.n_aggs;
+      std::vector<const Column*> kc(3, nullptr);
+      for (int k = 0; k < op.n_keys; k++)
+        if (op.key_src[k] < -1) kc[(size_t)k] = col_of(db, -2 - op.key_src[k]);
+      std::vector<std::array<const Column*, 3>> ac((size_t)na);
+      for (int a = 0; a < na; a++)
+        for (int j = 0; j < 3; j++) ac[(size_t)a][(size_t)j] = op.agg_col[a][j] >= 0 ? col_of(db, op.agg_col[a][j]) : nullptr;
+      std::unordered_map<int64_t, std::vector<__int128>> g;
+      for (int64_t i = 0; i < n; i++) {
+        int32_t r = in->tids[i];
+        int64_t key = 0;
+        for (int k = 0; k < op.n_keys; k++) {
+          int32_t c = op.key_src[k] >= 0 ? ((const int32_t*)in->vecs[(size_t)op.key_src[k]].ptr)[i]
+                                         : ((const int32_t*)kc[(size_t)k]->host)[r];
+          key |= (int64_t)(uint32_t)c << (21 * k);
+        }
+        auto& acc = g[key];
+        if (acc.empty()) acc.assign((size_t)na, 0);
+        for (int a = 0; a < na; a++) {
+          int kind = op.agg_kind[a];
+          __int128 v = 1;
+          if (kind != DDQ_AGG_COUNT) {
+            __int128 x = hcol(ac[(size_t)a][0], r);
+            if (kind == DDQ_AGG_SUM) v = x;
+            else {
+              __int128 y = hcol(ac[(size_t)a][1], r);
+              if (kind == DDQ_AGG_SUM_MUL) v = x * y;
+              else if (kind == DDQ_AGG_SUM_SUB) v = x - y;
+              else if (kind == DDQ_AGG_SUM_MUL_100M) v = x * (100 - y);
+              else v = x * (100 - y) * (100 + hcol(ac[(size_t)a][2], r));
+            }
+          }
+          acc[(size_t)a] += v;
+        }
+      }
+      auto keys = std::make_shared<std::vector<int64_t>>();
+      auto accs = std::make_shared<std::vector<int64_t>>();
+      for (auto& kv : g) {
+        keys->push_back(kv.first);
+        for (int a = 0; a < na; a++) {
+          unsigned __int128 u = (unsigned __int128)kv.second[(size_t)a];
+          accs->push_back((int64_t)(uint64_t)u);
+          accs->push_back((int64_t)(uint64_t)(u >> 64));
+        }
+      }
+      out.h_keys = keys;
+      out.h_accs = accs;
+      out.h_groups = (int64_t)keys->size();
+      return DDQ_OK;
+    }
+  }
+  return set_error(DDQ_EINVAL, "unknown operator");
+}
+
+// ------------------------------------------------------------ scheduling
+static bool columns_cached(ddq_db* db, const ddq_op& op) {
+  std::lock_guard<std::mutex> g(db->mu);
+  for (int c : op_columns(op)) {
+    const Column* col = col_of(db, c);
+    if (!col || !col->dev || col->evict_pending) return false;
+  }
+  return true;
+}
+
+static bool children_on_gpu(QueryState& q, int i) {
+  for (int c : op_children(q.plan.ops[i]))
+    if (q.inters[(size_t)c].on_host) return false;
+  return true;
+}
+
+// Operator-driven data placement for the GPU-only arm: make the
+// op's columns resident, evicting least-recently-used unreferenced columns.
+static ddq_status ensure_cached_lru(ddq_db* db, const ddq_op& op) {
+  std::lock_guard<std::mutex> g(db->mu);
+  for (int c : op_columns(op)) {
+    Column& col = *db->cols[(size_t)c];
+    if (col.dev && !col.evict_pending) {
+      db->stats.cache_hits++;
+      continue;
+    }
+    db->stats.cache_misses++;
+    uint64_t need = (uint64_t)std::max<int64_t>(col.n, 1) * col.width;
+    while (db->cache_used + need > db->cfg.cache_bytes) {
+      int victim = -1;
+      uint64_t best = UINT64_MAX;
+      std::vector<int> mine = op_columns(op);
+      for (size_t k = 0; k < db->cols.size(); k++) {
+        const Column& o = *db->cols[k];
+        if (!o.dev || o.refs > 0 || std::find(mine.begin(), mine.end(), (int)k) != mine.end()) continue;
+        if (o.last_access < best) {
+          best = o.last_access;
+          victim = (int)k;
+        }
+      }
+      if (victim < 0) return DDQ_ENOMEM_DEVICE;
+      evict_column_locked(db, victim);
+    }
+    ddq_status s = cache_column_locked(db, c, true);
+    if (s != DDQ_OK) return s;
+  }
+  return DDQ_OK;
+}
+
+static void hold_columns(ddq_db* db, const ddq_op& op, int delta) {
+  std::lock_guard<std::mutex> g(db->mu);
+  for (int c : op_columns(op)) {
+    Column& col = *db->cols[(size_t)c];
+    col.refs += delta;
+    if (delta < 0 && col.refs == 0 && col.evict_pending) evict_column_locked(db, c);
+  }
+}
+
+static void enqueue(ddq_db* db, std::shared_ptr<QueryState> q, int i);
+
+static void finish_query(ddq_db* db, QueryState& q) {
+  const ddq_op& root = q.plan.ops[q.plan.n_ops - 1];
+  Inter& r = q.inters.back();
+  ddq_result* res = nullptr;
+  ddq_status s = DDQ_OK;
+  if (root.kind == DDQ_OP_AGGREGATE) {
+    if (r.on_host) {
+      s = finalize_result(root, r.h_groups, r.h_keys->data(), r.h_accs->data(), &res);
+    } else {
+      cudaStream_t st;
+      cudaSetDevice(db->device);
+      cudaStreamCreateWithFlags(&st, cudaStreamNonBlocking);
+      uint32_t g = 0;
+      uint64_t t0 = now_ns();
+      cudaMemcpyAsync(&g, r.gb_groups, 4, cudaMemcpyDeviceToHost, st);
+      cudaStreamSynchronize(st);
+      std::vector<int64_t> keys(g), accs((size_t)g * root.n_aggs * 2);
+      if (g) {
+        cudaMemcpyAsync(keys.data(), r.gb_keys, (size_t)g * 8, cudaMemcpyDeviceToHost, st);
+        cudaMemcpyAsync(accs.data(), r.gb_accs, (size_t)g * root.n_aggs * 16, cudaMemcpyDeviceToHost, st);
+      }
+      cudaError_t e = cudaStreamSynchronize(st);
+      cudaStreamDestroy(st);
+      db->stats.d2h_bytes += 4 + (uint64_t)g * (8 + 16 * root.n_aggs);
+      db->stats.d2h_ns += now_ns() - t0;
+      s = e == cudaSuccess ? finalize_result(root, g, keys.data(), accs.data(), &res) : cuda_status(e, "fetch");
+    }
+  } else {
+    cudaStream_t st;
+    cudaSetDevice(db->device);
+    cudaStreamCreateWithFlags(&st, cudaStreamNonBlocking);
+    s = inter_to_host(db, r, st);
+    cudaStreamDestroy(st);
+    if (s == DDQ_OK) {
+      res = new ddq_result();
+      std::memset(res, 0, sizeof(*res));
+      int32_t* t = new int32_t[(size_t)std::max<int64_t>(r.count, 1)];
+      const int64_t base = db->tables[(size_t)root.table].row_begin;
+      for (int64_t i = 0; i < r.count; i++) t[i] = (int32_t)(r.tids[i] + base);
+      res->n_tids = r.count;
+      res->tids = t;
+    }
+  }
+  for (auto& x : q.inters) release_inter(db, x);
+  std::lock_guard<std::mutex> g(q.mu);
+  q.status = s;
+  if (s != DDQ_OK) q.error = ddq_last_error();
+  if (res) {
+    res->gpu_ops = q.gpu_ops;
+    res->host_ops = q.host_ops;
+    res->aborts = q.aborts;
+  }
+  q.t_done = now_ns();
+  if (res) res->exec_ms = (double)(q.t_done - q.t_submit) / 1e6;
+  q.result = res;
+  q.done = true;
+  db->stats.queries_done++;
+  q.cv.notify_all();
+}
+
+static void fail_query(ddq_db* db, QueryState& q, ddq_status s) {
+  std::string msg = ddq_last_error();
+  for (auto& x : q.inters) release_inter(db, x);
+  std::lock_guard<std::mutex> g(q.mu);
+  if (q.done) return;
+  q.status = s;
+  q.error = msg;
+  q.done = true;
+  q.cv.notify_all();
+}
+
+// Called when op i of q finished: notify parents, free consumed inputs.
+static void op_finished(ddq_db* db, std::shared_ptr<QueryState> q, int i) {
+  std::vector<int> ready;
+  bool last = false;
+  {
+    std::lock_guard<std::mutex> g(q->mu);
+    for (int p : q->parents[(size_t)i])
+      if (--q->pending[(size_t)p] == 0) ready.push_back(p);
+    // intermediates whose consumers are all done can be released
+    // (a GATHER output aliases its input's TIDs: such inputs live until the query ends)
+    for (int c : op_children(q->plan.ops[i]))
+      if (--q->consumers_left[(size_t)c] == 0 && q->plan.ops[i].kind != DDQ_OP_GATHER)
+        release_inter(db, q->inters[(size_t)c]);
+    last = --q->ops_left == 0;
+  }
+  for (int p : ready) enqueue(db, q, p);
+  if (last) finish_query(db, *q);
+}
+
+static int decide_place(ddq_db* db, QueryState& q, int i) {
+  const ddq_op& op = q.plan.ops[i];
+  if (!db->cfg.chopping && q.place[(size_t)i] != P_NONE) return q.place[(size_t)i];  // compile time
+  switch (db->cfg.placement) {
+    case DDQ_PLACE_CPU_ONLY: return P_HOST;
+    case DDQ_PLACE_GPU_ONLY: return P_GPU;
+    default:  // data-driven, run time
+      return (columns_cached(db, op) && children_on_gpu(q, i)) ? P_GPU : P_HOST;
+  }
+}
+
+static void enqueue(ddq_db* db, std::shared_ptr<QueryState> q, int i) {
+  int where = decide_place(db, *q, i);
+  std::lock_guard<std::mutex> g(db->qmu);
+  if (where == P_GPU) db->gpu_ready.emplace_back(q, i);
+  else db->host_ready.emplace_back(q, i);
+  db->qcv.notify_all();
+}
+
+static void run_on_host(ddq_db* db, std::shared_ptr<QueryState> q, int i, cudaStream_t st) {
+  const ddq_op& op = q->plan.ops[i];
+  for (int c : op_children(op)) {  // data follows the operator to the host
+    ddq_status s = inter_to_host(db, q->inters[(size_t)c], st);
+    if (s != DDQ_OK) {
+      fail_query(db, *q, s);
+      return;
+    }
+  }
+  Inter out;
+  ddq_status s = run_host_op(db, op, q->inters, out);
+  if (s != DDQ_OK) {
+    release_inter(db, out);
+    fail_query(db, *q, s);
+    return;
+  }
+  q->inters[(size_t)i] = std::move(out);
+  q->host_ops++;
+  db->stats.host_ops++;
+  op_finished(db, q, i);
+}
+
+static void run_on_gpu(ddq_db* db, std::shared_ptr<QueryState> q, int i, cudaStream_t st) {
+  const ddq_op& op = q->plan.ops[i];
+  const uint64_t t0 = now_ns();
+  ddq_status s = DDQ_OK;
+  if (db->cfg.placement == DDQ_PLACE_GPU_ONLY || !db->cfg.chopping) s = ensure_cached_lru(db, op);
+  bool abort = s == DDQ_ENOMEM_DEVICE;
+  if (s != DDQ_OK && !abort) {
+    fail_query(db, *q, s);
+    return;
+  }
+  if (!abort) {
+    for (int c : op_children(op)) {  // compile-time arm: copy host data back (Fig. 8)
+      s = inter_to_device(db, q->inters[(size_t)c], st);
+      if (s == DDQ_ENOMEM_DEVICE) {
+        abort = true;
+        break;
+      }
+      if (s != DDQ_OK) {
+        fail_query(db, *q, s);
+        return;
+      }
+    }
+  }
+  if (!abort && !columns_cached(db, op)) abort = true;  // evicted meanwhile: follow the data
+  Inter out;
+  if (!abort) {
+    hold_columns(db, op, +1);
+    GpuOpCtx ctx{db, st, &q->inters};
+    s = run_gpu_op(ctx, op, out);
+    if (s == DDQ_OK) {
+      cudaError_t e = cudaStreamSynchronize(st);
+      if (e != cudaSuccess) s = cuda_status(e, "gpu op");
+    }
+    hold_columns(db, op, -1);
+    if (s == DDQ_OK && out.d_count && op.kind != DDQ_OP_GATHER) {
+      uint32_t c = 0;
+      cudaMemcpy(&c, out.d_count, 4, cudaMemcpyDeviceToHost);
+      out.count = c;
+      out.cap = c;  // exact cardinality is known at run time: consumers allocate exactly
+    }
+    if (s == DDQ_OK && out.table_ptr && out.d_error) {
+      uint32_t e2 = 0;
+      cudaMemcpy(&e2, out.d_error, 4, cudaMemcpyDeviceToHost);
+      if (e2) s = set_error(e2 == 2 ? DDQ_EOVERFLOW : DDQ_EINVAL, "hash build failed (duplicate key or overflow)");
+    }
+    if (s == DDQ_ENOMEM_DEVICE) {
+      abort = true;
+      release_inter(db, out);
+    } else if (s != DDQ_OK) {
+      release_inter(db, out);
+      fail_query(db, *q, s);
+      return;
+    }
+  }
+  if (abort) {  // abort immediately, restart on the host
+    q->aborts++;
+    db->stats.aborts++;
+    db->stats.wasted_ns += now_ns() - t0;
+    run_on_host(db, q, i, st);
+    return;
+  }
+  if (op.kind == DDQ_OP_GATHER) out.count = q->inters[(size_t)op.input].count;
+  q->inters[(size_t)i] = std::move(out);
+  q->gpu_ops++;
+  db->stats.gpu_ops++;
+  op_finished(db, q, i);
+}
+
+static void worker_loop(ddq_db* db, bool gpu) {
+  cudaSetDevice(db->device);
+  cudaStream_t st;
+  cudaStreamCreateWithFlags(&st, cudaStreamNonBlocking);
+  while (true) {
+    std::shared_ptr<QueryState> q;
+    int i = -1;
+    {
+      std::unique_lock<std::mutex> g(db->qmu);
+      auto& Q = gpu ? db->gpu_ready : db->host_ready;
+      db->qcv.wait(g, [&] { return db->stopping || !Q.empty(); });
+      if (db->stopping) break;
+      q = Q.front().first;
+      i = Q.front().second;
+      Q.pop_front();
+    }
+    {
+      std::lock_guard<std::mutex> g(q->mu);
+      if (q->done) continue;  // failed query: drop remaining ops
+    }
+    if (gpu) run_on_gpu(db, q, i, st);
+    else run_on_host(db, q, i, st);
+  }
+  cudaStreamDestroy(st);
+}
+
+void driver_start(ddq_db* db) {
+  // chopping: a bounded pool pulls GPU operators; without chopping
+  // every operator gets its own thread (unbounded inter-operator parallelism).
+  int g = db->cfg.chopping ? db->cfg.gpu_workers : 64;
+  int h = db->cfg.chopping ? db->cfg.host_workers : std::max(db->cfg.host_workers, 16);
+  for (int i = 0; i < g; i++) db->workers.emplace_back(worker_loop, db, true);
+  for (int i = 0; i < h; i++) db->workers.emplace_back(worker_loop, db, false);
+}
+
+void driver_stop(ddq_db* db) {
+  {
+    std::lock_guard<std::mutex> g(db->qmu);
+    db->stopping = true;
+    db->qcv.notify_all();
+  }
+  for (auto& t : db->workers) t.join();
+  db->workers.clear();
+  for (auto& kv : db->queries) {
+    for (auto& x : kv.second->inters) release_inter(db, x);
+    if (kv.second->result) ddq_result_free(kv.second->result);
+  }
+  db->queries.clear();
+}
+
+}  // namespace ddq
+
+using namespace ddq;
+
+extern "C" {
+
+ddq_status ddq_submit(ddq_db* db, const ddq_plan* plan, ddq_query* out) {
+  if (!db || !out) return set_error(DDQ_EINVAL, "submit: null argument");
+  if (ddq_status s = validate_plan_public(db, plan)) return s;
+  auto q = std::make_shared<QueryState>();
+  q->plan = *plan;  // plans are copied at submit (S8(b))
+  const int n = plan->n_ops;
+  q->inters.resize((size_t)n);
+  q->pending.assign((size_t)n, 0);
+  q->parents.assign((size_t)n, {});
+  q->consumers_left.assign((size_t)n, 0);
+  q->place.assign((size_t)n, P_NONE);
+  q->ops_left = n;
+  q->t_submit = now_ns();
+  for (int i = 0; i < n; i++)
+    for (int c : op_children(plan->ops[i])) {
+      q->pending[(size_t)i]++;
+      q->parents[(size_t)c].push_back(i);
+      q->consumers_left[(size_t)c]++;
+    }
+  if (!db->cfg.chopping) {  // compile-time placement from the cache state at submit
+    for (int i = 0; i < n; i++) {
+      if (db->cfg.placement == DDQ_PLACE_CPU_ONLY) q->place[(size_t)i] = P_HOST;
+      else if (db->cfg.placement == DDQ_PLACE_GPU_ONLY) q->place[(size_t)i] = P_GPU;
+      else {
+        bool ok = columns_cached(db, plan->ops[i]);
+        for (int c : op_children(plan->ops[i])) ok = ok && q->place[(size_t)c] == P_GPU;
+        q->place[(size_t)i] = ok ? P_GPU : P_HOST;
+      }
+    }
+  }
+  {
+    std::lock_guard<std::mutex> g(db->qmu);
+    q->id = db->next_query++;
+    db->queries[q->id] = q;
+  }
+  *out = q->id;
+  // leaf operators enter the global operator stream
+  for (int i = 0; i < n; i++)
+    if (q->pending[(size_t)i] == 0) enqueue(db, q, i);
+  return DDQ_OK;
+}
+
+ddq_status ddq_wait(ddq_db* db, ddq_query id, int64_t timeout_ns) {
+  if (!db) return set_error(DDQ_EINVAL, "wait: null");
+  std::shared_ptr<QueryState> q;
+  {
+    std::lock_guard<std::mutex> g(db->qmu);
+    auto it = db->queries.find(id);
+    if (it == db->queries.end()) return set_error(DDQ_ENOTFOUND, "wait: unknown query");
+    q = it->second;
+  }
+  std::unique_lock<std::mutex> g(q->mu);
+  if (timeout_ns < 0) q->cv.wait(g, [&] { return q->done; });
+  else if (!q->cv.wait_for(g, std::chrono::nanoseconds(timeout_ns), [&] { return q->done; }))
+    return set_error(DDQ_ETIMEOUT, "wait: timeout");
+  if (q->status != DDQ_OK) return set_error(q->status, q->error);
+  return DDQ_OK;
+}
+
+ddq_status ddq_fetch(ddq_db* db, ddq_query id, ddq_result** out) {
+  if (!db || !out) return set_error(DDQ_EINVAL, "fetch: null");
+  std::shared_ptr<QueryState> q;
+  {
+    std::lock_guard<std::mutex> g(db->qmu);
+    auto it = db->queries.find(id);
+    if (it == db->queries.end()) return set_error(DDQ_ENOTFOUND, "fetch: unknown query");
+    q = it->second;
+  }
+  std::unique_lock<std::mutex> g(q->mu);
+  q->cv.wait(g, [&] { return q->done; });
+  if (q->status != DDQ_OK) return set_error(q->status, q->error);
+  *out = q->result;
+  q->result = nullptr;
+  g.unlock();
+  std::lock_guard<std::mutex> g2(db->qmu);
+  db->queries.erase(id);
+  return DDQ_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,1109 @@
+// engine.cpp -- libddq database: column store, device column cache (Algorithm 1),
+// heap-budget allocator, GPU operator runner, finalisation and prepared
+// (CUDA-graph) plans.  Citations: P:n = PAPER.md line n.
+#include <algorithm>
+#include <chrono>
+#include <cmath>
+#include <cstring>
+#include <numeric>
+
+#include "engine.h"
+#include "ops_internal.h"
+
+namespace ddq {
+
+uint64_t now_ns() {
+  return (uint64_t)std::chrono::duration_cast<std::chrono::nanoseconds>(
+             std::chrono::steady_clock::now().time_since_epoch())
+      .count();
+}
+
+int64_t pow2_at_least(int64_t x) {
+  int64_t p = 1;
+  while (p < x) p <<= 1;
+  return p;
+}
+
+// ---------------------------------------------------------------- heap
+// The rest of device memory after the cache is the heap for intermediates.
+// Allocation never waits: it fails immediately so the operator can abort and be
+// restarted elsewhere ("CoGaDB aborts operators immediately if an
+// allocation fails").
+static constexpr uint64_t kAlign = 256;
+
+ddq_status Heap::init(uint64_t bytes, uint32_t fault_every) {
+  cap_ = (bytes + kAlign - 1) / kAlign * kAlign;
+  fault_every_ = fault_every;
+  if (cap_ == 0) return DDQ_OK;
+  cudaError_t e = cudaMalloc(&base_, cap_);
+  if (e != cudaSuccess) return cuda_status(e, "heap cudaMalloc");
+  free_[0] = cap_;
+  return DDQ_OK;
+}
+
+Heap::~Heap() {
+  if (base_) cudaFree(base_);
+}
+
+void* Heap::try_alloc(uint64_t bytes) {
+  std::lock_guard<std::mutex> g(mu_);
+  n_allocs_++;
+  if (fault_every_ && n_allocs_ % fault_every_ == 0) return nullptr;  // fault injection
+  uint64_t need = std::max<uint64_t>(kAlign, (bytes + kAlign - 1) / kAlign * kAlign);
+  for (auto it = free_.begin(); it != free_.end(); ++it) {
+    if (it->second < need) continue;
+    uint64_t off = it->first, sz = it->second;
+    free_.erase(it);
+    if (sz > need) free_[off + need] = sz - need;
+    alloc_[off] = need;
+    used_ += need;
+    peak_ = std::max(peak_, used_);
+    return base_ + off;
+  }
+  return nullptr;
+}
+
+void Heap::free(void* p) {
+  if (!p) return;
+  std::lock_guard<std::mutex> g(mu_);
+  uint64_t off = (uint64_t)((char*)p - base_);
+  auto it = alloc_.find(off);
+  if (it == alloc_.end()) return;
+  uint64_t sz = it->second;
+  alloc_.erase(it);
+  used_ -= sz;
+  auto nx = free_.lower_bound(off);
+  if (nx != free_.end() && nx->first == off + sz) {
+    sz += nx->second;
+    nx = free_.erase(nx);
+  }
+  if (nx != free_.begin()) {
+    auto pv = std::prev(nx);
+    if (pv->first + pv->second == off) {
+      pv->second += sz;
+      return;
+    }
+  }
+  free_[off] = sz;
+}
+
+const Column* col_of(ddq_db* db, int c) {
+  if (c < 0 || c >= (int)db->cols.size()) return nullptr;
+  return db->cols[(size_t)c].get();
+}
+
+void release_inter(ddq_db* db, Inter& x) {
+  for (void* p : x.heap_blocks) db->heap.free(p);
+  for (void* p : x.host_blocks) std::free(p);
+  x.heap_blocks.clear();
+  x.host_blocks.clear();
+}
+
+// ----------------------------------------------------------- GPU operator runner
+struct Alloc {
+  ddq_db* db;
+  Inter* out;
+  const std::vector<void*>* reuse = nullptr;  // replay: hand back these blocks in order
+  size_t next = 0;
+  bool failed = false;
+  void* get(uint64_t bytes) {
+    if (failed) return nullptr;
+    if (reuse) {
+      if (next >= reuse->size()) {
+        failed = true;
+        return nullptr;
+      }
+      void* p = (*reuse)[next++];
+      out->heap_blocks.push_back(p);
+      return p;
+    }
+    void* p = db->heap.try_alloc(bytes);
+    if (!p) {
+      failed = true;
+      return nullptr;
+    }
+    out->heap_blocks.push_back(p);
+    return p;
+  }
+};
+
+static const void* dev_col(ddq_db* db, int c, bool count_access) {
+  const Column* col = col_of(db, c);
+  if (!col) return nullptr;
+  if (count_access) {
+    db->cols[(size_t)c]->access++;
+    db->cols[(size_t)c]->last_access = ++db->clock;
+  }
+  return col->dev;
+}
+
+ddq_status run_gpu_op(GpuOpCtx& ctx, const ddq_op& op, Inter& out) {
+  ddq_db* db = ctx.db;
+  const std::vector<Inter>& I = *ctx.inters;
+  cudaStream_t st = ctx.stream;
+  const bool acc = ctx.count_column_access;
+  Alloc A{db, &out};
+  A.reuse = ctx.reuse;
+  out = Inter();
+  out.table = op.table;
+  if (op.table < 0 || op.table >= (int)db->tables.size()) return set_error(DDQ_EINVAL, "op: bad table");
+  const Table& T = db->tables[(size_t)op.table];
+  const Inter* in = op.input >= 0 ? &I[(size_t)op.input] : nullptr;
+  if (in && in->on_host) return set_error(DDQ_ESTATE, "GPU op with a host-resident input");
+  const int32_t* in_tids = in ? in->tids : nullptr;
+  const uint32_t* in_cnt = in ? in->d_count : nullptr;
+  const int64_t in_cap = in ? in->cap : T.n_rows;
+  const int64_t out_cap = ctx.forced_cap >= 0 ? std::min<int64_t>(ctx.forced_cap, in_cap) : in_cap;
+  auto need_col = [&](int c) -> const void* {
+    const void* p = dev_col(db, c, acc);
+    return p;
+  };
+  switch (op.kind) {
+    case DDQ_OP_SELECT:
+    case DDQ_OP_HASH_PROBE: {
+      const bool probe = op.kind == DDQ_OP_HASH_PROBE;
+      ddq_dev_pred dp[DDQ_MAX_PREDS];
+      std::memset(dp, 0, sizeof(dp));
+      if (!probe) {
+        if (op.n_preds < 0 || op.n_preds > DDQ_MAX_PREDS) return set_error(DDQ_EINVAL, "select: bad n_preds");
+        for (int i = 0; i < op.n_preds; i++) {
+          const ddq_pred& p = op.preds[i];
+          const Column* c = col_of(db, p.column);
+          if (!c || c->table != op.table) return set_error(DDQ_EINVAL, "select: predicate column not in table");
+          dp[i].col = need_col(p.column);
+          if (!dp[i].col) return set_error(DDQ_ESTATE, "select: column not cached on the GPU");
+          dp[i].width = c->width;
+          dp[i].kind = p.kind;
+          dp[i].lo = p.lo;
+          dp[i].hi = p.hi;
+          dp[i].n_in = p.n_in;
+          for (int j = 0; j < DDQ_MAX_IN; j++) dp[i].in_vals[j] = p.in_vals[j];
+        }
+      }
+      const Inter* build = nullptr;
+      const int32_t* fk = nullptr;
+      if (probe) {
+        if (op.build < 0 || op.build >= (int)I.size()) return set_error(DDQ_EINVAL, "probe: bad build index");
+        build = &I[(size_t)op.build];
+        if (!build->table_ptr) return set_error(DDQ_ESTATE, "probe: build side is not a device hash table");
+        const Column* c = col_of(db, op.fk_col);
+        if (!c || c->table != op.table || c->width != 4) return set_error(DDQ_EINVAL, "probe: bad fk column");
+        fk = (const int32_t*)need_col(op.fk_col);
+        if (!fk) return set_error(DDQ_ESTATE, "probe: fk column not cached on the GPU");
+      }
+      // carried vectors (int32 only; int64 vectors are re-gathered by consumers)
+      std::vector<const int32_t*> cin;
+      std::vector<int32_t*> cout;
+      if (in) {
+        if (in->vecs.size() > DDQ_MAX_CARRY) return set_error(DDQ_EINVAL, "too many aligned vectors");
+        for (const Vec& v : in->vecs) {
+          if (v.width != 4) return set_error(DDQ_EINVAL, "only int32 vectors can be carried");
+          cin.push_back((const int32_t*)v.ptr);
+        }
+      }
+      out.cap = out_cap;
+      out.tids = (int32_t*)A.get((uint64_t)std::max<int64_t>(out_cap, 1) * 4);
+      out.d_count = (uint32_t*)A.get(64);
+      for (size_t c = 0; c < cin.size(); c++) {
+        int32_t* p = (int32_t*)A.get((uint64_t)std::max<int64_t>(out_cap, 1) * 4);
+        cout.push_back(p);
+        out.vecs.push_back(Vec{p, 4, false});
+      }
+      int32_t* payload = nullptr;
+      if (probe && op.emit_payload) {
+        payload = (int32_t*)A.get((uint64_t)std::max<int64_t>(out_cap, 1) * 4);
+        out.vecs.push_back(Vec{payload, 4, false});
+      }
+      size_t sb = filter_scratch_bytes(in_cap);
+      void* scratch = A.get(sb);
+      if (A.failed) return DDQ_ENOMEM_DEVICE;
+      FilterArgs fa;
+      fa.preds = dp;
+      fa.n_preds = probe ? 0 : op.n_preds;
+      fa.probe = probe;
+      if (probe) {
+        fa.table = build->table_ptr;
+        fa.capacity = build->table_cap;
+        fa.fk = fk;
+        fa.out_payload = payload;
+      }
+      fa.in_tids = in_tids;
+      fa.d_in_count = in_cnt;
+      fa.n_cap = in_cap;
+      fa.carry_in = cin.data();
+      fa.carry_out = cout.data();
+      fa.n_carry = (int)cin.size();
+      fa.out_tids = out.tids;
+      fa.d_out_count = out.d_count;
+      fa.out_cap = out_cap;
+      fa.d_overflow = ctx.forced_cap >= 0 && in && in->d_error ? in->d_error : nullptr;
+      fa.scratch = scratch;
+      // error cell propagates down the chain so a prepared plan can detect overflow
+      out.d_error = in ? in->d_error : nullptr;
+      if (!out.d_error) {
+        out.d_error = (uint32_t*)A.get(64);
+        if (A.failed) return DDQ_ENOMEM_DEVICE;
+        cudaMemsetAsync(out.d_error, 0, 4, st);
+      }
+      fa.d_overflow = out.d_error;
+      return cuda_status(launch_filter(fa, st), probe ? "probe" : "select");
+    }
+    case DDQ_OP_HASH_BUILD: {
+      const Column* kc = col_of(db, op.key_col);
+      if (!kc || kc->table != op.table || kc->width != 4) return set_error(DDQ_EINVAL, "build: bad key column");
+      const int32_t* keys = (const int32_t*)need_col(op.key_col);
+      const int32_t* payload = nullptr;
+      if (op.payload_col >= 0) {
+        const Column* pc = col_of(db, op.payload_col);
+        if (!pc || pc->table != op.table || pc->width != 4) return set_error(DDQ_EINVAL, "build: bad payload column");
+        payload = (const int32_t*)need_col(op.payload_col);
+        if (!payload) return set_error(DDQ_ESTATE, "build: payload column not cached on the GPU");
+      }
+      if (!keys) return set_error(DDQ_ESTATE, "build: key column not cached on the GPU");
+      int64_t cap = pow2_at_least(std::max<int64_t>(16, 2 * out_cap));
+      if (cap > (1ll << 31)) return set_error(DDQ_EINVAL, "build: table too large");
+      out.table_cap = (uint32_t)cap;
+      out.table_ptr = (uint64_t*)A.get((uint64_t)cap * 8);
+      out.d_error = (uint32_t*)A.get(64);
+      out.cap = 0;
+      if (A.failed) return DDQ_ENOMEM_DEVICE;
+      cudaMemsetAsync(out.d_error, 0, 4, st);
+      cudaError_t e = launch_hash_init(out.table_ptr, out.table_cap, st);
+      if (e == cudaSuccess)
+        e = launch_hash_build(keys, payload, in_tids, in_cnt, in_cap, out.table_ptr, out.table_cap, out.d_error, st);
+      return cuda_status(e, "hash_build");
+    }
+    case DDQ_OP_GATHER: {
+      const Column* c = col_of(db, op.gather_col);
+      if (!c || c->table != op.table) return set_error(DDQ_EINVAL, "gather: bad column");
+      if (!in) return set_error(DDQ_EINVAL, "gather needs an input TID list");
+      const void* src = need_col(op.gather_col);
+      if (!src) return set_error(DDQ_ESTATE, "gather: column not cached on the GPU");
+      // pass-through of the input's TIDs and vectors (no copy), plus the new vector
+      out.tids = in->tids;
+      out.d_count = in->d_count;
+      out.cap = in->cap;
+      out.vecs = in->vecs;
+      out.d_error = in->d_error;
+      void* dst = A.get((uint64_t)std::max<int64_t>(in->cap, 1) * c->width);
+      if (A.failed) return DDQ_ENOMEM_DEVICE;
+      out.vecs.push_back(Vec{dst, c->width, false});
+      return cuda_status(launch_gather(src, c->width, in->tids, in->d_count, in->cap, dst, st), "gather");
+    }
+    case DDQ_OP_AGGREGATE: {
+      if (!in) return set_error(DDQ_EINVAL, "aggregate needs an input TID list");
+      if (op.n_keys < 0 || op.n_keys > DDQ_MAX_KEYS || op.n_aggs < 1 || op.n_aggs > DDQ_MAX_AGGS)
+        return set_error(DDQ_EINVAL, "aggregate: bad key/agg counts");
+      const int32_t* kv[3] = {nullptr, nullptr, nullptr};
+      const int32_t* kc[3] = {nullptr, nullptr, nullptr};
+      for (int k = 0; k < op.n_keys; k++) {
+        int src = op.key_src[k];
+        if (src >= 0) {
+          if (src >= (int)in->vecs.size() || in->vecs[(size_t)src].width != 4)
+            return set_error(DDQ_EINVAL, "aggregate: bad key vector");
+          kv[k] = (const int32_t*)in->vecs[(size_t)src].ptr;
+        } else {
+          const Column* c = col_of(db, -2 - src);
+          if (!c || c->table != op.table || c->width != 4) return set_error(DDQ_EINVAL, "aggregate: bad key column");
+          kc[k] = (const int32_t*)need_col(-2 - src);
+          if (!kc[k]) return set_error(DDQ_ESTATE, "aggregate: key column not cached");
+        }
+      }
+      ddq_dev_agg ag[DDQ_MAX_AGGS];
+      std::memset(ag, 0, sizeof(ag));
+      for (int a = 0; a < op.n_aggs; a++) {
+        ag[a].kind = op.agg_kind[a];
+        int need = op.agg_kind[a] == DDQ_AGG_COUNT ? 0 : op.agg_kind[a] == DDQ_AGG_SUM ? 1
+                 : op.agg_kind[a] == DDQ_AGG_SUM_MUL_100M_100P ? 3 : 2;
+        for (int j = 0; j < need; j++) {
+          const Column* c = col_of(db, op.agg_col[a][j]);
+          if (!c || c->table != op.table) return set_error(DDQ_EINVAL, "aggregate: bad argument column");
+          ag[a].arg[j] = need_col(op.agg_col[a][j]);
+          ag[a].width[j] = c->width;
+          if (!ag[a].arg[j]) return set_error(DDQ_ESTATE, "aggregate: argument column not cached");
+        }
+      }
+      int64_t groups = op.max_groups > 0 ? std::min<int64_t>(op.max_groups, std::max<int64_t>(in->cap, 1))
+                                         : std::max<int64_t>(in->cap, 1);
+      int64_t cap = pow2_at_least(std::max<int64_t>(64, 2 * groups));
+      if (cap > (1ll << 31)) return set_error(DDQ_EINVAL, "aggregate: table too large");
+      out.gb_cap = (uint32_t)cap;
+      out.gb_table = A.get(groupby_table_bytes(out.gb_cap, op.n_aggs));
+      out.gb_keys = (int64_t*)A.get((uint64_t)cap * 8);
+      out.gb_accs = (int64_t*)A.get((uint64_t)cap * op.n_aggs * 16);
+      out.gb_groups = (uint32_t*)A.get(64);
+      out.d_error = in->d_error;
+      if (!out.d_error) {
+        out.d_error = (uint32_t*)A.get(64);
+        if (!A.failed) cudaMemsetAsync(out.d_error, 0, 4, st);
+      }
+      if (A.failed) return DDQ_ENOMEM_DEVICE;
+      cudaError_t e = launch_groupby_init(out.gb_table, out.gb_cap, op.n_aggs, st);
+      if (e == cudaSuccess)
+        e = launch_groupby(in->tids, in->d_count, in->cap, kv, kc, op.n_keys, ag, op.n_aggs, out.gb_table,
+                           out.gb_cap, out.d_error, st);
+      if (e == cudaSuccess)
+        e = launch_groupby_compact(out.gb_table, out.gb_cap, op.n_aggs, out.gb_keys, out.gb_accs, out.gb_groups, st);
+      return cuda_status(e, "aggregate");
+    }
+  }
+  return set_error(DDQ_EINVAL, "unknown operator kind");
+}
+
+// ------------------------------------------------------------ finalisation
+// S8(a7): decode the packed group key, ORDER BY (order-preserving codes, O4; the
+// O8 tie-break = remaining keys ascending is encoded in the plan), LIMIT.
+static inline __int128 acc128(const int64_t* accs, int64_t g, int n_aggs, int a) {
+  unsigned __int128 lo = (uint64_t)accs[(g * n_aggs + a) * 2];
+  __int128 hi = (__int128)accs[(g * n_aggs + a) * 2 + 1];
+  return (__int128)((unsigned __int128)(hi << 64) | lo);
+}
+
+ddq_status finalize_result(const ddq_op& root, int64_t n_groups, const int64_t* keys, const int64_t* accs,
+                           ddq_result** out) {
+  const int nk = root.n_keys, na = root.n_aggs;
+  std::vector<int64_t> idx((size_t)n_groups);
+  std::iota(idx.begin(), idx.end(), 0);
+  auto keyk = [&](int64_t g, int k) { return (keys[g] >> (21 * k)) & ((1ll << 21) - 1); };
+  std::sort(idx.begin(), idx.end(), [&](int64_t a, int64_t b) {
+    for (int o = 0; o < root.n_order; o++) {
+      int e = root.order_by[o];
+      bool desc = e < 0;
+      int v = desc ? -e : e;
+      int c = 0;
+      if (v >= 101) {
+        __int128 x = acc128(accs, a, na, v - 101), y = acc128(accs, b, na, v - 101);
+        c = x < y ? -1 : x > y ? 1 : 0;
+      } else {
+        int64_t x = keyk(a, v - 1), y = keyk(b, v - 1);
+        c = x < y ? -1 : x > y ? 1 : 0;
+      }
+      if (desc) c = -c;
+      if (c) return c < 0;
+    }
+    return keys[a] < keys[b];  // deterministic residual order
+  });
+  int64_t n = n_groups;
+  if (root.limit > 0 && n > root.limit) n = root.limit;
+  ddq_result* r = new ddq_result();
+  std::memset(r, 0, sizeof(*r));
+  int64_t* k = new int64_t[(size_t)std::max<int64_t>(1, n * nk)];
+  int64_t* a = new int64_t[(size_t)std::max<int64_t>(1, n * na * 2)];
+  for (int64_t i = 0; i < n; i++) {
+    int64_t g = idx[(size_t)i];
+    for (int j = 0; j < nk; j++) k[i * nk + j] = keyk(g, j);
+    for (int j = 0; j < na; j++) {
+      a[(i * na + j) * 2] = accs[(g * na + j) * 2];
+      a[(i * na + j) * 2 + 1] = accs[(g * na + j) * 2 + 1];
+    }
+  }
+  r->n_rows = n;
+  r->n_keys = nk;
+  r->n_aggs = na;
+  r->keys = k;
+  r->aggs = a;
+  *out = r;
+  return DDQ_OK;
+}
+
+}  // namespace ddq
+
+using namespace ddq;
+
+// ======================================================================= C ABI
+extern "C" {
+
+void ddq_config_default(ddq_config* c) {
+  std::memset(c, 0, sizeof(*c));
+  c->device = 0;
+  c->rank = 0;
+  c->world = 1;
+  c->cache_bytes = 64ull << 30;
+  c->heap_bytes = 32ull << 30;
+  c->gpu_workers = 4;  // O17
+  c->host_workers = 4;
+  c->placement = DDQ_PLACE_DATA_DRIVEN;
+  c->chopping = 1;
+  c->cache_policy = 0;
+  c->fault_alloc_every = 0;
+}
+
+
+ddq_status ddq_open(const ddq_config* cfg, ddq_db** out) {
+  if (!cfg || !out) return set_error(DDQ_EINVAL, "ddq_open: null argument");
+  ddq_db* db = new ddq_db();
+  db->cfg = *cfg;
+  if (db->cfg.gpu_workers < 1) db->cfg.gpu_workers = 1;
+  if (db->cfg.host_workers < 1) db->cfg.host_workers = 1;
+  int ndev = 0;
+  cudaError_t e = cudaGetDeviceCount(&ndev);
+  if (e != cudaSuccess || ndev == 0) {
+    delete db;
+    return set_error(DDQ_ECUDA, "ddq_open: no CUDA device (the product path has no CPU fallback)");
+  }
+  if (cfg->device < 0 || cfg->device >= ndev) {
+    delete db;
+    return set_error(DDQ_EINVAL, "ddq_open: bad device ordinal");
+  }
+  db->device = cfg->device;
+  cudaSetDevice(db->device);
+  e = cudaStreamCreateWithFlags(&db->copy_stream, cudaStreamNonBlocking);
+  if (e != cudaSuccess) {
+    delete db;
+    return cuda_status(e, "ddq_open stream");
+  }
+  ddq_status s = db->heap.init(cfg->heap_bytes, cfg->fault_alloc_every);
+  if (s != DDQ_OK) {
+    delete db;
+    return s;
+  }
+  ddq::driver_start(db);
+  *out = db;
+  return DDQ_OK;
+}
+
+void ddq_close(ddq_db* db) {
+  if (!db) return;
+  ddq::driver_stop(db);
+  cudaSetDevice(db->device);
+  cudaDeviceSynchronize();
+  for (auto& c : db->cols) {
+    if (c->dev) cudaFree(c->dev);
+    if (c->host) cudaFreeHost(c->host);
+  }
+  if (db->copy_stream) cudaStreamDestroy(db->copy_stream);
+  delete db;
+}
+
+ddq_status ddq_create_table(ddq_db* db, const char* name, int64_t n_rows, int64_t row_begin, ddq_table* out) {
+  if (!db || !name || n_rows < 0 || n_rows > INT32_MAX || !out) return set_error(DDQ_EINVAL, "create_table");
+  std::lock_guard<std::mutex> g(db->mu);
+  for (auto& t : db->tables)
+    if (t.name == name) return set_error(DDQ_EINVAL, "table exists");
+  Table t;
+  t.name = name;
+  t.n_rows = n_rows;
+  t.row_begin = row_begin;
+  db->tables.push_back(t);
+  *out = (ddq_table)(db->tables.size() - 1);
+  return DDQ_OK;
+}
+
+ddq_status ddq_load_column(ddq_db* db, ddq_table t, const char* name, ddq_type type, const void* host_data,
+                           int64_t n_rows, ddq_column* out) {
+  if (!db || !name || !host_data || !out) return set_error(DDQ_EINVAL, "load_column: null argument");
+  if (type != DDQ_I32 && type != DDQ_I64) return set_error(DDQ_EINVAL, "load_column: bad type");
+  std::lock_guard<std::mutex> g(db->mu);
+  if (t < 0 || t >= (int)db->tables.size()) return set_error(DDQ_ENOTFOUND, "load_column: bad table");
+  if (n_rows != db->tables[(size_t)t].n_rows) return set_error(DDQ_EINVAL, "load_column: row count mismatch");
+  auto c = std::make_unique<Column>();
+  c->name = name;
+  c->table = t;
+  c->type = type;
+  c->width = type == DDQ_I32 ? 4 : 8;
+  c->n = n_rows;
+  size_t bytes = (size_t)std::max<int64_t>(n_rows, 1) * c->width;
+  cudaError_t e = cudaHostAlloc(&c->host, bytes, cudaHostAllocPortable);
+  if (e != cudaSuccess) return set_error(DDQ_ENOMEM_HOST, "load_column: pinned alloc failed");
+  std::memcpy(c->host, host_data, (size_t)n_rows * c->width);
+  db->cols.push_back(std::move(c));
+  int id = (int)db->cols.size() - 1;
+  db->tables[(size_t)t].cols.push_back(id);
+  *out = id;
+  return DDQ_OK;
+}
+
+ddq_status ddq_find_column(ddq_db* db, const char* table, const char* name, ddq_column* out) {
+  if (!db || !table || !name || !out) return set_error(DDQ_EINVAL, "find_column");
+  std::lock_guard<std::mutex> g(db->mu);
+  for (size_t t = 0; t < db->tables.size(); t++) {
+    if (db->tables[t].name != table) continue;
+    for (int c : db->tables[t].cols)
+      if (db->cols[(size_t)c]->name == name) {
+        *out = c;
+        return DDQ_OK;
+      }
+  }
+  return set_error(DDQ_ENOTFOUND, std::string("column ") + table + "." + name);
+}
+
+}  // extern "C"
+
+namespace ddq {
+// H2D copy of one column into the cache (caller holds db->mu).
+ddq_status cache_column_locked(ddq_db* db, int c, bool on_demand) {
+  Column& col = *db->cols[(size_t)c];
+  if (col.dev) {
+    col.evict_pending = false;
+    return DDQ_OK;
+  }
+  uint64_t bytes = (uint64_t)std::max<int64_t>(col.n, 1) * col.width;
+  if (db->cache_used + bytes > db->cfg.cache_bytes)
+    return set_error(DDQ_ENOMEM_DEVICE, "cache budget exceeded for " + col.name);
+  cudaSetDevice(db->device);
+  void* p = nullptr;
+  cudaError_t e = cudaMalloc(&p, bytes);
+  if (e != cudaSuccess) return cuda_status(e, "cache cudaMalloc");
+  uint64_t t0 = now_ns();
+  e = cudaMemcpyAsync(p, col.host, (size_t)col.n * col.width, cudaMemcpyHostToDevice, db->copy_stream);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(db->copy_stream);
+  if (e != cudaSuccess) {
+    cudaFree(p);
+    return cuda_status(e, "cache H2D");
+  }
+  db->stats.h2d_ns += now_ns() - t0;
+  db->stats.h2d_bytes += (uint64_t)col.n * col.width;
+  col.dev = p;
+  col.on_demand = on_demand;
+  col.evict_pending = false;
+  db->cache_used += bytes;
+  return DDQ_OK;
+}
+
+// Evict (deferred while running operators hold references).
+void evict_column_locked(ddq_db* db, int c) {
+  Column& col = *db->cols[(size_t)c];
+  if (!col.dev) return;
+  if (col.refs > 0) {
+    col.evict_pending = true;
+    return;
+  }
+  cudaFree(col.dev);
+  col.dev = nullptr;
+  col.evict_pending = false;
+  db->cache_used -= (uint64_t)std::max<int64_t>(col.n, 1) * col.width;
+}
+}  // namespace ddq
+
+extern "C" {
+
+ddq_status ddq_cache_column(ddq_db* db, ddq_column c) {
+  if (!db || c < 0 || c >= (int)db->cols.size()) return set_error(DDQ_ENOTFOUND, "cache_column");
+  std::lock_guard<std::mutex> g(db->mu);
+  return cache_column_locked(db, c, false);
+}
+
+ddq_status ddq_evict_column(ddq_db* db, ddq_column c) {
+  if (!db || c < 0 || c >= (int)db->cols.size()) return set_error(DDQ_ENOTFOUND, "evict_column");
+  std::lock_guard<std::mutex> g(db->mu);
+  evict_column_locked(db, c);
+  return DDQ_OK;
+}
+
+int32_t ddq_column_is_cached(ddq_db* db, ddq_column c) {
+  if (!db || c < 0 || c >= (int)db->cols.size()) return 0;
+  std::lock_guard<std::mutex> g(db->mu);
+  return db->cols[(size_t)c]->dev && !db->cols[(size_t)c]->evict_pending ? 1 : 0;
+}
+
+const void* ddq_column_device_ptr(ddq_db* db, ddq_column c) {
+  if (!db || c < 0 || c >= (int)db->cols.size()) return nullptr;
+  std::lock_guard<std::mutex> g(db->mu);
+  return db->cols[(size_t)c]->dev;
+}
+
+uint64_t ddq_column_access_count(ddq_db* db, ddq_column c) {
+  if (!db || c < 0 || c >= (int)db->cols.size()) return 0;
+  return db->cols[(size_t)c]->access.load();
+}
+
+ddq_status ddq_reset_access_counts(ddq_db* db) {
+  if (!db) return set_error(DDQ_EINVAL, "reset_access_counts");
+  for (auto& c : db->cols) c->access = 0;
+  return DDQ_OK;
+}
+
+// Algorithm 1 (Sec. 3.2).  LFU by access count (cache_policy 0) or
+// LRU by last access (policy 1, App. E).  Reading O16: i runs over all
+// of K, ties by column id, and the loop stops at the first column that does not fit.
+ddq_status ddq_update_placement(ddq_db* db) {
+  if (!db) return set_error(DDQ_EINVAL, "update_placement");
+  std::lock_guard<std::mutex> g(db->mu);
+  std::vector<int> K(db->cols.size());
+  std::iota(K.begin(), K.end(), 0);
+  std::stable_sort(K.begin(), K.end(), [&](int a, int b) {
+    uint64_t x = db->cfg.cache_policy == 1 ? db->cols[(size_t)a]->last_access.load() : db->cols[(size_t)a]->access.load();
+    uint64_t y = db->cfg.cache_policy == 1 ? db->cols[(size_t)b]->last_access.load() : db->cols[(size_t)b]->access.load();
+    return x > y;
+  });
+  uint64_t used = 0;
+  std::vector<bool> keep(db->cols.size(), false);
+  for (size_t i = 0; i < K.size(); i++) {
+    const Column& c = *db->cols[(size_t)K[i]];
+    uint64_t sz = (uint64_t)std::max<int64_t>(c.n, 1) * c.width;
+    if (used + sz > db->cfg.cache_bytes) break;
+    keep[(size_t)K[i]] = true;
+    used += sz;
+  }
+  for (size_t c = 0; c < db->cols.size(); c++)  // evict(C_old \ C_new)
+    if (!keep[c] && db->cols[c]->dev) evict_column_locked(db, (int)c);
+  for (size_t c = 0; c < db->cols.size(); c++)  // cache(C_new \ C_old)
+    if (keep[c] && !db->cols[c]->dev) {
+      ddq_status s = cache_column_locked(db, (int)c, false);
+      if (s != DDQ_OK && s != DDQ_ENOMEM_DEVICE) return s;  // deferred evictions may still hold memory
+    }
+  return DDQ_OK;
+}
+
+ddq_status ddq_get_stats(ddq_db* db, ddq_stats* o) {
+  if (!db || !o) return set_error(DDQ_EINVAL, "get_stats");
+  std::memset(o, 0, sizeof(*o));
+  o->h2d_bytes = db->stats.h2d_bytes;
+  o->d2h_bytes = db->stats.d2h_bytes;
+  o->h2d_ns = db->stats.h2d_ns;
+  o->d2h_ns = db->stats.d2h_ns;
+  o->gpu_ops = db->stats.gpu_ops;
+  o->host_ops = db->stats.host_ops;
+  o->aborts = db->stats.aborts;
+  o->wasted_ns = db->stats.wasted_ns;
+  o->heap_peak_bytes = db->heap.peak();
+  o->heap_used_bytes = db->heap.used();
+  o->cache_used_bytes = db->cache_used;
+  o->cache_hits = db->stats.cache_hits;
+  o->cache_misses = db->stats.cache_misses;
+  o->queries_done = db->stats.queries_done;
+  return DDQ_OK;
+}
+
+ddq_status ddq_reset_stats(ddq_db* db) {
+  if (!db) return set_error(DDQ_EINVAL, "reset_stats");
+  db->stats.h2d_bytes = 0;
+  db->stats.d2h_bytes = 0;
+  db->stats.h2d_ns = 0;
+  db->stats.d2h_ns = 0;
+  db->stats.gpu_ops = 0;
+  db->stats.host_ops = 0;
+  db->stats.aborts = 0;
+  db->stats.wasted_ns = 0;
+  db->stats.cache_hits = 0;
+  db->stats.cache_misses = 0;
+  db->stats.queries_done = 0;
+  db->heap.reset_peak();
+  return DDQ_OK;
+}
+
+void* ddq_heap_try_alloc(ddq_db* db, uint64_t bytes) { return db ? db->heap.try_alloc(bytes) : nullptr; }
+void ddq_heap_free(ddq_db* db, void* p) {
+  if (db) db->heap.free(p);
+}
+
+void ddq_result_free(ddq_result* r) {
+  if (!r) return;
+  delete[] r->keys;
+  delete[] r->aggs;
+  delete[] r->tids;
+  delete r;
+}
+
+}  // extern "C"
+
+// ============================================================ prepared plans
+struct ddq_prepared {
+  ddq_db* db = nullptr;
+  ddq_plan plan{};
+  std::vector<ddq::Inter> inters;
+  std::vector<int64_t> forced;  // per-op output capacity (exact count + slack)
+  cudaGraph_t graph = nullptr;
+  cudaGraphExec_t exec = nullptr;
+  bool use_graph = false;
+  int kernels = 0;
+  cudaStream_t cap_stream = nullptr;
+};
+
+namespace ddq {
+
+static ddq_status validate_plan(ddq_db* db, const ddq_plan* plan) {
+  if (!plan || plan->n_ops < 1 || plan->n_ops > DDQ_MAX_OPS) return set_error(DDQ_EINVAL, "plan: bad op count");
+  for (int i = 0; i < plan->n_ops; i++) {
+    const ddq_op& op = plan->ops[i];
+    if (op.kind < DDQ_OP_SELECT || op.kind > DDQ_OP_AGGREGATE) return set_error(DDQ_EINVAL, "plan: bad op kind");
+    if (op.input >= i || op.input < -1) return set_error(DDQ_EINVAL, "plan: input must precede the op");
+    if (op.kind == DDQ_OP_HASH_PROBE && (op.build < 0 || op.build >= i ||
+                                         plan->ops[op.build].kind != DDQ_OP_HASH_BUILD))
+      return set_error(DDQ_EINVAL, "plan: probe must reference an earlier HASH_BUILD");
+    if (op.input >= 0 && plan->ops[op.input].kind == DDQ_OP_HASH_BUILD)
+      return set_error(DDQ_EINVAL, "plan: a hash table is not a TID input");
+    if (op.input >= 0 && plan->ops[op.input].kind == DDQ_OP_AGGREGATE)
+      return set_error(DDQ_EINVAL, "plan: an aggregate is not a TID input");
+    if (op.input >= 0 && plan->ops[op.input].table != op.table)
+      return set_error(DDQ_EINVAL, "plan: input TIDs belong to another table");
+    if (op.table < 0 || op.table >= (int)db->tables.size()) return set_error(DDQ_EINVAL, "plan: bad table");
+  }
+  const ddq_op& root = plan->ops[plan->n_ops - 1];
+  if (root.kind == DDQ_OP_HASH_BUILD) return set_error(DDQ_EINVAL, "plan: root cannot be a HASH_BUILD");
+  return DDQ_OK;
+}
+ddq_status validate_plan_public(ddq_db* db, const ddq_plan* plan) { return validate_plan(db, plan); }
+
+static int kernels_of(const ddq_op& op) {
+  switch (op.kind) {
+    case DDQ_OP_SELECT:
+    case DDQ_OP_HASH_PROBE: return 1;
+    case DDQ_OP_HASH_BUILD: return 2;
+    case DDQ_OP_GATHER: return 1;
+    case DDQ_OP_AGGREGATE: return 3;
+  }
+  return 0;
+}
+
+static void free_inters(ddq_db* db, std::vector<Inter>& v) {
+  for (auto& x : v) release_inter(db, x);
+  v.clear();
+}
+
+// Re-issue the launches of a prepared plan on its existing buffers.
+static ddq_status replay(ddq_prepared* P, cudaStream_t st) {
+  for (int i = 0; i < P->plan.n_ops; i++) {
+    std::vector<void*> blocks = P->inters[(size_t)i].heap_blocks;
+    GpuOpCtx ctx{P->db, st, &P->inters};
+    ctx.forced_cap = P->forced[(size_t)i];
+    ctx.count_column_access = false;
+    ctx.reuse = &blocks;
+    ddq_status s = run_gpu_op(ctx, P->plan.ops[i], P->inters[(size_t)i]);
+    if (s != DDQ_OK) return s;
+  }
+  return DDQ_OK;
+}
+
+void count_accesses(ddq_db* db, const ddq_op& op) {
+  auto touch = [&](int c) {
+    if (c < 0 || c >= (int)db->cols.size()) return;
+    db->cols[(size_t)c]->access++;
+    db->cols[(size_t)c]->last_access = ++db->clock;
+  };
+  switch (op.kind) {
+    case DDQ_OP_SELECT:
+      for (int i = 0; i < op.n_preds; i++) touch(op.preds[i].column);
+      break;
+    case DDQ_OP_HASH_BUILD: touch(op.key_col); touch(op.payload_col); break;
+    case DDQ_OP_HASH_PROBE: touch(op.fk_col); break;
+    case DDQ_OP_GATHER: touch(op.gather_col); break;
+    case DDQ_OP_AGGREGATE:
+      for (int k = 0; k < op.n_keys; k++)
+        if (op.key_src[k] < -1) touch(-2 - op.key_src[k]);
+      for (int a = 0; a < op.n_aggs; a++) {
+        int need = op.agg_kind[a] == DDQ_AGG_COUNT ? 0 : op.agg_kind[a] == DDQ_AGG_SUM ? 1
+                 : op.agg_kind[a] == DDQ_AGG_SUM_MUL_100M_100P ? 3 : 2;
+        for (int j = 0; j < need; j++) touch(op.agg_col[a][j]);
+      }
+      break;
+  }
+}
+
+}  // namespace ddq
+
+extern "C" {
+
+// Data-driven placement for the hot path: every input column must be
+// cached on this GPU; run once with worst-case capacities to learn the exact
+// intermediate cardinalities (run-time placement knows them), then
+// allocate exactly and capture the operator sequence into one CUDA graph.
+ddq_status ddq_prepare(ddq_db* db, const ddq_plan* plan, int32_t use_graph, ddq_prepared** out) {
+  if (!db || !out) return set_error(DDQ_EINVAL, "prepare: null argument");
+  if (ddq_status s = validate_plan(db, plan)) return s;
+  cudaSetDevice(db->device);
+  auto P = std::make_unique<ddq_prepared>();
+  P->db = db;
+  P->plan = *plan;
+  P->use_graph = use_graph != 0;
+  cudaStream_t st;
+  if (cudaStreamCreateWithFlags(&st, cudaStreamNonBlocking) != cudaSuccess)
+    return set_error(DDQ_ECUDA, "prepare: stream");
+  P->cap_stream = st;
+  auto fail = [&](ddq_status s) {
+    free_inters(db, P->inters);
+    cudaStreamDestroy(st);
+    P->cap_stream = nullptr;
+    return s;
+  };
+  // 1. calibration run (worst-case capacities) -> exact counts
+  std::vector<int64_t> counts((size_t)plan->n_ops, -1);
+  {
+    std::vector<Inter> cal((size_t)plan->n_ops);
+    GpuOpCtx ctx{db, st, &cal};
+    ctx.count_column_access = false;
+    uint32_t err = 0;
+    for (int i = 0; i < plan->n_ops; i++) {
+      ddq_status s = run_gpu_op(ctx, plan->ops[i], cal[(size_t)i]);
+      if (s != DDQ_OK) {
+        free_inters(db, cal);
+        return fail(s == DDQ_ENOMEM_DEVICE ? set_error(s, "prepare: device heap exhausted (calibration)") : s);
+      }
+      if (cal[(size_t)i].d_count && plan->ops[i].kind != DDQ_OP_GATHER) {
+        uint32_t c = 0;
+        cudaMemcpyAsync(&c, cal[(size_t)i].d_count, 4, cudaMemcpyDeviceToHost, st);
+        cudaError_t e = cudaStreamSynchronize(st);
+        if (e != cudaSuccess) {
+          free_inters(db, cal);
+          return fail(cuda_status(e, "prepare: calibration"));
+        }
+        counts[(size_t)i] = c;
+      }
+    }
+    for (auto& x : cal)
+      if (x.d_error) {
+        uint32_t e2 = 0;
+        cudaMemcpy(&e2, x.d_error, 4, cudaMemcpyDeviceToHost);
+        err = std::max(err, e2);
+      }
+    free_inters(db, cal);
+    if (err == 1 || err == 3) return fail(set_error(DDQ_EINVAL, "prepare: duplicate or invalid build key"));
+    if (err) return fail(set_error(DDQ_EOVERFLOW, "prepare: hash table overflow"));
+  }
+  // 2. exact capacities, allocate, eager run
+  P->forced.assign((size_t)plan->n_ops, -1);
+  for (int i = 0; i < plan->n_ops; i++) {
+    const ddq_op& op = plan->ops[i];
+    if (op.kind == DDQ_OP_HASH_BUILD && op.input >= 0) P->forced[(size_t)i] = counts[(size_t)op.input];
+    if (op.kind == DDQ_OP_SELECT || op.kind == DDQ_OP_HASH_PROBE)
+      P->forced[(size_t)i] = counts[(size_t)i] + counts[(size_t)i] / 64 + 256;
+  }
+  P->inters.resize((size_t)plan->n_ops);
+  for (int i = 0; i < plan->n_ops; i++) {
+    GpuOpCtx ctx{db, st, &P->inters};
+    ctx.forced_cap = P->forced[(size_t)i];
+    ctx.count_column_access = false;
+    ddq_status s = run_gpu_op(ctx, plan->ops[i], P->inters[(size_t)i]);
+    if (s != DDQ_OK) return fail(s == DDQ_ENOMEM_DEVICE ? set_error(s, "prepare: device heap exhausted") : s);
+    P->kernels += kernels_of(plan->ops[i]);
+  }
+  cudaError_t e = cudaStreamSynchronize(st);
+  if (e != cudaSuccess) return fail(cuda_status(e, "prepare: eager run"));
+  // 3. capture the same launches on the same buffers into one CUDA graph
+  if (P->use_graph) {
+    e = cudaStreamBeginCapture(st, cudaStreamCaptureModeThreadLocal);
+    if (e != cudaSuccess) return fail(cuda_status(e, "prepare: begin capture"));
+    ddq_status s = replay(P.get(), st);
+    cudaGraph_t g = nullptr;
+    e = cudaStreamEndCapture(st, &g);
+    if (s != DDQ_OK || e != cudaSuccess) {
+      if (g) cudaGraphDestroy(g);
+      return fail(s != DDQ_OK ? s : cuda_status(e, "prepare: end capture"));
+    }
+    P->graph = g;
+    e = cudaGraphInstantiate(&P->exec, g, 0);
+    if (e != cudaSuccess) return fail(cuda_status(e, "prepare: instantiate"));
+  }
+  *out = P.release();
+  return DDQ_OK;
+}
+
+ddq_status ddq_prepared_launch(ddq_prepared* p, void* stream) {
+  if (!p) return set_error(DDQ_EINVAL, "prepared_launch: null");
+  cudaStream_t st = (cudaStream_t)stream;
+  // column access counts (LFU statistics)
+  for (int i = 0; i < p->plan.n_ops; i++) count_accesses(p->db, p->plan.ops[i]);
+  p->db->stats.gpu_ops += (uint64_t)p->plan.n_ops;
+  if (p->use_graph) return cuda_status(cudaGraphLaunch(p->exec, st), "prepared_launch");
+  return replay(p, st);
+}
+
+int32_t ddq_prepared_kernel_count(ddq_prepared* p) { return p ? p->kernels : 0; }
+
+static double sector_bytes(double N, double m, int w) {
+  if (N <= 0 || m <= 0) return 0;
+  double rho = std::min(1.0, m / N);
+  return N * w * (1.0 - std::pow(1.0 - rho, 32.0 / w));
+}
+
+int32_t ddq_prepared_profile(ddq_prepared* p, void* stream, int32_t max_ops, float* op_ms, double* op_bytes,
+                             int32_t* op_class) {
+  if (!p) return set_error(DDQ_EINVAL, "prepared_profile: null");
+  cudaStream_t st = (cudaStream_t)stream;
+  const int n = p->plan.n_ops;
+  std::vector<cudaEvent_t> ev((size_t)n + 1);
+  for (auto& e : ev) cudaEventCreate(&e);
+  cudaEventRecord(ev[0], st);
+  for (int i = 0; i < n; i++) {
+    std::vector<void*> blocks = p->inters[(size_t)i].heap_blocks;
+    GpuOpCtx ctx{p->db, st, &p->inters};
+    ctx.forced_cap = p->forced[(size_t)i];
+    ctx.count_column_access = false;
+    ctx.reuse = &blocks;
+    ddq_status s = run_gpu_op(ctx, p->plan.ops[i], p->inters[(size_t)i]);
+    if (s != DDQ_OK) {
+      for (auto& e : ev) cudaEventDestroy(e);
+      return s;
+    }
+    cudaEventRecord(ev[(size_t)i + 1], st);
+  }
+  cudaError_t e = cudaStreamSynchronize(st);
+  if (e != cudaSuccess) {
+    for (auto& x : ev) cudaEventDestroy(x);
+    return cuda_status(e, "prepared_profile");
+  }
+  std::vector<int64_t> cnt((size_t)n, -1);
+  for (int i = 0; i < n; i++)
+    if (p->inters[(size_t)i].d_count) {
+      uint32_t c = 0;
+      cudaMemcpy(&c, p->inters[(size_t)i].d_count, 4, cudaMemcpyDeviceToHost);
+      cnt[(size_t)i] = c;
+    }
+  auto width = [&](int c) { const Column* col = col_of(p->db, c); return col ? col->width : 4; };
+  for (int i = 0; i < n && i < max_ops; i++) {
+    const ddq_op& op = p->plan.ops[i];
+    const Inter& o = p->inters[(size_t)i];
+    const double N = (double)p->db->tables[(size_t)op.table].n_rows;
+    const double m = op.input >= 0 ? (double)cnt[(size_t)op.input] : N;
+    const double out = cnt[(size_t)i] >= 0 ? (double)cnt[(size_t)i] : 0;
+    const int nvec_in = op.input >= 0 ? (int)p->inters[(size_t)op.input].vecs.size() : 0;
+    double bytes = 0;
+    int cls = 0;
+    float ms = 0;
+    cudaEventElapsedTime(&ms, ev[(size_t)i], ev[(size_t)i + 1]);
+    switch (op.kind) {
+      case DDQ_OP_SELECT:
+      case DDQ_OP_HASH_PROBE: {
+        std::vector<int> cols;
+        if (op.kind == DDQ_OP_SELECT)
+          for (int k = 0; k < op.n_preds; k++) cols.push_back(op.preds[k].column);
+        else
+          cols.push_back(op.fk_col);
+        const int emit = op.kind == DDQ_OP_HASH_PROBE && op.emit_payload ? 1 : 0;
+        if (op.input < 0) {
+          cls = 0;
+          for (int c : cols) bytes += N * width(c);
+        } else {
+          cls = 1;
+          bytes += m * 4;
+          for (int c : cols) bytes += sector_bytes(N, m, width(c));
+          bytes += out * 4 * nvec_in;  // carried vectors read at survivors
+        }
+        bytes += out * 4 * (1 + nvec_in + emit);
+      } break;
+      case DDQ_OP_HASH_BUILD:
+        cls = 2;
+        bytes = m * 4 * (op.payload_col >= 0 ? 2 : 1) + (double)o.table_cap * 8 * 2;
+        break;
+      case DDQ_OP_GATHER:
+        cls = 3;
+        bytes = m * 4 + sector_bytes(N, m, width(op.gather_col)) + m * width(op.gather_col);
+        break;
+      case DDQ_OP_AGGREGATE: {
+        cls = 4;
+        bytes = m * 4;
+        for (int k = 0; k < op.n_keys; k++) bytes += op.key_src[k] >= 0 ? m * 4 : sector_bytes(N, m, 4);
+        std::vector<int> seen;
+        for (int a = 0; a < op.n_aggs; a++)
+          for (int j = 0; j < 3; j++) {
+            int c = op.agg_col[a][j];
+            if (c < 0 || std::find(seen.begin(), seen.end(), c) != seen.end()) continue;
+            int need = op.agg_kind[a] == DDQ_AGG_COUNT ? 0 : op.agg_kind[a] == DDQ_AGG_SUM ? 1
+                     : op.agg_kind[a] == DDQ_AGG_SUM_MUL_100M_100P ? 3 : 2;
+            if (j >= need) continue;
+            seen.push_back(c);
+            bytes += sector_bytes(N, m, width(c));
+          }
+      } break;
+    }
+    if (op_ms) op_ms[i] = ms;
+    if (op_bytes) op_bytes[i] = bytes;
+    if (op_class) op_class[i] = cls;
+  }
+  for (auto& x : ev) cudaEventDestroy(x);
+  return n;
+}
+
+int64_t ddq_prepared_group_capacity(ddq_prepared* p) {
+  if (!p) return 0;
+  const Inter& r = p->inters.back();
+  return r.gb_cap ? (int64_t)r.gb_cap : r.cap;
+}
+
+static ddq_status check_errors(ddq_prepared* p, cudaStream_t st) {
+  uint32_t err = 0;
+  for (auto& x : p->inters)
+    if (x.d_error) {
+      uint32_t e2 = 0;
+      cudaMemcpyAsync(&e2, x.d_error, 4, cudaMemcpyDeviceToHost, st);
+      cudaError_t e = cudaStreamSynchronize(st);
+      if (e != cudaSuccess) return cuda_status(e, "prepared: error cell");
+      err = std::max(err, e2);
+    }
+  if (err == 1 || err == 3) return set_error(DDQ_EINVAL, "duplicate or invalid build key");
+  if (err == 4) return set_error(DDQ_EOVERFLOW, "intermediate exceeded its prepared capacity (data changed?)");
+  if (err) return set_error(DDQ_EOVERFLOW, "hash table overflow");
+  return DDQ_OK;
+}
+
+ddq_status ddq_prepared_partials(ddq_prepared* p, void* stream, int64_t* h_n_groups, int64_t* h_keys,
+                                 int64_t* h_accs, int64_t cap) {
+  if (!p || !h_n_groups) return set_error(DDQ_EINVAL, "prepared_partials: null");
+  cudaStream_t st = (cudaStream_t)stream;
+  const Inter& r = p->inters.back();
+  if (!r.gb_table) return set_error(DDQ_ESTATE, "prepared_partials: root is not an aggregate");
+  if (ddq_status s = check_errors(p, st)) return s;
+  uint32_t g = 0;
+  uint64_t t0 = now_ns();
+  cudaMemcpyAsync(&g, r.gb_groups, 4, cudaMemcpyDeviceToHost, st);
+  cudaError_t e = cudaStreamSynchronize(st);
+  if (e != cudaSuccess) return cuda_status(e, "prepared_partials");
+  if ((int64_t)g > cap) return set_error(DDQ_EINVAL, "prepared_partials: buffer too small");
+  const int na = p->plan.ops[p->plan.n_ops - 1].n_aggs;
+  if (g) {
+    cudaMemcpyAsync(h_keys, r.gb_keys, (size_t)g * 8, cudaMemcpyDeviceToHost, st);
+    cudaMemcpyAsync(h_accs, r.gb_accs, (size_t)g * na * 16, cudaMemcpyDeviceToHost, st);
+    e = cudaStreamSynchronize(st);
+    if (e != cudaSuccess) return cuda_status(e, "prepared_partials copy");
+  }
+  p->db->stats.d2h_bytes += 4 + (uint64_t)g * (8 + 16 * na);
+  p->db->stats.d2h_ns += now_ns() - t0;
+  *h_n_groups = g;
+  return DDQ_OK;
+}
+
+ddq_status ddq_prepared_finalize(ddq_prepared* p, int64_t n_groups, const int64_t* h_keys, const int64_t* h_accs,
+                                 ddq_result** out) {
+  if (!p || !out) return set_error(DDQ_EINVAL, "prepared_finalize: null");
+  return finalize_result(p->plan.ops[p->plan.n_ops - 1], n_groups, h_keys, h_accs, out);
+}
+
+ddq_status ddq_prepared_fetch(ddq_prepared* p, void* stream, ddq_result** out) {
+  if (!p || !out) return set_error(DDQ_EINVAL, "prepared_fetch: null");
+  cudaStream_t st = (cudaStream_t)stream;
+  const ddq_op& root = p->plan.ops[p->plan.n_ops - 1];
+  const Inter& r = p->inters.back();
+  if (root.kind != DDQ_OP_AGGREGATE) {  // select-* root: return the TID list
+    if (ddq_status s = check_errors(p, st)) return s;
+    uint32_t n = 0;
+    cudaMemcpyAsync(&n, r.d_count, 4, cudaMemcpyDeviceToHost, st);
+    cudaError_t e = cudaStreamSynchronize(st);
+    if (e != cudaSuccess) return cuda_status(e, "prepared_fetch");
+    ddq_result* res = new ddq_result();
+    std::memset(res, 0, sizeof(*res));
+    int32_t* t = new int32_t[std::max<uint32_t>(n, 1)];
+    if (n) cudaMemcpyAsync(t, r.tids, (size_t)n * 4, cudaMemcpyDeviceToHost, st);
+    e = cudaStreamSynchronize(st);
+    if (e != cudaSuccess) {
+      delete[] t;
+      delete res;
+      return cuda_status(e, "prepared_fetch tids");
+    }
+    const int64_t base = p->db->tables[(size_t)root.table].row_begin;
+    for (uint32_t i = 0; i < n; i++) t[i] = (int32_t)(t[i] + base);
+    res->n_tids = n;
+    res->tids = t;
+    res->gpu_ops = p->plan.n_ops;
+    *out = res;
+    return DDQ_OK;
+  }
+  const int na = root.n_aggs;
+  std::vector<int64_t> keys(r.gb_cap), accs((size_t)r.gb_cap * na * 2);
+  int64_t g = 0;
+  if (ddq_status s = ddq_prepared_partials(p, stream, &g, keys.data(), accs.data(), r.gb_cap)) return s;
+  ddq_status s = finalize_result(root, g, keys.data(), accs.data(), out);
+  if (s == DDQ_OK) (*out)->gpu_ops = p->plan.n_ops;
+  return s;
+}
+
+void ddq_prepared_free(ddq_prepared* p) {
+  if (!p) return;
+  if (p->cap_stream) cudaStreamSynchronize(p->cap_stream);
+  if (p->exec) cudaGraphExecDestroy(p->exec);
+  if (p->graph) cudaGraphDestroy(p->graph);
+  free_inters(p->db, p->inters);
+  if (p->cap_stream) cudaStreamDestroy(p->cap_stream);
+  delete p;
+}
+
+}  // extern "C"

@@ -1,0 +1,163 @@
+// engine.h -- internal structures of the libddq database (column store, device
+// cache, heap-budget allocator, operator runners).
+#pragma once
+#include <atomic>
+#include <condition_variable>
+#include <cstdint>
+#include <deque>
+#include <map>
+#include <memory>
+#include <mutex>
+#include <string>
+#include <thread>
+#include <vector>
+
+#include <cuda_runtime.h>
+
+#include "../../include/ddq.h"
+
+namespace ddq {
+
+ddq_status set_error(ddq_status s, const std::string& msg);
+ddq_status cuda_status(cudaError_t e, const char* where);
+uint64_t now_ns();
+
+// ---- heap-budget allocator (P:62 heap; P:113 fail fast, never wait) --------
+class Heap {
+ public:
+  ddq_status init(uint64_t bytes, uint32_t fault_every);
+  ~Heap();
+  void* try_alloc(uint64_t bytes);  // nullptr on failure (no waiting)
+  void free(void* p);
+  uint64_t used() const { return used_; }
+  uint64_t peak() const { return peak_; }
+  uint64_t capacity() const { return cap_; }
+  void reset_peak() { peak_ = used_; }
+
+ private:
+  std::mutex mu_;
+  char* base_ = nullptr;
+  uint64_t cap_ = 0, used_ = 0, peak_ = 0;
+  uint32_t fault_every_ = 0;
+  uint64_t n_allocs_ = 0;
+  std::map<uint64_t, uint64_t> free_;   // offset -> size
+  std::map<uint64_t, uint64_t> alloc_;  // offset -> size
+};
+
+struct Column {
+  std::string name;
+  int table = -1;
+  int type = DDQ_I32;
+  int width = 4;
+  int64_t n = 0;
+  void* host = nullptr;   // pinned host copy
+  void* dev = nullptr;    // device cache copy or nullptr
+  std::atomic<uint64_t> access{0};
+  std::atomic<uint64_t> last_access{0};
+  int refs = 0;             // running operators using `dev`
+  bool evict_pending = false;
+  bool on_demand = false;   // cached by operator-driven placement (GPU-only arm)
+};
+
+struct Table {
+  std::string name;
+  int64_t n_rows = 0;
+  int64_t row_begin = 0;
+  std::vector<int> cols;
+};
+
+struct Vec {
+  void* ptr = nullptr;  // device or host, aligned with the TID list
+  int width = 4;
+  bool host = false;
+};
+
+// A materialised intermediate: TIDs + aligned vectors, on one processor.
+struct Inter {
+  bool on_host = false;
+  bool all_rows = false;   // implicit TIDs 0..cap-1
+  int table = -1;
+  int32_t* tids = nullptr;
+  uint32_t* d_count = nullptr;  // device count cell (GPU)
+  int64_t cap = 0;              // capacity (upper bound on count)
+  int64_t count = -1;           // exact count when known on the host
+  std::vector<Vec> vecs;
+  // hash build output
+  uint64_t* table_ptr = nullptr;
+  uint32_t table_cap = 0;
+  uint32_t* d_error = nullptr;
+  // host-side hash table (host build)
+  std::shared_ptr<std::vector<uint64_t>> host_table;
+  // aggregate output
+  void* gb_table = nullptr;
+  uint32_t gb_cap = 0;
+  int64_t* gb_keys = nullptr;
+  int64_t* gb_accs = nullptr;
+  uint32_t* gb_groups = nullptr;
+  // host aggregate result (host executor)
+  std::shared_ptr<std::vector<int64_t>> h_keys, h_accs;
+  int64_t h_groups = 0;
+  // allocations owned by this intermediate (heap or host)
+  std::vector<void*> heap_blocks;
+  std::vector<void*> host_blocks;
+};
+
+struct Stats {
+  std::atomic<uint64_t> h2d_bytes{0}, d2h_bytes{0}, h2d_ns{0}, d2h_ns{0}, gpu_ops{0}, host_ops{0}, aborts{0},
+      wasted_ns{0}, cache_hits{0}, cache_misses{0}, queries_done{0};
+};
+
+struct QueryState;
+
+}  // namespace ddq
+
+struct ddq_db {
+  ddq_config cfg{};
+  int device = 0;
+  cudaStream_t copy_stream = nullptr;
+  ddq::Heap heap;
+  std::mutex mu;  // catalog + cache
+  std::condition_variable cache_cv;
+  std::vector<ddq::Table> tables;
+  std::vector<std::unique_ptr<ddq::Column>> cols;
+  uint64_t cache_used = 0;
+  std::atomic<uint64_t> clock{0};
+  ddq::Stats stats;
+  // chopping executor
+  std::mutex qmu;
+  std::condition_variable qcv;
+  std::deque<std::pair<std::shared_ptr<ddq::QueryState>, int>> gpu_ready, host_ready;
+  std::map<int64_t, std::shared_ptr<ddq::QueryState>> queries;
+  int64_t next_query = 1;
+  bool stopping = false;
+  std::vector<std::thread> workers;
+  int busy_gpu = 0;
+};
+
+namespace ddq {
+
+// Runs one operator on the GPU, allocating outputs from the heap (fail fast).
+// exact_caps: if non-null, output capacities to use (prepared plans), else the
+// input capacity.  Returns DDQ_ENOMEM_DEVICE when an allocation fails.
+struct GpuOpCtx {
+  ddq_db* db;
+  cudaStream_t stream;
+  const std::vector<Inter>* inters;  // outputs of earlier ops (same plan)
+  int64_t forced_cap = -1;           // output capacity override
+  bool count_column_access = true;
+  const std::vector<void*>* reuse = nullptr;  // replay on existing buffers
+};
+void count_accesses(ddq_db* db, const ddq_op& op);
+void driver_start(ddq_db* db);
+void driver_stop(ddq_db* db);
+ddq_status run_gpu_op(GpuOpCtx& ctx, const ddq_op& op, Inter& out);
+// Host executor (CPU fallback handler for every operator).
+ddq_status run_host_op(ddq_db* db, const ddq_op& op, const std::vector<Inter>& inters, Inter& out);
+void release_inter(ddq_db* db, Inter& x);
+ddq_status inter_to_host(ddq_db* db, Inter& x, cudaStream_t st);
+ddq_status finalize_result(const ddq_op& root, int64_t n_groups, const int64_t* keys, const int64_t* accs,
+                           ddq_result** out);
+int64_t pow2_at_least(int64_t x);
+const ddq::Column* col_of(ddq_db* db, int c);
+
+}  // namespace ddq

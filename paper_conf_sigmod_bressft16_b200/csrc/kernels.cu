@@ -1,0 +1,352 @@
+// kernels.cu -- hash build (S8(a3)), positional gather (S8(a5)) and group-by
+// aggregation (S8(a6)) for sm_100a.
+//
+// Group-by design: every warp aggregates its 32 rows per
+// distinct key first (__match_any_sync + a log-step peer reduction), the lowest
+// lane of each key group then updates a per-CTA shared-memory hash table, and each
+// CTA merges its table into the global open-addressing table once at the end.
+// Accumulators are exact int128 (two 64-bit atomics with carry), so results are
+// bit-identical whatever the scheduling (integer addition is associative).
+#include <cstdint>
+#include <cuda_runtime.h>
+
+#include "device_common.cuh"
+#include "ops_internal.h"
+
+namespace ddq {
+
+int num_sms() {
+  static int sms = 0;
+  if (!sms) {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    if (sms <= 0) sms = 1;
+  }
+  return sms;
+}
+
+static inline uint32_t read_count_host_cap(int64_t n_cap) { return (uint32_t)n_cap; }
+
+// ----------------------------------------------------------------- hash build
+__global__ void hash_init_kernel(uint64_t* table, uint32_t capacity) {
+  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < capacity; i += gridDim.x * blockDim.x)
+    table[i] = HT_EMPTY;
+}
+
+__global__ void hash_build_kernel(const int32_t* __restrict__ keys, const int32_t* __restrict__ payload,
+                                  const int32_t* __restrict__ in_tids, const uint32_t* d_in_count,
+                                  uint32_t n_static, uint64_t* table, uint32_t capacity, int shift,
+                                  uint32_t* d_error) {
+  const uint32_t n = d_in_count ? ld_relaxed_u32(d_in_count) : n_static;
+  const uint32_t mask = capacity - 1;
+  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
+    const int32_t r = in_tids ? in_tids[i] : (int32_t)i;
+    const int32_t k = keys[r];
+    const int32_t v = payload ? payload[r] : r;
+    if (k == INT32_MIN) {
+      atomicMax(d_error, 3u);
+      continue;
+    }
+    const uint64_t slot = ((uint64_t)(uint32_t)k << 32) | (uint32_t)v;
+    uint32_t h = ht_hash(k, shift);
+    uint32_t probes = 0;
+    while (true) {
+      unsigned long long old = atomicCAS(reinterpret_cast<unsigned long long*>(table + h),
+                                         (unsigned long long)HT_EMPTY, (unsigned long long)slot);
+      if (old == HT_EMPTY) break;
+      if (ht_key(old) == k) {  // PKs must be unique (reading O13)
+        atomicMax(d_error, 1u);
+        break;
+      }
+      h = (h + 1) & mask;
+      if (++probes >= capacity) {
+        atomicMax(d_error, 2u);
+        break;
+      }
+    }
+  }
+}
+
+cudaError_t launch_hash_init(uint64_t* table, uint32_t capacity, cudaStream_t st) {
+  int grid = (int)((capacity + 255) / 256);
+  if (grid > num_sms() * 8) grid = num_sms() * 8;
+  if (grid < 1) grid = 1;
+  hash_init_kernel<<<grid, 256, 0, st>>>(table, capacity);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_hash_build(const int32_t* keys, const int32_t* payload, const int32_t* in_tids,
+                              const uint32_t* d_in_count, int64_t n_cap, uint64_t* table, uint32_t capacity,
+                              uint32_t* d_error, cudaStream_t st) {
+  int lg = 0;
+  while ((1u << lg) < capacity) lg++;
+  int64_t g = (n_cap + 255) / 256;
+  int grid = (int)(g > num_sms() * 8 ? num_sms() * 8 : (g < 1 ? 1 : g));
+  hash_build_kernel<<<grid, 256, 0, st>>>(keys, payload, in_tids, d_in_count, read_count_host_cap(n_cap), table,
+                                          capacity, 32 - lg, d_error);
+  return cudaGetLastError();
+}
+
+// --------------------------------------------------------------------- gather
+template <int W>
+__global__ void gather_kernel(const void* __restrict__ col, const int32_t* __restrict__ tids,
+                              const uint32_t* d_count, uint32_t n_static, void* __restrict__ out) {
+  const uint32_t n = d_count ? ld_relaxed_u32(d_count) : n_static;
+  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
+    const int32_t r = tids[i];
+    if (W == 8)
+      reinterpret_cast<long long*>(out)[i] = __ldg(reinterpret_cast<const long long*>(col) + r);
+    else
+      reinterpret_cast<int*>(out)[i] = __ldg(reinterpret_cast<const int*>(col) + r);
+  }
+}
+
+cudaError_t launch_gather(const void* col, int width, const int32_t* tids, const uint32_t* d_count,
+                          int64_t n_cap, void* out, cudaStream_t st) {
+  int64_t g = (n_cap + 255) / 256;
+  int grid = (int)(g > num_sms() * 16 ? num_sms() * 16 : (g < 1 ? 1 : g));
+  if (width == 8)
+    gather_kernel<8><<<grid, 256, 0, st>>>(col, tids, d_count, (uint32_t)n_cap, out);
+  else
+    gather_kernel<4><<<grid, 256, 0, st>>>(col, tids, d_count, (uint32_t)n_cap, out);
+  return cudaGetLastError();
+}
+
+// -------------------------------------------------------------------- groupby
+constexpr int GB_THREADS = 256;
+constexpr int GB_SMEM_BUDGET = 32 * 1024;
+
+struct GroupbyParams {
+  const int32_t* tids;
+  const uint32_t* d_count;
+  uint32_t n_static;
+  int32_t n_keys;
+  const int32_t* key_vec[3];
+  const int32_t* key_col[3];
+  int32_t n_aggs;
+  int32_t kind[8];
+  int32_t width[8][3];
+  const void* arg[8][3];
+  long long* g_keys;
+  unsigned long long* g_accs;  // [(a * cap + slot) * 2 + {0: lo, 1: hi}]
+  uint32_t cap_mask;
+  int32_t shift;
+  uint32_t* d_error;
+  uint32_t s_slots;
+  int32_t s_shift;
+};
+
+__device__ __forceinline__ long long agg_value(const GroupbyParams& P, int a, int32_t r) {
+  const int k = P.kind[a];
+  if (k == DDQ_AGG_COUNT) return 1;
+  const long long x = col_at(P.arg[a][0], P.width[a][0], r);
+  if (k == DDQ_AGG_SUM) return x;
+  const long long y = col_at(P.arg[a][1], P.width[a][1], r);
+  if (k == DDQ_AGG_SUM_MUL) return x * y;
+  if (k == DDQ_AGG_SUM_SUB) return x - y;
+  if (k == DDQ_AGG_SUM_MUL_100M) return x * (100 - y);
+  const long long z = col_at(P.arg[a][2], P.width[a][2], r);
+  return x * (100 - y) * (100 + z);  // DDQ_AGG_SUM_MUL_100M_100P
+}
+
+// Sum of x over the lanes of `peers`; the total lands in the lowest peer lane.
+__device__ __forceinline__ long long peer_reduce(unsigned peers, long long x, int lane) {
+  unsigned rest = peers & (0xfffffffeu << lane);
+  unsigned rank = __popc(peers & ((1u << lane) - 1u));
+  while (__any_sync(FULL, rest != 0)) {
+    const int next = __ffs(rest);
+    const long long t = __shfl_sync(FULL, x, next ? next - 1 : lane);
+    if (next) x += t;
+    rest &= ~__ballot_sync(FULL, rank & 1u);
+    rank >>= 1;
+  }
+  return x;
+}
+
+// find-or-insert `key` into an open-addressing table of int64 keys; -1 if full
+__device__ __forceinline__ int64_t table_slot(long long* keys, uint32_t mask, uint32_t h, long long key) {
+  for (uint32_t probes = 0; probes <= mask; probes++) {
+    long long cur = keys[h];
+    if (cur == key) return h;
+    if (cur == GB_EMPTY) {
+      long long old = (long long)atomicCAS(reinterpret_cast<unsigned long long*>(keys + h),
+                                           (unsigned long long)GB_EMPTY, (unsigned long long)key);
+      if (old == GB_EMPTY || old == key) return h;
+    }
+    h = (h + 1) & mask;
+  }
+  return -1;
+}
+
+__global__ void __launch_bounds__(GB_THREADS) groupby_kernel(const __grid_constant__ GroupbyParams P) {
+  extern __shared__ unsigned long long s_mem[];
+  long long* s_keys = reinterpret_cast<long long*>(s_mem);
+  unsigned long long* s_accs = s_mem + P.s_slots;  // [(a * S + slot) * 2 + w]
+  const uint32_t S = P.s_slots, smask = S - 1;
+  for (uint32_t i = threadIdx.x; i < S; i += GB_THREADS) s_keys[i] = GB_EMPTY;
+  for (uint32_t i = threadIdx.x; i < S * 2 * P.n_aggs; i += GB_THREADS) s_accs[i] = 0;
+  __syncthreads();
+
+  const int lane = threadIdx.x & 31;
+  const uint32_t n = P.d_count ? ld_relaxed_u32(P.d_count) : P.n_static;
+  const uint32_t warps_total = gridDim.x * (GB_THREADS / 32);
+  const uint32_t gw = blockIdx.x * (GB_THREADS / 32) + (threadIdx.x >> 5);
+  for (uint32_t base = gw * 32; base < n; base += warps_total * 32) {
+    const uint32_t i = base + lane;
+    const bool valid = i < n;
+    int32_t r = 0;
+    long long key = LLONG_MIN;
+    if (valid) {
+      r = P.tids[i];
+      key = 0;
+      for (int k = 0; k < P.n_keys; k++) {
+        const int32_t c = P.key_vec[k] ? P.key_vec[k][i] : __ldg(P.key_col[k] + r);
+        key |= (long long)(uint32_t)c << (21 * k);
+      }
+    }
+    const unsigned peers = __match_any_sync(FULL, key);
+    const bool leader = (peers & ((1u << lane) - 1u)) == 0;
+    long long slot = -1;
+    bool global = false;
+    if (valid && leader) {
+      slot = table_slot(s_keys, smask, gb_hash(key, P.s_shift), key);
+      if (slot < 0) {
+        global = true;
+        slot = table_slot(P.g_keys, P.cap_mask, gb_hash(key, P.shift), key);
+        if (slot < 0) atomicMax(P.d_error, 2u);
+      }
+    }
+    for (int a = 0; a < P.n_aggs; a++) {
+      long long v = valid ? agg_value(P, a, r) : 0;
+      v = peer_reduce(peers, v, lane);
+      if (valid && leader && slot >= 0) {
+        if (!global)
+          atomic_add_i128(&s_accs[((size_t)a * S + slot) * 2], &s_accs[((size_t)a * S + slot) * 2 + 1], v);
+        else
+          atomic_add_i128(&P.g_accs[((size_t)a * (P.cap_mask + 1) + slot) * 2],
+                          &P.g_accs[((size_t)a * (P.cap_mask + 1) + slot) * 2 + 1], v);
+      }
+    }
+  }
+  __syncthreads();
+  // merge this CTA's table into the global one
+  for (uint32_t s = threadIdx.x; s < S; s += GB_THREADS) {
+    const long long key = s_keys[s];
+    if (key == GB_EMPTY) continue;
+    const long long g = table_slot(P.g_keys, P.cap_mask, gb_hash(key, P.shift), key);
+    if (g < 0) {
+      atomicMax(P.d_error, 2u);
+      continue;
+    }
+    for (int a = 0; a < P.n_aggs; a++) {
+      const unsigned long long lo = s_accs[((size_t)a * S + s) * 2], hi = s_accs[((size_t)a * S + s) * 2 + 1];
+      unsigned long long* glo = &P.g_accs[((size_t)a * (P.cap_mask + 1) + g) * 2];
+      const unsigned long long old = atomicAdd(glo, lo);
+      const unsigned long long carry = (old + lo < old) ? 1ull : 0ull;
+      if (hi + carry) atomicAdd(glo + 1, hi + carry);
+    }
+  }
+}
+
+size_t groupby_table_bytes(uint32_t capacity, int n_aggs) {
+  return (size_t)capacity * 8 + (size_t)capacity * n_aggs * 16;
+}
+
+__global__ void groupby_init_kernel(long long* keys, unsigned long long* accs, uint32_t capacity, int n_aggs) {
+  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < capacity; i += gridDim.x * blockDim.x) {
+    keys[i] = GB_EMPTY;
+    for (int a = 0; a < n_aggs; a++) {
+      accs[((size_t)a * capacity + i) * 2] = 0;
+      accs[((size_t)a * capacity + i) * 2 + 1] = 0;
+    }
+  }
+}
+
+cudaError_t launch_groupby_init(void* table, uint32_t capacity, int n_aggs, cudaStream_t st) {
+  int grid = (int)((capacity + 255) / 256);
+  if (grid > num_sms() * 8) grid = num_sms() * 8;
+  groupby_init_kernel<<<grid < 1 ? 1 : grid, 256, 0, st>>>(
+      reinterpret_cast<long long*>(table), reinterpret_cast<unsigned long long*>((char*)table + (size_t)capacity * 8),
+      capacity, n_aggs);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_groupby(const int32_t* tids, const uint32_t* d_count, int64_t n_cap,
+                           const int32_t* const* key_vec, const int32_t* const* key_col, int n_keys,
+                           const ddq_dev_agg* aggs, int n_aggs, void* table, uint32_t capacity,
+                           uint32_t* d_error, cudaStream_t st) {
+  GroupbyParams p{};
+  p.tids = tids;
+  p.d_count = d_count;
+  p.n_static = (uint32_t)n_cap;
+  p.n_keys = n_keys;
+  for (int k = 0; k < n_keys; k++) {
+    p.key_vec[k] = key_vec ? key_vec[k] : nullptr;
+    p.key_col[k] = key_col ? key_col[k] : nullptr;
+  }
+  p.n_aggs = n_aggs;
+  for (int a = 0; a < n_aggs; a++) {
+    p.kind[a] = aggs[a].kind;
+    for (int j = 0; j < 3; j++) {
+      p.width[a][j] = aggs[a].width[j];
+      p.arg[a][j] = aggs[a].arg[j];
+    }
+  }
+  p.g_keys = reinterpret_cast<long long*>(table);
+  p.g_accs = reinterpret_cast<unsigned long long*>((char*)table + (size_t)capacity * 8);
+  p.cap_mask = capacity - 1;
+  int lg = 0;
+  while ((1u << lg) < capacity) lg++;
+  p.shift = 64 - lg;
+  p.d_error = d_error;
+  uint32_t S = 1u << 12;
+  while (S > 64 && (size_t)S * (8 + 16 * (size_t)n_aggs) > GB_SMEM_BUDGET) S >>= 1;
+  // no point in a CTA table larger than the global one
+  while (S > 64 && S > capacity) S >>= 1;
+  int slg = 0;
+  while ((1u << slg) < S) slg++;
+  p.s_slots = S;
+  p.s_shift = 64 - slg;
+  const size_t smem = (size_t)S * (8 + 16 * (size_t)n_aggs);
+  static int occ = 0;
+  if (!occ) {
+    cudaFuncSetAttribute(groupby_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 160 * 1024);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, groupby_kernel, GB_THREADS, GB_SMEM_BUDGET);
+    if (occ < 1) occ = 1;
+  }
+  int64_t want = (n_cap + GB_THREADS - 1) / GB_THREADS;
+  int64_t maxb = (int64_t)num_sms() * occ;
+  int grid = (int)(want < 1 ? 1 : (want > maxb ? maxb : want));
+  groupby_kernel<<<grid, GB_THREADS, smem, st>>>(p);
+  return cudaGetLastError();
+}
+
+__global__ void groupby_compact_kernel(const long long* keys, const unsigned long long* accs, uint32_t capacity,
+                                       int n_aggs, int64_t* out_keys, int64_t* out_accs, uint32_t* d_out) {
+  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < capacity; i += gridDim.x * blockDim.x) {
+    const long long k = keys[i];
+    if (k == GB_EMPTY) continue;
+    const uint32_t pos = atomicAdd(d_out, 1u);
+    out_keys[pos] = k;
+    for (int a = 0; a < n_aggs; a++) {
+      out_accs[((size_t)pos * n_aggs + a) * 2] = (int64_t)accs[((size_t)a * capacity + i) * 2];
+      out_accs[((size_t)pos * n_aggs + a) * 2 + 1] = (int64_t)accs[((size_t)a * capacity + i) * 2 + 1];
+    }
+  }
+}
+
+cudaError_t launch_groupby_compact(const void* table, uint32_t capacity, int n_aggs, int64_t* out_keys,
+                                   int64_t* out_accs, uint32_t* d_out_groups, cudaStream_t st) {
+  cudaError_t e = cudaMemsetAsync(d_out_groups, 0, sizeof(uint32_t), st);
+  if (e != cudaSuccess) return e;
+  int grid = (int)((capacity + 255) / 256);
+  if (grid > num_sms() * 8) grid = num_sms() * 8;
+  groupby_compact_kernel<<<grid < 1 ? 1 : grid, 256, 0, st>>>(
+      reinterpret_cast<const long long*>(table),
+      reinterpret_cast<const unsigned long long*>((const char*)table + (size_t)capacity * 8), capacity, n_aggs,
+      out_keys, out_accs, d_out_groups);
+  return cudaGetLastError();
+}
+
+}  // namespace ddq

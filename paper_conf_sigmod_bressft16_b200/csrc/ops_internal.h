@@ -1,0 +1,54 @@
+// ops_internal.h -- host-side launch interfaces of the libddq kernels.
+#pragma once
+#include <cstddef>
+#include <cstdint>
+#include <cuda_runtime.h>
+
+#include "../../include/ddq.h"
+
+namespace ddq {
+
+struct FilterArgs {
+  const ddq_dev_pred* preds = nullptr;
+  int n_preds = 0;
+  bool probe = false;
+  bool no_smem = false;
+  const uint64_t* table = nullptr;
+  uint32_t capacity = 0;
+  const int32_t* fk = nullptr;
+  int32_t* out_payload = nullptr;
+  const int32_t* in_tids = nullptr;
+  const uint32_t* d_in_count = nullptr;
+  int64_t n_cap = 0;
+  const int32_t* const* carry_in = nullptr;
+  int32_t* const* carry_out = nullptr;
+  int n_carry = 0;
+  int32_t* out_tids = nullptr;
+  uint32_t* d_out_count = nullptr;
+  int64_t out_cap = 0;            // 0: n_cap
+  uint32_t* d_overflow = nullptr; // set to 4 when survivors exceed out_cap
+  void* scratch = nullptr;
+};
+
+size_t filter_scratch_bytes(int64_t n_cap);
+cudaError_t launch_filter(const FilterArgs& a, cudaStream_t st);
+
+cudaError_t launch_hash_init(uint64_t* table, uint32_t capacity, cudaStream_t st);
+cudaError_t launch_hash_build(const int32_t* keys, const int32_t* payload, const int32_t* in_tids,
+                              const uint32_t* d_in_count, int64_t n_cap, uint64_t* table, uint32_t capacity,
+                              uint32_t* d_error, cudaStream_t st);
+cudaError_t launch_gather(const void* col, int width, const int32_t* tids, const uint32_t* d_count,
+                          int64_t n_cap, void* out, cudaStream_t st);
+
+size_t groupby_table_bytes(uint32_t capacity, int n_aggs);
+cudaError_t launch_groupby_init(void* table, uint32_t capacity, int n_aggs, cudaStream_t st);
+cudaError_t launch_groupby(const int32_t* tids, const uint32_t* d_count, int64_t n_cap,
+                           const int32_t* const* key_vec, const int32_t* const* key_col, int n_keys,
+                           const ddq_dev_agg* aggs, int n_aggs, void* table, uint32_t capacity,
+                           uint32_t* d_error, cudaStream_t st);
+cudaError_t launch_groupby_compact(const void* table, uint32_t capacity, int n_aggs, int64_t* out_keys,
+                                   int64_t* out_accs, uint32_t* d_out_groups, cudaStream_t st);
+
+int num_sms();
+
+}  // namespace ddq

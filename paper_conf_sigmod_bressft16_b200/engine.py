@@ -1,0 +1,315 @@
+"""Python binding of the libddq database layer (include/ddq.h section 2).
+
+Argument marshalling only: plans are built here as C structs, every operator runs
+in libddq (sm_100a kernels or the C++ host executor the driver falls back to on an
+aborted GPU operator).  Names follow the paper: data cache + heap,
+data-driven placement, query chopping, Algorithm 1.
+"""
+from __future__ import annotations
+
+import ctypes
+from dataclasses import dataclass, field
+
+import numpy as np
+
+from . import _abi as A
+from ._abi import check, lib
+
+
+@dataclass
+class QueryResult:
+    """Rows (keys..., aggregates...) as Python ints, in ORDER BY order, or TIDs."""
+    rows: list = field(default_factory=list)
+    tids: np.ndarray | None = None
+    n_keys: int = 0
+    n_aggs: int = 0
+    gpu_ops: int = 0
+    host_ops: int = 0
+    aborts: int = 0
+    exec_ms: float = 0.0
+
+
+def _convert(res_ptr) -> QueryResult:
+    r = res_ptr.contents
+    out = QueryResult(n_keys=r.n_keys, n_aggs=r.n_aggs, gpu_ops=r.gpu_ops, host_ops=r.host_ops,
+                      aborts=r.aborts, exec_ms=r.exec_ms)
+    if r.n_tids > 0 or (r.n_rows == 0 and r.n_keys == 0 and r.n_aggs == 0):
+        out.tids = np.ctypeslib.as_array(r.tids, shape=(r.n_tids,)).copy() if r.n_tids else \
+            np.empty(0, np.int32)
+    nk, na = r.n_keys, r.n_aggs
+    for i in range(r.n_rows):
+        vals = [int(r.keys[i * nk + k]) for k in range(nk)]
+        for a in range(na):
+            lo = r.aggs[(i * na + a) * 2] & 0xFFFFFFFFFFFFFFFF
+            hi = r.aggs[(i * na + a) * 2 + 1]
+            vals.append((hi << 64) | lo)
+        out.rows.append(tuple(vals))
+    lib().ddq_result_free(res_ptr)
+    return out
+
+
+class PlanBuilder:
+    """Builds a ddq_plan (operator DAG, children before parents; last op = root)."""
+
+    def __init__(self, db: "Database"):
+        self.db = db
+        self.plan = A.Plan()
+        self.n = 0
+
+    def _op(self, kind: int, table: str, input: int = -1) -> tuple[int, A.Op]:
+        if self.n >= A.MAX_OPS:
+            raise ValueError("plan too long")
+        op = self.plan.ops[self.n]
+        ctypes.memset(ctypes.addressof(op), 0, ctypes.sizeof(op))
+        op.kind = kind
+        op.input = input
+        op.table = self.db.table_id(table)
+        op.build = -1
+        op.payload_col = -1
+        op.fk_col = -1
+        op.key_col = -1
+        op.gather_col = -1
+        idx = self.n
+        self.n += 1
+        self.plan.n_ops = self.n
+        return idx, op
+
+    def select(self, table: str, preds: list, input: int = -1) -> int:
+        """preds: list of (column, lo, hi) ranges or (column, [values]) IN-sets."""
+        idx, op = self._op(A.OP_SELECT, table, input)
+        if len(preds) > A.MAX_PREDS:
+            raise ValueError("too many predicates")
+        op.n_preds = len(preds)
+        for i, p in enumerate(preds):
+            pr = op.preds[i]
+            pr.column = self.db.col(table, p[0])
+            if len(p) == 3:
+                pr.kind, pr.lo, pr.hi = A.PRED_RANGE, int(p[1]), int(p[2])
+            else:
+                vals = list(p[1])
+                if not 1 <= len(vals) <= A.MAX_IN:
+                    raise ValueError("IN list must have 1..8 values")
+                pr.kind, pr.n_in = A.PRED_IN, len(vals)
+                for j, v in enumerate(vals):
+                    pr.in_vals[j] = int(v)
+        return idx
+
+    def build(self, table: str, key: str, payload: str | None = None, input: int = -1) -> int:
+        idx, op = self._op(A.OP_HASH_BUILD, table, input)
+        op.key_col = self.db.col(table, key)
+        op.payload_col = self.db.col(table, payload) if payload else -1
+        return idx
+
+    def probe(self, table: str, fk: str, build: int, input: int = -1, emit: bool = False) -> int:
+        idx, op = self._op(A.OP_HASH_PROBE, table, input)
+        op.fk_col = self.db.col(table, fk)
+        op.build = build
+        op.emit_payload = 1 if emit else 0
+        return idx
+
+    def gather(self, table: str, col: str, input: int) -> int:
+        idx, op = self._op(A.OP_GATHER, table, input)
+        op.gather_col = self.db.col(table, col)
+        return idx
+
+    def aggregate(self, table: str, input: int, keys: list, aggs: list, order_by: list | None = None,
+                  max_groups: int = 0, limit: int = 0) -> int:
+        """keys: int (aligned vector index) or str (column of `table`).
+        aggs: (kind, [cols]).  order_by: ints per include/ddq.h (+/-(1+k), +/-(101+a))."""
+        idx, op = self._op(A.OP_AGGREGATE, table, input)
+        op.n_keys = len(keys)
+        for k, src in enumerate(keys):
+            op.key_src[k] = src if isinstance(src, int) else -2 - self.db.col(table, src)
+        op.n_aggs = len(aggs)
+        for a, (kind, cols) in enumerate(aggs):
+            op.agg_kind[a] = kind
+            for j in range(3):
+                op.agg_col[a][j] = self.db.col(table, cols[j]) if j < len(cols) else -1
+        order_by = order_by or []
+        op.n_order = len(order_by)
+        for i, o in enumerate(order_by):
+            op.order_by[i] = o
+        op.max_groups = max_groups
+        op.limit = limit
+        return idx
+
+
+class Prepared:
+    """A plan placed entirely on the GPU and captured into one CUDA graph."""
+
+    def __init__(self, db: "Database", plan: A.Plan, use_graph: bool = True):
+        self.db = db
+        h = ctypes.c_void_p()
+        check(lib().ddq_prepare(db.h, ctypes.byref(plan), 1 if use_graph else 0, ctypes.byref(h)))
+        self.h = h
+        self.kernels = lib().ddq_prepared_kernel_count(h)
+
+    def launch(self, stream: int = 0) -> None:
+        check(lib().ddq_prepared_launch(self.h, ctypes.c_void_p(stream)))
+
+    def fetch(self, stream: int = 0) -> QueryResult:
+        p = ctypes.POINTER(A.Result)()
+        check(lib().ddq_prepared_fetch(self.h, ctypes.c_void_p(stream), ctypes.byref(p)))
+        return _convert(p)
+
+    def profile(self, stream: int = 0):
+        """Per-operator (ms, algorithmic bytes, class) from an event-timed replay."""
+        n = 64
+        ms = (ctypes.c_float * n)()
+        by = (ctypes.c_double * n)()
+        cl = (ctypes.c_int32 * n)()
+        k = lib().ddq_prepared_profile(self.h, ctypes.c_void_p(stream), n, ms, by, cl)
+        if k < 0:
+            check(k)
+        return [(float(ms[i]), float(by[i]), int(cl[i])) for i in range(k)]
+
+    def partials(self, stream: int = 0):
+        """Compacted partial group table (keys int64[g], accs int64[g, n_aggs, 2])."""
+        cap = lib().ddq_prepared_group_capacity(self.h)
+        keys = np.empty(max(cap, 1), np.int64)
+        na = self.db._root_aggs.get(id(self), 1)
+        accs = np.empty(max(cap, 1) * 16, np.int64)
+        g = ctypes.c_int64()
+        check(lib().ddq_prepared_partials(self.h, ctypes.c_void_p(stream), ctypes.byref(g),
+                                          keys.ctypes.data, accs.ctypes.data, cap))
+        return keys[:g.value], accs[:g.value * na * 2].reshape(g.value, na, 2)
+
+    def finalize(self, keys: np.ndarray, accs: np.ndarray) -> QueryResult:
+        keys = np.ascontiguousarray(keys, np.int64)
+        accs = np.ascontiguousarray(accs, np.int64)
+        p = ctypes.POINTER(A.Result)()
+        check(lib().ddq_prepared_finalize(self.h, keys.size, keys.ctypes.data, accs.ctypes.data, ctypes.byref(p)))
+        return _convert(p)
+
+    def close(self) -> None:
+        if self.h:
+            lib().ddq_prepared_free(self.h)
+            self.h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+class Database:
+    """A libddq database on one GPU: pinned host columns + device cache + heap."""
+
+    def __init__(self, device: int = 0, cache_bytes: int = 64 << 30, heap_bytes: int = 32 << 30,
+                 gpu_workers: int = 4, host_workers: int = 4, placement: int = A.PLACE_DATA_DRIVEN,
+                 chopping: bool = True, cache_policy: int = 0, fault_alloc_every: int = 0,
+                 rank: int = 0, world: int = 1):
+        cfg = A.Config()
+        lib().ddq_config_default(ctypes.byref(cfg))
+        cfg.device, cfg.rank, cfg.world = device, rank, world
+        cfg.cache_bytes, cfg.heap_bytes = cache_bytes, heap_bytes
+        cfg.gpu_workers, cfg.host_workers = gpu_workers, host_workers
+        cfg.placement, cfg.chopping = placement, 1 if chopping else 0
+        cfg.cache_policy, cfg.fault_alloc_every = cache_policy, fault_alloc_every
+        h = ctypes.c_void_p()
+        check(lib().ddq_open(ctypes.byref(cfg), ctypes.byref(h)))
+        self.h = h
+        self._tables: dict[str, int] = {}
+        self._cols: dict[tuple[str, str], int] = {}
+        self.dicts: dict[str, list[str]] = {}
+        self._root_aggs: dict = {}
+
+    def close(self) -> None:
+        if self.h:
+            lib().ddq_close(self.h)
+            self.h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    # ---- catalog -------------------------------------------------------------
+    def create_table(self, name: str, n_rows: int, row_begin: int = 0) -> int:
+        t = ctypes.c_int32()
+        check(lib().ddq_create_table(self.h, name.encode(), n_rows, row_begin, ctypes.byref(t)))
+        self._tables[name] = t.value
+        return t.value
+
+    def load_column(self, table: str, name: str, data: np.ndarray) -> int:
+        data = np.ascontiguousarray(data)
+        if data.dtype == np.int32:
+            ty = A.I32
+        elif data.dtype == np.int64:
+            ty = A.I64
+        else:
+            raise TypeError("columns are int32 or int64")
+        c = ctypes.c_int32()
+        check(lib().ddq_load_column(self.h, self._tables[table], name.encode(), ty, data.ctypes.data,
+                                    data.size, ctypes.byref(c)))
+        self._cols[(table, name)] = c.value
+        return c.value
+
+    def table_id(self, table: str) -> int:
+        return self._tables[table]
+
+    def col(self, table: str, name: str) -> int:
+        return self._cols[(table, name)]
+
+    def has_col(self, table: str, name: str) -> bool:
+        return (table, name) in self._cols
+
+    def cache(self, table: str, name: str) -> None:
+        check(lib().ddq_cache_column(self.h, self.col(table, name)))
+
+    def evict(self, table: str, name: str) -> None:
+        check(lib().ddq_evict_column(self.h, self.col(table, name)))
+
+    def is_cached(self, table: str, name: str) -> bool:
+        return bool(lib().ddq_column_is_cached(self.h, self.col(table, name)))
+
+    def device_ptr(self, table: str, name: str) -> int:
+        return lib().ddq_column_device_ptr(self.h, self.col(table, name)) or 0
+
+    def access_count(self, table: str, name: str) -> int:
+        return int(lib().ddq_column_access_count(self.h, self.col(table, name)))
+
+    def update_placement(self) -> None:
+        """Algorithm 1."""
+        check(lib().ddq_update_placement(self.h))
+
+    def reset_access_counts(self) -> None:
+        check(lib().ddq_reset_access_counts(self.h))
+
+    # ---- plans -----------------------------------------------------------------
+    def plan(self) -> PlanBuilder:
+        return PlanBuilder(self)
+
+    def submit(self, plan: PlanBuilder | A.Plan) -> int:
+        p = plan.plan if isinstance(plan, PlanBuilder) else plan
+        q = ctypes.c_int64()
+        check(lib().ddq_submit(self.h, ctypes.byref(p), ctypes.byref(q)))
+        return q.value
+
+    def wait(self, q: int, timeout_s: float | None = None) -> None:
+        check(lib().ddq_wait(self.h, q, -1 if timeout_s is None else int(timeout_s * 1e9)))
+
+    def fetch(self, q: int) -> QueryResult:
+        p = ctypes.POINTER(A.Result)()
+        check(lib().ddq_fetch(self.h, q, ctypes.byref(p)))
+        return _convert(p)
+
+    def run(self, plan: PlanBuilder | A.Plan) -> QueryResult:
+        return self.fetch(self.submit(plan))
+
+    def prepare(self, plan: PlanBuilder | A.Plan, use_graph: bool = True) -> Prepared:
+        p = plan.plan if isinstance(plan, PlanBuilder) else plan
+        pr = Prepared(self, p, use_graph)
+        self._root_aggs[id(pr)] = p.ops[p.n_ops - 1].n_aggs
+        return pr
+
+    # ---- statistics -----------------------------------------------------------
+    def stats(self) -> dict:
+        s = A.Stats()
+        check(lib().ddq_get_stats(self.h, ctypes.byref(s)))
+        return {n: int(getattr(s, n)) for n, _ in A.Stats._fields_}
+
+    def reset_stats(self) -> None:
+        check(lib().ddq_reset_stats(self.h))

@@ -1,0 +1,177 @@
+"""Operator-level parity of the sm_100a kernels against library routines on
+seeded random inputs (SURVEY.md 4.2 "Unit (GPU)"): select vs numpy.flatnonzero,
+build/probe vs numpy.isin + a dict, gather vs numpy.take, group-by vs numpy.unique
+with exact Python-int sums.  Sizes span several 4096-row tiles plus ragged tails,
+and the edge cases n = 0, 1, 31, 32, 33, all-pass and none-pass."""
+import numpy as np
+import pytest
+
+pytestmark = pytest.mark.gpu
+
+SIZES = [0, 1, 31, 32, 33, 4095, 4096, 4097, 100_003, 3_000_017]
+
+
+def _t(a):
+    import torch
+    return torch.from_numpy(np.ascontiguousarray(a)).cuda()
+
+
+@pytest.fixture(scope="module")
+def ops():
+    from paper_conf_sigmod_bressft16_b200 import ops
+    return ops
+
+
+@pytest.mark.parametrize("n", SIZES)
+def test_select_dense_int64_range(ops, n):
+    rng = np.random.default_rng(n)
+    a = rng.integers(0, 11, n, dtype=np.int64)
+    b = rng.integers(1, 51, n, dtype=np.int64)
+    tids, cnt, _ = ops.select([(_t(a), 4, 6), (_t(b), 26, 35)], n)
+    want = np.flatnonzero((a >= 4) & (a <= 6) & (b >= 26) & (b <= 35))
+    c = int(cnt[0].item())
+    assert c == want.size
+    assert np.array_equal(tids[:c].cpu().numpy(), want)
+
+
+@pytest.mark.parametrize("n", [0, 5, 4097, 1_000_001])
+def test_select_int32_in_set_and_all_none(ops, n):
+    rng = np.random.default_rng(7 + n)
+    a = rng.integers(0, 250, n, dtype=np.int32)
+    tids, cnt, _ = ops.select([(_t(a), [3, 17, 249, 0])], n)
+    want = np.flatnonzero(np.isin(a, [3, 17, 249, 0]))
+    c = int(cnt[0].item())
+    assert np.array_equal(tids[:c].cpu().numpy(), want)
+    _, cnt_all, _ = ops.select([(_t(a), -1, 1000)], n)
+    _, cnt_none, _ = ops.select([(_t(a), 1000, 2000)], n)
+    assert int(cnt_all[0].item()) == n and int(cnt_none[0].item()) == 0
+
+
+@pytest.mark.parametrize("n", [0, 33, 4097, 777_777])
+def test_select_at_tids_with_carry(ops, n):
+    import torch
+    rng = np.random.default_rng(11 + n)
+    N = max(n * 3, 1)
+    col = rng.integers(0, 100, N, dtype=np.int64)
+    tids_in = np.sort(rng.choice(N, size=n, replace=False)).astype(np.int32)
+    carry = rng.integers(-5, 5, n, dtype=np.int32)
+    cnt_in = ops.count_cell(n)
+    out, cnt, couts = ops.select([(_t(col), 10, 40)], n, in_tids=_t(tids_in) if n else
+                                 torch.empty(1, dtype=torch.int32, device="cuda"), in_count=cnt_in,
+                                 carry=[_t(carry) if n else torch.empty(1, dtype=torch.int32, device="cuda")])
+    keep = (col[tids_in] >= 10) & (col[tids_in] <= 40)
+    c = int(cnt[0].item())
+    assert c == int(keep.sum())
+    assert np.array_equal(out[:c].cpu().numpy(), tids_in[keep])
+    assert np.array_equal(couts[0][:c].cpu().numpy(), carry[keep])
+
+
+@pytest.mark.parametrize("ndim,nfact", [(2557, 4097), (40_000, 1_000_003), (600_000, 3_000_000), (1, 100)])
+def test_build_probe_semijoin_payload(ops, ndim, nfact):
+    rng = np.random.default_rng(ndim)
+    keys = rng.permutation(np.arange(1, 3 * ndim + 1, dtype=np.int32))[:ndim]  # sparse unique keys
+    payload = rng.integers(0, 1000, ndim, dtype=np.int32)
+    sel = np.flatnonzero(rng.random(ndim) < 0.3).astype(np.int32)
+    cap = 16
+    while cap < 2 * max(sel.size, 1):
+        cap *= 2
+    table, err = ops.hash_build(_t(keys), cap, payload=_t(payload), in_tids=_t(sel) if sel.size else None,
+                                in_count=ops.count_cell(sel.size) if sel.size else None, n=sel.size)
+    assert int(err[0].item()) == 0
+    fk = rng.integers(1, 3 * ndim + 1, nfact, dtype=np.int32)
+    out, pay, cnt, _ = ops.hash_probe(table, _t(fk), nfact, emit_payload=True)
+    m = dict(zip(keys[sel].tolist(), payload[sel].tolist()))
+    want = np.flatnonzero(np.isin(fk, keys[sel]))
+    c = int(cnt[0].item())
+    assert c == want.size
+    assert np.array_equal(out[:c].cpu().numpy(), want)
+    assert pay[:c].cpu().numpy().tolist() == [m[int(k)] for k in fk[want]]
+
+
+def test_build_rejects_duplicate_keys(ops):
+    keys = np.array([5, 9, 5, 1], dtype=np.int32)
+    _, err = ops.hash_build(_t(keys), 16)
+    assert int(err[0].item()) == 1
+
+
+def test_probe_chain_at_tids_carries_payload(ops):
+    rng = np.random.default_rng(3)
+    n = 200_000
+    fk1 = rng.integers(1, 1001, n, dtype=np.int32)
+    fk2 = rng.integers(1, 101, n, dtype=np.int32)
+    t1, _ = ops.hash_build(_t(np.arange(1, 501, dtype=np.int32)), 1024,
+                           payload=_t(np.arange(1, 501, dtype=np.int32) * 7))
+    t2, _ = ops.hash_build(_t(np.arange(1, 101, 3, dtype=np.int32)), 128)
+    o1, p1, c1, _ = ops.hash_probe(t1, _t(fk1), n, emit_payload=True)
+    n1 = int(c1[0].item())
+    o2, _, c2, carried = ops.hash_probe(t2, _t(fk2), n1, in_tids=o1, in_count=c1, carry=[p1])
+    n2 = int(c2[0].item())
+    m = (fk1 <= 500) & np.isin(fk2, np.arange(1, 101, 3))
+    want = np.flatnonzero(m)
+    assert np.array_equal(o2[:n2].cpu().numpy(), want)
+    assert np.array_equal(carried[0][:n2].cpu().numpy(), fk1[want] * 7)
+
+
+@pytest.mark.parametrize("dtype", [np.int32, np.int64])
+def test_gather(ops, dtype):
+    rng = np.random.default_rng(5)
+    col = rng.integers(-2**30, 2**30, 1_000_003).astype(dtype)
+    tids = np.sort(rng.choice(col.size, 123_457, replace=False)).astype(np.int32)
+    out = ops.gather(_t(col), _t(tids), ops.count_cell(tids.size), tids.size)
+    assert np.array_equal(out[:tids.size].cpu().numpy(), col[tids])
+
+
+def _acc_to_int(accs):
+    a = accs.cpu().numpy()
+    lo = a[..., 0].astype(np.uint64).astype(object)
+    hi = a[..., 1].astype(object)
+    return hi * (1 << 64) + lo
+
+
+@pytest.mark.parametrize("ngroups,n", [(1, 1_000_000), (7, 33), (800, 2_000_003), (50_000, 1_500_000)])
+def test_groupby_exact(ops, ngroups, n):
+    from paper_conf_sigmod_bressft16_b200 import _abi as A
+    rng = np.random.default_rng(ngroups)
+    N = n + 1000
+    tids = np.sort(rng.choice(N, n, replace=False)).astype(np.int32)
+    k0 = rng.integers(0, ngroups, n, dtype=np.int32)             # aligned vector key
+    kc = rng.integers(0, 3, N, dtype=np.int32)                   # column key at tid
+    ep = rng.integers(90_000 * 1, 209_900 * 50, N, dtype=np.int64)
+    d = rng.integers(0, 11, N, dtype=np.int64)
+    t = rng.integers(0, 9, N, dtype=np.int64)
+    sc = rng.integers(0, 10**7, N, dtype=np.int64) * 3
+    aggs = [(A.AGG_SUM_MUL, [_t(ep), _t(d)]), (A.AGG_COUNT, []), (A.AGG_SUM_SUB, [_t(d), _t(sc)]),
+            (A.AGG_SUM_MUL_100M_100P, [_t(ep), _t(d), _t(t)]), (A.AGG_SUM_MUL_100M, [_t(ep), _t(d)]),
+            (A.AGG_SUM, [_t(sc)])]
+    cap = 64
+    while cap < 2 * ngroups * 3:
+        cap *= 2
+    keys, accs, err = ops.groupby(_t(tids), ops.count_cell(n), n, key_vecs=[_t(k0), None],
+                                  key_cols=[None, _t(kc)], aggs=aggs, capacity=cap)
+    assert err == 0
+    keys = keys.cpu().numpy()
+    got = _acc_to_int(accs)
+    r = tids
+    key = k0.astype(np.int64) | (kc[r].astype(np.int64) << 21)
+    vals = [ep[r].astype(object) * d[r], np.ones(n, dtype=object), d[r].astype(object) - sc[r],
+            ep[r].astype(object) * (100 - d[r]) * (100 + t[r]), ep[r].astype(object) * (100 - d[r]),
+            sc[r].astype(object)]
+    uk = np.unique(key)
+    assert sorted(keys.tolist()) == uk.tolist()
+    pos = {int(k): i for i, k in enumerate(keys)}
+    for a, v in enumerate(vals):
+        want = {}
+        for kk, vv in zip(key.tolist(), v.tolist()):
+            want[kk] = want.get(kk, 0) + vv
+        for kk, vv in want.items():
+            assert got[pos[kk], a] == vv, (a, kk)
+
+
+def test_groupby_overflow_flagged(ops):
+    from paper_conf_sigmod_bressft16_b200 import _abi as A
+    n = 10_000
+    tids = np.arange(n, dtype=np.int32)
+    k = np.arange(n, dtype=np.int32)
+    _, _, err = ops.groupby(_t(tids), ops.count_cell(n), n, key_vecs=[_t(k)],
+                            aggs=[(A.AGG_COUNT, [])], capacity=1024)
+    assert err == 2
