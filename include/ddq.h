@@ -117,6 +117,26 @@ ddq_status ddq_op_hash_probe(const uint64_t* table, uint32_t capacity, const int
                              int32_t* out_tids, int32_t* out_payload, uint32_t* d_out_count,
                              void* scratch, size_t scratch_bytes, void* stream);
 
+/* Direct-mapped join index (S8(a3)/(a4), the build/probe used when the build key
+ * column spans a compact range [key_min, key_min + range)): a membership bitmap of
+ * `range` bits followed (16-byte aligned) by an int32 payload array of `range`
+ * entries; ddq_op_join_index_bytes(range) bytes, zero the bitmap with
+ * ddq_op_join_index_init.  Same semantics as hash build / probe: unique keys
+ * (duplicate -> *d_error = 1; key outside the range -> *d_error = 3), probe =
+ * semi-join + payload of survivors.  Chosen by the engine when range <= 16 x the
+ * dimension's rows (dimension primary keys); hash tables remain the general path. */
+size_t ddq_op_join_index_bytes(uint32_t range);
+ddq_status ddq_op_join_index_init(void* index, uint32_t range, void* stream);
+ddq_status ddq_op_join_index_build(const int32_t* keys, const int32_t* payload,
+                                   const int32_t* in_tids, const uint32_t* d_in_count, int64_t n_cap,
+                                   int32_t key_min, uint32_t range, void* index, uint32_t* d_error,
+                                   void* stream);
+ddq_status ddq_op_join_index_probe(const void* index, int32_t key_min, uint32_t range, const int32_t* fk,
+                                   const int32_t* in_tids, const uint32_t* d_in_count, int64_t n_cap,
+                                   const int32_t* const* carry_in, int32_t* const* carry_out, int32_t n_carry,
+                                   int32_t* out_tids, int32_t* out_payload, uint32_t* d_out_count,
+                                   void* scratch, size_t scratch_bytes, void* stream);
+
 /* Positional gather (S8(a5); P:107 materialisation): out[i] = col[tids[i]] for
  * i < *d_count; width 4 or 8. */
 ddq_status ddq_op_gather(const void* col, int32_t width, const int32_t* tids,

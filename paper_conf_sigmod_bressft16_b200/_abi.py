@@ -93,6 +93,11 @@ SIGNATURES = {
     "ddq_op_hash_init": (_i32, [_vp, _u32, _vp]),
     "ddq_op_hash_build": (_i32, [_vp, _vp, _vp, _vp, _i64, _vp, _u32, _vp, _vp]),
     "ddq_op_hash_probe": (_i32, [_vp, _u32, _vp, _vp, _vp, _i64, _pp, _pp, _i32, _vp, _vp, _vp, _vp, _sz, _vp]),
+    "ddq_op_join_index_bytes": (_sz, [_u32]),
+    "ddq_op_join_index_init": (_i32, [_vp, _u32, _vp]),
+    "ddq_op_join_index_build": (_i32, [_vp, _vp, _vp, _vp, _i64, _i32, _u32, _vp, _vp, _vp]),
+    "ddq_op_join_index_probe": (_i32, [_vp, _i32, _u32, _vp, _vp, _vp, _i64, _pp, _pp, _i32, _vp, _vp, _vp, _vp,
+                                       _sz, _vp]),
     "ddq_op_gather": (_i32, [_vp, _i32, _vp, _vp, _i64, _vp, _vp]),
     "ddq_op_groupby_table_bytes": (_sz, [_u32, _i32]),
     "ddq_op_groupby_init": (_i32, [_vp, _u32, _i32, _vp]),

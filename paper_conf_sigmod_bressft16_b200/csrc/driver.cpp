@@ -107,11 +107,21 @@ ddq_status inter_to_host(ddq_db* db, Inter& x, cudaStream_t st) {
     h.table_cap = x.table_cap;
     bytes += (uint64_t)x.table_cap * 8;
   }
+  if (x.jidx) {
+    const size_t words = ((size_t)x.jrange + 31) / 32;
+    auto bm = std::make_shared<std::vector<uint32_t>>(words);
+    auto pa = std::make_shared<std::vector<int32_t>>(x.jrange);
+    cudaMemcpyAsync(bm->data(), x.jidx, words * 4, cudaMemcpyDeviceToHost, st);
+    cudaMemcpyAsync(pa->data(), join_index_payload(x.jidx, x.jrange), (size_t)x.jrange * 4,
+                    cudaMemcpyDeviceToHost, st);
+    h.h_bitmap = bm;
+    h.h_payarr = pa;
+    h.jmin = x.jmin;
+    h.jrange = x.jrange;
+    bytes += words * 4 + (uint64_t)x.jrange * 4;
+  }
   if (x.gb_table) {
-    uint32_t g = 0;
-    cudaMemcpyAsync(&g, x.gb_groups, 4, cudaMemcpyDeviceToHost, st);
-    cudaStreamSynchronize(st);
-    // aggregate inputs are consumed by finalisation only; keep the arrays
+    // aggregate outputs are consumed by finalisation only
     return set_error(DDQ_ESTATE, "aggregate output cannot move");
   }
   if (x.tids || x.d_count) {
@@ -154,7 +164,21 @@ static ddq_status inter_to_device(ddq_db* db, Inter& x, cudaStream_t st) {
     if (p) d.heap_blocks.push_back(p);
     return p;
   };
-  if (x.host_table) {
+  if (x.h_bitmap) {
+    d.jmin = x.jmin;
+    d.jrange = x.jrange;
+    d.jidx = get(join_index_bytes(x.jrange));
+    d.d_error = (uint32_t*)get(64);
+    if (!d.jidx || !d.d_error) {
+      release_inter(db, d);
+      return DDQ_ENOMEM_DEVICE;
+    }
+    cudaMemsetAsync(d.d_error, 0, 4, st);
+    cudaMemcpyAsync(d.jidx, x.h_bitmap->data(), x.h_bitmap->size() * 4, cudaMemcpyHostToDevice, st);
+    cudaMemcpyAsync(join_index_payload(d.jidx, d.jrange), x.h_payarr->data(), (size_t)x.jrange * 4,
+                    cudaMemcpyHostToDevice, st);
+    bytes += x.h_bitmap->size() * 4 + (uint64_t)x.jrange * 4;
+  } else if (x.host_table) {
     d.table_cap = x.table_cap;
     d.table_ptr = (uint64_t*)get((uint64_t)x.table_cap * 8);
     d.d_error = (uint32_t*)get(64);
@@ -249,15 +273,16 @@ ddq_status run_host_op(ddq_db* db, const ddq_op& op, const std::vector<Inter>& I
     case DDQ_OP_HASH_PROBE: {
       const bool probe = op.kind == DDQ_OP_HASH_PROBE;
       const Inter* build = probe ? &I[(size_t)op.build] : nullptr;
-      if (probe && !build->host_table) return set_error(DDQ_ESTATE, "host probe needs a host table");
+      if (probe && !build->host_table && !build->h_bitmap) return set_error(DDQ_ESTATE, "host probe needs a host table");
+      const bool direct = probe && build->h_bitmap != nullptr;
       std::vector<const Column*> pc;
       for (int i = 0; i < op.n_preds && !probe; i++) pc.push_back(col_of(db, op.preds[i].column));
       const Column* fk = probe ? col_of(db, op.fk_col) : nullptr;
       int lg = 0;
-      if (probe)
+      if (probe && !direct)
         while ((1u << lg) < build->table_cap) lg++;
-      const uint64_t* tab = probe ? build->host_table->data() : nullptr;
-      const uint32_t mask = probe ? build->table_cap - 1 : 0;
+      const uint64_t* tab = (probe && !direct) ? build->host_table->data() : nullptr;
+      const uint32_t mask = (probe && !direct) ? build->table_cap - 1 : 0;
       int nchunks = (threads <= 1 || n < (1 << 16)) ? 1 : threads;
       std::vector<std::vector<int64_t>> sel((size_t)nchunks);     // positions i
       std::vector<std::vector<int32_t>> pay((size_t)nchunks);
@@ -281,6 +306,15 @@ ddq_status run_host_op(ddq_db* db, const ddq_op& op, const std::vector<Inter>& I
             if (ok) S.push_back(i);
           } else {
             int32_t k = ((const int32_t*)fk->host)[r];
+            if (direct) {
+              const uint32_t o = (uint32_t)(k - build->jmin);
+              ok = o < build->jrange && (((*build->h_bitmap)[o >> 5] >> (o & 31)) & 1u);
+              if (ok) {
+                Pv.push_back((*build->h_payarr)[o]);
+                S.push_back(i);
+              }
+              continue;
+            }
             uint32_t h = host_hash32(k, 32 - lg);
             while (true) {
               uint64_t s = tab[h];
@@ -511,6 +545,7 @@ static void finish_query(ddq_db* db, QueryState& q) {
       int32_t* t = new int32_t[(size_t)std::max<int64_t>(r.count, 1)];
       const int64_t base = db->tables[(size_t)root.table].row_begin;
       for (int64_t i = 0; i < r.count; i++) t[i] = (int32_t)(r.tids[i] + base);
+      std::sort(t, t + r.count);  // a select-* result is a set of rows: row order (S8(a7))
       res->n_tids = r.count;
       res->tids = t;
     }
@@ -643,7 +678,7 @@ static void run_on_gpu(ddq_db* db, std::shared_ptr<QueryState> q, int i, cudaStr
       out.count = c;
       out.cap = c;  // exact cardinality is known at run time: consumers allocate exactly
     }
-    if (s == DDQ_OK && out.table_ptr && out.d_error) {
+    if (s == DDQ_OK && (out.table_ptr || out.jidx) && out.d_error) {
       uint32_t e2 = 0;
       cudaMemcpy(&e2, out.d_error, 4, cudaMemcpyDeviceToHost);
       if (e2) s = set_error(e2 == 2 ? DDQ_EOVERFLOW : DDQ_EINVAL, "hash build failed (duplicate key or overflow)");
@@ -763,9 +798,12 @@ ddq_status ddq_submit(ddq_db* db, const ddq_plan* plan, ddq_query* out) {
     db->queries[q->id] = q;
   }
   *out = q->id;
-  // leaf operators enter the global operator stream
+  // leaf operators enter the global operator stream.  Collect them first:
+  // once one is enqueued, workers may finish it and make parents ready concurrently.
+  std::vector<int> leaves;
   for (int i = 0; i < n; i++)
-    if (q->pending[(size_t)i] == 0) enqueue(db, q, i);
+    if (q->pending[(size_t)i] == 0) leaves.push_back(i);
+  for (int i : leaves) enqueue(db, q, i);
   return DDQ_OK;
 }
 

@@ -99,6 +99,15 @@ void release_inter(ddq_db* db, Inter& x) {
   x.host_blocks.clear();
 }
 
+// A dimension key column whose values span a compact range gets a direct-mapped
+// join index (bitmap + payload array) instead of a hash table: one probe per row,
+// no collision chains.  Range <= 2^20 or <= 16 x the rows (primary keys 1..n).
+bool use_join_index(const Column& kc, int64_t n_rows) {
+  if (kc.vmax < kc.vmin) return false;
+  const int64_t r = kc.vmax - kc.vmin + 1;
+  return r <= (1ll << 28) && (r <= (1ll << 20) || r <= 16 * std::max<int64_t>(n_rows, 1));
+}
+
 // ----------------------------------------------------------- GPU operator runner
 struct Alloc {
   ddq_db* db;
@@ -185,7 +194,8 @@ ddq_status run_gpu_op(GpuOpCtx& ctx, const ddq_op& op, Inter& out) {
       if (probe) {
         if (op.build < 0 || op.build >= (int)I.size()) return set_error(DDQ_EINVAL, "probe: bad build index");
         build = &I[(size_t)op.build];
-        if (!build->table_ptr) return set_error(DDQ_ESTATE, "probe: build side is not a device hash table");
+        if (!build->table_ptr && !build->jidx)
+          return set_error(DDQ_ESTATE, "probe: build side is not a device hash table / join index");
         const Column* c = col_of(db, op.fk_col);
         if (!c || c->table != op.table || c->width != 4) return set_error(DDQ_EINVAL, "probe: bad fk column");
         fk = (const int32_t*)need_col(op.fk_col);
@@ -224,6 +234,12 @@ ddq_status run_gpu_op(GpuOpCtx& ctx, const ddq_op& op, Inter& out) {
       if (probe) {
         fa.table = build->table_ptr;
         fa.capacity = build->table_cap;
+        if (build->jidx) {
+          fa.bitmap = join_index_bitmap(build->jidx);
+          fa.payarr = join_index_payload(build->jidx, build->jrange);
+          fa.key_min = build->jmin;
+          fa.range = build->jrange;
+        }
         fa.fk = fk;
         fa.out_payload = payload;
       }
@@ -260,7 +276,23 @@ ddq_status run_gpu_op(GpuOpCtx& ctx, const ddq_op& op, Inter& out) {
         if (!payload) return set_error(DDQ_ESTATE, "build: payload column not cached on the GPU");
       }
       if (!keys) return set_error(DDQ_ESTATE, "build: key column not cached on the GPU");
+      if (use_join_index(*kc, T.n_rows)) {  // compact key range: direct-mapped join index
+        out.jmin = (int32_t)kc->vmin;
+        out.jrange = (uint32_t)(kc->vmax - kc->vmin + 1);
+        out.jidx = A.get(join_index_bytes(out.jrange));
+        out.d_error = (uint32_t*)A.get(64);
+        out.cap = 0;
+        if (A.failed) return DDQ_ENOMEM_DEVICE;
+        cudaMemsetAsync(out.d_error, 0, 4, st);
+        cudaError_t e = cudaMemsetAsync(out.jidx, 0, ((size_t)out.jrange + 31) / 32 * 4, st);
+        if (e == cudaSuccess)
+          e = launch_join_index_build(keys, payload, in_tids, in_cnt, in_cap, out.jmin, out.jrange, out.jidx,
+                                      out.d_error, st);
+        return cuda_status(e, "join_index_build");
+      }
+      // sparse keys: open addressing; small tables (shared-memory resident) get load <= 0.25
       int64_t cap = pow2_at_least(std::max<int64_t>(16, 2 * out_cap));
+      if (cap * 2 * 8 <= 64 * 1024) cap *= 2;
       if (cap > (1ll << 31)) return set_error(DDQ_EINVAL, "build: table too large");
       out.table_cap = (uint32_t)cap;
       out.table_ptr = (uint64_t*)A.get((uint64_t)cap * 8);
@@ -506,6 +538,11 @@ ddq_status ddq_load_column(ddq_db* db, ddq_table t, const char* name, ddq_type t
   cudaError_t e = cudaHostAlloc(&c->host, bytes, cudaHostAllocPortable);
   if (e != cudaSuccess) return set_error(DDQ_ENOMEM_HOST, "load_column: pinned alloc failed");
   std::memcpy(c->host, host_data, (size_t)n_rows * c->width);
+  for (int64_t i = 0; i < n_rows; i++) {
+    int64_t v = c->width == 4 ? ((const int32_t*)host_data)[i] : ((const int64_t*)host_data)[i];
+    if (i == 0 || v < c->vmin) c->vmin = v;
+    if (i == 0 || v > c->vmax) c->vmax = v;
+  }
   db->cols.push_back(std::move(c));
   int id = (int)db->cols.size() - 1;
   db->tables[(size_t)t].cols.push_back(id);
@@ -1079,6 +1116,8 @@ ddq_status ddq_prepared_fetch(ddq_prepared* p, void* stream, ddq_result** out) {
       delete res;
       return cuda_status(e, "prepared_fetch tids");
     }
+    // a select-* result is a set of rows; present it in row order (S8(a7))
+    std::sort(t, t + n);
     const int64_t base = p->db->tables[(size_t)root.table].row_begin;
     for (uint32_t i = 0; i < n; i++) t[i] = (int32_t)(t[i] + base);
     res->n_tids = n;

@@ -50,6 +50,7 @@ struct Column {
   int type = DDQ_I32;
   int width = 4;
   int64_t n = 0;
+  int64_t vmin = 0, vmax = -1;  // value range (computed at load; sizes join indexes)
   void* host = nullptr;   // pinned host copy
   void* dev = nullptr;    // device cache copy or nullptr
   std::atomic<uint64_t> access{0};
@@ -88,6 +89,12 @@ struct Inter {
   uint32_t* d_error = nullptr;
   // host-side hash table (host build)
   std::shared_ptr<std::vector<uint64_t>> host_table;
+  // direct-mapped join index (device: jidx; host copy: h_bitmap/h_payarr)
+  void* jidx = nullptr;
+  int32_t jmin = 0;
+  uint32_t jrange = 0;
+  std::shared_ptr<std::vector<uint32_t>> h_bitmap;
+  std::shared_ptr<std::vector<int32_t>> h_payarr;
   // aggregate output
   void* gb_table = nullptr;
   uint32_t gb_cap = 0;

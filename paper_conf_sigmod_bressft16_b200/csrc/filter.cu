@@ -50,6 +50,11 @@ struct FilterParams {
   int32_t shift;
   const int32_t* fk;
   int32_t* out_payload;
+  int32_t direct;  // direct-mapped join index instead of the hash table
+  const uint32_t* bitmap;
+  const int32_t* payarr;
+  int32_t key_min;
+  uint32_t range;
   // carries
   int32_t n_carry;
   const int32_t* carry_in[4];
@@ -177,23 +182,42 @@ filter_kernel(const __grid_constant__ FilterParams P) {
 #pragma unroll
         for (int k = 0; k < FT_ITEMS; k++) keys[k] = ((flags >> k) & 1u) ? __ldg(P.fk + rows[k]) : 0;
       }
-      uint32_t h[FT_ITEMS];
-      uint64_t sl[FT_ITEMS];
+      if (P.direct) {
+        uint32_t w[FT_ITEMS];
 #pragma unroll
-      for (int k = 0; k < FT_ITEMS; k++) {
-        h[k] = ht_hash(keys[k], P.shift);
-        sl[k] = ((flags >> k) & 1u) ? table[h[k]] : HT_EMPTY;
-      }
-#pragma unroll
-      for (int k = 0; k < FT_ITEMS; k++) {
-        uint64_t s = sl[k];
-        uint32_t hh = h[k];
-        while (s != HT_EMPTY && ht_key(s) != keys[k]) {
-          hh = (hh + 1) & P.cap_mask;
-          s = table[hh];
+        for (int k = 0; k < FT_ITEMS; k++) {
+          const uint32_t o = (uint32_t)(keys[k] - P.key_min);
+          w[k] = (((flags >> k) & 1u) && o < P.range) ? __ldg(P.bitmap + (o >> 5)) : 0u;
         }
-        if (s == HT_EMPTY) flags &= ~(1u << k);
-        payload[k] = ht_val(s);
+#pragma unroll
+        for (int k = 0; k < FT_ITEMS; k++) {
+          const uint32_t o = (uint32_t)(keys[k] - P.key_min);
+          if (!((w[k] >> (o & 31)) & 1u)) flags &= ~(1u << k);
+        }
+        if (P.out_payload) {
+#pragma unroll
+          for (int k = 0; k < FT_ITEMS; k++)
+            payload[k] = ((flags >> k) & 1u) ? __ldg(P.payarr + (uint32_t)(keys[k] - P.key_min)) : 0;
+        }
+      } else {
+        uint32_t h[FT_ITEMS];
+        uint64_t sl[FT_ITEMS];
+#pragma unroll
+        for (int k = 0; k < FT_ITEMS; k++) {
+          h[k] = ht_hash(keys[k], P.shift);
+          sl[k] = ((flags >> k) & 1u) ? table[h[k]] : HT_EMPTY;
+        }
+#pragma unroll
+        for (int k = 0; k < FT_ITEMS; k++) {
+          uint64_t s = sl[k];
+          uint32_t hh = h[k];
+          while (s != HT_EMPTY && ht_key(s) != keys[k]) {
+            hh = (hh + 1) & P.cap_mask;
+            s = table[hh];
+          }
+          if (s == HT_EMPTY) flags &= ~(1u << k);
+          payload[k] = ht_val(s);
+        }
       }
     }
 
@@ -285,6 +309,7 @@ size_t filter_scratch_bytes(int64_t n_cap) {
 constexpr size_t kSmemTableMax = 96 * 1024;
 
 cudaError_t launch_filter(const FilterArgs& a, cudaStream_t st) {
+  if (!a.stable && scan_supported(a)) return launch_scan(a, st);
   FilterParams p{};
   p.in_tids = a.in_tids;
   p.d_in_count = a.d_in_count;
@@ -306,6 +331,11 @@ cudaError_t launch_filter(const FilterArgs& a, cudaStream_t st) {
   p.shift = 32 - lg;
   p.fk = a.fk;
   p.out_payload = a.out_payload;
+  p.direct = a.bitmap != nullptr;
+  p.bitmap = a.bitmap;
+  p.payarr = a.payarr;
+  p.key_min = a.key_min;
+  p.range = a.range;
   p.n_carry = a.n_carry;
   for (int c = 0; c < a.n_carry && c < 4; c++) {
     p.carry_in[c] = a.carry_in[c];
@@ -325,7 +355,7 @@ cudaError_t launch_filter(const FilterArgs& a, cudaStream_t st) {
     return tids ? launch_t<true, false, false>(p, a.n_cap, 0, st) : launch_t<false, false, false>(p, a.n_cap, 0, st);
   }
   size_t tbytes = (size_t)a.capacity * 8;
-  if (tbytes <= kSmemTableMax && !a.no_smem) {
+  if (!p.direct && tbytes <= kSmemTableMax && !a.no_smem) {
     return tids ? launch_t<true, true, true>(p, a.n_cap, tbytes, st)
                 : launch_t<false, true, true>(p, a.n_cap, tbytes, st);
   }

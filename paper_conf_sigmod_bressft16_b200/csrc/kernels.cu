@@ -88,6 +88,39 @@ cudaError_t launch_hash_build(const int32_t* keys, const int32_t* payload, const
   return cudaGetLastError();
 }
 
+// ------------------------------------------------------- direct-mapped join index
+size_t join_index_bytes(uint32_t range) {
+  return ((((size_t)range + 31) / 32 * 4 + 15) / 16) * 16 + (size_t)range * 4;
+}
+
+__global__ void join_index_build_kernel(const int32_t* __restrict__ keys, const int32_t* __restrict__ payload,
+                                        const int32_t* __restrict__ in_tids, const uint32_t* d_in_count,
+                                        uint32_t n_static, int32_t key_min, uint32_t range, uint32_t* bitmap,
+                                        int32_t* payarr, uint32_t* d_error) {
+  const uint32_t n = d_in_count ? ld_relaxed_u32(d_in_count) : n_static;
+  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
+    const int32_t r = in_tids ? in_tids[i] : (int32_t)i;
+    const uint32_t o = (uint32_t)(keys[r] - key_min);
+    if (o >= range) {
+      atomicMax(d_error, 3u);
+      continue;
+    }
+    const uint32_t old = atomicOr(bitmap + (o >> 5), 1u << (o & 31));
+    if (old & (1u << (o & 31))) atomicMax(d_error, 1u);  // PKs are unique (O13)
+    payarr[o] = payload ? payload[r] : r;
+  }
+}
+
+cudaError_t launch_join_index_build(const int32_t* keys, const int32_t* payload, const int32_t* in_tids,
+                                    const uint32_t* d_in_count, int64_t n_cap, int32_t key_min, uint32_t range,
+                                    void* index, uint32_t* d_error, cudaStream_t st) {
+  int64_t g = (n_cap + 255) / 256;
+  int grid = (int)(g > num_sms() * 8 ? num_sms() * 8 : (g < 1 ? 1 : g));
+  join_index_build_kernel<<<grid, 256, 0, st>>>(keys, payload, in_tids, d_in_count, (uint32_t)n_cap, key_min, range,
+                                                join_index_bitmap(index), join_index_payload(index, range), d_error);
+  return cudaGetLastError();
+}
+
 // --------------------------------------------------------------------- gather
 template <int W>
 __global__ void gather_kernel(const void* __restrict__ col, const int32_t* __restrict__ tids,

@@ -40,7 +40,7 @@ ddq_status ddq_op_select(const ddq_dev_pred* preds, int32_t n_preds, const int32
     return set_error(DDQ_EINVAL, "select: bad predicate list");
   if (n_carry < 0 || n_carry > DDQ_MAX_CARRY) return set_error(DDQ_EINVAL, "select: bad carry count");
   for (int i = 0; i < n_preds; i++) {
-    if (!preds[i].col || (preds[i].width != 4 && preds[i].width != 8))
+    if ((n_cap > 0 && !preds[i].col) || (preds[i].width != 4 && preds[i].width != 8))
       return set_error(DDQ_EINVAL, "select: predicate column must be non-null int32/int64");
     if (preds[i].kind != DDQ_PRED_RANGE && preds[i].kind != DDQ_PRED_IN)
       return set_error(DDQ_EINVAL, "select: bad predicate kind");
@@ -88,7 +88,7 @@ ddq_status ddq_op_hash_probe(const uint64_t* table, uint32_t capacity, const int
                              int32_t* const* carry_out, int32_t n_carry, int32_t* out_tids, int32_t* out_payload,
                              uint32_t* d_out_count, void* scratch, size_t scratch_bytes, void* stream) {
   if (ddq_status s = check_cap(n_cap)) return s;
-  if (!table || !fk || capacity < 2 || (capacity & (capacity - 1)))
+  if (!table || (n_cap > 0 && !fk) || capacity < 2 || (capacity & (capacity - 1)))
     return set_error(DDQ_EINVAL, "hash_probe: bad table / fk");
   if (n_carry < 0 || n_carry > DDQ_MAX_CARRY) return set_error(DDQ_EINVAL, "hash_probe: bad carry count");
   if (!out_tids || !d_out_count || !scratch) return set_error(DDQ_EINVAL, "hash_probe: null output");
@@ -112,10 +112,61 @@ ddq_status ddq_op_hash_probe(const uint64_t* table, uint32_t capacity, const int
   return cuda_status(launch_filter(a, (cudaStream_t)stream), "ddq_op_hash_probe");
 }
 
+size_t ddq_op_join_index_bytes(uint32_t range) { return join_index_bytes(range); }
+
+ddq_status ddq_op_join_index_init(void* index, uint32_t range, void* stream) {
+  if (!index || range == 0) return set_error(DDQ_EINVAL, "join_index_init: bad arguments");
+  return cuda_status(cudaMemsetAsync(index, 0, ((size_t)range + 31) / 32 * 4, (cudaStream_t)stream),
+                     "ddq_op_join_index_init");
+}
+
+ddq_status ddq_op_join_index_build(const int32_t* keys, const int32_t* payload, const int32_t* in_tids,
+                                   const uint32_t* d_in_count, int64_t n_cap, int32_t key_min, uint32_t range,
+                                   void* index, uint32_t* d_error, void* stream) {
+  if (ddq_status s = check_cap(n_cap)) return s;
+  if ((n_cap > 0 && !keys) || !index || !d_error || range == 0)
+    return set_error(DDQ_EINVAL, "join_index_build: bad arguments");
+  if (in_tids && !d_in_count) return set_error(DDQ_EINVAL, "join_index_build: TID input needs a device count");
+  return cuda_status(launch_join_index_build(keys, payload, in_tids, d_in_count, n_cap, key_min, range, index, d_error,
+                                             (cudaStream_t)stream),
+                     "ddq_op_join_index_build");
+}
+
+ddq_status ddq_op_join_index_probe(const void* index, int32_t key_min, uint32_t range, const int32_t* fk,
+                                   const int32_t* in_tids, const uint32_t* d_in_count, int64_t n_cap,
+                                   const int32_t* const* carry_in, int32_t* const* carry_out, int32_t n_carry,
+                                   int32_t* out_tids, int32_t* out_payload, uint32_t* d_out_count, void* scratch,
+                                   size_t scratch_bytes, void* stream) {
+  if (ddq_status s = check_cap(n_cap)) return s;
+  if (!index || range == 0 || (n_cap > 0 && !fk)) return set_error(DDQ_EINVAL, "join_index_probe: bad index / fk");
+  if (n_carry < 0 || n_carry > DDQ_MAX_CARRY) return set_error(DDQ_EINVAL, "join_index_probe: bad carry count");
+  if (!out_tids || !d_out_count || !scratch) return set_error(DDQ_EINVAL, "join_index_probe: null output");
+  if (scratch_bytes < filter_scratch_bytes(n_cap)) return set_error(DDQ_EINVAL, "join_index_probe: scratch too small");
+  if (in_tids && !d_in_count) return set_error(DDQ_EINVAL, "join_index_probe: TID input needs a device count");
+  FilterArgs a;
+  a.probe = true;
+  a.bitmap = join_index_bitmap(const_cast<void*>(index));
+  a.payarr = join_index_payload(const_cast<void*>(index), range);
+  a.key_min = key_min;
+  a.range = range;
+  a.fk = fk;
+  a.out_payload = out_payload;
+  a.in_tids = in_tids;
+  a.d_in_count = d_in_count;
+  a.n_cap = n_cap;
+  a.carry_in = carry_in;
+  a.carry_out = carry_out;
+  a.n_carry = n_carry;
+  a.out_tids = out_tids;
+  a.d_out_count = d_out_count;
+  a.scratch = scratch;
+  return cuda_status(launch_filter(a, (cudaStream_t)stream), "ddq_op_join_index_probe");
+}
+
 ddq_status ddq_op_gather(const void* col, int32_t width, const int32_t* tids, const uint32_t* d_count,
                          int64_t n_cap, void* out, void* stream) {
   if (ddq_status s = check_cap(n_cap)) return s;
-  if (!col || !tids || !out || (width != 4 && width != 8)) return set_error(DDQ_EINVAL, "gather: bad arguments");
+  if ((n_cap > 0 && (!col || !tids || !out)) || (width != 4 && width != 8)) return set_error(DDQ_EINVAL, "gather: bad arguments");
   return cuda_status(launch_gather(col, width, tids, d_count, n_cap, out, (cudaStream_t)stream), "ddq_op_gather");
 }
 

@@ -13,8 +13,14 @@ struct FilterArgs {
   int n_preds = 0;
   bool probe = false;
   bool no_smem = false;
+  bool stable = false;  // dense inputs: force the single-pass look-back kernel (ascending TIDs)
   const uint64_t* table = nullptr;
   uint32_t capacity = 0;
+  // direct-mapped join index (probe): bitmap + payload array over [key_min, key_min+range)
+  const uint32_t* bitmap = nullptr;
+  const int32_t* payarr = nullptr;
+  int32_t key_min = 0;
+  uint32_t range = 0;
   const int32_t* fk = nullptr;
   int32_t* out_payload = nullptr;
   const int32_t* in_tids = nullptr;
@@ -31,12 +37,22 @@ struct FilterArgs {
 };
 
 size_t filter_scratch_bytes(int64_t n_cap);
+bool scan_supported(const FilterArgs& a);
+cudaError_t launch_scan(const FilterArgs& a, cudaStream_t st);
 cudaError_t launch_filter(const FilterArgs& a, cudaStream_t st);
 
 cudaError_t launch_hash_init(uint64_t* table, uint32_t capacity, cudaStream_t st);
 cudaError_t launch_hash_build(const int32_t* keys, const int32_t* payload, const int32_t* in_tids,
                               const uint32_t* d_in_count, int64_t n_cap, uint64_t* table, uint32_t capacity,
                               uint32_t* d_error, cudaStream_t st);
+size_t join_index_bytes(uint32_t range);
+inline uint32_t* join_index_bitmap(void* idx) { return reinterpret_cast<uint32_t*>(idx); }
+inline int32_t* join_index_payload(void* idx, uint32_t range) {
+  return reinterpret_cast<int32_t*>(reinterpret_cast<char*>(idx) + ((((size_t)range + 31) / 32 * 4 + 15) / 16) * 16);
+}
+cudaError_t launch_join_index_build(const int32_t* keys, const int32_t* payload, const int32_t* in_tids,
+                                    const uint32_t* d_in_count, int64_t n_cap, int32_t key_min, uint32_t range,
+                                    void* index, uint32_t* d_error, cudaStream_t st);
 cudaError_t launch_gather(const void* col, int width, const int32_t* tids, const uint32_t* d_count,
                           int64_t n_cap, void* out, cudaStream_t st);
 

@@ -92,6 +92,32 @@ def hash_probe(table, fk, n: int, in_tids=None, in_count=None, carry=(), emit_pa
     return out, pay, cnt, cout
 
 
+def join_index_build(keys, key_min: int, key_range: int, payload=None, in_tids=None, in_count=None,
+                     n: int | None = None):
+    """Direct-mapped join index over [key_min, key_min + key_range)."""
+    n = keys.numel() if n is None else n
+    idx = torch.empty(lib().ddq_op_join_index_bytes(key_range), dtype=torch.uint8, device="cuda")
+    err = count_cell()
+    check(lib().ddq_op_join_index_init(idx.data_ptr(), key_range, _stream()))
+    check(lib().ddq_op_join_index_build(keys.data_ptr(), _ptr(payload), _ptr(in_tids), _ptr(in_count), n, key_min,
+                                        key_range, idx.data_ptr(), err.data_ptr(), _stream()))
+    return idx, err
+
+
+def join_index_probe(idx, key_min: int, key_range: int, fk, n: int, in_tids=None, in_count=None, carry=(),
+                     emit_payload: bool = False):
+    out = torch.empty(max(n, 1), dtype=torch.int32, device="cuda")
+    pay = torch.empty(max(n, 1), dtype=torch.int32, device="cuda") if emit_payload else None
+    cnt = count_cell()
+    scratch = torch.empty(lib().ddq_op_scratch_bytes(n), dtype=torch.uint8, device="cuda")
+    cout = [torch.empty(max(n, 1), dtype=torch.int32, device="cuda") for _ in carry]
+    check(lib().ddq_op_join_index_probe(idx.data_ptr(), key_min, key_range, fk.data_ptr(), _ptr(in_tids),
+                                        _ptr(in_count), n, _ptr_array(list(carry)), _ptr_array(cout), len(carry),
+                                        out.data_ptr(), _ptr(pay), cnt.data_ptr(), scratch.data_ptr(),
+                                        scratch.numel(), _stream()))
+    return out, pay, cnt, cout
+
+
 def gather(col, tids, count, n: int):
     out = torch.empty(max(n, 1), dtype=col.dtype, device="cuda")
     check(lib().ddq_op_gather(col.data_ptr(), col.element_size(), tids.data_ptr(), _ptr(count), n,

@@ -16,6 +16,23 @@ def _t(a):
     return torch.from_numpy(np.ascontiguousarray(a)).cuda()
 
 
+TILE = 4096
+
+
+def tile_order(tids, *vecs):
+    """Dense scans emit TIDs ascending within each 4096-row tile, tiles in completion
+    order (reading O14').  Check that shape and return everything sorted."""
+    tids = np.asarray(tids)
+    if tids.size:
+        t = tids // TILE
+        starts = np.flatnonzero(np.r_[True, t[1:] != t[:-1]])
+        assert len(set(t[starts].tolist())) == starts.size, "a tile's rows are not contiguous"
+        run = np.repeat(np.arange(starts.size), np.diff(np.r_[starts, tids.size]))
+        assert np.all((np.diff(tids) > 0) | (np.diff(run) != 0)), "rows not ascending within a tile"
+    order = np.argsort(tids, kind="stable")
+    return (tids[order],) + tuple(np.asarray(v)[order] for v in vecs)
+
+
 @pytest.fixture(scope="module")
 def ops():
     from paper_conf_sigmod_bressft16_b200 import ops
@@ -31,7 +48,7 @@ def test_select_dense_int64_range(ops, n):
     want = np.flatnonzero((a >= 4) & (a <= 6) & (b >= 26) & (b <= 35))
     c = int(cnt[0].item())
     assert c == want.size
-    assert np.array_equal(tids[:c].cpu().numpy(), want)
+    assert np.array_equal(tile_order(tids[:c].cpu().numpy())[0], want)
 
 
 @pytest.mark.parametrize("n", [0, 5, 4097, 1_000_001])
@@ -41,7 +58,7 @@ def test_select_int32_in_set_and_all_none(ops, n):
     tids, cnt, _ = ops.select([(_t(a), [3, 17, 249, 0])], n)
     want = np.flatnonzero(np.isin(a, [3, 17, 249, 0]))
     c = int(cnt[0].item())
-    assert np.array_equal(tids[:c].cpu().numpy(), want)
+    assert np.array_equal(tile_order(tids[:c].cpu().numpy())[0], want)
     _, cnt_all, _ = ops.select([(_t(a), -1, 1000)], n)
     _, cnt_none, _ = ops.select([(_t(a), 1000, 2000)], n)
     assert int(cnt_all[0].item()) == n and int(cnt_none[0].item()) == 0
@@ -84,8 +101,52 @@ def test_build_probe_semijoin_payload(ops, ndim, nfact):
     want = np.flatnonzero(np.isin(fk, keys[sel]))
     c = int(cnt[0].item())
     assert c == want.size
-    assert np.array_equal(out[:c].cpu().numpy(), want)
-    assert pay[:c].cpu().numpy().tolist() == [m[int(k)] for k in fk[want]]
+    o, p = tile_order(out[:c].cpu().numpy(), pay[:c].cpu().numpy())
+    assert np.array_equal(o, want)
+    assert p.tolist() == [m[int(k)] for k in fk[want]]
+
+
+@pytest.mark.parametrize("ndim,nfact,smem", [(2557, 4097, True), (40_000, 1_000_003, True),
+                                             (1_000_000, 3_000_000, False), (1, 100, True)])
+def test_join_index_semijoin_payload(ops, ndim, nfact, smem):
+    """Direct-mapped join index: dense probe (bitmap staged in smem when <= 96 KB)
+    and the same probe at a TID list, vs numpy.isin + a dict."""
+    rng = np.random.default_rng(ndim + 1)
+    kmin = 1000
+    keys = (kmin + rng.permutation(ndim)).astype(np.int32)          # unique keys in the range
+    payload = rng.integers(0, 1 << 20, ndim, dtype=np.int32)
+    sel = np.flatnonzero(rng.random(ndim) < 0.2).astype(np.int32)
+    idx, err = ops.join_index_build(_t(keys), kmin, ndim, payload=_t(payload),
+                                    in_tids=_t(sel) if sel.size else None,
+                                    in_count=ops.count_cell(sel.size) if sel.size else None, n=sel.size)
+    assert int(err[0].item()) == 0
+    assert (((ndim + 31) // 32) * 4 <= 96 * 1024) == smem
+    fk = rng.integers(kmin - 50, kmin + ndim + 50, nfact, dtype=np.int32)  # includes out-of-range keys
+    m = dict(zip(keys[sel].tolist(), payload[sel].tolist()))
+    want = np.flatnonzero(np.isin(fk, keys[sel]))
+    out, pay, cnt, _ = ops.join_index_probe(idx, kmin, ndim, _t(fk), nfact, emit_payload=True)
+    c = int(cnt[0].item())
+    o, p = tile_order(out[:c].cpu().numpy(), pay[:c].cpu().numpy())
+    assert np.array_equal(o, want)
+    assert p.tolist() == [m[int(k)] for k in fk[want]]
+    # at TIDs (every other row), carrying a vector
+    tin = np.arange(0, nfact, 2, dtype=np.int32)
+    carry = (tin * 3).astype(np.int32)
+    out2, pay2, cnt2, cv = ops.join_index_probe(idx, kmin, ndim, _t(fk), tin.size, in_tids=_t(tin),
+                                                in_count=ops.count_cell(tin.size), carry=[_t(carry)],
+                                                emit_payload=True)
+    c2 = int(cnt2[0].item())
+    keep = np.isin(fk[tin], keys[sel])
+    assert np.array_equal(out2[:c2].cpu().numpy(), tin[keep])
+    assert np.array_equal(cv[0][:c2].cpu().numpy(), carry[keep])
+    assert pay2[:c2].cpu().numpy().tolist() == [m[int(k)] for k in fk[tin[keep]]]
+
+
+def test_join_index_rejects_duplicates_and_out_of_range(ops):
+    _, err = ops.join_index_build(_t(np.array([5, 9, 5], dtype=np.int32)), 0, 16)
+    assert int(err[0].item()) == 1
+    _, err = ops.join_index_build(_t(np.array([5, 99], dtype=np.int32)), 0, 16)
+    assert int(err[0].item()) == 3
 
 
 def test_build_rejects_duplicate_keys(ops):
@@ -108,8 +169,9 @@ def test_probe_chain_at_tids_carries_payload(ops):
     n2 = int(c2[0].item())
     m = (fk1 <= 500) & np.isin(fk2, np.arange(1, 101, 3))
     want = np.flatnonzero(m)
-    assert np.array_equal(o2[:n2].cpu().numpy(), want)
-    assert np.array_equal(carried[0][:n2].cpu().numpy(), fk1[want] * 7)
+    o, cv = tile_order(o2[:n2].cpu().numpy(), carried[0][:n2].cpu().numpy())
+    assert np.array_equal(o, want)
+    assert np.array_equal(cv, fk1[want] * 7)
 
 
 @pytest.mark.parametrize("dtype", [np.int32, np.int64])

@@ -1,0 +1,55 @@
+"""Per-operator profile of the 13 SSB plans (event-timed replay + byte model).
+
+usage: python tools/opprofile.py [--sf 20] [--queries ssb1.1,ssb3.1] [--launch N]
+  --launch N: only launch each prepared plan N times (for ncu), no table.
+"""
+import argparse
+import os
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--sf", type=float, default=20)
+    ap.add_argument("--queries", default="")
+    ap.add_argument("--launch", type=int, default=0)
+    a = ap.parse_args()
+    import torch
+    import datagen
+    from paper_conf_sigmod_bressft16_b200 import Database
+    from paper_conf_sigmod_bressft16_b200.ssb import SSB_QUERIES, load_ssb, ssb_plan
+    qs = a.queries.split(",") if a.queries else SSB_QUERIES
+    data = datagen.SSB(a.sf)
+    db = Database(cache_bytes=64 << 30, heap_bytes=24 << 30)
+    load_ssb(db, data)
+    preps = {q: db.prepare(ssb_plan(db, q)) for q in qs}
+    torch.cuda.synchronize()
+    if a.launch:
+        for _ in range(a.launch):
+            for p in preps.values():
+                p.launch()
+        torch.cuda.synchronize()
+        return
+    names = {0: "dense", 1: "at-tids", 2: "build", 3: "gather", 4: "agg"}
+    tot = {}
+    for q, p in preps.items():
+        for _ in range(3):
+            p.launch()
+        prof = p.profile()
+        prof = p.profile()
+        ops = p.db  # noqa
+        line = []
+        for i, (ms, by, cl) in enumerate(prof):
+            line.append(f"{names[cl]}:{ms*1e3:.0f}us/{by/1e6:.0f}MB/{by/ms/1e6 if ms else 0:.0f}GB/s")
+            t = tot.setdefault(names[cl], [0.0, 0.0])
+            t[0] += ms
+            t[1] += by
+        print(q, f"total {sum(x[0] for x in prof)*1e3:.0f}us", " | ".join(line))
+    for k, (ms, by) in tot.items():
+        print(f"{k:8s} {ms*1e3:9.0f} us {by/1e9:8.3f} GB {by/ms/1e6:8.0f} GB/s")
+
+
+if __name__ == "__main__":
+    main()
