@@ -579,7 +579,7 @@ ddq_status cache_column_locked(ddq_db* db, int c, bool on_demand) {
     return set_error(DDQ_ENOMEM_DEVICE, "cache budget exceeded for " + col.name);
   cudaSetDevice(db->device);
   void* p = nullptr;
-  cudaError_t e = cudaMalloc(&p, bytes);
+  cudaError_t e = cudaMalloc(&p, (bytes + 255) / 256 * 256);  // padded: TMA reads whole 16-byte chunks
   if (e != cudaSuccess) return cuda_status(e, "cache cudaMalloc");
   uint64_t t0 = now_ns();
   e = cudaMemcpyAsync(p, col.host, (size_t)col.n * col.width, cudaMemcpyHostToDevice, db->copy_stream);

@@ -70,42 +70,45 @@ struct ScanParams {
   uint32_t* d_overflow;
 };
 
-__device__ __forceinline__ void cp_async16(void* smem, const void* gmem, int src_bytes) {
-  const uint32_t s = (uint32_t)__cvta_generic_to_shared(smem);
-  asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(s), "l"(gmem), "r"(src_bytes) : "memory");
+// ---- TMA bulk copies (cp.async.bulk) completing on an mbarrier ---------------
+__device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
 }
-__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
-template <int N>
-__device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory"); }
-__device__ __forceinline__ void cp_async_wait_dyn(int n) {
-  switch (n) {
-    case 0: cp_async_wait<0>(); break;
-    case 1: cp_async_wait<1>(); break;
-    case 2: cp_async_wait<2>(); break;
-    case 3: cp_async_wait<3>(); break;
-    case 4: cp_async_wait<4>(); break;
-    case 5: cp_async_wait<5>(); break;
-    default: cp_async_wait<6>(); break;
+__device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t* bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+  uint32_t done = 0;
+  while (!done) {
+    asm volatile(
+        "{\n .reg .pred p;\n mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n selp.u32 %0, 1, 0, p;\n}"
+        : "=r"(done) : "r"(smem_u32(bar)), "r"(parity) : "memory");
   }
 }
+__device__ __forceinline__ void tma_load_1d(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+               ::"r"(smem_u32(dst)), "l"(src), "r"(bytes), "r"(smem_u32(bar)) : "memory");
+}
+__device__ __forceinline__ void fence_proxy_async() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
+__device__ __forceinline__ void fence_mbar_init() { asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory"); }
 
-// Issue the copies of tile `tile` into stage buffer `buf` (all threads).
-__device__ __forceinline__ void issue_tile(const ScanParams& P, uint8_t* buf, uint32_t tile) {
+// Thread 0: one bulk copy per column of tile `tile` into stage buffer `buf`.
+// Columns are readable up to the next 16-byte boundary (library allocations are
+// padded; torch allocations are 512-byte granular), so the tail tile is copied
+// rounded up to 16 bytes and its invalid rows are masked by the row bound.
+__device__ __forceinline__ void issue_tile(const ScanParams& P, uint8_t* buf, uint64_t* bar, uint32_t tile) {
   const uint64_t row0 = (uint64_t)tile * SC_TILE;
+  const uint64_t rows = (uint64_t)P.n - row0 < (uint64_t)SC_TILE ? (uint64_t)P.n - row0 : (uint64_t)SC_TILE;
+  uint32_t total = 0;
+  uint32_t bytes[SC_MAXCOLS];
   for (int c = 0; c < P.n_cols; c++) {
-    const int w = P.width[c];
-    const uint64_t base_b = row0 * w;
-    const uint64_t end_b = (uint64_t)P.n * w;
-    const int chunks = SC_TILE * w / 16;
-    const uint8_t* src = reinterpret_cast<const uint8_t*>(P.cols[c]);
-    uint8_t* dst = buf + P.col_off[c];
-    for (int j = threadIdx.x; j < chunks; j += SC_THREADS) {
-      const uint64_t off = base_b + (uint64_t)j * 16;
-      if (off >= end_b) break;
-      const uint64_t rem = end_b - off;
-      cp_async16(dst + j * 16, src + off, rem >= 16 ? 16 : (int)rem);
-    }
+    bytes[c] = (uint32_t)((rows * P.width[c] + 15) / 16 * 16);
+    total += bytes[c];
   }
+  mbar_arrive_expect_tx(bar, total);
+  for (int c = 0; c < P.n_cols; c++)
+    tma_load_1d(buf + P.col_off[c], reinterpret_cast<const uint8_t*>(P.cols[c]) + row0 * P.width[c], bytes[c], bar);
 }
 
 __device__ __forceinline__ bool scan_pred(const ScanPred& p, int64_t v) {
@@ -117,20 +120,24 @@ __device__ __forceinline__ bool scan_pred(const ScanPred& p, int64_t v) {
 }
 
 __global__ void __launch_bounds__(SC_THREADS, 2) scan_kernel(const __grid_constant__ ScanParams P) {
-  extern __shared__ __align__(16) uint8_t smem[];
+  extern __shared__ __align__(128) uint8_t smem[];
   __shared__ uint32_t s_warp_tot[SC_WARPS];
-  __shared__ uint32_t s_base;
+  __shared__ uint32_t s_base, s_tot;
+  __shared__ __align__(8) uint64_t s_full[8];  // one mbarrier per stage
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const uint32_t ntiles = (P.n + SC_TILE - 1) / SC_TILE;
   const int S = P.stages;
   uint8_t* ring = smem;
   uint64_t* s_table = reinterpret_cast<uint64_t*>(smem + (size_t)S * P.stage_bytes);
 
-  // prologue: put S-1 tiles in flight, then stage the hash table (overlaps them)
-  for (int k = 0; k < S - 1; k++) {
-    const uint32_t t = blockIdx.x + (uint32_t)k * gridDim.x;
-    if (t < ntiles) issue_tile(P, ring + (size_t)k * P.stage_bytes, t);
-    cp_async_commit();
+  // prologue: thread 0 puts S-1 tiles in flight; all threads stage the table meanwhile
+  if (threadIdx.x == 0) {
+    for (int k = 0; k < S; k++) mbar_init(&s_full[k], 1);
+    fence_mbar_init();
+    for (int k = 0; k < S - 1; k++) {
+      const uint32_t t = blockIdx.x + (uint32_t)k * gridDim.x;
+      if (t < ntiles) issue_tile(P, ring + (size_t)k * P.stage_bytes, &s_full[k], t);
+    }
   }
   if (P.probe && P.table_in_smem) {
     for (uint32_t i = threadIdx.x; i <= P.cap_mask; i += SC_THREADS) s_table[i] = P.table[i];
@@ -141,27 +148,33 @@ __global__ void __launch_bounds__(SC_THREADS, 2) scan_kernel(const __grid_consta
     for (uint32_t i = threadIdx.x; i < P.bitmap_words; i += SC_THREADS) s_bm[i] = P.bitmap[i];
   }
   const uint32_t* bm = (P.probe && P.direct && P.bitmap_in_smem) ? s_bm : P.bitmap;
+  __syncthreads();
 
   for (uint32_t k = 0;; k++) {
     const uint32_t tile = blockIdx.x + k * gridDim.x;
     if (tile >= ntiles) break;
-    {  // keep S-1 tiles in flight
+    if (threadIdx.x == 0) {  // keep S-1 tiles in flight (stage (k-1)%S was released by the last barrier)
       const uint32_t t = tile + (uint32_t)(S - 1) * gridDim.x;
-      if (t < ntiles) issue_tile(P, ring + (size_t)((k + S - 1) % S) * P.stage_bytes, t);
-      cp_async_commit();
+      if (t < ntiles) {
+        fence_proxy_async();
+        const int st = (int)((k + S - 1) % S);
+        issue_tile(P, ring + (size_t)st * P.stage_bytes, &s_full[st], t);
+      }
     }
-    cp_async_wait_dyn(S - 1);
-    __syncthreads();
+    mbar_wait(&s_full[k % S], (k / S) & 1u);
     const uint8_t* buf = ring + (size_t)(k % S) * P.stage_bytes;
     const uint32_t row0 = tile * SC_TILE;
     const uint32_t wrow = warp * (32 * SC_ITEMS);  // warp's first row inside the tile
 
-    uint32_t flags = 0;
+    uint32_t flags = 0xFFFFu;
+    if (row0 + SC_TILE > P.n) {  // tail tile only
+      flags = 0;
 #pragma unroll
-    for (int s = 0; s < 4; s++)
+      for (int s = 0; s < 4; s++)
 #pragma unroll
-      for (int v = 0; v < 4; v++)
-        flags |= (row0 + wrow + s * 128 + lane * 4 + v < P.n ? 1u : 0u) << (s * 4 + v);
+        for (int v = 0; v < 4; v++)
+          flags |= (row0 + wrow + s * 128 + lane * 4 + v < P.n ? 1u : 0u) << (s * 4 + v);
+    }
 
     int32_t payload[SC_ITEMS];
     if (!P.probe) {
@@ -180,9 +193,10 @@ __global__ void __launch_bounds__(SC_THREADS, 2) scan_kernel(const __grid_consta
             const int4 a = *reinterpret_cast<const int4*>(cb + (size_t)it * 4);
             v4[0] = a.x; v4[1] = a.y; v4[2] = a.z; v4[3] = a.w;
           }
+          uint32_t m = 0;
 #pragma unroll
-          for (int v = 0; v < 4; v++)
-            if (!scan_pred(pr, v4[v])) flags &= ~(1u << (s * 4 + v));
+          for (int v = 0; v < 4; v++) m |= (scan_pred(pr, v4[v]) ? 1u : 0u) << v;
+          flags &= ~((~m & 0xFu) << (s * 4));
         }
       }
     } else if (P.direct) {
@@ -194,11 +208,14 @@ __global__ void __launch_bounds__(SC_THREADS, 2) scan_kernel(const __grid_consta
         o[s * 4 + 0] = (uint32_t)(a.x - P.key_min); o[s * 4 + 1] = (uint32_t)(a.y - P.key_min);
         o[s * 4 + 2] = (uint32_t)(a.z - P.key_min); o[s * 4 + 3] = (uint32_t)(a.w - P.key_min);
       }
+      uint32_t m = 0;
 #pragma unroll
       for (int k2 = 0; k2 < SC_ITEMS; k2++) {
-        const bool in = o[k2] < P.range && ((bm[o[k2] >> 5] >> (o[k2] & 31)) & 1u);
-        if (!in) flags &= ~(1u << k2);
+        const uint32_t oo = o[k2] < P.range ? o[k2] : 0u;
+        const uint32_t w = bm[oo >> 5];
+        m |= ((o[k2] < P.range ? (w >> (oo & 31)) : 0u) & 1u) << k2;
       }
+      flags &= m;
       if (P.out_payload) {
 #pragma unroll
         for (int k2 = 0; k2 < SC_ITEMS; k2++) payload[k2] = ((flags >> k2) & 1u) ? __ldg(P.payarr + o[k2]) : 0;
@@ -251,34 +268,33 @@ __global__ void __launch_bounds__(SC_THREADS, 2) scan_kernel(const __grid_consta
 #pragma unroll
       for (int w = 0; w < SC_WARPS; w++) tot += s_warp_tot[w];
       s_base = tot ? atomicAdd(P.d_out_count, tot) : 0;
+      s_tot = tot;
     }
     uint32_t warp_off = 0;
 #pragma unroll
     for (int w = 0; w < SC_WARPS; w++) warp_off += (w < warp) ? s_warp_tot[w] : 0;
     __syncthreads();
-    const uint32_t base = s_base + warp_off;
+    const uint32_t tile_base = s_base;
+    const uint32_t base = tile_base + warp_off;
+    const bool fits = tile_base + s_tot <= P.out_cap;
 #pragma unroll
     for (int s = 0; s < 4; s++) {
-      uint32_t pos = base + slot_off[s] + ((excl >> (8 * s)) & 0xFFu);
+      const uint32_t m = (flags >> (4 * s)) & 0xFu;
+      const uint32_t sb = base + slot_off[s] + ((excl >> (8 * s)) & 0xFFu);
 #pragma unroll
       for (int v = 0; v < 4; v++) {
-        const int k2 = s * 4 + v;
-        if ((flags >> k2) & 1u) {
-          if (pos < P.out_cap) {
-            P.out_tids[pos] = (int32_t)(row0 + wrow + s * 128 + lane * 4 + v);
-            if (P.out_payload) P.out_payload[pos] = payload[k2];
-          } else if (P.d_overflow) {
-            atomicMax(P.d_overflow, 4u);
-          }
-          pos++;
+        const uint32_t pos = sb + __popc(m & ((1u << v) - 1u));
+        if (((m >> v) & 1u) && (fits || pos < P.out_cap)) {
+          P.out_tids[pos] = (int32_t)(row0 + wrow + s * 128 + lane * 4 + v);
+          if (P.out_payload) P.out_payload[pos] = payload[s * 4 + v];
         }
       }
     }
+    if (!fits && threadIdx.x == 0 && P.d_overflow) atomicMax(P.d_overflow, 4u);
+    __syncthreads();  // s_warp_tot / s_base reuse
   }
-  cp_async_wait<0>();
   // the last CTA to finish clamps the count to the output capacity (cell word 1 =
   // CTA completion counter, zeroed with the count before launch)
-  __syncthreads();
   if (threadIdx.x == 0) {
     __threadfence();
     if (atomicAdd(P.d_out_count + 1, 1u) == gridDim.x - 1) {
@@ -293,6 +309,10 @@ static int g_smem_optin = 0;
 bool scan_supported(const FilterArgs& a) {
   if (a.in_tids || a.n_carry) return false;  // dense inputs only
   if (!a.probe && (a.n_preds < 1 || a.n_preds > SC_MAXCOLS)) return false;
+  // TMA bulk copies need 16-byte aligned column bases
+  if (a.probe) return ((uintptr_t)a.fk & 15) == 0;
+  for (int i = 0; i < a.n_preds; i++)
+    if ((uintptr_t)a.preds[i].col & 15) return false;
   return true;
 }
 
