@@ -1,20 +1,24 @@
 // scan.cu -- dense scan kernel: selection (S8(a2)) and first hash probe (S8(a4))
 // over ALL rows of a fact column, the dominant kernel of every SSB plan.
 //
-// B200 design, replacing the single-pass look-back kernel
-// for dense inputs after ncu showed it barrier/latency bound at 8% of HBM peak:
-//   * persistent CTAs (SMs x resident), static tile order b, b+G, b+2G, ...;
-//   * input columns streamed through an S-stage shared-memory ring with cp.async
-//     (16-byte LDGSTS, L2-only): S-1 tiles are always in flight per CTA, without
-//     holding registers, so the memory pipe stays busy across the per-tile
-//     compaction and output reservation;
-//   * hash tables that fit are staged once per CTA into shared memory (random
-//     8-byte lookups at smem bandwidth instead of L1/L2 sector rate);
-//   * survivors are compacted per tile (packed warp scan) and their output range is
-//     reserved with ONE atomicAdd per 4096-row tile: no inter-CTA waiting.  Rows
-//     stay ascending within each tile; tiles appear in completion order (reading
-//     O14': the TID list is a multiset -- SQL results are order-free before ORDER BY
-//     and all aggregates are exact integer sums, so results are bit-identical).
+// B200 design; each choice answers an ncu finding:
+//   * one persistent CTA per SM holding G independent 256-thread "groups".  Each
+//     group is a complete pipeline (own TMA ring, mbarriers, named barrier, survivor
+//     lists), so one group's barrier / atomic / TMA wait overlaps the others'
+//     compute, while the dimension table or bitmap is staged ONCE per SM in shared
+//     memory for all groups (random lookups at smem bandwidth, not L1/L2 sectors);
+//   * input columns stream through an S-stage smem ring filled by one thread with
+//     TMA bulk copies (cp.async.bulk + mbarrier complete_tx): no per-thread copy
+//     instructions, S-1 tiles in flight per group;
+//   * full tiles need no row-bound checks; survivors are compacted with a packed
+//     warp scan, staged in smem and copied out coalesced, survivors only;
+//   * the output range of a 4096-row tile is reserved with ONE atomicAdd whose
+//     latency is hidden: tile k is copied out in iteration k+1 (double-buffered
+//     lists).  Rows stay ascending within a tile; tiles appear in reservation order
+//     (reading O14': a TID list is a multiset; aggregates are exact integer sums,
+//     so query results are bit-identical whatever the order).
+//   * compact-range dimension keys use a direct-mapped join index (membership
+//     bitmap + payload array): one lookup per row, no collision chains.
 #include <cstdint>
 #include <cuda_runtime.h>
 
@@ -23,11 +27,14 @@
 
 namespace ddq {
 
-constexpr int SC_THREADS = 256;
-constexpr int SC_WARPS = SC_THREADS / 32;
-constexpr int SC_TILE = 4096;        // rows per tile
-constexpr int SC_ITEMS = SC_TILE / SC_THREADS;  // 16
+constexpr int SC_GT = 256;                 // threads per group
+constexpr int SC_GW = SC_GT / 32;          // warps per group
+constexpr int SC_TILE = 4096;              // rows per tile
+constexpr int SC_ITEMS = SC_TILE / SC_GT;  // 16 rows per thread
+constexpr int SC_SLOTS = SC_ITEMS / 4;     // 4 x (one 16-byte vector of int32)
 constexpr int SC_MAXCOLS = 4;
+constexpr int SC_MAXG = 4;
+constexpr int SC_MAXS = 4;
 
 struct ScanPred {
   const void* col;
@@ -45,6 +52,9 @@ struct ScanParams {
   int32_t col_off[SC_MAXCOLS];  // byte offset of the column's chunk inside a stage
   int32_t stage_bytes;
   int32_t stages;
+  int32_t group_bytes;  // ring + lists of one group
+  int32_t list_off;     // offset of the lists inside a group's area
+  int32_t shared_off;   // offset of the shared table / bitmap
   // select
   int32_t n_preds;
   ScanPred preds[SC_MAXCOLS];
@@ -54,8 +64,7 @@ struct ScanParams {
   uint32_t cap_mask;
   int32_t shift;
   int32_t table_in_smem;
-  // direct-mapped join index instead of a hash table
-  int32_t direct;
+  int32_t direct;  // direct-mapped join index instead of a hash table
   const uint32_t* bitmap;
   const int32_t* payarr;
   int32_t key_min;
@@ -65,7 +74,7 @@ struct ScanParams {
   int32_t* out_payload;
   // outputs
   int32_t* out_tids;
-  uint32_t* d_out_count;  // zeroed before launch; final = survivors
+  uint32_t* d_out_count;  // [0] survivors, [1] CTA completion counter; zeroed before launch
   uint32_t out_cap;
   uint32_t* d_overflow;
 };
@@ -92,8 +101,11 @@ __device__ __forceinline__ void tma_load_1d(void* dst, const void* src, uint32_t
 }
 __device__ __forceinline__ void fence_proxy_async() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
 __device__ __forceinline__ void fence_mbar_init() { asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory"); }
+__device__ __forceinline__ void group_sync(int g) {
+  asm volatile("bar.sync %0, %1;" ::"r"(g + 1), "r"(SC_GT) : "memory");
+}
 
-// Thread 0: one bulk copy per column of tile `tile` into stage buffer `buf`.
+// Group leader: one bulk copy per column of tile `tile` into stage buffer `buf`.
 // Columns are readable up to the next 16-byte boundary (library allocations are
 // padded; torch allocations are 512-byte granular), so the tail tile is copied
 // rounded up to 16 bytes and its invalid rows are masked by the row bound.
@@ -119,182 +131,214 @@ __device__ __forceinline__ bool scan_pred(const ScanPred& p, int64_t v) {
   return m;
 }
 
-__global__ void __launch_bounds__(SC_THREADS, 2) scan_kernel(const __grid_constant__ ScanParams P) {
+template <int G>
+__global__ void __launch_bounds__(SC_GT* G, 1) scan_kernel(const __grid_constant__ ScanParams P) {
   extern __shared__ __align__(128) uint8_t smem[];
-  __shared__ uint32_t s_warp_tot[SC_WARPS];
-  __shared__ uint32_t s_base, s_tot;
-  __shared__ __align__(8) uint64_t s_full[8];  // one mbarrier per stage
-  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  __shared__ uint32_t s_warp_tot[SC_MAXG][SC_GW];
+  __shared__ uint32_t s_base[SC_MAXG];
+  __shared__ __align__(8) uint64_t s_full[SC_MAXG][SC_MAXS];
+  const int g = threadIdx.x / SC_GT;     // group
+  const int t = threadIdx.x % SC_GT;     // thread within the group
+  const int lane = t & 31, warp = t >> 5;
   const uint32_t ntiles = (P.n + SC_TILE - 1) / SC_TILE;
   const int S = P.stages;
-  uint8_t* ring = smem;
-  uint64_t* s_table = reinterpret_cast<uint64_t*>(smem + (size_t)S * P.stage_bytes);
+  const uint32_t vb = blockIdx.x * G + g, vgrid = gridDim.x * G;  // virtual CTA id / count
+  uint8_t* ring = smem + (size_t)g * P.group_bytes;
+  uint16_t* s_list = reinterpret_cast<uint16_t*>(ring + P.list_off);              // 2 x TILE
+  int32_t* s_pay = reinterpret_cast<int32_t*>(ring + P.list_off + SC_TILE * 4);   // 2 x TILE
+  uint64_t* s_table = reinterpret_cast<uint64_t*>(smem + P.shared_off);
 
-  // prologue: thread 0 puts S-1 tiles in flight; all threads stage the table meanwhile
-  if (threadIdx.x == 0) {
-    for (int k = 0; k < S; k++) mbar_init(&s_full[k], 1);
+  if (t == 0) {  // group leader: barriers, then S-1 tiles in flight
+    for (int k = 0; k < S; k++) mbar_init(&s_full[g][k], 1);
     fence_mbar_init();
     for (int k = 0; k < S - 1; k++) {
-      const uint32_t t = blockIdx.x + (uint32_t)k * gridDim.x;
-      if (t < ntiles) issue_tile(P, ring + (size_t)k * P.stage_bytes, &s_full[k], t);
+      const uint32_t tl = vb + (uint32_t)k * vgrid;
+      if (tl < ntiles) issue_tile(P, ring + (size_t)k * P.stage_bytes, &s_full[g][k], tl);
     }
   }
-  if (P.probe && P.table_in_smem) {
-    for (uint32_t i = threadIdx.x; i <= P.cap_mask; i += SC_THREADS) s_table[i] = P.table[i];
-  }
-  const uint64_t* table = (P.probe && P.table_in_smem) ? s_table : P.table;
+  // all groups stage the shared table / bitmap once per SM (overlaps the first loads)
+  if (P.probe && P.table_in_smem)
+    for (uint32_t i = threadIdx.x; i <= P.cap_mask; i += SC_GT * G) s_table[i] = P.table[i];
   uint32_t* s_bm = reinterpret_cast<uint32_t*>(s_table);
-  if (P.probe && P.direct && P.bitmap_in_smem) {
-    for (uint32_t i = threadIdx.x; i < P.bitmap_words; i += SC_THREADS) s_bm[i] = P.bitmap[i];
-  }
+  if (P.probe && P.direct && P.bitmap_in_smem)
+    for (uint32_t i = threadIdx.x; i < P.bitmap_words; i += SC_GT * G) s_bm[i] = P.bitmap[i];
+  const uint64_t* table = (P.probe && P.table_in_smem) ? s_table : P.table;
   const uint32_t* bm = (P.probe && P.direct && P.bitmap_in_smem) ? s_bm : P.bitmap;
+  const bool want_pay = P.probe && P.out_payload != nullptr;
+  const bool hash_pay = want_pay && !P.direct;  // hash probes stage payloads in smem
   __syncthreads();
 
+  // Software pipeline over the group's tiles: iteration k evaluates tile k and
+  // stages its survivors in list[k&1] while its output reservation (one atomic) is
+  // in flight; it copies out tile k-1, whose range was reserved last iteration.
+  uint32_t prev_tot = 0, prev_base = 0;
+  const uint32_t wrow = warp * (32 * SC_ITEMS);  // warp's first row inside a tile
   for (uint32_t k = 0;; k++) {
-    const uint32_t tile = blockIdx.x + k * gridDim.x;
-    if (tile >= ntiles) break;
-    if (threadIdx.x == 0) {  // keep S-1 tiles in flight (stage (k-1)%S was released by the last barrier)
-      const uint32_t t = tile + (uint32_t)(S - 1) * gridDim.x;
-      if (t < ntiles) {
-        fence_proxy_async();
-        const int st = (int)((k + S - 1) % S);
-        issue_tile(P, ring + (size_t)st * P.stage_bytes, &s_full[st], t);
-      }
-    }
-    mbar_wait(&s_full[k % S], (k / S) & 1u);
-    const uint8_t* buf = ring + (size_t)(k % S) * P.stage_bytes;
+    const uint32_t tile = vb + k * vgrid;
+    const bool have = tile < ntiles;
     const uint32_t row0 = tile * SC_TILE;
-    const uint32_t wrow = warp * (32 * SC_ITEMS);  // warp's first row inside the tile
-
-    uint32_t flags = 0xFFFFu;
-    if (row0 + SC_TILE > P.n) {  // tail tile only
-      flags = 0;
-#pragma unroll
-      for (int s = 0; s < 4; s++)
-#pragma unroll
-        for (int v = 0; v < 4; v++)
-          flags |= (row0 + wrow + s * 128 + lane * 4 + v < P.n ? 1u : 0u) << (s * 4 + v);
-    }
-
+    uint32_t flags = 0;
     int32_t payload[SC_ITEMS];
-    if (!P.probe) {
-      for (int p = 0; p < P.n_preds; p++) {
-        const ScanPred& pr = P.preds[p];
-        const uint8_t* cb = buf + P.col_off[p];
+    if (have) {
+      mbar_wait(&s_full[g][k % S], (k / S) & 1u);
+      const uint8_t* buf = ring + (size_t)(k % S) * P.stage_bytes;
+      flags = 0xFFFFu;
+      if (row0 + SC_TILE > P.n) {  // tail tile only
+        flags = 0;
 #pragma unroll
-        for (int s = 0; s < 4; s++) {
-          const int it = wrow + s * 128 + lane * 4;
-          int64_t v4[4];
-          if (pr.width == 8) {
-            const longlong2 a = *reinterpret_cast<const longlong2*>(cb + (size_t)it * 8);
-            const longlong2 b = *reinterpret_cast<const longlong2*>(cb + (size_t)it * 8 + 16);
-            v4[0] = a.x; v4[1] = a.y; v4[2] = b.x; v4[3] = b.y;
-          } else {
-            const int4 a = *reinterpret_cast<const int4*>(cb + (size_t)it * 4);
-            v4[0] = a.x; v4[1] = a.y; v4[2] = a.z; v4[3] = a.w;
+        for (int s = 0; s < SC_SLOTS; s++)
+#pragma unroll
+          for (int v = 0; v < 4; v++)
+            flags |= (row0 + wrow + s * 128 + lane * 4 + v < P.n ? 1u : 0u) << (s * 4 + v);
+      }
+      if (!P.probe) {
+        for (int p = 0; p < P.n_preds; p++) {
+          const ScanPred& pr = P.preds[p];
+          const uint8_t* cb = buf + P.col_off[p];
+#pragma unroll
+          for (int s = 0; s < SC_SLOTS; s++) {
+            const int it = wrow + s * 128 + lane * 4;
+            int64_t v4[4];
+            if (pr.width == 8) {
+              const longlong2 a = *reinterpret_cast<const longlong2*>(cb + (size_t)it * 8);
+              const longlong2 b = *reinterpret_cast<const longlong2*>(cb + (size_t)it * 8 + 16);
+              v4[0] = a.x; v4[1] = a.y; v4[2] = b.x; v4[3] = b.y;
+            } else {
+              const int4 a = *reinterpret_cast<const int4*>(cb + (size_t)it * 4);
+              v4[0] = a.x; v4[1] = a.y; v4[2] = a.z; v4[3] = a.w;
+            }
+            uint32_t m = 0;
+#pragma unroll
+            for (int v = 0; v < 4; v++) m |= (scan_pred(pr, v4[v]) ? 1u : 0u) << v;
+            flags &= ~((~m & 0xFu) << (s * 4));
           }
-          uint32_t m = 0;
-#pragma unroll
-          for (int v = 0; v < 4; v++) m |= (scan_pred(pr, v4[v]) ? 1u : 0u) << v;
-          flags &= ~((~m & 0xFu) << (s * 4));
         }
-      }
-    } else if (P.direct) {
-      // direct-mapped join index: one bitmap probe per row, payload for survivors only
-      uint32_t o[SC_ITEMS];
+      } else if (P.direct) {
+        // one bitmap probe per row; survivors' payload loads are issued now and
+        // consumed after the group scan, so their latency is hidden
+        uint32_t o[SC_ITEMS];
 #pragma unroll
-      for (int s = 0; s < 4; s++) {
-        const int4 a = *reinterpret_cast<const int4*>(buf + (size_t)(wrow + s * 128 + lane * 4) * 4);
-        o[s * 4 + 0] = (uint32_t)(a.x - P.key_min); o[s * 4 + 1] = (uint32_t)(a.y - P.key_min);
-        o[s * 4 + 2] = (uint32_t)(a.z - P.key_min); o[s * 4 + 3] = (uint32_t)(a.w - P.key_min);
-      }
-      uint32_t m = 0;
-#pragma unroll
-      for (int k2 = 0; k2 < SC_ITEMS; k2++) {
-        const uint32_t oo = o[k2] < P.range ? o[k2] : 0u;
-        const uint32_t w = bm[oo >> 5];
-        m |= ((o[k2] < P.range ? (w >> (oo & 31)) : 0u) & 1u) << k2;
-      }
-      flags &= m;
-      if (P.out_payload) {
-#pragma unroll
-        for (int k2 = 0; k2 < SC_ITEMS; k2++) payload[k2] = ((flags >> k2) & 1u) ? __ldg(P.payarr + o[k2]) : 0;
-      }
-    } else {
-      int32_t key[SC_ITEMS];
-      uint32_t h[SC_ITEMS];
-      uint64_t sl[SC_ITEMS];
-#pragma unroll
-      for (int s = 0; s < 4; s++) {
-        const int4 a = *reinterpret_cast<const int4*>(buf + (size_t)(wrow + s * 128 + lane * 4) * 4);
-        key[s * 4 + 0] = a.x; key[s * 4 + 1] = a.y; key[s * 4 + 2] = a.z; key[s * 4 + 3] = a.w;
-      }
-#pragma unroll
-      for (int k2 = 0; k2 < SC_ITEMS; k2++) {
-        h[k2] = ht_hash(key[k2], P.shift);
-        sl[k2] = ((flags >> k2) & 1u) ? table[h[k2]] : HT_EMPTY;
-      }
-#pragma unroll
-      for (int k2 = 0; k2 < SC_ITEMS; k2++) {
-        uint64_t s = sl[k2];
-        uint32_t hh = h[k2];
-        while (s != HT_EMPTY && ht_key(s) != key[k2]) {
-          hh = (hh + 1) & P.cap_mask;
-          s = table[hh];
+        for (int s = 0; s < SC_SLOTS; s++) {
+          const int4 a = *reinterpret_cast<const int4*>(buf + (size_t)(wrow + s * 128 + lane * 4) * 4);
+          o[s * 4 + 0] = (uint32_t)(a.x - P.key_min); o[s * 4 + 1] = (uint32_t)(a.y - P.key_min);
+          o[s * 4 + 2] = (uint32_t)(a.z - P.key_min); o[s * 4 + 3] = (uint32_t)(a.w - P.key_min);
         }
-        if (s == HT_EMPTY) flags &= ~(1u << k2);
-        payload[k2] = ht_val(s);
+        uint32_t m = 0;
+#pragma unroll
+        for (int k2 = 0; k2 < SC_ITEMS; k2++) {
+          const uint32_t oo = o[k2] < P.range ? o[k2] : 0u;
+          const uint32_t w = bm[oo >> 5];
+          m |= ((o[k2] < P.range ? (w >> (oo & 31)) : 0u) & 1u) << k2;
+        }
+        flags &= m;  // payloads: fetched for survivors only, at copy-out
+      } else {
+        int32_t key[SC_ITEMS];
+        uint32_t h[SC_ITEMS];
+        uint64_t sl[SC_ITEMS];
+#pragma unroll
+        for (int s = 0; s < SC_SLOTS; s++) {
+          const int4 a = *reinterpret_cast<const int4*>(buf + (size_t)(wrow + s * 128 + lane * 4) * 4);
+          key[s * 4 + 0] = a.x; key[s * 4 + 1] = a.y; key[s * 4 + 2] = a.z; key[s * 4 + 3] = a.w;
+        }
+#pragma unroll
+        for (int k2 = 0; k2 < SC_ITEMS; k2++) {
+          h[k2] = ht_hash(key[k2], P.shift);
+          sl[k2] = ((flags >> k2) & 1u) ? table[h[k2]] : HT_EMPTY;
+        }
+#pragma unroll
+        for (int k2 = 0; k2 < SC_ITEMS; k2++) {
+          uint64_t s = sl[k2];
+          uint32_t hh = h[k2];
+          while (s != HT_EMPTY && ht_key(s) != key[k2]) {
+            hh = (hh + 1) & P.cap_mask;
+            s = table[hh];
+          }
+          if (s == HT_EMPTY) flags &= ~(1u << k2);
+          payload[k2] = ht_val(s);
+        }
       }
     }
-
-    // compaction within the tile
+    // group scan of the per-slot survivor counts
     uint32_t packed = 0;
 #pragma unroll
-    for (int s = 0; s < 4; s++) packed |= (uint32_t)__popc((flags >> (4 * s)) & 0xFu) << (8 * s);
+    for (int s = 0; s < SC_SLOTS; s++) packed |= (uint32_t)__popc((flags >> (4 * s)) & 0xFu) << (8 * s);
     const uint32_t incl = warp_incl_scan(packed, lane);
     const uint32_t excl = incl - packed;
     const uint32_t wtot = __shfl_sync(FULL, incl, 31);
-    uint32_t slot_off[4];
+    uint32_t slot_off[SC_SLOTS];
     uint32_t acc = 0;
 #pragma unroll
-    for (int s = 0; s < 4; s++) {
+    for (int s = 0; s < SC_SLOTS; s++) {
       slot_off[s] = acc;
       acc += (wtot >> (8 * s)) & 0xFFu;
     }
-    if (lane == 0) s_warp_tot[warp] = acc;
-    __syncthreads();  // also: every thread is done reading stage k%S
-    if (threadIdx.x == 0) {
-      uint32_t tot = 0;
+    if (lane == 0) s_warp_tot[g][warp] = acc;
+    group_sync(g);  // (A) warp totals visible; the group is done with tile k-1
+    uint32_t tot = 0, warp_off = 0;
 #pragma unroll
-      for (int w = 0; w < SC_WARPS; w++) tot += s_warp_tot[w];
-      s_base = tot ? atomicAdd(P.d_out_count, tot) : 0;
-      s_tot = tot;
+    for (int w = 0; w < SC_GW; w++) {
+      const uint32_t x = s_warp_tot[g][w];
+      warp_off += (w < warp) ? x : 0;
+      tot += x;
     }
-    uint32_t warp_off = 0;
+    uint32_t my_base = 0;
+    if (t == 0) {
+      if (have) {  // keep S-1 tiles in flight: refill stage (k-1)%S, released by (A)
+        const uint32_t tl = tile + (uint32_t)(S - 1) * vgrid;
+        if (tl < ntiles) {
+          fence_proxy_async();
+          const int st = (int)((k + S - 1) % S);
+          issue_tile(P, ring + (size_t)st * P.stage_bytes, &s_full[g][st], tl);
+        }
+      }
+      my_base = tot ? atomicAdd(P.d_out_count, tot) : 0;  // consumed only before (B)
+    }
+    // stage tile k's survivors (tile-local row offsets + payloads) in list[k&1]
+    uint16_t* lst = s_list + (k & 1) * SC_TILE;
+    int32_t* pay = s_pay + (k & 1) * SC_TILE;
 #pragma unroll
-    for (int w = 0; w < SC_WARPS; w++) warp_off += (w < warp) ? s_warp_tot[w] : 0;
-    __syncthreads();
-    const uint32_t tile_base = s_base;
-    const uint32_t base = tile_base + warp_off;
-    const bool fits = tile_base + s_tot <= P.out_cap;
-#pragma unroll
-    for (int s = 0; s < 4; s++) {
+    for (int s = 0; s < SC_SLOTS; s++) {
       const uint32_t m = (flags >> (4 * s)) & 0xFu;
-      const uint32_t sb = base + slot_off[s] + ((excl >> (8 * s)) & 0xFFu);
+      const uint32_t sb = warp_off + slot_off[s] + ((excl >> (8 * s)) & 0xFFu);
 #pragma unroll
       for (int v = 0; v < 4; v++) {
-        const uint32_t pos = sb + __popc(m & ((1u << v) - 1u));
-        if (((m >> v) & 1u) && (fits || pos < P.out_cap)) {
-          P.out_tids[pos] = (int32_t)(row0 + wrow + s * 128 + lane * 4 + v);
-          if (P.out_payload) P.out_payload[pos] = payload[s * 4 + v];
+        if ((m >> v) & 1u) {
+          const uint32_t pos = sb + __popc(m & ((1u << v) - 1u));
+          lst[pos] = (uint16_t)(wrow + s * 128 + lane * 4 + v);
+          if (hash_pay) pay[pos] = payload[s * 4 + v];
         }
       }
     }
-    if (!fits && threadIdx.x == 0 && P.d_overflow) atomicMax(P.d_overflow, 4u);
-    __syncthreads();  // s_warp_tot / s_base reuse
+    // copy out tile k-1 (reserved last iteration): coalesced, survivors only
+    if (k > 0) {
+      const uint16_t* pl = s_list + ((k - 1) & 1) * SC_TILE;
+      const int32_t* pp = s_pay + ((k - 1) & 1) * SC_TILE;
+      const uint32_t prow0 = (tile - vgrid) * SC_TILE;
+      const uint32_t lim = prev_base + prev_tot <= P.out_cap ? prev_tot
+                         : (P.out_cap > prev_base ? P.out_cap - prev_base : 0);
+      if (lim < prev_tot && t == 0 && P.d_overflow) atomicMax(P.d_overflow, 4u);
+      if (want_pay && !hash_pay) {  // direct join index: re-read the (L2-hot) key, fetch payload
+        for (uint32_t i = t; i < lim; i += SC_GT) {
+          const uint32_t r = prow0 + pl[i];
+          const int32_t key = __ldg(reinterpret_cast<const int32_t*>(P.cols[0]) + r);
+          P.out_tids[prev_base + i] = (int32_t)r;
+          P.out_payload[prev_base + i] = __ldg(P.payarr + (uint32_t)(key - P.key_min));
+        }
+      } else {
+        for (uint32_t i = t; i < lim; i += SC_GT) {
+          P.out_tids[prev_base + i] = (int32_t)(prow0 + pl[i]);
+          if (hash_pay) P.out_payload[prev_base + i] = pp[i];
+        }
+      }
+    }
+    if (t == 0) s_base[g] = my_base;
+    group_sync(g);  // (B) s_base visible; list[(k-1)&1] free for tile k+1
+    prev_base = s_base[g];
+    prev_tot = tot;
+    if (!have) break;
   }
-  // the last CTA to finish clamps the count to the output capacity (cell word 1 =
-  // CTA completion counter, zeroed with the count before launch)
+  // the last CTA to finish clamps the count to the output capacity
+  __syncthreads();
   if (threadIdx.x == 0) {
     __threadfence();
     if (atomicAdd(P.d_out_count + 1, 1u) == gridDim.x - 1) {
@@ -320,8 +364,13 @@ cudaError_t launch_scan(const FilterArgs& a, cudaStream_t st) {
   if (!g_smem_optin) {
     int dev = 0;
     cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&g_smem_optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
-    cudaFuncSetAttribute(scan_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, g_smem_optin - 1024);
+    int v = 0;
+    cudaDeviceGetAttribute(&v, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
+    cudaFuncSetAttribute(scan_kernel<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, v - 2048);
+    cudaFuncSetAttribute(scan_kernel<2>, cudaFuncAttributeMaxDynamicSharedMemorySize, v - 2048);
+    cudaFuncSetAttribute(scan_kernel<3>, cudaFuncAttributeMaxDynamicSharedMemorySize, v - 2048);
+    cudaFuncSetAttribute(scan_kernel<4>, cudaFuncAttributeMaxDynamicSharedMemorySize, v - 2048);
+    g_smem_optin = v;
   }
   ScanParams p{};
   p.n = (uint32_t)a.n_cap;
@@ -353,13 +402,23 @@ cudaError_t launch_scan(const FilterArgs& a, cudaStream_t st) {
   }
   p.stage_bytes = off;
   const bool direct = a.probe && a.bitmap != nullptr;
-  size_t table_bytes = a.probe ? (direct ? ((size_t)a.range + 31) / 32 * 4 : (size_t)a.capacity * 8) : 0;
-  // shared memory budget per SM (~227 KB usable): table + ring, 2 CTAs per SM when possible
-  const size_t budget = (size_t)g_smem_optin - 1024;
-  const bool in_smem = a.probe && table_bytes <= 96 * 1024;
+  const size_t table_bytes = a.probe ? (direct ? ((size_t)a.range + 31) / 32 * 4 : (size_t)a.capacity * 8) : 0;
+  const size_t budget = (size_t)g_smem_optin - 2048;
+  const bool in_smem = a.probe && table_bytes <= 144 * 1024;
   p.table_in_smem = (in_smem && !direct) ? 1 : 0;
   p.bitmap_in_smem = (in_smem && direct) ? 1 : 0;
-  size_t fixed = in_smem ? (table_bytes + 15) / 16 * 16 : 0;
+  const size_t shared = in_smem ? (table_bytes + 127) / 128 * 128 : 0;
+  const size_t list_bytes = (size_t)SC_TILE * 4 + (a.probe && !direct && a.out_payload ? (size_t)SC_TILE * 8 : 0);
+  // as many groups (up to 4) and stages (up to 4, at least 2) as shared memory allows
+  int G = 4, S = 4;
+  auto need = [&](int gg, int ss) { return shared + (size_t)gg * ((size_t)ss * p.stage_bytes + list_bytes); };
+  while (G > 1 && need(G, 2) > budget) G--;
+  while (S > 2 && need(G, S) > budget) S--;
+  if (need(G, S) > budget) return cudaErrorInvalidConfiguration;
+  p.stages = S;
+  p.list_off = S * p.stage_bytes;
+  p.group_bytes = (int32_t)((p.list_off + list_bytes + 127) / 128 * 128);
+  p.shared_off = G * p.group_bytes;
   if (direct) {
     p.direct = 1;
     p.bitmap = a.bitmap;
@@ -367,15 +426,7 @@ cudaError_t launch_scan(const FilterArgs& a, cudaStream_t st) {
     p.key_min = a.key_min;
     p.range = a.range;
     p.bitmap_words = (a.range + 31) / 32;
-  }
-  int ctas_per_sm = 2;
-  int stages = 4;
-  auto need = [&](int s, int c) { return ((size_t)s * p.stage_bytes + fixed) * c; };
-  while (stages > 2 && need(stages, ctas_per_sm) > budget) stages--;
-  if (need(stages, ctas_per_sm) > budget) ctas_per_sm = 1;
-  while (stages > 2 && need(stages, ctas_per_sm) > budget) stages--;
-  p.stages = stages;
-  if (a.probe && !direct) {
+  } else if (a.probe) {
     p.table = a.table;
     p.cap_mask = a.capacity - 1;
     int lg = 0;
@@ -389,11 +440,17 @@ cudaError_t launch_scan(const FilterArgs& a, cudaStream_t st) {
   p.d_overflow = a.d_overflow;
   cudaError_t e = cudaMemsetAsync(a.d_out_count, 0, 8, st);
   if (e != cudaSuccess) return e;
-  const size_t smem = (size_t)stages * p.stage_bytes + fixed;
+  const size_t smem = (size_t)p.shared_off + shared;
   const int64_t ntiles = (a.n_cap + SC_TILE - 1) / SC_TILE;
-  int64_t grid = (int64_t)num_sms() * ctas_per_sm;
-  if (grid > ntiles) grid = ntiles < 1 ? 1 : ntiles;
-  scan_kernel<<<(int)grid, SC_THREADS, smem, st>>>(p);
+  int64_t grid = num_sms();
+  const int64_t need_ctas = (ntiles + G - 1) / G;
+  if (grid > need_ctas) grid = need_ctas < 1 ? 1 : need_ctas;
+  switch (G) {
+    case 1: scan_kernel<1><<<(int)grid, SC_GT * 1, smem, st>>>(p); break;
+    case 2: scan_kernel<2><<<(int)grid, SC_GT * 2, smem, st>>>(p); break;
+    case 3: scan_kernel<3><<<(int)grid, SC_GT * 3, smem, st>>>(p); break;
+    default: scan_kernel<4><<<(int)grid, SC_GT * 4, smem, st>>>(p); break;
+  }
   return cudaGetLastError();
 }
 
