@@ -230,22 +230,48 @@ def main():
         for p in preps:
             p.launch(sptr)
 
+    # N>1: the 13 compacted partial group tables of a step are packed on the device
+    # ([n, keys[cap], accs[cap*n_aggs*2]] per query) and exchanged with ONE NCCL
+    # all_gather; rank 0 merges them at finalisation (dist.py, S8(e)).
+    from paper_conf_sigmod_bressft16_b200 import dist as D
+
+    class _Dev:  # zero-copy torch view of a library-owned device buffer
+        def __init__(self, ptr, n, typestr):
+            self.__cuda_array_interface__ = {"data": (ptr, False), "shape": (n,), "typestr": typestr,
+                                             "version": 3}
+    views, offs, total = [], [], 0
+    if ws > 1:
+        for p in preps:
+            kp, ap, cp, cap = p.partials_device()
+            na = db._root_aggs[id(p)]
+            views.append((torch.as_tensor(_Dev(cp, 1, "<u4"), device="cuda"),
+                          torch.as_tensor(_Dev(kp, cap, "<i8"), device="cuda"),
+                          torch.as_tensor(_Dev(ap, cap * na * 2, "<i8"), device="cuda"), cap, na))
+            offs.append(total)
+            total += D.packed_words(cap, na)
+    packed = torch.zeros(max(total, 1), dtype=torch.int64, device="cuda")
+    gathered = torch.zeros(max(total, 1) * ws, dtype=torch.int64, device="cuda")
+
     def exchange():
-        """N>1: all_gather of every query's compacted partial group table."""
         if ws == 1:
-            return None
+            return
         import torch.distributed as dist
-        outs = []
         with torch.cuda.stream(stream):
-            for p in preps:
-                keys, accs = p.partials(sptr)  # D2H of <= 800 groups per query
-                t = torch.from_numpy(np.concatenate([[keys.size], keys, accs.reshape(-1)]).astype(np.int64))
-                pad = torch.zeros(1 + 2048 * (1 + 2 * 2), dtype=torch.int64)
-                pad[:t.numel()] = t
-                g = [torch.zeros_like(pad, device="cuda") for _ in range(ws)]
-                dist.all_gather(g, pad.cuda())
-                outs.append(g)
-        return outs
+            for (cnt, keys, accs, cap, na), o in zip(views, offs):
+                packed[o:o + 1].copy_(cnt.to(torch.int64))
+                packed[o + 1:o + 1 + cap].copy_(keys)
+                packed[o + 1 + cap:o + 1 + cap + cap * na * 2].copy_(accs)
+            dist.all_gather_into_tensor(gathered, packed)
+
+    def merged_results():
+        """rank 0: unpack every rank's partials per query and finalise (exact merge)."""
+        g = gathered.view(ws, -1).cpu().numpy()
+        res = {}
+        for q, p, (cnt, keys, accs, cap, na), o in zip(SSB_QUERIES, preps, views, offs):
+            flat = g[:, o:o + D.packed_words(cap, na)].reshape(-1)
+            k, a = D.unpack_gathered(flat, ws, cap, na)
+            res[q] = p.finalize(k, a).rows
+        return res
 
     if args.profile_only:
         for _ in range(2):
@@ -284,7 +310,8 @@ def main():
     value = total_rows * args.steps / (ms / 1e3)
 
     # results of the timed plans (validated against the oracle by tests/, here sanity only)
-    results = {q: p.fetch(sptr).rows for q, p in zip(SSB_QUERIES, preps)} if ws == 1 else {}
+    results = {q: p.fetch(sptr).rows for q, p in zip(SSB_QUERIES, preps)} if ws == 1 else \
+        (merged_results() if rank == 0 else {})
 
     # ---- roofline of the dominant kernel class from an event-timed profiling replay
     prof = [p.profile(sptr) for p in preps]

@@ -143,8 +143,9 @@ ddq_status ddq_op_gather(const void* col, int32_t width, const int32_t* tids,
                          const uint32_t* d_count, int64_t n_cap, void* out, void* stream);
 
 /* Group-by aggregation (S8(a6)).  For each input position i < *d_count with
- * row r = tids[i]: group key = k0 | k1 << 21 | k2 << 42 where kj is either the
- * aligned vector key_vec[j][i] or the column key_col[j][r] (int32, 0 <= kj < 2^21);
+ * row r = tids[i]: group key = k0 | k1 << b0 | k2 << (b0 + b1) (bj = key_bits[j],
+ * key_bits NULL or 0 -> 21) where kj is either the aligned vector key_vec[j][i] or
+ * the column key_col[j][r] (int32, 0 <= kj < 2^bj, sum of bits <= 63);
  * aggregate a adds expr_a(r) to the group's exact int128 accumulator.  The result
  * is an open-addressing table of `capacity` slots (power of two, >= 2x groups):
  *   keys  int64[capacity]           (empty = -1)
@@ -171,7 +172,7 @@ size_t ddq_op_groupby_table_bytes(uint32_t capacity, int32_t n_aggs);
 ddq_status ddq_op_groupby_init(void* table, uint32_t capacity, int32_t n_aggs, void* stream);
 ddq_status ddq_op_groupby(const int32_t* tids, const uint32_t* d_count, int64_t n_cap,
                           const int32_t* const* key_vec, const int32_t* const* key_col, int32_t n_keys,
-                          const ddq_dev_agg* aggs, int32_t n_aggs,
+                          const int32_t* key_bits, const ddq_dev_agg* aggs, int32_t n_aggs,
                           void* table, uint32_t capacity, uint32_t* d_error, void* stream);
 /* Compact the non-empty groups: out_keys int64[capacity], out_accs int64[n_aggs *
  * capacity * 2] (group-major: accs of group g at [(g * n_aggs + a) * 2]),
@@ -252,7 +253,9 @@ enum {
   DDQ_OP_HASH_BUILD = 2, /* hash table over input TIDs of `table` (key_col, payload_col) */
   DDQ_OP_HASH_PROBE = 3, /* semi-join input TIDs of `table` via fk_col against op `build` */
   DDQ_OP_GATHER = 4,     /* append vector col[tid] to the input's aligned vectors */
-  DDQ_OP_AGGREGATE = 5   /* group-by at input TIDs; root; finalised on the host */
+  DDQ_OP_AGGREGATE = 5,  /* group-by at input TIDs; root; finalised on the host */
+  DDQ_OP_FILTER_EQ = 6   /* keep input rows whose two aligned vectors are equal (TPC-H Q5's
+                            c_nationkey = s_nationkey); vectors carried */
 };
 
 typedef struct {
@@ -292,6 +295,13 @@ typedef struct {
   int32_t n_order;
   int32_t order_by[8];
   int64_t limit;           /* <= 0: no limit */
+  /* extensions (zero = default) */
+  int32_t key_bits[DDQ_MAX_KEYS]; /* AGGREGATE: bits of key k in the packed group key
+                                     (0 = 21); keys are packed low to high; sum <= 63 */
+  int32_t fk_vec;          /* HASH_PROBE: 1 + index of an aligned input vector holding the
+                              probe keys (instead of fk_col); 0 = use fk_col */
+  int32_t eq_vec[2];       /* FILTER_EQ: 1 + indexes of the two aligned vectors compared */
+  int32_t _pad2;
 } ddq_op;
 
 #define DDQ_MAX_OPS 32
@@ -347,6 +357,18 @@ int32_t ddq_prepared_kernel_count(ddq_prepared* p);
  * 2 hash build, 3 gather, 4 aggregate.  Returns the number of operators. */
 int32_t ddq_prepared_profile(ddq_prepared* p, void* stream, int32_t max_ops, float* op_ms, double* op_bytes,
                              int32_t* op_class);
+/* Device views of the compacted partial group table of the last launch (for an
+ * NCCL exchange without host copies): keys int64[cap], accs int64[cap*n_aggs*2],
+ * *count = number of valid groups (device uint32).  Library-owned; valid until
+ * ddq_prepared_free. */
+ddq_status ddq_prepared_partials_device(ddq_prepared* p, int64_t** keys, int64_t** accs, uint32_t** count,
+                                        int64_t* cap);
+/* Finalise partial group tables on the host, no GPU needed (S8(a7) + the S8(e)
+ * merge): rows with equal packed keys (e.g. the same group from several shards)
+ * are merged by exact int128 addition, then ORDER BY / LIMIT of `root` apply.
+ * keys: int64[n] packed group keys; accs: int64[n * root->n_aggs * 2]. */
+ddq_status ddq_finalize_partials(const ddq_op* root, int64_t n, const int64_t* keys, const int64_t* accs,
+                                 ddq_result** out);
 /* Finalise externally merged partials (keys/accs as returned above) into a result. */
 ddq_status ddq_prepared_finalize(ddq_prepared* p, int64_t n_groups, const int64_t* h_keys,
                                  const int64_t* h_accs, ddq_result** out);

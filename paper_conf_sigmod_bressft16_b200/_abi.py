@@ -19,7 +19,7 @@ STATUS = {0: "DDQ_OK", -1: "DDQ_EINVAL", -2: "DDQ_ENOTFOUND", -3: "DDQ_ENOMEM_HO
 
 PRED_RANGE, PRED_IN = 1, 2
 MAX_IN, MAX_PREDS, MAX_CARRY, MAX_AGGS, MAX_KEYS, MAX_OPS = 8, 4, 4, 8, 3, 32
-OP_SELECT, OP_HASH_BUILD, OP_HASH_PROBE, OP_GATHER, OP_AGGREGATE = 1, 2, 3, 4, 5
+OP_SELECT, OP_HASH_BUILD, OP_HASH_PROBE, OP_GATHER, OP_AGGREGATE, OP_FILTER_EQ = 1, 2, 3, 4, 5, 6
 AGG_COUNT, AGG_SUM, AGG_SUM_MUL, AGG_SUM_SUB, AGG_SUM_MUL_100M, AGG_SUM_MUL_100M_100P = 1, 2, 3, 4, 5, 6
 I32, I64 = 1, 2
 PLACE_DATA_DRIVEN, PLACE_GPU_ONLY, PLACE_CPU_ONLY = 0, 1, 2
@@ -59,7 +59,9 @@ class Op(ctypes.Structure):
                 ("n_aggs", ctypes.c_int32), ("agg_kind", ctypes.c_int32 * MAX_AGGS),
                 ("agg_col", (ctypes.c_int32 * 3) * MAX_AGGS),
                 ("max_groups", ctypes.c_int64), ("n_order", ctypes.c_int32),
-                ("order_by", ctypes.c_int32 * 8), ("limit", ctypes.c_int64)]
+                ("order_by", ctypes.c_int32 * 8), ("limit", ctypes.c_int64),
+                ("key_bits", ctypes.c_int32 * MAX_KEYS), ("fk_vec", ctypes.c_int32),
+                ("eq_vec", ctypes.c_int32 * 2), ("_pad2", ctypes.c_int32)]
 
 
 class Plan(ctypes.Structure):
@@ -101,7 +103,8 @@ SIGNATURES = {
     "ddq_op_gather": (_i32, [_vp, _i32, _vp, _vp, _i64, _vp, _vp]),
     "ddq_op_groupby_table_bytes": (_sz, [_u32, _i32]),
     "ddq_op_groupby_init": (_i32, [_vp, _u32, _i32, _vp]),
-    "ddq_op_groupby": (_i32, [_vp, _vp, _i64, _pp, _pp, _i32, ctypes.POINTER(DevAgg), _i32, _vp, _u32, _vp, _vp]),
+    "ddq_op_groupby": (_i32, [_vp, _vp, _i64, _pp, _pp, _i32, _vp, ctypes.POINTER(DevAgg), _i32, _vp, _u32, _vp,
+                              _vp]),
     "ddq_op_groupby_compact": (_i32, [_vp, _u32, _i32, _vp, _vp, _vp, _vp]),
     "ddq_config_default": (None, [ctypes.POINTER(Config)]),
     "ddq_open": (_i32, [ctypes.POINTER(Config), ctypes.POINTER(_vp)]),
@@ -128,6 +131,9 @@ SIGNATURES = {
     "ddq_prepared_kernel_count": (_i32, [_vp]),
     "ddq_prepared_profile": (_i32, [_vp, _vp, _i32, ctypes.POINTER(ctypes.c_float), ctypes.POINTER(ctypes.c_double),
                                     ctypes.POINTER(_i32)]),
+    "ddq_prepared_partials_device": (_i32, [_vp, ctypes.POINTER(_vp), ctypes.POINTER(_vp), ctypes.POINTER(_vp),
+                                            ctypes.POINTER(_i64)]),
+    "ddq_finalize_partials": (_i32, [ctypes.POINTER(Op), _i64, _vp, _vp, ctypes.POINTER(ctypes.POINTER(Result))]),
     "ddq_prepared_finalize": (_i32, [_vp, _i64, _vp, _vp, ctypes.POINTER(ctypes.POINTER(Result))]),
     "ddq_prepared_free": (None, [_vp]),
     "ddq_get_stats": (_i32, [_vp, ctypes.POINTER(Stats)]),

@@ -63,7 +63,10 @@ static std::vector<int> op_columns(const ddq_op& op) {
       c.push_back(op.key_col);
       if (op.payload_col >= 0) c.push_back(op.payload_col);
       break;
-    case DDQ_OP_HASH_PROBE: c.push_back(op.fk_col); break;
+    case DDQ_OP_HASH_PROBE:
+      if (op.fk_vec <= 0) c.push_back(op.fk_col);
+      break;
+    case DDQ_OP_FILTER_EQ: break;
     case DDQ_OP_GATHER: c.push_back(op.gather_col); break;
     case DDQ_OP_AGGREGATE:
       for (int k = 0; k < op.n_keys; k++)
@@ -270,14 +273,25 @@ ddq_status run_host_op(ddq_db* db, const ddq_op& op, const std::vector<Inter>& I
   }
   switch (op.kind) {
     case DDQ_OP_SELECT:
+    case DDQ_OP_FILTER_EQ:
     case DDQ_OP_HASH_PROBE: {
       const bool probe = op.kind == DDQ_OP_HASH_PROBE;
       const Inter* build = probe ? &I[(size_t)op.build] : nullptr;
       if (probe && !build->host_table && !build->h_bitmap) return set_error(DDQ_ESTATE, "host probe needs a host table");
       const bool direct = probe && build->h_bitmap != nullptr;
       std::vector<const Column*> pc;
-      for (int i = 0; i < op.n_preds && !probe; i++) pc.push_back(col_of(db, op.preds[i].column));
-      const Column* fk = probe ? col_of(db, op.fk_col) : nullptr;
+      for (int i = 0; i < op.n_preds && op.kind == DDQ_OP_SELECT; i++) pc.push_back(col_of(db, op.preds[i].column));
+      const int32_t* eqa = nullptr;
+      const int32_t* eqb = nullptr;
+      if (op.kind == DDQ_OP_FILTER_EQ) {
+        const int a = op.eq_vec[0] - 1, b = op.eq_vec[1] - 1;
+        if (!in || a < 0 || b < 0 || a >= (int)in->vecs.size() || b >= (int)in->vecs.size())
+          return set_error(DDQ_EINVAL, "filter_eq: bad vector indexes");
+        eqa = (const int32_t*)in->vecs[(size_t)a].ptr;
+        eqb = (const int32_t*)in->vecs[(size_t)b].ptr;
+      }
+      const Column* fk = (probe && op.fk_vec <= 0) ? col_of(db, op.fk_col) : nullptr;
+      const int32_t* fkv = (probe && op.fk_vec > 0) ? (const int32_t*)in->vecs[(size_t)op.fk_vec - 1].ptr : nullptr;
       int lg = 0;
       if (probe && !direct)
         while ((1u << lg) < build->table_cap) lg++;
@@ -292,7 +306,9 @@ ddq_status run_host_op(ddq_db* db, const ddq_op& op, const std::vector<Inter>& I
         for (int64_t i = b; i < e; i++) {
           int32_t r = row_of(i);
           bool ok = true;
-          if (!probe) {
+          if (eqa) {
+            if (eqa[i] == eqb[i]) S.push_back(i);
+          } else if (!probe) {
             for (int p = 0; p < op.n_preds && ok; p++) {
               int64_t v = hcol(pc[(size_t)p], r);
               const ddq_pred& pr = op.preds[p];
@@ -305,7 +321,7 @@ ddq_status run_host_op(ddq_db* db, const ddq_op& op, const std::vector<Inter>& I
             }
             if (ok) S.push_back(i);
           } else {
-            int32_t k = ((const int32_t*)fk->host)[r];
+            int32_t k = fkv ? fkv[i] : ((const int32_t*)fk->host)[r];
             if (direct) {
               const uint32_t o = (uint32_t)(k - build->jmin);
               ok = o < build->jrange && (((*build->h_bitmap)[o >> 5] >> (o & 31)) & 1u);
@@ -399,6 +415,11 @@ ddq_status run_host_op(ddq_db* db, const ddq_op& op, const std::vector<Inter>& I
       std::vector<std::array<const Column*, 3>> ac((size_t)na);
       for (int a = 0; a < na; a++)
         for (int j = 0; j < 3; j++) ac[(size_t)a][(size_t)j] = op.agg_col[a][j] >= 0 ? col_of(db, op.agg_col[a][j]) : nullptr;
+      int kshift[DDQ_MAX_KEYS];
+      for (int k = 0, sh = 0; k < DDQ_MAX_KEYS; k++) {
+        kshift[k] = sh;
+        sh += op.key_bits[k] > 0 ? op.key_bits[k] : 21;
+      }
       std::unordered_map<int64_t, std::vector<__int128>> g;
       for (int64_t i = 0; i < n; i++) {
         int32_t r = in->tids[i];
@@ -406,7 +427,7 @@ ddq_status run_host_op(ddq_db* db, const ddq_op& op, const std::vector<Inter>& I
         for (int k = 0; k < op.n_keys; k++) {
           int32_t c = op.key_src[k] >= 0 ? ((const int32_t*)in->vecs[(size_t)op.key_src[k]].ptr)[i]
                                          : ((const int32_t*)kc[(size_t)k]->host)[r];
-          key |= (int64_t)(uint32_t)c << (21 * k);
+          key |= (int64_t)(uint32_t)c << kshift[k];
         }
         auto& acc = g[key];
         if (acc.empty()) acc.assign((size_t)na, 0);

@@ -169,11 +169,22 @@ ddq_status run_gpu_op(GpuOpCtx& ctx, const ddq_op& op, Inter& out) {
   };
   switch (op.kind) {
     case DDQ_OP_SELECT:
+    case DDQ_OP_FILTER_EQ:
     case DDQ_OP_HASH_PROBE: {
       const bool probe = op.kind == DDQ_OP_HASH_PROBE;
       ddq_dev_pred dp[DDQ_MAX_PREDS];
       std::memset(dp, 0, sizeof(dp));
-      if (!probe) {
+      const int32_t* eq_a = nullptr;
+      const int32_t* eq_b = nullptr;
+      if (op.kind == DDQ_OP_FILTER_EQ) {
+        if (!in) return set_error(DDQ_EINVAL, "filter_eq needs an input with aligned vectors");
+        const int a = op.eq_vec[0] - 1, b = op.eq_vec[1] - 1;
+        if (a < 0 || b < 0 || a >= (int)in->vecs.size() || b >= (int)in->vecs.size() ||
+            in->vecs[(size_t)a].width != 4 || in->vecs[(size_t)b].width != 4)
+          return set_error(DDQ_EINVAL, "filter_eq: bad vector indexes");
+        eq_a = (const int32_t*)in->vecs[(size_t)a].ptr;
+        eq_b = (const int32_t*)in->vecs[(size_t)b].ptr;
+      } else if (!probe) {
         if (op.n_preds < 0 || op.n_preds > DDQ_MAX_PREDS) return set_error(DDQ_EINVAL, "select: bad n_preds");
         for (int i = 0; i < op.n_preds; i++) {
           const ddq_pred& p = op.preds[i];
@@ -196,10 +207,16 @@ ddq_status run_gpu_op(GpuOpCtx& ctx, const ddq_op& op, Inter& out) {
         build = &I[(size_t)op.build];
         if (!build->table_ptr && !build->jidx)
           return set_error(DDQ_ESTATE, "probe: build side is not a device hash table / join index");
-        const Column* c = col_of(db, op.fk_col);
-        if (!c || c->table != op.table || c->width != 4) return set_error(DDQ_EINVAL, "probe: bad fk column");
-        fk = (const int32_t*)need_col(op.fk_col);
-        if (!fk) return set_error(DDQ_ESTATE, "probe: fk column not cached on the GPU");
+        if (op.fk_vec > 0) {  // probe keys from an aligned vector of the input
+          if (!in || op.fk_vec - 1 >= (int)in->vecs.size() || in->vecs[(size_t)op.fk_vec - 1].width != 4)
+            return set_error(DDQ_EINVAL, "probe: bad fk vector");
+          fk = (const int32_t*)in->vecs[(size_t)op.fk_vec - 1].ptr;
+        } else {
+          const Column* c = col_of(db, op.fk_col);
+          if (!c || c->table != op.table || c->width != 4) return set_error(DDQ_EINVAL, "probe: bad fk column");
+          fk = (const int32_t*)need_col(op.fk_col);
+          if (!fk) return set_error(DDQ_ESTATE, "probe: fk column not cached on the GPU");
+        }
       }
       // carried vectors (int32 only; int64 vectors are re-gathered by consumers)
       std::vector<const int32_t*> cin;
@@ -241,8 +258,11 @@ ddq_status run_gpu_op(GpuOpCtx& ctx, const ddq_op& op, Inter& out) {
           fa.range = build->jrange;
         }
         fa.fk = fk;
+        fa.fk_by_pos = op.fk_vec > 0;
         fa.out_payload = payload;
       }
+      fa.eq_a = eq_a;
+      fa.eq_b = eq_b;
       fa.in_tids = in_tids;
       fa.d_in_count = in_cnt;
       fa.n_cap = in_cap;
@@ -372,7 +392,7 @@ ddq_status run_gpu_op(GpuOpCtx& ctx, const ddq_op& op, Inter& out) {
       if (A.failed) return DDQ_ENOMEM_DEVICE;
       cudaError_t e = launch_groupby_init(out.gb_table, out.gb_cap, op.n_aggs, st);
       if (e == cudaSuccess)
-        e = launch_groupby(in->tids, in->d_count, in->cap, kv, kc, op.n_keys, ag, op.n_aggs, out.gb_table,
+        e = launch_groupby(in->tids, in->d_count, in->cap, kv, kc, op.n_keys, op.key_bits, ag, op.n_aggs, out.gb_table,
                            out.gb_cap, out.d_error, st);
       if (e == cudaSuccess)
         e = launch_groupby_compact(out.gb_table, out.gb_cap, op.n_aggs, out.gb_keys, out.gb_accs, out.gb_groups, st);
@@ -391,12 +411,57 @@ static inline __int128 acc128(const int64_t* accs, int64_t g, int n_aggs, int a)
   return (__int128)((unsigned __int128)(hi << 64) | lo);
 }
 
+static ddq_status finalize_unique(const ddq_op& root, int64_t n_groups, const int64_t* keys, const int64_t* accs,
+                                  ddq_result** out);
+
+// Merge equal packed keys (partials of several shards, S8(e)) by exact int128
+// addition, then finalise.
 ddq_status finalize_result(const ddq_op& root, int64_t n_groups, const int64_t* keys, const int64_t* accs,
                            ddq_result** out) {
+  const int na = root.n_aggs;
+  std::vector<int64_t> idx((size_t)n_groups);
+  std::iota(idx.begin(), idx.end(), 0);
+  std::sort(idx.begin(), idx.end(), [&](int64_t a, int64_t b) { return keys[a] < keys[b]; });
+  bool dup = false;
+  for (size_t i = 1; i < idx.size() && !dup; i++) dup = keys[idx[i]] == keys[idx[i - 1]];
+  if (!dup) return finalize_unique(root, n_groups, keys, accs, out);
+  std::vector<int64_t> mk, ma;
+  for (size_t i = 0; i < idx.size(); i++) {
+    const int64_t g = idx[i];
+    if (i == 0 || keys[g] != mk.back()) {
+      mk.push_back(keys[g]);
+      for (int a = 0; a < na; a++) {
+        ma.push_back(accs[(g * na + a) * 2]);
+        ma.push_back(accs[(g * na + a) * 2 + 1]);
+      }
+    } else {
+      const size_t m = mk.size() - 1;
+      for (int a = 0; a < na; a++) {
+        unsigned __int128 x = ((unsigned __int128)(uint64_t)ma[(m * na + a) * 2 + 1] << 64) |
+                              (uint64_t)ma[(m * na + a) * 2];
+        unsigned __int128 y = ((unsigned __int128)(uint64_t)accs[(g * na + a) * 2 + 1] << 64) |
+                              (uint64_t)accs[(g * na + a) * 2];
+        x += y;
+        ma[(m * na + a) * 2] = (int64_t)(uint64_t)x;
+        ma[(m * na + a) * 2 + 1] = (int64_t)(uint64_t)(x >> 64);
+      }
+    }
+  }
+  return finalize_unique(root, (int64_t)mk.size(), mk.data(), ma.data(), out);
+}
+
+static ddq_status finalize_unique(const ddq_op& root, int64_t n_groups, const int64_t* keys, const int64_t* accs,
+                                  ddq_result** out) {
   const int nk = root.n_keys, na = root.n_aggs;
   std::vector<int64_t> idx((size_t)n_groups);
   std::iota(idx.begin(), idx.end(), 0);
-  auto keyk = [&](int64_t g, int k) { return (keys[g] >> (21 * k)) & ((1ll << 21) - 1); };
+  int shift[DDQ_MAX_KEYS], bits[DDQ_MAX_KEYS];
+  for (int k = 0, sh = 0; k < DDQ_MAX_KEYS; k++) {
+    bits[k] = root.key_bits[k] > 0 ? root.key_bits[k] : 21;
+    shift[k] = sh;
+    sh += bits[k];
+  }
+  auto keyk = [&](int64_t g, int k) { return (keys[g] >> shift[k]) & ((1ll << bits[k]) - 1); };
   std::sort(idx.begin(), idx.end(), [&](int64_t a, int64_t b) {
     for (int o = 0; o < root.n_order; o++) {
       int e = root.order_by[o];
@@ -753,7 +818,15 @@ static ddq_status validate_plan(ddq_db* db, const ddq_plan* plan) {
   if (!plan || plan->n_ops < 1 || plan->n_ops > DDQ_MAX_OPS) return set_error(DDQ_EINVAL, "plan: bad op count");
   for (int i = 0; i < plan->n_ops; i++) {
     const ddq_op& op = plan->ops[i];
-    if (op.kind < DDQ_OP_SELECT || op.kind > DDQ_OP_AGGREGATE) return set_error(DDQ_EINVAL, "plan: bad op kind");
+    if (op.kind < DDQ_OP_SELECT || op.kind > DDQ_OP_FILTER_EQ) return set_error(DDQ_EINVAL, "plan: bad op kind");
+    if (op.kind == DDQ_OP_FILTER_EQ && op.input < 0) return set_error(DDQ_EINVAL, "plan: filter_eq needs an input");
+    if (op.kind == DDQ_OP_HASH_PROBE && op.fk_vec > 0 && op.input < 0)
+      return set_error(DDQ_EINVAL, "plan: a vector-keyed probe needs an input");
+    if (op.kind == DDQ_OP_AGGREGATE) {
+      int bits = 0;
+      for (int k = 0; k < op.n_keys && k < DDQ_MAX_KEYS; k++) bits += op.key_bits[k] > 0 ? op.key_bits[k] : 21;
+      if (bits > 63) return set_error(DDQ_EINVAL, "plan: packed group key wider than 63 bits");
+    }
     if (op.input >= i || op.input < -1) return set_error(DDQ_EINVAL, "plan: input must precede the op");
     if (op.kind == DDQ_OP_HASH_PROBE && (op.build < 0 || op.build >= i ||
                                          plan->ops[op.build].kind != DDQ_OP_HASH_BUILD))
@@ -779,6 +852,7 @@ static int kernels_of(const ddq_op& op) {
     case DDQ_OP_HASH_BUILD: return 2;
     case DDQ_OP_GATHER: return 1;
     case DDQ_OP_AGGREGATE: return 3;
+    case DDQ_OP_FILTER_EQ: return 1;
   }
   return 0;
 }
@@ -1008,6 +1082,10 @@ int32_t ddq_prepared_profile(ddq_prepared* p, void* stream, int32_t max_ops, flo
         }
         bytes += out * 4 * (1 + nvec_in + emit);
       } break;
+      case DDQ_OP_FILTER_EQ:
+        cls = 1;
+        bytes = m * 4 + m * 8 + out * 4 * (1 + 2 * nvec_in);
+        break;
       case DDQ_OP_HASH_BUILD:
         cls = 2;
         bytes = m * 4 * (op.payload_col >= 0 ? 2 : 1) + (double)o.table_cap * 8 * 2;
@@ -1087,6 +1165,27 @@ ddq_status ddq_prepared_partials(ddq_prepared* p, void* stream, int64_t* h_n_gro
   p->db->stats.d2h_ns += now_ns() - t0;
   *h_n_groups = g;
   return DDQ_OK;
+}
+
+ddq_status ddq_prepared_partials_device(ddq_prepared* p, int64_t** keys, int64_t** accs, uint32_t** count,
+                                        int64_t* cap) {
+  if (!p || !keys || !accs || !count || !cap) return set_error(DDQ_EINVAL, "prepared_partials_device: null");
+  const Inter& r = p->inters.back();
+  if (!r.gb_table) return set_error(DDQ_ESTATE, "prepared_partials_device: root is not an aggregate");
+  *keys = r.gb_keys;
+  *accs = r.gb_accs;
+  *count = r.gb_groups;
+  *cap = r.gb_cap;
+  return DDQ_OK;
+}
+
+ddq_status ddq_finalize_partials(const ddq_op* root, int64_t n, const int64_t* keys, const int64_t* accs,
+                                 ddq_result** out) {
+  if (!root || !out || n < 0 || (n > 0 && (!keys || !accs))) return set_error(DDQ_EINVAL, "finalize_partials");
+  if (root->kind != DDQ_OP_AGGREGATE || root->n_aggs < 1 || root->n_aggs > DDQ_MAX_AGGS ||
+      root->n_keys < 0 || root->n_keys > DDQ_MAX_KEYS)
+    return set_error(DDQ_EINVAL, "finalize_partials: root must be an AGGREGATE");
+  return finalize_result(*root, n, keys, accs, out);
 }
 
 ddq_status ddq_prepared_finalize(ddq_prepared* p, int64_t n_groups, const int64_t* h_keys, const int64_t* h_accs,

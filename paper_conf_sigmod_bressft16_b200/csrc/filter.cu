@@ -50,6 +50,9 @@ struct FilterParams {
   int32_t shift;
   const int32_t* fk;
   int32_t* out_payload;
+  int32_t fk_by_pos;    // probe keys are an aligned vector (fk[i]), not a column (fk[row])
+  const int32_t* eq_a;  // FILTER_EQ vectors (positional), or null
+  const int32_t* eq_b;
   int32_t direct;  // direct-mapped join index instead of the hash table
   const uint32_t* bitmap;
   const int32_t* payarr;
@@ -164,6 +167,13 @@ filter_kernel(const __grid_constant__ FilterParams P) {
         for (int k = 0; k < FT_ITEMS; k++)
           if (!eval_pred(pr, vals[k])) flags &= ~(1u << k);
       }
+      if (P.eq_a) {  // FILTER_EQ: two aligned (positional) vectors must be equal
+#pragma unroll
+        for (int k = 0; k < FT_ITEMS; k++) {
+          const int64_t pos = wbase + (k >> 2) * 128 + lane * 4 + (k & 3);
+          if (((flags >> k) & 1u) && __ldg(P.eq_a + pos) != __ldg(P.eq_b + pos)) flags &= ~(1u << k);
+        }
+      }
     } else {
       int32_t keys[FT_ITEMS];
       if (!kTids) {
@@ -180,7 +190,10 @@ filter_kernel(const __grid_constant__ FilterParams P) {
         }
       } else {
 #pragma unroll
-        for (int k = 0; k < FT_ITEMS; k++) keys[k] = ((flags >> k) & 1u) ? __ldg(P.fk + rows[k]) : 0;
+        for (int k = 0; k < FT_ITEMS; k++) {
+          const int64_t pos = wbase + (k >> 2) * 128 + lane * 4 + (k & 3);
+          keys[k] = ((flags >> k) & 1u) ? __ldg(P.fk + (P.fk_by_pos ? pos : (int64_t)rows[k])) : 0;
+        }
       }
       if (P.direct) {
         uint32_t w[FT_ITEMS];
@@ -331,6 +344,9 @@ cudaError_t launch_filter(const FilterArgs& a, cudaStream_t st) {
   p.shift = 32 - lg;
   p.fk = a.fk;
   p.out_payload = a.out_payload;
+  p.fk_by_pos = a.fk_by_pos ? 1 : 0;
+  p.eq_a = a.eq_a;
+  p.eq_b = a.eq_b;
   p.direct = a.bitmap != nullptr;
   p.bitmap = a.bitmap;
   p.payarr = a.payarr;

@@ -157,6 +157,7 @@ struct GroupbyParams {
   int32_t n_keys;
   const int32_t* key_vec[3];
   const int32_t* key_col[3];
+  int32_t key_shift[3];
   int32_t n_aggs;
   int32_t kind[8];
   int32_t width[8][3];
@@ -235,7 +236,7 @@ __global__ void __launch_bounds__(GB_THREADS) groupby_kernel(const __grid_consta
       key = 0;
       for (int k = 0; k < P.n_keys; k++) {
         const int32_t c = P.key_vec[k] ? P.key_vec[k][i] : __ldg(P.key_col[k] + r);
-        key |= (long long)(uint32_t)c << (21 * k);
+        key |= (long long)(uint32_t)c << P.key_shift[k];
       }
     }
     const unsigned peers = __match_any_sync(FULL, key);
@@ -307,6 +308,7 @@ cudaError_t launch_groupby_init(void* table, uint32_t capacity, int n_aggs, cuda
 
 cudaError_t launch_groupby(const int32_t* tids, const uint32_t* d_count, int64_t n_cap,
                            const int32_t* const* key_vec, const int32_t* const* key_col, int n_keys,
+                           const int32_t* key_bits,
                            const ddq_dev_agg* aggs, int n_aggs, void* table, uint32_t capacity,
                            uint32_t* d_error, cudaStream_t st) {
   GroupbyParams p{};
@@ -314,6 +316,10 @@ cudaError_t launch_groupby(const int32_t* tids, const uint32_t* d_count, int64_t
   p.d_count = d_count;
   p.n_static = (uint32_t)n_cap;
   p.n_keys = n_keys;
+  for (int k = 0, sh = 0; k < 3; k++) {
+    p.key_shift[k] = sh;
+    sh += (key_bits && key_bits[k] > 0) ? key_bits[k] : 21;
+  }
   for (int k = 0; k < n_keys; k++) {
     p.key_vec[k] = key_vec ? key_vec[k] : nullptr;
     p.key_col[k] = key_col ? key_col[k] : nullptr;

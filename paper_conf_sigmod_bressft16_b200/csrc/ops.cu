@@ -179,9 +179,15 @@ ddq_status ddq_op_groupby_init(void* table, uint32_t capacity, int32_t n_aggs, v
 }
 
 ddq_status ddq_op_groupby(const int32_t* tids, const uint32_t* d_count, int64_t n_cap, const int32_t* const* key_vec,
-                          const int32_t* const* key_col, int32_t n_keys, const ddq_dev_agg* aggs, int32_t n_aggs,
-                          void* table, uint32_t capacity, uint32_t* d_error, void* stream) {
+                          const int32_t* const* key_col, int32_t n_keys, const int32_t* key_bits,
+                          const ddq_dev_agg* aggs, int32_t n_aggs, void* table, uint32_t capacity, uint32_t* d_error,
+                          void* stream) {
   if (ddq_status s = check_cap(n_cap)) return s;
+  {
+    int bits = 0;
+    for (int k = 0; k < n_keys && k < DDQ_MAX_KEYS; k++) bits += (key_bits && key_bits[k] > 0) ? key_bits[k] : 21;
+    if (bits > 63) return set_error(DDQ_EINVAL, "groupby: packed key wider than 63 bits");
+  }
   if (!tids || !table || !d_error || capacity < 2 || (capacity & (capacity - 1)))
     return set_error(DDQ_EINVAL, "groupby: bad arguments");
   if (n_keys < 0 || n_keys > DDQ_MAX_KEYS || n_aggs < 1 || n_aggs > DDQ_MAX_AGGS || !aggs)
@@ -197,7 +203,8 @@ ddq_status ddq_op_groupby(const int32_t* tids, const uint32_t* d_count, int64_t 
       if (!aggs[a].arg[j] || (aggs[a].width[j] != 4 && aggs[a].width[j] != 8))
         return set_error(DDQ_EINVAL, "groupby: bad aggregate argument");
   }
-  return cuda_status(launch_groupby(tids, d_count, n_cap, key_vec, key_col, n_keys, aggs, n_aggs, table, capacity,
+  return cuda_status(launch_groupby(tids, d_count, n_cap, key_vec, key_col, n_keys, key_bits, aggs, n_aggs, table,
+                                    capacity,
                                     d_error, (cudaStream_t)stream),
                      "ddq_op_groupby");
 }

@@ -14,6 +14,9 @@ struct FilterArgs {
   bool probe = false;
   bool no_smem = false;
   bool stable = false;  // dense inputs: force the single-pass look-back kernel (ascending TIDs)
+  bool fk_by_pos = false;          // probe keys from an aligned vector (TID inputs)
+  const int32_t* eq_a = nullptr;   // FILTER_EQ positional vectors (TID inputs)
+  const int32_t* eq_b = nullptr;
   const uint64_t* table = nullptr;
   uint32_t capacity = 0;
   // direct-mapped join index (probe): bitmap + payload array over [key_min, key_min+range)
@@ -60,6 +63,7 @@ size_t groupby_table_bytes(uint32_t capacity, int n_aggs);
 cudaError_t launch_groupby_init(void* table, uint32_t capacity, int n_aggs, cudaStream_t st);
 cudaError_t launch_groupby(const int32_t* tids, const uint32_t* d_count, int64_t n_cap,
                            const int32_t* const* key_vec, const int32_t* const* key_col, int n_keys,
+                           const int32_t* key_bits,
                            const ddq_dev_agg* aggs, int n_aggs, void* table, uint32_t capacity,
                            uint32_t* d_error, cudaStream_t st);
 cudaError_t launch_groupby_compact(const void* table, uint32_t capacity, int n_aggs, int64_t* out_keys,

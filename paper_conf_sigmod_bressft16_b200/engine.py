@@ -100,11 +100,21 @@ class PlanBuilder:
         op.payload_col = self.db.col(table, payload) if payload else -1
         return idx
 
-    def probe(self, table: str, fk: str, build: int, input: int = -1, emit: bool = False) -> int:
+    def probe(self, table: str, fk, build: int, input: int = -1, emit: bool = False) -> int:
+        """fk: a column of `table`, or an int = index of an aligned input vector."""
         idx, op = self._op(A.OP_HASH_PROBE, table, input)
-        op.fk_col = self.db.col(table, fk)
+        if isinstance(fk, int):
+            op.fk_vec = fk + 1
+        else:
+            op.fk_col = self.db.col(table, fk)
         op.build = build
         op.emit_payload = 1 if emit else 0
+        return idx
+
+    def filter_eq(self, table: str, input: int, vec_a: int, vec_b: int) -> int:
+        """Keep rows whose aligned vectors vec_a and vec_b are equal."""
+        idx, op = self._op(A.OP_FILTER_EQ, table, input)
+        op.eq_vec[0], op.eq_vec[1] = vec_a + 1, vec_b + 1
         return idx
 
     def gather(self, table: str, col: str, input: int) -> int:
@@ -113,10 +123,13 @@ class PlanBuilder:
         return idx
 
     def aggregate(self, table: str, input: int, keys: list, aggs: list, order_by: list | None = None,
-                  max_groups: int = 0, limit: int = 0) -> int:
+                  max_groups: int = 0, limit: int = 0, key_bits: list | None = None) -> int:
         """keys: int (aligned vector index) or str (column of `table`).
-        aggs: (kind, [cols]).  order_by: ints per include/ddq.h (+/-(1+k), +/-(101+a))."""
+        aggs: (kind, [cols]).  order_by: ints per include/ddq.h (+/-(1+k), +/-(101+a)).
+        key_bits: bits per key in the packed group key (default 21 each, sum <= 63)."""
         idx, op = self._op(A.OP_AGGREGATE, table, input)
+        for k, b in enumerate(key_bits or []):
+            op.key_bits[k] = b
         op.n_keys = len(keys)
         for k, src in enumerate(keys):
             op.key_src[k] = src if isinstance(src, int) else -2 - self.db.col(table, src)
@@ -132,6 +145,37 @@ class PlanBuilder:
         op.max_groups = max_groups
         op.limit = limit
         return idx
+
+
+def finalize_partials(root: A.Op, keys: np.ndarray, accs: np.ndarray) -> QueryResult:
+    """Host finalisation of (possibly duplicated) partial groups: exact merge of equal
+    packed keys, ORDER BY / LIMIT of the root AGGREGATE (no GPU needed)."""
+    keys = np.ascontiguousarray(keys, np.int64)
+    accs = np.ascontiguousarray(accs, np.int64)
+    p = ctypes.POINTER(A.Result)()
+    check(lib().ddq_finalize_partials(ctypes.byref(root), keys.size, keys.ctypes.data, accs.ctypes.data,
+                                      ctypes.byref(p)))
+    return _convert(p)
+
+
+class Catalog:
+    """Name -> id catalogue without a device (plans for host-only finalisation)."""
+
+    def __init__(self, dicts: dict[str, list[str]]):
+        self.dicts = dicts
+        self._ids: dict = {}
+
+    def _id(self, key) -> int:
+        return self._ids.setdefault(key, len(self._ids))
+
+    def table_id(self, table: str) -> int:
+        return self._id(("t", table))
+
+    def col(self, table: str, name: str) -> int:
+        return self._id(("c", table, name))
+
+    def plan(self) -> "PlanBuilder":
+        return PlanBuilder(self)
 
 
 class Prepared:
@@ -173,6 +217,14 @@ class Prepared:
         check(lib().ddq_prepared_partials(self.h, ctypes.c_void_p(stream), ctypes.byref(g),
                                           keys.ctypes.data, accs.ctypes.data, cap))
         return keys[:g.value], accs[:g.value * na * 2].reshape(g.value, na, 2)
+
+    def partials_device(self):
+        """(keys_ptr, accs_ptr, count_ptr, capacity) of the device partial table."""
+        k, a, c = ctypes.c_void_p(), ctypes.c_void_p(), ctypes.c_void_p()
+        cap = ctypes.c_int64()
+        check(lib().ddq_prepared_partials_device(self.h, ctypes.byref(k), ctypes.byref(a), ctypes.byref(c),
+                                                 ctypes.byref(cap)))
+        return k.value, a.value, c.value, cap.value
 
     def finalize(self, keys: np.ndarray, accs: np.ndarray) -> QueryResult:
         keys = np.ascontiguousarray(keys, np.int64)

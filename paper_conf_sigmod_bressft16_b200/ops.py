@@ -125,7 +125,7 @@ def gather(col, tids, count, n: int):
     return out
 
 
-def groupby(tids, count, n: int, key_vecs=(), key_cols=(), aggs=(), capacity: int = 1024):
+def groupby(tids, count, n: int, key_vecs=(), key_cols=(), aggs=(), capacity: int = 1024, key_bits=None):
     """aggs: list of (kind, [arg column tensors]).  Returns (keys[g], accs[g, n_aggs, 2], g)."""
     nk = max(len(key_vecs), len(key_cols))
     kv = (ctypes.c_void_p * 3)(*[(key_vecs[k].data_ptr() if k < len(key_vecs) and key_vecs[k] is not None
@@ -142,7 +142,8 @@ def groupby(tids, count, n: int, key_vecs=(), key_cols=(), aggs=(), capacity: in
     table = torch.empty(lib().ddq_op_groupby_table_bytes(capacity, na), dtype=torch.uint8, device="cuda")
     err = count_cell()
     check(lib().ddq_op_groupby_init(table.data_ptr(), capacity, na, _stream()))
-    check(lib().ddq_op_groupby(tids.data_ptr(), _ptr(count), n, kv, kc, nk, da, na, table.data_ptr(), capacity,
+    kb = (ctypes.c_int32 * 3)(*(list(key_bits or []) + [0, 0, 0])[:3])
+    check(lib().ddq_op_groupby(tids.data_ptr(), _ptr(count), n, kv, kc, nk, kb, da, na, table.data_ptr(), capacity,
                                err.data_ptr(), _stream()))
     keys = torch.empty(capacity, dtype=torch.int64, device="cuda")
     accs = torch.empty(capacity * max(na, 1) * 2, dtype=torch.int64, device="cuda")

@@ -1,0 +1,96 @@
+"""TPC-H Q1, Q3, Q5, Q6 on libddq (BASELINE config 4; the paper runs TPC-H,
+PAPER.md:305, App. C.2).  Decimals are scale-2 int64 (reading O5); dates
+are int32 yyyymmdd with folded constants (O11).  Query texts: SURVEY.md App. A.2.
+"""
+from __future__ import annotations
+
+from . import _abi as A
+from .engine import Database, PlanBuilder
+from .ssb import code
+
+TPCH_QUERIES = ["tpch1", "tpch3", "tpch5", "tpch6"]
+
+TABLE_COLUMNS = {
+    "nation": ["n_nationkey", "n_name", "n_regionkey"],
+    "region": ["r_regionkey", "r_name"],
+    "customer": ["c_custkey", "c_nationkey", "c_mktsegment"],
+    "supplier": ["s_suppkey", "s_nationkey"],
+    "orders": ["o_orderkey", "o_custkey", "o_orderdate", "o_shippriority"],
+    "lineitem": ["l_orderkey", "l_suppkey", "l_quantity", "l_extendedprice", "l_discount", "l_tax",
+                 "l_returnflag", "l_linestatus", "l_shipdate"],
+}
+STRING_DICTS = {"n_name": "nation", "r_name": "region", "c_mktsegment": "mktsegment",
+                "l_returnflag": "returnflag", "l_linestatus": "linestatus"}
+QUERY_TABLES = {"tpch1": ["lineitem"], "tpch6": ["lineitem"],
+                "tpch3": ["customer", "orders", "lineitem"],
+                "tpch5": ["region", "nation", "supplier", "customer", "orders", "lineitem"]}
+
+
+def load_tpch(db: Database, data, cache: bool = True, tables=None) -> None:
+    """data: ``data.col(table, col)``, ``data.rows(table)``, ``data.dict_for(col)``."""
+    for t in (tables or TABLE_COLUMNS):
+        db.create_table(t, data.rows(t))
+        for c in TABLE_COLUMNS[t]:
+            db.load_column(t, c, data.col(t, c))
+            if cache:
+                db.cache(t, c)
+    for c, d in STRING_DICTS.items():
+        db.dicts[d] = data.dict_for(c)
+
+
+def tpch_plan(db: Database, q: str, limit: int = 0) -> PlanBuilder:
+    P = db.plan()
+    li = "lineitem"
+    if q == "tpch1":
+        # l_shipdate <= date '1998-12-01' - interval '90' day  (= 19980902, O11)
+        t = P.select(li, [("l_shipdate", -2**31, 19980902)])
+        P.aggregate(li, t, keys=["l_returnflag", "l_linestatus"],
+                    aggs=[(A.AGG_SUM, ["l_quantity"]), (A.AGG_SUM, ["l_extendedprice"]),
+                          (A.AGG_SUM_MUL_100M, ["l_extendedprice", "l_discount"]),
+                          (A.AGG_SUM_MUL_100M_100P, ["l_extendedprice", "l_discount", "l_tax"]),
+                          (A.AGG_SUM, ["l_discount"]), (A.AGG_COUNT, [])],
+                    order_by=[1, 2], max_groups=6)
+        return P
+    if q == "tpch6":
+        # shipdate in 1994 (15 %) first; discount 0.05..0.07 and quantity < 24 at its TIDs
+        t = P.select(li, [("l_shipdate", 19940101, 19941231)])
+        t = P.select(li, [("l_discount", 5, 7)], input=t)
+        t = P.select(li, [("l_quantity", -2**62, 2399)], input=t)
+        P.aggregate(li, t, keys=[], aggs=[(A.AGG_SUM_MUL, ["l_extendedprice", "l_discount"]),
+                                          (A.AGG_COUNT, [])], max_groups=1)
+        return P
+    if q == "tpch3":
+        c = P.select("customer", [("c_mktsegment", [code(db, "mktsegment", "BUILDING")])])
+        hc = P.build("customer", "c_custkey", input=c)
+        o = P.select("orders", [("o_orderdate", -2**31, 19950314)])        # < 1995-03-15
+        o = P.probe("orders", "o_custkey", hc, input=o)
+        hod = P.build("orders", "o_orderkey", "o_orderdate", input=o)
+        hos = P.build("orders", "o_orderkey", "o_shippriority", input=o)
+        t = P.select(li, [("l_shipdate", 19950316, 2**31 - 1)])            # > 1995-03-15
+        t = P.probe(li, "l_orderkey", hod, input=t, emit=True)            # vec0 = o_orderdate
+        t = P.probe(li, "l_orderkey", hos, input=t, emit=True)            # vec1 = o_shippriority
+        # group by l_orderkey, o_orderdate, o_shippriority; order by revenue desc,
+        # o_orderdate, then l_orderkey (O9)
+        P.aggregate(li, t, keys=["l_orderkey", 0, 1], key_bits=[28, 25, 10],
+                    aggs=[(A.AGG_SUM_MUL_100M, ["l_extendedprice", "l_discount"])],
+                    order_by=[-101, 2, 1], max_groups=1 << 22, limit=limit)
+        return P
+    if q == "tpch5":
+        r = P.select("region", [("r_name", [code(db, "region", "ASIA")])])
+        hr = P.build("region", "r_regionkey", input=r)
+        n = P.probe("nation", "n_regionkey", hr)                         # nations of ASIA
+        hn = P.build("nation", "n_nationkey", "n_name", input=n)
+        s = P.probe("supplier", "s_nationkey", hn)                       # suppliers in ASIA
+        hs = P.build("supplier", "s_suppkey", "s_nationkey", input=s)
+        hc = P.build("customer", "c_custkey", "c_nationkey")
+        o = P.select("orders", [("o_orderdate", 19940101, 19941231)])
+        ho = P.build("orders", "o_orderkey", "o_custkey", input=o)
+        t = P.probe(li, "l_orderkey", ho, emit=True)                     # vec0 = o_custkey
+        t = P.probe(li, "l_suppkey", hs, input=t, emit=True)             # vec1 = s_nationkey
+        t = P.probe(li, 0, hc, input=t, emit=True)                       # vec2 = c_nationkey
+        t = P.filter_eq(li, t, 1, 2)                                     # c_nationkey = s_nationkey
+        t = P.probe(li, 1, hn, input=t, emit=True)                       # vec3 = n_name
+        P.aggregate(li, t, keys=[3], aggs=[(A.AGG_SUM_MUL_100M, ["l_extendedprice", "l_discount"])],
+                    order_by=[-101, 1], max_groups=25)
+        return P
+    raise KeyError(q)
