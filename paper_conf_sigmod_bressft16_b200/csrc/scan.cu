@@ -1,22 +1,24 @@
-// scan.cu -- dense scan kernel: selection (S8(a2)) and first hash probe (S8(a4))
-// over ALL rows of a fact column, the dominant kernel of every SSB plan.
+// scan.cu -- the filter kernel of the hot path: selection (S8(a1)/(a2)), hash /
+// join-index probe (S8(a4)) and FILTER_EQ, over ALL rows of a column ("dense") or
+// over a TID list ("gather"), emitting the compacted survivors.
 //
-// B200 design (DESIGN.md "dense scan"); each choice answers an ncu finding:
+// B200 design (DESIGN.md "scan"); each choice answers an ncu finding:
 //   * one persistent CTA per SM holding G independent 256-thread "groups".  Each
 //     group is a complete pipeline (own TMA ring, mbarriers, named barrier, survivor
 //     lists), so one group's barrier / atomic / TMA wait overlaps the others'
 //     compute, while the dimension table or bitmap is staged ONCE per SM in shared
 //     memory for all groups (random lookups at smem bandwidth, not L1/L2 sectors);
-//   * input columns stream through an S-stage smem ring filled by one thread with
-//     TMA bulk copies (cp.async.bulk + mbarrier complete_tx): no per-thread copy
-//     instructions, S-1 tiles in flight per group;
+//   * the streamed input (fact columns, or the TID list) goes through an S-stage
+//     smem ring filled by one thread with TMA bulk copies (cp.async.bulk + mbarrier
+//     complete_tx): no per-thread copy instructions, tiles in flight per group;
+//     gathered columns (TID mode) are 16 independent loads per thread;
 //   * full tiles need no row-bound checks; survivors are compacted with a packed
 //     warp scan, staged in smem and copied out coalesced, survivors only;
-//   * the output range of a 4096-row tile is reserved with ONE atomicAdd whose
+//   * the output range of a 4096-item tile is reserved with ONE atomicAdd whose
 //     latency is hidden: tile k is copied out in iteration k+1 (double-buffered
-//     lists).  Rows stay ascending within a tile; tiles appear in reservation order
-//     (reading O14': a TID list is a multiset; aggregates are exact integer sums,
-//     so query results are bit-identical whatever the order).
+//     lists).  Items stay in input order within a tile; tiles appear in reservation
+//     order (reading O14': a TID list is a multiset; aggregates are exact integer
+//     sums, so query results are bit-identical whatever the order);
 //   * compact-range dimension keys use a direct-mapped join index (membership
 //     bitmap + payload array): one lookup per row, no collision chains.
 #include <cstdint>
@@ -29,8 +31,8 @@ namespace ddq {
 
 constexpr int SC_GT = 256;                 // threads per group
 constexpr int SC_GW = SC_GT / 32;          // warps per group
-constexpr int SC_TILE = 4096;              // rows per tile
-constexpr int SC_ITEMS = SC_TILE / SC_GT;  // 16 rows per thread
+constexpr int SC_TILE = 4096;              // items per tile
+constexpr int SC_ITEMS = SC_TILE / SC_GT;  // 16 items per thread
 constexpr int SC_SLOTS = SC_ITEMS / 4;     // 4 x (one 16-byte vector of int32)
 constexpr int SC_MAXCOLS = 4;
 constexpr int SC_MAXG = 4;
@@ -45,8 +47,9 @@ struct ScanPred {
 };
 
 struct ScanParams {
-  uint32_t n;  // rows
-  int32_t n_cols;
+  uint32_t n;                  // items (dense: rows); TID mode: read from d_in_count
+  const uint32_t* d_in_count;  // TID mode
+  int32_t n_cols;              // streamed columns (dense: predicate / fk columns; TID mode: the TIDs)
   const void* cols[SC_MAXCOLS];
   int32_t width[SC_MAXCOLS];
   int32_t col_off[SC_MAXCOLS];  // byte offset of the column's chunk inside a stage
@@ -58,8 +61,12 @@ struct ScanParams {
   // select
   int32_t n_preds;
   ScanPred preds[SC_MAXCOLS];
-  // probe (fk = cols[0])
+  const int32_t* eq_a;  // FILTER_EQ (positional vectors)
+  const int32_t* eq_b;
+  // probe
   int32_t probe;
+  const int32_t* fk;  // probe keys: column (indexed by row) or vector (by position)
+  int32_t fk_by_pos;
   const uint64_t* table;
   uint32_t cap_mask;
   int32_t shift;
@@ -72,6 +79,10 @@ struct ScanParams {
   uint32_t bitmap_words;
   int32_t bitmap_in_smem;
   int32_t* out_payload;
+  // carried vectors (TID mode)
+  int32_t n_carry;
+  const int32_t* carry_in[4];
+  int32_t* carry_out[4];
   // outputs
   int32_t* out_tids;
   uint32_t* d_out_count;  // [0] survivors, [1] CTA completion counter; zeroed before launch
@@ -105,13 +116,14 @@ __device__ __forceinline__ void group_sync(int g) {
   asm volatile("bar.sync %0, %1;" ::"r"(g + 1), "r"(SC_GT) : "memory");
 }
 
-// Group leader: one bulk copy per column of tile `tile` into stage buffer `buf`.
-// Columns are readable up to the next 16-byte boundary (library allocations are
+// Group leader: one bulk copy per streamed column of tile `tile` into `buf`.
+// Buffers are readable up to the next 16-byte boundary (library allocations are
 // padded; torch allocations are 512-byte granular), so the tail tile is copied
-// rounded up to 16 bytes and its invalid rows are masked by the row bound.
-__device__ __forceinline__ void issue_tile(const ScanParams& P, uint8_t* buf, uint64_t* bar, uint32_t tile) {
+// rounded up to 16 bytes and its invalid items are masked by the item bound.
+__device__ __forceinline__ void issue_tile(const ScanParams& P, uint32_t n, uint8_t* buf, uint64_t* bar,
+                                           uint32_t tile) {
   const uint64_t row0 = (uint64_t)tile * SC_TILE;
-  const uint64_t rows = (uint64_t)P.n - row0 < (uint64_t)SC_TILE ? (uint64_t)P.n - row0 : (uint64_t)SC_TILE;
+  const uint64_t rows = (uint64_t)n - row0 < (uint64_t)SC_TILE ? (uint64_t)n - row0 : (uint64_t)SC_TILE;
   uint32_t total = 0;
   uint32_t bytes[SC_MAXCOLS];
   for (int c = 0; c < P.n_cols; c++) {
@@ -131,7 +143,44 @@ __device__ __forceinline__ bool scan_pred(const ScanPred& p, int64_t v) {
   return m;
 }
 
-template <int G>
+// Membership (+ lookup) of 16 keys; clears the flag bits of misses.
+template <bool kHashPayload>
+__device__ __forceinline__ void probe16(const ScanParams& P, const uint64_t* table, const uint32_t* bm,
+                                        const int32_t (&key)[SC_ITEMS], uint32_t& flags,
+                                        int32_t (&payload)[SC_ITEMS]) {
+  if (P.direct) {
+    uint32_t m = 0;
+#pragma unroll
+    for (int k = 0; k < SC_ITEMS; k++) {
+      const uint32_t o = (uint32_t)(key[k] - P.key_min);
+      const uint32_t oo = o < P.range ? o : 0u;
+      const uint32_t w = bm[oo >> 5];
+      m |= ((o < P.range ? (w >> (oo & 31)) : 0u) & 1u) << k;
+    }
+    flags &= m;  // payloads: fetched for survivors only, at copy-out
+  } else {
+    uint32_t h[SC_ITEMS];
+    uint64_t sl[SC_ITEMS];
+#pragma unroll
+    for (int k = 0; k < SC_ITEMS; k++) {
+      h[k] = ht_hash(key[k], P.shift);
+      sl[k] = ((flags >> k) & 1u) ? table[h[k]] : HT_EMPTY;
+    }
+#pragma unroll
+    for (int k = 0; k < SC_ITEMS; k++) {
+      uint64_t s = sl[k];
+      uint32_t hh = h[k];
+      while (s != HT_EMPTY && ht_key(s) != key[k]) {
+        hh = (hh + 1) & P.cap_mask;
+        s = table[hh];
+      }
+      if (s == HT_EMPTY) flags &= ~(1u << k);
+      if (kHashPayload) payload[k] = ht_val(s);
+    }
+  }
+}
+
+template <int G, bool kTids>
 __global__ void __launch_bounds__(SC_GT* G, 1) scan_kernel(const __grid_constant__ ScanParams P) {
   extern __shared__ __align__(128) uint8_t smem[];
   __shared__ uint32_t s_warp_tot[SC_MAXG][SC_GW];
@@ -140,20 +189,25 @@ __global__ void __launch_bounds__(SC_GT* G, 1) scan_kernel(const __grid_constant
   const int g = threadIdx.x / SC_GT;     // group
   const int t = threadIdx.x % SC_GT;     // thread within the group
   const int lane = t & 31, warp = t >> 5;
-  const uint32_t ntiles = (P.n + SC_TILE - 1) / SC_TILE;
+  const uint32_t n = kTids ? ld_relaxed_u32(P.d_in_count) : P.n;
+  const uint32_t ntiles = (n + SC_TILE - 1) / SC_TILE;
   const int S = P.stages;
+  // S-1 tiles in flight ahead of the current one; stage (k-1)%S is refilled with
+  // tile k+S-1 right after (A) in dense mode, after (B) in TID mode (whose copy-out
+  // of tile k-1 reads its TIDs from that stage)
+  const int ahead = S - 1;
   const uint32_t vb = blockIdx.x * G + g, vgrid = gridDim.x * G;  // virtual CTA id / count
   uint8_t* ring = smem + (size_t)g * P.group_bytes;
   uint16_t* s_list = reinterpret_cast<uint16_t*>(ring + P.list_off);              // 2 x TILE
   int32_t* s_pay = reinterpret_cast<int32_t*>(ring + P.list_off + SC_TILE * 4);   // 2 x TILE
   uint64_t* s_table = reinterpret_cast<uint64_t*>(smem + P.shared_off);
 
-  if (t == 0) {  // group leader: barriers, then S-1 tiles in flight
+  if (t == 0) {  // group leader: barriers, then the first tiles in flight
     for (int k = 0; k < S; k++) mbar_init(&s_full[g][k], 1);
     fence_mbar_init();
-    for (int k = 0; k < S - 1; k++) {
+    for (int k = 0; k < ahead; k++) {
       const uint32_t tl = vb + (uint32_t)k * vgrid;
-      if (tl < ntiles) issue_tile(P, ring + (size_t)k * P.stage_bytes, &s_full[g][k], tl);
+      if (tl < ntiles) issue_tile(P, n, ring + (size_t)k * P.stage_bytes, &s_full[g][k], tl);
     }
   }
   // all groups stage the shared table / bitmap once per SM (overlaps the first loads)
@@ -172,26 +226,65 @@ __global__ void __launch_bounds__(SC_GT* G, 1) scan_kernel(const __grid_constant
   // stages its survivors in list[k&1] while its output reservation (one atomic) is
   // in flight; it copies out tile k-1, whose range was reserved last iteration.
   uint32_t prev_tot = 0, prev_base = 0;
-  const uint32_t wrow = warp * (32 * SC_ITEMS);  // warp's first row inside a tile
+  const uint32_t wrow = warp * (32 * SC_ITEMS);  // warp's first item inside a tile
   for (uint32_t k = 0;; k++) {
     const uint32_t tile = vb + k * vgrid;
     const bool have = tile < ntiles;
-    const uint32_t row0 = tile * SC_TILE;
+    const uint32_t row0 = tile * SC_TILE;  // first item of the tile
     uint32_t flags = 0;
     int32_t payload[SC_ITEMS];
     if (have) {
       mbar_wait(&s_full[g][k % S], (k / S) & 1u);
       const uint8_t* buf = ring + (size_t)(k % S) * P.stage_bytes;
       flags = 0xFFFFu;
-      if (row0 + SC_TILE > P.n) {  // tail tile only
+      if (row0 + SC_TILE > n) {  // tail tile only
         flags = 0;
 #pragma unroll
         for (int s = 0; s < SC_SLOTS; s++)
 #pragma unroll
           for (int v = 0; v < 4; v++)
-            flags |= (row0 + wrow + s * 128 + lane * 4 + v < P.n ? 1u : 0u) << (s * 4 + v);
+            flags |= (row0 + wrow + s * 128 + lane * 4 + v < n ? 1u : 0u) << (s * 4 + v);
       }
-      if (!P.probe) {
+      if (kTids) {
+        // ---- TID mode: rows from the staged TID list, values gathered ----------
+        int32_t row[SC_ITEMS];
+#pragma unroll
+        for (int s = 0; s < SC_SLOTS; s++) {
+          const int4 a = *reinterpret_cast<const int4*>(buf + (size_t)(wrow + s * 128 + lane * 4) * 4);
+          row[s * 4 + 0] = a.x; row[s * 4 + 1] = a.y; row[s * 4 + 2] = a.z; row[s * 4 + 3] = a.w;
+        }
+        if (!P.probe) {
+          for (int p = 0; p < P.n_preds; p++) {
+            const ScanPred& pr = P.preds[p];
+            int64_t v[SC_ITEMS];
+#pragma unroll
+            for (int k2 = 0; k2 < SC_ITEMS; k2++) v[k2] = ((flags >> k2) & 1u) ? col_at(pr.col, pr.width, row[k2]) : 0;
+            uint32_t m = 0;
+#pragma unroll
+            for (int k2 = 0; k2 < SC_ITEMS; k2++) m |= (scan_pred(pr, v[k2]) ? 1u : 0u) << k2;
+            flags &= m;
+          }
+          if (P.eq_a) {
+            uint32_t m = 0;
+#pragma unroll
+            for (int k2 = 0; k2 < SC_ITEMS; k2++) {
+              const uint32_t pos = row0 + wrow + (k2 >> 2) * 128 + lane * 4 + (k2 & 3);
+              m |= (((flags >> k2) & 1u) && __ldg(P.eq_a + pos) == __ldg(P.eq_b + pos) ? 1u : 0u) << k2;
+            }
+            flags &= m;
+          }
+        } else {
+          int32_t key[SC_ITEMS];
+#pragma unroll
+          for (int k2 = 0; k2 < SC_ITEMS; k2++) {
+            const uint32_t pos = row0 + wrow + (k2 >> 2) * 128 + lane * 4 + (k2 & 3);
+            key[k2] = ((flags >> k2) & 1u) ? __ldg(P.fk + (P.fk_by_pos ? (int64_t)pos : (int64_t)row[k2])) : 0;
+          }
+          if (hash_pay) probe16<true>(P, table, bm, key, flags, payload);
+          else probe16<false>(P, table, bm, key, flags, payload);
+        }
+      } else if (!P.probe) {
+        // ---- dense select: values from the staged columns ----------------------
         for (int p = 0; p < P.n_preds; p++) {
           const ScanPred& pr = P.preds[p];
           const uint8_t* cb = buf + P.col_off[p];
@@ -213,49 +306,16 @@ __global__ void __launch_bounds__(SC_GT* G, 1) scan_kernel(const __grid_constant
             flags &= ~((~m & 0xFu) << (s * 4));
           }
         }
-      } else if (P.direct) {
-        // one bitmap probe per row; survivors' payload loads are issued now and
-        // consumed after the group scan, so their latency is hidden
-        uint32_t o[SC_ITEMS];
-#pragma unroll
-        for (int s = 0; s < SC_SLOTS; s++) {
-          const int4 a = *reinterpret_cast<const int4*>(buf + (size_t)(wrow + s * 128 + lane * 4) * 4);
-          o[s * 4 + 0] = (uint32_t)(a.x - P.key_min); o[s * 4 + 1] = (uint32_t)(a.y - P.key_min);
-          o[s * 4 + 2] = (uint32_t)(a.z - P.key_min); o[s * 4 + 3] = (uint32_t)(a.w - P.key_min);
-        }
-        uint32_t m = 0;
-#pragma unroll
-        for (int k2 = 0; k2 < SC_ITEMS; k2++) {
-          const uint32_t oo = o[k2] < P.range ? o[k2] : 0u;
-          const uint32_t w = bm[oo >> 5];
-          m |= ((o[k2] < P.range ? (w >> (oo & 31)) : 0u) & 1u) << k2;
-        }
-        flags &= m;  // payloads: fetched for survivors only, at copy-out
       } else {
+        // ---- dense probe: keys from the staged fk column -------------------------
         int32_t key[SC_ITEMS];
-        uint32_t h[SC_ITEMS];
-        uint64_t sl[SC_ITEMS];
 #pragma unroll
         for (int s = 0; s < SC_SLOTS; s++) {
           const int4 a = *reinterpret_cast<const int4*>(buf + (size_t)(wrow + s * 128 + lane * 4) * 4);
           key[s * 4 + 0] = a.x; key[s * 4 + 1] = a.y; key[s * 4 + 2] = a.z; key[s * 4 + 3] = a.w;
         }
-#pragma unroll
-        for (int k2 = 0; k2 < SC_ITEMS; k2++) {
-          h[k2] = ht_hash(key[k2], P.shift);
-          sl[k2] = ((flags >> k2) & 1u) ? table[h[k2]] : HT_EMPTY;
-        }
-#pragma unroll
-        for (int k2 = 0; k2 < SC_ITEMS; k2++) {
-          uint64_t s = sl[k2];
-          uint32_t hh = h[k2];
-          while (s != HT_EMPTY && ht_key(s) != key[k2]) {
-            hh = (hh + 1) & P.cap_mask;
-            s = table[hh];
-          }
-          if (s == HT_EMPTY) flags &= ~(1u << k2);
-          payload[k2] = ht_val(s);
-        }
+        if (hash_pay) probe16<true>(P, table, bm, key, flags, payload);
+        else probe16<false>(P, table, bm, key, flags, payload);
       }
     }
     // group scan of the per-slot survivor counts
@@ -273,7 +333,7 @@ __global__ void __launch_bounds__(SC_GT* G, 1) scan_kernel(const __grid_constant
       acc += (wtot >> (8 * s)) & 0xFFu;
     }
     if (lane == 0) s_warp_tot[g][warp] = acc;
-    group_sync(g);  // (A) warp totals visible; the group is done with tile k-1
+    group_sync(g);  // (A) warp totals visible; the group is done computing on tile k-1
     uint32_t tot = 0, warp_off = 0;
 #pragma unroll
     for (int w = 0; w < SC_GW; w++) {
@@ -283,17 +343,17 @@ __global__ void __launch_bounds__(SC_GT* G, 1) scan_kernel(const __grid_constant
     }
     uint32_t my_base = 0;
     if (t == 0) {
-      if (have) {  // keep S-1 tiles in flight: refill stage (k-1)%S, released by (A)
-        const uint32_t tl = tile + (uint32_t)(S - 1) * vgrid;
+      if (!kTids && have) {  // dense: refill stage (k-1)%S, released by (A)
+        const uint32_t tl = tile + (uint32_t)ahead * vgrid;
         if (tl < ntiles) {
           fence_proxy_async();
-          const int st = (int)((k + S - 1) % S);
-          issue_tile(P, ring + (size_t)st * P.stage_bytes, &s_full[g][st], tl);
+          const int st = (int)((k + ahead) % S);
+          issue_tile(P, n, ring + (size_t)st * P.stage_bytes, &s_full[g][st], tl);
         }
       }
       my_base = tot ? atomicAdd(P.d_out_count, tot) : 0;  // consumed only before (B)
     }
-    // stage tile k's survivors (tile-local row offsets + payloads) in list[k&1]
+    // stage tile k's survivors (tile-local item offsets + hash payloads) in list[k&1]
     uint16_t* lst = s_list + (k & 1) * SC_TILE;
     int32_t* pay = s_pay + (k & 1) * SC_TILE;
 #pragma unroll
@@ -314,25 +374,38 @@ __global__ void __launch_bounds__(SC_GT* G, 1) scan_kernel(const __grid_constant
       const uint16_t* pl = s_list + ((k - 1) & 1) * SC_TILE;
       const int32_t* pp = s_pay + ((k - 1) & 1) * SC_TILE;
       const uint32_t prow0 = (tile - vgrid) * SC_TILE;
+      const int32_t* ptid = reinterpret_cast<const int32_t*>(ring + (size_t)((k - 1) % S) * P.stage_bytes);
       const uint32_t lim = prev_base + prev_tot <= P.out_cap ? prev_tot
                          : (P.out_cap > prev_base ? P.out_cap - prev_base : 0);
       if (lim < prev_tot && t == 0 && P.d_overflow) atomicMax(P.d_overflow, 4u);
-      if (want_pay && !hash_pay) {  // direct join index: re-read the (L2-hot) key, fetch payload
-        for (uint32_t i = t; i < lim; i += SC_GT) {
-          const uint32_t r = prow0 + pl[i];
-          const int32_t key = __ldg(reinterpret_cast<const int32_t*>(P.cols[0]) + r);
-          P.out_tids[prev_base + i] = (int32_t)r;
-          P.out_payload[prev_base + i] = __ldg(P.payarr + (uint32_t)(key - P.key_min));
+      for (uint32_t i = t; i < lim; i += SC_GT) {
+        const uint32_t it = pl[i];
+        const int32_t r = kTids ? ptid[it] : (int32_t)(prow0 + it);
+        P.out_tids[prev_base + i] = r;
+        if (want_pay) {
+          int32_t pv;
+          if (hash_pay) {
+            pv = pp[i];
+          } else {  // direct join index: re-read the (L2-hot) key, fetch the payload
+            const int64_t ki = (kTids && P.fk_by_pos) ? (int64_t)(prow0 + it) : (int64_t)r;
+            pv = __ldg(P.payarr + (uint32_t)(__ldg(P.fk + ki) - P.key_min));
+          }
+          P.out_payload[prev_base + i] = pv;
         }
-      } else {
-        for (uint32_t i = t; i < lim; i += SC_GT) {
-          P.out_tids[prev_base + i] = (int32_t)(prow0 + pl[i]);
-          if (hash_pay) P.out_payload[prev_base + i] = pp[i];
-        }
+        if (kTids)
+          for (int c = 0; c < P.n_carry; c++) P.carry_out[c][prev_base + i] = __ldg(P.carry_in[c] + prow0 + it);
       }
     }
     if (t == 0) s_base[g] = my_base;
-    group_sync(g);  // (B) s_base visible; list[(k-1)&1] free for tile k+1
+    group_sync(g);  // (B) s_base visible; list[(k-1)&1] and (TID mode) stage (k-1)%S free
+    if (kTids && t == 0 && have) {  // TID mode: refill stage (k-1)%S now
+      const uint32_t tl = tile + (uint32_t)ahead * vgrid;
+      if (tl < ntiles) {
+        fence_proxy_async();
+        const int st = (int)((k + ahead) % S);
+        issue_tile(P, n, ring + (size_t)st * P.stage_bytes, &s_full[g][st], tl);
+      }
+    }
     prev_base = s_base[g];
     prev_tot = tot;
     if (!have) break;
@@ -350,14 +423,34 @@ __global__ void __launch_bounds__(SC_GT* G, 1) scan_kernel(const __grid_constant
 
 static int g_smem_optin = 0;
 
+template <bool kTids>
+static void set_attrs(int v) {
+  cudaFuncSetAttribute(scan_kernel<1, kTids>, cudaFuncAttributeMaxDynamicSharedMemorySize, v - 2048);
+  cudaFuncSetAttribute(scan_kernel<2, kTids>, cudaFuncAttributeMaxDynamicSharedMemorySize, v - 2048);
+  cudaFuncSetAttribute(scan_kernel<3, kTids>, cudaFuncAttributeMaxDynamicSharedMemorySize, v - 2048);
+  cudaFuncSetAttribute(scan_kernel<4, kTids>, cudaFuncAttributeMaxDynamicSharedMemorySize, v - 2048);
+}
+
 bool scan_supported(const FilterArgs& a) {
-  if (a.in_tids || a.n_carry) return false;  // dense inputs only
-  if (!a.probe && (a.n_preds < 1 || a.n_preds > SC_MAXCOLS)) return false;
-  // TMA bulk copies need 16-byte aligned column bases
+  if (a.n_carry > 4) return false;
+  if (!a.probe && a.n_preds > SC_MAXCOLS) return false;
+  if (!a.probe && a.n_preds < 1 && !a.eq_a) return false;
+  if (a.in_tids) return ((uintptr_t)a.in_tids & 15) == 0;  // TMA needs 16-byte aligned bases
+  if (a.eq_a || a.fk_by_pos || a.n_carry) return false;    // vectors exist only for TID inputs
   if (a.probe) return ((uintptr_t)a.fk & 15) == 0;
   for (int i = 0; i < a.n_preds; i++)
     if ((uintptr_t)a.preds[i].col & 15) return false;
   return true;
+}
+
+template <bool kTids>
+static void launch_g(int G, int64_t grid, size_t smem, cudaStream_t st, const ScanParams& p) {
+  switch (G) {
+    case 1: scan_kernel<1, kTids><<<(int)grid, SC_GT * 1, smem, st>>>(p); break;
+    case 2: scan_kernel<2, kTids><<<(int)grid, SC_GT * 2, smem, st>>>(p); break;
+    case 3: scan_kernel<3, kTids><<<(int)grid, SC_GT * 3, smem, st>>>(p); break;
+    default: scan_kernel<4, kTids><<<(int)grid, SC_GT * 4, smem, st>>>(p); break;
+  }
 }
 
 cudaError_t launch_scan(const FilterArgs& a, cudaStream_t st) {
@@ -366,41 +459,51 @@ cudaError_t launch_scan(const FilterArgs& a, cudaStream_t st) {
     cudaGetDevice(&dev);
     int v = 0;
     cudaDeviceGetAttribute(&v, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
-    cudaFuncSetAttribute(scan_kernel<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, v - 2048);
-    cudaFuncSetAttribute(scan_kernel<2>, cudaFuncAttributeMaxDynamicSharedMemorySize, v - 2048);
-    cudaFuncSetAttribute(scan_kernel<3>, cudaFuncAttributeMaxDynamicSharedMemorySize, v - 2048);
-    cudaFuncSetAttribute(scan_kernel<4>, cudaFuncAttributeMaxDynamicSharedMemorySize, v - 2048);
+    set_attrs<false>(v);
+    set_attrs<true>(v);
     g_smem_optin = v;
   }
+  const bool tids = a.in_tids != nullptr;
   ScanParams p{};
   p.n = (uint32_t)a.n_cap;
+  p.d_in_count = a.d_in_count;
   int off = 0;
-  if (a.probe) {
-    p.probe = 1;
+  if (tids) {  // stream the TID list; columns are gathered
+    p.n_cols = 1;
+    p.cols[0] = a.in_tids;
+    p.width[0] = 4;
+    off = SC_TILE * 4;
+  } else if (a.probe) {
     p.n_cols = 1;
     p.cols[0] = a.fk;
     p.width[0] = 4;
-    p.col_off[0] = 0;
     off = SC_TILE * 4;
   } else {
     p.n_cols = a.n_preds;
-    p.n_preds = a.n_preds;
     for (int i = 0; i < a.n_preds; i++) {
-      const ddq_dev_pred& d = a.preds[i];
-      p.cols[i] = d.col;
-      p.width[i] = d.width;
+      p.cols[i] = a.preds[i].col;
+      p.width[i] = a.preds[i].width;
       p.col_off[i] = off;
-      off += SC_TILE * d.width;
-      p.preds[i].col = d.col;
-      p.preds[i].width = d.width;
-      p.preds[i].kind = d.kind;
-      p.preds[i].lo = d.lo;
-      p.preds[i].hi = d.hi;
-      p.preds[i].n_in = d.n_in;
-      for (int j = 0; j < 8; j++) p.preds[i].in_vals[j] = d.in_vals[j];
+      off += SC_TILE * a.preds[i].width;
     }
   }
+  p.n_preds = a.probe ? 0 : a.n_preds;
+  for (int i = 0; i < p.n_preds; i++) {
+    const ddq_dev_pred& d = a.preds[i];
+    p.preds[i].col = d.col;
+    p.preds[i].width = d.width;
+    p.preds[i].kind = d.kind;
+    p.preds[i].lo = d.lo;
+    p.preds[i].hi = d.hi;
+    p.preds[i].n_in = d.n_in;
+    for (int j = 0; j < 8; j++) p.preds[i].in_vals[j] = d.in_vals[j];
+  }
+  p.eq_a = a.eq_a;
+  p.eq_b = a.eq_b;
   p.stage_bytes = off;
+  p.probe = a.probe ? 1 : 0;
+  p.fk = a.fk;
+  p.fk_by_pos = a.fk_by_pos ? 1 : 0;
   const bool direct = a.probe && a.bitmap != nullptr;
   const size_t table_bytes = a.probe ? (direct ? ((size_t)a.range + 31) / 32 * 4 : (size_t)a.capacity * 8) : 0;
   const size_t budget = (size_t)g_smem_optin - 2048;
@@ -410,10 +513,11 @@ cudaError_t launch_scan(const FilterArgs& a, cudaStream_t st) {
   const size_t shared = in_smem ? (table_bytes + 127) / 128 * 128 : 0;
   const size_t list_bytes = (size_t)SC_TILE * 4 + (a.probe && !direct && a.out_payload ? (size_t)SC_TILE * 8 : 0);
   // as many groups (up to 4) and stages (up to 4, at least 2) as shared memory allows
+  const int min_s = 2;
   int G = 4, S = 4;
   auto need = [&](int gg, int ss) { return shared + (size_t)gg * ((size_t)ss * p.stage_bytes + list_bytes); };
-  while (G > 1 && need(G, 2) > budget) G--;
-  while (S > 2 && need(G, S) > budget) S--;
+  while (G > 1 && need(G, min_s) > budget) G--;
+  while (S > min_s && need(G, S) > budget) S--;
   if (need(G, S) > budget) return cudaErrorInvalidConfiguration;
   p.stages = S;
   p.list_off = S * p.stage_bytes;
@@ -434,6 +538,11 @@ cudaError_t launch_scan(const FilterArgs& a, cudaStream_t st) {
     p.shift = 32 - lg;
   }
   if (a.probe) p.out_payload = a.out_payload;
+  p.n_carry = a.n_carry;
+  for (int c = 0; c < a.n_carry; c++) {
+    p.carry_in[c] = a.carry_in[c];
+    p.carry_out[c] = a.carry_out[c];
+  }
   p.out_tids = a.out_tids;
   p.d_out_count = a.d_out_count;
   p.out_cap = (uint32_t)(a.out_cap > 0 ? a.out_cap : a.n_cap);
@@ -441,16 +550,12 @@ cudaError_t launch_scan(const FilterArgs& a, cudaStream_t st) {
   cudaError_t e = cudaMemsetAsync(a.d_out_count, 0, 8, st);
   if (e != cudaSuccess) return e;
   const size_t smem = (size_t)p.shared_off + shared;
-  const int64_t ntiles = (a.n_cap + SC_TILE - 1) / SC_TILE;
+  const int64_t ntiles = (a.n_cap + SC_TILE - 1) / SC_TILE;  // upper bound (TID mode: capacity)
   int64_t grid = num_sms();
   const int64_t need_ctas = (ntiles + G - 1) / G;
   if (grid > need_ctas) grid = need_ctas < 1 ? 1 : need_ctas;
-  switch (G) {
-    case 1: scan_kernel<1><<<(int)grid, SC_GT * 1, smem, st>>>(p); break;
-    case 2: scan_kernel<2><<<(int)grid, SC_GT * 2, smem, st>>>(p); break;
-    case 3: scan_kernel<3><<<(int)grid, SC_GT * 3, smem, st>>>(p); break;
-    default: scan_kernel<4><<<(int)grid, SC_GT * 4, smem, st>>>(p); break;
-  }
+  if (tids) launch_g<true>(G, grid, smem, st, p);
+  else launch_g<false>(G, grid, smem, st, p);
   return cudaGetLastError();
 }
 

@@ -1,0 +1,61 @@
+"""Parity at BASELINE full size, in the launch configuration bench.py times:
+all 13 SSB queries at SF20 (120 M lineorder rows) through prepared CUDA-graph plans,
+element-by-element equal to the oracle (run in parallel threads: the C++ oracle
+releases the GIL).  Also TPC-H Q1/Q6 at SF30 (180 M lineitem rows)."""
+import concurrent.futures as cf
+import os
+
+import pytest
+
+import datagen
+import oracle
+
+pytestmark = [pytest.mark.gpu, pytest.mark.slow]
+
+
+def _norm(q, rows):
+    if q.startswith("ssb1") and rows == []:
+        return [(0, 0)]
+    return [tuple(r) for r in rows]
+
+
+def test_ssb_sf20_all_queries_equal_oracle():
+    from paper_conf_sigmod_bressft16_b200 import Database
+    from paper_conf_sigmod_bressft16_b200.ssb import SSB_QUERIES, load_ssb, ssb_plan
+    data = datagen.SSB(20)
+    db = Database(cache_bytes=64 << 30, heap_bytes=24 << 30)
+    load_ssb(db, data)
+    got = {}
+    for q in SSB_QUERIES:
+        p = db.prepare(ssb_plan(db, q))
+        for _ in range(2):
+            p.launch()
+        got[q] = p.fetch().rows
+        p.close()
+    db.close()
+    # the oracle reads only the columns each query needs; generate them up front
+    for c in set(sum(oracle.SSB_QUERY_COLUMNS.values(), [])):
+        data[c]
+    with cf.ThreadPoolExecutor(max_workers=min(13, os.cpu_count() or 4)) as ex:
+        want = dict(zip(SSB_QUERIES, ex.map(lambda q: oracle.run(data, q), SSB_QUERIES)))
+    for q in SSB_QUERIES:
+        assert _norm(q, got[q]) == _norm(q, want[q]), q
+
+
+def test_tpch_sf30_q1_q6_equal_oracle():
+    from paper_conf_sigmod_bressft16_b200 import Database
+    from paper_conf_sigmod_bressft16_b200.tpch import load_tpch, tpch_plan
+    data = datagen.TPCH(30)
+    db = Database(cache_bytes=64 << 30, heap_bytes=24 << 30)
+    load_tpch(db, data, tables=["lineitem"])
+    got = {}
+    for q in ("tpch1", "tpch6"):
+        p = db.prepare(tpch_plan(db, q))
+        p.launch()
+        got[q] = p.fetch().rows
+        p.close()
+    db.close()
+    with cf.ThreadPoolExecutor(max_workers=2) as ex:
+        want = dict(zip(("tpch1", "tpch6"), ex.map(lambda q: oracle.run(data, q), ("tpch1", "tpch6"))))
+    for q in got:
+        assert got[q] == [tuple(r) for r in want[q]], q
