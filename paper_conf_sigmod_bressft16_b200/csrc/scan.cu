@@ -514,7 +514,8 @@ cudaError_t launch_scan(const FilterArgs& a, cudaStream_t st) {
   const size_t list_bytes = (size_t)SC_TILE * 4 + (a.probe && !direct && a.out_payload ? (size_t)SC_TILE * 8 : 0);
   // as many groups (up to 4) and stages (up to 4, at least 2) as shared memory allows
   const int min_s = 2;
-  int G = 4, S = 4;
+  // TID mode holds 16 gathered values per thread: > 2 groups spill registers (ptxas)
+  int G = tids ? 2 : 4, S = 4;
   auto need = [&](int gg, int ss) { return shared + (size_t)gg * ((size_t)ss * p.stage_bytes + list_bytes); };
   while (G > 1 && need(G, min_s) > budget) G--;
   while (S > min_s && need(G, S) > budget) S--;
