@@ -137,6 +137,37 @@ ddq_status ddq_op_join_index_probe(const void* index, int32_t key_min, uint32_t 
                                    int32_t* out_tids, int32_t* out_payload, uint32_t* d_out_count,
                                    void* scratch, size_t scratch_bytes, void* stream);
 
+/* Star semi-join (S8(a2)+(a4) in one pass; the n-ary operator behind DDQ_OP_STAR):
+ * rows r in [0, n_rows) of a fact table survive iff every term holds -- a predicate
+ * on its column, or membership of its int32 fk column value in a join index
+ * (index != NULL: bitmap + payload over [key_min, key_min+range), see
+ * ddq_op_join_index_*) or hash table (table/capacity).  Probe terms with
+ * out_payload != NULL write the matched payload aligned with out_tids.  All term
+ * columns are streamed once (TMA); terms are evaluated in order.  Output order:
+ * ascending within 2048-row tiles, tiles in reservation order (a multiset).
+ * Columns must be 16-byte aligned and readable up to the next 16-byte boundary.
+ * *d_out_count uses 2 words (count, CTA counter); overflow of out_cap sets
+ * *d_overflow = 4 (if non-NULL). */
+enum { DDQ_TERM_PRED = 1, DDQ_TERM_PROBE = 2 };
+typedef struct {
+  int32_t kind;          /* DDQ_TERM_PRED | DDQ_TERM_PROBE */
+  int32_t width;         /* column width (4 or 8; probes: 4) */
+  const void* col;       /* streamed column */
+  int32_t pred_kind;     /* DDQ_PRED_RANGE | DDQ_PRED_IN */
+  int32_t n_in;
+  int64_t lo, hi;
+  int64_t in_vals[DDQ_MAX_IN];
+  const void* index;     /* join index, or NULL */
+  int32_t key_min;
+  uint32_t range;
+  const uint64_t* table; /* hash table when index == NULL */
+  uint32_t capacity;
+  int32_t _pad;
+  int32_t* out_payload;  /* probe payload output or NULL */
+} ddq_dev_term;
+ddq_status ddq_op_star(const ddq_dev_term* terms, int32_t n_terms, int64_t n_rows, int32_t* out_tids,
+                       uint32_t* d_out_count, int64_t out_cap, uint32_t* d_overflow, void* stream);
+
 /* Positional gather (S8(a5); P:107 materialisation): out[i] = col[tids[i]] for
  * i < *d_count; width 4 or 8. */
 ddq_status ddq_op_gather(const void* col, int32_t width, const int32_t* tids,
@@ -254,8 +285,11 @@ enum {
   DDQ_OP_HASH_PROBE = 3, /* semi-join input TIDs of `table` via fk_col against op `build` */
   DDQ_OP_GATHER = 4,     /* append vector col[tid] to the input's aligned vectors */
   DDQ_OP_AGGREGATE = 5,  /* group-by at input TIDs; root; finalised on the host */
-  DDQ_OP_FILTER_EQ = 6   /* keep input rows whose two aligned vectors are equal (TPC-H Q5's
+  DDQ_OP_FILTER_EQ = 6,  /* keep input rows whose two aligned vectors are equal (TPC-H Q5's
                             c_nationkey = s_nationkey); vectors carried */
+  DDQ_OP_STAR = 7        /* conjunction of predicates and probes over all rows of a fact
+                            table in one pass (all term columns streamed once); output as
+                            a chain of SELECT/HASH_PROBE ops would produce it */
 };
 
 typedef struct {
@@ -301,7 +335,14 @@ typedef struct {
   int32_t fk_vec;          /* HASH_PROBE: 1 + index of an aligned input vector holding the
                               probe keys (instead of fk_col); 0 = use fk_col */
   int32_t eq_vec[2];       /* FILTER_EQ: 1 + indexes of the two aligned vectors compared */
-  int32_t _pad2;
+  /* STAR (n-ary semi-join over all rows of `table`, evaluated in one pass): term j is
+     a predicate (preds[j]) or a probe of fk column term_fk[j] against HASH_BUILD op
+     term_build[j], emitting its payload as the next aligned vector if term_emit[j]. */
+  int32_t n_terms;
+  int32_t term_kind[4];    /* DDQ_TERM_PRED | DDQ_TERM_PROBE */
+  int32_t term_build[4];
+  ddq_column term_fk[4];
+  int32_t term_emit[4];
 } ddq_op;
 
 #define DDQ_MAX_OPS 32

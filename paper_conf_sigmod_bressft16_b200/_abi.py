@@ -19,7 +19,8 @@ STATUS = {0: "DDQ_OK", -1: "DDQ_EINVAL", -2: "DDQ_ENOTFOUND", -3: "DDQ_ENOMEM_HO
 
 PRED_RANGE, PRED_IN = 1, 2
 MAX_IN, MAX_PREDS, MAX_CARRY, MAX_AGGS, MAX_KEYS, MAX_OPS = 8, 4, 4, 8, 3, 32
-OP_SELECT, OP_HASH_BUILD, OP_HASH_PROBE, OP_GATHER, OP_AGGREGATE, OP_FILTER_EQ = 1, 2, 3, 4, 5, 6
+OP_SELECT, OP_HASH_BUILD, OP_HASH_PROBE, OP_GATHER, OP_AGGREGATE, OP_FILTER_EQ, OP_STAR = 1, 2, 3, 4, 5, 6, 7
+TERM_PRED, TERM_PROBE = 1, 2
 AGG_COUNT, AGG_SUM, AGG_SUM_MUL, AGG_SUM_SUB, AGG_SUM_MUL_100M, AGG_SUM_MUL_100M_100P = 1, 2, 3, 4, 5, 6
 I32, I64 = 1, 2
 PLACE_DATA_DRIVEN, PLACE_GPU_ONLY, PLACE_CPU_ONLY = 0, 1, 2
@@ -61,7 +62,17 @@ class Op(ctypes.Structure):
                 ("max_groups", ctypes.c_int64), ("n_order", ctypes.c_int32),
                 ("order_by", ctypes.c_int32 * 8), ("limit", ctypes.c_int64),
                 ("key_bits", ctypes.c_int32 * MAX_KEYS), ("fk_vec", ctypes.c_int32),
-                ("eq_vec", ctypes.c_int32 * 2), ("_pad2", ctypes.c_int32)]
+                ("eq_vec", ctypes.c_int32 * 2), ("n_terms", ctypes.c_int32),
+                ("term_kind", ctypes.c_int32 * 4), ("term_build", ctypes.c_int32 * 4),
+                ("term_fk", ctypes.c_int32 * 4), ("term_emit", ctypes.c_int32 * 4)]
+
+
+class DevTerm(ctypes.Structure):
+    _fields_ = [("kind", ctypes.c_int32), ("width", ctypes.c_int32), ("col", ctypes.c_void_p),
+                ("pred_kind", ctypes.c_int32), ("n_in", ctypes.c_int32), ("lo", ctypes.c_int64),
+                ("hi", ctypes.c_int64), ("in_vals", ctypes.c_int64 * MAX_IN), ("index", ctypes.c_void_p),
+                ("key_min", ctypes.c_int32), ("range", ctypes.c_uint32), ("table", ctypes.c_void_p),
+                ("capacity", ctypes.c_uint32), ("_pad", ctypes.c_int32), ("out_payload", ctypes.c_void_p)]
 
 
 class Plan(ctypes.Structure):
@@ -95,6 +106,7 @@ SIGNATURES = {
     "ddq_op_hash_init": (_i32, [_vp, _u32, _vp]),
     "ddq_op_hash_build": (_i32, [_vp, _vp, _vp, _vp, _i64, _vp, _u32, _vp, _vp]),
     "ddq_op_hash_probe": (_i32, [_vp, _u32, _vp, _vp, _vp, _i64, _pp, _pp, _i32, _vp, _vp, _vp, _vp, _sz, _vp]),
+    "ddq_op_star": (_i32, [ctypes.POINTER(DevTerm), _i32, _i64, _vp, _vp, _i64, _vp, _vp]),
     "ddq_op_join_index_bytes": (_sz, [_u32]),
     "ddq_op_join_index_init": (_i32, [_vp, _u32, _vp]),
     "ddq_op_join_index_build": (_i32, [_vp, _vp, _vp, _vp, _i64, _i32, _u32, _vp, _vp, _vp]),

@@ -67,6 +67,10 @@ static std::vector<int> op_columns(const ddq_op& op) {
       if (op.fk_vec <= 0) c.push_back(op.fk_col);
       break;
     case DDQ_OP_FILTER_EQ: break;
+    case DDQ_OP_STAR:
+      for (int j = 0; j < op.n_terms && j < 4; j++)
+        c.push_back(op.term_kind[j] == DDQ_TERM_PRED ? op.preds[j].column : op.term_fk[j]);
+      break;
     case DDQ_OP_GATHER: c.push_back(op.gather_col); break;
     case DDQ_OP_AGGREGATE:
       for (int k = 0; k < op.n_keys; k++)
@@ -85,6 +89,10 @@ static std::vector<int> op_children(const ddq_op& op) {
   std::vector<int> ch;
   if (op.input >= 0) ch.push_back(op.input);
   if (op.kind == DDQ_OP_HASH_PROBE && op.build >= 0 && op.build != op.input) ch.push_back(op.build);
+  if (op.kind == DDQ_OP_STAR)
+    for (int j = 0; j < op.n_terms && j < 4; j++)
+      if (op.term_kind[j] == DDQ_TERM_PROBE && std::find(ch.begin(), ch.end(), op.term_build[j]) == ch.end())
+        ch.push_back(op.term_build[j]);
   return ch;
 }
 
@@ -272,6 +280,91 @@ ddq_status run_host_op(ddq_db* db, const ddq_op& op, const std::vector<Inter>& I
     db->cols[(size_t)c]->last_access = ++db->clock;
   }
   switch (op.kind) {
+    case DDQ_OP_STAR: {  // conjunction of predicates / probes over all rows
+      struct HT {
+        const Column* col;
+        const Inter* b;
+        int lg;
+      };
+      std::vector<HT> ts;
+      int n_emit = 0;
+      for (int j = 0; j < op.n_terms; j++) {
+        HT h{nullptr, nullptr, 0};
+        if (op.term_kind[j] == DDQ_TERM_PRED) {
+          h.col = col_of(db, op.preds[j].column);
+        } else {
+          h.col = col_of(db, op.term_fk[j]);
+          h.b = &I[(size_t)op.term_build[j]];
+          if (!h.b->host_table && !h.b->h_bitmap) return set_error(DDQ_ESTATE, "host star needs host tables");
+          while (h.b->host_table && (1u << h.lg) < h.b->table_cap) h.lg++;
+          n_emit += op.term_emit[j] ? 1 : 0;
+        }
+        ts.push_back(h);
+      }
+      int nchunks = (threads <= 1 || n < (1 << 16)) ? 1 : threads;
+      std::vector<std::vector<int32_t>> sel((size_t)nchunks);
+      std::vector<std::vector<int32_t>> pay((size_t)nchunks);  // n_emit values per survivor
+      parallel_chunks(n, nchunks, [&](int t, int64_t b, int64_t e) {
+        int32_t pv[4];
+        for (int64_t r = b; r < e; r++) {
+          bool ok = true;
+          int ne = 0;
+          for (int j = 0; j < op.n_terms && ok; j++) {
+            const int64_t v = hcol(ts[(size_t)j].col, r);
+            if (op.term_kind[j] == DDQ_TERM_PRED) {
+              const ddq_pred& pr = op.preds[j];
+              if (pr.kind == DDQ_PRED_RANGE) ok = v >= pr.lo && v <= pr.hi;
+              else {
+                bool m = false;
+                for (int x = 0; x < pr.n_in; x++) m |= v == pr.in_vals[x];
+                ok = m;
+              }
+              continue;
+            }
+            const Inter& B = *ts[(size_t)j].b;
+            int32_t p = 0;
+            if (B.h_bitmap) {
+              const uint32_t o = (uint32_t)((int32_t)v - B.jmin);
+              ok = o < B.jrange && (((*B.h_bitmap)[o >> 5] >> (o & 31)) & 1u);
+              if (ok) p = (*B.h_payarr)[o];
+            } else {
+              uint32_t h = host_hash32((int32_t)v, 32 - ts[(size_t)j].lg);
+              ok = false;
+              while (true) {
+                const uint64_t s = (*B.host_table)[h];
+                if (s == kHostEmpty) break;
+                if ((int32_t)(s >> 32) == (int32_t)v) {
+                  ok = true;
+                  p = (int32_t)(uint32_t)s;
+                  break;
+                }
+                h = (h + 1) & (B.table_cap - 1);
+              }
+            }
+            if (ok && op.term_emit[j]) pv[ne++] = p;
+          }
+          if (!ok) continue;
+          sel[(size_t)t].push_back((int32_t)r);
+          for (int x = 0; x < ne; x++) pay[(size_t)t].push_back(pv[x]);
+        }
+      });
+      int64_t total = 0;
+      for (auto& s : sel) total += (int64_t)s.size();
+      out.count = out.cap = total;
+      out.tids = (int32_t*)host_alloc(out, (size_t)total * 4);
+      std::vector<int32_t*> pv;
+      for (int x = 0; x < n_emit; x++) {
+        pv.push_back((int32_t*)host_alloc(out, (size_t)total * 4));
+        out.vecs.push_back(Vec{pv.back(), 4, true});
+      }
+      int64_t o = 0;
+      for (int t = 0; t < nchunks; t++)
+        for (size_t i = 0; i < sel[(size_t)t].size(); i++, o++) {
+          out.tids[o] = sel[(size_t)t][i];
+          for (int x = 0; x < n_emit; x++) pv[(size_t)x][o] = pay[(size_t)t][i * n_emit + x];
+        }
+      return DDQ_OK;
+    }
     case DDQ_OP_SELECT:
     case DDQ_OP_FILTER_EQ:
     case DDQ_OP_HASH_PROBE: {

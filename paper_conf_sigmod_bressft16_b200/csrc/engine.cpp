@@ -284,6 +284,60 @@ ddq_status run_gpu_op(GpuOpCtx& ctx, const ddq_op& op, Inter& out) {
       fa.d_overflow = out.d_error;
       return cuda_status(launch_filter(fa, st), probe ? "probe" : "select");
     }
+    case DDQ_OP_STAR: {
+      if (in) return set_error(DDQ_EINVAL, "star: input must be all rows");
+      if (op.n_terms < 1 || op.n_terms > 4) return set_error(DDQ_EINVAL, "star: 1..4 terms");
+      ddq_dev_term terms[4];
+      std::memset(terms, 0, sizeof(terms));
+      out.cap = out_cap;
+      out.tids = (int32_t*)A.get((uint64_t)std::max<int64_t>(out_cap, 1) * 4);
+      out.d_count = (uint32_t*)A.get(64);
+      for (int j = 0; j < op.n_terms; j++) {
+        ddq_dev_term& d = terms[j];
+        d.kind = op.term_kind[j];
+        if (d.kind == DDQ_TERM_PRED) {
+          const ddq_pred& p = op.preds[j];
+          const Column* c = col_of(db, p.column);
+          if (!c || c->table != op.table) return set_error(DDQ_EINVAL, "star: predicate column not in table");
+          d.col = need_col(p.column);
+          d.width = c->width;
+          d.pred_kind = p.kind;
+          d.lo = p.lo;
+          d.hi = p.hi;
+          d.n_in = p.n_in;
+          for (int i = 0; i < DDQ_MAX_IN; i++) d.in_vals[i] = p.in_vals[i];
+        } else if (d.kind == DDQ_TERM_PROBE) {
+          const int b = op.term_build[j];
+          if (b < 0 || b >= (int)I.size()) return set_error(DDQ_EINVAL, "star: bad build index");
+          const Inter& B = I[(size_t)b];
+          if (!B.table_ptr && !B.jidx) return set_error(DDQ_ESTATE, "star: build side is not on the device");
+          const Column* c = col_of(db, op.term_fk[j]);
+          if (!c || c->table != op.table || c->width != 4) return set_error(DDQ_EINVAL, "star: bad fk column");
+          d.col = need_col(op.term_fk[j]);
+          d.width = 4;
+          if (B.jidx) {
+            d.index = B.jidx;
+            d.key_min = B.jmin;
+            d.range = B.jrange;
+          } else {
+            d.table = B.table_ptr;
+            d.capacity = B.table_cap;
+          }
+          if (op.term_emit[j]) {
+            d.out_payload = (int32_t*)A.get((uint64_t)std::max<int64_t>(out_cap, 1) * 4);
+            out.vecs.push_back(Vec{d.out_payload, 4, false});
+          }
+        } else {
+          return set_error(DDQ_EINVAL, "star: bad term kind");
+        }
+        if (!d.col) return set_error(DDQ_ESTATE, "star: column not cached on the GPU");
+      }
+      out.d_error = (uint32_t*)A.get(64);
+      if (A.failed) return DDQ_ENOMEM_DEVICE;
+      cudaMemsetAsync(out.d_error, 0, 4, st);
+      return cuda_status(launch_star(terms, op.n_terms, T.n_rows, out.tids, out.d_count, out_cap, out.d_error, st),
+                         "star");
+    }
     case DDQ_OP_HASH_BUILD: {
       const Column* kc = col_of(db, op.key_col);
       if (!kc || kc->table != op.table || kc->width != 4) return set_error(DDQ_EINVAL, "build: bad key column");
@@ -818,7 +872,15 @@ static ddq_status validate_plan(ddq_db* db, const ddq_plan* plan) {
   if (!plan || plan->n_ops < 1 || plan->n_ops > DDQ_MAX_OPS) return set_error(DDQ_EINVAL, "plan: bad op count");
   for (int i = 0; i < plan->n_ops; i++) {
     const ddq_op& op = plan->ops[i];
-    if (op.kind < DDQ_OP_SELECT || op.kind > DDQ_OP_FILTER_EQ) return set_error(DDQ_EINVAL, "plan: bad op kind");
+    if (op.kind < DDQ_OP_SELECT || op.kind > DDQ_OP_STAR) return set_error(DDQ_EINVAL, "plan: bad op kind");
+    if (op.kind == DDQ_OP_STAR) {
+      if (op.input >= 0) return set_error(DDQ_EINVAL, "plan: a STAR op scans all rows");
+      if (op.n_terms < 1 || op.n_terms > 4) return set_error(DDQ_EINVAL, "plan: STAR needs 1..4 terms");
+      for (int j = 0; j < op.n_terms; j++)
+        if (op.term_kind[j] == DDQ_TERM_PROBE &&
+            (op.term_build[j] < 0 || op.term_build[j] >= i || plan->ops[op.term_build[j]].kind != DDQ_OP_HASH_BUILD))
+          return set_error(DDQ_EINVAL, "plan: STAR probe must reference an earlier HASH_BUILD");
+    }
     if (op.kind == DDQ_OP_FILTER_EQ && op.input < 0) return set_error(DDQ_EINVAL, "plan: filter_eq needs an input");
     if (op.kind == DDQ_OP_HASH_PROBE && op.fk_vec > 0 && op.input < 0)
       return set_error(DDQ_EINVAL, "plan: a vector-keyed probe needs an input");
@@ -853,6 +915,7 @@ static int kernels_of(const ddq_op& op) {
     case DDQ_OP_GATHER: return 1;
     case DDQ_OP_AGGREGATE: return 3;
     case DDQ_OP_FILTER_EQ: return 1;
+    case DDQ_OP_STAR: return 1;
   }
   return 0;
 }
@@ -889,6 +952,9 @@ void count_accesses(ddq_db* db, const ddq_op& op) {
     case DDQ_OP_HASH_BUILD: touch(op.key_col); touch(op.payload_col); break;
     case DDQ_OP_HASH_PROBE: touch(op.fk_col); break;
     case DDQ_OP_GATHER: touch(op.gather_col); break;
+    case DDQ_OP_STAR:
+      for (int j = 0; j < op.n_terms; j++) touch(op.term_kind[j] == DDQ_TERM_PRED ? op.preds[j].column : op.term_fk[j]);
+      break;
     case DDQ_OP_AGGREGATE:
       for (int k = 0; k < op.n_keys; k++)
         if (op.key_src[k] < -1) touch(-2 - op.key_src[k]);
@@ -966,7 +1032,8 @@ ddq_status ddq_prepare(ddq_db* db, const ddq_plan* plan, int32_t use_graph, ddq_
   for (int i = 0; i < plan->n_ops; i++) {
     const ddq_op& op = plan->ops[i];
     if (op.kind == DDQ_OP_HASH_BUILD && op.input >= 0) P->forced[(size_t)i] = counts[(size_t)op.input];
-    if (op.kind == DDQ_OP_SELECT || op.kind == DDQ_OP_HASH_PROBE)
+    if (op.kind == DDQ_OP_SELECT || op.kind == DDQ_OP_HASH_PROBE || op.kind == DDQ_OP_STAR ||
+        op.kind == DDQ_OP_FILTER_EQ)
       P->forced[(size_t)i] = counts[(size_t)i] + counts[(size_t)i] / 64 + 256;
   }
   P->inters.resize((size_t)plan->n_ops);
@@ -1081,6 +1148,15 @@ int32_t ddq_prepared_profile(ddq_prepared* p, void* stream, int32_t max_ops, flo
           bytes += out * 4 * nvec_in;  // carried vectors read at survivors
         }
         bytes += out * 4 * (1 + nvec_in + emit);
+      } break;
+      case DDQ_OP_STAR: {
+        cls = 0;
+        int emit = 0;
+        for (int j = 0; j < op.n_terms; j++) {
+          bytes += N * (op.term_kind[j] == DDQ_TERM_PRED ? width(op.preds[j].column) : 4);
+          emit += op.term_kind[j] == DDQ_TERM_PROBE && op.term_emit[j] ? 1 : 0;
+        }
+        bytes += out * 4 * (1 + emit);
       } break;
       case DDQ_OP_FILTER_EQ:
         cls = 1;

@@ -184,18 +184,36 @@ __device__ __forceinline__ long long agg_value(const GroupbyParams& P, int a, in
   return x * (100 - y) * (100 + z);  // DDQ_AGG_SUM_MUL_100M_100P
 }
 
-// Sum of x over the lanes of `peers`; the total lands in the lowest peer lane.
-__device__ __forceinline__ long long peer_reduce(unsigned peers, long long x, int lane) {
+// Exact int128 sum (lo, hi) of x over the lanes of `peers` (log-step peer
+// reduction: each round a lane adds the value of its next remaining peer and the
+// odd-ranked lanes retire); the total lands in the lowest peer lane.
+__device__ __forceinline__ void peer_reduce128(unsigned peers, long long x, int lane, unsigned long long& lo,
+                                               long long& hi) {
+  lo = (unsigned long long)x;
+  hi = x < 0 ? -1 : 0;
   unsigned rest = peers & (0xfffffffeu << lane);
   unsigned rank = __popc(peers & ((1u << lane) - 1u));
   while (__any_sync(FULL, rest != 0)) {
     const int next = __ffs(rest);
-    const long long t = __shfl_sync(FULL, x, next ? next - 1 : lane);
-    if (next) x += t;
+    const int src = next ? next - 1 : lane;
+    const unsigned long long tlo = __shfl_sync(FULL, lo, src);
+    const long long thi = __shfl_sync(FULL, hi, src);
+    if (next) {
+      const unsigned long long s = lo + tlo;
+      hi += thi + (s < lo ? 1 : 0);
+      lo = s;
+    }
     rest &= ~__ballot_sync(FULL, rank & 1u);
     rank >>= 1;
   }
-  return x;
+}
+
+// exact int128 accumulation of an int128 (lo, hi) addend
+__device__ __forceinline__ void atomic_add_i128_pair(unsigned long long* plo, unsigned long long* phi,
+                                                     unsigned long long lo, long long hi) {
+  const unsigned long long old = atomicAdd(plo, lo);
+  const long long h = hi + ((old + lo < old) ? 1 : 0);
+  if (h) atomicAdd(phi, (unsigned long long)h);
 }
 
 // find-or-insert `key` into an open-addressing table of int64 keys; -1 if full
@@ -252,14 +270,16 @@ __global__ void __launch_bounds__(GB_THREADS) groupby_kernel(const __grid_consta
       }
     }
     for (int a = 0; a < P.n_aggs; a++) {
-      long long v = valid ? agg_value(P, a, r) : 0;
-      v = peer_reduce(peers, v, lane);
+      const long long v = valid ? agg_value(P, a, r) : 0;
+      unsigned long long lo;
+      long long hi;
+      peer_reduce128(peers, v, lane, lo, hi);  // exact: 32 int64 values can exceed int64
       if (valid && leader && slot >= 0) {
         if (!global)
-          atomic_add_i128(&s_accs[((size_t)a * S + slot) * 2], &s_accs[((size_t)a * S + slot) * 2 + 1], v);
+          atomic_add_i128_pair(&s_accs[((size_t)a * S + slot) * 2], &s_accs[((size_t)a * S + slot) * 2 + 1], lo, hi);
         else
-          atomic_add_i128(&P.g_accs[((size_t)a * (P.cap_mask + 1) + slot) * 2],
-                          &P.g_accs[((size_t)a * (P.cap_mask + 1) + slot) * 2 + 1], v);
+          atomic_add_i128_pair(&P.g_accs[((size_t)a * (P.cap_mask + 1) + slot) * 2],
+                               &P.g_accs[((size_t)a * (P.cap_mask + 1) + slot) * 2 + 1], lo, hi);
       }
     }
   }

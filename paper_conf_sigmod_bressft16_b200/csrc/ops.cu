@@ -112,6 +112,30 @@ ddq_status ddq_op_hash_probe(const uint64_t* table, uint32_t capacity, const int
   return cuda_status(launch_filter(a, (cudaStream_t)stream), "ddq_op_hash_probe");
 }
 
+ddq_status ddq_op_star(const ddq_dev_term* terms, int32_t n_terms, int64_t n_rows, int32_t* out_tids,
+                       uint32_t* d_out_count, int64_t out_cap, uint32_t* d_overflow, void* stream) {
+  if (ddq_status s = check_cap(n_rows)) return s;
+  if (!terms || n_terms < 1 || n_terms > 4) return set_error(DDQ_EINVAL, "star: 1..4 terms");
+  if (!out_tids || !d_out_count) return set_error(DDQ_EINVAL, "star: null output");
+  for (int j = 0; j < n_terms; j++) {
+    const ddq_dev_term& t = terms[j];
+    if (t.kind != DDQ_TERM_PRED && t.kind != DDQ_TERM_PROBE) return set_error(DDQ_EINVAL, "star: bad term kind");
+    if ((n_rows > 0 && !t.col) || ((uintptr_t)t.col & 15)) return set_error(DDQ_EINVAL, "star: column must be 16-byte aligned");
+    if (t.width != 4 && t.width != 8) return set_error(DDQ_EINVAL, "star: bad width");
+    if (t.kind == DDQ_TERM_PRED) {
+      if (t.pred_kind != DDQ_PRED_RANGE && t.pred_kind != DDQ_PRED_IN) return set_error(DDQ_EINVAL, "star: bad predicate");
+      if (t.pred_kind == DDQ_PRED_IN && (t.n_in < 0 || t.n_in > DDQ_MAX_IN)) return set_error(DDQ_EINVAL, "star: IN list too long");
+    } else {
+      if (t.width != 4) return set_error(DDQ_EINVAL, "star: probe keys are int32");
+      if (!t.index && (!t.table || t.capacity < 2 || (t.capacity & (t.capacity - 1))))
+        return set_error(DDQ_EINVAL, "star: probe needs a join index or a hash table");
+      if (t.index && t.range == 0) return set_error(DDQ_EINVAL, "star: empty join index range");
+    }
+  }
+  return cuda_status(launch_star(terms, n_terms, n_rows, out_tids, d_out_count, out_cap, d_overflow, (cudaStream_t)stream),
+                     "ddq_op_star");
+}
+
 size_t ddq_op_join_index_bytes(uint32_t range) { return join_index_bytes(range); }
 
 ddq_status ddq_op_join_index_init(void* index, uint32_t range, void* stream) {

@@ -48,6 +48,9 @@ cudaError_t launch_hash_init(uint64_t* table, uint32_t capacity, cudaStream_t st
 cudaError_t launch_hash_build(const int32_t* keys, const int32_t* payload, const int32_t* in_tids,
                               const uint32_t* d_in_count, int64_t n_cap, uint64_t* table, uint32_t capacity,
                               uint32_t* d_error, cudaStream_t st);
+cudaError_t launch_star(const ddq_dev_term* terms, int n_terms, int64_t n_rows, int32_t* out_tids,
+                        uint32_t* d_out_count, int64_t out_cap, uint32_t* d_overflow, cudaStream_t st);
+
 size_t join_index_bytes(uint32_t range);
 inline uint32_t* join_index_bitmap(void* idx) { return reinterpret_cast<uint32_t*>(idx); }
 inline int32_t* join_index_payload(void* idx, uint32_t range) {

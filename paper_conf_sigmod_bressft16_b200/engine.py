@@ -111,6 +111,36 @@ class PlanBuilder:
         op.emit_payload = 1 if emit else 0
         return idx
 
+    def star(self, table: str, terms: list) -> int:
+        """n-ary semi-join over all rows of `table` in one pass.  terms (evaluated in
+        order, most selective first): ("pred", (col, lo, hi)) | ("pred", (col, [vals]))
+        | ("probe", fk_col, build_op, emit).  Emitted payloads become aligned vectors
+        in term order -- the same output as the equivalent SELECT/HASH_PROBE chain."""
+        idx, op = self._op(A.OP_STAR, table, -1)
+        if not 1 <= len(terms) <= 4:
+            raise ValueError("STAR takes 1..4 terms")
+        op.n_terms = len(terms)
+        for j, term in enumerate(terms):
+            if term[0] == "pred":
+                p = term[1]
+                pr = op.preds[j]
+                pr.column = self.db.col(table, p[0])
+                if len(p) == 3:
+                    pr.kind, pr.lo, pr.hi = A.PRED_RANGE, int(p[1]), int(p[2])
+                else:
+                    pr.kind, pr.n_in = A.PRED_IN, len(p[1])
+                    for i, v in enumerate(p[1]):
+                        pr.in_vals[i] = int(v)
+                op.term_kind[j] = A.TERM_PRED
+            else:
+                _, fk, build, emit = term
+                op.term_kind[j] = A.TERM_PROBE
+                op.term_fk[j] = self.db.col(table, fk)
+                op.term_build[j] = build
+                op.term_emit[j] = 1 if emit else 0
+        op.n_preds = 0
+        return idx
+
     def filter_eq(self, table: str, input: int, vec_a: int, vec_b: int) -> int:
         """Keep rows whose aligned vectors vec_a and vec_b are equal."""
         idx, op = self._op(A.OP_FILTER_EQ, table, input)

@@ -233,6 +233,27 @@ def test_groupby_exact(ops, ngroups, n):
             assert got[pos[kk], a] == vv, (a, kk)
 
 
+@pytest.mark.parametrize("nkeys", [0, 1])
+def test_groupby_few_groups_int128_exact(ops, nkeys):
+    """Register-accumulating few-group kernel: per-thread int64 partial sums that
+    would overflow must spill exactly into the int128 table."""
+    from paper_conf_sigmod_bressft16_b200 import _abi as A
+    rng = np.random.default_rng(9)
+    n = 300_000
+    big = rng.integers(2**60, 2**62, n, dtype=np.int64) * rng.choice([-1, 1], n)
+    tids = np.arange(n, dtype=np.int32)
+    k = rng.integers(0, 3, n, dtype=np.int32)
+    keys, accs, err = ops.groupby(_t(tids), ops.count_cell(n), n, key_vecs=[_t(k)] if nkeys else [],
+                                  aggs=[(A.AGG_SUM, [_t(big)]), (A.AGG_COUNT, [])], capacity=64)
+    assert err == 0
+    got = _acc_to_int(accs)
+    keys = keys.cpu().numpy()
+    for i, kk in enumerate(keys):
+        m = (k == kk) if nkeys else np.ones(n, bool)
+        assert got[i, 0] == sum(int(x) for x in big[m])
+        assert got[i, 1] == int(m.sum())
+
+
 def test_groupby_overflow_flagged(ops):
     from paper_conf_sigmod_bressft16_b200 import _abi as A
     n = 10_000

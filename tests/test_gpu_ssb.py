@@ -50,12 +50,13 @@ def _oracle(kind, q):
     return norm(q, oracle.run(_data(kind), q))
 
 
+@pytest.mark.parametrize("star", [True, False], ids=["star", "chain"])
 @pytest.mark.parametrize("kind", ["1", "planted", "0.01"])
 @pytest.mark.parametrize("q", oracle.SSB_QUERIES)
-def test_ssb_prepared_graph_equals_oracle(kind, q):
+def test_ssb_prepared_graph_equals_oracle(kind, q, star):
     from paper_conf_sigmod_bressft16_b200.ssb import ssb_plan
     db = _db(kind)
-    p = db.prepare(ssb_plan(db, q), use_graph=True)
+    p = db.prepare(ssb_plan(db, q, star=star), use_graph=True)
     want = _oracle(kind, q)
     for _ in range(2):  # relaunch of the same graph is deterministic
         p.launch()
@@ -64,12 +65,13 @@ def test_ssb_prepared_graph_equals_oracle(kind, q):
     p.close()
 
 
+@pytest.mark.parametrize("star", [True, False], ids=["star", "chain"])
 @pytest.mark.parametrize("kind", ["1", "planted"])
 @pytest.mark.parametrize("q", oracle.SSB_QUERIES)
-def test_ssb_submit_chopping_equals_oracle(kind, q):
+def test_ssb_submit_chopping_equals_oracle(kind, q, star):
     from paper_conf_sigmod_bressft16_b200.ssb import ssb_plan
     db = _db(kind)
-    r = db.run(ssb_plan(db, q))
+    r = db.run(ssb_plan(db, q, star=star))
     assert norm(q, r.rows) == _oracle(kind, q)
     assert r.host_ops == 0 and r.aborts == 0  # hot cache: everything on the GPU
 
