@@ -15,13 +15,14 @@
 //   * full tiles need no row-bound checks; survivors are compacted with a packed
 //     warp scan, staged in smem and copied out coalesced, survivors only;
 //   * the output range of a 4096-item tile is reserved with ONE atomicAdd whose
-//     latency is hidden: tile k is copied out in iteration k+1 (double-buffered
-//     lists).  Items stay in input order within a tile; tiles appear in reservation
+//     latency is hidden: tile k is copied out in iteration k+1 (the survivor list is
+//     staged after barrier (B)).  Items stay in input order within a tile; tiles appear in reservation
 //     order (reading O14': a TID list is a multiset; aggregates are exact integer
 //     sums, so query results are bit-identical whatever the order);
 //   * compact-range dimension keys use a direct-mapped join index (membership
 //     bitmap + payload array): one lookup per row, no collision chains.
 #include <cstdint>
+#include <cstdlib>
 #include <cuda_runtime.h>
 
 #include "device_common.cuh"
@@ -44,6 +45,23 @@ struct ScanPred {
   int64_t lo, hi;
   int32_t n_in, _pad;
   int64_t in_vals[8];
+  // RANGE, precomputed on the host: lo <= v <= hi  <=>  (unsigned)(v - lo) <= d
+  // (one subtract + one compare per value); `empty` when no int32 value qualifies
+  int32_t lo32;
+  uint32_t d32;
+  uint64_t d64;
+  int32_t empty32, empty64;
+};
+
+// Kernel variants: the predicate / probe code is specialised at compile time so a
+// tile costs only the instructions its operator needs (ncu: the generic path was
+// issue-bound -- math-pipe throttle + not-selected stalls).
+// The *_R probe variants stream the key column through registers (coalesced 16-byte
+// loads one tile ahead) instead of the TMA ring: no ring in shared memory, so a
+// large smem bitmap / table leaves room for 4 groups.
+enum ScanMode : int {
+  SM_SEL_GENERIC = 0, SM_SEL_RANGE = 1, SM_PROBE_DIRECT = 2, SM_PROBE_HASH = 3, SM_PROBE_DIRECT_R = 4,
+  SM_PROBE_HASH_R = 5
 };
 
 struct ScanParams {
@@ -78,6 +96,8 @@ struct ScanParams {
   uint32_t range;
   uint32_t bitmap_words;
   int32_t bitmap_in_smem;
+  int32_t payarr_in_smem;  // payload array staged after the bitmap (at payarr_off)
+  int32_t payarr_off;
   int32_t* out_payload;
   // carried vectors (TID mode)
   int32_t n_carry;
@@ -143,21 +163,36 @@ __device__ __forceinline__ bool scan_pred(const ScanPred& p, int64_t v) {
   return m;
 }
 
-// Membership (+ lookup) of 16 keys; clears the flag bits of misses.
-template <bool kHashPayload>
+// Membership (+ payload lookup) of 16 keys; clears the flag bits of misses.  Payloads
+// are loaded for hits only, right after the probe, so their latency overlaps the
+// survivor scan and barrier (they are staged in smem with the survivor list).
+template <int kMode, bool kPay>
 __device__ __forceinline__ void probe16(const ScanParams& P, const uint64_t* table, const uint32_t* bm,
-                                        const int32_t (&key)[SC_ITEMS], uint32_t& flags,
-                                        int32_t (&payload)[SC_ITEMS]) {
-  if (P.direct) {
+                                        const int32_t* pa, bool bm_padded, const int32_t (&key)[SC_ITEMS],
+                                        uint32_t& flags, int32_t (&payload)[SC_ITEMS]) {
+  if (kMode == SM_PROBE_DIRECT) {
     uint32_t m = 0;
+    if (bm_padded) {  // smem bitmap with a zero word past its end: clamp instead of test
 #pragma unroll
-    for (int k = 0; k < SC_ITEMS; k++) {
-      const uint32_t o = (uint32_t)(key[k] - P.key_min);
-      const uint32_t oo = o < P.range ? o : 0u;
-      const uint32_t w = bm[oo >> 5];
-      m |= ((o < P.range ? (w >> (oo & 31)) : 0u) & 1u) << k;
+      for (int k = 0; k < SC_ITEMS; k++) {
+        const uint32_t oo = min((uint32_t)(key[k] - P.key_min), P.range);
+        m |= ((bm[oo >> 5] >> (oo & 31)) & 1u) << k;
+      }
+    } else {
+#pragma unroll
+      for (int k = 0; k < SC_ITEMS; k++) {
+        const uint32_t o = (uint32_t)(key[k] - P.key_min);
+        const uint32_t oo = o < P.range ? o : 0u;
+        const uint32_t w = bm[oo >> 5];
+        m |= ((o < P.range ? (w >> (oo & 31)) : 0u) & 1u) << k;
+      }
     }
-    flags &= m;  // payloads: fetched for survivors only, at copy-out
+    flags &= m;
+    if (kPay) {
+#pragma unroll
+      for (int k = 0; k < SC_ITEMS; k++)
+        payload[k] = ((flags >> k) & 1u) ? pa[(uint32_t)(key[k] - P.key_min)] : 0;
+    }
   } else {
     uint32_t h[SC_ITEMS];
     uint64_t sl[SC_ITEMS];
@@ -175,13 +210,92 @@ __device__ __forceinline__ void probe16(const ScanParams& P, const uint64_t* tab
         s = table[hh];
       }
       if (s == HT_EMPTY) flags &= ~(1u << k);
-      if (kHashPayload) payload[k] = ht_val(s);
+      if (kPay) payload[k] = ht_val(s);
     }
   }
 }
 
-template <int G, bool kTids>
+// Gathered values (TID mode) against predicate p.
+template <int kMode>
+__device__ __forceinline__ void pred16_gathered(const ScanPred& pr, const int32_t (&row)[SC_ITEMS], uint32_t& flags) {
+  int64_t v[SC_ITEMS];
+#pragma unroll
+  for (int k = 0; k < SC_ITEMS; k++) v[k] = ((flags >> k) & 1u) ? col_at(pr.col, pr.width, row[k]) : 0;
+  if (kMode == SM_SEL_RANGE) {
+    if (pr.empty64) flags = 0;
+#pragma unroll
+    for (int k = 0; k < SC_ITEMS; k++)
+      if ((uint64_t)(v[k] - pr.lo) > pr.d64) flags &= ~(1u << k);
+  } else {
+    uint32_t m = 0;
+#pragma unroll
+    for (int k = 0; k < SC_ITEMS; k++) m |= (scan_pred(pr, v[k]) ? 1u : 0u) << k;
+    flags &= m;
+  }
+}
+
+// Staged (dense) column chunk against predicate p.
+template <int kMode>
+__device__ __forceinline__ void pred16_staged(const ScanPred& pr, const uint8_t* cb, int wrow, int lane,
+                                              uint32_t& flags) {
+#pragma unroll
+  for (int s = 0; s < SC_SLOTS; s++) {
+    const int it = wrow + s * 128 + lane * 4;
+    if (kMode == SM_SEL_RANGE && pr.width == 4) {
+      const int4 a = *reinterpret_cast<const int4*>(cb + (size_t)it * 4);
+      const int32_t v4[4] = {a.x, a.y, a.z, a.w};
+#pragma unroll
+      for (int v = 0; v < 4; v++)
+        if ((uint32_t)(v4[v] - pr.lo32) > pr.d32) flags &= ~(1u << (s * 4 + v));
+      continue;
+    }
+    int64_t v4[4];
+    if (pr.width == 8) {
+      const longlong2 a = *reinterpret_cast<const longlong2*>(cb + (size_t)it * 8);
+      const longlong2 b = *reinterpret_cast<const longlong2*>(cb + (size_t)it * 8 + 16);
+      v4[0] = a.x; v4[1] = a.y; v4[2] = b.x; v4[3] = b.y;
+    } else {
+      const int4 a = *reinterpret_cast<const int4*>(cb + (size_t)it * 4);
+      v4[0] = a.x; v4[1] = a.y; v4[2] = a.z; v4[3] = a.w;
+    }
+    if (kMode == SM_SEL_RANGE) {
+#pragma unroll
+      for (int v = 0; v < 4; v++)
+        if ((uint64_t)(v4[v] - pr.lo) > pr.d64) flags &= ~(1u << (s * 4 + v));
+    } else {
+      uint32_t m = 0;
+#pragma unroll
+      for (int v = 0; v < 4; v++) m |= (scan_pred(pr, v4[v]) ? 1u : 0u) << v;
+      flags &= ~((~m & 0xFu) << (s * 4));
+    }
+  }
+}
+
+// One tile's keys (dense probe, register-streamed): 4 x 16-byte loads per thread.
+__device__ __forceinline__ void load_keys(const int32_t* fk, uint32_t n, uint32_t row0, uint32_t wrow, int lane,
+                                          int4 (&r)[SC_SLOTS]) {
+  if (row0 + SC_TILE <= n) {
+#pragma unroll
+    for (int s = 0; s < SC_SLOTS; s++) r[s] = ld_stream_i4(fk + (size_t)row0 + wrow + s * 128 + lane * 4);
+  } else {
+#pragma unroll
+    for (int s = 0; s < SC_SLOTS; s++) {
+      const uint32_t i = row0 + wrow + s * 128 + lane * 4;
+      r[s].x = i < n ? fk[i] : 0;
+      r[s].y = i + 1 < n ? fk[i + 1] : 0;
+      r[s].z = i + 2 < n ? fk[i + 2] : 0;
+      r[s].w = i + 3 < n ? fk[i + 3] : 0;
+    }
+  }
+}
+
+template <int G, bool kTids, int kMode>
 __global__ void __launch_bounds__(SC_GT* G, 1) scan_kernel(const __grid_constant__ ScanParams P) {
+  constexpr bool kProbe = kMode >= SM_PROBE_DIRECT;
+  constexpr bool kDirect = kMode == SM_PROBE_DIRECT || kMode == SM_PROBE_DIRECT_R;
+  constexpr bool kHash = kProbe && !kDirect;
+  constexpr bool kReg = kMode >= SM_PROBE_DIRECT_R;  // dense only
+  constexpr int kPM = kDirect ? SM_PROBE_DIRECT : SM_PROBE_HASH;
   extern __shared__ __align__(128) uint8_t smem[];
   __shared__ uint32_t s_warp_tot[SC_MAXG][SC_GW];
   __shared__ uint32_t s_base[SC_MAXG];
@@ -198,11 +312,14 @@ __global__ void __launch_bounds__(SC_GT* G, 1) scan_kernel(const __grid_constant
   const int ahead = S - 1;
   const uint32_t vb = blockIdx.x * G + g, vgrid = gridDim.x * G;  // virtual CTA id / count
   uint8_t* ring = smem + (size_t)g * P.group_bytes;
-  uint16_t* s_list = reinterpret_cast<uint16_t*>(ring + P.list_off);              // 2 x TILE
-  int32_t* s_pay = reinterpret_cast<int32_t*>(ring + P.list_off + SC_TILE * 4);   // 2 x TILE
+  uint16_t* s_list = reinterpret_cast<uint16_t*>(ring + P.list_off);             // TILE
+  int32_t* s_pay = reinterpret_cast<int32_t*>(ring + P.list_off + SC_TILE * 2);  // TILE
   uint64_t* s_table = reinterpret_cast<uint64_t*>(smem + P.shared_off);
 
-  if (t == 0) {  // group leader: barriers, then the first tiles in flight
+  const uint32_t wrow = warp * (32 * SC_ITEMS);  // warp's first item inside a tile
+  int4 nk[SC_SLOTS];                             // register-streamed keys of the next tile
+  if (kReg && vb < ntiles) load_keys(P.fk, n, vb * SC_TILE, wrow, lane, nk);
+  if (t == 0 && !kReg) {  // group leader: barriers, then the first tiles in flight
     for (int k = 0; k < S; k++) mbar_init(&s_full[g][k], 1);
     fence_mbar_init();
     for (int k = 0; k < ahead; k++) {
@@ -210,23 +327,30 @@ __global__ void __launch_bounds__(SC_GT* G, 1) scan_kernel(const __grid_constant
       if (tl < ntiles) issue_tile(P, n, ring + (size_t)k * P.stage_bytes, &s_full[g][k], tl);
     }
   }
-  // all groups stage the shared table / bitmap once per SM (overlaps the first loads)
-  if (P.probe && P.table_in_smem)
-    for (uint32_t i = threadIdx.x; i <= P.cap_mask; i += SC_GT * G) s_table[i] = P.table[i];
+  // all groups stage the shared table / bitmap (+ payload array) once per SM
+  // (overlaps the first loads); the smem bitmap gets one zero word past its end
   uint32_t* s_bm = reinterpret_cast<uint32_t*>(s_table);
-  if (P.probe && P.direct && P.bitmap_in_smem)
-    for (uint32_t i = threadIdx.x; i < P.bitmap_words; i += SC_GT * G) s_bm[i] = P.bitmap[i];
-  const uint64_t* table = (P.probe && P.table_in_smem) ? s_table : P.table;
-  const uint32_t* bm = (P.probe && P.direct && P.bitmap_in_smem) ? s_bm : P.bitmap;
-  const bool want_pay = P.probe && P.out_payload != nullptr;
-  const bool hash_pay = want_pay && !P.direct;  // hash probes stage payloads in smem
+  int32_t* s_pa = reinterpret_cast<int32_t*>(smem + P.shared_off + P.payarr_off);
+  if (kHash && P.table_in_smem)
+    for (uint32_t i = threadIdx.x; i <= P.cap_mask; i += SC_GT * G) s_table[i] = P.table[i];
+  if (kDirect && P.bitmap_in_smem) {
+    for (uint32_t i = threadIdx.x; i <= P.bitmap_words; i += SC_GT * G)
+      s_bm[i] = i < P.bitmap_words ? P.bitmap[i] : 0u;
+    if (P.payarr_in_smem)
+      for (uint32_t i = threadIdx.x; i < P.range; i += SC_GT * G) s_pa[i] = P.payarr[i];
+  }
+  const uint64_t* table = (kHash && P.table_in_smem) ? s_table : P.table;
+  const uint32_t* bm = (kDirect && P.bitmap_in_smem) ? s_bm : P.bitmap;
+  const int32_t* pa = (kDirect && P.payarr_in_smem) ? s_pa : P.payarr;
+  const bool bm_padded = P.bitmap_in_smem != 0;
+  const bool want_pay = kProbe && P.out_payload != nullptr;  // payloads staged with the list
   __syncthreads();
 
-  // Software pipeline over the group's tiles: iteration k evaluates tile k and
-  // stages its survivors in list[k&1] while its output reservation (one atomic) is
-  // in flight; it copies out tile k-1, whose range was reserved last iteration.
+  // Software pipeline over the group's tiles: iteration k evaluates tile k, then
+  // (while its output reservation -- one atomic -- is in flight) copies out tile
+  // k-1, whose range was reserved last iteration, from the survivor list; after (B)
+  // it stages tile k's survivors in that list (one buffer: half the smem of two).
   uint32_t prev_tot = 0, prev_base = 0;
-  const uint32_t wrow = warp * (32 * SC_ITEMS);  // warp's first item inside a tile
   for (uint32_t k = 0;; k++) {
     const uint32_t tile = vb + k * vgrid;
     const bool have = tile < ntiles;
@@ -234,7 +358,7 @@ __global__ void __launch_bounds__(SC_GT* G, 1) scan_kernel(const __grid_constant
     uint32_t flags = 0;
     int32_t payload[SC_ITEMS];
     if (have) {
-      mbar_wait(&s_full[g][k % S], (k / S) & 1u);
+      if (!kReg) mbar_wait(&s_full[g][k % S], (k / S) & 1u);
       const uint8_t* buf = ring + (size_t)(k % S) * P.stage_bytes;
       flags = 0xFFFFu;
       if (row0 + SC_TILE > n) {  // tail tile only
@@ -253,17 +377,8 @@ __global__ void __launch_bounds__(SC_GT* G, 1) scan_kernel(const __grid_constant
           const int4 a = *reinterpret_cast<const int4*>(buf + (size_t)(wrow + s * 128 + lane * 4) * 4);
           row[s * 4 + 0] = a.x; row[s * 4 + 1] = a.y; row[s * 4 + 2] = a.z; row[s * 4 + 3] = a.w;
         }
-        if (!P.probe) {
-          for (int p = 0; p < P.n_preds; p++) {
-            const ScanPred& pr = P.preds[p];
-            int64_t v[SC_ITEMS];
-#pragma unroll
-            for (int k2 = 0; k2 < SC_ITEMS; k2++) v[k2] = ((flags >> k2) & 1u) ? col_at(pr.col, pr.width, row[k2]) : 0;
-            uint32_t m = 0;
-#pragma unroll
-            for (int k2 = 0; k2 < SC_ITEMS; k2++) m |= (scan_pred(pr, v[k2]) ? 1u : 0u) << k2;
-            flags &= m;
-          }
+        if (!kProbe) {
+          for (int p = 0; p < P.n_preds; p++) pred16_gathered<kMode>(P.preds[p], row, flags);
           if (P.eq_a) {
             uint32_t m = 0;
 #pragma unroll
@@ -280,42 +395,27 @@ __global__ void __launch_bounds__(SC_GT* G, 1) scan_kernel(const __grid_constant
             const uint32_t pos = row0 + wrow + (k2 >> 2) * 128 + lane * 4 + (k2 & 3);
             key[k2] = ((flags >> k2) & 1u) ? __ldg(P.fk + (P.fk_by_pos ? (int64_t)pos : (int64_t)row[k2])) : 0;
           }
-          if (hash_pay) probe16<true>(P, table, bm, key, flags, payload);
-          else probe16<false>(P, table, bm, key, flags, payload);
+          if (want_pay) probe16<kPM, true>(P, table, bm, pa, bm_padded, key, flags, payload);
+          else probe16<kPM, false>(P, table, bm, pa, bm_padded, key, flags, payload);
         }
-      } else if (!P.probe) {
+      } else if (!kProbe) {
         // ---- dense select: values from the staged columns ----------------------
         for (int p = 0; p < P.n_preds; p++) {
           const ScanPred& pr = P.preds[p];
-          const uint8_t* cb = buf + P.col_off[p];
-#pragma unroll
-          for (int s = 0; s < SC_SLOTS; s++) {
-            const int it = wrow + s * 128 + lane * 4;
-            int64_t v4[4];
-            if (pr.width == 8) {
-              const longlong2 a = *reinterpret_cast<const longlong2*>(cb + (size_t)it * 8);
-              const longlong2 b = *reinterpret_cast<const longlong2*>(cb + (size_t)it * 8 + 16);
-              v4[0] = a.x; v4[1] = a.y; v4[2] = b.x; v4[3] = b.y;
-            } else {
-              const int4 a = *reinterpret_cast<const int4*>(cb + (size_t)it * 4);
-              v4[0] = a.x; v4[1] = a.y; v4[2] = a.z; v4[3] = a.w;
-            }
-            uint32_t m = 0;
-#pragma unroll
-            for (int v = 0; v < 4; v++) m |= (scan_pred(pr, v4[v]) ? 1u : 0u) << v;
-            flags &= ~((~m & 0xFu) << (s * 4));
-          }
+          if (kMode == SM_SEL_RANGE && (pr.width == 4 ? pr.empty32 : pr.empty64)) flags = 0;
+          pred16_staged<kMode>(pr, buf + P.col_off[p], wrow, lane, flags);
         }
       } else {
         // ---- dense probe: keys from the staged fk column -------------------------
         int32_t key[SC_ITEMS];
 #pragma unroll
         for (int s = 0; s < SC_SLOTS; s++) {
-          const int4 a = *reinterpret_cast<const int4*>(buf + (size_t)(wrow + s * 128 + lane * 4) * 4);
+          const int4 a = kReg ? nk[s] : *reinterpret_cast<const int4*>(buf + (size_t)(wrow + s * 128 + lane * 4) * 4);
           key[s * 4 + 0] = a.x; key[s * 4 + 1] = a.y; key[s * 4 + 2] = a.z; key[s * 4 + 3] = a.w;
         }
-        if (hash_pay) probe16<true>(P, table, bm, key, flags, payload);
-        else probe16<false>(P, table, bm, key, flags, payload);
+        if (kReg && tile + vgrid < ntiles) load_keys(P.fk, n, (tile + vgrid) * SC_TILE, wrow, lane, nk);
+        if (want_pay) probe16<kPM, true>(P, table, bm, pa, bm_padded, key, flags, payload);
+        else probe16<kPM, false>(P, table, bm, pa, bm_padded, key, flags, payload);
       }
     }
     // group scan of the per-slot survivor counts
@@ -343,7 +443,7 @@ __global__ void __launch_bounds__(SC_GT* G, 1) scan_kernel(const __grid_constant
     }
     uint32_t my_base = 0;
     if (t == 0) {
-      if (!kTids && have) {  // dense: refill stage (k-1)%S, released by (A)
+      if (!kTids && !kReg && have) {  // dense: refill stage (k-1)%S, released by (A)
         const uint32_t tl = tile + (uint32_t)ahead * vgrid;
         if (tl < ntiles) {
           fence_proxy_async();
@@ -353,26 +453,10 @@ __global__ void __launch_bounds__(SC_GT* G, 1) scan_kernel(const __grid_constant
       }
       my_base = tot ? atomicAdd(P.d_out_count, tot) : 0;  // consumed only before (B)
     }
-    // stage tile k's survivors (tile-local item offsets + hash payloads) in list[k&1]
-    uint16_t* lst = s_list + (k & 1) * SC_TILE;
-    int32_t* pay = s_pay + (k & 1) * SC_TILE;
-#pragma unroll
-    for (int s = 0; s < SC_SLOTS; s++) {
-      const uint32_t m = (flags >> (4 * s)) & 0xFu;
-      const uint32_t sb = warp_off + slot_off[s] + ((excl >> (8 * s)) & 0xFFu);
-#pragma unroll
-      for (int v = 0; v < 4; v++) {
-        if ((m >> v) & 1u) {
-          const uint32_t pos = sb + __popc(m & ((1u << v) - 1u));
-          lst[pos] = (uint16_t)(wrow + s * 128 + lane * 4 + v);
-          if (hash_pay) pay[pos] = payload[s * 4 + v];
-        }
-      }
-    }
     // copy out tile k-1 (reserved last iteration): coalesced, survivors only
     if (k > 0) {
-      const uint16_t* pl = s_list + ((k - 1) & 1) * SC_TILE;
-      const int32_t* pp = s_pay + ((k - 1) & 1) * SC_TILE;
+      const uint16_t* pl = s_list;
+      const int32_t* pp = s_pay;
       const uint32_t prow0 = (tile - vgrid) * SC_TILE;
       const int32_t* ptid = reinterpret_cast<const int32_t*>(ring + (size_t)((k - 1) % S) * P.stage_bytes);
       const uint32_t lim = prev_base + prev_tot <= P.out_cap ? prev_tot
@@ -382,28 +466,36 @@ __global__ void __launch_bounds__(SC_GT* G, 1) scan_kernel(const __grid_constant
         const uint32_t it = pl[i];
         const int32_t r = kTids ? ptid[it] : (int32_t)(prow0 + it);
         P.out_tids[prev_base + i] = r;
-        if (want_pay) {
-          int32_t pv;
-          if (hash_pay) {
-            pv = pp[i];
-          } else {  // direct join index: re-read the (L2-hot) key, fetch the payload
-            const int64_t ki = (kTids && P.fk_by_pos) ? (int64_t)(prow0 + it) : (int64_t)r;
-            pv = __ldg(P.payarr + (uint32_t)(__ldg(P.fk + ki) - P.key_min));
-          }
-          P.out_payload[prev_base + i] = pv;
-        }
+        if (want_pay) P.out_payload[prev_base + i] = pp[i];
         if (kTids)
           for (int c = 0; c < P.n_carry; c++) P.carry_out[c][prev_base + i] = __ldg(P.carry_in[c] + prow0 + it);
       }
     }
     if (t == 0) s_base[g] = my_base;
-    group_sync(g);  // (B) s_base visible; list[(k-1)&1] and (TID mode) stage (k-1)%S free
+    group_sync(g);  // (B) s_base visible; the list and (TID mode) stage (k-1)%S free
     if (kTids && t == 0 && have) {  // TID mode: refill stage (k-1)%S now
       const uint32_t tl = tile + (uint32_t)ahead * vgrid;
       if (tl < ntiles) {
         fence_proxy_async();
         const int st = (int)((k + ahead) % S);
         issue_tile(P, n, ring + (size_t)st * P.stage_bytes, &s_full[g][st], tl);
+      }
+    }
+    // stage tile k's survivors (tile-local item offsets + payloads) in the list,
+    // which (B) released; (A) of the next iteration publishes it to the copy-out
+    if (flags) {
+#pragma unroll
+      for (int s = 0; s < SC_SLOTS; s++) {
+        const uint32_t m = (flags >> (4 * s)) & 0xFu;
+        const uint32_t sb = warp_off + slot_off[s] + ((excl >> (8 * s)) & 0xFFu);
+#pragma unroll
+        for (int v = 0; v < 4; v++) {
+          if ((m >> v) & 1u) {
+            const uint32_t pos = sb + __popc(m & ((1u << v) - 1u));
+            s_list[pos] = (uint16_t)(wrow + s * 128 + lane * 4 + v);
+            if (want_pay) s_pay[pos] = payload[s * 4 + v];
+          }
+        }
       }
     }
     prev_base = s_base[g];
@@ -423,12 +515,18 @@ __global__ void __launch_bounds__(SC_GT* G, 1) scan_kernel(const __grid_constant
 
 static int g_smem_optin = 0;
 
-template <bool kTids>
-static void set_attrs(int v) {
-  cudaFuncSetAttribute(scan_kernel<1, kTids>, cudaFuncAttributeMaxDynamicSharedMemorySize, v - 2048);
-  cudaFuncSetAttribute(scan_kernel<2, kTids>, cudaFuncAttributeMaxDynamicSharedMemorySize, v - 2048);
-  cudaFuncSetAttribute(scan_kernel<3, kTids>, cudaFuncAttributeMaxDynamicSharedMemorySize, v - 2048);
-  cudaFuncSetAttribute(scan_kernel<4, kTids>, cudaFuncAttributeMaxDynamicSharedMemorySize, v - 2048);
+template <int G, bool kTids>
+static void set_attrs_g(int v) {
+  cudaFuncSetAttribute(scan_kernel<G, kTids, SM_SEL_GENERIC>, cudaFuncAttributeMaxDynamicSharedMemorySize, v - 2048);
+  cudaFuncSetAttribute(scan_kernel<G, kTids, SM_SEL_RANGE>, cudaFuncAttributeMaxDynamicSharedMemorySize, v - 2048);
+  cudaFuncSetAttribute(scan_kernel<G, kTids, SM_PROBE_DIRECT>, cudaFuncAttributeMaxDynamicSharedMemorySize, v - 2048);
+  cudaFuncSetAttribute(scan_kernel<G, kTids, SM_PROBE_HASH>, cudaFuncAttributeMaxDynamicSharedMemorySize, v - 2048);
+  if (!kTids) {
+    cudaFuncSetAttribute(scan_kernel<G, false, SM_PROBE_DIRECT_R>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         v - 2048);
+    cudaFuncSetAttribute(scan_kernel<G, false, SM_PROBE_HASH_R>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         v - 2048);
+  }
 }
 
 bool scan_supported(const FilterArgs& a) {
@@ -443,13 +541,19 @@ bool scan_supported(const FilterArgs& a) {
   return true;
 }
 
-template <bool kTids>
-static void launch_g(int G, int64_t grid, size_t smem, cudaStream_t st, const ScanParams& p) {
-  switch (G) {
-    case 1: scan_kernel<1, kTids><<<(int)grid, SC_GT * 1, smem, st>>>(p); break;
-    case 2: scan_kernel<2, kTids><<<(int)grid, SC_GT * 2, smem, st>>>(p); break;
-    case 3: scan_kernel<3, kTids><<<(int)grid, SC_GT * 3, smem, st>>>(p); break;
-    default: scan_kernel<4, kTids><<<(int)grid, SC_GT * 4, smem, st>>>(p); break;
+template <int G, bool kTids>
+static void launch_m(int mode, int64_t grid, size_t smem, cudaStream_t st, const ScanParams& p) {
+  switch (mode) {
+    case SM_SEL_GENERIC: scan_kernel<G, kTids, SM_SEL_GENERIC><<<(int)grid, SC_GT * G, smem, st>>>(p); break;
+    case SM_SEL_RANGE: scan_kernel<G, kTids, SM_SEL_RANGE><<<(int)grid, SC_GT * G, smem, st>>>(p); break;
+    case SM_PROBE_DIRECT: scan_kernel<G, kTids, SM_PROBE_DIRECT><<<(int)grid, SC_GT * G, smem, st>>>(p); break;
+    case SM_PROBE_HASH: scan_kernel<G, kTids, SM_PROBE_HASH><<<(int)grid, SC_GT * G, smem, st>>>(p); break;
+    case SM_PROBE_DIRECT_R:
+      if (!kTids) scan_kernel<G, false, SM_PROBE_DIRECT_R><<<(int)grid, SC_GT * G, smem, st>>>(p);
+      break;
+    default:
+      if (!kTids) scan_kernel<G, false, SM_PROBE_HASH_R><<<(int)grid, SC_GT * G, smem, st>>>(p);
+      break;
   }
 }
 
@@ -459,8 +563,12 @@ cudaError_t launch_scan(const FilterArgs& a, cudaStream_t st) {
     cudaGetDevice(&dev);
     int v = 0;
     cudaDeviceGetAttribute(&v, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
-    set_attrs<false>(v);
-    set_attrs<true>(v);
+    set_attrs_g<1, false>(v);
+    set_attrs_g<2, false>(v);
+    set_attrs_g<3, false>(v);
+    set_attrs_g<4, false>(v);
+    set_attrs_g<1, true>(v);
+    set_attrs_g<2, true>(v);
     g_smem_optin = v;
   }
   const bool tids = a.in_tids != nullptr;
@@ -488,15 +596,24 @@ cudaError_t launch_scan(const FilterArgs& a, cudaStream_t st) {
     }
   }
   p.n_preds = a.probe ? 0 : a.n_preds;
+  bool all_range = true;
   for (int i = 0; i < p.n_preds; i++) {
     const ddq_dev_pred& d = a.preds[i];
-    p.preds[i].col = d.col;
-    p.preds[i].width = d.width;
-    p.preds[i].kind = d.kind;
-    p.preds[i].lo = d.lo;
-    p.preds[i].hi = d.hi;
-    p.preds[i].n_in = d.n_in;
-    for (int j = 0; j < 8; j++) p.preds[i].in_vals[j] = d.in_vals[j];
+    ScanPred& q = p.preds[i];
+    q.col = d.col;
+    q.width = d.width;
+    q.kind = d.kind;
+    q.lo = d.lo;
+    q.hi = d.hi;
+    q.n_in = d.n_in;
+    for (int j = 0; j < 8; j++) q.in_vals[j] = d.in_vals[j];
+    all_range = all_range && d.kind == DDQ_PRED_RANGE;
+    q.empty64 = d.hi < d.lo;
+    q.d64 = q.empty64 ? 0 : (uint64_t)d.hi - (uint64_t)d.lo;
+    const int64_t lo32 = d.lo < INT32_MIN ? INT32_MIN : d.lo, hi32 = d.hi > INT32_MAX ? INT32_MAX : d.hi;
+    q.empty32 = hi32 < lo32;
+    q.lo32 = q.empty32 ? 0 : (int32_t)lo32;
+    q.d32 = q.empty32 ? 0 : (uint32_t)(hi32 - lo32);
   }
   p.eq_a = a.eq_a;
   p.eq_b = a.eq_b;
@@ -505,13 +622,23 @@ cudaError_t launch_scan(const FilterArgs& a, cudaStream_t st) {
   p.fk = a.fk;
   p.fk_by_pos = a.fk_by_pos ? 1 : 0;
   const bool direct = a.probe && a.bitmap != nullptr;
-  const size_t table_bytes = a.probe ? (direct ? ((size_t)a.range + 31) / 32 * 4 : (size_t)a.capacity * 8) : 0;
+  int mode = a.probe ? (direct ? SM_PROBE_DIRECT : SM_PROBE_HASH)
+                           : (all_range && !a.eq_a ? SM_SEL_RANGE : SM_SEL_GENERIC);
+  // smem-resident structure: hash table, or join-index bitmap (+1 zero word) and,
+  // when it fits too, the payload array
+  const size_t kSmemTable = 144 * 1024;
+  const size_t bm_bytes = direct ? ((size_t)a.range + 31) / 32 * 4 + 4 : 0;
+  const size_t table_bytes = a.probe ? (direct ? bm_bytes : (size_t)a.capacity * 8) : 0;
   const size_t budget = (size_t)g_smem_optin - 2048;
-  const bool in_smem = a.probe && table_bytes <= 144 * 1024;
+  const bool in_smem = a.probe && table_bytes <= kSmemTable;
   p.table_in_smem = (in_smem && !direct) ? 1 : 0;
   p.bitmap_in_smem = (in_smem && direct) ? 1 : 0;
-  const size_t shared = in_smem ? (table_bytes + 127) / 128 * 128 : 0;
-  const size_t list_bytes = (size_t)SC_TILE * 4 + (a.probe && !direct && a.out_payload ? (size_t)SC_TILE * 8 : 0);
+  const size_t pa_off = (bm_bytes + 15) / 16 * 16;
+  const bool pa_smem = in_smem && direct && a.out_payload && pa_off + (size_t)a.range * 4 <= kSmemTable;
+  p.payarr_in_smem = pa_smem ? 1 : 0;
+  p.payarr_off = (int32_t)pa_off;
+  const size_t shared = in_smem ? ((pa_smem ? pa_off + (size_t)a.range * 4 : table_bytes) + 127) / 128 * 128 : 0;
+  const size_t list_bytes = (size_t)SC_TILE * 2 + (a.probe && a.out_payload ? (size_t)SC_TILE * 4 : 0);
   // as many groups (up to 4) and stages (up to 4, at least 2) as shared memory allows
   const int min_s = 2;
   // TID mode holds 16 gathered values per thread: > 2 groups spill registers (ptxas)
@@ -520,6 +647,22 @@ cudaError_t launch_scan(const FilterArgs& a, cudaStream_t st) {
   while (G > 1 && need(G, min_s) > budget) G--;
   while (S > min_s && need(G, S) > budget) S--;
   if (need(G, S) > budget) return cudaErrorInvalidConfiguration;
+  // dense probes stream the keys through registers (microbench, 120M keys: 73 KB
+  // bitmap + payloads 389 -> 258 us, 122 KB bitmap 431 -> 201 us vs the TMA ring,
+  // whose smem competes with the bitmap); DDQ_SCAN_REG=0 selects the ring
+  bool reg = false;
+  if (a.probe && !tids) {
+    static const char* env = getenv("DDQ_SCAN_REG");
+    reg = env ? env[0] == '1' : true;
+  }
+  if (reg) {
+    mode = direct ? SM_PROBE_DIRECT_R : SM_PROBE_HASH_R;
+    p.n_cols = 0;
+    p.stage_bytes = 0;
+    S = 1;
+    G = a.out_payload ? 3 : 4;  // register budget (ptxas: no spills)
+    while (G > 1 && shared + (size_t)G * list_bytes > budget) G--;
+  }
   p.stages = S;
   p.list_off = S * p.stage_bytes;
   p.group_bytes = (int32_t)((p.list_off + list_bytes + 127) / 128 * 128);
@@ -555,8 +698,17 @@ cudaError_t launch_scan(const FilterArgs& a, cudaStream_t st) {
   int64_t grid = num_sms();
   const int64_t need_ctas = (ntiles + G - 1) / G;
   if (grid > need_ctas) grid = need_ctas < 1 ? 1 : need_ctas;
-  if (tids) launch_g<true>(G, grid, smem, st, p);
-  else launch_g<false>(G, grid, smem, st, p);
+  if (tids) {
+    if (G == 1) launch_m<1, true>(mode, grid, smem, st, p);
+    else launch_m<2, true>(mode, grid, smem, st, p);
+  } else {
+    switch (G) {
+      case 1: launch_m<1, false>(mode, grid, smem, st, p); break;
+      case 2: launch_m<2, false>(mode, grid, smem, st, p); break;
+      case 3: launch_m<3, false>(mode, grid, smem, st, p); break;
+      default: launch_m<4, false>(mode, grid, smem, st, p); break;
+    }
+  }
   return cudaGetLastError();
 }
 

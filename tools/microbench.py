@@ -48,20 +48,22 @@ def main():
         ms = timeit(sel(col, lo, hi))
         gb = n * col.element_size() / 1e9
         print(f"select {name:14s} {ms*1e3:8.1f} us  {gb/ms*1e3:8.1f} GB/s (input only)", flush=True)
-    for frac in (0.2, 0.05):
-        keys = torch.arange(1, 600_001, dtype=torch.int32, device="cuda")
-        sel_rows = torch.nonzero(torch.rand(600_000, device="cuda", generator=g) < frac).int().flatten()
-        idx, err = ops.join_index_build(keys, 1, 600_000, payload=keys, in_tids=sel_rows,
+    for rng_keys, frac in ((600_000, 0.2), (600_000, 0.05), (1_000_000, 0.04)):
+        fk = c32 if rng_keys == 600_000 else torch.randint(1, rng_keys + 1, (n,), device="cuda", dtype=torch.int32,
+                                                           generator=g)
+        keys = torch.arange(1, rng_keys + 1, dtype=torch.int32, device="cuda")
+        sel_rows = torch.nonzero(torch.rand(rng_keys, device="cuda", generator=g) < frac).int().flatten()
+        idx, err = ops.join_index_build(keys, 1, rng_keys, payload=keys, in_tids=sel_rows,
                                         in_count=ops.count_cell(sel_rows.numel()), n=sel_rows.numel())
         for emit in (False, True):
             def probe():
-                ops.check(ops.lib().ddq_op_join_index_probe(idx.data_ptr(), 1, 600_000, c32.data_ptr(), None, None,
+                ops.check(ops.lib().ddq_op_join_index_probe(idx.data_ptr(), 1, rng_keys, fk.data_ptr(), None, None,
                                                             n, None, None, 0, out.data_ptr(),
                                                             pay.data_ptr() if emit else None, cnt.data_ptr(),
                                                             scratch.data_ptr(), scratch.numel(), ops._stream()))
             ms = timeit(probe)
-            print(f"probe  bitmap75KB pass {frac:.2f} emit={emit} {ms*1e3:8.1f} us  {n*4/1e9/ms*1e3:8.1f} GB/s",
-                  flush=True)
+            print(f"probe  bitmap{(rng_keys + 7) // 8 // 1024}KB pass {frac:.2f} emit={emit} {ms*1e3:8.1f} us"
+                  f"  {n*4/1e9/ms*1e3:8.1f} GB/s", flush=True)
     ms = timeit(lambda: out.copy_(c32))
     print(f"torch copy int32 (read+write) {ms*1e3:8.1f} us  {2*n*4/1e9/ms*1e3:8.1f} GB/s")
 

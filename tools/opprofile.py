@@ -15,7 +15,7 @@ def main():
     ap.add_argument("--sf", type=float, default=20)
     ap.add_argument("--queries", default="")
     ap.add_argument("--launch", type=int, default=0)
-    ap.add_argument("--chain", action="store_true", help="binary-operator chains instead of STAR")
+    ap.add_argument("--star", action="store_true", help="n-ary STAR operator instead of binary-operator chains")
     a = ap.parse_args()
     import torch
     import datagen
@@ -25,7 +25,7 @@ def main():
     data = datagen.SSB(a.sf)
     db = Database(cache_bytes=64 << 30, heap_bytes=24 << 30)
     load_ssb(db, data)
-    preps = {q: db.prepare(ssb_plan(db, q, star=not a.chain)) for q in qs}
+    preps = {q: db.prepare(ssb_plan(db, q, star=a.star)) for q in qs}
     torch.cuda.synchronize()
     if a.launch:
         for _ in range(a.launch):
