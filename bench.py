@@ -328,7 +328,7 @@ def main():
     hbm_peak = pk.get("hbm_gbs", 6650.0)
     achieved = cls_bytes[dom] / (cls_ms[dom] / 1e3) / 1e9
     step_bytes = sum(cls_bytes.values())
-    roofline = {"bound": "hbm", "kernel": "filter_kernel: " + names[dom], "achieved": round(achieved, 1),
+    roofline = {"bound": "hbm", "kernel": "scan_kernel: " + names[dom], "achieved": round(achieved, 1),
                 "peak": hbm_peak, "unit": "GB/s", "frac": round(achieved / hbm_peak, 4), "traffic": None,
                 "launches_per_step": cls_n[dom], "share_of_step": round(cls_ms[dom] / sum(cls_ms.values()), 3),
                 "peak_source": "MEASURED_PEAKS.json hbm_gbs (measured)" if "hbm_gbs" in pk else "fallback 6.65 TB/s",

@@ -163,9 +163,9 @@ __device__ __forceinline__ bool scan_pred(const ScanPred& p, int64_t v) {
   return m;
 }
 
-// Membership (+ payload lookup) of 16 keys; clears the flag bits of misses.  Payloads
-// are loaded for hits only, right after the probe, so their latency overlaps the
-// survivor scan and barrier (they are staged in smem with the survivor list).
+// Membership of 16 keys; clears the flag bits of misses.  kPay: hash probes return
+// the payloads (read with the slot); join-index probes return the payload-array
+// offsets, looked up at copy-out for the survivors only (batched loads).
 template <int kMode, bool kPay>
 __device__ __forceinline__ void probe16(const ScanParams& P, const uint64_t* table, const uint32_t* bm,
                                         const int32_t* pa, bool bm_padded, const int32_t (&key)[SC_ITEMS],
@@ -188,10 +188,9 @@ __device__ __forceinline__ void probe16(const ScanParams& P, const uint64_t* tab
       }
     }
     flags &= m;
-    if (kPay) {
+    if (kPay) {  // the hits' offsets; their payloads are fetched at copy-out (survivors only)
 #pragma unroll
-      for (int k = 0; k < SC_ITEMS; k++)
-        payload[k] = ((flags >> k) & 1u) ? pa[(uint32_t)(key[k] - P.key_min)] : 0;
+      for (int k = 0; k < SC_ITEMS; k++) payload[k] = (int32_t)(key[k] - P.key_min);
     }
   } else {
     uint32_t h[SC_ITEMS];
@@ -462,13 +461,32 @@ __global__ void __launch_bounds__(SC_GT* G, 1) scan_kernel(const __grid_constant
       const uint32_t lim = prev_base + prev_tot <= P.out_cap ? prev_tot
                          : (P.out_cap > prev_base ? P.out_cap - prev_base : 0);
       if (lim < prev_tot && t == 0 && P.d_overflow) atomicMax(P.d_overflow, 4u);
-      for (uint32_t i = t; i < lim; i += SC_GT) {
-        const uint32_t it = pl[i];
-        const int32_t r = kTids ? ptid[it] : (int32_t)(prow0 + it);
-        P.out_tids[prev_base + i] = r;
-        if (want_pay) P.out_payload[prev_base + i] = pp[i];
-        if (kTids)
-          for (int c = 0; c < P.n_carry; c++) P.carry_out[c][prev_base + i] = __ldg(P.carry_in[c] + prow0 + it);
+      constexpr int U = 4;  // survivors per thread per batch: independent loads in flight
+      for (uint32_t i0 = t; i0 < lim; i0 += U * SC_GT) {
+        uint32_t it[U];
+        int32_t pv[U];
+#pragma unroll
+        for (int u = 0; u < U; u++) {
+          const uint32_t i = i0 + u * SC_GT;
+          it[u] = i < lim ? pl[i] : 0u;
+          pv[u] = (want_pay && i < lim) ? pp[i] : 0;
+        }
+        if (kDirect && want_pay) {
+#pragma unroll
+          for (int u = 0; u < U; u++)
+            if (i0 + u * SC_GT < lim) pv[u] = pa[(uint32_t)pv[u]];
+        }
+#pragma unroll
+        for (int u = 0; u < U; u++) {
+          const uint32_t i = i0 + u * SC_GT;
+          if (i < lim) {
+            P.out_tids[prev_base + i] = kTids ? ptid[it[u]] : (int32_t)(prow0 + it[u]);
+            if (want_pay) P.out_payload[prev_base + i] = pv[u];
+            if (kTids)
+              for (int c = 0; c < P.n_carry; c++)
+                P.carry_out[c][prev_base + i] = __ldg(P.carry_in[c] + prow0 + it[u]);
+          }
+        }
       }
     }
     if (t == 0) s_base[g] = my_base;
