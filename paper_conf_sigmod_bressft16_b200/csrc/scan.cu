@@ -98,6 +98,7 @@ struct ScanParams {
   int32_t bitmap_in_smem;
   int32_t payarr_in_smem;  // payload array staged after the bitmap (at payarr_off)
   int32_t payarr_off;
+  int32_t tid_off;  // TID mode: survivor TID list, offset inside a group's area
   int32_t* out_payload;
   // carried vectors (TID mode)
   int32_t n_carry;
@@ -145,14 +146,11 @@ __device__ __forceinline__ void issue_tile(const ScanParams& P, uint32_t n, uint
   const uint64_t row0 = (uint64_t)tile * SC_TILE;
   const uint64_t rows = (uint64_t)n - row0 < (uint64_t)SC_TILE ? (uint64_t)n - row0 : (uint64_t)SC_TILE;
   uint32_t total = 0;
-  uint32_t bytes[SC_MAXCOLS];
-  for (int c = 0; c < P.n_cols; c++) {
-    bytes[c] = (uint32_t)((rows * P.width[c] + 15) / 16 * 16);
-    total += bytes[c];
-  }
+  for (int c = 0; c < P.n_cols; c++) total += (uint32_t)((rows * P.width[c] + 15) / 16 * 16);
   mbar_arrive_expect_tx(bar, total);
   for (int c = 0; c < P.n_cols; c++)
-    tma_load_1d(buf + P.col_off[c], reinterpret_cast<const uint8_t*>(P.cols[c]) + row0 * P.width[c], bytes[c], bar);
+    tma_load_1d(buf + P.col_off[c], reinterpret_cast<const uint8_t*>(P.cols[c]) + row0 * P.width[c],
+                (uint32_t)((rows * P.width[c] + 15) / 16 * 16), bar);
 }
 
 __device__ __forceinline__ bool scan_pred(const ScanPred& p, int64_t v) {
@@ -293,7 +291,9 @@ __global__ void __launch_bounds__(SC_GT* G, 1) scan_kernel(const __grid_constant
   constexpr bool kProbe = kMode >= SM_PROBE_DIRECT;
   constexpr bool kDirect = kMode == SM_PROBE_DIRECT || kMode == SM_PROBE_DIRECT_R;
   constexpr bool kHash = kProbe && !kDirect;
-  constexpr bool kReg = kMode >= SM_PROBE_DIRECT_R;  // dense only
+  // register-streamed input: dense probe keys (*_R variants) or the TID list (TID
+  // mode: no ring; the TIDs of the survivors are staged with the survivor list)
+  constexpr bool kReg = kMode >= SM_PROBE_DIRECT_R || kTids;
   constexpr int kPM = kDirect ? SM_PROBE_DIRECT : SM_PROBE_HASH;
   extern __shared__ __align__(128) uint8_t smem[];
   __shared__ uint32_t s_warp_tot[SC_MAXG][SC_GW];
@@ -305,19 +305,20 @@ __global__ void __launch_bounds__(SC_GT* G, 1) scan_kernel(const __grid_constant
   const uint32_t n = kTids ? ld_relaxed_u32(P.d_in_count) : P.n;
   const uint32_t ntiles = (n + SC_TILE - 1) / SC_TILE;
   const int S = P.stages;
-  // S-1 tiles in flight ahead of the current one; stage (k-1)%S is refilled with
-  // tile k+S-1 right after (A) in dense mode, after (B) in TID mode (whose copy-out
-  // of tile k-1 reads its TIDs from that stage)
+  // ring mode: S-1 tiles in flight ahead of the current one; stage (k-1)%S is
+  // refilled with tile k+S-1 right after (A)
   const int ahead = S - 1;
   const uint32_t vb = blockIdx.x * G + g, vgrid = gridDim.x * G;  // virtual CTA id / count
   uint8_t* ring = smem + (size_t)g * P.group_bytes;
   uint16_t* s_list = reinterpret_cast<uint16_t*>(ring + P.list_off);             // TILE
   int32_t* s_pay = reinterpret_cast<int32_t*>(ring + P.list_off + SC_TILE * 2);  // TILE
+  int32_t* s_tid = reinterpret_cast<int32_t*>(ring + P.tid_off);                   // TILE (TID mode)
+  const int32_t* scol = kTids ? reinterpret_cast<const int32_t*>(P.cols[0]) : P.fk;  // streamed column
   uint64_t* s_table = reinterpret_cast<uint64_t*>(smem + P.shared_off);
 
   const uint32_t wrow = warp * (32 * SC_ITEMS);  // warp's first item inside a tile
   int4 nk[SC_SLOTS];                             // register-streamed keys of the next tile
-  if (kReg && vb < ntiles) load_keys(P.fk, n, vb * SC_TILE, wrow, lane, nk);
+  if (kReg && vb < ntiles) load_keys(scol, n, vb * SC_TILE, wrow, lane, nk);
   if (t == 0 && !kReg) {  // group leader: barriers, then the first tiles in flight
     for (int k = 0; k < S; k++) mbar_init(&s_full[g][k], 1);
     fence_mbar_init();
@@ -350,15 +351,18 @@ __global__ void __launch_bounds__(SC_GT* G, 1) scan_kernel(const __grid_constant
   // k-1, whose range was reserved last iteration, from the survivor list; after (B)
   // it stages tile k's survivors in that list (one buffer: half the smem of two).
   uint32_t prev_tot = 0, prev_base = 0;
+  int stg = 0;        // ring stage of tile k (k % S)
+  uint32_t ph = 0;    // its mbarrier phase parity ((k / S) & 1)
   for (uint32_t k = 0;; k++) {
     const uint32_t tile = vb + k * vgrid;
     const bool have = tile < ntiles;
     const uint32_t row0 = tile * SC_TILE;  // first item of the tile
     uint32_t flags = 0;
     int32_t payload[SC_ITEMS];
+    int32_t row[SC_ITEMS];  // TID mode: the tile's TIDs
     if (have) {
-      if (!kReg) mbar_wait(&s_full[g][k % S], (k / S) & 1u);
-      const uint8_t* buf = ring + (size_t)(k % S) * P.stage_bytes;
+      if (!kReg) mbar_wait(&s_full[g][stg], ph);
+      const uint8_t* buf = ring + (size_t)stg * P.stage_bytes;
       flags = 0xFFFFu;
       if (row0 + SC_TILE > n) {  // tail tile only
         flags = 0;
@@ -370,12 +374,11 @@ __global__ void __launch_bounds__(SC_GT* G, 1) scan_kernel(const __grid_constant
       }
       if (kTids) {
         // ---- TID mode: rows from the staged TID list, values gathered ----------
-        int32_t row[SC_ITEMS];
 #pragma unroll
         for (int s = 0; s < SC_SLOTS; s++) {
-          const int4 a = *reinterpret_cast<const int4*>(buf + (size_t)(wrow + s * 128 + lane * 4) * 4);
-          row[s * 4 + 0] = a.x; row[s * 4 + 1] = a.y; row[s * 4 + 2] = a.z; row[s * 4 + 3] = a.w;
+          row[s * 4 + 0] = nk[s].x; row[s * 4 + 1] = nk[s].y; row[s * 4 + 2] = nk[s].z; row[s * 4 + 3] = nk[s].w;
         }
+        if (tile + vgrid < ntiles) load_keys(scol, n, (tile + vgrid) * SC_TILE, wrow, lane, nk);
         if (!kProbe) {
           for (int p = 0; p < P.n_preds; p++) pred16_gathered<kMode>(P.preds[p], row, flags);
           if (P.eq_a) {
@@ -389,10 +392,15 @@ __global__ void __launch_bounds__(SC_GT* G, 1) scan_kernel(const __grid_constant
           }
         } else {
           int32_t key[SC_ITEMS];
+          if (P.fk_by_pos) {  // positional key vector: coalesced
 #pragma unroll
-          for (int k2 = 0; k2 < SC_ITEMS; k2++) {
-            const uint32_t pos = row0 + wrow + (k2 >> 2) * 128 + lane * 4 + (k2 & 3);
-            key[k2] = ((flags >> k2) & 1u) ? __ldg(P.fk + (P.fk_by_pos ? (int64_t)pos : (int64_t)row[k2])) : 0;
+            for (int k2 = 0; k2 < SC_ITEMS; k2++) {
+              const uint32_t pos = row0 + wrow + (k2 >> 2) * 128 + lane * 4 + (k2 & 3);
+              key[k2] = ((flags >> k2) & 1u) ? __ldg(P.fk + pos) : 0;
+            }
+          } else {  // key column gathered at the TIDs
+#pragma unroll
+            for (int k2 = 0; k2 < SC_ITEMS; k2++) key[k2] = ((flags >> k2) & 1u) ? __ldg(P.fk + (uint32_t)row[k2]) : 0;
           }
           if (want_pay) probe16<kPM, true>(P, table, bm, pa, bm_padded, key, flags, payload);
           else probe16<kPM, false>(P, table, bm, pa, bm_padded, key, flags, payload);
@@ -442,11 +450,11 @@ __global__ void __launch_bounds__(SC_GT* G, 1) scan_kernel(const __grid_constant
     }
     uint32_t my_base = 0;
     if (t == 0) {
-      if (!kTids && !kReg && have) {  // dense: refill stage (k-1)%S, released by (A)
+      if (!kReg && have) {  // ring: refill stage (k-1)%S, released by (A)
         const uint32_t tl = tile + (uint32_t)ahead * vgrid;
         if (tl < ntiles) {
           fence_proxy_async();
-          const int st = (int)((k + ahead) % S);
+          const int st = stg == 0 ? S - 1 : stg - 1;  // (k + S - 1) % S
           issue_tile(P, n, ring + (size_t)st * P.stage_bytes, &s_full[g][st], tl);
         }
       }
@@ -457,7 +465,6 @@ __global__ void __launch_bounds__(SC_GT* G, 1) scan_kernel(const __grid_constant
       const uint16_t* pl = s_list;
       const int32_t* pp = s_pay;
       const uint32_t prow0 = (tile - vgrid) * SC_TILE;
-      const int32_t* ptid = reinterpret_cast<const int32_t*>(ring + (size_t)((k - 1) % S) * P.stage_bytes);
       const uint32_t lim = prev_base + prev_tot <= P.out_cap ? prev_tot
                          : (P.out_cap > prev_base ? P.out_cap - prev_base : 0);
       if (lim < prev_tot && t == 0 && P.d_overflow) atomicMax(P.d_overflow, 4u);
@@ -480,7 +487,7 @@ __global__ void __launch_bounds__(SC_GT* G, 1) scan_kernel(const __grid_constant
         for (int u = 0; u < U; u++) {
           const uint32_t i = i0 + u * SC_GT;
           if (i < lim) {
-            P.out_tids[prev_base + i] = kTids ? ptid[it[u]] : (int32_t)(prow0 + it[u]);
+            P.out_tids[prev_base + i] = kTids ? s_tid[i] : (int32_t)(prow0 + it[u]);
             if (want_pay) P.out_payload[prev_base + i] = pv[u];
             if (kTids)
               for (int c = 0; c < P.n_carry; c++)
@@ -490,15 +497,7 @@ __global__ void __launch_bounds__(SC_GT* G, 1) scan_kernel(const __grid_constant
       }
     }
     if (t == 0) s_base[g] = my_base;
-    group_sync(g);  // (B) s_base visible; the list and (TID mode) stage (k-1)%S free
-    if (kTids && t == 0 && have) {  // TID mode: refill stage (k-1)%S now
-      const uint32_t tl = tile + (uint32_t)ahead * vgrid;
-      if (tl < ntiles) {
-        fence_proxy_async();
-        const int st = (int)((k + ahead) % S);
-        issue_tile(P, n, ring + (size_t)st * P.stage_bytes, &s_full[g][st], tl);
-      }
-    }
+    group_sync(g);  // (B) s_base visible; the list is free
     // stage tile k's survivors (tile-local item offsets + payloads) in the list,
     // which (B) released; (A) of the next iteration publishes it to the copy-out
     if (flags) {
@@ -512,12 +511,17 @@ __global__ void __launch_bounds__(SC_GT* G, 1) scan_kernel(const __grid_constant
             const uint32_t pos = sb + __popc(m & ((1u << v) - 1u));
             s_list[pos] = (uint16_t)(wrow + s * 128 + lane * 4 + v);
             if (want_pay) s_pay[pos] = payload[s * 4 + v];
+            if (kTids) s_tid[pos] = row[s * 4 + v];
           }
         }
       }
     }
     prev_base = s_base[g];
     prev_tot = tot;
+    if (++stg == S) {
+      stg = 0;
+      ph ^= 1u;
+    }
     if (!have) break;
   }
   // the last CTA to finish clamps the count to the output capacity
@@ -656,10 +660,13 @@ cudaError_t launch_scan(const FilterArgs& a, cudaStream_t st) {
   p.payarr_in_smem = pa_smem ? 1 : 0;
   p.payarr_off = (int32_t)pa_off;
   const size_t shared = in_smem ? ((pa_smem ? pa_off + (size_t)a.range * 4 : table_bytes) + 127) / 128 * 128 : 0;
-  const size_t list_bytes = (size_t)SC_TILE * 2 + (a.probe && a.out_payload ? (size_t)SC_TILE * 4 : 0);
+  const size_t pay_bytes = a.probe && a.out_payload ? (size_t)SC_TILE * 4 : 0;
+  const size_t list_bytes = (size_t)SC_TILE * 2 + pay_bytes + (tids ? (size_t)SC_TILE * 4 : 0);
   // as many groups (up to 4) and stages (up to 4, at least 2) as shared memory allows
   const int min_s = 2;
-  // TID mode holds 16 gathered values per thread: > 2 groups spill registers (ptxas)
+  // TID mode: 2 groups (opprofile SF20: G=1 2105 us, G=2 1753 us, G=3 1894 us of
+  // at-TID ops -- the 85-register cap of G=3 serialises the gathers; so did a
+  // software-pipelined one-tile-ahead gather at G=2: spills, 1915 us)
   int G = tids ? 2 : 4, S = 4;
   auto need = [&](int gg, int ss) { return shared + (size_t)gg * ((size_t)ss * p.stage_bytes + list_bytes); };
   while (G > 1 && need(G, min_s) > budget) G--;
@@ -668,22 +675,26 @@ cudaError_t launch_scan(const FilterArgs& a, cudaStream_t st) {
   // dense probes stream the keys through registers (microbench, 120M keys: 73 KB
   // bitmap + payloads 389 -> 258 us, 122 KB bitmap 431 -> 201 us vs the TMA ring,
   // whose smem competes with the bitmap); DDQ_SCAN_REG=0 selects the ring
-  bool reg = false;
+  // TID mode always streams the TID list through registers (no ring)
+  bool reg = tids;
   if (a.probe && !tids) {
     static const char* env = getenv("DDQ_SCAN_REG");
     reg = env ? env[0] == '1' : true;
   }
   if (reg) {
-    mode = direct ? SM_PROBE_DIRECT_R : SM_PROBE_HASH_R;
-    p.n_cols = 0;
+    if (!tids) mode = direct ? SM_PROBE_DIRECT_R : SM_PROBE_HASH_R;
+    p.n_cols = tids ? 1 : 0;  // cols[0]: the TID list (streamed by the kernel itself)
     p.stage_bytes = 0;
     S = 1;
-    G = a.out_payload ? 3 : 4;  // register budget (ptxas: no spills)
+    // register budget (ptxas: no spills); hash probes hold 16 slots more
+    G = tids ? 2 : (a.out_payload ? 3 : 4) - (direct ? 0 : 1);
     while (G > 1 && shared + (size_t)G * list_bytes > budget) G--;
+    if (shared + (size_t)G * list_bytes > budget) return cudaErrorInvalidConfiguration;
   }
   p.stages = S;
   p.list_off = S * p.stage_bytes;
   p.group_bytes = (int32_t)((p.list_off + list_bytes + 127) / 128 * 128);
+  p.tid_off = (int32_t)(p.list_off + SC_TILE * 2 + pay_bytes);
   p.shared_off = G * p.group_bytes;
   if (direct) {
     p.direct = 1;

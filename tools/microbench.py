@@ -25,6 +25,7 @@ def timeit(fn, reps=10):
 
 def main():
     import torch
+    only = sys.argv[1] if len(sys.argv) > 1 else ""
     from paper_conf_sigmod_bressft16_b200 import ops
     n = 120_000_000
     g = torch.Generator(device="cuda").manual_seed(1)
@@ -45,6 +46,8 @@ def main():
     for name, col, lo, hi in [("i64 pass 0", c64, 1000, 2000), ("i64 pass 15%", c64, 0, 14),
                               ("i64 pass 100%", c64, 0, 100), ("i32 pass 0", c32, -5, -1),
                               ("i32 pass 20%", c32, 1, 120000)]:
+        if only and only not in "select " + name:
+            continue
         ms = timeit(sel(col, lo, hi))
         gb = n * col.element_size() / 1e9
         print(f"select {name:14s} {ms*1e3:8.1f} us  {gb/ms*1e3:8.1f} GB/s (input only)", flush=True)
@@ -56,6 +59,10 @@ def main():
         idx, err = ops.join_index_build(keys, 1, rng_keys, payload=keys, in_tids=sel_rows,
                                         in_count=ops.count_cell(sel_rows.numel()), n=sel_rows.numel())
         for emit in (False, True):
+            tag = f"probe bitmap{(rng_keys + 7) // 8 // 1024}KB pass {frac:.2f} emit={emit}"
+            if only and only not in tag:
+                continue
+
             def probe():
                 ops.check(ops.lib().ddq_op_join_index_probe(idx.data_ptr(), 1, rng_keys, fk.data_ptr(), None, None,
                                                             n, None, None, 0, out.data_ptr(),
@@ -64,6 +71,8 @@ def main():
             ms = timeit(probe)
             print(f"probe  bitmap{(rng_keys + 7) // 8 // 1024}KB pass {frac:.2f} emit={emit} {ms*1e3:8.1f} us"
                   f"  {n*4/1e9/ms*1e3:8.1f} GB/s", flush=True)
+    if only:
+        return
     ms = timeit(lambda: out.copy_(c32))
     print(f"torch copy int32 (read+write) {ms*1e3:8.1f} us  {2*n*4/1e9/ms*1e3:8.1f} GB/s")
 
