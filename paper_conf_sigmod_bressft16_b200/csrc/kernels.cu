@@ -169,6 +169,12 @@ struct GroupbyParams {
   uint32_t* d_error;
   uint32_t s_slots;
   int32_t s_shift;
+  // small-domain kernel: the distinct argument columns, loaded once per row, and
+  // each aggregate's arguments as indices into them
+  int32_t n_ucols;
+  const void* ucol[8];
+  int32_t uwidth[8];
+  int32_t uidx[8][3];
 };
 
 __device__ __forceinline__ long long agg_value(const GroupbyParams& P, int a, int32_t r) {
@@ -303,6 +309,136 @@ __global__ void __launch_bounds__(GB_THREADS) groupby_kernel(const __grid_consta
   }
 }
 
+// ---- small key domain (every key dictionary-coded in key_bits, D = 2^sum(bits)
+// groups, D * n_aggs <= GBS_MAX_DA): no warp reduction and no atomics per row.
+// Every thread owns D x n_aggs int64 partial sums in shared memory ([entry][thread],
+// conflict-free) updated with a plain read-modify-write; a signed-overflow test
+// per add spills the partial into a per-CTA int128 accumulator (exact for any
+// data).  At the end one warp per entry sums the CTA's partials in int128 and adds
+// them to the global table -- only for groups some row hit (`present` mask).
+constexpr int GBS_THREADS = 128;
+constexpr int GBS_ROWS = 4;  // rows per thread per iteration (independent gathers in flight)
+constexpr int GBS_MAX_DA = 64;
+
+__global__ void __launch_bounds__(GBS_THREADS) groupby_small_kernel(const __grid_constant__ GroupbyParams P,
+                                                                     uint32_t D) {
+  extern __shared__ unsigned long long s_mem[];
+  const int A = P.n_aggs;
+  const uint32_t DA = D * (uint32_t)A;
+  long long* part = reinterpret_cast<long long*>(s_mem);       // [DA][GBS_THREADS]
+  unsigned long long* spill = s_mem + (size_t)DA * GBS_THREADS;  // [DA][2] int128
+  uint32_t* present = reinterpret_cast<uint32_t*>(spill + (size_t)DA * 2);
+  const int tid = threadIdx.x;
+  for (uint32_t e = 0; e < DA; e++) part[(size_t)e * GBS_THREADS + tid] = 0;
+  for (uint32_t i = tid; i < DA * 2; i += GBS_THREADS) spill[i] = 0;
+  if (tid == 0) *present = 0;
+  __syncthreads();
+
+  const uint32_t n = P.d_count ? ld_relaxed_u32(P.d_count) : P.n_static;
+  uint32_t pm = 0;  // groups this thread hit
+  for (uint32_t base = blockIdx.x * (GBS_THREADS * GBS_ROWS); base < n;
+       base += gridDim.x * (GBS_THREADS * GBS_ROWS)) {
+    int32_t r[GBS_ROWS];
+    uint32_t d[GBS_ROWS];
+#pragma unroll
+    for (int j = 0; j < GBS_ROWS; j++) {
+      const uint32_t i = base + j * GBS_THREADS + tid;
+      r[j] = i < n ? P.tids[i] : -1;
+    }
+#pragma unroll
+    for (int j = 0; j < GBS_ROWS; j++) {
+      const uint32_t i = base + j * GBS_THREADS + tid;
+      uint32_t key = 0;
+      if (r[j] >= 0)
+        for (int k = 0; k < P.n_keys; k++) {
+          const int32_t c = P.key_vec[k] ? P.key_vec[k][i] : __ldg(P.key_col[k] + r[j]);
+          key |= (uint32_t)c << P.key_shift[k];
+        }
+      d[j] = key & (D - 1);
+      if (r[j] >= 0) pm |= 1u << d[j];
+    }
+    // every distinct argument column of the GBS_ROWS rows: independent loads in flight
+    long long val[8][GBS_ROWS];
+#pragma unroll
+    for (int c = 0; c < 8; c++)
+      if (c < P.n_ucols)
+#pragma unroll
+        for (int j = 0; j < GBS_ROWS; j++) val[c][j] = col_at(P.ucol[c], P.uwidth[c], r[j] < 0 ? 0 : r[j]);
+#pragma unroll
+    for (int a = 0; a < 8; a++) {
+      if (a >= A) break;
+      const int kind = P.kind[a], i0 = P.uidx[a][0], i1 = P.uidx[a][1], i2 = P.uidx[a][2];
+#pragma unroll
+      for (int j = 0; j < GBS_ROWS; j++) {
+        if (r[j] < 0) continue;
+        long long x = 0, y = 0, z = 0;
+#pragma unroll
+        for (int c = 0; c < 8; c++) {  // register selects, no dynamic indexing
+          x = c == i0 ? val[c][j] : x;
+          y = c == i1 ? val[c][j] : y;
+          z = c == i2 ? val[c][j] : z;
+        }
+        const long long v = kind == DDQ_AGG_COUNT ? 1
+                          : kind == DDQ_AGG_SUM ? x
+                          : kind == DDQ_AGG_SUM_MUL ? x * y
+                          : kind == DDQ_AGG_SUM_SUB ? x - y
+                          : kind == DDQ_AGG_SUM_MUL_100M ? x * (100 - y)
+                          : x * (100 - y) * (100 + z);
+        long long* slot = part + (size_t)(d[j] * A + a) * GBS_THREADS + tid;
+        const long long old = *slot;
+        const long long sum = (long long)((unsigned long long)old + (unsigned long long)v);
+        if (((old ^ sum) & (v ^ sum)) < 0) {  // signed overflow: spill the partial exactly
+          unsigned long long* sp = spill + (size_t)(d[j] * A + a) * 2;
+          atomic_add_i128_pair(sp, sp + 1, (unsigned long long)old, old < 0 ? -1 : 0);
+          *slot = v;
+        } else {
+          *slot = sum;
+        }
+      }
+    }
+  }
+  if (pm) atomicOr(present, pm);
+  __syncthreads();
+  // one warp per entry: int128 sum of the CTA's partials, then into the global table
+  const int lane = tid & 31, warp = tid >> 5;
+  const uint32_t pres = *present;
+  for (uint32_t e = warp; e < DA; e += GBS_THREADS / 32) {
+    const uint32_t g = e / A;
+    const int a = (int)(e % A);
+    if (!((pres >> g) & 1u)) continue;
+    unsigned long long lo = 0;
+    long long hi = 0;
+    for (int t = lane; t < GBS_THREADS; t += 32) {
+      const long long x = part[(size_t)e * GBS_THREADS + t];
+      const unsigned long long s2 = lo + (unsigned long long)x;
+      hi += (x < 0 ? -1 : 0) + (s2 < lo ? 1 : 0);
+      lo = s2;
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+      const unsigned long long tlo = __shfl_down_sync(FULL, lo, o);
+      const long long thi = __shfl_down_sync(FULL, hi, o);
+      const unsigned long long s2 = lo + tlo;
+      hi += thi + (s2 < lo ? 1 : 0);
+      lo = s2;
+    }
+    if (lane == 0) {
+      const unsigned long long slo = spill[(size_t)e * 2], shi = spill[(size_t)e * 2 + 1];
+      const unsigned long long s2 = lo + slo;
+      hi += (long long)shi + (s2 < lo ? 1 : 0);
+      lo = s2;
+      const long long key = (long long)g;
+      const int64_t slot = table_slot(P.g_keys, P.cap_mask, gb_hash(key, P.shift), key);
+      if (slot < 0) {
+        atomicMax(P.d_error, 2u);
+      } else {
+        unsigned long long* glo = &P.g_accs[((size_t)a * (P.cap_mask + 1) + slot) * 2];
+        atomic_add_i128_pair(glo, glo + 1, lo, hi);
+      }
+    }
+  }
+}
+
 size_t groupby_table_bytes(uint32_t capacity, int n_aggs) {
   return (size_t)capacity * 8 + (size_t)capacity * n_aggs * 16;
 }
@@ -359,6 +495,51 @@ cudaError_t launch_groupby(const int32_t* tids, const uint32_t* d_count, int64_t
   while ((1u << lg) < capacity) lg++;
   p.shift = 64 - lg;
   p.d_error = d_error;
+  // small key domain: every key dictionary-coded (key_bits), D * n_aggs <= 64
+  int total_bits = 0;
+  bool coded = n_keys == 0 || key_bits != nullptr;
+  for (int k = 0; k < n_keys && coded; k++) {
+    coded = key_bits[k] > 0;
+    total_bits += coded ? key_bits[k] : 0;
+  }
+  bool ucols_ok = true;  // the small kernel loads at most 8 distinct argument columns
+  p.n_ucols = 0;
+  for (int a = 0; a < n_aggs; a++)
+    for (int j = 0; j < 3; j++) {
+      p.uidx[a][j] = -1;
+      const int need = aggs[a].kind == DDQ_AGG_COUNT ? 0 : aggs[a].kind == DDQ_AGG_SUM ? 1
+                     : aggs[a].kind == DDQ_AGG_SUM_MUL_100M_100P ? 3 : 2;
+      if (j >= need) continue;
+      int c = 0;
+      while (c < p.n_ucols && !(p.ucol[c] == aggs[a].arg[j] && p.uwidth[c] == aggs[a].width[j])) c++;
+      if (c == p.n_ucols) {
+        if (c == 8) {
+          ucols_ok = false;
+          continue;
+        }
+        p.ucol[c] = aggs[a].arg[j];
+        p.uwidth[c] = aggs[a].width[j];
+        p.n_ucols++;
+      }
+      p.uidx[a][j] = c;
+    }
+  if (ucols_ok && coded && total_bits <= 6 && (n_aggs << total_bits) <= GBS_MAX_DA && p.tids != nullptr) {
+    const uint32_t D = 1u << total_bits;
+    const size_t smem = (size_t)D * n_aggs * (GBS_THREADS * 8 + 16) + 16;
+    static int occs = 0;
+    if (!occs) {
+      cudaFuncSetAttribute(groupby_small_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                           GBS_MAX_DA * (GBS_THREADS * 8 + 16) + 16);
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occs, groupby_small_kernel, GBS_THREADS,
+                                                    GBS_MAX_DA * (GBS_THREADS * 8 + 16) + 16);
+      if (occs < 1) occs = 1;
+    }
+    const int64_t want = (n_cap + GBS_THREADS * GBS_ROWS - 1) / (GBS_THREADS * GBS_ROWS);
+    const int64_t maxb = (int64_t)num_sms() * occs;
+    const int grid = (int)(want < 1 ? 1 : (want > maxb ? maxb : want));
+    groupby_small_kernel<<<grid, GBS_THREADS, smem, st>>>(p, D);
+    return cudaGetLastError();
+  }
   uint32_t S = 1u << 12;
   while (S > 64 && (size_t)S * (8 + 16 * (size_t)n_aggs) > GB_SMEM_BUDGET) S >>= 1;
   // no point in a CTA table larger than the global one

@@ -668,6 +668,13 @@ cudaError_t launch_scan(const FilterArgs& a, cudaStream_t st) {
   // at-TID ops -- the 85-register cap of G=3 serialises the gathers; so did a
   // software-pipelined one-tile-ahead gather at G=2: spills, 1915 us)
   int G = tids ? 2 : 4, S = 4;
+  {
+    static const char* env = getenv("DDQ_SCAN_SMALL");
+    if (env && a.n_cap <= atoll(env)) {
+      G = 1;
+      S = 2;
+    }
+  }
   auto need = [&](int gg, int ss) { return shared + (size_t)gg * ((size_t)ss * p.stage_bytes + list_bytes); };
   while (G > 1 && need(G, min_s) > budget) G--;
   while (S > min_s && need(G, S) > budget) S--;

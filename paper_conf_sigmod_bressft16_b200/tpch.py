@@ -49,7 +49,8 @@ def tpch_plan(db: Database, q: str, limit: int = 0) -> PlanBuilder:
                           (A.AGG_SUM_MUL_100M, ["l_extendedprice", "l_discount"]),
                           (A.AGG_SUM_MUL_100M_100P, ["l_extendedprice", "l_discount", "l_tax"]),
                           (A.AGG_SUM, ["l_discount"]), (A.AGG_COUNT, [])],
-                    order_by=[1, 2], max_groups=6)
+                    order_by=[1, 2], max_groups=6,
+                    key_bits=[2, 1])  # dictionary codes: returnflag A/N/R, linestatus F/O
         return P
     if q == "tpch6":
         # shipdate in 1994 (15 %) first; discount 0.05..0.07 and quantity < 24 at its TIDs

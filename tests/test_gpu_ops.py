@@ -254,6 +254,43 @@ def test_groupby_few_groups_int128_exact(ops, nkeys):
         assert got[i, 1] == int(m.sum())
 
 
+@pytest.mark.parametrize("n", [1, 517, 2_000_003])
+@pytest.mark.parametrize("bits", [(1,), (2, 1), (3, 2, 1)])
+def test_groupby_small_domain_exact(ops, n, bits):
+    """Dictionary-coded keys with sum(key_bits) <= 6: the small-domain kernel
+    (thread-private int64 partials in smem, overflow spills to int128) must give
+    the exact per-group sums, only for groups that occur (tids: every 3rd row)."""
+    from paper_conf_sigmod_bressft16_b200 import _abi as A
+    rng = np.random.default_rng(n + len(bits))
+    N = 3 * n + 7
+    tids = np.arange(0, 3 * n, 3, dtype=np.int32)
+    nk = len(bits)
+    codes = [rng.integers(0, max(1, (1 << b) - 1), N if k else n, dtype=np.int32) for k, b in enumerate(bits)]
+    big = rng.integers(2**61, 2**62, N, dtype=np.int64) * rng.choice([-1, 1], N)
+    ep = rng.integers(1, 10**7, N, dtype=np.int64)
+    d = rng.integers(0, 11, N, dtype=np.int64)
+    t = rng.integers(0, 9, N, dtype=np.int64)
+    aggs = [(A.AGG_SUM, [_t(big)]), (A.AGG_COUNT, []), (A.AGG_SUM_MUL_100M_100P, [_t(ep), _t(d), _t(t)])]
+    keys, accs, err = ops.groupby(_t(tids), ops.count_cell(n), n, key_vecs=[_t(codes[0])] + [None] * (nk - 1),
+                                  key_cols=[None] + [_t(c) for c in codes[1:]], aggs=aggs, capacity=128,
+                                  key_bits=list(bits))
+    assert err == 0
+    r = tids
+    key = codes[0].astype(np.int64)
+    sh = bits[0]
+    for k in range(1, nk):
+        key = key | (codes[k][r].astype(np.int64) << sh)
+        sh += bits[k]
+    got = _acc_to_int(accs)
+    keys = keys.cpu().numpy()
+    assert sorted(keys.tolist()) == sorted(set(key.tolist()))
+    vals = [big[r].astype(object), np.ones(n, dtype=object), ep[r].astype(object) * (100 - d[r]) * (100 + t[r])]
+    for i, kk in enumerate(keys):
+        m = key == kk
+        for a, v in enumerate(vals):
+            assert got[i, a] == sum(v[m]), (kk, a)
+
+
 def test_groupby_overflow_flagged(ops):
     from paper_conf_sigmod_bressft16_b200 import _abi as A
     n = 10_000

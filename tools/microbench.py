@@ -51,6 +51,14 @@ def main():
         ms = timeit(sel(col, lo, hi))
         gb = n * col.element_size() / 1e9
         print(f"select {name:14s} {ms*1e3:8.1f} us  {gb/ms*1e3:8.1f} GB/s (input only)", flush=True)
+    for small in (2556, 40_000, 600_000):
+        if only and only != "small":
+            break
+        ms = timeit(lambda: ops.check(ops.lib().ddq_op_select(ops._dev_preds([(c32, 1, 120000)]), 1, None, None, small,
+                                                               None, None, 0, out.data_ptr(), cnt.data_ptr(),
+                                                               scratch.data_ptr(), scratch.numel(), ops._stream())),
+                    reps=50)
+        print(f"select i32 n={small:8d} {ms*1e3:8.1f} us", flush=True)
     for rng_keys, frac in ((600_000, 0.2), (600_000, 0.05), (1_000_000, 0.04)):
         fk = c32 if rng_keys == 600_000 else torch.randint(1, rng_keys + 1, (n,), device="cuda", dtype=torch.int32,
                                                            generator=g)
