@@ -62,6 +62,7 @@ static std::vector<int> op_columns(const ddq_op& op) {
     case DDQ_OP_HASH_BUILD:
       c.push_back(op.key_col);
       if (op.payload_col >= 0) c.push_back(op.payload_col);
+      for (int i = 0; i < op.n_preds; i++) c.push_back(op.preds[i].column);  // fused selection
       break;
     case DDQ_OP_HASH_PROBE:
       if (op.fk_vec <= 0) c.push_back(op.fk_col);
@@ -467,8 +468,23 @@ ddq_status run_host_op(ddq_db* db, const ddq_op& op, const std::vector<Inter>& I
       int lg = 0;
       while ((1ll << lg) < cap) lg++;
       auto t = std::make_shared<std::vector<uint64_t>>((size_t)cap, kHostEmpty);
+      std::vector<const Column*> bpc;  // fused selection (BUILD op with predicates)
+      for (int p = 0; p < op.n_preds; p++) bpc.push_back(col_of(db, op.preds[p].column));
       for (int64_t i = 0; i < n; i++) {
         int32_t r = row_of(i);
+        bool ok = true;
+        for (int p = 0; p < op.n_preds && ok; p++) {
+          const int64_t v = hcol(bpc[(size_t)p], r);
+          const ddq_pred& pr = op.preds[p];
+          if (pr.kind == DDQ_PRED_RANGE) {
+            ok = v >= pr.lo && v <= pr.hi;
+          } else {
+            bool m = false;
+            for (int j = 0; j < pr.n_in; j++) m |= v == pr.in_vals[j];
+            ok = m;
+          }
+        }
+        if (!ok) continue;
         int32_t k = ((const int32_t*)kc->host)[r];
         int32_t v = pc ? ((const int32_t*)pc->host)[r] : r;
         uint32_t h = host_hash32(k, 32 - lg);

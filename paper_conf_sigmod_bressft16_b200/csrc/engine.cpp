@@ -350,6 +350,26 @@ ddq_status run_gpu_op(GpuOpCtx& ctx, const ddq_op& op, Inter& out) {
         if (!payload) return set_error(DDQ_ESTATE, "build: payload column not cached on the GPU");
       }
       if (!keys) return set_error(DDQ_ESTATE, "build: key column not cached on the GPU");
+      // fused selection (BUILD op with predicates): evaluated per input row in the
+      // build kernel
+      if (op.n_preds < 0 || op.n_preds > DDQ_MAX_PREDS) return set_error(DDQ_EINVAL, "build: bad n_preds");
+      BuildPreds bp;
+      bp.n = op.n_preds;
+      for (int i = 0; i < op.n_preds; i++) {
+        const ddq_pred& p = op.preds[i];
+        const Column* c = col_of(db, p.column);
+        if (!c || c->table != op.table) return set_error(DDQ_EINVAL, "build: predicate column not in table");
+        ddq_dev_pred& d = bp.p[i];
+        std::memset(&d, 0, sizeof(d));
+        d.col = need_col(p.column);
+        if (!d.col) return set_error(DDQ_ESTATE, "build: predicate column not cached on the GPU");
+        d.width = c->width;
+        d.kind = p.kind;
+        d.lo = p.lo;
+        d.hi = p.hi;
+        d.n_in = p.n_in;
+        for (int j = 0; j < DDQ_MAX_IN; j++) d.in_vals[j] = p.in_vals[j];
+      }
       if (use_join_index(*kc, T.n_rows)) {  // compact key range: direct-mapped join index
         out.jmin = (int32_t)kc->vmin;
         out.jrange = (uint32_t)(kc->vmax - kc->vmin + 1);
@@ -361,7 +381,7 @@ ddq_status run_gpu_op(GpuOpCtx& ctx, const ddq_op& op, Inter& out) {
         cudaError_t e = cudaMemsetAsync(out.jidx, 0, ((size_t)out.jrange + 31) / 32 * 4, st);
         if (e == cudaSuccess)
           e = launch_join_index_build(keys, payload, in_tids, in_cnt, in_cap, out.jmin, out.jrange, out.jidx,
-                                      out.d_error, st);
+                                      out.d_error, st, &bp);
         return cuda_status(e, "join_index_build");
       }
       // sparse keys: open addressing; small tables (shared-memory resident) get load <= 0.25
@@ -376,7 +396,8 @@ ddq_status run_gpu_op(GpuOpCtx& ctx, const ddq_op& op, Inter& out) {
       cudaMemsetAsync(out.d_error, 0, 4, st);
       cudaError_t e = launch_hash_init(out.table_ptr, out.table_cap, st);
       if (e == cudaSuccess)
-        e = launch_hash_build(keys, payload, in_tids, in_cnt, in_cap, out.table_ptr, out.table_cap, out.d_error, st);
+        e = launch_hash_build(keys, payload, in_tids, in_cnt, in_cap, out.table_ptr, out.table_cap, out.d_error, st,
+                              &bp);
       return cuda_status(e, "hash_build");
     }
     case DDQ_OP_GATHER: {
@@ -949,7 +970,11 @@ void count_accesses(ddq_db* db, const ddq_op& op) {
     case DDQ_OP_SELECT:
       for (int i = 0; i < op.n_preds; i++) touch(op.preds[i].column);
       break;
-    case DDQ_OP_HASH_BUILD: touch(op.key_col); touch(op.payload_col); break;
+    case DDQ_OP_HASH_BUILD:
+      touch(op.key_col);
+      touch(op.payload_col);
+      for (int i = 0; i < op.n_preds; i++) touch(op.preds[i].column);
+      break;
     case DDQ_OP_HASH_PROBE: touch(op.fk_col); break;
     case DDQ_OP_GATHER: touch(op.gather_col); break;
     case DDQ_OP_STAR:
@@ -1165,6 +1190,7 @@ int32_t ddq_prepared_profile(ddq_prepared* p, void* stream, int32_t max_ops, flo
       case DDQ_OP_HASH_BUILD:
         cls = 2;
         bytes = m * 4 * (op.payload_col >= 0 ? 2 : 1) + (double)o.table_cap * 8 * 2;
+        for (int k = 0; k < op.n_preds; k++) bytes += m * width(op.preds[k].column);  // fused selection
         break;
       case DDQ_OP_GATHER:
         cls = 3;

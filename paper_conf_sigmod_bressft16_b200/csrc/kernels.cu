@@ -29,6 +29,22 @@ int num_sms() {
 static inline uint32_t read_count_host_cap(int64_t n_cap) { return (uint32_t)n_cap; }
 
 // ----------------------------------------------------------------- hash build
+__device__ __forceinline__ bool build_row_passes(const BuildPreds& bp, int32_t r) {
+  for (int i = 0; i < bp.n; i++) {
+    const ddq_dev_pred& p = bp.p[i];
+    const int64_t v = col_at(p.col, p.width, r);
+    bool m = false;
+    if (p.kind == DDQ_PRED_RANGE) {
+      m = v >= p.lo && v <= p.hi;
+    } else {
+#pragma unroll
+      for (int j = 0; j < DDQ_MAX_IN; j++) m |= j < p.n_in && v == p.in_vals[j];
+    }
+    if (!m) return false;
+  }
+  return true;
+}
+
 __global__ void hash_init_kernel(uint64_t* table, uint32_t capacity) {
   for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < capacity; i += gridDim.x * blockDim.x)
     table[i] = HT_EMPTY;
@@ -37,11 +53,12 @@ __global__ void hash_init_kernel(uint64_t* table, uint32_t capacity) {
 __global__ void hash_build_kernel(const int32_t* __restrict__ keys, const int32_t* __restrict__ payload,
                                   const int32_t* __restrict__ in_tids, const uint32_t* d_in_count,
                                   uint32_t n_static, uint64_t* table, uint32_t capacity, int shift,
-                                  uint32_t* d_error) {
+                                  uint32_t* d_error, const __grid_constant__ BuildPreds bp) {
   const uint32_t n = d_in_count ? ld_relaxed_u32(d_in_count) : n_static;
   const uint32_t mask = capacity - 1;
   for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
     const int32_t r = in_tids ? in_tids[i] : (int32_t)i;
+    if (bp.n && !build_row_passes(bp, r)) continue;
     const int32_t k = keys[r];
     const int32_t v = payload ? payload[r] : r;
     if (k == INT32_MIN) {
@@ -78,13 +95,14 @@ cudaError_t launch_hash_init(uint64_t* table, uint32_t capacity, cudaStream_t st
 
 cudaError_t launch_hash_build(const int32_t* keys, const int32_t* payload, const int32_t* in_tids,
                               const uint32_t* d_in_count, int64_t n_cap, uint64_t* table, uint32_t capacity,
-                              uint32_t* d_error, cudaStream_t st) {
+                              uint32_t* d_error, cudaStream_t st, const BuildPreds* preds) {
   int lg = 0;
   while ((1u << lg) < capacity) lg++;
   int64_t g = (n_cap + 255) / 256;
   int grid = (int)(g > num_sms() * 8 ? num_sms() * 8 : (g < 1 ? 1 : g));
+  const BuildPreds bp = preds ? *preds : BuildPreds{};
   hash_build_kernel<<<grid, 256, 0, st>>>(keys, payload, in_tids, d_in_count, read_count_host_cap(n_cap), table,
-                                          capacity, 32 - lg, d_error);
+                                          capacity, 32 - lg, d_error, bp);
   return cudaGetLastError();
 }
 
@@ -96,10 +114,11 @@ size_t join_index_bytes(uint32_t range) {
 __global__ void join_index_build_kernel(const int32_t* __restrict__ keys, const int32_t* __restrict__ payload,
                                         const int32_t* __restrict__ in_tids, const uint32_t* d_in_count,
                                         uint32_t n_static, int32_t key_min, uint32_t range, uint32_t* bitmap,
-                                        int32_t* payarr, uint32_t* d_error) {
+                                        int32_t* payarr, uint32_t* d_error, const __grid_constant__ BuildPreds bp) {
   const uint32_t n = d_in_count ? ld_relaxed_u32(d_in_count) : n_static;
   for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
     const int32_t r = in_tids ? in_tids[i] : (int32_t)i;
+    if (bp.n && !build_row_passes(bp, r)) continue;
     const uint32_t o = (uint32_t)(keys[r] - key_min);
     if (o >= range) {
       atomicMax(d_error, 3u);
@@ -113,11 +132,13 @@ __global__ void join_index_build_kernel(const int32_t* __restrict__ keys, const 
 
 cudaError_t launch_join_index_build(const int32_t* keys, const int32_t* payload, const int32_t* in_tids,
                                     const uint32_t* d_in_count, int64_t n_cap, int32_t key_min, uint32_t range,
-                                    void* index, uint32_t* d_error, cudaStream_t st) {
+                                    void* index, uint32_t* d_error, cudaStream_t st, const BuildPreds* preds) {
+  const BuildPreds bp = preds ? *preds : BuildPreds{};
   int64_t g = (n_cap + 255) / 256;
   int grid = (int)(g > num_sms() * 8 ? num_sms() * 8 : (g < 1 ? 1 : g));
   join_index_build_kernel<<<grid, 256, 0, st>>>(keys, payload, in_tids, d_in_count, (uint32_t)n_cap, key_min, range,
-                                                join_index_bitmap(index), join_index_payload(index, range), d_error);
+                                                join_index_bitmap(index), join_index_payload(index, range), d_error,
+                                                bp);
   return cudaGetLastError();
 }
 

@@ -44,10 +44,18 @@ bool scan_supported(const FilterArgs& a);
 cudaError_t launch_scan(const FilterArgs& a, cudaStream_t st);
 cudaError_t launch_filter(const FilterArgs& a, cudaStream_t st);
 
+// HASH_BUILD with a fused selection (a BUILD op carrying predicates): rows that
+// fail any predicate are not inserted -- the select -> build pair of a dimension
+// table in one kernel, without the intermediate TID list.
+struct BuildPreds {
+  int32_t n = 0;
+  ddq_dev_pred p[DDQ_MAX_PREDS];
+};
+
 cudaError_t launch_hash_init(uint64_t* table, uint32_t capacity, cudaStream_t st);
 cudaError_t launch_hash_build(const int32_t* keys, const int32_t* payload, const int32_t* in_tids,
                               const uint32_t* d_in_count, int64_t n_cap, uint64_t* table, uint32_t capacity,
-                              uint32_t* d_error, cudaStream_t st);
+                              uint32_t* d_error, cudaStream_t st, const BuildPreds* preds = nullptr);
 cudaError_t launch_star(const ddq_dev_term* terms, int n_terms, int64_t n_rows, int32_t* out_tids,
                         uint32_t* d_out_count, int64_t out_cap, uint32_t* d_overflow, cudaStream_t st);
 
@@ -58,7 +66,8 @@ inline int32_t* join_index_payload(void* idx, uint32_t range) {
 }
 cudaError_t launch_join_index_build(const int32_t* keys, const int32_t* payload, const int32_t* in_tids,
                                     const uint32_t* d_in_count, int64_t n_cap, int32_t key_min, uint32_t range,
-                                    void* index, uint32_t* d_error, cudaStream_t st);
+                                    void* index, uint32_t* d_error, cudaStream_t st,
+                                    const BuildPreds* preds = nullptr);
 cudaError_t launch_gather(const void* col, int width, const int32_t* tids, const uint32_t* d_count,
                           int64_t n_cap, void* out, cudaStream_t st);
 

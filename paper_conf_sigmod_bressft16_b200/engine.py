@@ -77,6 +77,10 @@ class PlanBuilder:
     def select(self, table: str, preds: list, input: int = -1) -> int:
         """preds: list of (column, lo, hi) ranges or (column, [values]) IN-sets."""
         idx, op = self._op(A.OP_SELECT, table, input)
+        self._preds(op, table, preds)
+        return idx
+
+    def _preds(self, op, table: str, preds: list):
         if len(preds) > A.MAX_PREDS:
             raise ValueError("too many predicates")
         op.n_preds = len(preds)
@@ -92,12 +96,16 @@ class PlanBuilder:
                 pr.kind, pr.n_in = A.PRED_IN, len(vals)
                 for j, v in enumerate(vals):
                     pr.in_vals[j] = int(v)
-        return idx
 
-    def build(self, table: str, key: str, payload: str | None = None, input: int = -1) -> int:
+    def build(self, table: str, key: str, payload: str | None = None, input: int = -1,
+              where: list | None = None) -> int:
+        """where: predicates evaluated on the input rows inside the build (a fused
+        selection: no intermediate TID list), same forms as select()."""
         idx, op = self._op(A.OP_HASH_BUILD, table, input)
         op.key_col = self.db.col(table, key)
         op.payload_col = self.db.col(table, payload) if payload else -1
+        if where:
+            self._preds(op, table, where)
         return idx
 
     def probe(self, table: str, fk, build: int, input: int = -1, emit: bool = False) -> int:

@@ -50,13 +50,19 @@ def _oracle(kind, q):
     return norm(q, oracle.run(_data(kind), q))
 
 
-@pytest.mark.parametrize("star", [True, False], ids=["star", "chain"])
+VARIANTS = {"star": dict(star=True), "chain": dict(star=False),
+            "chain_unfused": dict(star=False, fused_build=False)}
+
+
+@pytest.mark.parametrize("variant", list(VARIANTS))
 @pytest.mark.parametrize("kind", ["1", "planted", "0.01"])
 @pytest.mark.parametrize("q", oracle.SSB_QUERIES)
-def test_ssb_prepared_graph_equals_oracle(kind, q, star):
+def test_ssb_prepared_graph_equals_oracle(kind, q, variant):
+    """star: one STAR operator; chain: binary operators, dimension selections fused
+    into their builds; chain_unfused: SELECT -> BUILD on every dimension."""
     from paper_conf_sigmod_bressft16_b200.ssb import ssb_plan
     db = _db(kind)
-    p = db.prepare(ssb_plan(db, q, star=star), use_graph=True)
+    p = db.prepare(ssb_plan(db, q, **VARIANTS[variant]), use_graph=True)
     want = _oracle(kind, q)
     for _ in range(2):  # relaunch of the same graph is deterministic
         p.launch()
@@ -65,13 +71,13 @@ def test_ssb_prepared_graph_equals_oracle(kind, q, star):
     p.close()
 
 
-@pytest.mark.parametrize("star", [True, False], ids=["star", "chain"])
+@pytest.mark.parametrize("variant", list(VARIANTS))
 @pytest.mark.parametrize("kind", ["1", "planted"])
 @pytest.mark.parametrize("q", oracle.SSB_QUERIES)
-def test_ssb_submit_chopping_equals_oracle(kind, q, star):
+def test_ssb_submit_chopping_equals_oracle(kind, q, variant):
     from paper_conf_sigmod_bressft16_b200.ssb import ssb_plan
     db = _db(kind)
-    r = db.run(ssb_plan(db, q, star=star))
+    r = db.run(ssb_plan(db, q, **VARIANTS[variant]))
     assert norm(q, r.rows) == _oracle(kind, q)
     assert r.host_ops == 0 and r.aborts == 0  # hot cache: everything on the GPU
 
