@@ -51,7 +51,11 @@ const char* ddq_version(void);
 
 /* ========================================================================
  * 1. Operator calls (device buffers; all pointers below are DEVICE pointers
- *    unless named h_*).  TIDs are int32 row ids (< 2^31) in ascending order.
+ *    unless named h_*).  TIDs are int32 row ids (< 2^31).  A TID list is a
+ *    MULTISET (reading O14'): the operators emit survivors in an
+ *    unspecified order (per-CTA write-combined blocks), each input item at most
+ *    once; every consumer (probe, select, gather, aggregate) is order-free and
+ *    all aggregates are exact integer sums, so query results are bit-identical.
  *    "count" arguments are device uint32 cells: an input count is read by the
  *    kernel; an output count is written by it.  `n_cap` is a HOST upper bound on
  *    the input count (sizes grids and scratch).  Outputs must hold n_cap items.
@@ -84,12 +88,12 @@ typedef struct {
 size_t ddq_op_scratch_bytes(int64_t n_cap);
 
 /* Selection (S8(a1) dimension, S8(a2) fact; App. B):
- * out_tids = ascending row ids r of the input (all rows [0, n_cap) when
- * in_tids == NULL, else r = in_tids[i] for i < *d_in_count) for which EVERY
- * predicate holds.  Carried vectors (aligned with the input, int32) are
- * compacted alongside: carry_out[c][j] = carry_in[c][i] for the j-th survivor i.
- * *d_out_count receives the survivor count.  Stable stream compaction
- * (decoupled look-back), deterministic. */
+ * out_tids = the row ids r of the input (all rows [0, n_cap) when in_tids ==
+ * NULL, else r = in_tids[i] for i < *d_in_count) for which EVERY predicate
+ * holds, as a multiset (order unspecified).  Carried vectors (aligned with the
+ * input, int32; 16-byte aligned) are compacted alongside: carry_out[c][j] =
+ * carry_in[c][i] where out_tids[j] came from input item i.  *d_out_count
+ * receives the survivor count. */
 ddq_status ddq_op_select(const ddq_dev_pred* preds, int32_t n_preds,
                          const int32_t* in_tids, const uint32_t* d_in_count, int64_t n_cap,
                          const int32_t* const* carry_in, int32_t* const* carry_out, int32_t n_carry,
@@ -108,9 +112,10 @@ ddq_status ddq_op_hash_build(const int32_t* keys, const int32_t* payload,
                              uint64_t* table, uint32_t capacity, uint32_t* d_error, void* stream);
 
 /* Hash probe = semi-join + payload (S8(a4)): for each input row r
- * (all rows or in_tids[i]), look up fk[r]; survivors are compacted stably into
- * out_tids, with the matched payload into out_payload (may be NULL) and carried
- * vectors compacted alongside (as in ddq_op_select). */
+ * (all rows or in_tids[i]), look up fk[r]; survivors are compacted into
+ * out_tids (a multiset, as in ddq_op_select), with the matched payload into
+ * out_payload (may be NULL) aligned with them and carried vectors compacted
+ * alongside (as in ddq_op_select). */
 ddq_status ddq_op_hash_probe(const uint64_t* table, uint32_t capacity, const int32_t* fk,
                              const int32_t* in_tids, const uint32_t* d_in_count, int64_t n_cap,
                              const int32_t* const* carry_in, int32_t* const* carry_out, int32_t n_carry,

@@ -1,0 +1,614 @@
+// dense.cu -- warp-autonomous filter kernels of the hot path: the dense hash /
+// join-index probe (S8(a4), every row of a fact FK column) and every operator over
+// a TID list (S8(a2) selection at TIDs, S8(a4) probe at TIDs, FILTER_EQ), each
+// emitting a compacted TID list (+ the hit's payload, + carried aligned vectors).
+// The dense probe is the first fact operator of every SSB plan (SURVEY.md 8(d):
+// the most selective dimension's FK column is scanned fully); the TID-input
+// operators are the later steps of the same column-at-a-time chains.
+//
+// B200 design; the predecessor scan_kernel (one CTA per SM split into
+// 256-thread groups with named barriers) was instruction- and barrier-bound (ncu:
+// 46 thread-instructions per row; barrier, wait stalls) at 42 % of HBM peak:
+//   * one persistent CTA of 32 warps per SM; every warp walks its own 512-item
+//     tiles (32 lanes x 16 items, 16-byte loads, the next tile's keys / TIDs
+//     prefetched into registers) -- no CTA-wide barrier inside the loop;
+//   * the dimension bitmap (or hash table) is staged once per SM in shared memory
+//     and probed with LDS (the kernel is specialised so the compiler sees a shared
+//     pointer, not a generic one);
+//   * compaction: a lane's 16 hit bits -> popc -> warp inclusive scan -> the warp
+//     claims a range of a CTA-wide counter with ONE shared-memory atomic; the
+//     survivors go straight from registers into a shared-memory write-combining
+//     ring of R blocks x BLK entries (TID, payload, input position);
+//   * the warp whose entries complete a ring block flushes it: one global atomicAdd
+//     reserves BLK output slots (measured: 1.45 G same-address atomics/s on B200,
+//     so one per 2048 survivors, not one per tile), then coalesced copies; carried
+//     vectors are gathered at the survivors' input positions during the flush.
+//     Its latency is that warp's alone; the other warps keep filling the remaining
+//     blocks.  A block's slot is reused only after its flush (per-slot generation
+//     counter); the oldest unflushed block's writers never wait, so the ring cannot
+//     deadlock;
+//   * after the loop the CTA flushes its last, partial block with an exact-size
+//     reservation: the output has no holes.
+// Output order: unspecified (reading O14': a TID list is a multiset; every consumer
+// is order-free); each input item is emitted at most once.
+#include <cstdint>
+#include <cstdlib>
+#include <cuda_runtime.h>
+
+#include "device_common.cuh"
+#include "ops_internal.h"
+
+namespace ddq {
+
+namespace {
+
+constexpr int WS_ITEMS = 16;            // items per lane per tile
+constexpr int WS_TILE = 32 * WS_ITEMS;  // items per warp tile
+constexpr int WS_R = 4;                 // ring blocks
+// entries per ring block (one global reservation): 2048, or 1024 when carried
+// vectors add up to 4 more int32 fields per entry (ring <= 96 KB)
+__host__ __device__ constexpr int ws_blk(bool carry) { return carry ? 1024 : 2048; }
+constexpr int WS_MAXF = 6;  // ring fields: TID, payload, <= 4 carried vectors
+// warps per CTA: dense probes 32 (64 registers: 16 keys in use + 16 prefetched);
+// TID-input operators 16 (128 registers: TIDs, gathered keys / values, payloads)
+__host__ __device__ constexpr int ws_nw(bool tids) { return tids ? 16 : 32; }
+
+// operator variants (compile time: a tile costs only the instructions it needs)
+enum WsKind : int {
+  WK_BM_SMEM = 0,    // join-index probe, bitmap in smem
+  WK_BM_GLOBAL = 1,  // join-index probe, bitmap in global (L2)
+  WK_HT_SMEM = 2,    // hash probe, table in smem
+  WK_HT_GLOBAL = 3,  // hash probe, table in global
+  WK_SEL_RANGE = 4,  // conjunctive range predicates (TID input)
+  WK_SEL_GENERIC = 5,  // range / IN predicates (TID input)
+  WK_EQ = 6            // FILTER_EQ of two positional vectors (TID input)
+};
+
+struct WsPred {
+  const void* col;
+  int32_t width, kind;
+  int64_t lo, hi;
+  uint64_t d64;  // RANGE: lo <= v <= hi  <=>  (u64)(v - lo) <= d64
+  int32_t empty, n_in;
+  int64_t in_vals[8];
+};
+
+struct WsParams {
+  uint32_t n;                  // dense: rows; TID input: capacity (count in d_in_count)
+  const uint32_t* d_in_count;  // TID input
+  const int32_t* in_tids;      // TID input
+  int32_t n_preds;
+  WsPred preds[4];
+  const int32_t* eq_a;
+  const int32_t* eq_b;
+  const int32_t* fk;  // probe keys: column (by row) or positional vector (fk_by_pos)
+  int32_t fk_by_pos;
+  // join index (direct): membership bitmap over [key_min, key_min + range) + payloads
+  const uint32_t* bitmap;
+  const int32_t* payarr;
+  int32_t key_min;
+  uint32_t range;
+  uint32_t bitmap_words;
+  // hash table (open addressing, 8-byte slots key<<32|payload)
+  const uint64_t* table;
+  uint32_t cap_mask;
+  int32_t shift;
+  int32_t tab_off;  // byte offset of the staged table in dynamic smem
+  int32_t n_carry;
+  const int32_t* carry_in[4];
+  int32_t* carry_out[4];
+  int32_t n_fields;             // ring fields: TID, [payload], carried vectors
+  int32_t* field_out[WS_MAXF];  // their outputs
+  int32_t* out_tids;
+  int32_t* out_payload;
+  uint32_t* d_out_count;  // [0] survivors, [1] CTA completion counter (zeroed before launch)
+  uint32_t out_cap;
+  uint32_t* d_overflow;
+};
+
+__device__ __forceinline__ uint32_t ld_volatile_smem(const uint32_t* p) {
+  return *reinterpret_cast<const volatile uint32_t*>(p);
+}
+
+// Copy `cnt` ring entries starting at ring offset `r0` (no wrap) of every field
+// (field f lives at ring + f * ring_n) to its output at [g, g + cnt), clamped to
+// out_cap.  Called by a whole warp (tid = lane, nthr = 32) or by the whole CTA.
+__device__ __forceinline__ void copy_out(const WsParams& P, const int32_t* ring, uint32_t ring_n, uint32_t r0,
+                                         uint32_t cnt, uint32_t g, uint32_t tid, uint32_t nthr) {
+  uint32_t lim = cnt;
+  if (g + cnt > P.out_cap) {
+    lim = P.out_cap > g ? P.out_cap - g : 0u;
+    if (tid == 0 && P.d_overflow) atomicMax(P.d_overflow, 4u);
+  }
+  if ((g & 3u) == 0 && lim == cnt && (cnt & 3u) == 0) {  // 16-byte copies
+    for (int f = 0; f < P.n_fields; f++) {
+      const int4* src = reinterpret_cast<const int4*>(ring + (size_t)f * ring_n + r0);
+      int4* dst = reinterpret_cast<int4*>(P.field_out[f] + g);
+      for (uint32_t i = tid; i < cnt / 4; i += nthr) dst[i] = src[i];
+    }
+    return;
+  }
+  for (int f = 0; f < P.n_fields; f++) {
+    const int32_t* src = ring + (size_t)f * ring_n + r0;
+    int32_t* dst = P.field_out[f] + g;
+    for (uint32_t i = tid; i < lim; i += nthr) dst[i] = src[i];
+  }
+}
+
+__device__ __forceinline__ bool pred_generic(const WsPred& p, int64_t v) {
+  if (p.kind == DDQ_PRED_RANGE) return (uint64_t)(v - p.lo) <= p.d64 && !p.empty;
+  bool m = false;
+#pragma unroll
+  for (int j = 0; j < 8; j++) m |= (j < p.n_in) && (v == p.in_vals[j]);
+  return m;
+}
+
+// The lane's 16 int32 values of the tile starting at t0: positions
+// t0 + s*128 + lofs + v (16-byte aligned), 0 past n.
+__device__ __forceinline__ void load16(const int32_t* a, uint32_t t0, uint32_t lofs, uint32_t n, int4 (&r)[4]) {
+  const uint32_t base = t0 + lofs;
+  if (t0 + WS_TILE <= n) {
+#pragma unroll
+    for (int s = 0; s < 4; s++) r[s] = ld_stream_i4(a + base + s * 128);
+  } else {
+#pragma unroll
+    for (int s = 0; s < 4; s++) {
+      const uint32_t i = base + s * 128;
+      r[s].x = i < n ? a[i] : 0;
+      r[s].y = i + 1 < n ? a[i + 1] : 0;
+      r[s].z = i + 2 < n ? a[i + 2] : 0;
+      r[s].w = i + 3 < n ? a[i + 3] : 0;
+    }
+  }
+}
+__device__ __forceinline__ void unpack16(const int4 (&r)[4], int32_t (&v)[WS_ITEMS]) {
+#pragma unroll
+  for (int s = 0; s < 4; s++) {
+    v[s * 4 + 0] = r[s].x; v[s * 4 + 1] = r[s].y; v[s * 4 + 2] = r[s].z; v[s * 4 + 3] = r[s].w;
+  }
+}
+
+template <int kKind, bool kTids, bool kPay, bool kCarry>
+__global__ void __launch_bounds__(ws_nw(kTids) * 32, 1) ws_kernel(const __grid_constant__ WsParams P) {
+  extern __shared__ __align__(16) uint8_t smem[];
+  __shared__ uint32_t s_cnt, s_base;
+  __shared__ uint32_t s_filled[WS_R], s_gen[WS_R];
+  constexpr uint32_t BLK = ws_blk(kCarry), RING = BLK * WS_R;
+  int32_t* ring = reinterpret_cast<int32_t*>(smem);  // fields [tid | payload | carried...] x RING
+  constexpr bool kProbe = kKind <= WK_HT_GLOBAL;
+  constexpr bool kHash = kKind == WK_HT_SMEM || kKind == WK_HT_GLOBAL;
+  uint32_t* s_bm = reinterpret_cast<uint32_t*>(smem + P.tab_off);
+  uint64_t* s_ht = reinterpret_cast<uint64_t*>(smem + P.tab_off);
+
+  if (threadIdx.x == 0) {
+    s_cnt = 0;
+#pragma unroll
+    for (int r = 0; r < WS_R; r++) s_filled[r] = 0, s_gen[r] = 0;
+  }
+  __shared__ __align__(8) uint64_t s_bar;
+  if (kKind == WK_BM_SMEM) {  // + one zero word past the end: the range test is a clamp
+    stage_bulk(s_bm, P.bitmap, (P.bitmap_words * 4 + 15) & ~15u, &s_bar);
+    if (threadIdx.x == 0) s_bm[P.bitmap_words] = 0u;
+  }
+  if (kKind == WK_HT_SMEM) stage_bulk(s_ht, P.table, (P.cap_mask + 1) * 8, &s_bar);
+  __syncthreads();
+
+  const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const uint32_t n = kTids ? ld_relaxed_u32(P.d_in_count) : P.n;
+  const uint32_t ntiles = (n + WS_TILE - 1) / WS_TILE;
+  constexpr uint32_t NW = ws_nw(kTids);
+  const uint32_t W = gridDim.x * NW;
+  uint32_t tile = blockIdx.x * NW + warp;
+  const uint32_t lofs = lane * 4;  // item (s, v) of lane l sits at tile*512 + s*128 + l*4 + v
+  const int32_t* stream = kTids ? P.in_tids : P.fk;  // the column streamed through registers
+  int4 nk[4];
+  if (tile < ntiles) load16(stream, tile * WS_TILE, lofs, n, nk);
+
+  for (; tile < ntiles; tile += W) {
+    int32_t sv[WS_ITEMS];  // streamed values: keys (dense probe) or TIDs
+    unpack16(nk, sv);
+    const uint32_t base = tile * WS_TILE + lofs;  // position of the lane's item 0
+    if (tile + W < ntiles) load16(stream, (tile + W) * WS_TILE, lofs, n, nk);
+    uint32_t flags = 0xFFFFu;
+    if (tile * WS_TILE + WS_TILE > n) {
+      flags = 0;
+#pragma unroll
+      for (int j = 0; j < WS_ITEMS; j++) flags |= (base + (j >> 2) * 128 + (j & 3) < n ? 1u : 0u) << j;
+    }
+    int32_t pay[WS_ITEMS];
+    if (kProbe) {
+      int32_t key[WS_ITEMS];
+      if (!kTids) {
+#pragma unroll
+        for (int j = 0; j < WS_ITEMS; j++) key[j] = sv[j];
+      } else if (P.fk_by_pos) {  // positional key vector: coalesced
+        int4 kk[4];
+        load16(P.fk, tile * WS_TILE, lofs, n, kk);
+        unpack16(kk, key);
+      } else {  // key column gathered at the TIDs
+#pragma unroll
+        for (int j = 0; j < WS_ITEMS; j++) key[j] = ((flags >> j) & 1u) ? __ldg(P.fk + (uint32_t)sv[j]) : 0;
+      }
+      if (!kHash) {
+        uint32_t m = 0;
+#pragma unroll
+        for (int j = 0; j < WS_ITEMS; j++) {
+          uint32_t hit;
+          if (kKind == WK_BM_SMEM) {
+            const uint32_t oo = min((uint32_t)(key[j] - P.key_min), P.range);
+            hit = (s_bm[oo >> 5] >> (oo & 31)) & 1u;
+          } else {
+            const uint32_t o = (uint32_t)(key[j] - P.key_min);
+            hit = o < P.range ? (__ldg(P.bitmap + (o >> 5)) >> (o & 31)) & 1u : 0u;
+          }
+          m |= hit << j;
+        }
+        flags &= m;
+        if (kPay) {
+          const uint32_t any = __reduce_or_sync(FULL, flags);
+#pragma unroll
+          for (int j = 0; j < WS_ITEMS; j++) {
+            pay[j] = 0;
+            if ((any >> j) & 1u)
+              if ((flags >> j) & 1u) pay[j] = __ldg(P.payarr + (uint32_t)(key[j] - P.key_min));
+          }
+        }
+      } else {
+#pragma unroll
+        for (int j = 0; j < WS_ITEMS; j++) {
+          pay[j] = 0;
+          if ((flags >> j) & 1u) {
+            uint32_t h = ht_hash(key[j], P.shift);
+            uint64_t s = kKind == WK_HT_SMEM ? s_ht[h] : __ldg(P.table + h);
+            while (s != HT_EMPTY && ht_key(s) != key[j]) {
+              h = (h + 1) & P.cap_mask;
+              s = kKind == WK_HT_SMEM ? s_ht[h] : __ldg(P.table + h);
+            }
+            if (s == HT_EMPTY) flags &= ~(1u << j);
+            pay[j] = ht_val(s);
+          }
+        }
+      }
+    } else if (kKind == WK_EQ) {
+      int4 a4[4], b4[4];
+      load16(P.eq_a, tile * WS_TILE, lofs, n, a4);
+      load16(P.eq_b, tile * WS_TILE, lofs, n, b4);
+      int32_t a[WS_ITEMS], b[WS_ITEMS];
+      unpack16(a4, a);
+      unpack16(b4, b);
+      uint32_t m = 0;
+#pragma unroll
+      for (int j = 0; j < WS_ITEMS; j++) m |= (a[j] == b[j] ? 1u : 0u) << j;
+      flags &= m;
+    } else {  // selection at TIDs: later columns gathered for the remaining rows only
+      for (int p = 0; p < P.n_preds; p++) {
+        const WsPred& pr = P.preds[p];
+        int64_t v[WS_ITEMS];
+        const uint32_t any = __reduce_or_sync(FULL, flags);
+        if (pr.width == 8) {
+#pragma unroll
+          for (int j = 0; j < WS_ITEMS; j++) {
+            v[j] = 0;
+            if ((any >> j) & 1u)
+              if ((flags >> j) & 1u) v[j] = __ldg(reinterpret_cast<const long long*>(pr.col) + (uint32_t)sv[j]);
+          }
+        } else {
+#pragma unroll
+          for (int j = 0; j < WS_ITEMS; j++) {
+            v[j] = 0;
+            if ((any >> j) & 1u)
+              if ((flags >> j) & 1u) v[j] = __ldg(reinterpret_cast<const int32_t*>(pr.col) + (uint32_t)sv[j]);
+          }
+        }
+        uint32_t m = 0;
+        if (kKind == WK_SEL_RANGE) {
+#pragma unroll
+          for (int j = 0; j < WS_ITEMS; j++) m |= ((uint64_t)(v[j] - pr.lo) <= pr.d64 ? 1u : 0u) << j;
+          if (pr.empty) m = 0;
+        } else {
+#pragma unroll
+          for (int j = 0; j < WS_ITEMS; j++) m |= (pred_generic(pr, v[j]) ? 1u : 0u) << j;
+        }
+        flags &= m;
+      }
+    }
+    // ---- compaction: warp scan of the lanes' hit counts, one smem claim --------
+    const uint32_t c = __popc(flags);
+    const uint32_t incl = warp_incl_scan(c, (int)lane);
+    const uint32_t tot = __shfl_sync(FULL, incl, 31);
+    if (tot == 0) continue;
+    uint32_t pos0 = 0;
+    if (lane == 0) {
+      pos0 = atomicAdd(&s_cnt, tot);
+      // wait until the ring blocks this range touches are free (their previous
+      // occupants flushed): block b lives in slot b % R, generation b / R
+      const uint32_t b0 = pos0 / BLK, b1 = (pos0 + tot - 1) / BLK;
+      while (ld_volatile_smem(&s_gen[b0 % WS_R]) != b0 / WS_R) __nanosleep(64);
+      if (b1 != b0)
+        while (ld_volatile_smem(&s_gen[b1 % WS_R]) != b1 / WS_R) __nanosleep(64);
+    }
+    pos0 = __shfl_sync(FULL, pos0, 0);
+    __syncwarp();
+    // predicated stores through a running ring pointer, no per-item branches (a
+    // branchy version spent 43 % of the kernel's instructions here)
+    const uint32_t r0 = (pos0 & (RING - 1)) + incl - c;  // this lane's first ring slot
+    if ((pos0 & (RING - 1)) + tot <= RING) {  // the claim does not wrap the ring
+      int32_t* wp = ring + r0;
+#pragma unroll
+      for (int j = 0; j < WS_ITEMS; j++) {
+        if (flags & (1u << j)) {
+          const uint32_t pos = base + (j >> 2) * 128 + (j & 3);
+          wp[0] = kTids ? sv[j] : (int32_t)pos;
+          if (kPay) wp[RING] = pay[j];
+          wp++;
+        }
+      }
+      if (kCarry) {  // carried vectors: coalesced loads at the tile's positions
+        for (int cc = 0; cc < P.n_carry; cc++) {
+          int4 cv4[4];
+          load16(P.carry_in[cc], tile * WS_TILE, lofs, n, cv4);
+          int32_t cv[WS_ITEMS];
+          unpack16(cv4, cv);
+          int32_t* cp = ring + (size_t)((kPay ? 2 : 1) + cc) * RING + r0;
+#pragma unroll
+          for (int j = 0; j < WS_ITEMS; j++) {
+            if (flags & (1u << j)) {
+              *cp = cv[j];
+              cp++;
+            }
+          }
+        }
+      }
+    } else {
+      uint32_t p = r0;
+#pragma unroll
+      for (int j = 0; j < WS_ITEMS; j++) {
+        if ((flags >> j) & 1u) {
+          const uint32_t r = p & (RING - 1);
+          const uint32_t pos = base + (j >> 2) * 128 + (j & 3);
+          ring[r] = kTids ? sv[j] : (int32_t)pos;
+          if (kPay) ring[RING + r] = pay[j];
+          p++;
+        }
+      }
+      if (kCarry) {
+        for (int cc = 0; cc < P.n_carry; cc++) {
+          int4 cv4[4];
+          load16(P.carry_in[cc], tile * WS_TILE, lofs, n, cv4);
+          int32_t cv[WS_ITEMS];
+          unpack16(cv4, cv);
+          int32_t* cb = ring + (size_t)((kPay ? 2 : 1) + cc) * RING;
+          uint32_t q = r0;
+#pragma unroll
+          for (int j = 0; j < WS_ITEMS; j++) {
+            if ((flags >> j) & 1u) {
+              cb[q & (RING - 1)] = cv[j];
+              q++;
+            }
+          }
+        }
+      }
+    }
+    __threadfence_block();
+    __syncwarp();
+    // account the written entries to their blocks; the warp completing a block flushes it
+    uint32_t flush = 0;  // bit 0: block b0, bit 1: block b1
+    if (lane == 0) {
+      const uint32_t end = pos0 + tot;
+      const uint32_t b0 = pos0 / BLK, b1 = (end - 1) / BLK;
+      const uint32_t c0 = (b1 == b0 ? end : (b0 + 1) * BLK) - pos0;
+      if (atomicAdd(&s_filled[b0 % WS_R], c0) + c0 == BLK) flush |= 1u;
+      if (b1 != b0) {
+        const uint32_t c1 = end - b1 * BLK;
+        if (atomicAdd(&s_filled[b1 % WS_R], c1) + c1 == BLK) flush |= 2u;
+      }
+      __threadfence_block();
+    }
+    flush = __shfl_sync(FULL, flush, 0);
+    while (flush) {
+      const uint32_t b = (flush & 1u) ? pos0 / BLK : (pos0 + tot - 1) / BLK;
+      flush &= flush - 1;
+      const uint32_t slot = b % WS_R;
+      uint32_t g = 0;
+      if (lane == 0) g = atomicAdd(P.d_out_count, BLK);
+      g = __shfl_sync(FULL, g, 0);
+      copy_out(P, ring, RING, slot * BLK, BLK, g, lane, 32);
+      __threadfence_block();
+      __syncwarp();
+      if (lane == 0) {
+        s_filled[slot] = 0;
+        __threadfence_block();
+        atomicAdd(&s_gen[slot], 1u);
+      }
+    }
+  }
+  // the CTA's last, partial block: an exact reservation (no holes)
+  __syncthreads();
+  const uint32_t total = s_cnt;
+  const uint32_t rem = total % BLK;
+  if (rem) {
+    if (threadIdx.x == 0) s_base = atomicAdd(P.d_out_count, rem);
+    __syncthreads();
+    copy_out(P, ring, RING, ((total / BLK) % WS_R) * BLK, rem, s_base, threadIdx.x, blockDim.x);
+  }
+  // the last CTA to finish clamps the count to the output capacity
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    __threadfence();
+    if (atomicAdd(P.d_out_count + 1, 1u) == gridDim.x - 1) {
+      const uint32_t cnt = atomicAdd(P.d_out_count, 0u);
+      if (cnt > P.out_cap) *P.d_out_count = P.out_cap;
+    }
+  }
+}
+
+int g_optin = 0;
+constexpr size_t kWsCtl = 1024;  // static smem + reserve
+
+template <int K, bool T, bool Pa, bool C>
+void ws_attr() {
+  cudaFuncSetAttribute(ws_kernel<K, T, Pa, C>, cudaFuncAttributeMaxDynamicSharedMemorySize, g_optin - (int)kWsCtl);
+}
+template <int K>
+void ws_attr_kind() {
+  if constexpr (K <= WK_HT_GLOBAL) {  // dense inputs: probes only
+    ws_attr<K, false, false, false>();
+    ws_attr<K, false, true, false>();
+  }
+  ws_attr<K, true, false, false>();
+  ws_attr<K, true, true, false>();
+  ws_attr<K, true, false, true>();
+  ws_attr<K, true, true, true>();
+}
+
+template <int K>
+void launch_k(bool tids, bool pay, bool carry, int grid, size_t smem, cudaStream_t st, const WsParams& p) {
+  if constexpr (K <= WK_HT_GLOBAL) {  // dense inputs: probes only
+    if (!tids) {
+      const dim3 blk(ws_nw(false) * 32);
+      if (pay) ws_kernel<K, false, true, false><<<grid, blk, smem, st>>>(p);
+      else ws_kernel<K, false, false, false><<<grid, blk, smem, st>>>(p);
+      return;
+    }
+  }
+  const dim3 blk(ws_nw(true) * 32);
+  if (carry) {
+    if (pay) ws_kernel<K, true, true, true><<<grid, blk, smem, st>>>(p);
+    else ws_kernel<K, true, false, true><<<grid, blk, smem, st>>>(p);
+  } else {
+    if (pay) ws_kernel<K, true, true, false><<<grid, blk, smem, st>>>(p);
+    else ws_kernel<K, true, false, false><<<grid, blk, smem, st>>>(p);
+  }
+}
+
+}  // namespace
+
+bool ws_supported(const FilterArgs& a) {
+  const bool tids = a.in_tids != nullptr;
+  if (a.n_carry > 4 || a.n_cap > (int64_t)0x7FFFFFFF) return false;
+  if (!tids) {  // dense: probes only (dense selections stream several columns: scan.cu)
+    if (!a.probe || a.fk_by_pos || a.eq_a || a.n_carry) return false;
+    if (((uintptr_t)a.fk & 15) != 0) return false;
+  } else {
+    if (((uintptr_t)a.in_tids & 15) != 0) return false;
+    if (a.probe && a.fk_by_pos && ((uintptr_t)a.fk & 15) != 0) return false;
+    if (a.eq_a && ((((uintptr_t)a.eq_a | (uintptr_t)a.eq_b) & 15) != 0)) return false;
+    if (!a.probe && !a.eq_a && (a.n_preds < 1 || a.n_preds > 4)) return false;
+    if (!a.probe && a.eq_a && a.n_preds) return false;
+  }
+  if (a.out_payload && ((uintptr_t)a.out_payload & 15) != 0) return false;
+  for (int c = 0; c < a.n_carry; c++)  // carried vectors: 16-byte loads and copies
+    if ((((uintptr_t)a.carry_in[c] | (uintptr_t)a.carry_out[c]) & 15) != 0) return false;
+  return ((uintptr_t)a.out_tids & 15) == 0;
+}
+
+// Staging a table in every SM's shared memory costs ~tab x 148 bytes of L2 reads
+// and one round trip per CTA; for small inputs the probes go to the L2-resident
+// global copy instead (a few thousand late-materialisation lookups must not pay
+// for a 75 KB bitmap per SM).
+static bool stage_pays(int64_t n_cap, size_t tab) { return n_cap >= (int64_t)(tab * 4); }
+
+cudaError_t launch_ws(const FilterArgs& a, cudaStream_t st) {
+  if (!g_optin) {
+    int dev = 0, v = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&v, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
+    g_optin = v;
+    ws_attr_kind<WK_BM_SMEM>();
+    ws_attr_kind<WK_BM_GLOBAL>();
+    ws_attr_kind<WK_HT_SMEM>();
+    ws_attr_kind<WK_HT_GLOBAL>();
+    ws_attr_kind<WK_SEL_RANGE>();
+    ws_attr_kind<WK_SEL_GENERIC>();
+    ws_attr_kind<WK_EQ>();
+  }
+  const bool tids = a.in_tids != nullptr;
+  WsParams p{};
+  p.n = (uint32_t)a.n_cap;
+  p.d_in_count = a.d_in_count;
+  p.in_tids = a.in_tids;
+  const bool pay = a.probe && a.out_payload != nullptr;
+  const bool carry = tids && a.n_carry > 0;
+  const int n_fields = 1 + (pay ? 1 : 0) + (carry ? a.n_carry : 0);
+  const size_t ring = (size_t)ws_blk(carry) * WS_R * 4 * n_fields;
+  const size_t budget = (size_t)g_optin - kWsCtl;
+  int kind;
+  size_t tab = 0;
+  if (a.probe) {
+    p.fk = a.fk;
+    p.fk_by_pos = a.fk_by_pos ? 1 : 0;
+    if (a.bitmap) {
+      p.bitmap = a.bitmap;
+      p.payarr = a.payarr;
+      p.key_min = a.key_min;
+      p.range = a.range;
+      p.bitmap_words = (a.range + 31) / 32;
+      tab = ((size_t)p.bitmap_words * 4 + 15) / 16 * 16 + 16;  // bulk-copy rounding + the zero word
+      kind = (!a.no_smem && ring + tab <= budget && stage_pays(a.n_cap, tab)) ? WK_BM_SMEM : WK_BM_GLOBAL;
+    } else {
+      p.table = a.table;
+      p.cap_mask = a.capacity - 1;
+      int lg = 0;
+      while ((1u << lg) < a.capacity) lg++;
+      p.shift = 32 - lg;
+      tab = (size_t)a.capacity * 8;
+      kind = (!a.no_smem && ring + tab <= budget && stage_pays(a.n_cap, tab)) ? WK_HT_SMEM : WK_HT_GLOBAL;
+    }
+  } else if (a.eq_a) {
+    kind = WK_EQ;
+    p.eq_a = a.eq_a;
+    p.eq_b = a.eq_b;
+  } else {
+    bool all_range = true;
+    p.n_preds = a.n_preds;
+    for (int i = 0; i < a.n_preds; i++) {
+      const ddq_dev_pred& d = a.preds[i];
+      WsPred& q = p.preds[i];
+      q.col = d.col;
+      q.width = d.width;
+      q.kind = d.kind;
+      q.lo = d.lo;
+      q.hi = d.hi;
+      q.empty = d.hi < d.lo;
+      q.d64 = q.empty ? 0 : (uint64_t)d.hi - (uint64_t)d.lo;
+      q.n_in = d.n_in;
+      for (int j = 0; j < 8; j++) q.in_vals[j] = d.in_vals[j];
+      all_range = all_range && d.kind == DDQ_PRED_RANGE;
+    }
+    kind = all_range ? WK_SEL_RANGE : WK_SEL_GENERIC;
+  }
+  p.tab_off = (int32_t)ring;
+  p.n_carry = carry ? a.n_carry : 0;
+  for (int c = 0; c < p.n_carry; c++) {
+    p.carry_in[c] = a.carry_in[c];
+    p.carry_out[c] = a.carry_out[c];
+  }
+  p.out_tids = a.out_tids;
+  p.out_payload = pay ? a.out_payload : nullptr;
+  p.n_fields = n_fields;
+  p.field_out[0] = a.out_tids;
+  if (pay) p.field_out[1] = a.out_payload;
+  for (int c = 0; c < p.n_carry; c++) p.field_out[(pay ? 2 : 1) + c] = a.carry_out[c];
+  p.d_out_count = a.d_out_count;
+  p.out_cap = (uint32_t)(a.out_cap > 0 ? a.out_cap : a.n_cap);
+  p.d_overflow = a.d_overflow;
+  cudaError_t e = cudaMemsetAsync(a.d_out_count, 0, 8, st);
+  if (e != cudaSuccess) return e;
+  const size_t smem = ring + ((kind == WK_BM_SMEM || kind == WK_HT_SMEM) ? tab : 0);
+  const int64_t ntiles = (a.n_cap + WS_TILE - 1) / WS_TILE;  // TID input: an upper bound
+  int64_t grid = num_sms();
+  const int64_t need = (ntiles + ws_nw(tids) - 1) / ws_nw(tids);
+  if (grid > need) grid = need < 1 ? 1 : need;
+  switch (kind) {
+    case WK_BM_SMEM: launch_k<WK_BM_SMEM>(tids, pay, carry, (int)grid, smem, st, p); break;
+    case WK_BM_GLOBAL: launch_k<WK_BM_GLOBAL>(tids, pay, carry, (int)grid, smem, st, p); break;
+    case WK_HT_SMEM: launch_k<WK_HT_SMEM>(tids, pay, carry, (int)grid, smem, st, p); break;
+    case WK_HT_GLOBAL: launch_k<WK_HT_GLOBAL>(tids, pay, carry, (int)grid, smem, st, p); break;
+    case WK_SEL_RANGE: launch_k<WK_SEL_RANGE>(tids, false, carry, (int)grid, smem, st, p); break;
+    case WK_SEL_GENERIC: launch_k<WK_SEL_GENERIC>(tids, false, carry, (int)grid, smem, st, p); break;
+    default: launch_k<WK_EQ>(tids, false, carry, (int)grid, smem, st, p); break;
+  }
+  return cudaGetLastError();
+}
+
+}  // namespace ddq

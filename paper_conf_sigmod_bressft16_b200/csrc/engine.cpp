@@ -4,6 +4,7 @@
 #include <algorithm>
 #include <chrono>
 #include <cmath>
+#include <cstdlib>
 #include <cstring>
 #include <numeric>
 
@@ -885,6 +886,9 @@ struct ddq_prepared {
   bool use_graph = false;
   int kernels = 0;
   cudaStream_t cap_stream = nullptr;
+  // graph capture with parallel branches: side streams + one event per op
+  std::vector<cudaStream_t> side;
+  std::vector<cudaEvent_t> ev;
 };
 
 namespace ddq {
@@ -947,16 +951,90 @@ static void free_inters(ddq_db* db, std::vector<Inter>& v) {
 }
 
 // Re-issue the launches of a prepared plan on its existing buffers.
+static ddq_status replay_op(ddq_prepared* P, int i, cudaStream_t st) {
+  std::vector<void*> blocks = P->inters[(size_t)i].heap_blocks;
+  GpuOpCtx ctx{P->db, st, &P->inters};
+  ctx.forced_cap = P->forced[(size_t)i];
+  ctx.count_column_access = false;
+  ctx.reuse = &blocks;
+  return run_gpu_op(ctx, P->plan.ops[i], P->inters[(size_t)i]);
+}
 static ddq_status replay(ddq_prepared* P, cudaStream_t st) {
-  for (int i = 0; i < P->plan.n_ops; i++) {
-    std::vector<void*> blocks = P->inters[(size_t)i].heap_blocks;
-    GpuOpCtx ctx{P->db, st, &P->inters};
-    ctx.forced_cap = P->forced[(size_t)i];
-    ctx.count_column_access = false;
-    ctx.reuse = &blocks;
-    ddq_status s = run_gpu_op(ctx, P->plan.ops[i], P->inters[(size_t)i]);
-    if (s != DDQ_OK) return s;
+  for (int i = 0; i < P->plan.n_ops; i++)
+    if (ddq_status s = replay_op(P, i, st)) return s;
+  return DDQ_OK;
+}
+
+// The plan DAG's edges: an op depends on its TID input, its build side and the
+// builds its STAR terms probe (every other buffer it reads -- carried vectors,
+// error cells -- comes down its input chain).
+static std::vector<int> op_deps(const ddq_op& op, int i) {
+  std::vector<int> d;
+  auto add = [&](int x) {
+    if (x >= 0 && x < i && std::find(d.begin(), d.end(), x) == d.end()) d.push_back(x);
+  };
+  add(op.input);
+  if (op.kind == DDQ_OP_HASH_PROBE) add(op.build);
+  if (op.kind == DDQ_OP_STAR)
+    for (int j = 0; j < op.n_terms && j < 4; j++)
+      if (op.term_kind[j] == DDQ_TERM_PROBE) add(op.term_build[j]);
+  return d;
+}
+
+// Capture the plan as a graph whose branches follow the DAG: independent
+// operators (the dimension builds of a star query, and the fact chain's first
+// probe against the builds it does not read) run concurrently, so the small,
+// latency-bound build kernels leave the critical path.  An op continues the
+// stream of its first dependency when it is that stream's last op, else forks a
+// side stream; other dependencies are event waits.  All branches join `st`.
+static ddq_status replay_branches(ddq_prepared* P, cudaStream_t st) {
+  const int n = P->plan.n_ops;
+  if ((int)P->ev.size() < n + 1) {
+    for (int i = (int)P->ev.size(); i < n + 1; i++) {
+      cudaEvent_t e;
+      if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess)
+        return set_error(DDQ_ECUDA, "prepare: event");
+      P->ev.push_back(e);
+    }
   }
+  std::vector<cudaStream_t> streams;  // capture lanes; lane 0 = st
+  std::vector<int> tail;              // last op on each lane
+  std::vector<int> lane_of((size_t)n, -1);
+  streams.push_back(st);
+  tail.push_back(-1);
+  cudaEvent_t start = P->ev[(size_t)n];
+  if (cudaEventRecord(start, st) != cudaSuccess) return set_error(DDQ_ECUDA, "prepare: fork");
+  size_t next_side = 0;
+  for (int i = 0; i < n; i++) {
+    const std::vector<int> d = op_deps(P->plan.ops[i], i);
+    int lane = -1;
+    if (!d.empty() && tail[(size_t)lane_of[(size_t)d[0]]] == d[0]) lane = lane_of[(size_t)d[0]];
+    if (lane < 0 && d.empty() && tail[0] == -1) lane = 0;  // the first root op stays on st
+    if (lane < 0) {
+      if (next_side == P->side.size()) {
+        cudaStream_t s2;
+        if (cudaStreamCreateWithFlags(&s2, cudaStreamNonBlocking) != cudaSuccess)
+          return set_error(DDQ_ECUDA, "prepare: side stream");
+        P->side.push_back(s2);
+      }
+      streams.push_back(P->side[next_side++]);
+      tail.push_back(-1);
+      lane = (int)streams.size() - 1;
+      if (d.empty() && cudaStreamWaitEvent(streams[(size_t)lane], start, 0) != cudaSuccess)
+        return set_error(DDQ_ECUDA, "prepare: fork");
+    }
+    for (int x : d)
+      if (lane_of[(size_t)x] != lane && cudaStreamWaitEvent(streams[(size_t)lane], P->ev[(size_t)x], 0) != cudaSuccess)
+        return set_error(DDQ_ECUDA, "prepare: edge");
+    if (ddq_status s = replay_op(P, i, streams[(size_t)lane])) return s;
+    if (cudaEventRecord(P->ev[(size_t)i], streams[(size_t)lane]) != cudaSuccess)
+      return set_error(DDQ_ECUDA, "prepare: event record");
+    lane_of[(size_t)i] = lane;
+    tail[(size_t)lane] = i;
+  }
+  for (size_t l = 1; l < streams.size(); l++)
+    if (tail[l] >= 0 && cudaStreamWaitEvent(st, P->ev[(size_t)tail[l]], 0) != cudaSuccess)
+      return set_error(DDQ_ECUDA, "prepare: join");
   return DDQ_OK;
 }
 
@@ -1076,7 +1154,9 @@ ddq_status ddq_prepare(ddq_db* db, const ddq_plan* plan, int32_t use_graph, ddq_
   if (P->use_graph) {
     e = cudaStreamBeginCapture(st, cudaStreamCaptureModeThreadLocal);
     if (e != cudaSuccess) return fail(cuda_status(e, "prepare: begin capture"));
-    ddq_status s = replay(P.get(), st);
+    static const char* env = getenv("DDQ_GRAPH_BRANCHES");  // "0": one serial chain
+    const bool branches = !env || env[0] != '0';
+    ddq_status s = branches ? replay_branches(P.get(), st) : replay(P.get(), st);
     cudaGraph_t g = nullptr;
     e = cudaStreamEndCapture(st, &g);
     if (s != DDQ_OK || e != cudaSuccess) {
@@ -1343,6 +1423,8 @@ void ddq_prepared_free(ddq_prepared* p) {
   if (p->graph) cudaGraphDestroy(p->graph);
   free_inters(p->db, p->inters);
   if (p->cap_stream) cudaStreamDestroy(p->cap_stream);
+  for (cudaStream_t s2 : p->side) cudaStreamDestroy(s2);
+  for (cudaEvent_t e : p->ev) cudaEventDestroy(e);
   delete p;
 }
 

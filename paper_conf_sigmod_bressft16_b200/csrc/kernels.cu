@@ -8,6 +8,7 @@
 // Accumulators are exact int128 (two 64-bit atomics with carry), so results are
 // bit-identical whatever the scheduling (integer addition is associative).
 #include <cstdint>
+#include <cstdlib>
 #include <cuda_runtime.h>
 
 #include "device_common.cuh"
@@ -488,6 +489,12 @@ cudaError_t launch_groupby(const int32_t* tids, const uint32_t* d_count, int64_t
                            const int32_t* key_bits,
                            const ddq_dev_agg* aggs, int n_aggs, void* table, uint32_t capacity,
                            uint32_t* d_error, cudaStream_t st) {
+  if (agg_ws_supported(tids, key_vec, n_keys, n_aggs, capacity) && d_count) {
+    static const char* env = getenv("DDQ_AGG_WS");  // "0": the warp-match kernels below
+    if (!env || env[0] != '0')
+      return launch_agg_ws(tids, d_count, n_cap, key_vec, key_col, n_keys, key_bits, aggs, n_aggs, table, capacity,
+                           d_error, st);
+  }
   GroupbyParams p{};
   p.tids = tids;
   p.d_count = d_count;

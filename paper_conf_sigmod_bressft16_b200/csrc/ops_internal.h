@@ -43,6 +43,9 @@ size_t filter_scratch_bytes(int64_t n_cap);
 bool scan_supported(const FilterArgs& a);
 cudaError_t launch_scan(const FilterArgs& a, cudaStream_t st);
 cudaError_t launch_filter(const FilterArgs& a, cudaStream_t st);
+// warp-autonomous filter kernels (dense.cu): dense probes and every TID-input operator
+bool ws_supported(const FilterArgs& a);
+cudaError_t launch_ws(const FilterArgs& a, cudaStream_t st);
 
 // HASH_BUILD with a fused selection (a BUILD op carrying predicates): rows that
 // fail any predicate are not inserted -- the select -> build pair of a dimension
@@ -78,6 +81,13 @@ cudaError_t launch_groupby(const int32_t* tids, const uint32_t* d_count, int64_t
                            const int32_t* key_bits,
                            const ddq_dev_agg* aggs, int n_aggs, void* table, uint32_t capacity,
                            uint32_t* d_error, cudaStream_t st);
+// warp-autonomous aggregation for <= 2 aggregates and small group counts (agg.cu)
+bool agg_ws_supported(const int32_t* tids, const int32_t* const* key_vec, int n_keys, int n_aggs,
+                      uint32_t capacity);
+cudaError_t launch_agg_ws(const int32_t* tids, const uint32_t* d_count, int64_t n_cap,
+                          const int32_t* const* key_vec, const int32_t* const* key_col, int n_keys,
+                          const int32_t* key_bits, const ddq_dev_agg* aggs, int n_aggs, void* table,
+                          uint32_t capacity, uint32_t* d_error, cudaStream_t st);
 cudaError_t launch_groupby_compact(const void* table, uint32_t capacity, int n_aggs, int64_t* out_keys,
                                    int64_t* out_accs, uint32_t* d_out_groups, cudaStream_t st);
 

@@ -51,7 +51,8 @@ def _oracle(kind, q):
 
 
 VARIANTS = {"star": dict(star=True), "chain": dict(star=False),
-            "chain_unfused": dict(star=False, fused_build=False)}
+            "chain_eager": dict(star=False, late=False),
+            "chain_unfused": dict(star=False, fused_build=False, late=False)}
 
 
 @pytest.mark.parametrize("variant", list(VARIANTS))
@@ -59,7 +60,9 @@ VARIANTS = {"star": dict(star=True), "chain": dict(star=False),
 @pytest.mark.parametrize("q", oracle.SSB_QUERIES)
 def test_ssb_prepared_graph_equals_oracle(kind, q, variant):
     """star: one STAR operator; chain: binary operators, dimension selections fused
-    into their builds; chain_unfused: SELECT -> BUILD on every dimension."""
+    into their builds, the first probe's payload fetched at the final TIDs;
+    chain_eager: payloads emitted by the first probe and carried; chain_unfused:
+    SELECT -> BUILD on every dimension."""
     from paper_conf_sigmod_bressft16_b200.ssb import ssb_plan
     db = _db(kind)
     p = db.prepare(ssb_plan(db, q, **VARIANTS[variant]), use_graph=True)
