@@ -46,6 +46,9 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--profile-only", action="store_true", help="short run for ncu")
+    ap.add_argument("--streams", type=int, default=1,
+                    help="concurrent query streams inside a step (the 13 plans round-robin over K streams, "
+                         "the paper's parallel users P:358); 1 = back to back on one stream")
     return ap.parse_args()
 
 
@@ -226,9 +229,20 @@ def main():
     sptr = stream.cuda_stream
     kernels_per_step = sum(p.kernels for p in preps)
 
+    side = [torch.cuda.Stream() for _ in range(max(args.streams, 1) - 1)]
+
     def step():
-        for p in preps:
-            p.launch(sptr)
+        if not side:
+            for p in preps:
+                p.launch(sptr)
+            return
+        lanes = [stream] + side
+        for s2 in side:
+            s2.wait_stream(stream)
+        for i, p in enumerate(preps):
+            p.launch(lanes[i % len(lanes)].cuda_stream)
+        for s2 in side:
+            stream.wait_stream(s2)
 
     # N>1: the 13 compacted partial group tables of a step are packed on the device
     # ([n, keys[cap], accs[cap*n_aggs*2]] per query) and exchanged with ONE NCCL
@@ -379,6 +393,7 @@ def main():
                 "config": {"workload": f"SSB SF{sf_total:g}, all 13 queries, hot cache (BASELINE configs[1])",
                            "lineorder_rows": n_lo, "rows_per_gpu": shard_rows, "queries": 13,
                            "parallelism": f"row-sharded x{ws}" if ws > 1 else "1 GPU",
+                           "query_streams": max(args.streams, 1),
                            "l2": "inputs (6.7 GB/GPU) larger than L2; no flush"},
                 "queries_per_s": 13 * args.steps / (ms / 1e3),
                 "gpu_launches": kernels_per_step * args.steps,

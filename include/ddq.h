@@ -310,7 +310,8 @@ typedef struct {
   int32_t kind;            /* DDQ_OP_* */
   int32_t input;           /* child op index whose output TIDs are consumed, or -1 = all rows */
   ddq_table table;         /* row space of input and output TIDs */
-  /* SELECT */
+  /* SELECT; also HASH_BUILD and AGGREGATE, where they are a fused selection of the
+     op's input rows (readings O25, O26) */
   int32_t n_preds;
   ddq_pred preds[DDQ_MAX_PREDS];
   /* HASH_BUILD */

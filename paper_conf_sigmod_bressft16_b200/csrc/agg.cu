@@ -13,8 +13,11 @@
 //     touches the shared-memory table only when its key changes -- a single-group
 //     query (Q1.x, Q6) never does until the end, a 150-group one does per row but
 //     with conflict-free random slots (no warp match / shuffle reduction);
-//   * the per-CTA shared-memory table (open addressing, int128 accumulators by two
-//     64-bit atomics with carry) is merged into the global table once per CTA.
+//   * the shared-memory table accumulates every aggregate as TWO int64 words,
+//     L += S mod 2^32 and H += S >> 32 (arithmetic), with non-returning atomics:
+//     exact for any CTA (L < 2^32 * 2^32 adds, |H| < 2^62 for |sum| < 2^94) and
+//     no carry round trip; the CTA's (H, L) become one int128 = H * 2^32 + L that
+//     is merged into the global table (two 64-bit atomics with carry) once per CTA.
 // Sums are exact int128 whatever the order (integer addition is associative).
 #include <climits>
 #include <cstdint>
@@ -49,6 +52,17 @@ struct AggParams {
   uint32_t* d_error;
   uint32_t s_slots;
   int32_t s_shift;
+  // fused predicates (reading O26): conjunction evaluated at the TIDs first
+  int32_t n_preds;
+  struct Pred {
+    const void* col;
+    int32_t width, kind;
+    int64_t lo;
+    uint64_t d64;  // RANGE: (u64)(v - lo) <= d64
+    int32_t empty, n_in;
+    int64_t in_vals[8];
+  } preds[4];
+  uint32_t* d_rows;
 };
 
 __device__ __forceinline__ int64_t find_or_insert(long long* keys, uint32_t mask, uint32_t h, long long key) {
@@ -78,11 +92,11 @@ __device__ __forceinline__ void gather8(const void* col, int width, const int32_
   if (width == 8) {
 #pragma unroll
     for (int j = 0; j < AG_ITEMS; j++)
-      v[j] = ((valid >> j) & 1u) ? __ldg(reinterpret_cast<const long long*>(col) + (uint32_t)tid[j]) : 0;
+      v[j] = ((valid >> j) & 1u) ? ldg_gather(reinterpret_cast<const long long*>(col) + (uint32_t)tid[j]) : 0;
   } else {
 #pragma unroll
     for (int j = 0; j < AG_ITEMS; j++)
-      v[j] = ((valid >> j) & 1u) ? (long long)__ldg(reinterpret_cast<const int32_t*>(col) + (uint32_t)tid[j]) : 0;
+      v[j] = ((valid >> j) & 1u) ? (long long)ldg_gather(reinterpret_cast<const int32_t*>(col) + (uint32_t)tid[j]) : 0;
   }
 }
 
@@ -116,14 +130,19 @@ __device__ __forceinline__ void agg_values(const AggParams& P, int a, const int3
   }
 }
 
+__device__ __forceinline__ uint32_t hash32(long long k, int shift) {
+  const uint32_t x = (uint32_t)k ^ (uint32_t)((unsigned long long)k >> 32);
+  return (x * 0x9E3779B1u) >> shift;  // shift = 32 - log2(slots)
+}
+
 template <int NA>
 __global__ void __launch_bounds__(AG_NW * 32, 1) agg_ws_kernel(const __grid_constant__ AggParams P) {
   extern __shared__ __align__(16) unsigned long long ag_smem[];
   long long* s_keys = reinterpret_cast<long long*>(ag_smem);
-  unsigned long long* s_accs = ag_smem + P.s_slots;  // [(a * S + slot) * 2 + w]
+  unsigned long long* s_acc = ag_smem + P.s_slots;  // [(a * S + slot) * 2 + {0: L, 1: H}]
   const uint32_t S = P.s_slots, smask = S - 1;
   for (uint32_t i = threadIdx.x; i < S; i += blockDim.x) s_keys[i] = GB_EMPTY;
-  for (uint32_t i = threadIdx.x; i < S * 2 * NA; i += blockDim.x) s_accs[i] = 0;
+  for (uint32_t i = threadIdx.x; i < S * 2 * NA; i += blockDim.x) s_acc[i] = 0;
   __syncthreads();
 
   const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
@@ -139,11 +158,31 @@ __global__ void __launch_bounds__(AG_NW * 32, 1) agg_ws_kernel(const __grid_cons
   for (int a = 0; a < NA; a++) lo[a] = 0, hi[a] = 0;
   auto flush = [&]() {
     if (cur == GB_EMPTY) return;
-    int64_t slot = find_or_insert(s_keys, smask, gb_hash(cur, P.s_shift), cur);
+    uint32_t h = hash32(cur, P.s_shift);
+    int64_t slot = -1;
+    for (uint32_t probes = 0; probes <= smask; probes++) {
+      const long long k = s_keys[h];
+      if (k == cur) {
+        slot = h;
+        break;
+      }
+      if (k == GB_EMPTY) {
+        const long long old = (long long)atomicCAS(reinterpret_cast<unsigned long long*>(s_keys + h),
+                                                   (unsigned long long)GB_EMPTY, (unsigned long long)cur);
+        if (old == GB_EMPTY || old == cur) {
+          slot = h;
+          break;
+        }
+      }
+      h = (h + 1) & smask;
+    }
     if (slot >= 0) {
 #pragma unroll
-      for (int a = 0; a < NA; a++)
-        add_i128(&s_accs[((size_t)a * S + slot) * 2], &s_accs[((size_t)a * S + slot) * 2 + 1], lo[a], hi[a]);
+      for (int a = 0; a < NA; a++) {  // split accumulation, fire-and-forget atomics
+        atomicAdd(&s_acc[((size_t)a * S + slot) * 2], lo[a] & 0xFFFFFFFFull);
+        atomicAdd(&s_acc[((size_t)a * S + slot) * 2 + 1],
+                  (unsigned long long)(long long)((lo[a] >> 32) | ((unsigned long long)hi[a] << 32)));
+      }
     } else {  // CTA table full: straight into the global table
       slot = find_or_insert(P.g_keys, P.cap_mask, gb_hash(cur, P.shift), cur);
       if (slot < 0) {
@@ -163,16 +202,17 @@ __global__ void __launch_bounds__(AG_NW * 32, 1) agg_ws_kernel(const __grid_cons
       r[1] = ld_stream_i4(base_ptr + t0 + 128 + lofs);
     } else {
 #pragma unroll
-      for (int s = 0; s < 2; s++) {
-        const uint32_t i = t0 + s * 128 + lofs;
-        r[s].x = i < n ? base_ptr[i] : 0;
-        r[s].y = i + 1 < n ? base_ptr[i + 1] : 0;
-        r[s].z = i + 2 < n ? base_ptr[i + 2] : 0;
-        r[s].w = i + 3 < n ? base_ptr[i + 3] : 0;
+      for (int s2 = 0; s2 < 2; s2++) {
+        const uint32_t i = t0 + s2 * 128 + lofs;
+        r[s2].x = i < n ? base_ptr[i] : 0;
+        r[s2].y = i + 1 < n ? base_ptr[i + 1] : 0;
+        r[s2].z = i + 2 < n ? base_ptr[i + 2] : 0;
+        r[s2].w = i + 3 < n ? base_ptr[i + 3] : 0;
       }
     }
   };
   uint32_t tile = blockIdx.x * AG_NW + warp;
+  uint32_t rows = 0;  // rows passing the fused predicates (d_rows)
   int4 nt[2];
   if (tile < ntiles) load8(P.tids, tile * AG_TILE, nt);
   for (; tile < ntiles; tile += W) {
@@ -185,6 +225,27 @@ __global__ void __launch_bounds__(AG_NW * 32, 1) agg_ws_kernel(const __grid_cons
 #pragma unroll
       for (int j = 0; j < AG_ITEMS; j++) valid |= (t0 + (j >> 2) * 128 + lofs + (j & 3) < n ? 1u : 0u) << j;
     }
+    for (int p = 0; p < P.n_preds; p++) {  // fused selection: later columns only for live rows
+      const AggParams::Pred& pr = P.preds[p];
+      long long x[AG_ITEMS];
+      gather8(pr.col, pr.width, tid, valid, x);
+      uint32_t m = 0;
+      if (pr.kind == DDQ_PRED_RANGE) {
+#pragma unroll
+        for (int j = 0; j < AG_ITEMS; j++) m |= ((uint64_t)(x[j] - pr.lo) <= pr.d64 ? 1u : 0u) << j;
+        if (pr.empty) m = 0;
+      } else {
+#pragma unroll
+        for (int j = 0; j < AG_ITEMS; j++) {
+          bool hit = false;
+#pragma unroll
+          for (int q = 0; q < 8; q++) hit |= (q < pr.n_in) && (x[j] == pr.in_vals[q]);
+          m |= (hit ? 1u : 0u) << j;
+        }
+      }
+      valid &= m;
+    }
+    if (P.d_rows) rows += __popc(valid);
     long long key[AG_ITEMS];
 #pragma unroll
     for (int j = 0; j < AG_ITEMS; j++) key[j] = 0;
@@ -197,7 +258,7 @@ __global__ void __launch_bounds__(AG_NW * 32, 1) agg_ws_kernel(const __grid_cons
         c[4] = r[1].x; c[5] = r[1].y; c[6] = r[1].z; c[7] = r[1].w;
       } else {
 #pragma unroll
-        for (int j = 0; j < AG_ITEMS; j++) c[j] = ((valid >> j) & 1u) ? __ldg(P.key_col[k] + (uint32_t)tid[j]) : 0;
+        for (int j = 0; j < AG_ITEMS; j++) c[j] = ((valid >> j) & 1u) ? ldg_gather(P.key_col[k] + (uint32_t)tid[j]) : 0;
       }
 #pragma unroll
       for (int j = 0; j < AG_ITEMS; j++) key[j] |= (long long)(uint32_t)c[j] << P.key_shift[k];
@@ -216,17 +277,21 @@ __global__ void __launch_bounds__(AG_NW * 32, 1) agg_ws_kernel(const __grid_cons
       }
 #pragma unroll
       for (int a = 0; a < NA; a++) {  // exact int128 running sum
-        const unsigned long long s = lo[a] + (unsigned long long)v[a][j];
-        hi[a] += (v[a][j] < 0 ? -1 : 0) + (s < lo[a] ? 1 : 0);
-        lo[a] = s;
+        const unsigned long long s2 = lo[a] + (unsigned long long)v[a][j];
+        hi[a] += (v[a][j] < 0 ? -1 : 0) + (s2 < lo[a] ? 1 : 0);
+        lo[a] = s2;
       }
     }
   }
   flush();
+  if (P.d_rows) {
+    rows = __reduce_add_sync(FULL, rows);
+    if (lane == 0 && rows) atomicAdd(P.d_rows, rows);
+  }
   __syncthreads();
-  // merge this CTA's table into the global one
-  for (uint32_t s = threadIdx.x; s < S; s += blockDim.x) {
-    const long long key = s_keys[s];
+  // merge this CTA's table into the global one: int128 = H * 2^32 + L
+  for (uint32_t s2 = threadIdx.x; s2 < S; s2 += blockDim.x) {
+    const long long key = s_keys[s2];
     if (key == GB_EMPTY) continue;
     const int64_t g = find_or_insert(P.g_keys, P.cap_mask, gb_hash(key, P.shift), key);
     if (g < 0) {
@@ -234,9 +299,17 @@ __global__ void __launch_bounds__(AG_NW * 32, 1) agg_ws_kernel(const __grid_cons
       continue;
     }
 #pragma unroll
-    for (int a = 0; a < NA; a++)
+    for (int a = 0; a < NA; a++) {
+      const unsigned long long L = s_acc[((size_t)a * S + s2) * 2];
+      const long long H = (long long)s_acc[((size_t)a * S + s2) * 2 + 1];
+      // (H << 32) + L as int128 (lo, hi)
+      const unsigned long long hl = (unsigned long long)H << 32;
+      const long long hh = H >> 32;
+      const unsigned long long lo2 = hl + L;
+      const long long hi2 = hh + (lo2 < hl ? 1 : 0);
       add_i128(&P.g_accs[((size_t)a * (P.cap_mask + 1) + g) * 2], &P.g_accs[((size_t)a * (P.cap_mask + 1) + g) * 2 + 1],
-               s_accs[((size_t)a * S + s) * 2], (long long)s_accs[((size_t)a * S + s) * 2 + 1]);
+               lo2, hi2);
+    }
   }
 }
 
@@ -253,8 +326,25 @@ bool agg_ws_supported(const int32_t* tids, const int32_t* const* key_vec, int n_
 cudaError_t launch_agg_ws(const int32_t* tids, const uint32_t* d_count, int64_t n_cap,
                           const int32_t* const* key_vec, const int32_t* const* key_col, int n_keys,
                           const int32_t* key_bits, const ddq_dev_agg* aggs, int n_aggs, void* table,
-                          uint32_t capacity, uint32_t* d_error, cudaStream_t st) {
+                          uint32_t capacity, uint32_t* d_error, cudaStream_t st, const BuildPreds* preds,
+                          uint32_t* d_rows) {
   AggParams p{};
+  p.d_rows = d_rows;
+  if (preds) {
+    p.n_preds = preds->n;
+    for (int i = 0; i < preds->n && i < 4; i++) {
+      const ddq_dev_pred& d = preds->p[i];
+      AggParams::Pred& q = p.preds[i];
+      q.col = d.col;
+      q.width = d.width;
+      q.kind = d.kind;
+      q.lo = d.lo;
+      q.empty = d.hi < d.lo;
+      q.d64 = q.empty ? 0 : (uint64_t)d.hi - (uint64_t)d.lo;
+      q.n_in = d.n_in;
+      for (int j = 0; j < 8; j++) q.in_vals[j] = d.in_vals[j];
+    }
+  }
   p.tids = tids;
   p.d_count = d_count;
   p.n_keys = n_keys;
@@ -284,7 +374,7 @@ cudaError_t launch_agg_ws(const int32_t* tids, const uint32_t* d_count, int64_t 
   int slg = 0;
   while ((1u << slg) < S) slg++;
   p.s_slots = S;
-  p.s_shift = 64 - slg;
+  p.s_shift = 32 - slg;
   const size_t smem = (size_t)S * (8 + 16 * (size_t)n_aggs);
   static bool attr = false;
   if (!attr) {

@@ -227,7 +227,7 @@ __global__ void __launch_bounds__(ws_nw(kTids) * 32, 1) ws_kernel(const __grid_c
         unpack16(kk, key);
       } else {  // key column gathered at the TIDs
 #pragma unroll
-        for (int j = 0; j < WS_ITEMS; j++) key[j] = ((flags >> j) & 1u) ? __ldg(P.fk + (uint32_t)sv[j]) : 0;
+        for (int j = 0; j < WS_ITEMS; j++) key[j] = ((flags >> j) & 1u) ? ldg_gather(P.fk + (uint32_t)sv[j]) : 0;
       }
       if (!kHash) {
         uint32_t m = 0;
@@ -239,7 +239,7 @@ __global__ void __launch_bounds__(ws_nw(kTids) * 32, 1) ws_kernel(const __grid_c
             hit = (s_bm[oo >> 5] >> (oo & 31)) & 1u;
           } else {
             const uint32_t o = (uint32_t)(key[j] - P.key_min);
-            hit = o < P.range ? (__ldg(P.bitmap + (o >> 5)) >> (o & 31)) & 1u : 0u;
+            hit = o < P.range ? (ldg_gather(P.bitmap + (o >> 5)) >> (o & 31)) & 1u : 0u;
           }
           m |= hit << j;
         }
@@ -250,7 +250,7 @@ __global__ void __launch_bounds__(ws_nw(kTids) * 32, 1) ws_kernel(const __grid_c
           for (int j = 0; j < WS_ITEMS; j++) {
             pay[j] = 0;
             if ((any >> j) & 1u)
-              if ((flags >> j) & 1u) pay[j] = __ldg(P.payarr + (uint32_t)(key[j] - P.key_min));
+              if ((flags >> j) & 1u) pay[j] = ldg_gather(P.payarr + (uint32_t)(key[j] - P.key_min));
           }
         }
       } else {
@@ -259,10 +259,10 @@ __global__ void __launch_bounds__(ws_nw(kTids) * 32, 1) ws_kernel(const __grid_c
           pay[j] = 0;
           if ((flags >> j) & 1u) {
             uint32_t h = ht_hash(key[j], P.shift);
-            uint64_t s = kKind == WK_HT_SMEM ? s_ht[h] : __ldg(P.table + h);
+            uint64_t s = kKind == WK_HT_SMEM ? s_ht[h] : ldg_gather(P.table + h);
             while (s != HT_EMPTY && ht_key(s) != key[j]) {
               h = (h + 1) & P.cap_mask;
-              s = kKind == WK_HT_SMEM ? s_ht[h] : __ldg(P.table + h);
+              s = kKind == WK_HT_SMEM ? s_ht[h] : ldg_gather(P.table + h);
             }
             if (s == HT_EMPTY) flags &= ~(1u << j);
             pay[j] = ht_val(s);
@@ -290,14 +290,14 @@ __global__ void __launch_bounds__(ws_nw(kTids) * 32, 1) ws_kernel(const __grid_c
           for (int j = 0; j < WS_ITEMS; j++) {
             v[j] = 0;
             if ((any >> j) & 1u)
-              if ((flags >> j) & 1u) v[j] = __ldg(reinterpret_cast<const long long*>(pr.col) + (uint32_t)sv[j]);
+              if ((flags >> j) & 1u) v[j] = ldg_gather(reinterpret_cast<const long long*>(pr.col) + (uint32_t)sv[j]);
           }
         } else {
 #pragma unroll
           for (int j = 0; j < WS_ITEMS; j++) {
             v[j] = 0;
             if ((any >> j) & 1u)
-              if ((flags >> j) & 1u) v[j] = __ldg(reinterpret_cast<const int32_t*>(pr.col) + (uint32_t)sv[j]);
+              if ((flags >> j) & 1u) v[j] = ldg_gather(reinterpret_cast<const int32_t*>(pr.col) + (uint32_t)sv[j]);
           }
         }
         uint32_t m = 0;
@@ -592,7 +592,7 @@ cudaError_t launch_ws(const FilterArgs& a, cudaStream_t st) {
   p.d_out_count = a.d_out_count;
   p.out_cap = (uint32_t)(a.out_cap > 0 ? a.out_cap : a.n_cap);
   p.d_overflow = a.d_overflow;
-  cudaError_t e = cudaMemsetAsync(a.d_out_count, 0, 8, st);
+  cudaError_t e = init_fill(a.d_out_count, 8, 0, st);
   if (e != cudaSuccess) return e;
   const size_t smem = ring + ((kind == WK_BM_SMEM || kind == WK_HT_SMEM) ? tab : 0);
   const int64_t ntiles = (a.n_cap + WS_TILE - 1) / WS_TILE;  // TID input: an upper bound

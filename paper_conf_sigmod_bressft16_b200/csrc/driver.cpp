@@ -74,6 +74,7 @@ static std::vector<int> op_columns(const ddq_op& op) {
       break;
     case DDQ_OP_GATHER: c.push_back(op.gather_col); break;
     case DDQ_OP_AGGREGATE:
+      for (int i = 0; i < op.n_preds; i++) c.push_back(op.preds[i].column);  // fused selection
       for (int k = 0; k < op.n_keys; k++)
         if (op.key_src[k] < -1) c.push_back(-2 - op.key_src[k]);
       for (int a = 0; a < op.n_aggs; a++) {
@@ -530,8 +531,23 @@ ddq_status run_host_op(ddq_db* db, const ddq_op& op, const std::vector<Inter>& I
         sh += op.key_bits[k] > 0 ? op.key_bits[k] : 21;
       }
       std::unordered_map<int64_t, std::vector<__int128>> g;
+      std::vector<const Column*> apc;  // fused selection (AGGREGATE op with predicates)
+      for (int p = 0; p < op.n_preds; p++) apc.push_back(col_of(db, op.preds[p].column));
       for (int64_t i = 0; i < n; i++) {
         int32_t r = in->tids[i];
+        bool ok = true;
+        for (int p = 0; p < op.n_preds && ok; p++) {
+          const int64_t v = hcol(apc[(size_t)p], r);
+          const ddq_pred& pr = op.preds[p];
+          if (pr.kind == DDQ_PRED_RANGE) {
+            ok = v >= pr.lo && v <= pr.hi;
+          } else {
+            bool m = false;
+            for (int j = 0; j < pr.n_in; j++) m |= v == pr.in_vals[j];
+            ok = m;
+          }
+        }
+        if (!ok) continue;
         int64_t key = 0;
         for (int k = 0; k < op.n_keys; k++) {
           int32_t c = op.key_src[k] >= 0 ? ((const int32_t*)in->vecs[(size_t)op.key_src[k]].ptr)[i]

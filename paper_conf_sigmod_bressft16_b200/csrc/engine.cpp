@@ -280,7 +280,7 @@ ddq_status run_gpu_op(GpuOpCtx& ctx, const ddq_op& op, Inter& out) {
       if (!out.d_error) {
         out.d_error = (uint32_t*)A.get(64);
         if (A.failed) return DDQ_ENOMEM_DEVICE;
-        cudaMemsetAsync(out.d_error, 0, 4, st);
+        init_fill(out.d_error, 4, 0, st);
       }
       fa.d_overflow = out.d_error;
       return cuda_status(launch_filter(fa, st), probe ? "probe" : "select");
@@ -335,7 +335,7 @@ ddq_status run_gpu_op(GpuOpCtx& ctx, const ddq_op& op, Inter& out) {
       }
       out.d_error = (uint32_t*)A.get(64);
       if (A.failed) return DDQ_ENOMEM_DEVICE;
-      cudaMemsetAsync(out.d_error, 0, 4, st);
+      init_fill(out.d_error, 4, 0, st);
       return cuda_status(launch_star(terms, op.n_terms, T.n_rows, out.tids, out.d_count, out_cap, out.d_error, st),
                          "star");
     }
@@ -378,8 +378,8 @@ ddq_status run_gpu_op(GpuOpCtx& ctx, const ddq_op& op, Inter& out) {
         out.d_error = (uint32_t*)A.get(64);
         out.cap = 0;
         if (A.failed) return DDQ_ENOMEM_DEVICE;
-        cudaMemsetAsync(out.d_error, 0, 4, st);
-        cudaError_t e = cudaMemsetAsync(out.jidx, 0, ((size_t)out.jrange + 31) / 32 * 4, st);
+        init_fill(out.d_error, 4, 0, st);
+        cudaError_t e = init_fill(out.jidx, ((size_t)out.jrange + 31) / 32 * 4, 0, st);
         if (e == cudaSuccess)
           e = launch_join_index_build(keys, payload, in_tids, in_cnt, in_cap, out.jmin, out.jrange, out.jidx,
                                       out.d_error, st, &bp);
@@ -394,7 +394,7 @@ ddq_status run_gpu_op(GpuOpCtx& ctx, const ddq_op& op, Inter& out) {
       out.d_error = (uint32_t*)A.get(64);
       out.cap = 0;
       if (A.failed) return DDQ_ENOMEM_DEVICE;
-      cudaMemsetAsync(out.d_error, 0, 4, st);
+      init_fill(out.d_error, 4, 0, st);
       cudaError_t e = launch_hash_init(out.table_ptr, out.table_cap, st);
       if (e == cudaSuccess)
         e = launch_hash_build(keys, payload, in_tids, in_cnt, in_cap, out.table_ptr, out.table_cap, out.d_error, st,
@@ -463,13 +463,82 @@ ddq_status run_gpu_op(GpuOpCtx& ctx, const ddq_op& op, Inter& out) {
       out.d_error = in->d_error;
       if (!out.d_error) {
         out.d_error = (uint32_t*)A.get(64);
-        if (!A.failed) cudaMemsetAsync(out.d_error, 0, 4, st);
+        if (!A.failed) init_fill(out.d_error, 4, 0, st);
       }
       if (A.failed) return DDQ_ENOMEM_DEVICE;
+      // fused selection (reading O26): an AGGREGATE carrying predicates aggregates
+      // only the input rows that pass them
+      if (op.n_preds < 0 || op.n_preds > DDQ_MAX_PREDS) return set_error(DDQ_EINVAL, "aggregate: bad n_preds");
+      BuildPreds bp;
+      bp.n = op.n_preds;
+      for (int i = 0; i < op.n_preds; i++) {
+        const ddq_pred& p = op.preds[i];
+        const Column* c = col_of(db, p.column);
+        if (!c || c->table != op.table) return set_error(DDQ_EINVAL, "aggregate: predicate column not in table");
+        ddq_dev_pred& d = bp.p[i];
+        std::memset(&d, 0, sizeof(d));
+        d.col = need_col(p.column);
+        if (!d.col) return set_error(DDQ_ESTATE, "aggregate: predicate column not cached on the GPU");
+        d.width = c->width;
+        d.kind = p.kind;
+        d.lo = p.lo;
+        d.hi = p.hi;
+        d.n_in = p.n_in;
+        for (int j = 0; j < DDQ_MAX_IN; j++) d.in_vals[j] = p.in_vals[j];
+      }
+      const int32_t* g_tids = in->tids;
+      const uint32_t* g_count = in->d_count;
+      if (op.n_preds > 0 && !agg_ws_supported(in->tids, kv, op.n_keys, op.n_aggs, out.gb_cap)) {
+        // no fused kernel for this shape: a selection into a temporary TID list
+        // (carrying the key vectors) feeds the aggregation
+        int32_t* ft = (int32_t*)A.get((uint64_t)std::max<int64_t>(in->cap, 1) * 4);
+        uint32_t* fc = (uint32_t*)A.get(64);
+        void* fscr = A.get(filter_scratch_bytes(in->cap));
+        const int32_t* cin[3] = {nullptr, nullptr, nullptr};
+        int32_t* cout2[3] = {nullptr, nullptr, nullptr};
+        int nc = 0;
+        for (int k = 0; k < op.n_keys; k++)
+          if (kv[k]) {
+            cin[nc] = kv[k];
+            cout2[nc] = (int32_t*)A.get((uint64_t)std::max<int64_t>(in->cap, 1) * 4);
+            kv[k] = cout2[nc];
+            nc++;
+          }
+        if (A.failed) return DDQ_ENOMEM_DEVICE;
+        FilterArgs fa;
+        fa.preds = bp.p;
+        fa.n_preds = bp.n;
+        fa.in_tids = in->tids;
+        fa.d_in_count = in->d_count;
+        fa.n_cap = in->cap;
+        fa.carry_in = cin;
+        fa.carry_out = cout2;
+        fa.n_carry = nc;
+        fa.out_tids = ft;
+        fa.d_out_count = fc;
+        fa.out_cap = in->cap;
+        fa.d_overflow = out.d_error;
+        fa.scratch = fscr;
+        cudaError_t e0 = launch_filter(fa, st);
+        if (e0 != cudaSuccess) return cuda_status(e0, "aggregate: fused selection");
+        g_tids = ft;
+        g_count = fc;
+        bp.n = 0;
+      }
+      if (op.n_preds > 0 && bp.n > 0) {
+        out.d_rows = (uint32_t*)A.get(64);
+        if (A.failed) return DDQ_ENOMEM_DEVICE;
+        init_fill(out.d_rows, 4, 0, st);
+      }
       cudaError_t e = launch_groupby_init(out.gb_table, out.gb_cap, op.n_aggs, st);
-      if (e == cudaSuccess)
-        e = launch_groupby(in->tids, in->d_count, in->cap, kv, kc, op.n_keys, op.key_bits, ag, op.n_aggs, out.gb_table,
-                           out.gb_cap, out.d_error, st);
+      if (e == cudaSuccess) {
+        if (bp.n > 0)
+          e = launch_agg_ws(g_tids, g_count, in->cap, kv, kc, op.n_keys, op.key_bits, ag, op.n_aggs, out.gb_table,
+                            out.gb_cap, out.d_error, st, &bp, out.d_rows);
+        else
+          e = launch_groupby(g_tids, g_count, in->cap, kv, kc, op.n_keys, op.key_bits, ag, op.n_aggs, out.gb_table,
+                             out.gb_cap, out.d_error, st);
+      }
       if (e == cudaSuccess)
         e = launch_groupby_compact(out.gb_table, out.gb_cap, op.n_aggs, out.gb_keys, out.gb_accs, out.gb_groups, st);
       return cuda_status(e, "aggregate");
@@ -889,6 +958,7 @@ struct ddq_prepared {
   // graph capture with parallel branches: side streams + one event per op
   std::vector<cudaStream_t> side;
   std::vector<cudaEvent_t> ev;
+  std::vector<ddq::FillRec> fills;  // buffer initialisations, hoisted to the graph root
 };
 
 namespace ddq {
@@ -932,13 +1002,15 @@ static ddq_status validate_plan(ddq_db* db, const ddq_plan* plan) {
 }
 ddq_status validate_plan_public(ddq_db* db, const ddq_plan* plan) { return validate_plan(db, plan); }
 
+// kernels an operator launches in a prepared graph (its buffer initialisations are
+// hoisted into the graph's one multi-range fill kernel, counted separately)
 static int kernels_of(const ddq_op& op) {
   switch (op.kind) {
     case DDQ_OP_SELECT:
     case DDQ_OP_HASH_PROBE: return 1;
-    case DDQ_OP_HASH_BUILD: return 2;
+    case DDQ_OP_HASH_BUILD: return 1;
     case DDQ_OP_GATHER: return 1;
-    case DDQ_OP_AGGREGATE: return 3;
+    case DDQ_OP_AGGREGATE: return 2;
     case DDQ_OP_FILTER_EQ: return 1;
     case DDQ_OP_STAR: return 1;
   }
@@ -1059,6 +1131,7 @@ void count_accesses(ddq_db* db, const ddq_op& op) {
       for (int j = 0; j < op.n_terms; j++) touch(op.term_kind[j] == DDQ_TERM_PRED ? op.preds[j].column : op.term_fk[j]);
       break;
     case DDQ_OP_AGGREGATE:
+      for (int i = 0; i < op.n_preds; i++) touch(op.preds[i].column);  // fused selection
       for (int k = 0; k < op.n_keys; k++)
         if (op.key_src[k] < -1) touch(-2 - op.key_src[k]);
       for (int a = 0; a < op.n_aggs; a++) {
@@ -1140,14 +1213,19 @@ ddq_status ddq_prepare(ddq_db* db, const ddq_plan* plan, int32_t use_graph, ddq_
       P->forced[(size_t)i] = counts[(size_t)i] + counts[(size_t)i] / 64 + 256;
   }
   P->inters.resize((size_t)plan->n_ops);
+  fill_hoist().rec = &P->fills;  // record every buffer initialisation of the eager run
   for (int i = 0; i < plan->n_ops; i++) {
     GpuOpCtx ctx{db, st, &P->inters};
     ctx.forced_cap = P->forced[(size_t)i];
     ctx.count_column_access = false;
     ddq_status s = run_gpu_op(ctx, plan->ops[i], P->inters[(size_t)i]);
-    if (s != DDQ_OK) return fail(s == DDQ_ENOMEM_DEVICE ? set_error(s, "prepare: device heap exhausted") : s);
+    if (s != DDQ_OK) {
+      fill_hoist().rec = nullptr;
+      return fail(s == DDQ_ENOMEM_DEVICE ? set_error(s, "prepare: device heap exhausted") : s);
+    }
     P->kernels += kernels_of(plan->ops[i]);
   }
+  fill_hoist().rec = nullptr;
   cudaError_t e = cudaStreamSynchronize(st);
   if (e != cudaSuccess) return fail(cuda_status(e, "prepare: eager run"));
   // 3. capture the same launches on the same buffers into one CUDA graph
@@ -1156,7 +1234,16 @@ ddq_status ddq_prepare(ddq_db* db, const ddq_plan* plan, int32_t use_graph, ddq_
     if (e != cudaSuccess) return fail(cuda_status(e, "prepare: begin capture"));
     static const char* env = getenv("DDQ_GRAPH_BRANCHES");  // "0": one serial chain
     const bool branches = !env || env[0] != '0';
-    ddq_status s = branches ? replay_branches(P.get(), st) : replay(P.get(), st);
+    // all buffer initialisations as ONE fill kernel at the graph root; the
+    // operators' own fills are skipped while capturing
+    ddq_status s = DDQ_OK;
+    if (branches) {
+      if (launch_multi_fill(P->fills, st) != cudaSuccess) s = set_error(DDQ_ECUDA, "prepare: fill");
+      fill_hoist().skip = true;
+    }
+    if (s == DDQ_OK) s = branches ? replay_branches(P.get(), st) : replay(P.get(), st);
+    fill_hoist().skip = false;
+    if (branches) P->kernels += (int)((P->fills.size() + 47) / 48);
     cudaGraph_t g = nullptr;
     e = cudaStreamEndCapture(st, &g);
     if (s != DDQ_OK || e != cudaSuccess) {
@@ -1249,7 +1336,10 @@ int32_t ddq_prepared_profile(ddq_prepared* p, void* stream, int32_t max_ops, flo
         } else {
           cls = 1;
           bytes += m * 4;
-          for (int c : cols) bytes += sector_bytes(N, m, width(c));
+          // a conjunction reads its first column at every input TID and the
+          // others only at rows still alive (counted at the final survivors: a
+          // lower bound, intermediate counts are not kept)
+          for (size_t k = 0; k < cols.size(); k++) bytes += sector_bytes(N, k == 0 ? m : out, width(cols[k]));
           bytes += out * 4 * nvec_in;  // carried vectors read at survivors
         }
         bytes += out * 4 * (1 + nvec_in + emit);
@@ -1279,7 +1369,16 @@ int32_t ddq_prepared_profile(ddq_prepared* p, void* stream, int32_t max_ops, flo
       case DDQ_OP_AGGREGATE: {
         cls = 4;
         bytes = m * 4;
-        for (int k = 0; k < op.n_keys; k++) bytes += op.key_src[k] >= 0 ? m * 4 : sector_bytes(N, m, 4);
+        // fused selection: first predicate column at every input TID, the rest
+        // and everything below at the rows that passed (d_rows)
+        double mr = m;
+        if (op.n_preds > 0 && o.d_rows) {
+          uint32_t r = 0;
+          cudaMemcpy(&r, o.d_rows, 4, cudaMemcpyDeviceToHost);
+          mr = r;
+          for (int k = 0; k < op.n_preds; k++) bytes += sector_bytes(N, k == 0 ? m : mr, width(op.preds[k].column));
+        }
+        for (int k = 0; k < op.n_keys; k++) bytes += op.key_src[k] >= 0 ? m * 4 : sector_bytes(N, mr, 4);
         std::vector<int> seen;
         for (int a = 0; a < op.n_aggs; a++)
           for (int j = 0; j < 3; j++) {
@@ -1289,7 +1388,7 @@ int32_t ddq_prepared_profile(ddq_prepared* p, void* stream, int32_t max_ops, flo
                      : op.agg_kind[a] == DDQ_AGG_SUM_MUL_100M_100P ? 3 : 2;
             if (j >= need) continue;
             seen.push_back(c);
-            bytes += sector_bytes(N, m, width(c));
+            bytes += sector_bytes(N, mr, width(c));
           }
       } break;
     }

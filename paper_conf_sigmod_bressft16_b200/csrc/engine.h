@@ -101,6 +101,7 @@ struct Inter {
   int64_t* gb_keys = nullptr;
   int64_t* gb_accs = nullptr;
   uint32_t* gb_groups = nullptr;
+  uint32_t* d_rows = nullptr;  // AGGREGATE with fused predicates: rows that passed (profile)
   // host aggregate result (host executor)
   std::shared_ptr<std::vector<int64_t>> h_keys, h_accs;
   int64_t h_groups = 0;

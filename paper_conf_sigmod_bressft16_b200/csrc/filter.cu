@@ -368,7 +368,7 @@ cudaError_t launch_filter(const FilterArgs& a, cudaStream_t st) {
   uint8_t* sc = reinterpret_cast<uint8_t*>(a.scratch);
   p.tile_counter = reinterpret_cast<uint32_t*>(sc);
   p.tile_status = reinterpret_cast<uint64_t*>(sc + 256);
-  cudaError_t e = cudaMemsetAsync(a.scratch, 0, filter_scratch_bytes(a.n_cap), st);
+  cudaError_t e = init_fill(a.scratch, filter_scratch_bytes(a.n_cap), 0, st);
   if (e != cudaSuccess) return e;
   const bool tids = a.in_tids != nullptr;
   if (!a.probe) {

@@ -7,6 +7,7 @@
 // CTA merges its table into the global open-addressing table once at the end.
 // Accumulators are exact int128 (two 64-bit atomics with carry), so results are
 // bit-identical whatever the scheduling (integer addition is associative).
+#include <algorithm>
 #include <cstdint>
 #include <cstdlib>
 #include <cuda_runtime.h>
@@ -87,11 +88,55 @@ __global__ void hash_build_kernel(const int32_t* __restrict__ keys, const int32_
 }
 
 cudaError_t launch_hash_init(uint64_t* table, uint32_t capacity, cudaStream_t st) {
-  int grid = (int)((capacity + 255) / 256);
-  if (grid > num_sms() * 8) grid = num_sms() * 8;
-  if (grid < 1) grid = 1;
-  hash_init_kernel<<<grid, 256, 0, st>>>(table, capacity);
-  return cudaGetLastError();
+  return init_fill(table, (size_t)capacity * 8, HT_EMPTY, st);
+}
+
+// ---- buffer initialisation -------------------------------------------------
+constexpr int MF_MAX = 48;
+struct MultiFill {
+  int32_t n;
+  FillRec r[MF_MAX];
+};
+
+__global__ void multi_fill_kernel(const __grid_constant__ MultiFill M) {
+  const FillRec& f = M.r[blockIdx.y];
+  uint64_t* p = reinterpret_cast<uint64_t*>(f.ptr);
+  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < f.n64; i += (uint64_t)gridDim.x * blockDim.x)
+    p[i] = f.pattern;
+}
+
+FillHoist& fill_hoist() {
+  static thread_local FillHoist h;
+  return h;
+}
+
+cudaError_t launch_multi_fill(const std::vector<FillRec>& recs, cudaStream_t st) {
+  for (size_t b = 0; b < recs.size(); b += MF_MAX) {
+    MultiFill M{};
+    M.n = (int32_t)std::min<size_t>(MF_MAX, recs.size() - b);
+    uint64_t mx = 1;
+    for (int i = 0; i < M.n; i++) {
+      M.r[i] = recs[b + (size_t)i];
+      mx = std::max<uint64_t>(mx, M.r[i].n64);
+    }
+    uint64_t gx = (mx + 255) / 256;
+    if (gx > (uint64_t)num_sms() * 2) gx = (uint64_t)num_sms() * 2;
+    multi_fill_kernel<<<dim3((unsigned)gx, (unsigned)M.n), 256, 0, st>>>(M);
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return e;
+  }
+  return cudaSuccess;
+}
+
+cudaError_t init_fill(void* ptr, size_t bytes, uint64_t pattern, cudaStream_t st) {
+  if (bytes == 0) return cudaSuccess;
+  FillHoist& h = fill_hoist();
+  if (h.skip) return cudaSuccess;
+  const uint64_t n64 = (bytes + 7) / 8;
+  if (h.rec) h.rec->push_back(FillRec{ptr, n64, pattern});
+  if (pattern == 0) return cudaMemsetAsync(ptr, 0, n64 * 8, st);
+  std::vector<FillRec> one{FillRec{ptr, n64, pattern}};
+  return launch_multi_fill(one, st);
 }
 
 cudaError_t launch_hash_build(const int32_t* keys, const int32_t* payload, const int32_t* in_tids,
@@ -151,9 +196,9 @@ __global__ void gather_kernel(const void* __restrict__ col, const int32_t* __res
   for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
     const int32_t r = tids[i];
     if (W == 8)
-      reinterpret_cast<long long*>(out)[i] = __ldg(reinterpret_cast<const long long*>(col) + r);
+      reinterpret_cast<long long*>(out)[i] = ldg_gather(reinterpret_cast<const long long*>(col) + r);
     else
-      reinterpret_cast<int*>(out)[i] = __ldg(reinterpret_cast<const int*>(col) + r);
+      reinterpret_cast<int*>(out)[i] = ldg_gather(reinterpret_cast<const int32_t*>(col) + r);
   }
 }
 
@@ -281,7 +326,7 @@ __global__ void __launch_bounds__(GB_THREADS) groupby_kernel(const __grid_consta
       r = P.tids[i];
       key = 0;
       for (int k = 0; k < P.n_keys; k++) {
-        const int32_t c = P.key_vec[k] ? P.key_vec[k][i] : __ldg(P.key_col[k] + r);
+        const int32_t c = P.key_vec[k] ? P.key_vec[k][i] : ldg_gather(P.key_col[k] + r);
         key |= (long long)(uint32_t)c << P.key_shift[k];
       }
     }
@@ -373,7 +418,7 @@ __global__ void __launch_bounds__(GBS_THREADS) groupby_small_kernel(const __grid
       uint32_t key = 0;
       if (r[j] >= 0)
         for (int k = 0; k < P.n_keys; k++) {
-          const int32_t c = P.key_vec[k] ? P.key_vec[k][i] : __ldg(P.key_col[k] + r[j]);
+          const int32_t c = P.key_vec[k] ? P.key_vec[k][i] : ldg_gather(P.key_col[k] + r[j]);
           key |= (uint32_t)c << P.key_shift[k];
         }
       d[j] = key & (D - 1);
@@ -476,12 +521,9 @@ __global__ void groupby_init_kernel(long long* keys, unsigned long long* accs, u
 }
 
 cudaError_t launch_groupby_init(void* table, uint32_t capacity, int n_aggs, cudaStream_t st) {
-  int grid = (int)((capacity + 255) / 256);
-  if (grid > num_sms() * 8) grid = num_sms() * 8;
-  groupby_init_kernel<<<grid < 1 ? 1 : grid, 256, 0, st>>>(
-      reinterpret_cast<long long*>(table), reinterpret_cast<unsigned long long*>((char*)table + (size_t)capacity * 8),
-      capacity, n_aggs);
-  return cudaGetLastError();
+  cudaError_t e = init_fill(table, (size_t)capacity * 8, (uint64_t)GB_EMPTY, st);  // keys
+  if (e != cudaSuccess) return e;
+  return init_fill((char*)table + (size_t)capacity * 8, (size_t)capacity * n_aggs * 16, 0, st);  // accs
 }
 
 cudaError_t launch_groupby(const int32_t* tids, const uint32_t* d_count, int64_t n_cap,
@@ -606,7 +648,7 @@ __global__ void groupby_compact_kernel(const long long* keys, const unsigned lon
 
 cudaError_t launch_groupby_compact(const void* table, uint32_t capacity, int n_aggs, int64_t* out_keys,
                                    int64_t* out_accs, uint32_t* d_out_groups, cudaStream_t st) {
-  cudaError_t e = cudaMemsetAsync(d_out_groups, 0, sizeof(uint32_t), st);
+  cudaError_t e = init_fill(d_out_groups, sizeof(uint32_t), 0, st);
   if (e != cudaSuccess) return e;
   int grid = (int)((capacity + 255) / 256);
   if (grid > num_sms() * 8) grid = num_sms() * 8;

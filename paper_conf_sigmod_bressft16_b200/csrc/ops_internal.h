@@ -2,11 +2,31 @@
 #pragma once
 #include <cstddef>
 #include <cstdint>
+#include <vector>
 #include <cuda_runtime.h>
 
 #include "../../include/ddq.h"
 
 namespace ddq {
+
+// ---- buffer initialisation (counters, error cells, bitmaps, empty tables) ----
+// Every operator's "zero this / fill that before the kernel" goes through
+// init_fill.  A prepared plan records them in its eager run and captures ONE
+// multi-range fill kernel at the root of its graph instead (fill_hoist().skip
+// during capture), so no memset node sits on the operator chain.
+struct FillRec {
+  void* ptr;
+  uint64_t n64;      // 8-byte words
+  uint64_t pattern;  // 64-bit fill value
+};
+struct FillHoist {
+  std::vector<FillRec>* rec = nullptr;  // record (and still perform) every fill
+  bool skip = false;                    // fills were hoisted: do nothing
+};
+FillHoist& fill_hoist();  // per host thread
+// bytes are rounded up to a multiple of 8 (every target allocation is padded)
+cudaError_t init_fill(void* ptr, size_t bytes, uint64_t pattern, cudaStream_t st);
+cudaError_t launch_multi_fill(const std::vector<FillRec>& recs, cudaStream_t st);
 
 struct FilterArgs {
   const ddq_dev_pred* preds = nullptr;
@@ -81,13 +101,16 @@ cudaError_t launch_groupby(const int32_t* tids, const uint32_t* d_count, int64_t
                            const int32_t* key_bits,
                            const ddq_dev_agg* aggs, int n_aggs, void* table, uint32_t capacity,
                            uint32_t* d_error, cudaStream_t st);
+// AGGREGATE with fused predicates (reading O26): only input rows passing every
+// predicate contribute; *d_rows (optional) += the number that did.
 // warp-autonomous aggregation for <= 2 aggregates and small group counts (agg.cu)
 bool agg_ws_supported(const int32_t* tids, const int32_t* const* key_vec, int n_keys, int n_aggs,
                       uint32_t capacity);
 cudaError_t launch_agg_ws(const int32_t* tids, const uint32_t* d_count, int64_t n_cap,
                           const int32_t* const* key_vec, const int32_t* const* key_col, int n_keys,
                           const int32_t* key_bits, const ddq_dev_agg* aggs, int n_aggs, void* table,
-                          uint32_t capacity, uint32_t* d_error, cudaStream_t st);
+                          uint32_t capacity, uint32_t* d_error, cudaStream_t st,
+                          const BuildPreds* preds = nullptr, uint32_t* d_rows = nullptr);
 cudaError_t launch_groupby_compact(const void* table, uint32_t capacity, int n_aggs, int64_t* out_keys,
                                    int64_t* out_accs, uint32_t* d_out_groups, cudaStream_t st);
 

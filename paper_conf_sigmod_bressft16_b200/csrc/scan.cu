@@ -705,7 +705,7 @@ cudaError_t launch_scan(const FilterArgs& a, cudaStream_t st) {
   p.d_out_count = a.d_out_count;
   p.out_cap = (uint32_t)(a.out_cap > 0 ? a.out_cap : a.n_cap);
   p.d_overflow = a.d_overflow;
-  cudaError_t e = cudaMemsetAsync(a.d_out_count, 0, 8, st);
+  cudaError_t e = init_fill(a.d_out_count, 8, 0, st);
   if (e != cudaSuccess) return e;
   const size_t smem = (size_t)p.shared_off + shared;
   const int64_t ntiles = (a.n_cap + SC_TILE - 1) / SC_TILE;  // upper bound (TID mode: capacity)

@@ -415,7 +415,7 @@ cudaError_t launch_star(const ddq_dev_term* terms, int n_terms, int64_t n_rows, 
   p.d_out_count = d_out_count;
   p.out_cap = (uint32_t)(out_cap > 0 ? out_cap : n_rows);
   p.d_overflow = d_overflow;
-  cudaError_t e = cudaMemsetAsync(d_out_count, 0, 8, st);
+  cudaError_t e = init_fill(d_out_count, 8, 0, st);
   if (e != cudaSuccess) return e;
   const size_t smem = (size_t)shared_base + shared;
   const int64_t ntiles = (n_rows + p.tile - 1) / p.tile;

@@ -161,11 +161,16 @@ class PlanBuilder:
         return idx
 
     def aggregate(self, table: str, input: int, keys: list, aggs: list, order_by: list | None = None,
-                  max_groups: int = 0, limit: int = 0, key_bits: list | None = None) -> int:
+                  max_groups: int = 0, limit: int = 0, key_bits: list | None = None,
+                  where: list | None = None) -> int:
         """keys: int (aligned vector index) or str (column of `table`).
         aggs: (kind, [cols]).  order_by: ints per include/ddq.h (+/-(1+k), +/-(101+a)).
-        key_bits: bits per key in the packed group key (default 21 each, sum <= 63)."""
+        key_bits: bits per key in the packed group key (default 21 each, sum <= 63).
+        where: predicates on the input rows evaluated inside the aggregation (a fused
+        selection, reading O26), same forms as select()."""
         idx, op = self._op(A.OP_AGGREGATE, table, input)
+        if where:
+            self._preds(op, table, where)
         for k, b in enumerate(key_bits or []):
             op.key_bits[k] = b
         op.n_keys = len(keys)

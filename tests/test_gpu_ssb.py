@@ -52,7 +52,7 @@ def _oracle(kind, q):
 
 VARIANTS = {"star": dict(star=True), "chain": dict(star=False),
             "chain_eager": dict(star=False, late=False),
-            "chain_unfused": dict(star=False, fused_build=False, late=False)}
+            "chain_unfused": dict(star=False, fused_build=False, late=False, fused_agg=False)}
 
 
 @pytest.mark.parametrize("variant", list(VARIANTS))

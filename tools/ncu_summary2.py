@@ -30,17 +30,13 @@ def main(path):
                 try:
                     unit = rows[1][idx[k]]
                     v = float(r[idx[k]].replace(",", ""))
-                    if unit in ("usecond",) and lab == "us":
-                        v *= 1e3
-                    if unit == "msecond" and lab == "us":
-                        v *= 1e6
-                    if unit == "Kbyte":
-                        v *= 1e3
-                    if unit == "Gbyte":
-                        v *= 1e9
-                    if unit == "Mbyte":
-                        v *= 1e6
-                    parts.append(f"{lab}={v*sc:.1f}")
+                    scale = {"nsecond": 1e-3, "usecond": 1.0, "msecond": 1e3, "byte": 1e-6, "Kbyte": 1e-3,
+                             "Mbyte": 1.0, "Gbyte": 1e3}.get(unit)
+                    if lab in ("us", "MB_rd", "MB_wr") and scale is not None:
+                        v = v * scale
+                    else:
+                        v = v * sc
+                    parts.append(f"{lab}={v:.1f}")
                 except ValueError:
                     pass
         stalls = []

@@ -35,6 +35,22 @@ def main():
         return
     names = {0: "dense", 1: "at-tids", 2: "build", 3: "gather", 4: "agg"}
     tot = {}
+    # whole-graph time per query (the plan's CUDA graph, branches overlapped)
+    stream = torch.cuda.Stream()
+    gsum = 0.0
+    for q, p in preps.items():
+        for _ in range(3):
+            p.launch(stream.cuda_stream)
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        for _ in range(20):
+            p.launch(stream.cuda_stream)
+        e1.record(stream)
+        torch.cuda.synchronize()
+        g = e0.elapsed_time(e1) / 20
+        gsum += g
+        print(f"{q} graph {g*1e3:.0f}us")
+    print(f"graphs   {gsum*1e3:9.0f} us (sum of per-query graph times)")
     for q, p in preps.items():
         for _ in range(3):
             p.launch()
