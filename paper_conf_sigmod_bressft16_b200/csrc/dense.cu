@@ -77,6 +77,8 @@ struct WsParams {
   uint32_t n;                  // dense: rows; TID input: capacity (count in d_in_count)
   const uint32_t* d_in_count;  // TID input
   const int32_t* in_tids;      // TID input
+  const uint32_t* in_bits;     // row-bitmap input (n = rows): 16 words per 512-row tile
+  uint32_t* out_bits;          // row-bitmap output (dense probe / select, no payload)
   int32_t n_preds;
   WsPred preds[4];
   const int32_t* eq_a;
@@ -168,8 +170,14 @@ __device__ __forceinline__ void unpack16(const int4 (&r)[4], int32_t (&v)[WS_ITE
   }
 }
 
-template <int kKind, bool kTids, bool kPay, bool kCarry>
-__global__ void __launch_bounds__(ws_nw(kTids) * 32, 1) ws_kernel(const __grid_constant__ WsParams P) {
+// kIn: 0 = every row of the table (keys streamed), 1 = a TID list, 2 = a row
+// bitmap (tiles of 16 words; item j of lane l is row tile*512 + j*32 + l, so the
+// gathers of one item index are coalesced).  kOutBits: the survivors are written as
+// a row bitmap (no ring, no TIDs): one 32-bit word per 32 rows, from the lanes'
+// hit nibbles OR-reduced over groups of 8 lanes.
+template <int kKind, int kIn, bool kPay, bool kCarry, bool kOutBits>
+__global__ void __launch_bounds__(ws_nw(kIn != 0) * 32, 1) ws_kernel(const __grid_constant__ WsParams P) {
+  constexpr bool kTids = kIn != 0;  // sv[] holds TIDs (gathers at them)
   extern __shared__ __align__(16) uint8_t smem[];
   __shared__ uint32_t s_cnt, s_base;
   __shared__ uint32_t s_filled[WS_R], s_gen[WS_R];
@@ -194,23 +202,40 @@ __global__ void __launch_bounds__(ws_nw(kTids) * 32, 1) ws_kernel(const __grid_c
   __syncthreads();
 
   const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  const uint32_t n = kTids ? ld_relaxed_u32(P.d_in_count) : P.n;
+  const uint32_t n = kIn == 1 ? ld_relaxed_u32(P.d_in_count) : P.n;
   const uint32_t ntiles = (n + WS_TILE - 1) / WS_TILE;
   constexpr uint32_t NW = ws_nw(kTids);
   const uint32_t W = gridDim.x * NW;
   uint32_t tile = blockIdx.x * NW + warp;
   const uint32_t lofs = lane * 4;  // item (s, v) of lane l sits at tile*512 + s*128 + l*4 + v
-  const int32_t* stream = kTids ? P.in_tids : P.fk;  // the column streamed through registers
-  int4 nk[4];
-  if (tile < ntiles) load16(stream, tile * WS_TILE, lofs, n, nk);
+  const int32_t* stream = kIn == 1 ? P.in_tids : P.fk;  // the column streamed through registers
+  int4 nk[4];  // next tile: 16 keys / TIDs of this lane, or the tile's 16 bitmap words (kIn 2)
+  auto fetch = [&](uint32_t t) {
+    if (kIn == 2) {
+      const int4* wp = reinterpret_cast<const int4*>(P.in_bits + (size_t)t * 16);
+#pragma unroll
+      for (int s2 = 0; s2 < 4; s2++) nk[s2] = __ldg(wp + s2);  // same 64 B for every lane
+    } else {
+      load16(stream, t * WS_TILE, lofs, n, nk);
+    }
+  };
+  if (tile < ntiles) fetch(tile);
+  uint32_t bits_cnt = 0;  // kOutBits: survivors of this lane
 
   for (; tile < ntiles; tile += W) {
     int32_t sv[WS_ITEMS];  // streamed values: keys (dense probe) or TIDs
     unpack16(nk, sv);
-    const uint32_t base = tile * WS_TILE + lofs;  // position of the lane's item 0
-    if (tile + W < ntiles) load16(stream, (tile + W) * WS_TILE, lofs, n, nk);
+    const uint32_t base = tile * WS_TILE + lofs;  // position of the lane's item 0 (kIn 0, 1)
+    if (tile + W < ntiles) fetch(tile + W);
     uint32_t flags = 0xFFFFu;
-    if (tile * WS_TILE + WS_TILE > n) {
+    if (kIn == 2) {  // bitmap words -> this lane's rows of the tile
+      flags = 0;
+#pragma unroll
+      for (int j = 0; j < WS_ITEMS; j++) flags |= (((uint32_t)sv[j] >> lane) & 1u) << j;
+      if (__all_sync(FULL, flags == 0)) continue;  // an empty 512-row tile
+#pragma unroll
+      for (int j = 0; j < WS_ITEMS; j++) sv[j] = (int32_t)(tile * WS_TILE + j * 32 + lane);
+    } else if (tile * WS_TILE + WS_TILE > n) {
       flags = 0;
 #pragma unroll
       for (int j = 0; j < WS_ITEMS; j++) flags |= (base + (j >> 2) * 128 + (j & 3) < n ? 1u : 0u) << j;
@@ -221,7 +246,7 @@ __global__ void __launch_bounds__(ws_nw(kTids) * 32, 1) ws_kernel(const __grid_c
       if (!kTids) {
 #pragma unroll
         for (int j = 0; j < WS_ITEMS; j++) key[j] = sv[j];
-      } else if (P.fk_by_pos) {  // positional key vector: coalesced
+      } else if (kIn == 1 && P.fk_by_pos) {  // positional key vector: coalesced
         int4 kk[4];
         load16(P.fk, tile * WS_TILE, lofs, n, kk);
         unpack16(kk, key);
@@ -239,7 +264,7 @@ __global__ void __launch_bounds__(ws_nw(kTids) * 32, 1) ws_kernel(const __grid_c
             hit = (s_bm[oo >> 5] >> (oo & 31)) & 1u;
           } else {
             const uint32_t o = (uint32_t)(key[j] - P.key_min);
-            hit = o < P.range ? (ldg_gather(P.bitmap + (o >> 5)) >> (o & 31)) & 1u : 0u;
+            hit = o < P.range ? (__ldg(P.bitmap + (o >> 5)) >> (o & 31)) & 1u : 0u;
           }
           m |= hit << j;
         }
@@ -250,7 +275,7 @@ __global__ void __launch_bounds__(ws_nw(kTids) * 32, 1) ws_kernel(const __grid_c
           for (int j = 0; j < WS_ITEMS; j++) {
             pay[j] = 0;
             if ((any >> j) & 1u)
-              if ((flags >> j) & 1u) pay[j] = ldg_gather(P.payarr + (uint32_t)(key[j] - P.key_min));
+              if ((flags >> j) & 1u) pay[j] = __ldg(P.payarr + (uint32_t)(key[j] - P.key_min));
           }
         }
       } else {
@@ -259,17 +284,17 @@ __global__ void __launch_bounds__(ws_nw(kTids) * 32, 1) ws_kernel(const __grid_c
           pay[j] = 0;
           if ((flags >> j) & 1u) {
             uint32_t h = ht_hash(key[j], P.shift);
-            uint64_t s = kKind == WK_HT_SMEM ? s_ht[h] : ldg_gather(P.table + h);
+            uint64_t s = kKind == WK_HT_SMEM ? s_ht[h] : __ldg(P.table + h);
             while (s != HT_EMPTY && ht_key(s) != key[j]) {
               h = (h + 1) & P.cap_mask;
-              s = kKind == WK_HT_SMEM ? s_ht[h] : ldg_gather(P.table + h);
+              s = kKind == WK_HT_SMEM ? s_ht[h] : __ldg(P.table + h);
             }
             if (s == HT_EMPTY) flags &= ~(1u << j);
             pay[j] = ht_val(s);
           }
         }
       }
-    } else if (kKind == WK_EQ) {
+    } else if (kKind == WK_EQ && kIn == 1) {
       int4 a4[4], b4[4];
       load16(P.eq_a, tile * WS_TILE, lofs, n, a4);
       load16(P.eq_b, tile * WS_TILE, lofs, n, b4);
@@ -311,6 +336,18 @@ __global__ void __launch_bounds__(ws_nw(kTids) * 32, 1) ws_kernel(const __grid_c
         }
         flags &= m;
       }
+    }
+    if (kOutBits) {  // ---- row bitmap output: word (s, q) covers rows s*128 + 32q .. +32
+      bits_cnt += __popc(flags);
+#pragma unroll
+      for (int s2 = 0; s2 < 4; s2++) {
+        uint32_t w = ((flags >> (4 * s2)) & 0xFu) << (4 * (lane & 7));
+        w |= __shfl_xor_sync(FULL, w, 1);
+        w |= __shfl_xor_sync(FULL, w, 2);
+        w |= __shfl_xor_sync(FULL, w, 4);
+        if ((lane & 7) == 0) P.out_bits[(size_t)tile * 16 + s2 * 4 + (lane >> 3)] = w;
+      }
+      continue;
     }
     // ---- compaction: warp scan of the lanes' hit counts, one smem claim --------
     const uint32_t c = __popc(flags);
@@ -422,6 +459,13 @@ __global__ void __launch_bounds__(ws_nw(kTids) * 32, 1) ws_kernel(const __grid_c
       }
     }
   }
+  if (kOutBits) {  // survivor count: warp sum -> CTA -> one global atomic
+    bits_cnt = __reduce_add_sync(FULL, bits_cnt);
+    if (lane == 0 && bits_cnt) atomicAdd(&s_cnt, bits_cnt);
+    __syncthreads();
+    if (threadIdx.x == 0 && s_cnt) atomicAdd(P.d_out_count, s_cnt);
+    return;
+  }
   // the CTA's last, partial block: an exact reservation (no holes)
   __syncthreads();
   const uint32_t total = s_cnt;
@@ -445,40 +489,66 @@ __global__ void __launch_bounds__(ws_nw(kTids) * 32, 1) ws_kernel(const __grid_c
 int g_optin = 0;
 constexpr size_t kWsCtl = 1024;  // static smem + reserve
 
-template <int K, bool T, bool Pa, bool C>
+template <int K, int In, bool Pa, bool C, bool Ob>
 void ws_attr() {
-  cudaFuncSetAttribute(ws_kernel<K, T, Pa, C>, cudaFuncAttributeMaxDynamicSharedMemorySize, g_optin - (int)kWsCtl);
+  cudaFuncSetAttribute(ws_kernel<K, In, Pa, C, Ob>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                       g_optin - (int)kWsCtl);
 }
 template <int K>
 void ws_attr_kind() {
-  if constexpr (K <= WK_HT_GLOBAL) {  // dense inputs: probes only
-    ws_attr<K, false, false, false>();
-    ws_attr<K, false, true, false>();
+  constexpr bool kProbe = K <= WK_HT_GLOBAL;
+  if constexpr (kProbe) {  // dense inputs: probes only (payload, or a bitmap of the survivors)
+    ws_attr<K, 0, false, false, false>();
+    ws_attr<K, 0, true, false, false>();
+    ws_attr<K, 0, false, false, true>();
   }
-  ws_attr<K, true, false, false>();
-  ws_attr<K, true, true, false>();
-  ws_attr<K, true, false, true>();
-  ws_attr<K, true, true, true>();
+  ws_attr<K, 1, false, false, false>();
+  ws_attr<K, 1, false, true, false>();
+  if constexpr (kProbe) {
+    ws_attr<K, 1, true, false, false>();
+    ws_attr<K, 1, true, true, false>();
+  }
+  if constexpr (K != WK_EQ) {  // bitmap inputs carry no vectors
+    ws_attr<K, 2, false, false, false>();
+    if constexpr (kProbe) ws_attr<K, 2, true, false, false>();
+  }
 }
 
 template <int K>
-void launch_k(bool tids, bool pay, bool carry, int grid, size_t smem, cudaStream_t st, const WsParams& p) {
-  if constexpr (K <= WK_HT_GLOBAL) {  // dense inputs: probes only
-    if (!tids) {
+void launch_k(int in, bool pay, bool carry, bool obits, int grid, size_t smem, cudaStream_t st,
+              const WsParams& p) {
+  constexpr bool kProbe = K <= WK_HT_GLOBAL;
+  if constexpr (kProbe) {
+    if (in == 0) {
       const dim3 blk(ws_nw(false) * 32);
-      if (pay) ws_kernel<K, false, true, false><<<grid, blk, smem, st>>>(p);
-      else ws_kernel<K, false, false, false><<<grid, blk, smem, st>>>(p);
+      if (obits) ws_kernel<K, 0, false, false, true><<<grid, blk, smem, st>>>(p);
+      else if (pay) ws_kernel<K, 0, true, false, false><<<grid, blk, smem, st>>>(p);
+      else ws_kernel<K, 0, false, false, false><<<grid, blk, smem, st>>>(p);
       return;
     }
   }
   const dim3 blk(ws_nw(true) * 32);
-  if (carry) {
-    if (pay) ws_kernel<K, true, true, true><<<grid, blk, smem, st>>>(p);
-    else ws_kernel<K, true, false, true><<<grid, blk, smem, st>>>(p);
-  } else {
-    if (pay) ws_kernel<K, true, true, false><<<grid, blk, smem, st>>>(p);
-    else ws_kernel<K, true, false, false><<<grid, blk, smem, st>>>(p);
+  if constexpr (K != WK_EQ) {
+    if (in == 2) {
+      if constexpr (kProbe) {
+        if (pay) {
+          ws_kernel<K, 2, true, false, false><<<grid, blk, smem, st>>>(p);
+          return;
+        }
+      }
+      ws_kernel<K, 2, false, false, false><<<grid, blk, smem, st>>>(p);
+      return;
+    }
   }
+  if constexpr (kProbe) {
+    if (pay) {
+      if (carry) ws_kernel<K, 1, true, true, false><<<grid, blk, smem, st>>>(p);
+      else ws_kernel<K, 1, true, false, false><<<grid, blk, smem, st>>>(p);
+      return;
+    }
+  }
+  if (carry) ws_kernel<K, 1, false, true, false><<<grid, blk, smem, st>>>(p);
+  else ws_kernel<K, 1, false, false, false><<<grid, blk, smem, st>>>(p);
 }
 
 }  // namespace
@@ -486,7 +556,11 @@ void launch_k(bool tids, bool pay, bool carry, int grid, size_t smem, cudaStream
 bool ws_supported(const FilterArgs& a) {
   const bool tids = a.in_tids != nullptr;
   if (a.n_carry > 4 || a.n_cap > (int64_t)0x7FFFFFFF) return false;
-  if (!tids) {  // dense: probes only (dense selections stream several columns: scan.cu)
+  if (a.out_bits && (a.in_tids || a.in_bits || !a.probe || a.out_payload)) return false;
+  if (a.in_bits) {  // row bitmap input: probes at a key column and selections, no vectors
+    if (a.fk_by_pos || a.eq_a || a.n_carry || ((uintptr_t)a.in_bits & 15) != 0) return false;
+    if (!a.probe && (a.n_preds < 1 || a.n_preds > 4)) return false;
+  } else if (!tids) {  // dense: probes only (dense selections stream several columns: scan.cu)
     if (!a.probe || a.fk_by_pos || a.eq_a || a.n_carry) return false;
     if (((uintptr_t)a.fk & 15) != 0) return false;
   } else {
@@ -522,15 +596,19 @@ cudaError_t launch_ws(const FilterArgs& a, cudaStream_t st) {
     ws_attr_kind<WK_SEL_GENERIC>();
     ws_attr_kind<WK_EQ>();
   }
-  const bool tids = a.in_tids != nullptr;
+  const int in = a.in_bits ? 2 : (a.in_tids ? 1 : 0);
+  const bool tids = in != 0;
   WsParams p{};
   p.n = (uint32_t)a.n_cap;
   p.d_in_count = a.d_in_count;
   p.in_tids = a.in_tids;
+  p.in_bits = a.in_bits;
+  p.out_bits = a.out_bits;
+  const bool obits = a.out_bits != nullptr;
   const bool pay = a.probe && a.out_payload != nullptr;
-  const bool carry = tids && a.n_carry > 0;
+  const bool carry = in == 1 && a.n_carry > 0;
   const int n_fields = 1 + (pay ? 1 : 0) + (carry ? a.n_carry : 0);
-  const size_t ring = (size_t)ws_blk(carry) * WS_R * 4 * n_fields;
+  const size_t ring = obits ? 0 : (size_t)ws_blk(carry) * WS_R * 4 * n_fields;
   const size_t budget = (size_t)g_optin - kWsCtl;
   int kind;
   size_t tab = 0;
@@ -600,13 +678,13 @@ cudaError_t launch_ws(const FilterArgs& a, cudaStream_t st) {
   const int64_t need = (ntiles + ws_nw(tids) - 1) / ws_nw(tids);
   if (grid > need) grid = need < 1 ? 1 : need;
   switch (kind) {
-    case WK_BM_SMEM: launch_k<WK_BM_SMEM>(tids, pay, carry, (int)grid, smem, st, p); break;
-    case WK_BM_GLOBAL: launch_k<WK_BM_GLOBAL>(tids, pay, carry, (int)grid, smem, st, p); break;
-    case WK_HT_SMEM: launch_k<WK_HT_SMEM>(tids, pay, carry, (int)grid, smem, st, p); break;
-    case WK_HT_GLOBAL: launch_k<WK_HT_GLOBAL>(tids, pay, carry, (int)grid, smem, st, p); break;
-    case WK_SEL_RANGE: launch_k<WK_SEL_RANGE>(tids, false, carry, (int)grid, smem, st, p); break;
-    case WK_SEL_GENERIC: launch_k<WK_SEL_GENERIC>(tids, false, carry, (int)grid, smem, st, p); break;
-    default: launch_k<WK_EQ>(tids, false, carry, (int)grid, smem, st, p); break;
+    case WK_BM_SMEM: launch_k<WK_BM_SMEM>(in, pay, carry, obits, (int)grid, smem, st, p); break;
+    case WK_BM_GLOBAL: launch_k<WK_BM_GLOBAL>(in, pay, carry, obits, (int)grid, smem, st, p); break;
+    case WK_HT_SMEM: launch_k<WK_HT_SMEM>(in, pay, carry, obits, (int)grid, smem, st, p); break;
+    case WK_HT_GLOBAL: launch_k<WK_HT_GLOBAL>(in, pay, carry, obits, (int)grid, smem, st, p); break;
+    case WK_SEL_RANGE: launch_k<WK_SEL_RANGE>(in, false, carry, false, (int)grid, smem, st, p); break;
+    case WK_SEL_GENERIC: launch_k<WK_SEL_GENERIC>(in, false, carry, false, (int)grid, smem, st, p); break;
+    default: launch_k<WK_EQ>(in, false, carry, false, (int)grid, smem, st, p); break;
   }
   return cudaGetLastError();
 }

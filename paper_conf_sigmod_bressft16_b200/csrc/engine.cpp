@@ -160,6 +160,8 @@ ddq_status run_gpu_op(GpuOpCtx& ctx, const ddq_op& op, Inter& out) {
   const Table& T = db->tables[(size_t)op.table];
   const Inter* in = op.input >= 0 ? &I[(size_t)op.input] : nullptr;
   if (in && in->on_host) return set_error(DDQ_ESTATE, "GPU op with a host-resident input");
+  if (in && in->bits && op.kind != DDQ_OP_SELECT && op.kind != DDQ_OP_HASH_PROBE)
+    return set_error(DDQ_ESTATE, "op cannot read a row-bitmap input");
   const int32_t* in_tids = in ? in->tids : nullptr;
   const uint32_t* in_cnt = in ? in->d_count : nullptr;
   const int64_t in_cap = in ? in->cap : T.n_rows;
@@ -229,8 +231,10 @@ ddq_status run_gpu_op(GpuOpCtx& ctx, const ddq_op& op, Inter& out) {
           cin.push_back((const int32_t*)v.ptr);
         }
       }
-      out.cap = out_cap;
-      out.tids = (int32_t*)A.get((uint64_t)std::max<int64_t>(out_cap, 1) * 4);
+      const bool obits = ctx.bits_out && !in && probe && !op.emit_payload;
+      out.cap = obits ? T.n_rows : out_cap;
+      if (obits) out.bits = (uint32_t*)A.get(row_bitmap_bytes(T.n_rows));
+      else out.tids = (int32_t*)A.get((uint64_t)std::max<int64_t>(out_cap, 1) * 4);
       out.d_count = (uint32_t*)A.get(64);
       for (size_t c = 0; c < cin.size(); c++) {
         int32_t* p = (int32_t*)A.get((uint64_t)std::max<int64_t>(out_cap, 1) * 4);
@@ -267,6 +271,13 @@ ddq_status run_gpu_op(GpuOpCtx& ctx, const ddq_op& op, Inter& out) {
       fa.in_tids = in_tids;
       fa.d_in_count = in_cnt;
       fa.n_cap = in_cap;
+      if (in && in->bits) {  // row bitmap input: every row of the table, masked
+        fa.in_bits = in->bits;
+        fa.in_tids = nullptr;
+        fa.d_in_count = nullptr;
+        fa.n_cap = T.n_rows;
+      }
+      if (obits) fa.out_bits = out.bits;
       fa.carry_in = cin.data();
       fa.carry_out = cout.data();
       fa.n_carry = (int)cin.size();
@@ -950,6 +961,7 @@ struct ddq_prepared {
   ddq_plan plan{};
   std::vector<ddq::Inter> inters;
   std::vector<int64_t> forced;  // per-op output capacity (exact count + slack)
+  std::vector<char> bits_out;   // per op: survivors as a row bitmap (see GpuOpCtx)
   cudaGraph_t graph = nullptr;
   cudaGraphExec_t exec = nullptr;
   bool use_graph = false;
@@ -1029,6 +1041,7 @@ static ddq_status replay_op(ddq_prepared* P, int i, cudaStream_t st) {
   ctx.forced_cap = P->forced[(size_t)i];
   ctx.count_column_access = false;
   ctx.reuse = &blocks;
+  ctx.bits_out = P->bits_out[(size_t)i] != 0;
   return run_gpu_op(ctx, P->plan.ops[i], P->inters[(size_t)i]);
 }
 static ddq_status replay(ddq_prepared* P, cudaStream_t st) {
@@ -1212,12 +1225,33 @@ ddq_status ddq_prepare(ddq_db* db, const ddq_plan* plan, int32_t use_graph, ddq_
         op.kind == DDQ_OP_FILTER_EQ)
       P->forced[(size_t)i] = counts[(size_t)i] + counts[(size_t)i] / 64 + 256;
   }
+  // a dense semi-join probe (no payload) whose consumers are all probes / selections
+  // of its output hands them a row bitmap (N/8 bytes) instead of a TID list
+  P->bits_out.assign((size_t)plan->n_ops, 0);
+  {
+    static const char* env = getenv("DDQ_ROW_BITMAPS");  // "0": TID lists only
+    const bool allow = !env || env[0] != '0';
+    for (int i = 0; i < plan->n_ops && allow; i++) {
+      const ddq_op& op = plan->ops[i];
+      if (op.kind != DDQ_OP_HASH_PROBE || op.input >= 0 || op.emit_payload || op.fk_vec > 0) continue;
+      int consumers = 0;
+      bool ok = true;
+      for (int j = i + 1; j < plan->n_ops; j++) {
+        const ddq_op& c = plan->ops[j];
+        if (c.input != i) continue;
+        consumers++;
+        ok = ok && ((c.kind == DDQ_OP_HASH_PROBE && c.fk_vec <= 0) || c.kind == DDQ_OP_SELECT);
+      }
+      P->bits_out[(size_t)i] = (ok && consumers > 0) ? 1 : 0;
+    }
+  }
   P->inters.resize((size_t)plan->n_ops);
   fill_hoist().rec = &P->fills;  // record every buffer initialisation of the eager run
   for (int i = 0; i < plan->n_ops; i++) {
     GpuOpCtx ctx{db, st, &P->inters};
     ctx.forced_cap = P->forced[(size_t)i];
     ctx.count_column_access = false;
+    ctx.bits_out = P->bits_out[(size_t)i] != 0;
     ddq_status s = run_gpu_op(ctx, plan->ops[i], P->inters[(size_t)i]);
     if (s != DDQ_OK) {
       fill_hoist().rec = nullptr;
@@ -1290,6 +1324,7 @@ int32_t ddq_prepared_profile(ddq_prepared* p, void* stream, int32_t max_ops, flo
     ctx.forced_cap = p->forced[(size_t)i];
     ctx.count_column_access = false;
     ctx.reuse = &blocks;
+    ctx.bits_out = p->bits_out[(size_t)i] != 0;
     ddq_status s = run_gpu_op(ctx, p->plan.ops[i], p->inters[(size_t)i]);
     if (s != DDQ_OK) {
       for (auto& e : ev) cudaEventDestroy(e);
@@ -1330,19 +1365,20 @@ int32_t ddq_prepared_profile(ddq_prepared* p, void* stream, int32_t max_ops, flo
         else
           cols.push_back(op.fk_col);
         const int emit = op.kind == DDQ_OP_HASH_PROBE && op.emit_payload ? 1 : 0;
+        const bool in_bits = op.input >= 0 && p->inters[(size_t)op.input].bits;
         if (op.input < 0) {
           cls = 0;
           for (int c : cols) bytes += N * width(c);
         } else {
           cls = 1;
-          bytes += m * 4;
+          bytes += in_bits ? N / 8 : m * 4;  // the input: a row bitmap or a TID list
           // a conjunction reads its first column at every input TID and the
           // others only at rows still alive (counted at the final survivors: a
           // lower bound, intermediate counts are not kept)
           for (size_t k = 0; k < cols.size(); k++) bytes += sector_bytes(N, k == 0 ? m : out, width(cols[k]));
           bytes += out * 4 * nvec_in;  // carried vectors read at survivors
         }
-        bytes += out * 4 * (1 + nvec_in + emit);
+        bytes += o.bits ? N / 8 : out * 4 * (1 + nvec_in + emit);  // row bitmap or TIDs + vectors
       } break;
       case DDQ_OP_STAR: {
         cls = 0;

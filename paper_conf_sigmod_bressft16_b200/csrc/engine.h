@@ -79,6 +79,7 @@ struct Inter {
   bool all_rows = false;   // implicit TIDs 0..cap-1
   int table = -1;
   int32_t* tids = nullptr;
+  uint32_t* bits = nullptr;     // row bitmap instead of a TID list (prepared plans, see bits_out)
   uint32_t* d_count = nullptr;  // device count cell (GPU)
   int64_t cap = 0;              // capacity (upper bound on count)
   int64_t count = -1;           // exact count when known on the host
@@ -154,6 +155,9 @@ struct GpuOpCtx {
   int64_t forced_cap = -1;           // output capacity override
   bool count_column_access = true;
   const std::vector<void*>* reuse = nullptr;  // replay on existing buffers
+  // a dense semi-join probe writes its survivors as a row bitmap (1 bit per row)
+  // instead of a TID list: set by ddq_prepare when every consumer reads bitmaps
+  bool bits_out = false;
 };
 void count_accesses(ddq_db* db, const ddq_op& op);
 void driver_start(ddq_db* db);

@@ -322,6 +322,10 @@ size_t filter_scratch_bytes(int64_t n_cap) {
 constexpr size_t kSmemTableMax = 96 * 1024;
 
 cudaError_t launch_filter(const FilterArgs& a, cudaStream_t st) {
+  if (a.in_bits || a.out_bits) {  // row bitmaps exist only for the warp-autonomous kernels
+    if (!ws_supported(a)) return cudaErrorInvalidValue;
+    return launch_ws(a, st);
+  }
   if (!a.stable && ws_supported(a)) {
     static const char* env = getenv("DDQ_WS");  // "0": the group-pipelined scan kernel (scan.cu)
     if (!env || env[0] != '0') return launch_ws(a, st);

@@ -48,6 +48,10 @@ struct FilterArgs {
   int32_t* out_payload = nullptr;
   const int32_t* in_tids = nullptr;
   const uint32_t* d_in_count = nullptr;
+  // row bitmap input (instead of in_tids; n_cap = the table's rows): 16 words per
+  // 512-row tile; row bitmap output of a dense probe (instead of out_tids); see dense.cu
+  const uint32_t* in_bits = nullptr;
+  uint32_t* out_bits = nullptr;
   int64_t n_cap = 0;
   const int32_t* const* carry_in = nullptr;
   int32_t* const* carry_out = nullptr;
@@ -65,6 +69,7 @@ cudaError_t launch_scan(const FilterArgs& a, cudaStream_t st);
 cudaError_t launch_filter(const FilterArgs& a, cudaStream_t st);
 // warp-autonomous filter kernels (dense.cu): dense probes and every TID-input operator
 bool ws_supported(const FilterArgs& a);
+inline size_t row_bitmap_bytes(int64_t rows) { return (size_t)((rows + 511) / 512) * 64; }
 cudaError_t launch_ws(const FilterArgs& a, cudaStream_t st);
 
 // HASH_BUILD with a fused selection (a BUILD op carrying predicates): rows that
