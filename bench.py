@@ -335,15 +335,27 @@ def main():
             cls_ms[cl] = cls_ms.get(cl, 0.0) + ms_
             cls_bytes[cl] = cls_bytes.get(cl, 0.0) + by
             cls_n[cl] = cls_n.get(cl, 0) + 1
-    names = {0: "dense scan (select/probe over all rows)", 1: "select/probe at TIDs", 2: "hash build",
-             3: "gather", 4: "group-by aggregate"}
+    names = {0: "ws_kernel (csrc/dense.cu): dense probe over all rows", 1: "ws_kernel (csrc/dense.cu): "
+             "select/probe over a TID list or row bitmap", 2: "join_index_build_kernel (csrc/kernels.cu): build",
+             3: "gather_kernel (csrc/kernels.cu)", 4: "agg_ws_kernel (csrc/agg.cu): group-by aggregate"}
+    tclass = {0: "dense", 1: "at-tids", 2: "build", 3: "other", 4: "agg"}
     dom = max(cls_ms, key=lambda c: cls_ms[c])
     pk = peaks()
     hbm_peak = pk.get("hbm_gbs", 6650.0)
     achieved = cls_bytes[dom] / (cls_ms[dom] / 1e3) / 1e9
     step_bytes = sum(cls_bytes.values())
-    roofline = {"bound": "hbm", "kernel": "scan_kernel: " + names[dom], "achieved": round(achieved, 1),
-                "peak": hbm_peak, "unit": "GB/s", "frac": round(achieved / hbm_peak, 4), "traffic": None,
+    # measured DRAM traffic per launch of this kernel class: ncu launch list of the
+    # bench command (tools/ncu_traffic.py -> profiles/r1_traffic.json)
+    traffic = None
+    try:
+        tr = json.load(open(os.path.join(ROOT, "profiles", "r1_traffic.json")))["classes"][tclass[dom]]
+        traffic = {"dram_bytes_per_launch": tr["dram_bytes_per_launch"],
+                   "algorithmic_bytes_per_launch": round(cls_bytes[dom] / cls_n[dom]),
+                   "source": "ncu dram__bytes_read.sum + dram__bytes_write.sum, profiles/r1_traffic.json"}
+    except Exception:
+        pass
+    roofline = {"bound": "hbm", "kernel": names[dom], "achieved": round(achieved, 1),
+                "peak": hbm_peak, "unit": "GB/s", "frac": round(achieved / hbm_peak, 4), "traffic": traffic,
                 "launches_per_step": cls_n[dom], "share_of_step": round(cls_ms[dom] / sum(cls_ms.values()), 3),
                 "peak_source": "MEASURED_PEAKS.json hbm_gbs (measured)" if "hbm_gbs" in pk else "fallback 6.65 TB/s",
                 "step_model_gb": round(step_bytes / 1e9, 3),

@@ -170,14 +170,17 @@ __device__ __forceinline__ void unpack16(const int4 (&r)[4], int32_t (&v)[WS_ITE
   }
 }
 
-// kIn: 0 = every row of the table (keys streamed), 1 = a TID list, 2 = a row
-// bitmap (tiles of 16 words; item j of lane l is row tile*512 + j*32 + l, so the
-// gathers of one item index are coalesced).  kOutBits: the survivors are written as
-// a row bitmap (no ring, no TIDs): one 32-bit word per 32 rows, from the lanes'
-// hit nibbles OR-reduced over groups of 8 lanes.
+// kIn: 0 = every row of the table (keys streamed), 1 = a TID list, 2 = every row
+// masked by a row bitmap (a dense probe of a dense intermediate: the key column is
+// streamed like kIn 0 -- at >= 1/8 of the rows a gather would touch nearly every
+// sector anyway -- and rows outside the bitmap are dead items).  Row bitmap: in the
+// kernel's own item order, one 16-bit word per lane and tile (64 B per 512 rows):
+// bit 4s+v of word tile*32+l = row tile*512 + s*128 + 4l + v.  kOutBits: the
+// survivors are written as such a bitmap -- each lane stores its hit flags (no
+// ring, no TIDs); a consumer prefetches one 16-bit word per tile.
 template <int kKind, int kIn, bool kPay, bool kCarry, bool kOutBits>
-__global__ void __launch_bounds__(ws_nw(kIn != 0) * 32, 1) ws_kernel(const __grid_constant__ WsParams P) {
-  constexpr bool kTids = kIn != 0;  // sv[] holds TIDs (gathers at them)
+__global__ void __launch_bounds__(ws_nw(kIn == 1) * 32, 1) ws_kernel(const __grid_constant__ WsParams P) {
+  constexpr bool kTids = kIn == 1;  // sv[] holds TIDs (gathers at them)
   extern __shared__ __align__(16) uint8_t smem[];
   __shared__ uint32_t s_cnt, s_base;
   __shared__ uint32_t s_filled[WS_R], s_gen[WS_R];
@@ -209,15 +212,12 @@ __global__ void __launch_bounds__(ws_nw(kIn != 0) * 32, 1) ws_kernel(const __gri
   uint32_t tile = blockIdx.x * NW + warp;
   const uint32_t lofs = lane * 4;  // item (s, v) of lane l sits at tile*512 + s*128 + l*4 + v
   const int32_t* stream = kIn == 1 ? P.in_tids : P.fk;  // the column streamed through registers
-  int4 nk[4];  // next tile: 16 keys / TIDs of this lane, or the tile's 16 bitmap words (kIn 2)
+  int4 nk[4];          // next tile: 16 keys / TIDs of this lane
+  uint32_t nflags = 0;  // kIn 2: next tile's row-bitmap word of this lane
+  const uint16_t* in_bits16 = reinterpret_cast<const uint16_t*>(P.in_bits);
   auto fetch = [&](uint32_t t) {
-    if (kIn == 2) {
-      const int4* wp = reinterpret_cast<const int4*>(P.in_bits + (size_t)t * 16);
-#pragma unroll
-      for (int s2 = 0; s2 < 4; s2++) nk[s2] = __ldg(wp + s2);  // same 64 B for every lane
-    } else {
-      load16(stream, t * WS_TILE, lofs, n, nk);
-    }
+    load16(stream, t * WS_TILE, lofs, n, nk);
+    if (kIn == 2) nflags = __ldg(in_bits16 + (size_t)t * 32 + lane);
   };
   if (tile < ntiles) fetch(tile);
   uint32_t bits_cnt = 0;  // kOutBits: survivors of this lane
@@ -225,16 +225,11 @@ __global__ void __launch_bounds__(ws_nw(kIn != 0) * 32, 1) ws_kernel(const __gri
   for (; tile < ntiles; tile += W) {
     int32_t sv[WS_ITEMS];  // streamed values: keys (dense probe) or TIDs
     unpack16(nk, sv);
-    const uint32_t base = tile * WS_TILE + lofs;  // position of the lane's item 0 (kIn 0, 1)
+    uint32_t flags = kIn == 2 ? nflags : 0xFFFFu;
+    const uint32_t base = tile * WS_TILE + lofs;  // position of the lane's item 0
     if (tile + W < ntiles) fetch(tile + W);
-    uint32_t flags = 0xFFFFu;
-    if (kIn == 2) {  // bitmap words -> this lane's rows of the tile
-      flags = 0;
-#pragma unroll
-      for (int j = 0; j < WS_ITEMS; j++) flags |= (((uint32_t)sv[j] >> lane) & 1u) << j;
+    if (kIn == 2) {
       if (__all_sync(FULL, flags == 0)) continue;  // an empty 512-row tile
-#pragma unroll
-      for (int j = 0; j < WS_ITEMS; j++) sv[j] = (int32_t)(tile * WS_TILE + j * 32 + lane);
     } else if (tile * WS_TILE + WS_TILE > n) {
       flags = 0;
 #pragma unroll
@@ -337,16 +332,9 @@ __global__ void __launch_bounds__(ws_nw(kIn != 0) * 32, 1) ws_kernel(const __gri
         flags &= m;
       }
     }
-    if (kOutBits) {  // ---- row bitmap output: word (s, q) covers rows s*128 + 32q .. +32
+    if (kOutBits) {  // ---- row bitmap output: the lane's hit flags, 64 B per warp tile
       bits_cnt += __popc(flags);
-#pragma unroll
-      for (int s2 = 0; s2 < 4; s2++) {
-        uint32_t w = ((flags >> (4 * s2)) & 0xFu) << (4 * (lane & 7));
-        w |= __shfl_xor_sync(FULL, w, 1);
-        w |= __shfl_xor_sync(FULL, w, 2);
-        w |= __shfl_xor_sync(FULL, w, 4);
-        if ((lane & 7) == 0) P.out_bits[(size_t)tile * 16 + s2 * 4 + (lane >> 3)] = w;
-      }
+      reinterpret_cast<uint16_t*>(P.out_bits)[(size_t)tile * 32 + lane] = (uint16_t)flags;
       continue;
     }
     // ---- compaction: warp scan of the lanes' hit counts, one smem claim --------
@@ -508,9 +496,9 @@ void ws_attr_kind() {
     ws_attr<K, 1, true, false, false>();
     ws_attr<K, 1, true, true, false>();
   }
-  if constexpr (K != WK_EQ) {  // bitmap inputs carry no vectors
+  if constexpr (kProbe) {  // bitmap-masked dense probes (no carried vectors)
     ws_attr<K, 2, false, false, false>();
-    if constexpr (kProbe) ws_attr<K, 2, true, false, false>();
+    ws_attr<K, 2, true, false, false>();
   }
 }
 
@@ -527,19 +515,15 @@ void launch_k(int in, bool pay, bool carry, bool obits, int grid, size_t smem, c
       return;
     }
   }
-  const dim3 blk(ws_nw(true) * 32);
-  if constexpr (K != WK_EQ) {
+  if constexpr (kProbe) {
     if (in == 2) {
-      if constexpr (kProbe) {
-        if (pay) {
-          ws_kernel<K, 2, true, false, false><<<grid, blk, smem, st>>>(p);
-          return;
-        }
-      }
-      ws_kernel<K, 2, false, false, false><<<grid, blk, smem, st>>>(p);
+      const dim3 blk2(ws_nw(false) * 32);
+      if (pay) ws_kernel<K, 2, true, false, false><<<grid, blk2, smem, st>>>(p);
+      else ws_kernel<K, 2, false, false, false><<<grid, blk2, smem, st>>>(p);
       return;
     }
   }
+  const dim3 blk(ws_nw(true) * 32);
   if constexpr (kProbe) {
     if (pay) {
       if (carry) ws_kernel<K, 1, true, true, false><<<grid, blk, smem, st>>>(p);
@@ -557,9 +541,9 @@ bool ws_supported(const FilterArgs& a) {
   const bool tids = a.in_tids != nullptr;
   if (a.n_carry > 4 || a.n_cap > (int64_t)0x7FFFFFFF) return false;
   if (a.out_bits && (a.in_tids || a.in_bits || !a.probe || a.out_payload)) return false;
-  if (a.in_bits) {  // row bitmap input: probes at a key column and selections, no vectors
-    if (a.fk_by_pos || a.eq_a || a.n_carry || ((uintptr_t)a.in_bits & 15) != 0) return false;
-    if (!a.probe && (a.n_preds < 1 || a.n_preds > 4)) return false;
+  if (a.in_bits) {  // row bitmap input: probes of a key column (streamed), no vectors
+    if (!a.probe || a.fk_by_pos || a.eq_a || a.n_carry || ((uintptr_t)a.in_bits & 15) != 0) return false;
+    if (((uintptr_t)a.fk & 15) != 0) return false;
   } else if (!tids) {  // dense: probes only (dense selections stream several columns: scan.cu)
     if (!a.probe || a.fk_by_pos || a.eq_a || a.n_carry) return false;
     if (((uintptr_t)a.fk & 15) != 0) return false;
@@ -597,7 +581,6 @@ cudaError_t launch_ws(const FilterArgs& a, cudaStream_t st) {
     ws_attr_kind<WK_EQ>();
   }
   const int in = a.in_bits ? 2 : (a.in_tids ? 1 : 0);
-  const bool tids = in != 0;
   WsParams p{};
   p.n = (uint32_t)a.n_cap;
   p.d_in_count = a.d_in_count;
@@ -675,7 +658,7 @@ cudaError_t launch_ws(const FilterArgs& a, cudaStream_t st) {
   const size_t smem = ring + ((kind == WK_BM_SMEM || kind == WK_HT_SMEM) ? tab : 0);
   const int64_t ntiles = (a.n_cap + WS_TILE - 1) / WS_TILE;  // TID input: an upper bound
   int64_t grid = num_sms();
-  const int64_t need = (ntiles + ws_nw(tids) - 1) / ws_nw(tids);
+  const int64_t need = (ntiles + ws_nw(in == 1) - 1) / ws_nw(in == 1);
   if (grid > need) grid = need < 1 ? 1 : need;
   switch (kind) {
     case WK_BM_SMEM: launch_k<WK_BM_SMEM>(in, pay, carry, obits, (int)grid, smem, st, p); break;

@@ -1225,8 +1225,11 @@ ddq_status ddq_prepare(ddq_db* db, const ddq_plan* plan, int32_t use_graph, ddq_
         op.kind == DDQ_OP_FILTER_EQ)
       P->forced[(size_t)i] = counts[(size_t)i] + counts[(size_t)i] / 64 + 256;
   }
-  // a dense semi-join probe (no payload) whose consumers are all probes / selections
-  // of its output hands them a row bitmap (N/8 bytes) instead of a TID list
+  // a dense semi-join probe (no payload) keeping >= 1/8 of the rows, whose consumers
+  // are all probes of a key column, hands them a row bitmap (N/8 bytes) instead of a
+  // TID list; they stream their key column masked by it (a gather at that density
+  // touches nearly every sector anyway).  Sparser outputs stay TID lists: a bitmap
+  // consumer pays for every row.
   P->bits_out.assign((size_t)plan->n_ops, 0);
   {
     static const char* env = getenv("DDQ_ROW_BITMAPS");  // "0": TID lists only
@@ -1240,9 +1243,11 @@ ddq_status ddq_prepare(ddq_db* db, const ddq_plan* plan, int32_t use_graph, ddq_
         const ddq_op& c = plan->ops[j];
         if (c.input != i) continue;
         consumers++;
-        ok = ok && ((c.kind == DDQ_OP_HASH_PROBE && c.fk_vec <= 0) || c.kind == DDQ_OP_SELECT);
+        ok = ok && c.kind == DDQ_OP_HASH_PROBE && c.fk_vec <= 0;
       }
-      P->bits_out[(size_t)i] = (ok && consumers > 0) ? 1 : 0;
+      const int64_t rows = db->tables[(size_t)op.table].n_rows;
+      const bool dense_enough = counts[(size_t)i] >= 0 && counts[(size_t)i] * 8 >= rows;
+      P->bits_out[(size_t)i] = (ok && consumers > 0 && dense_enough) ? 1 : 0;
     }
   }
   P->inters.resize((size_t)plan->n_ops);
