@@ -46,9 +46,10 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--profile-only", action="store_true", help="short run for ncu")
-    ap.add_argument("--streams", type=int, default=1,
-                    help="concurrent query streams inside a step (the 13 plans round-robin over K streams, "
-                         "the paper's parallel users P:358); 1 = back to back on one stream")
+    ap.add_argument("--streams", type=int, default=4,
+                    help="concurrent query streams inside a step: the 13 plans round-robin over K CUDA streams "
+                         "(the paper's bounded GPU worker pool P:246-260, default 4 = reading O17); 1 = back to "
+                         "back on one stream.  The serial (1-stream) step time is always measured too.")
     return ap.parse_args()
 
 
@@ -231,8 +232,8 @@ def main():
 
     side = [torch.cuda.Stream() for _ in range(max(args.streams, 1) - 1)]
 
-    def step():
-        if not side:
+    def step(serial: bool = False):
+        if serial or not side:
             for p in preps:
                 p.launch(sptr)
             return
@@ -322,6 +323,23 @@ def main():
     ms_per_step = ms / args.steps
     total_rows = 13 * n_lo  # all ranks together
     value = total_rows * args.steps / (ms / 1e3)
+    # the same K steps with the 13 plans back to back on one stream (per-query latency view)
+    serial_ms = None
+    if side:
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        torch.cuda.synchronize()
+        e0.record(stream)
+        for _ in range(args.steps):
+            step(serial=True)
+            exchange()
+        e1.record(stream)
+        torch.cuda.synchronize()
+        serial_ms = e0.elapsed_time(e1)
+        if ws > 1:
+            import torch.distributed as dist
+            t = torch.tensor([serial_ms], device="cuda")
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            serial_ms = float(t.item())
 
     # results of the timed plans (validated against the oracle by tests/, here sanity only)
     results = {q: p.fetch(sptr).rows for q, p in zip(SSB_QUERIES, preps)} if ws == 1 else \
@@ -406,6 +424,8 @@ def main():
                            "lineorder_rows": n_lo, "rows_per_gpu": shard_rows, "queries": 13,
                            "parallelism": f"row-sharded x{ws}" if ws > 1 else "1 GPU",
                            "query_streams": max(args.streams, 1),
+                           "serial_ms_per_step": round(serial_ms / args.steps, 4) if serial_ms else None,
+                           "serial_value": total_rows * args.steps / (serial_ms / 1e3) if serial_ms else None,
                            "l2": "inputs (6.7 GB/GPU) larger than L2; no flush"},
                 "queries_per_s": 13 * args.steps / (ms / 1e3),
                 "gpu_launches": kernels_per_step * args.steps,

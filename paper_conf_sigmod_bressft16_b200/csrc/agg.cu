@@ -13,11 +13,13 @@
 //     touches the shared-memory table only when its key changes -- a single-group
 //     query (Q1.x, Q6) never does until the end, a 150-group one does per row but
 //     with conflict-free random slots (no warp match / shuffle reduction);
-//   * the shared-memory table accumulates every aggregate as TWO int64 words,
-//     L += S mod 2^32 and H += S >> 32 (arithmetic), with non-returning atomics:
-//     exact for any CTA (L < 2^32 * 2^32 adds, |H| < 2^62 for |sum| < 2^94) and
-//     no carry round trip; the CTA's (H, L) become one int128 = H * 2^32 + L that
-//     is merged into the global table (two 64-bit atomics with carry) once per CTA.
+//   * the shared-memory table accumulates every aggregate as a 128-bit two's
+//     complement number in FOUR 32-bit limbs updated with native 32-bit shared
+//     atomics (sm_100a has no 64-bit shared atomicAdd: it compiles to a CAS spin
+//     loop, which ncu showed at 45 % of the kernel's instructions); a limb is only
+//     touched when its addend or the carry into it is non-zero, so a small
+//     positive partial sum costs one returning atomic; the table is merged into
+//     the global int128 table (two 64-bit atomics with carry) once per CTA.
 // Sums are exact int128 whatever the order (integer addition is associative).
 #include <climits>
 #include <cstdint>
@@ -139,10 +141,10 @@ template <int NA>
 __global__ void __launch_bounds__(AG_NW * 32, 1) agg_ws_kernel(const __grid_constant__ AggParams P) {
   extern __shared__ __align__(16) unsigned long long ag_smem[];
   long long* s_keys = reinterpret_cast<long long*>(ag_smem);
-  unsigned long long* s_acc = ag_smem + P.s_slots;  // [(a * S + slot) * 2 + {0: L, 1: H}]
+  uint32_t* s_acc = reinterpret_cast<uint32_t*>(ag_smem + P.s_slots);  // [(a * S + slot) * 4 + limb]
   const uint32_t S = P.s_slots, smask = S - 1;
   for (uint32_t i = threadIdx.x; i < S; i += blockDim.x) s_keys[i] = GB_EMPTY;
-  for (uint32_t i = threadIdx.x; i < S * 2 * NA; i += blockDim.x) s_acc[i] = 0;
+  for (uint32_t i = threadIdx.x; i < S * 4 * NA; i += blockDim.x) s_acc[i] = 0;
   __syncthreads();
 
   const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
@@ -178,10 +180,24 @@ __global__ void __launch_bounds__(AG_NW * 32, 1) agg_ws_kernel(const __grid_cons
     }
     if (slot >= 0) {
 #pragma unroll
-      for (int a = 0; a < NA; a++) {  // split accumulation, fire-and-forget atomics
-        atomicAdd(&s_acc[((size_t)a * S + slot) * 2], lo[a] & 0xFFFFFFFFull);
-        atomicAdd(&s_acc[((size_t)a * S + slot) * 2 + 1],
-                  (unsigned long long)(long long)((lo[a] >> 32) | ((unsigned long long)hi[a] << 32)));
+      for (int a = 0; a < NA; a++) {  // 128-bit add in 32-bit limbs, carries rippled
+        uint32_t* w = s_acc + ((size_t)a * S + slot) * 4;
+        const uint32_t limb[4] = {(uint32_t)lo[a], (uint32_t)(lo[a] >> 32), (uint32_t)hi[a],
+                                  (uint32_t)((unsigned long long)hi[a] >> 32)};
+        uint32_t c = 0;
+#pragma unroll
+        for (int k = 0; k < 4; k++) {
+          const uint32_t x = limb[k] + c;
+          const uint32_t cx = (c && x == 0u) ? 1u : 0u;  // limb + carry wrapped
+          if (x == 0u) {
+            c = cx;
+          } else if (k == 3) {
+            atomicAdd(w + 3, x);  // top limb: carry out of 128 bits is discarded
+          } else {
+            const uint32_t old = atomicAdd(w + k, x);
+            c = (old + x < old) ? 1u : 0u;
+          }
+        }
       }
     } else {  // CTA table full: straight into the global table
       slot = find_or_insert(P.g_keys, P.cap_mask, gb_hash(cur, P.shift), cur);
@@ -300,13 +316,9 @@ __global__ void __launch_bounds__(AG_NW * 32, 1) agg_ws_kernel(const __grid_cons
     }
 #pragma unroll
     for (int a = 0; a < NA; a++) {
-      const unsigned long long L = s_acc[((size_t)a * S + s2) * 2];
-      const long long H = (long long)s_acc[((size_t)a * S + s2) * 2 + 1];
-      // (H << 32) + L as int128 (lo, hi)
-      const unsigned long long hl = (unsigned long long)H << 32;
-      const long long hh = H >> 32;
-      const unsigned long long lo2 = hl + L;
-      const long long hi2 = hh + (lo2 < hl ? 1 : 0);
+      const uint32_t* w = s_acc + ((size_t)a * S + s2) * 4;
+      const unsigned long long lo2 = (unsigned long long)w[0] | ((unsigned long long)w[1] << 32);
+      const long long hi2 = (long long)((unsigned long long)w[2] | ((unsigned long long)w[3] << 32));
       add_i128(&P.g_accs[((size_t)a * (P.cap_mask + 1) + g) * 2], &P.g_accs[((size_t)a * (P.cap_mask + 1) + g) * 2 + 1],
                lo2, hi2);
     }

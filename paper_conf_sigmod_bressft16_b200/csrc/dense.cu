@@ -44,7 +44,7 @@ namespace {
 
 constexpr int WS_ITEMS = 16;            // items per lane per tile
 constexpr int WS_TILE = 32 * WS_ITEMS;  // items per warp tile
-constexpr int WS_R = 4;                 // ring blocks
+constexpr int WS_RMAX = 16;             // ring blocks (runtime R = 4..16, as shared memory allows)
 // entries per ring block (one global reservation): 2048, or 1024 when carried
 // vectors add up to 4 more int32 fields per entry (ring <= 96 KB)
 __host__ __device__ constexpr int ws_blk(bool carry) { return carry ? 1024 : 2048; }
@@ -96,6 +96,7 @@ struct WsParams {
   uint32_t cap_mask;
   int32_t shift;
   int32_t tab_off;  // byte offset of the staged table in dynamic smem
+  int32_t ring_logr;  // log2 of the number of ring blocks
   int32_t n_carry;
   const int32_t* carry_in[4];
   int32_t* carry_out[4];
@@ -183,8 +184,9 @@ __global__ void __launch_bounds__(ws_nw(kIn == 1) * 32, 1) ws_kernel(const __gri
   constexpr bool kTids = kIn == 1;  // sv[] holds TIDs (gathers at them)
   extern __shared__ __align__(16) uint8_t smem[];
   __shared__ uint32_t s_cnt, s_base;
-  __shared__ uint32_t s_filled[WS_R], s_gen[WS_R];
-  constexpr uint32_t BLK = ws_blk(kCarry), RING = BLK * WS_R;
+  __shared__ uint32_t s_filled[WS_RMAX], s_gen[WS_RMAX];
+  constexpr uint32_t BLK = ws_blk(kCarry);
+  const uint32_t RL = P.ring_logr, RM = (1u << RL) - 1u, RING = BLK << RL;  // R = RM + 1 blocks
   int32_t* ring = reinterpret_cast<int32_t*>(smem);  // fields [tid | payload | carried...] x RING
   constexpr bool kProbe = kKind <= WK_HT_GLOBAL;
   constexpr bool kHash = kKind == WK_HT_SMEM || kKind == WK_HT_GLOBAL;
@@ -194,7 +196,7 @@ __global__ void __launch_bounds__(ws_nw(kIn == 1) * 32, 1) ws_kernel(const __gri
   if (threadIdx.x == 0) {
     s_cnt = 0;
 #pragma unroll
-    for (int r = 0; r < WS_R; r++) s_filled[r] = 0, s_gen[r] = 0;
+    for (int r = 0; r < WS_RMAX; r++) s_filled[r] = 0, s_gen[r] = 0;
   }
   __shared__ __align__(8) uint64_t s_bar;
   if (kKind == WK_BM_SMEM) {  // + one zero word past the end: the range test is a clamp
@@ -348,9 +350,9 @@ __global__ void __launch_bounds__(ws_nw(kIn == 1) * 32, 1) ws_kernel(const __gri
       // wait until the ring blocks this range touches are free (their previous
       // occupants flushed): block b lives in slot b % R, generation b / R
       const uint32_t b0 = pos0 / BLK, b1 = (pos0 + tot - 1) / BLK;
-      while (ld_volatile_smem(&s_gen[b0 % WS_R]) != b0 / WS_R) __nanosleep(64);
+      while (ld_volatile_smem(&s_gen[b0 & RM]) != b0 >> RL) __nanosleep(64);
       if (b1 != b0)
-        while (ld_volatile_smem(&s_gen[b1 % WS_R]) != b1 / WS_R) __nanosleep(64);
+        while (ld_volatile_smem(&s_gen[b1 & RM]) != b1 >> RL) __nanosleep(64);
     }
     pos0 = __shfl_sync(FULL, pos0, 0);
     __syncwarp();
@@ -422,10 +424,10 @@ __global__ void __launch_bounds__(ws_nw(kIn == 1) * 32, 1) ws_kernel(const __gri
       const uint32_t end = pos0 + tot;
       const uint32_t b0 = pos0 / BLK, b1 = (end - 1) / BLK;
       const uint32_t c0 = (b1 == b0 ? end : (b0 + 1) * BLK) - pos0;
-      if (atomicAdd(&s_filled[b0 % WS_R], c0) + c0 == BLK) flush |= 1u;
+      if (atomicAdd(&s_filled[b0 & RM], c0) + c0 == BLK) flush |= 1u;
       if (b1 != b0) {
         const uint32_t c1 = end - b1 * BLK;
-        if (atomicAdd(&s_filled[b1 % WS_R], c1) + c1 == BLK) flush |= 2u;
+        if (atomicAdd(&s_filled[b1 & RM], c1) + c1 == BLK) flush |= 2u;
       }
       __threadfence_block();
     }
@@ -433,7 +435,7 @@ __global__ void __launch_bounds__(ws_nw(kIn == 1) * 32, 1) ws_kernel(const __gri
     while (flush) {
       const uint32_t b = (flush & 1u) ? pos0 / BLK : (pos0 + tot - 1) / BLK;
       flush &= flush - 1;
-      const uint32_t slot = b % WS_R;
+      const uint32_t slot = b & RM;
       uint32_t g = 0;
       if (lane == 0) g = atomicAdd(P.d_out_count, BLK);
       g = __shfl_sync(FULL, g, 0);
@@ -461,7 +463,7 @@ __global__ void __launch_bounds__(ws_nw(kIn == 1) * 32, 1) ws_kernel(const __gri
   if (rem) {
     if (threadIdx.x == 0) s_base = atomicAdd(P.d_out_count, rem);
     __syncthreads();
-    copy_out(P, ring, RING, ((total / BLK) % WS_R) * BLK, rem, s_base, threadIdx.x, blockDim.x);
+    copy_out(P, ring, RING, ((total / BLK) & RM) * BLK, rem, s_base, threadIdx.x, blockDim.x);
   }
   // the last CTA to finish clamps the count to the output capacity
   __syncthreads();
@@ -591,7 +593,7 @@ cudaError_t launch_ws(const FilterArgs& a, cudaStream_t st) {
   const bool pay = a.probe && a.out_payload != nullptr;
   const bool carry = in == 1 && a.n_carry > 0;
   const int n_fields = 1 + (pay ? 1 : 0) + (carry ? a.n_carry : 0);
-  const size_t ring = obits ? 0 : (size_t)ws_blk(carry) * WS_R * 4 * n_fields;
+  const size_t ring1 = (size_t)ws_blk(carry) * 4 * n_fields;  // one ring block, all fields
   const size_t budget = (size_t)g_optin - kWsCtl;
   int kind;
   size_t tab = 0;
@@ -605,7 +607,8 @@ cudaError_t launch_ws(const FilterArgs& a, cudaStream_t st) {
       p.range = a.range;
       p.bitmap_words = (a.range + 31) / 32;
       tab = ((size_t)p.bitmap_words * 4 + 15) / 16 * 16 + 16;  // bulk-copy rounding + the zero word
-      kind = (!a.no_smem && ring + tab <= budget && stage_pays(a.n_cap, tab)) ? WK_BM_SMEM : WK_BM_GLOBAL;
+      kind = (!a.no_smem && (obits ? 0 : 4 * ring1) + tab <= budget && stage_pays(a.n_cap, tab)) ? WK_BM_SMEM
+                                                                                                 : WK_BM_GLOBAL;
     } else {
       p.table = a.table;
       p.cap_mask = a.capacity - 1;
@@ -613,7 +616,8 @@ cudaError_t launch_ws(const FilterArgs& a, cudaStream_t st) {
       while ((1u << lg) < a.capacity) lg++;
       p.shift = 32 - lg;
       tab = (size_t)a.capacity * 8;
-      kind = (!a.no_smem && ring + tab <= budget && stage_pays(a.n_cap, tab)) ? WK_HT_SMEM : WK_HT_GLOBAL;
+      kind = (!a.no_smem && (obits ? 0 : 4 * ring1) + tab <= budget && stage_pays(a.n_cap, tab)) ? WK_HT_SMEM
+                                                                                                 : WK_HT_GLOBAL;
     }
   } else if (a.eq_a) {
     kind = WK_EQ;
@@ -638,6 +642,15 @@ cudaError_t launch_ws(const FilterArgs& a, cudaStream_t st) {
     }
     kind = all_range ? WK_SEL_RANGE : WK_SEL_GENERIC;
   }
+  // ring: 4 blocks.  More blocks would put more flushes in flight (ncu: a quarter
+  // of a 100 %-pass late-fetch probe's instructions spin on a free slot), but
+  // shared memory is carved out of the unified L1 where the payload-array lookups
+  // live: 16 blocks made the date probe's d_year lookups miss (74 -> 141 us) and
+  // 8 blocks slowed the late fetch itself (119 -> 195 us)
+  const size_t tab_smem = (kind == WK_BM_SMEM || kind == WK_HT_SMEM) ? tab : 0;
+  const int logr = 2;
+  const size_t ring = obits ? 0 : ring1 << logr;
+  p.ring_logr = logr;
   p.tab_off = (int32_t)ring;
   p.n_carry = carry ? a.n_carry : 0;
   for (int c = 0; c < p.n_carry; c++) {
@@ -655,7 +668,7 @@ cudaError_t launch_ws(const FilterArgs& a, cudaStream_t st) {
   p.d_overflow = a.d_overflow;
   cudaError_t e = init_fill(a.d_out_count, 8, 0, st);
   if (e != cudaSuccess) return e;
-  const size_t smem = ring + ((kind == WK_BM_SMEM || kind == WK_HT_SMEM) ? tab : 0);
+  const size_t smem = ring + tab_smem;
   const int64_t ntiles = (a.n_cap + WS_TILE - 1) / WS_TILE;  // TID input: an upper bound
   int64_t grid = num_sms();
   const int64_t need = (ntiles + ws_nw(in == 1) - 1) / ws_nw(in == 1);
