@@ -349,6 +349,12 @@ typedef struct {
   int32_t term_build[4];
   ddq_column term_fk[4];
   int32_t term_emit[4];
+  /* GATHER through a join (dimension attribute fetch): 1 + index of a HASH_BUILD op;
+     0 = plain column gather.  The new vector is then payload(build, gather_col[r])
+     for every input row r (gather_col = the fact FK column), INT32_MIN where r's key
+     has no match -- a fetch after a semi-join probe of the same build (late
+     materialisation) never has one.  int32 output. */
+  int32_t fetch_build;
 } ddq_op;
 
 #define DDQ_MAX_OPS 32

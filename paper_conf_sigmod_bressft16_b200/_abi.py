@@ -64,7 +64,8 @@ class Op(ctypes.Structure):
                 ("key_bits", ctypes.c_int32 * MAX_KEYS), ("fk_vec", ctypes.c_int32),
                 ("eq_vec", ctypes.c_int32 * 2), ("n_terms", ctypes.c_int32),
                 ("term_kind", ctypes.c_int32 * 4), ("term_build", ctypes.c_int32 * 4),
-                ("term_fk", ctypes.c_int32 * 4), ("term_emit", ctypes.c_int32 * 4)]
+                ("term_fk", ctypes.c_int32 * 4), ("term_emit", ctypes.c_int32 * 4),
+                ("fetch_build", ctypes.c_int32)]
 
 
 class DevTerm(ctypes.Structure):

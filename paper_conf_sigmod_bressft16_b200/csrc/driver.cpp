@@ -91,6 +91,8 @@ static std::vector<int> op_children(const ddq_op& op) {
   std::vector<int> ch;
   if (op.input >= 0) ch.push_back(op.input);
   if (op.kind == DDQ_OP_HASH_PROBE && op.build >= 0 && op.build != op.input) ch.push_back(op.build);
+  if (op.kind == DDQ_OP_GATHER && op.fetch_build > 0 && op.fetch_build - 1 != op.input)
+    ch.push_back(op.fetch_build - 1);
   if (op.kind == DDQ_OP_STAR)
     for (int j = 0; j < op.n_terms && j < 4; j++)
       if (op.term_kind[j] == DDQ_TERM_PROBE && std::find(ch.begin(), ch.end(), op.term_build[j]) == ch.end())
@@ -508,6 +510,35 @@ ddq_status run_host_op(ddq_db* db, const ddq_op& op, const std::vector<Inter>& I
         void* p = host_alloc(out, (size_t)n * v.width);
         std::memcpy(p, v.ptr, (size_t)n * v.width);
         out.vecs.push_back(Vec{p, v.width, true});
+      }
+      if (op.fetch_build > 0) {  // dimension attribute fetch (INT32_MIN for a missing key)
+        const Inter* B = &I[(size_t)op.fetch_build - 1];
+        if (!B->host_table && !B->h_bitmap) return set_error(DDQ_ESTATE, "host fetch needs a host table");
+        int32_t* dst = (int32_t*)host_alloc(out, (size_t)n * 4);
+        int lg = 0;
+        while (B->host_table && (1u << lg) < B->table_cap) lg++;
+        for (int64_t i = 0; i < n; i++) {
+          const int32_t k = ((const int32_t*)c->host)[in->tids[i]];
+          int32_t v = INT32_MIN;
+          if (B->h_bitmap) {
+            const uint32_t o = (uint32_t)(k - B->jmin);
+            if (o < B->jrange && (((*B->h_bitmap)[o >> 5] >> (o & 31)) & 1u)) v = (*B->h_payarr)[o];
+          } else {
+            uint32_t h = host_hash32(k, 32 - lg);
+            while (true) {
+              const uint64_t sl = (*B->host_table)[h];
+              if (sl == kHostEmpty) break;
+              if ((int32_t)(sl >> 32) == k) {
+                v = (int32_t)(uint32_t)sl;
+                break;
+              }
+              h = (h + 1) & (B->table_cap - 1);
+            }
+          }
+          dst[i] = v;
+        }
+        out.vecs.push_back(Vec{dst, 4, true});
+        return DDQ_OK;
       }
       void* dst = host_alloc(out, (size_t)n * c->width);
       for (int64_t i = 0; i < n; i++) {

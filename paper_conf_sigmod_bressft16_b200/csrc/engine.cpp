@@ -424,6 +424,21 @@ ddq_status run_gpu_op(GpuOpCtx& ctx, const ddq_op& op, Inter& out) {
       out.cap = in->cap;
       out.vecs = in->vecs;
       out.d_error = in->d_error;
+      if (op.fetch_build > 0) {  // dimension attribute fetch through the build's index
+        const int b = op.fetch_build - 1;
+        if (b >= (int)I.size() || c->width != 4) return set_error(DDQ_EINVAL, "fetch: bad build / fk column");
+        const Inter& B = I[(size_t)b];
+        if (!B.table_ptr && !B.jidx) return set_error(DDQ_ESTATE, "fetch: build side is not on the device");
+        if (!in->d_count) return set_error(DDQ_ESTATE, "fetch: input without a device count");
+        int32_t* dst = (int32_t*)A.get((uint64_t)std::max<int64_t>(in->cap, 1) * 4);
+        if (A.failed) return DDQ_ENOMEM_DEVICE;
+        out.vecs.push_back(Vec{dst, 4, false});
+        return cuda_status(launch_fetch(in->tids, in->d_count, in->cap, (const int32_t*)src,
+                                        B.jidx ? join_index_bitmap(B.jidx) : nullptr,
+                                        B.jidx ? join_index_payload(B.jidx, B.jrange) : nullptr, B.jmin, B.jrange,
+                                        B.table_ptr, B.table_cap, dst, st),
+                           "fetch");
+      }
       void* dst = A.get((uint64_t)std::max<int64_t>(in->cap, 1) * c->width);
       if (A.failed) return DDQ_ENOMEM_DEVICE;
       out.vecs.push_back(Vec{dst, c->width, false});
@@ -989,6 +1004,9 @@ static ddq_status validate_plan(ddq_db* db, const ddq_plan* plan) {
           return set_error(DDQ_EINVAL, "plan: STAR probe must reference an earlier HASH_BUILD");
     }
     if (op.kind == DDQ_OP_FILTER_EQ && op.input < 0) return set_error(DDQ_EINVAL, "plan: filter_eq needs an input");
+    if (op.fetch_build != 0 && (op.kind != DDQ_OP_GATHER || op.fetch_build - 1 < 0 || op.fetch_build - 1 >= i ||
+                                plan->ops[op.fetch_build - 1].kind != DDQ_OP_HASH_BUILD))
+      return set_error(DDQ_EINVAL, "plan: a fetch must be a GATHER referencing an earlier HASH_BUILD");
     if (op.kind == DDQ_OP_HASH_PROBE && op.fk_vec > 0 && op.input < 0)
       return set_error(DDQ_EINVAL, "plan: a vector-keyed probe needs an input");
     if (op.kind == DDQ_OP_AGGREGATE) {
@@ -1060,6 +1078,7 @@ static std::vector<int> op_deps(const ddq_op& op, int i) {
   };
   add(op.input);
   if (op.kind == DDQ_OP_HASH_PROBE) add(op.build);
+  if (op.kind == DDQ_OP_GATHER && op.fetch_build > 0) add(op.fetch_build - 1);
   if (op.kind == DDQ_OP_STAR)
     for (int j = 0; j < op.n_terms && j < 4; j++)
       if (op.term_kind[j] == DDQ_TERM_PROBE) add(op.term_build[j]);
@@ -1407,8 +1426,8 @@ int32_t ddq_prepared_profile(ddq_prepared* p, void* stream, int32_t max_ops, flo
         for (int k = 0; k < op.n_preds; k++) bytes += m * width(op.preds[k].column);  // fused selection
         break;
       case DDQ_OP_GATHER:
-        cls = 3;
-        bytes = m * 4 + sector_bytes(N, m, width(op.gather_col)) + m * width(op.gather_col);
+        cls = op.fetch_build > 0 ? 1 : 3;  // a fetch is an at-TIDs lookup like a probe
+        bytes = m * 4 + sector_bytes(N, m, width(op.gather_col)) + m * (op.fetch_build > 0 ? 4 : width(op.gather_col));
         break;
       case DDQ_OP_AGGREGATE: {
         cls = 4;

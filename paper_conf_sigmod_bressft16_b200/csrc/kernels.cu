@@ -8,6 +8,7 @@
 // Accumulators are exact int128 (two 64-bit atomics with carry), so results are
 // bit-identical whatever the scheduling (integer addition is associative).
 #include <algorithm>
+#include <climits>
 #include <cstdint>
 #include <cstdlib>
 #include <cuda_runtime.h>
@@ -200,6 +201,61 @@ __global__ void gather_kernel(const void* __restrict__ col, const int32_t* __res
     else
       reinterpret_cast<int*>(out)[i] = ldg_gather(reinterpret_cast<const int32_t*>(col) + r);
   }
+}
+
+// Dimension attribute fetch (GATHER through a join index / hash table): for every
+// input TID r, out[i] = payload of fk[r] (INT32_MIN if fk[r] has no match).  Pure
+// streaming -- TIDs and out coalesced, fk gathered (64 B chunks), the index L2-
+// resident -- no compaction: a late-materialisation fetch after a semi-join of the
+// same build passes every row, so a probe's ring, reservation and TID copy would be
+// wasted work (opprofile SF20 Q3.1: 119 us as an emitting probe).
+constexpr int FT_PER = 4;  // items per thread (independent gathers in flight)
+__global__ void __launch_bounds__(256) fetch_kernel(const int32_t* __restrict__ tids, const uint32_t* d_count,
+                                                    const int32_t* __restrict__ fk, const uint32_t* __restrict__ bitmap,
+                                                    const int32_t* __restrict__ payarr, int32_t key_min, uint32_t range,
+                                                    const uint64_t* __restrict__ table, uint32_t cap_mask, int shift,
+                                                    int32_t* __restrict__ out) {
+  const uint32_t n = ld_relaxed_u32(d_count);
+  const uint32_t stride = gridDim.x * blockDim.x;
+  for (uint32_t i0 = blockIdx.x * blockDim.x + threadIdx.x; i0 < n; i0 += FT_PER * stride) {
+    int32_t k[FT_PER];
+#pragma unroll
+    for (int u = 0; u < FT_PER; u++) {
+      const uint32_t i = i0 + u * stride;
+      k[u] = i < n ? ldg_gather(fk + (uint32_t)tids[i]) : 0;
+    }
+#pragma unroll
+    for (int u = 0; u < FT_PER; u++) {
+      const uint32_t i = i0 + u * stride;
+      if (i >= n) continue;
+      int32_t v = INT32_MIN;
+      if (bitmap) {
+        const uint32_t o = (uint32_t)(k[u] - key_min);
+        if (o < range && ((__ldg(bitmap + (o >> 5)) >> (o & 31)) & 1u)) v = __ldg(payarr + o);
+      } else {
+        uint32_t h = ht_hash(k[u], shift);
+        uint64_t sl = __ldg(table + h);
+        while (sl != HT_EMPTY && ht_key(sl) != k[u]) {
+          h = (h + 1) & cap_mask;
+          sl = __ldg(table + h);
+        }
+        if (sl != HT_EMPTY) v = ht_val(sl);
+      }
+      out[i] = v;
+    }
+  }
+}
+
+cudaError_t launch_fetch(const int32_t* tids, const uint32_t* d_count, int64_t n_cap, const int32_t* fk,
+                         const uint32_t* bitmap, const int32_t* payarr, int32_t key_min, uint32_t range,
+                         const uint64_t* table, uint32_t capacity, int32_t* out, cudaStream_t st) {
+  int lg = 0;
+  while (capacity && (1u << lg) < capacity) lg++;
+  int64_t g = (n_cap + 256 * FT_PER - 1) / (256 * FT_PER);
+  int grid = (int)(g > num_sms() * 8 ? num_sms() * 8 : (g < 1 ? 1 : g));
+  fetch_kernel<<<grid, 256, 0, st>>>(tids, d_count, fk, bitmap, payarr, key_min, range, table,
+                                     capacity ? capacity - 1 : 0, 32 - lg, out);
+  return cudaGetLastError();
 }
 
 cudaError_t launch_gather(const void* col, int width, const int32_t* tids, const uint32_t* d_count,

@@ -96,6 +96,10 @@ cudaError_t launch_join_index_build(const int32_t* keys, const int32_t* payload,
                                     const uint32_t* d_in_count, int64_t n_cap, int32_t key_min, uint32_t range,
                                     void* index, uint32_t* d_error, cudaStream_t st,
                                     const BuildPreds* preds = nullptr);
+// dimension attribute fetch (GATHER through a join): join index (bitmap != NULL) or hash table
+cudaError_t launch_fetch(const int32_t* tids, const uint32_t* d_count, int64_t n_cap, const int32_t* fk,
+                         const uint32_t* bitmap, const int32_t* payarr, int32_t key_min, uint32_t range,
+                         const uint64_t* table, uint32_t capacity, int32_t* out, cudaStream_t st);
 cudaError_t launch_gather(const void* col, int width, const int32_t* tids, const uint32_t* d_count,
                           int64_t n_cap, void* out, cudaStream_t st);
 

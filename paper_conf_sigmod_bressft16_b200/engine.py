@@ -160,6 +160,15 @@ class PlanBuilder:
         op.gather_col = self.db.col(table, col)
         return idx
 
+    def fetch(self, table: str, fk: str, build: int, input: int) -> int:
+        """Dimension attribute fetch (a GATHER through a join): appends the payload of
+        `build` matched by fk[r] for every input row r as an aligned vector (late
+        materialisation after a semi-join probe of the same build)."""
+        idx, op = self._op(A.OP_GATHER, table, input)
+        op.gather_col = self.db.col(table, fk)
+        op.fetch_build = build + 1
+        return idx
+
     def aggregate(self, table: str, input: int, keys: list, aggs: list, order_by: list | None = None,
                   max_groups: int = 0, limit: int = 0, key_bits: list | None = None,
                   where: list | None = None) -> int:

@@ -142,3 +142,43 @@ def test_placement_invariance(arm):
         assert st["host_ops"] == 0 or st["aborts"] > 0
         assert st["h2d_bytes"] > 0
     db.close()
+
+
+@pytest.mark.parametrize("path", ["prepared", "submit"])
+def test_fetch_through_join_with_misses(path):
+    """GATHER through a join (dimension attribute fetch, include/ddq.h fetch_build):
+    rows whose key has no match get INT32_MIN.  Fetch c_nation through an
+    ASIA-only customer index at EVERY lineorder row of SF 0.01, then count rows per
+    fetched value; expected counts from numpy on the same columns (the ASIA
+    customers' nations, and the rest under the miss value)."""
+    import numpy as np
+    from paper_conf_sigmod_bressft16_b200 import _abi as A
+    from paper_conf_sigmod_bressft16_b200.ssb import code
+    data = _data("0.01")
+    db = _db("0.01")
+    asia = code(db, "region", "ASIA")
+    P = db.plan()
+    hc = P.build("customer", "c_custkey", "c_nation", where=[("c_region", [asia])])
+    t = P.select("lineorder", [("lo_quantity", 1, 50)])  # every row
+    t = P.fetch("lineorder", "lo_custkey", hc, input=t)
+    P.aggregate("lineorder", t, keys=[0], aggs=[(A.AGG_COUNT, [])], key_bits=[32], max_groups=64)
+    if path == "prepared":
+        p = db.prepare(P, use_graph=True)
+        p.launch()
+        rows = p.fetch().rows
+        p.close()
+    else:
+        rows = db.run(P).rows
+    ck, reg, nat = data["c_custkey"], data["c_region"], data["c_nation"]
+    nation_of = dict(zip(ck.tolist(), nat.tolist()))
+    in_asia = dict(zip(ck.tolist(), (reg == asia).tolist()))
+    want = {}
+    for k in data["lo_custkey"].tolist():
+        v = nation_of[k] if in_asia[k] else -2**31
+        want[v] = want.get(v, 0) + 1
+    got = {}
+    for r in rows:
+        key = int(r[0])
+        key = key - 2**32 if key >= 2**31 else key  # the miss value as an int32
+        got[key] = got.get(key, 0) + int(r[1])
+    assert got == want

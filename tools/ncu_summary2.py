@@ -30,7 +30,7 @@ def main(path):
                 try:
                     unit = rows[1][idx[k]]
                     v = float(r[idx[k]].replace(",", ""))
-                    scale = {"nsecond": 1e-3, "usecond": 1.0, "msecond": 1e3, "byte": 1e-6, "Kbyte": 1e-3,
+                    scale = {"nsecond": 1e-3, "ns": 1e-3, "usecond": 1.0, "us": 1.0, "msecond": 1e3, "ms": 1e3, "byte": 1e-6, "Kbyte": 1e-3,
                              "Mbyte": 1.0, "Gbyte": 1e3}.get(unit)
                     if lab in ("us", "MB_rd", "MB_wr") and scale is not None:
                         v = v * scale

@@ -41,8 +41,8 @@ def main(path: str, out: str | None):
         k = (d["ID"], d["Kernel Name"])
         v = float(d["Metric Value"].replace(",", ""))
         unit = d.get("Metric Unit", "")
-        scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "nsecond": 1e-3, "usecond": 1.0,
-                 "msecond": 1e3}.get(unit, 1.0)
+        scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "nsecond": 1e-3, "ns": 1e-3,
+                 "usecond": 1.0, "us": 1.0, "msecond": 1e3, "ms": 1e3}.get(unit, 1.0)
         per.setdefault(k, {})[d["Metric Name"]] = v * scale
     cls = {}
     for (i, name), m in per.items():
