@@ -27,7 +27,7 @@
 
 namespace ddq {
 
-ddq_status cache_column_locked(ddq_db* db, int c, bool on_demand);
+ddq_status cache_column_locked(ddq_db* db, int c, bool on_demand, std::unique_lock<std::mutex>& lk);
 void evict_column_locked(ddq_db* db, int c);
 ddq_status validate_plan_public(ddq_db* db, const ddq_plan* plan);
 
@@ -642,9 +642,10 @@ static bool children_on_gpu(QueryState& q, int i) {
 // Operator-driven data placement for the GPU-only arm: make the
 // op's columns resident, evicting least-recently-used unreferenced columns.
 static ddq_status ensure_cached_lru(ddq_db* db, const ddq_op& op) {
-  std::lock_guard<std::mutex> g(db->mu);
+  std::unique_lock<std::mutex> g(db->mu);
   for (int c : op_columns(op)) {
     Column& col = *db->cols[(size_t)c];
+    while (col.loading) db->cache_cv.wait(g);  // another worker is copying it
     if (col.dev && !col.evict_pending) {
       db->stats.cache_hits++;
       continue;
@@ -666,7 +667,7 @@ static ddq_status ensure_cached_lru(ddq_db* db, const ddq_op& op) {
       if (victim < 0) return DDQ_ENOMEM_DEVICE;
       evict_column_locked(db, victim);
     }
-    ddq_status s = cache_column_locked(db, c, true);
+    ddq_status s = cache_column_locked(db, c, true, g);
     if (s != DDQ_OK) return s;
   }
   return DDQ_OK;
@@ -679,6 +680,19 @@ static void hold_columns(ddq_db* db, const ddq_op& op, int delta) {
     col.refs += delta;
     if (delta < 0 && col.refs == 0 && col.evict_pending) evict_column_locked(db, c);
   }
+}
+
+// Pin the op's columns iff all are resident (check and pin under one lock, so an
+// eviction cannot slip between them).
+static bool hold_if_cached(ddq_db* db, const ddq_op& op) {
+  std::lock_guard<std::mutex> g(db->mu);
+  const std::vector<int> cols = op_columns(op);
+  for (int c : cols) {
+    const Column* col = col_of(db, c);
+    if (!col || !col->dev || col->evict_pending) return false;
+  }
+  for (int c : cols) db->cols[(size_t)c]->refs++;
+  return true;
 }
 
 static void enqueue(ddq_db* db, std::shared_ptr<QueryState> q, int i);
@@ -838,10 +852,9 @@ static void run_on_gpu(ddq_db* db, std::shared_ptr<QueryState> q, int i, cudaStr
       }
     }
   }
-  if (!abort && !columns_cached(db, op)) abort = true;  // evicted meanwhile: follow the data
+  if (!abort && !hold_if_cached(db, op)) abort = true;  // evicted meanwhile: follow the data
   Inter out;
   if (!abort) {
-    hold_columns(db, op, +1);
     GpuOpCtx ctx{db, st, &q->inters};
     s = run_gpu_op(ctx, op, out);
     if (s == DDQ_OK) {

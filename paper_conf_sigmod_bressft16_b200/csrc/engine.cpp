@@ -720,6 +720,20 @@ ddq_status ddq_open(const ddq_config* cfg, ddq_db** out) {
     delete db;
     return cuda_status(e, "ddq_open stream");
   }
+  {
+    cudaMemPoolProps pp{};
+    pp.allocType = cudaMemAllocationTypePinned;
+    pp.location.type = cudaMemLocationTypeDevice;
+    pp.location.id = db->device;
+    e = cudaMemPoolCreate(&db->cache_pool, &pp);
+    if (e != cudaSuccess) {
+      cudaStreamDestroy(db->copy_stream);
+      delete db;
+      return cuda_status(e, "ddq_open cache pool");
+    }
+    uint64_t thr = UINT64_MAX;
+    cudaMemPoolSetAttribute(db->cache_pool, cudaMemPoolAttrReleaseThreshold, &thr);
+  }
   ddq_status s = db->heap.init(cfg->heap_bytes, cfg->fault_alloc_every);
   if (s != DDQ_OK) {
     delete db;
@@ -736,9 +750,11 @@ void ddq_close(ddq_db* db) {
   cudaSetDevice(db->device);
   cudaDeviceSynchronize();
   for (auto& c : db->cols) {
-    if (c->dev) cudaFree(c->dev);
+    if (c->dev) cudaFreeAsync(c->dev, db->copy_stream);
     if (c->host) cudaFreeHost(c->host);
   }
+  cudaStreamSynchronize(db->copy_stream);
+  if (db->cache_pool) cudaMemPoolDestroy(db->cache_pool);
   if (db->copy_stream) cudaStreamDestroy(db->copy_stream);
   delete db;
 }
@@ -803,9 +819,13 @@ ddq_status ddq_find_column(ddq_db* db, const char* table, const char* name, ddq_
 }  // extern "C"
 
 namespace ddq {
-// H2D copy of one column into the cache (caller holds db->mu).
-ddq_status cache_column_locked(ddq_db* db, int c, bool on_demand) {
+// H2D copy of one column into the cache.  The caller holds db->mu through `lk`;
+// it is released for the copy itself, so operators of other queries keep
+// launching while PCIe is busy (a concurrent request for the same column waits
+// on cache_cv).  The bytes are reserved against the budget before unlocking.
+ddq_status cache_column_locked(ddq_db* db, int c, bool on_demand, std::unique_lock<std::mutex>& lk) {
   Column& col = *db->cols[(size_t)c];
+  while (col.loading) db->cache_cv.wait(lk);
   if (col.dev) {
     col.evict_pending = false;
     return DDQ_OK;
@@ -815,25 +835,43 @@ ddq_status cache_column_locked(ddq_db* db, int c, bool on_demand) {
     return set_error(DDQ_ENOMEM_DEVICE, "cache budget exceeded for " + col.name);
   cudaSetDevice(db->device);
   void* p = nullptr;
-  cudaError_t e = cudaMalloc(&p, (bytes + 255) / 256 * 256);  // padded: TMA reads whole 16-byte chunks
-  if (e != cudaSuccess) return cuda_status(e, "cache cudaMalloc");
+  // padded: TMA reads whole 16-byte chunks
+  cudaError_t e = cudaMallocFromPoolAsync(&p, (bytes + 255) / 256 * 256, db->cache_pool, db->copy_stream);
+  if (e != cudaSuccess) return cuda_status(e, "cache pool alloc");
+  cudaEvent_t done = nullptr;
+  e = cudaEventCreateWithFlags(&done, cudaEventDisableTiming);
+  if (e != cudaSuccess) {
+    cudaFreeAsync(p, db->copy_stream);
+    return cuda_status(e, "cache event");
+  }
+  db->cache_used += bytes;
+  col.loading = true;
+  lk.unlock();
   uint64_t t0 = now_ns();
   e = cudaMemcpyAsync(p, col.host, (size_t)col.n * col.width, cudaMemcpyHostToDevice, db->copy_stream);
-  if (e == cudaSuccess) e = cudaStreamSynchronize(db->copy_stream);
+  if (e == cudaSuccess) e = cudaEventRecord(done, db->copy_stream);
+  if (e == cudaSuccess) e = cudaEventSynchronize(done);
+  const uint64_t dt = now_ns() - t0;
+  cudaEventDestroy(done);
+  lk.lock();
+  col.loading = false;
+  db->cache_cv.notify_all();
   if (e != cudaSuccess) {
-    cudaFree(p);
+    cudaFreeAsync(p, db->copy_stream);
+    db->cache_used -= bytes;
     return cuda_status(e, "cache H2D");
   }
-  db->stats.h2d_ns += now_ns() - t0;
+  db->stats.h2d_ns += dt;
   db->stats.h2d_bytes += (uint64_t)col.n * col.width;
   col.dev = p;
   col.on_demand = on_demand;
   col.evict_pending = false;
-  db->cache_used += bytes;
   return DDQ_OK;
 }
 
-// Evict (deferred while running operators hold references).
+// Evict (deferred while running operators hold references).  Prepared
+// plans launched asynchronously may still read the column: wait for the device
+// (cudaFree's implicit synchronisation), then return the block to the pool.
 void evict_column_locked(ddq_db* db, int c) {
   Column& col = *db->cols[(size_t)c];
   if (!col.dev) return;
@@ -841,7 +879,9 @@ void evict_column_locked(ddq_db* db, int c) {
     col.evict_pending = true;
     return;
   }
-  cudaFree(col.dev);
+  cudaSetDevice(db->device);
+  cudaDeviceSynchronize();
+  cudaFreeAsync(col.dev, db->copy_stream);
   col.dev = nullptr;
   col.evict_pending = false;
   db->cache_used -= (uint64_t)std::max<int64_t>(col.n, 1) * col.width;
@@ -852,8 +892,8 @@ extern "C" {
 
 ddq_status ddq_cache_column(ddq_db* db, ddq_column c) {
   if (!db || c < 0 || c >= (int)db->cols.size()) return set_error(DDQ_ENOTFOUND, "cache_column");
-  std::lock_guard<std::mutex> g(db->mu);
-  return cache_column_locked(db, c, false);
+  std::unique_lock<std::mutex> g(db->mu);
+  return cache_column_locked(db, c, false, g);
 }
 
 ddq_status ddq_evict_column(ddq_db* db, ddq_column c) {
@@ -891,7 +931,7 @@ ddq_status ddq_reset_access_counts(ddq_db* db) {
 // of K, ties by column id, and the loop stops at the first column that does not fit.
 ddq_status ddq_update_placement(ddq_db* db) {
   if (!db) return set_error(DDQ_EINVAL, "update_placement");
-  std::lock_guard<std::mutex> g(db->mu);
+  std::unique_lock<std::mutex> lk(db->mu);
   std::vector<int> K(db->cols.size());
   std::iota(K.begin(), K.end(), 0);
   std::stable_sort(K.begin(), K.end(), [&](int a, int b) {
@@ -912,7 +952,7 @@ ddq_status ddq_update_placement(ddq_db* db) {
     if (!keep[c] && db->cols[c]->dev) evict_column_locked(db, (int)c);
   for (size_t c = 0; c < db->cols.size(); c++)  // cache(C_new \ C_old)
     if (keep[c] && !db->cols[c]->dev) {
-      ddq_status s = cache_column_locked(db, (int)c, false);
+      ddq_status s = cache_column_locked(db, (int)c, false, lk);
       if (s != DDQ_OK && s != DDQ_ENOMEM_DEVICE) return s;  // deferred evictions may still hold memory
     }
   return DDQ_OK;

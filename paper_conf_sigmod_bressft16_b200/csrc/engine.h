@@ -58,6 +58,7 @@ struct Column {
   int refs = 0;             // running operators using `dev`
   bool evict_pending = false;
   bool on_demand = false;   // cached by operator-driven placement (GPU-only arm)
+  bool loading = false;     // H2D copy in flight (db->mu released; waiters use cache_cv)
 };
 
 struct Table {
@@ -124,6 +125,10 @@ struct ddq_db {
   ddq_config cfg{};
   int device = 0;
   cudaStream_t copy_stream = nullptr;
+  // device column cache: a stream-ordered pool that keeps freed blocks (release
+  // threshold = max), so evict + re-cache reuses device memory without a
+  // cudaMalloc/cudaFree round trip through the driver per column
+  cudaMemPool_t cache_pool = nullptr;
   ddq::Heap heap;
   std::mutex mu;  // catalog + cache
   std::condition_variable cache_cv;
