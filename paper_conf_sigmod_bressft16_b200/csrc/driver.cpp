@@ -565,7 +565,7 @@ ddq_status run_host_op(ddq_db* db, const ddq_op& op, const std::vector<Inter>& I
       std::vector<const Column*> apc;  // fused selection (AGGREGATE op with predicates)
       for (int p = 0; p < op.n_preds; p++) apc.push_back(col_of(db, op.preds[p].column));
       for (int64_t i = 0; i < n; i++) {
-        int32_t r = in->tids[i];
+        int32_t r = row_of(i);
         bool ok = true;
         for (int p = 0; p < op.n_preds && ok; p++) {
           const int64_t v = hcol(apc[(size_t)p], r);

@@ -445,7 +445,8 @@ ddq_status run_gpu_op(GpuOpCtx& ctx, const ddq_op& op, Inter& out) {
       return cuda_status(launch_gather(src, c->width, in->tids, in->d_count, in->cap, dst, st), "gather");
     }
     case DDQ_OP_AGGREGATE: {
-      if (!in) return set_error(DDQ_EINVAL, "aggregate needs an input TID list");
+      // no input: every row of op.table (a dense aggregation, e.g. TPC-H Q1 with
+      // its selection fused, O26); keys must then be columns
       if (op.n_keys < 0 || op.n_keys > DDQ_MAX_KEYS || op.n_aggs < 1 || op.n_aggs > DDQ_MAX_AGGS)
         return set_error(DDQ_EINVAL, "aggregate: bad key/agg counts");
       const int32_t* kv[3] = {nullptr, nullptr, nullptr};
@@ -453,7 +454,7 @@ ddq_status run_gpu_op(GpuOpCtx& ctx, const ddq_op& op, Inter& out) {
       for (int k = 0; k < op.n_keys; k++) {
         int src = op.key_src[k];
         if (src >= 0) {
-          if (src >= (int)in->vecs.size() || in->vecs[(size_t)src].width != 4)
+          if (!in || src >= (int)in->vecs.size() || in->vecs[(size_t)src].width != 4)
             return set_error(DDQ_EINVAL, "aggregate: bad key vector");
           kv[k] = (const int32_t*)in->vecs[(size_t)src].ptr;
         } else {
@@ -477,8 +478,9 @@ ddq_status run_gpu_op(GpuOpCtx& ctx, const ddq_op& op, Inter& out) {
           if (!ag[a].arg[j]) return set_error(DDQ_ESTATE, "aggregate: argument column not cached");
         }
       }
-      int64_t groups = op.max_groups > 0 ? std::min<int64_t>(op.max_groups, std::max<int64_t>(in->cap, 1))
-                                         : std::max<int64_t>(in->cap, 1);
+      const int64_t in_cap = in ? in->cap : db->tables[(size_t)op.table].n_rows;
+      int64_t groups = op.max_groups > 0 ? std::min<int64_t>(op.max_groups, std::max<int64_t>(in_cap, 1))
+                                         : std::max<int64_t>(in_cap, 1);
       int64_t cap = pow2_at_least(std::max<int64_t>(64, 2 * groups));
       if (cap > (1ll << 31)) return set_error(DDQ_EINVAL, "aggregate: table too large");
       out.gb_cap = (uint32_t)cap;
@@ -486,7 +488,7 @@ ddq_status run_gpu_op(GpuOpCtx& ctx, const ddq_op& op, Inter& out) {
       out.gb_keys = (int64_t*)A.get((uint64_t)cap * 8);
       out.gb_accs = (int64_t*)A.get((uint64_t)cap * op.n_aggs * 16);
       out.gb_groups = (uint32_t*)A.get(64);
-      out.d_error = in->d_error;
+      out.d_error = in ? in->d_error : nullptr;
       if (!out.d_error) {
         out.d_error = (uint32_t*)A.get(64);
         if (!A.failed) init_fill(out.d_error, 4, 0, st);
@@ -512,21 +514,42 @@ ddq_status run_gpu_op(GpuOpCtx& ctx, const ddq_op& op, Inter& out) {
         d.n_in = p.n_in;
         for (int j = 0; j < DDQ_MAX_IN; j++) d.in_vals[j] = p.in_vals[j];
       }
-      const int32_t* g_tids = in->tids;
-      const uint32_t* g_count = in->d_count;
-      if (op.n_preds > 0 && !agg_ws_supported(in->tids, kv, op.n_keys, op.n_aggs, out.gb_cap)) {
+      if (!in && agg_dense_supported(in_cap, &bp, kc, op.n_keys, op.key_bits, ag, op.n_aggs)) {
+        out.d_rows = (uint32_t*)A.get(64);
+        if (A.failed) return DDQ_ENOMEM_DEVICE;
+        init_fill(out.d_rows, 4, 0, st);
+        cudaError_t e = launch_groupby_init(out.gb_table, out.gb_cap, op.n_aggs, st);
+        if (e == cudaSuccess)
+          e = launch_agg_dense(in_cap, kc, op.n_keys, op.key_bits, ag, op.n_aggs, out.gb_table, out.gb_cap,
+                               out.d_error, st, &bp, out.d_rows);
+        if (e == cudaSuccess)
+          e = launch_groupby_compact(out.gb_table, out.gb_cap, op.n_aggs, out.gb_keys, out.gb_accs, out.gb_groups, st);
+        return cuda_status(e, "aggregate (dense)");
+      }
+      const int32_t* g_tids = in ? in->tids : nullptr;
+      const uint32_t* g_count = in ? in->d_count : nullptr;
+      if (!in && op.n_preds == 0) {  // other dense shapes: an all-rows TID list feeds the generic kernels
+        int32_t* ft = (int32_t*)A.get((uint64_t)std::max<int64_t>(in_cap, 1) * 4);
+        uint32_t* fc = (uint32_t*)A.get(64);
+        if (A.failed) return DDQ_ENOMEM_DEVICE;
+        cudaError_t e0 = launch_iota(ft, in_cap, fc, st);
+        if (e0 != cudaSuccess) return cuda_status(e0, "aggregate: row list");
+        g_tids = ft;
+        g_count = fc;
+      }
+      if (op.n_preds > 0 && (!in || !agg_ws_supported(in->tids, kv, op.n_keys, op.n_aggs, out.gb_cap))) {
         // no fused kernel for this shape: a selection into a temporary TID list
         // (carrying the key vectors) feeds the aggregation
-        int32_t* ft = (int32_t*)A.get((uint64_t)std::max<int64_t>(in->cap, 1) * 4);
+        int32_t* ft = (int32_t*)A.get((uint64_t)std::max<int64_t>(in_cap, 1) * 4);
         uint32_t* fc = (uint32_t*)A.get(64);
-        void* fscr = A.get(filter_scratch_bytes(in->cap));
+        void* fscr = A.get(filter_scratch_bytes(in_cap));
         const int32_t* cin[3] = {nullptr, nullptr, nullptr};
         int32_t* cout2[3] = {nullptr, nullptr, nullptr};
         int nc = 0;
         for (int k = 0; k < op.n_keys; k++)
           if (kv[k]) {
             cin[nc] = kv[k];
-            cout2[nc] = (int32_t*)A.get((uint64_t)std::max<int64_t>(in->cap, 1) * 4);
+            cout2[nc] = (int32_t*)A.get((uint64_t)std::max<int64_t>(in_cap, 1) * 4);
             kv[k] = cout2[nc];
             nc++;
           }
@@ -534,15 +557,15 @@ ddq_status run_gpu_op(GpuOpCtx& ctx, const ddq_op& op, Inter& out) {
         FilterArgs fa;
         fa.preds = bp.p;
         fa.n_preds = bp.n;
-        fa.in_tids = in->tids;
-        fa.d_in_count = in->d_count;
-        fa.n_cap = in->cap;
+        fa.in_tids = in ? in->tids : nullptr;
+        fa.d_in_count = in ? in->d_count : nullptr;
+        fa.n_cap = in_cap;
         fa.carry_in = cin;
         fa.carry_out = cout2;
         fa.n_carry = nc;
         fa.out_tids = ft;
         fa.d_out_count = fc;
-        fa.out_cap = in->cap;
+        fa.out_cap = in_cap;
         fa.d_overflow = out.d_error;
         fa.scratch = fscr;
         cudaError_t e0 = launch_filter(fa, st);
@@ -559,10 +582,10 @@ ddq_status run_gpu_op(GpuOpCtx& ctx, const ddq_op& op, Inter& out) {
       cudaError_t e = launch_groupby_init(out.gb_table, out.gb_cap, op.n_aggs, st);
       if (e == cudaSuccess) {
         if (bp.n > 0)
-          e = launch_agg_ws(g_tids, g_count, in->cap, kv, kc, op.n_keys, op.key_bits, ag, op.n_aggs, out.gb_table,
+          e = launch_agg_ws(g_tids, g_count, in_cap, kv, kc, op.n_keys, op.key_bits, ag, op.n_aggs, out.gb_table,
                             out.gb_cap, out.d_error, st, &bp, out.d_rows);
         else
-          e = launch_groupby(g_tids, g_count, in->cap, kv, kc, op.n_keys, op.key_bits, ag, op.n_aggs, out.gb_table,
+          e = launch_groupby(g_tids, g_count, in_cap, kv, kc, op.n_keys, op.key_bits, ag, op.n_aggs, out.gb_table,
                              out.gb_cap, out.d_error, st);
       }
       if (e == cudaSuccess)
@@ -1049,6 +1072,9 @@ static ddq_status validate_plan(ddq_db* db, const ddq_plan* plan) {
       return set_error(DDQ_EINVAL, "plan: a fetch must be a GATHER referencing an earlier HASH_BUILD");
     if (op.kind == DDQ_OP_HASH_PROBE && op.fk_vec > 0 && op.input < 0)
       return set_error(DDQ_EINVAL, "plan: a vector-keyed probe needs an input");
+    if (op.kind == DDQ_OP_AGGREGATE && op.input < 0)
+      for (int k = 0; k < op.n_keys && k < DDQ_MAX_KEYS; k++)
+        if (op.key_src[k] >= 0) return set_error(DDQ_EINVAL, "plan: an aggregate over all rows keys on columns only");
     if (op.kind == DDQ_OP_AGGREGATE) {
       int bits = 0;
       for (int k = 0; k < op.n_keys && k < DDQ_MAX_KEYS; k++) bits += op.key_bits[k] > 0 ? op.key_bits[k] : 21;
@@ -1471,7 +1497,7 @@ int32_t ddq_prepared_profile(ddq_prepared* p, void* stream, int32_t max_ops, flo
         break;
       case DDQ_OP_AGGREGATE: {
         cls = 4;
-        bytes = m * 4;
+        bytes = op.input >= 0 ? m * 4 : 0;  // the input TID list (none over all rows)
         // fused selection: first predicate column at every input TID, the rest
         // and everything below at the rows that passed (d_rows)
         double mr = m;

@@ -113,6 +113,13 @@ cudaError_t launch_groupby(const int32_t* tids, const uint32_t* d_count, int64_t
 // AGGREGATE with fused predicates (reading O26): only input rows passing every
 // predicate contribute; *d_rows (optional) += the number that did.
 // warp-autonomous aggregation for <= 2 aggregates and small group counts (agg.cu)
+// dense small-domain aggregation over every row of a table (agg.cu)
+bool agg_dense_supported(int64_t n_rows, const struct BuildPreds* preds, const int32_t* const* key_col, int n_keys,
+                         const int32_t* key_bits, const ddq_dev_agg* aggs, int n_aggs);
+cudaError_t launch_agg_dense(int64_t n_rows, const int32_t* const* key_col, int n_keys, const int32_t* key_bits,
+                             const ddq_dev_agg* aggs, int n_aggs, void* table, uint32_t capacity, uint32_t* d_error,
+                             cudaStream_t st, const struct BuildPreds* preds, uint32_t* d_rows);
+cudaError_t launch_iota(int32_t* out, int64_t n, uint32_t* d_count, cudaStream_t st);
 bool agg_ws_supported(const int32_t* tids, const int32_t* const* key_vec, int n_keys, int n_aggs,
                       uint32_t capacity);
 cudaError_t launch_agg_ws(const int32_t* tids, const uint32_t* d_count, int64_t n_cap,

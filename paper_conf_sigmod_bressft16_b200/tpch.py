@@ -38,13 +38,17 @@ def load_tpch(db: Database, data, cache: bool = True, tables=None) -> None:
         db.dicts[d] = data.dict_for(c)
 
 
-def tpch_plan(db: Database, q: str, limit: int = 0) -> PlanBuilder:
+def tpch_plan(db: Database, q: str, limit: int = 0, dense: bool = True) -> PlanBuilder:
+    """dense (Q1): one AGGREGATE over every lineitem row with the shipdate predicate
+    fused (agg_dense_small_kernel, reading O26); False: select -> TID list ->
+    aggregate at the TIDs (the paper's operator granularity, kept under test)."""
     P = db.plan()
     li = "lineitem"
     if q == "tpch1":
         # l_shipdate <= date '1998-12-01' - interval '90' day  (= 19980902, O11)
-        t = P.select(li, [("l_shipdate", -2**31, 19980902)])
-        P.aggregate(li, t, keys=["l_returnflag", "l_linestatus"],
+        ship = [("l_shipdate", -2**31, 19980902)]
+        t = -1 if dense else P.select(li, ship)
+        P.aggregate(li, t, where=ship if dense else None, keys=["l_returnflag", "l_linestatus"],
                     aggs=[(A.AGG_SUM, ["l_quantity"]), (A.AGG_SUM, ["l_extendedprice"]),
                           (A.AGG_SUM_MUL_100M, ["l_extendedprice", "l_discount"]),
                           (A.AGG_SUM_MUL_100M_100P, ["l_extendedprice", "l_discount", "l_tax"]),

@@ -1,7 +1,8 @@
 """Parity at BASELINE full size, in the launch configuration bench.py times:
 all 13 SSB queries at SF20 (120 M lineorder rows) through prepared CUDA-graph plans,
 element-by-element equal to the oracle (run in parallel threads: the C++ oracle
-releases the GIL).  Also TPC-H Q1/Q6 at SF30 (180 M lineitem rows)."""
+releases the GIL), launched like bench.py (4 concurrent streams).  Also TPC-H
+Q1/Q3/Q5/Q6 at SF30 (180 M lineitem rows)."""
 import concurrent.futures as cf
 import os
 
@@ -25,12 +26,17 @@ def test_ssb_sf20_all_queries_equal_oracle():
     data = datagen.SSB(20)
     db = Database(cache_bytes=64 << 30, heap_bytes=24 << 30)
     load_ssb(db, data)
-    got = {}
-    for q in SSB_QUERIES:
-        p = db.prepare(ssb_plan(db, q))
-        for _ in range(2):
-            p.launch()
-        got[q] = p.fetch().rows
+    import torch
+    # bench.py's launch configuration: the 13 prepared graphs round-robin over 4
+    # concurrent streams, twice (the second launch reuses every buffer)
+    preps = [db.prepare(ssb_plan(db, q), use_graph=True) for q in SSB_QUERIES]
+    lanes = [torch.cuda.Stream() for _ in range(4)]
+    for _ in range(2):
+        for i, p in enumerate(preps):
+            p.launch(lanes[i % 4].cuda_stream)
+    torch.cuda.synchronize()
+    got = {q: p.fetch().rows for q, p in zip(SSB_QUERIES, preps)}
+    for p in preps:
         p.close()
     db.close()
     # the oracle reads only the columns each query needs; generate them up front
@@ -42,20 +48,21 @@ def test_ssb_sf20_all_queries_equal_oracle():
         assert _norm(q, got[q]) == _norm(q, want[q]), q
 
 
-def test_tpch_sf30_q1_q6_equal_oracle():
+def test_tpch_sf30_all_queries_equal_oracle():
     from paper_conf_sigmod_bressft16_b200 import Database
     from paper_conf_sigmod_bressft16_b200.tpch import load_tpch, tpch_plan
     data = datagen.TPCH(30)
     db = Database(cache_bytes=64 << 30, heap_bytes=24 << 30)
-    load_tpch(db, data, tables=["lineitem"])
+    load_tpch(db, data)
+    qs = ("tpch1", "tpch3", "tpch5", "tpch6")
     got = {}
-    for q in ("tpch1", "tpch6"):
+    for q in qs:
         p = db.prepare(tpch_plan(db, q))
         p.launch()
         got[q] = p.fetch().rows
         p.close()
     db.close()
-    with cf.ThreadPoolExecutor(max_workers=2) as ex:
-        want = dict(zip(("tpch1", "tpch6"), ex.map(lambda q: oracle.run(data, q), ("tpch1", "tpch6"))))
+    with cf.ThreadPoolExecutor(max_workers=4) as ex:
+        want = dict(zip(qs, ex.map(lambda q: oracle.run(data, q), qs)))
     for q in got:
         assert got[q] == [tuple(r) for r in want[q]], q

@@ -71,3 +71,63 @@ def test_tpch_cold_path_gpu_only():
     st = db.stats()
     assert st["h2d_bytes"] > 0 and st["cache_misses"] > 0
     db.close()
+
+
+def test_tpch1_unfused_variant():
+    """select -> TID list -> aggregate (the operator-at-a-time plan) = the dense
+    fused aggregation = the oracle."""
+    from paper_conf_sigmod_bressft16_b200.tpch import tpch_plan
+    db = _db()
+    p = db.prepare(tpch_plan(db, "tpch1", dense=False))
+    p.launch()
+    got = p.fetch().rows
+    p.close()
+    assert got == _want("tpch1")
+
+
+@pytest.mark.parametrize("shape", ["count_only", "no_pred", "wide_domain", "seven_cols", "in_pred"])
+def test_dense_aggregate_shapes(shape):
+    """AGGREGATE over all rows (no input): the dense small-domain kernel and the
+    fallbacks (all-rows TID list, fused selection) vs numpy on the same columns."""
+    import numpy as np
+    from paper_conf_sigmod_bressft16_b200 import _abi as A
+    db, d = _db(), _data()
+    li = "lineitem"
+    P = db.plan()
+    rf, ls = d.col(li, "l_returnflag").astype(np.int64), d.col(li, "l_linestatus").astype(np.int64)
+    qty, ep = d.col(li, "l_quantity").astype(np.int64), d.col(li, "l_extendedprice").astype(np.int64)
+    disc, tax = d.col(li, "l_discount").astype(np.int64), d.col(li, "l_tax").astype(np.int64)
+    ship = d.col(li, "l_shipdate").astype(np.int64)
+    keys, bits, where = ["l_returnflag", "l_linestatus"], [2, 1], [("l_shipdate", 19950101, 19961231)]
+    mask = (ship >= 19950101) & (ship <= 19961231)
+    aggs = [(A.AGG_SUM, ["l_quantity"]), (A.AGG_COUNT, [])]
+    vals = [qty, np.ones_like(qty)]
+    if shape == "count_only":
+        aggs, vals = [(A.AGG_COUNT, [])], [np.ones_like(qty)]
+    elif shape == "no_pred":
+        where, mask = None, np.ones_like(mask)
+    elif shape == "wide_domain":  # 21-bit keys: not a small domain -> generic kernels
+        bits = None
+    elif shape == "seven_cols":  # > 6 distinct argument columns -> generic kernels
+        aggs = [(A.AGG_SUM, ["l_quantity"]), (A.AGG_SUM, ["l_extendedprice"]), (A.AGG_SUM, ["l_discount"]),
+                (A.AGG_SUM, ["l_tax"]), (A.AGG_SUM, ["l_shipdate"]), (A.AGG_SUM, ["l_orderkey"]),
+                (A.AGG_SUM, ["l_suppkey"])]
+        vals = [qty, ep, disc, tax, ship, d.col(li, "l_orderkey").astype(np.int64),
+                d.col(li, "l_suppkey").astype(np.int64)]
+    elif shape == "in_pred":
+        where = [("l_discount", [1, 4, 9])]
+        mask = np.isin(disc, [1, 4, 9])
+        aggs = [(A.AGG_SUM_MUL_100M_100P, ["l_extendedprice", "l_discount", "l_tax"]), (A.AGG_COUNT, [])]
+        vals = [ep * (100 - disc) * (100 + tax), np.ones_like(qty)]
+    P.aggregate(li, -1, keys=keys, key_bits=bits, aggs=aggs, where=where, order_by=[1, 2], max_groups=64)
+    r = db.run(P)
+    p = db.prepare(P)
+    p.launch()
+    got = p.fetch().rows
+    p.close()
+    assert r.rows == got
+    want = []
+    for a in sorted(set(zip(rf[mask].tolist(), ls[mask].tolist()))):
+        m = mask & (rf == a[0]) & (ls == a[1])
+        want.append(a + tuple(int(v[m].sum()) for v in vals))
+    assert [tuple(x) for x in got] == want
