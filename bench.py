@@ -221,7 +221,9 @@ def main():
 
     shard = Shard()
     t_setup = time.perf_counter()
-    db = Database(device=local, cache_bytes=64 << 30, heap_bytes=24 << 30, rank=rank, world=ws)
+    # heap: intermediates scale with the shard (24 GiB at SF20's 120 M rows)
+    heap = min(110 << 30, max(24 << 30, int((24 << 30) * shard_rows / 120_000_000)))
+    db = Database(device=local, cache_bytes=64 << 30, heap_bytes=heap, rank=rank, world=ws)
 
     load_ssb(db, shard, row_begin=b, row_end=e, presliced=True)
     preps = [db.prepare(ssb_plan(db, q), use_graph=True) for q in SSB_QUERIES]
@@ -383,7 +385,7 @@ def main():
     #      H2D from pinned host memory inside the timed region (GPU-only placement)
     e2e = None
     if not args.no_e2e and ws == 1:
-        cold = Database(device=local, cache_bytes=64 << 30, heap_bytes=24 << 30, placement=A.PLACE_GPU_ONLY)
+        cold = Database(device=local, cache_bytes=64 << 30, heap_bytes=heap, placement=A.PLACE_GPU_ONLY)
         load_ssb(cold, shard, row_begin=b, row_end=e, cache=False, presliced=True)
         plans = [ssb_plan(cold, q) for q in SSB_QUERIES]
         all_cols = [(t, c) for (t, c) in cold._cols]

@@ -20,11 +20,13 @@ def _norm(q, rows):
     return [tuple(r) for r in rows]
 
 
-def test_ssb_sf20_all_queries_equal_oracle():
+@pytest.mark.parametrize("sf", [20, pytest.param(100, marks=pytest.mark.skipif(
+    os.environ.get("DDQ_SF100") != "1", reason="SF100 (600 M rows, ~70 GB host RAM): set DDQ_SF100=1"))])
+def test_ssb_all_queries_equal_oracle(sf):
     from paper_conf_sigmod_bressft16_b200 import Database
     from paper_conf_sigmod_bressft16_b200.ssb import SSB_QUERIES, load_ssb, ssb_plan
-    data = datagen.SSB(20)
-    db = Database(cache_bytes=64 << 30, heap_bytes=24 << 30)
+    data = datagen.SSB(sf)
+    db = Database(cache_bytes=64 << 30, heap_bytes=(24 << 30) * sf // 20)
     load_ssb(db, data)
     import torch
     # bench.py's launch configuration: the 13 prepared graphs round-robin over 4
