@@ -248,6 +248,11 @@ typedef struct {
                                     0: compile-time placement, one thread per operator */
   int32_t cache_policy;          /* 0 = LFU (Alg. 1), 1 = LRU (App. E) */
   uint32_t fault_alloc_every;    /* fault injection: fail every Nth device heap alloc (0=off) */
+  int32_t transfer_packing;      /* 1 (default): ddq_load_column also keeps a frame-of-reference
+                                    byte-packed pinned copy (value - min in 1..4 bytes) and a
+                                    cold cache load copies that and widens it on the device
+                                    (fewer bytes over PCIe);
+                                    0: copy the raw column */
 } ddq_config;
 
 void ddq_config_default(ddq_config* cfg);

@@ -41,7 +41,8 @@ class Config(ctypes.Structure):
                 ("cache_bytes", ctypes.c_uint64), ("heap_bytes", ctypes.c_uint64),
                 ("gpu_workers", ctypes.c_int32), ("host_workers", ctypes.c_int32),
                 ("placement", ctypes.c_int32), ("chopping", ctypes.c_int32),
-                ("cache_policy", ctypes.c_int32), ("fault_alloc_every", ctypes.c_uint32)]
+                ("cache_policy", ctypes.c_int32), ("fault_alloc_every", ctypes.c_uint32),
+                ("transfer_packing", ctypes.c_int32)]
 
 
 class Pred(ctypes.Structure):

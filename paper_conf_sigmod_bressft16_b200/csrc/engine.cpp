@@ -717,6 +717,7 @@ void ddq_config_default(ddq_config* c) {
   c->chopping = 1;
   c->cache_policy = 0;
   c->fault_alloc_every = 0;
+  c->transfer_packing = 1;
 }
 
 
@@ -775,6 +776,7 @@ void ddq_close(ddq_db* db) {
   for (auto& c : db->cols) {
     if (c->dev) cudaFreeAsync(c->dev, db->copy_stream);
     if (c->host) cudaFreeHost(c->host);
+    if (c->host_packed) cudaFreeHost(c->host_packed);
   }
   cudaStreamSynchronize(db->copy_stream);
   if (db->cache_pool) cudaMemPoolDestroy(db->cache_pool);
@@ -817,6 +819,27 @@ ddq_status ddq_load_column(ddq_db* db, ddq_table t, const char* name, ddq_type t
     int64_t v = c->width == 4 ? ((const int32_t*)host_data)[i] : ((const int64_t*)host_data)[i];
     if (i == 0 || v < c->vmin) c->vmin = v;
     if (i == 0 || v > c->vmax) c->vmax = v;
+  }
+  // transfer encoding: value - vmin in the fewest whole bytes (<= 4, < width)
+  if (db->cfg.transfer_packing && n_rows > 0) {
+    const uint64_t range = (uint64_t)c->vmax - (uint64_t)c->vmin;
+    int tw = range < (1ull << 8) ? 1 : range < (1ull << 16) ? 2 : range < (1ull << 24) ? 3 : range < (1ull << 32) ? 4 : 0;
+    if (tw && tw < c->width &&
+        cudaHostAlloc(&c->host_packed, packed_bytes(n_rows, tw), cudaHostAllocPortable) == cudaSuccess) {
+      uint8_t* dst = (uint8_t*)c->host_packed;
+      std::memset(dst + (size_t)n_rows * tw, 0, packed_bytes(n_rows, tw) - (size_t)n_rows * tw);
+      for (int64_t i = 0; i < n_rows; i++) {
+        const int64_t v = c->width == 4 ? ((const int32_t*)host_data)[i] : ((const int64_t*)host_data)[i];
+        const uint32_t d = (uint32_t)((uint64_t)v - (uint64_t)c->vmin);
+        switch (tw) {
+          case 1: dst[i] = (uint8_t)d; break;
+          case 2: ((uint16_t*)dst)[i] = (uint16_t)d; break;
+          case 4: ((uint32_t*)dst)[i] = d; break;
+          default: std::memcpy(dst + (size_t)i * 3, &d, 3); break;  // little endian
+        }
+      }
+      c->tw = tw;
+    }
   }
   db->cols.push_back(std::move(c));
   int id = (int)db->cols.size() - 1;
@@ -869,9 +892,25 @@ ddq_status cache_column_locked(ddq_db* db, int c, bool on_demand, std::unique_lo
   }
   db->cache_used += bytes;
   col.loading = true;
+  // packed transfer: stage the packed bytes in a pool block, widen into the column
+  void* stage = nullptr;
+  const size_t pbytes = col.tw ? packed_bytes(col.n, col.tw) : 0;
+  if (col.tw && cudaMallocFromPoolAsync(&stage, pbytes, db->cache_pool, db->copy_stream) != cudaSuccess) {
+    cudaGetLastError();
+    stage = nullptr;  // no room for the staging block: send the raw column
+  }
   lk.unlock();
   uint64_t t0 = now_ns();
-  e = cudaMemcpyAsync(p, col.host, (size_t)col.n * col.width, cudaMemcpyHostToDevice, db->copy_stream);
+  uint64_t moved = 0;
+  if (stage) {
+    e = cudaMemcpyAsync(stage, col.host_packed, pbytes, cudaMemcpyHostToDevice, db->copy_stream);
+    if (e == cudaSuccess) e = launch_unpack(stage, col.tw, col.vmin, p, col.width, col.n, db->copy_stream);
+    if (e == cudaSuccess) e = cudaFreeAsync(stage, db->copy_stream);
+    moved = pbytes;
+  } else {
+    e = cudaMemcpyAsync(p, col.host, (size_t)col.n * col.width, cudaMemcpyHostToDevice, db->copy_stream);
+    moved = (uint64_t)col.n * col.width;
+  }
   if (e == cudaSuccess) e = cudaEventRecord(done, db->copy_stream);
   if (e == cudaSuccess) e = cudaEventSynchronize(done);
   const uint64_t dt = now_ns() - t0;
@@ -885,7 +924,7 @@ ddq_status cache_column_locked(ddq_db* db, int c, bool on_demand, std::unique_lo
     return cuda_status(e, "cache H2D");
   }
   db->stats.h2d_ns += dt;
-  db->stats.h2d_bytes += (uint64_t)col.n * col.width;
+  db->stats.h2d_bytes += moved;
   col.dev = p;
   col.on_demand = on_demand;
   col.evict_pending = false;

@@ -303,7 +303,7 @@ class Database:
     def __init__(self, device: int = 0, cache_bytes: int = 64 << 30, heap_bytes: int = 32 << 30,
                  gpu_workers: int = 4, host_workers: int = 4, placement: int = A.PLACE_DATA_DRIVEN,
                  chopping: bool = True, cache_policy: int = 0, fault_alloc_every: int = 0,
-                 rank: int = 0, world: int = 1):
+                 rank: int = 0, world: int = 1, transfer_packing: bool = True):
         cfg = A.Config()
         lib().ddq_config_default(ctypes.byref(cfg))
         cfg.device, cfg.rank, cfg.world = device, rank, world
@@ -311,6 +311,7 @@ class Database:
         cfg.gpu_workers, cfg.host_workers = gpu_workers, host_workers
         cfg.placement, cfg.chopping = placement, 1 if chopping else 0
         cfg.cache_policy, cfg.fault_alloc_every = cache_policy, fault_alloc_every
+        cfg.transfer_packing = 1 if transfer_packing else 0
         h = ctypes.c_void_p()
         check(lib().ddq_open(ctypes.byref(cfg), ctypes.byref(h)))
         self.h = h
