@@ -359,7 +359,16 @@ __global__ void __launch_bounds__(ws_nw(kIn == 1) * 32, 1) ws_kernel(const __gri
     // predicated stores through a running ring pointer, no per-item branches (a
     // branchy version spent 43 % of the kernel's instructions here)
     const uint32_t r0 = (pos0 & (RING - 1)) + incl - c;  // this lane's first ring slot
-    if ((pos0 & (RING - 1)) + tot <= RING) {  // the claim does not wrap the ring
+    if ((kIn != 1 && !kPay && !kCarry) && (pos0 & (RING - 1)) + tot <= RING) {
+      // positions only (a dense semi-join): visit the lane's set bits, not all 16
+      // items -- most first probes keep <= 4 % of the rows, where 16 predicated
+      // stores per lane and tile were mostly no-ops
+      int32_t* wp = ring + r0;
+      for (uint32_t f = flags; f; f &= f - 1) {
+        const uint32_t j = __ffs(f) - 1;
+        *wp++ = (int32_t)(base + (j >> 2) * 128 + (j & 3));
+      }
+    } else if ((pos0 & (RING - 1)) + tot <= RING) {  // the claim does not wrap the ring
       int32_t* wp = ring + r0;
 #pragma unroll
       for (int j = 0; j < WS_ITEMS; j++) {
