@@ -20,7 +20,9 @@ def klass(name: str) -> str:
         return "dense" if m.group(1) == "0" else "at-tids"
     if "scan_kernel" in name or "star_kernel" in name or "filter_kernel" in name:
         return "dense" if re.search(r"scan_kernel<\d+, (?:\(bool\))?(?:0|false)", name) else "at-tids"
-    if "agg_ws" in name or "groupby" in name:
+    if "fetch_kernel" in name:  # late payload fetch through a join index: an at-TIDs lookup
+        return "at-tids"
+    if "agg_ws" in name or "agg_dense" in name or "groupby" in name:
         return "agg"
     if "build" in name:
         return "build"
