@@ -347,6 +347,7 @@ constexpr int DS_R = 4;               // rows per thread per stage
 constexpr int DS_SR = DS_T * DS_R;    // rows per ring stage
 constexpr int DS_MAXC = 12;           // distinct columns streamed
 constexpr int DS_MAX_DA = 64;
+static_assert(4 /*DS_R*/ * 8 <= 32, "overflow mask: DS_R x A bits");
 constexpr size_t DS_SMEM_MAX = 227 * 1024 - 1024;
 
 struct DenseAggParams {
@@ -483,59 +484,65 @@ __global__ void __launch_bounds__(DS_T, 1) agg_dense_small_kernel(const __grid_c
       idx[j] = d * (uint32_t)(A * DS_T) + tid;
     }
     nrows += __popc(livem);
+    long long v[A][DS_R];  // every aggregate's value for the thread's rows (dead rows: 0)
 #pragma unroll
     for (int a = 0; a < A; a++) {
       const int kind = KINDS == DS_RUNTIME ? P.kind[a] : (int)((KINDS >> (3 * a)) & 7u);
       const long long* xs = reinterpret_cast<const long long*>(stage + P.off[P.acol[a][0]]) + tid;
       const long long* ys = reinterpret_cast<const long long*>(stage + P.off[P.acol[a][1]]) + tid;
       const long long* zs = reinterpret_cast<const long long*>(stage + P.off[P.acol[a][2]]) + tid;
-      long long v[DS_R];
       if (kind == DDQ_AGG_COUNT) {
 #pragma unroll
-        for (int j = 0; j < DS_R; j++) v[j] = 1;
+        for (int j = 0; j < DS_R; j++) v[a][j] = 1;
       } else if (kind == DDQ_AGG_SUM) {
 #pragma unroll
-        for (int j = 0; j < DS_R; j++) v[j] = xs[j * DS_T];
+        for (int j = 0; j < DS_R; j++) v[a][j] = xs[j * DS_T];
       } else if (kind == DDQ_AGG_SUM_MUL) {
 #pragma unroll
-        for (int j = 0; j < DS_R; j++) v[j] = xs[j * DS_T] * ys[j * DS_T];
+        for (int j = 0; j < DS_R; j++) v[a][j] = xs[j * DS_T] * ys[j * DS_T];
       } else if (kind == DDQ_AGG_SUM_SUB) {
 #pragma unroll
-        for (int j = 0; j < DS_R; j++) v[j] = xs[j * DS_T] - ys[j * DS_T];
+        for (int j = 0; j < DS_R; j++) v[a][j] = xs[j * DS_T] - ys[j * DS_T];
       } else if (kind == DDQ_AGG_SUM_MUL_100M) {
 #pragma unroll
-        for (int j = 0; j < DS_R; j++) v[j] = xs[j * DS_T] * (100 - ys[j * DS_T]);
+        for (int j = 0; j < DS_R; j++) v[a][j] = xs[j * DS_T] * (100 - ys[j * DS_T]);
       } else {
 #pragma unroll
-        for (int j = 0; j < DS_R; j++) v[j] = xs[j * DS_T] * (100 - ys[j * DS_T]) * (100 + zs[j * DS_T]);
+        for (int j = 0; j < DS_R; j++) v[a][j] = xs[j * DS_T] * (100 - ys[j * DS_T]) * (100 + zs[j * DS_T]);
       }
-      bool ovf = false;
+      if (livem != (1u << DS_R) - 1u) {
 #pragma unroll
-      for (int j = 0; j < DS_R; j++) {
-        const long long vj = ((livem >> j) & 1u) ? v[j] : 0;
-        long long* slot = part + idx[j] + (uint32_t)a * DS_T;
-        const long long old = *slot;
-        const long long sum = (long long)((unsigned long long)old + (unsigned long long)vj);
-        const bool o = ((old ^ sum) & (vj ^ sum)) < 0;
-        ovf |= o;
-        *slot = o ? old : sum;
+        for (int j = 0; j < DS_R; j++) v[a][j] = ((livem >> j) & 1u) ? v[a][j] : 0;
       }
-      if (__builtin_expect(ovf, 0)) {  // signed overflow (never for SSB/TPC-H data): spill exactly
+    }
+    // row-major read-modify-writes: the A partials of one row are distinct slots
+    // (independent loads, one shared-memory latency per row); consecutive rows of a
+    // thread may hit the same group, which the in-order LSU keeps correct
+    // partials wrap modulo 2^64; a signed overflow (never for SSB/TPC-H data) adds
+    // +-2^64 to the entry's int128 cell, so slot + cell stays exact
+    uint32_t omask = 0;
 #pragma unroll
-        for (int j = 0; j < DS_R; j++) {
-          const long long vj = ((livem >> j) & 1u) ? v[j] : 0;
-          long long* slot = part + idx[j] + (uint32_t)a * DS_T;
-          const long long old = *slot;
-          const long long sum = (long long)((unsigned long long)old + (unsigned long long)vj);
-          if (((old ^ sum) & (vj ^ sum)) < 0) {
+    for (int j = 0; j < DS_R; j++) {
+      long long* row = part + idx[j];
+      long long old[A];
+#pragma unroll
+      for (int a = 0; a < A; a++) old[a] = row[a * DS_T];
+#pragma unroll
+      for (int a = 0; a < A; a++) {
+        const long long sum = (long long)((unsigned long long)old[a] + (unsigned long long)v[a][j]);
+        row[a * DS_T] = sum;
+        omask |= (((old[a] ^ sum) & (v[a][j] ^ sum)) < 0 ? 1u : 0u) << (j * A + a);
+      }
+    }
+    if (__builtin_expect(omask != 0, 0)) {
+#pragma unroll
+      for (int j = 0; j < DS_R; j++)
+#pragma unroll
+        for (int a = 0; a < A; a++)
+          if ((omask >> (j * A + a)) & 1u) {
             unsigned long long* sp = spill + (size_t)(idx[j] - tid + (uint32_t)a * DS_T) / DS_T * 2;
-            add_i128(sp, sp + 1, (unsigned long long)old, old < 0 ? -1 : 0);
-            *slot = vj;
-          } else {
-            *slot = sum;
+            add_i128(sp, sp + 1, 0ull, v[a][j] > 0 ? 1 : -1);
           }
-        }
-      }
     }
     __syncthreads();  // every thread is done with this slot: refill it
     if (tid == 0 && blockIdx.x + (k + S) * gridDim.x < nch) issue(k + S);

@@ -131,3 +131,33 @@ def test_dense_aggregate_shapes(shape):
         m = mask & (rf == a[0]) & (ls == a[1])
         want.append(a + tuple(int(v[m].sum()) for v in vals))
     assert [tuple(x) for x in got] == want
+
+
+@pytest.mark.parametrize("n", [1000, 200_003])
+def test_dense_aggregate_int64_overflow_is_exact(n):
+    """Per-thread int64 partials overflow (values near 2^62, both signs): the
+    dense kernel spills into int128 cells, the group sums stay exact."""
+    import numpy as np
+    from paper_conf_sigmod_bressft16_b200 import Database
+    from paper_conf_sigmod_bressft16_b200 import _abi as A
+    rng = np.random.default_rng(n)
+    g = rng.integers(0, 3, size=n).astype(np.int32)
+    x = rng.integers((1 << 62) - 1000, (1 << 62), size=n, dtype=np.int64)
+    x[rng.random(n) < 0.3] *= -1
+    y = rng.integers(0, 50, size=n).astype(np.int64)
+    db = Database(cache_bytes=1 << 30, heap_bytes=1 << 28)
+    db.create_table("t", n)
+    for name, col in (("g", g), ("x", x), ("y", y)):
+        db.load_column("t", name, col)
+        db.cache("t", name)
+    P = db.plan()
+    P.aggregate("t", -1, keys=["g"], key_bits=[2], aggs=[(A.AGG_SUM, ["x"]), (A.AGG_SUM, ["y"]), (A.AGG_COUNT, [])],
+                order_by=[1], max_groups=4)
+    p = db.prepare(P)
+    p.launch()
+    got = p.fetch().rows
+    p.close()
+    db.close()
+    want = [(k, int(sum(int(v) for v in x[g == k])), int(y[g == k].sum()), int((g == k).sum()))
+            for k in sorted(set(g.tolist()))]
+    assert [tuple(r) for r in got] == want
