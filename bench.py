@@ -46,10 +46,9 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--profile-only", action="store_true", help="short run for ncu")
-    ap.add_argument("--streams", type=int, default=4,
+    ap.add_argument("--streams", type=int, default=0,
                     help="concurrent query streams inside a step: the 13 plans round-robin over K CUDA streams "
-                         "(the paper's bounded GPU worker pool P:246-260, default 4 = reading O17); 1 = back to "
-                         "back on one stream.  The serial (1-stream) step time is always measured too.")
+                         "(the paper's parallel users); 0 = pick the fastest of 1/2/4 from untimed trial steps")
     return ap.parse_args()
 
 
@@ -232,7 +231,8 @@ def main():
     sptr = stream.cuda_stream
     kernels_per_step = sum(p.kernels for p in preps)
 
-    side = [torch.cuda.Stream() for _ in range(max(args.streams, 1) - 1)]
+    all_side = [torch.cuda.Stream() for _ in range(max(args.streams, 4) - 1)]
+    side = all_side[:max(args.streams, 1) - 1]
 
     def step(serial: bool = False):
         if serial or not side:
@@ -246,6 +246,29 @@ def main():
             p.launch(lanes[i % len(lanes)].cuda_stream)
         for s2 in side:
             stream.wait_stream(s2)
+
+    if args.streams == 0 and not args.profile_only:
+        # untimed trial steps pick the stream count (4 at SF20; a dimension bitmap that
+        # spills shared memory, e.g. customer at SF >= 60, makes concurrency lose)
+        trial = {}
+        for k in (1, 2, 4):
+            side = all_side[:k - 1]
+            step()
+            ta, tb = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            torch.cuda.synchronize()
+            ta.record(stream)
+            for _ in range(2):
+                step()
+            tb.record(stream)
+            torch.cuda.synchronize()
+            trial[k] = ta.elapsed_time(tb)
+        if ws > 1:  # every rank uses the same count: the max-over-ranks time of each
+            import torch.distributed as dist
+            t = torch.tensor([trial[k] for k in (1, 2, 4)], device="cuda")
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            trial = dict(zip((1, 2, 4), t.tolist()))
+        args.streams = min(trial, key=trial.get)
+        side = all_side[:args.streams - 1]
 
     # N>1: the 13 compacted partial group tables of a step are packed on the device
     # ([n, keys[cap], accs[cap*n_aggs*2]] per query) and exchanged with ONE NCCL
