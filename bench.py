@@ -44,6 +44,9 @@ def parse():
     ap.add_argument("--sf", type=float, default=SF_PER_GPU, help="scale factor per GPU")
     ap.add_argument("--e2e-steps", type=int, default=5)
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--emulate-world", type=int, default=0,
+                    help="diagnostic: size the data for W ranks (dimensions of SF sf*W) and run rank 0's "
+                         "lineorder shard on this single process (per-GPU step of a W-GPU weak-scaling run)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--profile-only", action="store_true", help="short run for ncu")
     ap.add_argument("--streams", type=int, default=0,
@@ -196,10 +199,11 @@ def main():
     if ws > 1:
         import torch.distributed as dist
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
-    sf_total = args.sf * ws
+    dws = args.emulate_world if (args.emulate_world and ws == 1) else ws  # ranks the data is sized for
+    sf_total = args.sf * dws
     data = datagen.SSB(sf_total)
     n_lo = data.rows("lineorder")
-    b, e = rank * n_lo // ws, (rank + 1) * n_lo // ws
+    b, e = rank * n_lo // dws, (rank + 1) * n_lo // dws
     shard_rows = e - b
 
     class Shard:  # dimension tables whole, lineorder rows [b, e) only
@@ -346,7 +350,7 @@ def main():
         ms = float(t.item())
         dist.barrier()
     ms_per_step = ms / args.steps
-    total_rows = 13 * n_lo  # all ranks together
+    total_rows = 13 * n_lo * ws // dws  # all ranks together (emulation: this shard only)
     value = total_rows * args.steps / (ms / 1e3)
     # the same K steps with the 13 plans back to back on one stream (per-query latency view)
     serial_ms = None

@@ -213,9 +213,13 @@ def finalize_partials(root: A.Op, keys: np.ndarray, accs: np.ndarray) -> QueryRe
 class Catalog:
     """Name -> id catalogue without a device (plans for host-only finalisation)."""
 
-    def __init__(self, dicts: dict[str, list[str]]):
+    def __init__(self, dicts: dict[str, list[str]], rows: dict[str, int] | None = None):
         self.dicts = dicts
         self._ids: dict = {}
+        self._rows = rows or {}  # table sizes the plans' join orders depend on (reading O30)
+
+    def table_rows(self, table: str) -> int:
+        return self._rows.get(table, 0)
 
     def _id(self, key) -> int:
         return self._ids.setdefault(key, len(self._ids))
@@ -316,6 +320,7 @@ class Database:
         check(lib().ddq_open(ctypes.byref(cfg), ctypes.byref(h)))
         self.h = h
         self._tables: dict[str, int] = {}
+        self._rows: dict[str, int] = {}
         self._cols: dict[tuple[str, str], int] = {}
         self.dicts: dict[str, list[str]] = {}
         self._root_aggs: dict = {}
@@ -336,7 +341,12 @@ class Database:
         t = ctypes.c_int32()
         check(lib().ddq_create_table(self.h, name.encode(), n_rows, row_begin, ctypes.byref(t)))
         self._tables[name] = t.value
+        self._rows[name] = n_rows
         return t.value
+
+    def table_rows(self, table: str) -> int:
+        """Rows of `table` in this process (a shard's rows for row-sharded tables)."""
+        return self._rows[table]
 
     def load_column(self, table: str, name: str, data: np.ndarray) -> int:
         data = np.ascontiguousarray(data)

@@ -182,3 +182,20 @@ def test_fetch_through_join_with_misses(path):
         key = key - 2**32 if key >= 2**31 else key  # the miss value as an int32
         got[key] = got.get(key, 0) + int(r[1])
     assert got == want
+
+
+def test_o30_supplier_first_orders_equal_oracle(monkeypatch):
+    """O30: with the customer bitmap declared too large for shared memory, Q3.x,
+    Q4.1 and Q4.2 probe supplier first; results equal the oracle (SF1 and planted)."""
+    from paper_conf_sigmod_bressft16_b200 import ssb as S
+    monkeypatch.setattr(S, "SMEM_BITMAP_KEYS", 1)
+    for kind in ("1", "planted"):
+        db = _db(kind)
+        for q in ("ssb3.1", "ssb3.2", "ssb3.3", "ssb3.4", "ssb4.1", "ssb4.2"):
+            for variant in ("chain", "chain_eager", "star"):
+                p = db.prepare(S.ssb_plan(db, q, **VARIANTS[variant]))
+                p.launch()
+                got = p.fetch().rows
+                p.close()
+                assert norm(q, got) == _oracle(kind, q), (kind, q, variant)
+            assert norm(q, db.run(S.ssb_plan(db, q)).rows) == _oracle(kind, q), (kind, q)
