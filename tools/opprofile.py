@@ -16,15 +16,32 @@ def main():
     ap.add_argument("--queries", default="")
     ap.add_argument("--launch", type=int, default=0)
     ap.add_argument("--star", action="store_true", help="n-ary STAR operator instead of binary-operator chains")
+    ap.add_argument("--world", type=int, default=1,
+                    help="dimensions of SF sf*W, lineorder = rank 0's shard of W (a weak-scaling rank)")
     a = ap.parse_args()
     import torch
     import datagen
     from paper_conf_sigmod_bressft16_b200 import Database
     from paper_conf_sigmod_bressft16_b200.ssb import SSB_QUERIES, load_ssb, ssb_plan
     qs = a.queries.split(",") if a.queries else SSB_QUERIES
-    data = datagen.SSB(a.sf)
+    data = datagen.SSB(a.sf * a.world)
     db = Database(cache_bytes=64 << 30, heap_bytes=24 << 30)
-    load_ssb(db, data)
+    if a.world > 1:
+        e = data.rows("lineorder") // a.world
+        sf_total = a.sf * a.world
+
+        class Shard:  # dimensions whole, lineorder rows [0, e) only
+            def __getitem__(self, col):
+                return datagen.ssb_column(col, sf_total, begin=0, end=e) if col.startswith("lo_") else data[col]
+
+            def rows(self, t):
+                return data.rows(t)
+
+            def dict_for(self, col):
+                return data.dict_for(col)
+        load_ssb(db, Shard(), row_begin=0, row_end=e, presliced=True)
+    else:
+        load_ssb(db, data)
     preps = {q: db.prepare(ssb_plan(db, q, star=a.star)) for q in qs}
     torch.cuda.synchronize()
     if a.launch:
