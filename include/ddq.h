@@ -125,7 +125,10 @@ ddq_status ddq_op_hash_probe(const uint64_t* table, uint32_t capacity, const int
 /* Direct-mapped join index (S8(a3)/(a4), the build/probe used when the build key
  * column spans a compact range [key_min, key_min + range)): a membership bitmap of
  * `range` bits followed (16-byte aligned) by an int32 payload array of `range`
- * entries; ddq_op_join_index_bytes(range) bytes, zero the bitmap with
+ * entries and, when range > 1.5 M keys (a bitmap too large for one SM's shared
+ * memory), a coarse bitmap (1 bit per 2^cg keys, set by the build; probes filter
+ * with it in shared memory and read exact bits from L2 only for its hits);
+ * ddq_op_join_index_bytes(range) bytes, zero the bitmaps with
  * ddq_op_join_index_init.  Same semantics as hash build / probe: unique keys
  * (duplicate -> *d_error = 1; key outside the range -> *d_error = 3), probe =
  * semi-join + payload of survivors.  Chosen by the engine when range <= 16 x the

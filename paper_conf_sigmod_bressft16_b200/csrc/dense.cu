@@ -61,7 +61,9 @@ enum WsKind : int {
   WK_HT_GLOBAL = 3,  // hash probe, table in global
   WK_SEL_RANGE = 4,  // conjunctive range predicates (TID input)
   WK_SEL_GENERIC = 5,  // range / IN predicates (TID input)
-  WK_EQ = 6            // FILTER_EQ of two positional vectors (TID input)
+  WK_EQ = 6,           // FILTER_EQ of two positional vectors (TID input)
+  WK_BM_COARSE = 7     // join-index probe: a coarse bitmap (1 bit per 2^cg keys) in smem
+                       // filters, the exact bit is read from the global (L2) bitmap
 };
 
 struct WsPred {
@@ -91,6 +93,8 @@ struct WsParams {
   int32_t key_min;
   uint32_t range;
   uint32_t bitmap_words;
+  uint32_t cg;              // WK_BM_COARSE: log2 keys per coarse bit
+  const uint32_t* coarse;   // WK_BM_COARSE: the index's coarse bitmap (global)
   // hash table (open addressing, 8-byte slots key<<32|payload)
   const uint64_t* table;
   uint32_t cap_mask;
@@ -188,7 +192,7 @@ __global__ void __launch_bounds__(ws_nw(kIn == 1) * 32, 1) ws_kernel(const __gri
   constexpr uint32_t BLK = ws_blk(kCarry);
   const uint32_t RL = P.ring_logr, RM = (1u << RL) - 1u, RING = BLK << RL;  // R = RM + 1 blocks
   int32_t* ring = reinterpret_cast<int32_t*>(smem);  // fields [tid | payload | carried...] x RING
-  constexpr bool kProbe = kKind <= WK_HT_GLOBAL;
+  constexpr bool kProbe = kKind <= WK_HT_GLOBAL || kKind == WK_BM_COARSE;
   constexpr bool kHash = kKind == WK_HT_SMEM || kKind == WK_HT_GLOBAL;
   uint32_t* s_bm = reinterpret_cast<uint32_t*>(smem + P.tab_off);
   uint64_t* s_ht = reinterpret_cast<uint64_t*>(smem + P.tab_off);
@@ -204,6 +208,8 @@ __global__ void __launch_bounds__(ws_nw(kIn == 1) * 32, 1) ws_kernel(const __gri
     if (threadIdx.x == 0) s_bm[P.bitmap_words] = 0u;
   }
   if (kKind == WK_HT_SMEM) stage_bulk(s_ht, P.table, (P.cap_mask + 1) * 8, &s_bar);
+  if (kKind == WK_BM_COARSE)  // the index's precomputed coarse bitmap
+    stage_bulk(s_bm, P.coarse, (uint32_t)((((P.range >> P.cg) + 1 + 31) / 32 * 4 + 15) & ~15u), &s_bar);
   __syncthreads();
 
   const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
@@ -259,11 +265,30 @@ __global__ void __launch_bounds__(ws_nw(kIn == 1) * 32, 1) ws_kernel(const __gri
           if (kKind == WK_BM_SMEM) {
             const uint32_t oo = min((uint32_t)(key[j] - P.key_min), P.range);
             hit = (s_bm[oo >> 5] >> (oo & 31)) & 1u;
+          } else if (kKind == WK_BM_COARSE) {  // coarse filter here, exact bit below
+            const uint32_t oo = min((uint32_t)(key[j] - P.key_min), P.range);
+            const uint32_t cb = oo >> P.cg;
+            hit = (s_bm[cb >> 5] >> (cb & 31)) & (oo < P.range ? 1u : 0u);
           } else {
             const uint32_t o = (uint32_t)(key[j] - P.key_min);
             hit = o < P.range ? (__ldg(P.bitmap + (o >> 5)) >> (o & 31)) & 1u : 0u;
           }
           m |= hit << j;
+        }
+        if (kKind == WK_BM_COARSE) {  // the exact bits of the coarse hits, loads in flight together
+          uint32_t fine[WS_ITEMS];
+#pragma unroll
+          for (int j = 0; j < WS_ITEMS; j++) {
+            const uint32_t o = (uint32_t)(key[j] - P.key_min);
+            fine[j] = ((m >> j) & 1u) ? __ldg(P.bitmap + (o >> 5)) : 0u;
+          }
+          uint32_t m2 = 0;
+#pragma unroll
+          for (int j = 0; j < WS_ITEMS; j++) {
+            const uint32_t o = (uint32_t)(key[j] - P.key_min);
+            m2 |= ((fine[j] >> (o & 31)) & 1u) << j;
+          }
+          m = m2;
         }
         flags &= m;
         if (kPay) {
@@ -495,7 +520,7 @@ void ws_attr() {
 }
 template <int K>
 void ws_attr_kind() {
-  constexpr bool kProbe = K <= WK_HT_GLOBAL;
+  constexpr bool kProbe = K <= WK_HT_GLOBAL || K == WK_BM_COARSE;
   if constexpr (kProbe) {  // dense inputs: probes only (payload, or a bitmap of the survivors)
     ws_attr<K, 0, false, false, false>();
     ws_attr<K, 0, true, false, false>();
@@ -516,7 +541,7 @@ void ws_attr_kind() {
 template <int K>
 void launch_k(int in, bool pay, bool carry, bool obits, int grid, size_t smem, cudaStream_t st,
               const WsParams& p) {
-  constexpr bool kProbe = K <= WK_HT_GLOBAL;
+  constexpr bool kProbe = K <= WK_HT_GLOBAL || K == WK_BM_COARSE;
   if constexpr (kProbe) {
     if (in == 0) {
       const dim3 blk(ws_nw(false) * 32);
@@ -590,6 +615,7 @@ cudaError_t launch_ws(const FilterArgs& a, cudaStream_t st) {
     ws_attr_kind<WK_SEL_RANGE>();
     ws_attr_kind<WK_SEL_GENERIC>();
     ws_attr_kind<WK_EQ>();
+    ws_attr_kind<WK_BM_COARSE>();
   }
   const int in = a.in_bits ? 2 : (a.in_tids ? 1 : 0);
   WsParams p{};
@@ -618,6 +644,23 @@ cudaError_t launch_ws(const FilterArgs& a, cudaStream_t st) {
       tab = ((size_t)p.bitmap_words * 4 + 15) / 16 * 16 + 16;  // bulk-copy rounding + the zero word
       kind = (!a.no_smem && (obits ? 0 : 4 * ring1) + tab <= budget && stage_pays(a.n_cap, tab)) ? WK_BM_SMEM
                                                                                                  : WK_BM_GLOBAL;
+      // a bitmap too large for one SM (customer at SF > 50, part at SF >= 128): the
+      // index's coarse bitmap (1 bit per 2^cg keys) filters in shared memory; only
+      // coarse hits read the exact bit from L2
+      static const char* co_env = getenv("DDQ_BM_COARSE");  // "0": exact lookups in L2 instead
+      // Probes of every row only: at a TID list (or row bitmap) the exact lookups
+      // are L1-cached, and the coarse table's shared memory shrinks that L1 (SF80
+      // Q3.1's customer probe at 24 M TIDs: 514 -> 720 us with it)
+      if (kind == WK_BM_GLOBAL && a.coarse && in == 0 && !a.no_smem && !(co_env && co_env[0] == '0')) {
+        const uint32_t cg = join_index_cg(a.range);
+        const size_t ctab = ji_coarse_bytes_cg(a.range, cg);
+        if ((obits ? 0 : 4 * ring1) + ctab <= budget && stage_pays(a.n_cap, ctab)) {
+          kind = WK_BM_COARSE;
+          p.cg = cg;
+          p.coarse = a.coarse;
+          tab = ctab;
+        }
+      }
     } else {
       p.table = a.table;
       p.cap_mask = a.capacity - 1;
@@ -656,7 +699,7 @@ cudaError_t launch_ws(const FilterArgs& a, cudaStream_t st) {
   // shared memory is carved out of the unified L1 where the payload-array lookups
   // live: 16 blocks made the date probe's d_year lookups miss (74 -> 141 us) and
   // 8 blocks slowed the late fetch itself (119 -> 195 us)
-  const size_t tab_smem = (kind == WK_BM_SMEM || kind == WK_HT_SMEM) ? tab : 0;
+  const size_t tab_smem = (kind == WK_BM_SMEM || kind == WK_HT_SMEM || kind == WK_BM_COARSE) ? tab : 0;
   const int logr = 2;
   const size_t ring = obits ? 0 : ring1 << logr;
   p.ring_logr = logr;
@@ -689,6 +732,7 @@ cudaError_t launch_ws(const FilterArgs& a, cudaStream_t st) {
     case WK_HT_GLOBAL: launch_k<WK_HT_GLOBAL>(in, pay, carry, obits, (int)grid, smem, st, p); break;
     case WK_SEL_RANGE: launch_k<WK_SEL_RANGE>(in, false, carry, false, (int)grid, smem, st, p); break;
     case WK_SEL_GENERIC: launch_k<WK_SEL_GENERIC>(in, false, carry, false, (int)grid, smem, st, p); break;
+    case WK_BM_COARSE: launch_k<WK_BM_COARSE>(in, pay, carry, obits, (int)grid, smem, st, p); break;
     default: launch_k<WK_EQ>(in, false, carry, false, (int)grid, smem, st, p); break;
   }
   return cudaGetLastError();

@@ -193,6 +193,13 @@ static ddq_status inter_to_device(ddq_db* db, Inter& x, cudaStream_t st) {
     cudaMemcpyAsync(join_index_payload(d.jidx, d.jrange), x.h_payarr->data(), (size_t)x.jrange * 4,
                     cudaMemcpyHostToDevice, st);
     bytes += x.h_bitmap->size() * 4 + (uint64_t)x.jrange * 4;
+    if (join_index_cg(x.jrange)) {  // derived from the membership bits (a host-built index)
+      std::vector<uint32_t> co(join_index_coarse_bytes(x.jrange) / 4);
+      join_index_coarse_host(x.h_bitmap->data(), x.jrange, co.data());
+      cudaMemcpyAsync(join_index_coarse(d.jidx, d.jrange), co.data(), co.size() * 4, cudaMemcpyHostToDevice, st);
+      cudaStreamSynchronize(st);  // `co` is a stack buffer
+      bytes += co.size() * 4;
+    }
   } else if (x.host_table) {
     d.table_cap = x.table_cap;
     d.table_ptr = (uint64_t*)get((uint64_t)x.table_cap * 8);

@@ -259,6 +259,7 @@ ddq_status run_gpu_op(GpuOpCtx& ctx, const ddq_op& op, Inter& out) {
         if (build->jidx) {
           fa.bitmap = join_index_bitmap(build->jidx);
           fa.payarr = join_index_payload(build->jidx, build->jrange);
+          fa.coarse = join_index_coarse(build->jidx, build->jrange);
           fa.key_min = build->jmin;
           fa.range = build->jrange;
         }
@@ -390,7 +391,7 @@ ddq_status run_gpu_op(GpuOpCtx& ctx, const ddq_op& op, Inter& out) {
         out.cap = 0;
         if (A.failed) return DDQ_ENOMEM_DEVICE;
         init_fill(out.d_error, 4, 0, st);
-        cudaError_t e = init_fill(out.jidx, ((size_t)out.jrange + 31) / 32 * 4, 0, st);
+        cudaError_t e = join_index_init(out.jidx, out.jrange, st);
         if (e == cudaSuccess)
           e = launch_join_index_build(keys, payload, in_tids, in_cnt, in_cap, out.jmin, out.jrange, out.jidx,
                                       out.d_error, st, &bp);

@@ -10,6 +10,7 @@
 #include <algorithm>
 #include <climits>
 #include <cstdint>
+#include <cstring>
 #include <cstdlib>
 #include <cuda_runtime.h>
 
@@ -154,14 +155,45 @@ cudaError_t launch_hash_build(const int32_t* keys, const int32_t* payload, const
 }
 
 // ------------------------------------------------------- direct-mapped join index
+uint32_t ji_smem_keys() {
+  static const uint32_t v = [] {
+    const char* e = getenv("DDQ_JI_SMEM_KEYS");
+    return e ? (uint32_t)strtoul(e, nullptr, 10) : 1500000u;
+  }();
+  return v;
+}
+size_t ji_coarse_max() {
+  static const size_t v = [] {
+    const char* e = getenv("DDQ_JI_COARSE_MAX");
+    return e ? (size_t)strtoull(e, nullptr, 10) : (size_t)160 * 1024;
+  }();
+  return v;
+}
+
 size_t join_index_bytes(uint32_t range) {
-  return ((((size_t)range + 31) / 32 * 4 + 15) / 16) * 16 + (size_t)range * 4;
+  return ji_fine_bytes(range) + ((size_t)range * 4 + 15) / 16 * 16 + join_index_coarse_bytes(range);
+}
+
+cudaError_t join_index_init(void* idx, uint32_t range, cudaStream_t st) {
+  cudaError_t e = init_fill(idx, ((size_t)range + 31) / 32 * 4, 0, st);
+  if (e == cudaSuccess && join_index_cg(range))
+    e = init_fill(join_index_coarse(idx, range), join_index_coarse_bytes(range), 0, st);
+  return e;
+}
+
+void join_index_coarse_host(const uint32_t* bitmap, uint32_t range, uint32_t* coarse) {
+  const uint32_t cg = join_index_cg(range);
+  if (!cg) return;
+  std::memset(coarse, 0, join_index_coarse_bytes(range));
+  for (uint32_t o = 0; o < range; o++)
+    if ((bitmap[o >> 5] >> (o & 31)) & 1u) coarse[(o >> cg) >> 5] |= 1u << ((o >> cg) & 31);
 }
 
 __global__ void join_index_build_kernel(const int32_t* __restrict__ keys, const int32_t* __restrict__ payload,
                                         const int32_t* __restrict__ in_tids, const uint32_t* d_in_count,
                                         uint32_t n_static, int32_t key_min, uint32_t range, uint32_t* bitmap,
-                                        int32_t* payarr, uint32_t* d_error, const __grid_constant__ BuildPreds bp) {
+                                        int32_t* payarr, uint32_t* coarse, uint32_t cg, uint32_t* d_error,
+                                        const __grid_constant__ BuildPreds bp) {
   const uint32_t n = d_in_count ? ld_relaxed_u32(d_in_count) : n_static;
   for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
     const int32_t r = in_tids ? in_tids[i] : (int32_t)i;
@@ -173,6 +205,7 @@ __global__ void join_index_build_kernel(const int32_t* __restrict__ keys, const 
     }
     const uint32_t old = atomicOr(bitmap + (o >> 5), 1u << (o & 31));
     if (old & (1u << (o & 31))) atomicMax(d_error, 1u);  // PKs are unique (O13)
+    if (coarse) atomicOr(coarse + ((o >> cg) >> 5), 1u << ((o >> cg) & 31));
     payarr[o] = payload ? payload[r] : r;
   }
 }
@@ -184,8 +217,8 @@ cudaError_t launch_join_index_build(const int32_t* keys, const int32_t* payload,
   int64_t g = (n_cap + 255) / 256;
   int grid = (int)(g > num_sms() * 8 ? num_sms() * 8 : (g < 1 ? 1 : g));
   join_index_build_kernel<<<grid, 256, 0, st>>>(keys, payload, in_tids, d_in_count, (uint32_t)n_cap, key_min, range,
-                                                join_index_bitmap(index), join_index_payload(index, range), d_error,
-                                                bp);
+                                                join_index_bitmap(index), join_index_payload(index, range),
+                                                join_index_coarse(index, range), join_index_cg(range), d_error, bp);
   return cudaGetLastError();
 }
 

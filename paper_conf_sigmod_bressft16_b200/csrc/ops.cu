@@ -140,8 +140,7 @@ size_t ddq_op_join_index_bytes(uint32_t range) { return join_index_bytes(range);
 
 ddq_status ddq_op_join_index_init(void* index, uint32_t range, void* stream) {
   if (!index || range == 0) return set_error(DDQ_EINVAL, "join_index_init: bad arguments");
-  return cuda_status(cudaMemsetAsync(index, 0, ((size_t)range + 31) / 32 * 4, (cudaStream_t)stream),
-                     "ddq_op_join_index_init");
+  return cuda_status(join_index_init(index, range, (cudaStream_t)stream), "ddq_op_join_index_init");
 }
 
 ddq_status ddq_op_join_index_build(const int32_t* keys, const int32_t* payload, const int32_t* in_tids,
@@ -171,6 +170,7 @@ ddq_status ddq_op_join_index_probe(const void* index, int32_t key_min, uint32_t 
   a.probe = true;
   a.bitmap = join_index_bitmap(const_cast<void*>(index));
   a.payarr = join_index_payload(const_cast<void*>(index), range);
+  a.coarse = join_index_coarse(const_cast<void*>(index), range);
   a.key_min = key_min;
   a.range = range;
   a.fk = fk;

@@ -45,6 +45,7 @@ struct FilterArgs {
   // direct-mapped join index (probe): bitmap + payload array over [key_min, key_min+range)
   const uint32_t* bitmap = nullptr;
   const int32_t* payarr = nullptr;
+  const uint32_t* coarse = nullptr;  // the index's coarse bitmap (join_index_coarse), or null
   int32_t key_min = 0;
   uint32_t range = 0;
   const int32_t* fk = nullptr;
@@ -90,11 +91,44 @@ cudaError_t launch_hash_build(const int32_t* keys, const int32_t* payload, const
 cudaError_t launch_star(const ddq_dev_term* terms, int n_terms, int64_t n_rows, int32_t* out_tids,
                         uint32_t* d_out_count, int64_t out_cap, uint32_t* d_overflow, cudaStream_t st);
 
+// Direct-mapped join index over [key_min, key_min + range):
+//   [membership bitmap, range bits][payload int32 x range][coarse bitmap]
+// The coarse bitmap (1 bit per 2^cg keys, OR of the group; set by the build) exists
+// only when the bitmap is too large for one SM's shared memory next to a probe's
+// compaction ring (range > JI_SMEM_KEYS); probes then filter with the coarse bitmap
+// in shared memory and read exact bits from L2 for coarse hits only (dense.cu).
+// thresholds (defaults 1.5 M keys, 160 KB; env DDQ_JI_SMEM_KEYS / DDQ_JI_COARSE_MAX
+// override them for tests that force coarse bitmaps on small data)
+uint32_t ji_smem_keys();
+size_t ji_coarse_max();
+inline size_t ji_fine_bytes(uint32_t range) { return ((((size_t)range + 31) / 32 * 4 + 15) / 16) * 16; }
+inline size_t ji_coarse_bytes_cg(uint32_t range, uint32_t cg) {
+  return (((size_t)(range >> cg) + 1 + 31) / 32 * 4 + 15) / 16 * 16;
+}
+inline uint32_t join_index_cg(uint32_t range) {
+  if (range <= ji_smem_keys()) return 0;
+  uint32_t cg = 1;
+  while (cg < 16 && ji_coarse_bytes_cg(range, cg) > ji_coarse_max()) cg++;
+  return cg;
+}
+inline size_t join_index_coarse_bytes(uint32_t range) {
+  const uint32_t cg = join_index_cg(range);
+  return cg ? ji_coarse_bytes_cg(range, cg) : 0;
+}
 size_t join_index_bytes(uint32_t range);
 inline uint32_t* join_index_bitmap(void* idx) { return reinterpret_cast<uint32_t*>(idx); }
 inline int32_t* join_index_payload(void* idx, uint32_t range) {
-  return reinterpret_cast<int32_t*>(reinterpret_cast<char*>(idx) + ((((size_t)range + 31) / 32 * 4 + 15) / 16) * 16);
+  return reinterpret_cast<int32_t*>(reinterpret_cast<char*>(idx) + ji_fine_bytes(range));
 }
+inline uint32_t* join_index_coarse(void* idx, uint32_t range) {
+  return join_index_cg(range) ? reinterpret_cast<uint32_t*>(reinterpret_cast<char*>(idx) + ji_fine_bytes(range) +
+                                                            ((size_t)range * 4 + 15) / 16 * 16)
+                              : nullptr;
+}
+// zero the membership and coarse bitmaps of an index (the payload needs no init)
+cudaError_t join_index_init(void* idx, uint32_t range, cudaStream_t st);
+// the coarse words of a host-side membership bitmap (a host-built index moving to the GPU)
+void join_index_coarse_host(const uint32_t* bitmap, uint32_t range, uint32_t* coarse);
 cudaError_t launch_join_index_build(const int32_t* keys, const int32_t* payload, const int32_t* in_tids,
                                     const uint32_t* d_in_count, int64_t n_cap, int32_t key_min, uint32_t range,
                                     void* index, uint32_t* d_error, cudaStream_t st,
