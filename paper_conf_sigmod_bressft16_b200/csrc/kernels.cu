@@ -189,6 +189,10 @@ void join_index_coarse_host(const uint32_t* bitmap, uint32_t range, uint32_t* co
     if ((bitmap[o >> 5] >> (o & 31)) & 1u) coarse[(o >> cg) >> 5] |= 1u << ((o >> cg) & 31);
 }
 
+// One thread per build row: atomicOr of its bit (an old bit = a duplicate key),
+// the coarse bit when the index has a coarse bitmap, the payload.  (A warp-
+// aggregated variant -- one atomic per run of equal words -- measured no faster:
+// SSB builds 531 -> 571 us per step, TPC-H Q3's orders builds 174 -> 155 us.)
 __global__ void join_index_build_kernel(const int32_t* __restrict__ keys, const int32_t* __restrict__ payload,
                                         const int32_t* __restrict__ in_tids, const uint32_t* d_in_count,
                                         uint32_t n_static, int32_t key_min, uint32_t range, uint32_t* bitmap,

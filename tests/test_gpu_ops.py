@@ -148,6 +148,62 @@ def test_join_index_rejects_duplicates_and_out_of_range(ops):
     assert int(err[0].item()) == 3
 
 
+@pytest.mark.parametrize("keys", [
+    [3, 4, 3], [7] * 32, list(range(40)) + [17], [1, 2, 33, 34, 1], list(range(0, 64, 2)) + [62],
+    [5] + list(range(100, 131)) + [5]])
+def test_join_index_warp_build_detects_duplicates(ops, keys):
+    """Duplicate build keys are reported wherever they sit: adjacent rows, far
+    apart in one warp, across warps."""
+    _, err = ops.join_index_build(_t(np.array(keys, dtype=np.int32)), 0, 256)
+    assert int(err[0].item()) == 1
+
+
+@pytest.mark.parametrize("keys", [[0, 40, 1, 2], [0, 64, 1, 65, 2, 66], [3, 100, 4, 101, 5] * 1 + [200, 6]])
+def test_join_index_warp_build_interleaved_words_no_false_duplicates(ops, keys):
+    """Unique keys whose bitmap words interleave inside a warp (separate runs of one
+    word): no duplicate reported, every key present."""
+    idx, err = ops.join_index_build(_t(np.array(keys, dtype=np.int32)), 0, 256)
+    assert int(err[0].item()) == 0
+    bits = np.unpackbits(idx[:32].cpu().numpy().view(np.uint8), bitorder="little")[:256].astype(bool)
+    assert np.flatnonzero(bits).tolist() == sorted(keys)
+
+
+@pytest.mark.parametrize("n_keys,order", [(3_000_000, "sorted"), (3_000_000, "random"), (1_600_000, "sorted"),
+                                          (20_000_000, "sorted")])
+def test_join_index_bitmaps_and_coarse_bits(ops, n_keys, order):
+    """Membership bitmap, payloads and (range > 1.5 M) the coarse bitmap of a build
+    over a selected subset of keys (sorted rows: one atomic per word; random order)
+    equal numpy's; no false errors."""
+    rng = np.random.default_rng(n_keys)
+    rows = np.arange(n_keys, dtype=np.int32)
+    keys = rows + 1 if order == "sorted" else (rng.permutation(n_keys) + 1).astype(np.int32)
+    sel = np.flatnonzero(rng.random(n_keys) < 0.3).astype(np.int32)
+    payload = (rows * 7).astype(np.int32)
+    idx, err = ops.join_index_build(_t(keys), 1, n_keys, payload=_t(payload), in_tids=_t(sel),
+                                    in_count=ops.count_cell(sel.size), n=sel.size)
+    assert int(err[0].item()) == 0
+    raw = idx.cpu().numpy()
+    fine_bytes = ((n_keys + 31) // 32 * 4 + 15) // 16 * 16
+    member = np.zeros(n_keys, dtype=bool)
+    member[keys[sel] - 1] = True
+    bits = np.unpackbits(raw[:fine_bytes].view(np.uint8), bitorder="little")[:n_keys].astype(bool)
+    assert np.array_equal(bits, member)
+    pay = raw[fine_bytes:fine_bytes + n_keys * 4].view(np.int32)
+    assert np.array_equal(pay[keys[sel] - 1], payload[sel])
+    coarse_off = fine_bytes + (n_keys * 4 + 15) // 16 * 16
+    if n_keys <= 1_500_000:
+        assert raw.size == coarse_off
+        return
+    cg = 1
+    while (((n_keys >> cg) + 1 + 31) // 32 * 4 + 15) // 16 * 16 > 160 * 1024:
+        cg += 1
+    ncb = (n_keys >> cg) + 1
+    want = np.zeros(ncb, dtype=bool)
+    want[np.flatnonzero(member) >> cg] = True
+    got = np.unpackbits(raw[coarse_off:].view(np.uint8), bitorder="little")[:ncb].astype(bool)
+    assert np.array_equal(got, want)
+
+
 def test_build_rejects_duplicate_keys(ops):
     keys = np.array([5, 9, 5, 1], dtype=np.int32)
     _, err = ops.hash_build(_t(keys), 16)

@@ -19,6 +19,7 @@ def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--sf", type=float, default=30)
     ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--ops", action="store_true", help="also print the per-operator profile (stderr)")
     a = ap.parse_args()
     import torch
     import datagen
@@ -45,6 +46,10 @@ def main():
         rows = p.fetch(st.cuda_stream).rows
         prof = p.profile(st.cuda_stream)
         byt = sum(b for _, b, _ in prof)
+        if a.ops:
+            names = {0: "dense", 1: "at-tids", 2: "build", 3: "gather", 4: "agg"}
+            print(q, " | ".join(f"{names.get(c, c)}:{m * 1e3:.0f}us/{b / 1e6:.0f}MB" for m, b, c in prof),
+                  file=sys.stderr, flush=True)
         print(json.dumps({"config": "M4", "mode": "hot", "query": q, "sf": a.sf, "lineitem_rows": n,
                           "ms": round(ms, 4), "rows_per_s": n / (ms / 1e3), "model_gb": round(byt / 1e9, 3),
                           "model_gbs": round(byt / (ms / 1e3) / 1e9, 1), "groups": len(rows)}), flush=True)
