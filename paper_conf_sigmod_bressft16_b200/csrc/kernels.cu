@@ -209,7 +209,11 @@ __global__ void join_index_build_kernel(const int32_t* __restrict__ keys, const 
     }
     const uint32_t old = atomicOr(bitmap + (o >> 5), 1u << (o & 31));
     if (old & (1u << (o & 31))) atomicMax(d_error, 1u);  // PKs are unique (O13)
-    if (coarse) atomicOr(coarse + ((o >> cg) >> 5), 1u << ((o >> cg) & 31));
+    if (coarse) {  // most coarse bits are set early: test before the atomic
+      uint32_t* cw = coarse + ((o >> cg) >> 5);
+      const uint32_t cb = 1u << ((o >> cg) & 31);
+      if (!(*reinterpret_cast<volatile uint32_t*>(cw) & cb)) atomicOr(cw, cb);
+    }
     payarr[o] = payload ? payload[r] : r;
   }
 }

@@ -2,7 +2,7 @@
 the build; used when a dimension's bitmap does not fit one SM, e.g. customer at
 SF > 50): probes filter with it in shared memory and read exact bits from L2
 (WK_BM_COARSE).  Forced on small data by lowering the thresholds (every index over
-more than 1000 keys; coarse budgets of 160 KB and of 256 bytes for large cg): every
+more than 1000 keys; coarse budgets of 160 KB and of 1 KB for cg 2-3): every
 SSB query -- dense probes, probes at TIDs, bitmap-masked probes, host-built indexes
 moved to the GPU (GPU-only placement) -- equals the oracle."""
 import os
@@ -55,7 +55,7 @@ print("ok")
 """
 
 
-@pytest.mark.parametrize("coarse_max", ["163840", "256"])
+@pytest.mark.parametrize("coarse_max", ["163840", "1024"])
 def test_ssb_with_coarse_bitmaps_equals_oracle(coarse_max):
     env = dict(os.environ, DDQ_JI_SMEM_KEYS="1000", DDQ_JI_COARSE_MAX=coarse_max)
     out = subprocess.run([sys.executable, "-c", SCRIPT.format(root=ROOT)], env=env, capture_output=True,
