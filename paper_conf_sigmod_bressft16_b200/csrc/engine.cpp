@@ -779,6 +779,8 @@ void ddq_close(ddq_db* db) {
     if (c->host) cudaFreeHost(c->host);
     if (c->host_packed) cudaFreeHost(c->host_packed);
   }
+  for (auto& kv : db->cache_free) cudaFreeAsync(kv.second, db->copy_stream);
+  db->cache_free.clear();
   cudaStreamSynchronize(db->copy_stream);
   if (db->cache_pool) cudaMemPoolDestroy(db->cache_pool);
   if (db->copy_stream) cudaStreamDestroy(db->copy_stream);
@@ -866,6 +868,31 @@ ddq_status ddq_find_column(ddq_db* db, const char* table, const char* name, ddq_
 }  // extern "C"
 
 namespace ddq {
+// Cache blocks: an exact-size free list in front of the stream-ordered pool.  The
+// pool alone let cold steps stretch from 52 ms to 150-600 ms (tools/e2e_steps.py):
+// blocks freed and re-requested in a different order each step.
+static void* cache_block(ddq_db* db, size_t bytes) {
+  auto it = db->cache_free.find(bytes);
+  if (it != db->cache_free.end()) {
+    void* p = it->second;
+    db->cache_free.erase(it);
+    return p;
+  }
+  void* p = nullptr;
+  if (cudaMallocFromPoolAsync(&p, bytes, db->cache_pool, db->copy_stream) != cudaSuccess) {
+    cudaGetLastError();
+    // drop the free list back into the pool and retry once
+    for (auto& kv : db->cache_free) cudaFreeAsync(kv.second, db->copy_stream);
+    db->cache_free.clear();
+    if (cudaMallocFromPoolAsync(&p, bytes, db->cache_pool, db->copy_stream) != cudaSuccess) {
+      cudaGetLastError();
+      return nullptr;
+    }
+  }
+  return p;
+}
+static void cache_unblock(ddq_db* db, void* p, size_t bytes) { db->cache_free.emplace(bytes, p); }
+
 // H2D copy of one column into the cache.  The caller holds db->mu through `lk`;
 // it is released for the copy itself, so operators of other queries keep
 // launching while PCIe is busy (a concurrent request for the same column waits
@@ -883,12 +910,14 @@ ddq_status cache_column_locked(ddq_db* db, int c, bool on_demand, std::unique_lo
   cudaSetDevice(db->device);
   void* p = nullptr;
   // padded: TMA reads whole 16-byte chunks
-  cudaError_t e = cudaMallocFromPoolAsync(&p, (bytes + 255) / 256 * 256, db->cache_pool, db->copy_stream);
-  if (e != cudaSuccess) return cuda_status(e, "cache pool alloc");
+  const size_t dbytes = (bytes + 255) / 256 * 256;
+  p = cache_block(db, dbytes);
+  if (!p) return set_error(DDQ_ENOMEM_DEVICE, "cache: device memory exhausted for " + col.name);
+  cudaError_t e = cudaSuccess;
   cudaEvent_t done = nullptr;
   e = cudaEventCreateWithFlags(&done, cudaEventDisableTiming);
   if (e != cudaSuccess) {
-    cudaFreeAsync(p, db->copy_stream);
+    cache_unblock(db, p, dbytes);
     return cuda_status(e, "cache event");
   }
   db->cache_used += bytes;
@@ -896,17 +925,13 @@ ddq_status cache_column_locked(ddq_db* db, int c, bool on_demand, std::unique_lo
   // packed transfer: stage the packed bytes in a pool block, widen into the column
   void* stage = nullptr;
   const size_t pbytes = col.tw ? packed_bytes(col.n, col.tw) : 0;
-  if (col.tw && cudaMallocFromPoolAsync(&stage, pbytes, db->cache_pool, db->copy_stream) != cudaSuccess) {
-    cudaGetLastError();
-    stage = nullptr;  // no room for the staging block: send the raw column
-  }
+  if (col.tw) stage = cache_block(db, pbytes);  // null: no room, send the raw column
   lk.unlock();
   uint64_t t0 = now_ns();
   uint64_t moved = 0;
   if (stage) {
     e = cudaMemcpyAsync(stage, col.host_packed, pbytes, cudaMemcpyHostToDevice, db->copy_stream);
     if (e == cudaSuccess) e = launch_unpack(stage, col.tw, col.vmin, p, col.width, col.n, db->copy_stream);
-    if (e == cudaSuccess) e = cudaFreeAsync(stage, db->copy_stream);
     moved = pbytes;
   } else {
     e = cudaMemcpyAsync(p, col.host, (size_t)col.n * col.width, cudaMemcpyHostToDevice, db->copy_stream);
@@ -919,8 +944,9 @@ ddq_status cache_column_locked(ddq_db* db, int c, bool on_demand, std::unique_lo
   lk.lock();
   col.loading = false;
   db->cache_cv.notify_all();
+  if (stage) cache_unblock(db, stage, pbytes);  // later users are ordered after the unpack on copy_stream
   if (e != cudaSuccess) {
-    cudaFreeAsync(p, db->copy_stream);
+    cache_unblock(db, p, dbytes);
     db->cache_used -= bytes;
     return cuda_status(e, "cache H2D");
   }
@@ -944,7 +970,7 @@ void evict_column_locked(ddq_db* db, int c) {
   }
   cudaSetDevice(db->device);
   cudaDeviceSynchronize();
-  cudaFreeAsync(col.dev, db->copy_stream);
+  cache_unblock(db, col.dev, ((size_t)std::max<int64_t>(col.n, 1) * col.width + 255) / 256 * 256);
   col.dev = nullptr;
   col.evict_pending = false;
   db->cache_used -= (uint64_t)std::max<int64_t>(col.n, 1) * col.width;

@@ -131,6 +131,9 @@ struct ddq_db {
   // threshold = max), so evict + re-cache reuses device memory without a
   // cudaMalloc/cudaFree round trip through the driver per column
   cudaMemPool_t cache_pool = nullptr;
+  // freed cache blocks by exact size (evict + re-cache of the same columns reuses
+  // them without the pool allocator; db->mu guards it)
+  std::multimap<size_t, void*> cache_free;
   ddq::Heap heap;
   std::mutex mu;  // catalog + cache
   std::condition_variable cache_cv;
