@@ -161,12 +161,13 @@ def run_reference(args):
         return
     import datagen  # noqa: F401
     sample = 2_000_000
+    sf = args.sf * max(args.gpus, ws, 1)  # our arm's workload at N GPUs: SF 20 x N (weak scaling)
     vals = []
     for _ in range(args.warmup):
-        cpu_baseline(args.sf, sample)
+        cpu_baseline(sf, sample)
     t_total = 0.0
     for _ in range(args.steps):
-        r = cpu_baseline(args.sf, sample)
+        r = cpu_baseline(sf, sample)
         vals.append(r["value"])
         t_total += 13 * sample / r["value"]
     value = 13 * sample * args.steps / t_total
@@ -174,10 +175,10 @@ def run_reference(args):
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * t_total / args.steps,
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "int64",
             "data": "synthetic (datagen, seed 0x5EED2016)",
-            "config": {"workload": f"SSB SF{args.sf:g}, all 13 queries (bounded sample: first {sample} lineorder "
+            "config": {"workload": f"SSB SF{sf:g}, all 13 queries (bounded sample: first {sample} lineorder "
                                    f"rows per step)", "queries": 13},
             "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle",
-                             "sample": f"first {sample} lineorder rows of SF{args.sf:g} per step"},
+                             "sample": f"first {sample} lineorder rows of SF{sf:g} per step"},
             "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
 
