@@ -196,10 +196,18 @@ def main():
 
     ws, rank, local = dist_env()
     assert ws == args.gpus or ws == 1, "launch N>1 with torchrun --nproc-per-node N"
+    # DDQ_BENCH_BACKEND=gloo (test only): N ranks sharing the visible GPUs (rank ->
+    # GPU local % count), to exercise the exchange and merge on a 1-GPU box
+    backend = os.environ.get("DDQ_BENCH_BACKEND", "nccl")
+    if backend != "nccl":
+        local = local % max(torch.cuda.device_count(), 1)
     torch.cuda.set_device(local)
     if ws > 1:
         import torch.distributed as dist
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        else:
+            dist.init_process_group(backend)
     dws = args.emulate_world if (args.emulate_world and ws == 1) else ws  # ranks the data is sized for
     sf_total = args.sf * dws
     data = datagen.SSB(sf_total)
