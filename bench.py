@@ -44,6 +44,8 @@ def parse():
     ap.add_argument("--sf", type=float, default=SF_PER_GPU, help="scale factor per GPU")
     ap.add_argument("--e2e-steps", type=int, default=5)
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--dump-results", default="",
+                    help="rank 0 writes the 13 (merged) query results of the timed plans as JSON (tests)")
     ap.add_argument("--emulate-world", type=int, default=0,
                     help="diagnostic: size the data for W ranks (dimensions of SF sf*W) and run rank 0's "
                          "lineorder shard on this single process (per-GPU step of a W-GPU weak-scaling run)")
@@ -382,6 +384,9 @@ def main():
     # results of the timed plans (validated against the oracle by tests/, here sanity only)
     results = {q: p.fetch(sptr).rows for q, p in zip(SSB_QUERIES, preps)} if ws == 1 else \
         (merged_results() if rank == 0 else {})
+    if args.dump_results and rank == 0:
+        with open(args.dump_results, "w") as f:
+            json.dump({q: [list(r) for r in rows] for q, rows in results.items()}, f)
 
     # ---- roofline of the dominant kernel class from an event-timed profiling replay
     prof = [p.profile(sptr) for p in preps]
