@@ -229,6 +229,13 @@ __global__ void __launch_bounds__(ws_nw(kIn == 1) * 32, 1) ws_kernel(const __gri
   };
   if (tile < ntiles) fetch(tile);
   uint32_t bits_cnt = 0;  // kOutBits: survivors of this lane
+  // kDefer (a dense semi-join: survivors are positions only): a tile's hit flags
+  // wait for the warp's next tile and both are compacted with ONE scan / claim /
+  // ring accounting (the per-tile compaction was ~60 instructions and three
+  // dependent shared-memory atomics for a handful of survivors)
+  constexpr bool kDefer = kIn == 0 && !kPay && !kCarry && !kOutBits;
+  uint32_t pend = 0, pend_base = 0;
+  bool have_pend = false;  // warp-uniform
 
   for (; tile < ntiles; tile += W) {
     int32_t sv[WS_ITEMS];  // streamed values: keys (dense probe) or TIDs
@@ -364,11 +371,20 @@ __global__ void __launch_bounds__(ws_nw(kIn == 1) * 32, 1) ws_kernel(const __gri
       reinterpret_cast<uint16_t*>(P.out_bits)[(size_t)tile * 32 + lane] = (uint16_t)flags;
       continue;
     }
+    if (kDefer && !have_pend && tile + W < ntiles) {  // hold this tile, compact with the next
+      pend = flags;
+      pend_base = base;
+      have_pend = true;
+      continue;
+    }
     // ---- compaction: warp scan of the lanes' hit counts, one smem claim --------
-    const uint32_t c = __popc(flags);
+    const uint32_t c = __popc(flags) + (kDefer && have_pend ? __popc(pend) : 0u);
     const uint32_t incl = warp_incl_scan(c, (int)lane);
     const uint32_t tot = __shfl_sync(FULL, incl, 31);
-    if (tot == 0) continue;
+    if (tot == 0) {
+      have_pend = false;
+      continue;
+    }
     uint32_t pos0 = 0;
     if (lane == 0) {
       pos0 = atomicAdd(&s_cnt, tot);
@@ -389,6 +405,11 @@ __global__ void __launch_bounds__(ws_nw(kIn == 1) * 32, 1) ws_kernel(const __gri
       // items -- most first probes keep <= 4 % of the rows, where 16 predicated
       // stores per lane and tile were mostly no-ops
       int32_t* wp = ring + r0;
+      if (kDefer && have_pend)
+        for (uint32_t f = pend; f; f &= f - 1) {
+          const uint32_t j = __ffs(f) - 1;
+          *wp++ = (int32_t)(pend_base + (j >> 2) * 128 + (j & 3));
+        }
       for (uint32_t f = flags; f; f &= f - 1) {
         const uint32_t j = __ffs(f) - 1;
         *wp++ = (int32_t)(base + (j >> 2) * 128 + (j & 3));
@@ -422,6 +443,12 @@ __global__ void __launch_bounds__(ws_nw(kIn == 1) * 32, 1) ws_kernel(const __gri
       }
     } else {
       uint32_t p = r0;
+      if (kDefer && have_pend)  // the held tile's positions first (ring wrap)
+        for (uint32_t f = pend; f; f &= f - 1) {
+          const uint32_t j = __ffs(f) - 1;
+          ring[p & (RING - 1)] = (int32_t)(pend_base + (j >> 2) * 128 + (j & 3));
+          p++;
+        }
 #pragma unroll
       for (int j = 0; j < WS_ITEMS; j++) {
         if ((flags >> j) & 1u) {
@@ -452,6 +479,7 @@ __global__ void __launch_bounds__(ws_nw(kIn == 1) * 32, 1) ws_kernel(const __gri
     }
     __threadfence_block();
     __syncwarp();
+    have_pend = false;
     // account the written entries to their blocks; the warp completing a block flushes it
     uint32_t flush = 0;  // bit 0: block b0, bit 1: block b1
     if (lane == 0) {
