@@ -165,13 +165,14 @@ TPCH_COLUMNS = {
     "customer": ["c_custkey", "c_nationkey", "c_mktsegment"],
     "supplier": ["s_suppkey", "s_nationkey"],
     "part": ["p_partkey", "p_retailprice"],
-    "orders": ["o_orderkey", "o_custkey", "o_orderdate", "o_shippriority"],
+    "orders": ["o_orderkey", "o_custkey", "o_orderdate", "o_shippriority", "o_orderpriority"],
     "lineitem": ["l_orderkey", "l_partkey", "l_suppkey", "l_linenumber", "l_quantity",
                  "l_extendedprice", "l_discount", "l_tax", "l_returnflag", "l_linestatus",
                  "l_shipdate", "l_commitdate", "l_receiptdate"],
 }
 TPCH_STRING_COLUMNS = {"n_name": "nation", "r_name": "region", "c_mktsegment": "mktsegment",
-                       "l_returnflag": "returnflag", "l_linestatus": "linestatus"}
+                       "l_returnflag": "returnflag", "l_linestatus": "linestatus",
+                       "o_orderpriority": "orderpriority"}
 
 
 def tpch_rows(table: str, sf: float) -> int:

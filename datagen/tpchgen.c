@@ -22,13 +22,13 @@ enum { R_REGIONKEY = 0, R_NAME };
 enum { HC_CUSTKEY = 0, HC_NATIONKEY, HC_MKTSEGMENT };
 enum { HS_SUPPKEY = 0, HS_NATIONKEY };
 enum { HP_PARTKEY = 0, HP_RETAILPRICE };
-enum { O_ORDERKEY = 0, O_CUSTKEY, O_ORDERDATE, O_SHIPPRIORITY };
+enum { O_ORDERKEY = 0, O_CUSTKEY, O_ORDERDATE, O_SHIPPRIORITY, O_ORDERPRIORITY };
 enum { L_ORDERKEY = 0, L_PARTKEY, L_SUPPKEY, L_LINENUMBER, L_QUANTITY, L_EXTENDEDPRICE,
        L_DISCOUNT, L_TAX, L_RETURNFLAG, L_LINESTATUS, L_SHIPDATE, L_COMMITDATE, L_RECEIPTDATE,
        L_NCOLS };
 enum { DRH_NATION = 1, DRH_SEGMENT = 2, DRH_CUST = 10, DRH_ODATE = 11, DRH_PART = 12, DRH_SUPP = 13,
        DRH_QTY = 14, DRH_DISC = 15, DRH_TAX = 16, DRH_SHIP = 17, DRH_RECEIPT = 18, DRH_COMMIT = 19,
-       DRH_RFLAG = 20 };
+       DRH_RFLAG = 20, DRH_OPRIO = 21 };
 
 #define N_ORDERDATES 2406
 #define CUTOFF_19950617 19950617
@@ -64,7 +64,7 @@ int ddqgen_tpch_width(int table, int col) {
     case TH_CUSTOMER: return (col >= 0 && col <= HC_MKTSEGMENT) ? 4 : 0;
     case TH_SUPPLIER: return (col >= 0 && col <= HS_NATIONKEY) ? 4 : 0;
     case TH_PART: return col == HP_RETAILPRICE ? 8 : col == HP_PARTKEY ? 4 : 0;
-    case TH_ORDERS: return (col >= 0 && col <= O_SHIPPRIORITY) ? 4 : 0;
+    case TH_ORDERS: return (col >= 0 && col <= O_ORDERPRIORITY) ? 4 : 0;
     case TH_LINEITEM:
       if (col < 0 || col >= L_NCOLS) return 0;
       return (col >= L_QUANTITY && col <= L_TAX) ? 8 : 4;
@@ -103,6 +103,8 @@ static void gen_rows_h(uint64_t seed, double sf, int table, int col, int64_t b, 
         else if (col == O_CUSTKEY) o32[k] = (int32_t)(1 + ddqgen_hash(seed, TH_ORDERS, DRH_CUST, (uint64_t)i) % (uint64_t)n_c);
         else if (col == O_ORDERDATE)
           o32[k] = ddqgen_datekey_of_index((int64_t)(ddqgen_hash(seed, TH_ORDERS, DRH_ODATE, (uint64_t)i) % N_ORDERDATES));
+        else if (col == O_ORDERPRIORITY) /* dict "1-URGENT".."5-LOW" (sorted == priority) */
+          o32[k] = (int32_t)(ddqgen_hash(seed, TH_ORDERS, DRH_OPRIO, (uint64_t)i) % 5u);
         else o32[k] = 0;
         break;
       case TH_LINEITEM: {

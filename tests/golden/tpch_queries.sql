@@ -1,4 +1,4 @@
--- TPC-H Q1, Q3, Q5, Q6 with validation parameters (BASELINE config 4; the paper
+-- TPC-H Q1, Q3, Q4, Q5, Q6 with validation parameters (BASELINE config 4; the paper
 -- runs TPC-H, PAPER.md:305, :595).  Texts: SURVEY.md App. A.2, rewritten for the
 -- stored representation ONLY as the DESIGN.md readings require:
 --   O5  decimals are scale-2 integers: (1 - l_discount) -> (100 - l_discount),
@@ -6,7 +6,8 @@
 --       Results are therefore scaled integers (scale 2, 4 or 6).
 --   O11 dates are int yyyymmdd and date arithmetic is folded:
 --       date '1998-12-01' - interval '90' day = 19980902,
---       date '1994-01-01' + interval '1' year = 19950101.
+--       date '1994-01-01' + interval '1' year = 19950101,
+--       date '1993-07-01' + interval '3' month = 19931001.
 --   avg(x) is reported as sum(x) and count(*) (O10: the average is a double
 --   computed at finalisation).  Q1's avg_disc uses sum(l_discount).
 --   LIMIT 10 of Q3 is dropped here so the whole pre-LIMIT group set is compared (O9).
@@ -23,6 +24,11 @@ select l_orderkey, o_orderdate, o_shippriority, sum(l_extendedprice*(100-l_disco
  where c_mktsegment = 'BUILDING' and c_custkey = o_custkey and l_orderkey = o_orderkey
    and o_orderdate < 19950315 and l_shipdate > 19950315
  group by l_orderkey, o_orderdate, o_shippriority order by revenue desc, o_orderdate;
+-- @tpch4
+select o_orderpriority, count(*) as order_count from orders
+ where o_orderdate >= 19930701 and o_orderdate < 19931001
+   and exists (select * from lineitem where l_orderkey = o_orderkey and l_commitdate < l_receiptdate)
+ group by o_orderpriority order by o_orderpriority;
 -- @tpch5
 select n_name, sum(l_extendedprice*(100-l_discount)) as revenue
   from customer, orders, lineitem, supplier, nation, region
