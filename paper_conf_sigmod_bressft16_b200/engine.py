@@ -149,11 +149,18 @@ class PlanBuilder:
         op.n_preds = 0
         return idx
 
-    def filter_eq(self, table: str, input: int, vec_a: int, vec_b: int) -> int:
-        """Keep rows whose aligned vectors vec_a and vec_b are equal."""
+    def filter_eq(self, table: str, input: int, vec_a: int, vec_b: int, cmp: int = A.CMP_EQ) -> int:
+        """Keep rows whose aligned vectors satisfy vec_a == vec_b (cmp=CMP_EQ) or
+        vec_a < vec_b (cmp=CMP_LT)."""
         idx, op = self._op(A.OP_FILTER_EQ, table, input)
         op.eq_vec[0], op.eq_vec[1] = vec_a + 1, vec_b + 1
+        op.eq_cmp = cmp
         return idx
+
+    def filter_lt(self, table: str, input: int, vec_a: int, vec_b: int) -> int:
+        """Keep rows whose aligned vectors satisfy vec_a < vec_b (column-column
+        comparison, e.g. TPC-H Q4's l_commitdate < l_receiptdate)."""
+        return self.filter_eq(table, input, vec_a, vec_b, A.CMP_LT)
 
     def gather(self, table: str, col: str, input: int) -> int:
         idx, op = self._op(A.OP_GATHER, table, input)

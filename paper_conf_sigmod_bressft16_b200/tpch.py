@@ -1,4 +1,4 @@
-"""TPC-H Q1, Q3, Q5, Q6 on libddq (BASELINE config 4; the paper runs TPC-H,
+"""TPC-H Q1, Q3, Q4, Q5, Q6 on libddq (BASELINE config 4; the paper runs TPC-H,
 PAPER.md:305, App. C.2).  Decimals are scale-2 int64 (reading O5); dates
 are int32 yyyymmdd with folded constants (O11).  Query texts: SURVEY.md App. A.2.
 """
@@ -8,21 +8,23 @@ from . import _abi as A
 from .engine import Database, PlanBuilder
 from .ssb import code
 
-TPCH_QUERIES = ["tpch1", "tpch3", "tpch5", "tpch6"]
+TPCH_QUERIES = ["tpch1", "tpch3", "tpch4", "tpch5", "tpch6"]
 
 TABLE_COLUMNS = {
     "nation": ["n_nationkey", "n_name", "n_regionkey"],
     "region": ["r_regionkey", "r_name"],
     "customer": ["c_custkey", "c_nationkey", "c_mktsegment"],
     "supplier": ["s_suppkey", "s_nationkey"],
-    "orders": ["o_orderkey", "o_custkey", "o_orderdate", "o_shippriority"],
+    "orders": ["o_orderkey", "o_custkey", "o_orderdate", "o_shippriority", "o_orderpriority"],
     "lineitem": ["l_orderkey", "l_suppkey", "l_quantity", "l_extendedprice", "l_discount", "l_tax",
-                 "l_returnflag", "l_linestatus", "l_shipdate"],
+                 "l_returnflag", "l_linestatus", "l_shipdate", "l_commitdate", "l_receiptdate"],
 }
 STRING_DICTS = {"n_name": "nation", "r_name": "region", "c_mktsegment": "mktsegment",
-                "l_returnflag": "returnflag", "l_linestatus": "linestatus"}
+                "l_returnflag": "returnflag", "l_linestatus": "linestatus",
+                "o_orderpriority": "orderpriority"}
 QUERY_TABLES = {"tpch1": ["lineitem"], "tpch6": ["lineitem"],
                 "tpch3": ["customer", "orders", "lineitem"],
+                "tpch4": ["orders", "lineitem"],
                 "tpch5": ["region", "nation", "supplier", "customer", "orders", "lineitem"]}
 
 
@@ -79,6 +81,21 @@ def tpch_plan(db: Database, q: str, limit: int = 0, dense: bool = True) -> PlanB
         P.aggregate(li, t, keys=["l_orderkey", 0, 1], key_bits=[28, 25, 10],
                     aggs=[(A.AGG_SUM_MUL_100M, ["l_extendedprice", "l_discount"])],
                     order_by=[-101, 2, 1], max_groups=1 << 22, limit=limit)
+        return P
+    if q == "tpch4":
+        # EXISTS (lineitem of the order with l_commitdate < l_receiptdate) is a
+        # semi-join: the late lineitems of the quarter's orders build a join index
+        # over l_orderkey (duplicates collapse into one bit), the orders probe it.
+        o = P.select("orders", [("o_orderdate", 19930701, 19930930)])    # [1993-07-01, 1993-10-01)
+        ho = P.build("orders", "o_orderkey", input=o)
+        t = P.probe(li, "l_orderkey", ho)                                # lineitems of those orders
+        t = P.gather(li, "l_commitdate", t)                              # vec0
+        t = P.gather(li, "l_receiptdate", t)                             # vec1
+        t = P.filter_lt(li, t, 0, 1)                                     # l_commitdate < l_receiptdate
+        hl = P.build(li, "l_orderkey", input=t)
+        o = P.probe("orders", "o_orderkey", hl, input=o)
+        P.aggregate("orders", o, keys=["o_orderpriority"], aggs=[(A.AGG_COUNT, [])],
+                    order_by=[1], max_groups=5, key_bits=[3])  # codes sorted == string order (O4)
         return P
     if q == "tpch5":
         r = P.select("region", [("r_name", [code(db, "region", "ASIA")])])
