@@ -14,7 +14,7 @@ Parity status per function:
                      on planted tables, group-count / sum-conservation invariants
   listing1..8        pinned: closed form (empty by the SSB value domains), brute force
   listing2b          pinned: numpy.flatnonzero of the predicate, binomial bounds
-  tpch1,3,4,5,6      pinned: SQLite 3.45 on decoded tables (tpch4: EXISTS subquery)
+  tpch1,3,4,5,6,7    pinned: SQLite 3.45 on decoded tables (tpch4: EXISTS subquery)
 """
 from __future__ import annotations
 
@@ -98,6 +98,11 @@ TPCH_QUERY_COLUMNS = {
     4: [("orders", "o_orderkey"), ("orders", "o_orderdate"), ("orders", "o_orderpriority"),
         ("lineitem", "l_orderkey"), ("lineitem", "l_commitdate"), ("lineitem", "l_receiptdate")],
     6: [("lineitem", c) for c in ["l_shipdate", "l_discount", "l_quantity", "l_extendedprice"]],
+    7: [("nation", "n_nationkey"), ("nation", "n_name"), ("supplier", "s_suppkey"),
+        ("supplier", "s_nationkey"), ("customer", "c_custkey"), ("customer", "c_nationkey"),
+        ("orders", "o_orderkey"), ("orders", "o_custkey"), ("lineitem", "l_orderkey"),
+        ("lineitem", "l_suppkey"), ("lineitem", "l_shipdate"), ("lineitem", "l_extendedprice"),
+        ("lineitem", "l_discount")],
 }
 
 
@@ -179,7 +184,7 @@ def ssb_db(db: "datagen.SSB", query: str, fact_rows: int | None = None) -> Oracl
 
 def run(db, query: str, fact_rows: int | None = None):
     """Evaluate `query` ("ssb1.1".."ssb4.3", "listing1".."listing8", "listing2b",
-    "tpch1", "tpch3", "tpch4", "tpch5", "tpch6") on a datagen database."""
+    "tpch1", "tpch3", "tpch4", "tpch5", "tpch6", "tpch7") on a datagen database."""
     if query.startswith("tpch"):
         odb = OracleDB()
         _set_dicts(odb)

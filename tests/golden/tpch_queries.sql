@@ -1,4 +1,4 @@
--- TPC-H Q1, Q3, Q4, Q5, Q6 with validation parameters (BASELINE config 4; the paper
+-- TPC-H Q1, Q3, Q4, Q5, Q6, Q7 with validation parameters (BASELINE config 4; the paper
 -- runs TPC-H, PAPER.md:305, :595).  Texts: SURVEY.md App. A.2, rewritten for the
 -- stored representation ONLY as the DESIGN.md readings require:
 --   O5  decimals are scale-2 integers: (1 - l_discount) -> (100 - l_discount),
@@ -7,7 +7,8 @@
 --   O11 dates are int yyyymmdd and date arithmetic is folded:
 --       date '1998-12-01' - interval '90' day = 19980902,
 --       date '1994-01-01' + interval '1' year = 19950101,
---       date '1993-07-01' + interval '3' month = 19931001.
+--       date '1993-07-01' + interval '3' month = 19931001,
+--       extract(year from l_shipdate) = l_shipdate / 10000.
 --   avg(x) is reported as sum(x) and count(*) (O10: the average is a double
 --   computed at finalisation).  Q1's avg_disc uses sum(l_discount).
 --   LIMIT 10 of Q3 is dropped here so the whole pre-LIMIT group set is compared (O9).
@@ -40,3 +41,12 @@ select n_name, sum(l_extendedprice*(100-l_discount)) as revenue
 select sum(l_extendedprice*l_discount) as revenue, count(*) from lineitem
  where l_shipdate >= 19940101 and l_shipdate < 19950101
    and l_discount between 5 and 7 and l_quantity < 2400;
+-- @tpch7
+select n1.n_name as supp_nation, n2.n_name as cust_nation, l_shipdate / 10000 as l_year,
+       sum(l_extendedprice*(100-l_discount)) as revenue
+  from supplier, lineitem, orders, customer, nation n1, nation n2
+ where s_suppkey = l_suppkey and o_orderkey = l_orderkey and c_custkey = o_custkey
+   and s_nationkey = n1.n_nationkey and c_nationkey = n2.n_nationkey
+   and ((n1.n_name = 'FRANCE' and n2.n_name = 'GERMANY') or (n1.n_name = 'GERMANY' and n2.n_name = 'FRANCE'))
+   and l_shipdate between 19950101 and 19961231
+ group by supp_nation, cust_nation, l_year order by supp_nation, cust_nation, l_year;

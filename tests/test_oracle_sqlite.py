@@ -98,6 +98,9 @@ def tpch_to_sql(q, rows):
     if q == "tpch4":
         pr = datagen.dictionary("orderpriority")
         return [(pr[r[0]], r[1]) for r in rows]
+    if q == "tpch7":
+        nat = datagen.dictionary("nation")
+        return [(nat[r[0]], nat[r[1]]) + tuple(r[2:]) for r in rows]
     if q == "tpch5":
         nat = datagen.dictionary("nation")
         return [(nat[r[0]], r[1]) for r in rows]
@@ -106,7 +109,7 @@ def tpch_to_sql(q, rows):
     return [tuple(r) for r in rows]
 
 
-@pytest.mark.parametrize("q", ["tpch1", "tpch3", "tpch4", "tpch5", "tpch6"])
+@pytest.mark.parametrize("q", ["tpch1", "tpch3", "tpch4", "tpch5", "tpch6", "tpch7"])
 def test_tpch_oracle_equals_sqlite(q):
     db, con = _tpch(0.01)
     want = [tuple(r) for r in con.execute(load_sql("tpch_queries.sql")[q]).fetchall()]
@@ -117,5 +120,5 @@ def test_tpch_oracle_equals_sqlite(q):
         assert [(r[3], r[1]) for r in got] == [(r[3], r[1]) for r in want]
     if q == "tpch5":
         assert [r[1] for r in got] == [r[1] for r in want]
-    if q == "tpch4":  # order by o_orderpriority (decoded string)
+    if q in ("tpch4", "tpch7"):  # order by decoded strings (and l_year)
         assert got == want
