@@ -365,12 +365,14 @@ typedef struct {
   int32_t fetch_build;
   /* FILTER_EQ comparison: DDQ_CMP_EQ (0, default) keeps rows with vec_a == vec_b,
      DDQ_CMP_LT keeps rows with vec_a < vec_b (signed int32; TPC-H Q4's
-     l_commitdate < l_receiptdate).  Other values: DDQ_EINVAL. */
+     l_commitdate < l_receiptdate), DDQ_CMP_NE keeps vec_a != vec_b (TPC-H Q7's
+     pair of distinct nations).  Other values: DDQ_EINVAL. */
   int32_t eq_cmp;
 } ddq_op;
 
 #define DDQ_CMP_EQ 0
 #define DDQ_CMP_LT 1
+#define DDQ_CMP_NE 2
 
 #define DDQ_MAX_OPS 32
 typedef struct {

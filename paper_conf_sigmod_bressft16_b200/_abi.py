@@ -19,7 +19,7 @@ STATUS = {0: "DDQ_OK", -1: "DDQ_EINVAL", -2: "DDQ_ENOTFOUND", -3: "DDQ_ENOMEM_HO
 
 PRED_RANGE, PRED_IN = 1, 2
 MAX_IN, MAX_PREDS, MAX_CARRY, MAX_AGGS, MAX_KEYS, MAX_OPS = 8, 4, 4, 8, 3, 32
-CMP_EQ, CMP_LT = 0, 1  # FILTER_EQ comparison (ddq_op.eq_cmp)
+CMP_EQ, CMP_LT, CMP_NE = 0, 1, 2  # FILTER_EQ comparison (ddq_op.eq_cmp)
 OP_SELECT, OP_HASH_BUILD, OP_HASH_PROBE, OP_GATHER, OP_AGGREGATE, OP_FILTER_EQ, OP_STAR = 1, 2, 3, 4, 5, 6, 7
 TERM_PRED, TERM_PROBE = 1, 2
 AGG_COUNT, AGG_SUM, AGG_SUM_MUL, AGG_SUM_SUB, AGG_SUM_MUL_100M, AGG_SUM_MUL_100M_100P = 1, 2, 3, 4, 5, 6

@@ -85,7 +85,7 @@ struct WsParams {
   WsPred preds[4];
   const int32_t* eq_a;
   const int32_t* eq_b;
-  int eq_lt;  // FILTER_EQ comparison: 0 keep a == b, 1 keep a < b (DDQ_CMP_LT)
+  int eq_cmp;  // FILTER_EQ comparison: 0 a == b, 1 a < b, 2 a != b (DDQ_CMP_*)
   const int32_t* fk;  // probe keys: column (by row) or positional vector (fk_by_pos)
   int32_t fk_by_pos;
   // join index (direct): membership bitmap over [key_min, key_min + range) + payloads
@@ -333,7 +333,7 @@ __global__ void __launch_bounds__(ws_nw(kIn == 1) * 32, 1) ws_kernel(const __gri
       unpack16(b4, b);
       uint32_t m = 0;
 #pragma unroll
-      for (int j = 0; j < WS_ITEMS; j++) m |= ((P.eq_lt ? a[j] < b[j] : a[j] == b[j]) ? 1u : 0u) << j;
+      for (int j = 0; j < WS_ITEMS; j++) m |= (vec_cmp(P.eq_cmp, a[j], b[j]) ? 1u : 0u) << j;
       flags &= m;
     } else {  // selection at TIDs: later columns gathered for the remaining rows only
       for (int p = 0; p < P.n_preds; p++) {
@@ -704,7 +704,7 @@ cudaError_t launch_ws(const FilterArgs& a, cudaStream_t st) {
     kind = WK_EQ;
     p.eq_a = a.eq_a;
     p.eq_b = a.eq_b;
-    p.eq_lt = a.eq_lt ? 1 : 0;
+    p.eq_cmp = a.eq_cmp;
   } else {
     bool all_range = true;
     p.n_preds = a.n_preds;

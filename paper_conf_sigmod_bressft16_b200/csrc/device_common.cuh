@@ -10,6 +10,12 @@ constexpr unsigned FULL = 0xffffffffu;
 
 // ---- loads ---------------------------------------------------------------
 // Streaming 128-bit loads that do not allocate in L1 (each column byte is read once).
+// FILTER_EQ comparison of two aligned int32 vector entries (ddq_op.eq_cmp:
+// DDQ_CMP_EQ 0, DDQ_CMP_LT 1, DDQ_CMP_NE 2).
+__device__ __forceinline__ bool vec_cmp(int cmp, int32_t a, int32_t b) {
+  return cmp == 1 ? a < b : cmp == 2 ? a != b : a == b;
+}
+
 __device__ __forceinline__ int4 ld_stream_i4(const void* p) {
   int4 r;
   asm volatile("ld.global.nc.L1::no_allocate.v4.s32 {%0,%1,%2,%3}, [%4];"

@@ -393,7 +393,7 @@ ddq_status run_host_op(ddq_db* db, const ddq_op& op, const std::vector<Inter>& I
           return set_error(DDQ_EINVAL, "filter_eq: bad vector indexes");
         eqa = (const int32_t*)in->vecs[(size_t)a].ptr;
         eqb = (const int32_t*)in->vecs[(size_t)b].ptr;
-        if (op.eq_cmp != DDQ_CMP_EQ && op.eq_cmp != DDQ_CMP_LT) return set_error(DDQ_EINVAL, "filter_eq: bad eq_cmp");
+        if (op.eq_cmp < DDQ_CMP_EQ || op.eq_cmp > DDQ_CMP_NE) return set_error(DDQ_EINVAL, "filter_eq: bad eq_cmp");
       }
       const Column* fk = (probe && op.fk_vec <= 0) ? col_of(db, op.fk_col) : nullptr;
       const int32_t* fkv = (probe && op.fk_vec > 0) ? (const int32_t*)in->vecs[(size_t)op.fk_vec - 1].ptr : nullptr;
@@ -412,7 +412,9 @@ ddq_status run_host_op(ddq_db* db, const ddq_op& op, const std::vector<Inter>& I
           int32_t r = row_of(i);
           bool ok = true;
           if (eqa) {
-            if (op.eq_cmp == DDQ_CMP_LT ? eqa[i] < eqb[i] : eqa[i] == eqb[i]) S.push_back(i);
+            const bool keep = op.eq_cmp == DDQ_CMP_LT ? eqa[i] < eqb[i]
+                            : op.eq_cmp == DDQ_CMP_NE ? eqa[i] != eqb[i] : eqa[i] == eqb[i];
+            if (keep) S.push_back(i);
           } else if (!probe) {
             for (int p = 0; p < op.n_preds && ok; p++) {
               int64_t v = hcol(pc[(size_t)p], r);

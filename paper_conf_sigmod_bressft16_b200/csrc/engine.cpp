@@ -187,7 +187,7 @@ ddq_status run_gpu_op(GpuOpCtx& ctx, const ddq_op& op, Inter& out) {
           return set_error(DDQ_EINVAL, "filter_eq: bad vector indexes");
         eq_a = (const int32_t*)in->vecs[(size_t)a].ptr;
         eq_b = (const int32_t*)in->vecs[(size_t)b].ptr;
-        if (op.eq_cmp != DDQ_CMP_EQ && op.eq_cmp != DDQ_CMP_LT) return set_error(DDQ_EINVAL, "filter_eq: bad eq_cmp");
+        if (op.eq_cmp < DDQ_CMP_EQ || op.eq_cmp > DDQ_CMP_NE) return set_error(DDQ_EINVAL, "filter_eq: bad eq_cmp");
       } else if (!probe) {
         if (op.n_preds < 0 || op.n_preds > DDQ_MAX_PREDS) return set_error(DDQ_EINVAL, "select: bad n_preds");
         for (int i = 0; i < op.n_preds; i++) {
@@ -270,7 +270,7 @@ ddq_status run_gpu_op(GpuOpCtx& ctx, const ddq_op& op, Inter& out) {
       }
       fa.eq_a = eq_a;
       fa.eq_b = eq_b;
-      fa.eq_lt = op.kind == DDQ_OP_FILTER_EQ && op.eq_cmp == DDQ_CMP_LT;
+      fa.eq_cmp = op.kind == DDQ_OP_FILTER_EQ ? op.eq_cmp : DDQ_CMP_EQ;
       fa.in_tids = in_tids;
       fa.d_in_count = in_cnt;
       fa.n_cap = in_cap;

@@ -53,7 +53,7 @@ struct FilterParams {
   int32_t fk_by_pos;    // probe keys are an aligned vector (fk[i]), not a column (fk[row])
   const int32_t* eq_a;  // FILTER_EQ vectors (positional), or null
   const int32_t* eq_b;
-  int eq_lt;            // FILTER_EQ comparison: 0 keep a == b, 1 keep a < b
+  int eq_cmp;  // FILTER_EQ comparison: 0 a == b, 1 a < b, 2 a != b (DDQ_CMP_*)
   int32_t direct;  // direct-mapped join index instead of the hash table
   const uint32_t* bitmap;
   const int32_t* payarr;
@@ -174,7 +174,7 @@ filter_kernel(const __grid_constant__ FilterParams P) {
           const int64_t pos = wbase + (k >> 2) * 128 + lane * 4 + (k & 3);
           if ((flags >> k) & 1u) {
             const int32_t va = __ldg(P.eq_a + pos), vb = __ldg(P.eq_b + pos);
-            if (P.eq_lt ? !(va < vb) : va != vb) flags &= ~(1u << k);
+            if (!vec_cmp(P.eq_cmp, va, vb)) flags &= ~(1u << k);
           }
         }
       }
@@ -359,7 +359,7 @@ cudaError_t launch_filter(const FilterArgs& a, cudaStream_t st) {
   p.fk_by_pos = a.fk_by_pos ? 1 : 0;
   p.eq_a = a.eq_a;
   p.eq_b = a.eq_b;
-  p.eq_lt = a.eq_lt ? 1 : 0;
+  p.eq_cmp = a.eq_cmp;
   p.direct = a.bitmap != nullptr;
   p.bitmap = a.bitmap;
   p.payarr = a.payarr;

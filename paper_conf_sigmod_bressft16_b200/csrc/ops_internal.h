@@ -40,7 +40,7 @@ struct FilterArgs {
   bool fk_by_pos = false;          // probe keys from an aligned vector (TID inputs)
   const int32_t* eq_a = nullptr;   // FILTER_EQ positional vectors (TID inputs)
   const int32_t* eq_b = nullptr;
-  bool eq_lt = false;              // FILTER_EQ with DDQ_CMP_LT: keep eq_a < eq_b
+  int eq_cmp = 0;                  // FILTER_EQ comparison: DDQ_CMP_EQ / _LT / _NE
   const uint64_t* table = nullptr;
   uint32_t capacity = 0;
   // direct-mapped join index (probe): bitmap + payload array over [key_min, key_min+range)

@@ -81,7 +81,7 @@ struct ScanParams {
   ScanPred preds[SC_MAXCOLS];
   const int32_t* eq_a;  // FILTER_EQ (positional vectors)
   const int32_t* eq_b;
-  int eq_lt;  // FILTER_EQ comparison: 0 keep a == b, 1 keep a < b
+  int eq_cmp;  // FILTER_EQ comparison: 0 a == b, 1 a < b, 2 a != b (DDQ_CMP_*)
   // probe
   int32_t probe;
   const int32_t* fk;  // probe keys: column (indexed by row) or vector (by position)
@@ -366,7 +366,7 @@ __global__ void __launch_bounds__(SC_GT* G, 1) scan_kernel(const __grid_constant
             for (int k2 = 0; k2 < SC_ITEMS; k2++) {
               const uint32_t pos = row0 + wrow + (k2 >> 2) * 128 + lane * 4 + (k2 & 3);
               const int32_t va = __ldg(P.eq_a + pos), vb = __ldg(P.eq_b + pos);
-              m |= (((flags >> k2) & 1u) && (P.eq_lt ? va < vb : va == vb) ? 1u : 0u) << k2;
+              m |= (((flags >> k2) & 1u) && vec_cmp(P.eq_cmp, va, vb) ? 1u : 0u) << k2;
             }
             flags &= m;
           }
@@ -619,7 +619,7 @@ cudaError_t launch_scan(const FilterArgs& a, cudaStream_t st) {
   }
   p.eq_a = a.eq_a;
   p.eq_b = a.eq_b;
-  p.eq_lt = a.eq_lt ? 1 : 0;
+  p.eq_cmp = a.eq_cmp;
   p.stage_bytes = off;
   p.probe = a.probe ? 1 : 0;
   p.fk = a.fk;

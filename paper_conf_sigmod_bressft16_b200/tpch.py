@@ -1,4 +1,4 @@
-"""TPC-H Q1, Q3, Q4, Q5, Q6 on libddq (BASELINE config 4; the paper runs TPC-H,
+"""TPC-H Q1, Q3, Q4, Q5, Q6, Q7 on libddq (BASELINE config 4; the paper runs TPC-H,
 PAPER.md:305, App. C.2).  Decimals are scale-2 int64 (reading O5); dates
 are int32 yyyymmdd with folded constants (O11).  Query texts: SURVEY.md App. A.2.
 """
@@ -8,7 +8,9 @@ from . import _abi as A
 from .engine import Database, PlanBuilder
 from .ssb import code
 
-TPCH_QUERIES = ["tpch1", "tpch3", "tpch4", "tpch5", "tpch6"]
+import numpy as np
+
+TPCH_QUERIES = ["tpch1", "tpch3", "tpch4", "tpch5", "tpch6", "tpch7"]
 
 TABLE_COLUMNS = {
     "nation": ["n_nationkey", "n_name", "n_regionkey"],
@@ -25,15 +27,29 @@ STRING_DICTS = {"n_name": "nation", "r_name": "region", "c_mktsegment": "mktsegm
 QUERY_TABLES = {"tpch1": ["lineitem"], "tpch6": ["lineitem"],
                 "tpch3": ["customer", "orders", "lineitem"],
                 "tpch4": ["orders", "lineitem"],
+                "tpch7": ["nation", "supplier", "customer", "orders", "lineitem", "calendar"],
                 "tpch5": ["region", "nation", "supplier", "customer", "orders", "lineitem"]}
+
+
+def calendar_table() -> dict:
+    """The date dimension (one row per day 1992-01-01 .. 1998-12-31, TPC-H's date
+    domain): d_datekey (int yyyymmdd, reading O11) and d_year.  extract(year from
+    l_shipdate) of Q7 is a join of l_shipdate with it (reading O36), as SSB's
+    lo_orderdate joins its date table."""
+    days = np.arange(np.datetime64("1992-01-01"), np.datetime64("1999-01-01"))
+    y = days.astype("datetime64[Y]").astype(np.int64) + 1970
+    m = days.astype("datetime64[M]").astype(np.int64) % 12 + 1
+    d = (days - days.astype("datetime64[M]")).astype(np.int64) + 1
+    return {"d_datekey": (y * 10000 + m * 100 + d).astype(np.int32), "d_year": y.astype(np.int32)}
 
 
 def load_tpch(db: Database, data, cache: bool = True, tables=None) -> None:
     """data: ``data.col(table, col)``, ``data.rows(table)``, ``data.dict_for(col)``."""
-    for t in (tables or TABLE_COLUMNS):
-        db.create_table(t, data.rows(t))
-        for c in TABLE_COLUMNS[t]:
-            db.load_column(t, c, data.col(t, c))
+    for t in (tables or list(TABLE_COLUMNS) + ["calendar"]):
+        cols = calendar_table() if t == "calendar" else {c: data.col(t, c) for c in TABLE_COLUMNS[t]}
+        db.create_table(t, len(next(iter(cols.values()))))
+        for c, v in cols.items():
+            db.load_column(t, c, v)
             if cache:
                 db.cache(t, c)
     for c, d in STRING_DICTS.items():
@@ -114,5 +130,29 @@ def tpch_plan(db: Database, q: str, limit: int = 0, dense: bool = True) -> PlanB
         t = P.probe(li, 1, hn, input=t, emit=True)                       # vec3 = n_name
         P.aggregate(li, t, keys=[3], aggs=[(A.AGG_SUM_MUL_100M, ["l_extendedprice", "l_discount"])],
                     order_by=[-101, 1], max_groups=25)
+        return P
+    if q == "tpch7":
+        n = P.select("nation", [("n_name", [code(db, "nation", "FRANCE"), code(db, "nation", "GERMANY")])])
+        hn = P.build("nation", "n_nationkey", "n_name", input=n)
+        s = P.probe("supplier", "s_nationkey", hn)
+        hs = P.build("supplier", "s_suppkey", "s_nationkey", input=s)
+        c = P.probe("customer", "c_nationkey", hn)
+        hc = P.build("customer", "c_custkey", "c_nationkey", input=c)
+        o = P.probe("orders", "o_custkey", hc)                           # orders of FR/DE customers
+        ho = P.build("orders", "o_orderkey", "o_custkey", input=o)
+        hy = P.build("calendar", "d_datekey", "d_year")
+        t = P.select(li, [("l_shipdate", 19950101, 19961231)])
+        t = P.probe(li, "l_suppkey", hs, input=t, emit=True)             # vec0 = s_nationkey
+        t = P.probe(li, "l_orderkey", ho, input=t, emit=True)            # vec1 = o_custkey
+        t = P.probe(li, 1, hc, input=t, emit=True)                       # vec2 = c_nationkey
+        # (n1 = FRANCE and n2 = GERMANY) or (n1 = GERMANY and n2 = FRANCE), both
+        # nations already restricted to {FRANCE, GERMANY}: s_nationkey != c_nationkey
+        t = P.filter_eq(li, t, 0, 2, A.CMP_NE)
+        t = P.probe(li, 0, hn, input=t, emit=True)                       # vec3 = supp_nation
+        t = P.probe(li, 2, hn, input=t, emit=True)                       # vec4 = cust_nation
+        t = P.fetch(li, "l_shipdate", hy, t)                             # vec5 = l_year
+        P.aggregate(li, t, keys=[3, 4, 5], key_bits=[5, 5, 12],
+                    aggs=[(A.AGG_SUM_MUL_100M, ["l_extendedprice", "l_discount"])],
+                    order_by=[1, 2, 3], max_groups=64)
         return P
     raise KeyError(q)

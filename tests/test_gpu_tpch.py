@@ -1,4 +1,4 @@
-"""TPC-H Q1/Q3/Q4/Q5/Q6 parity (BASELINE config 4): libddq through the C ABI vs the
+"""TPC-H Q1/Q3/Q4/Q5/Q6/Q7 parity (BASELINE config 4): libddq through the C ABI vs the
 oracle, exact (scale-2 decimals as int64, int128 sums), prepared CUDA-graph plans
 and the chopping driver, plus the cold path (GPU-only placement on an empty cache:
 every column copied from pinned host memory)."""
@@ -33,7 +33,7 @@ def _want(q):
     return [tuple(r) for r in oracle.run(_data(), q)]
 
 
-@pytest.mark.parametrize("q", ["tpch1", "tpch3", "tpch4", "tpch5", "tpch6"])
+@pytest.mark.parametrize("q", ["tpch1", "tpch3", "tpch4", "tpch5", "tpch6", "tpch7"])
 def test_tpch_prepared_equals_oracle(q):
     from paper_conf_sigmod_bressft16_b200.tpch import tpch_plan
     db = _db()
@@ -44,7 +44,7 @@ def test_tpch_prepared_equals_oracle(q):
     assert got and got == _want(q)
 
 
-@pytest.mark.parametrize("q", ["tpch1", "tpch3", "tpch4", "tpch5", "tpch6"])
+@pytest.mark.parametrize("q", ["tpch1", "tpch3", "tpch4", "tpch5", "tpch6", "tpch7"])
 def test_tpch_submit_equals_oracle(q):
     from paper_conf_sigmod_bressft16_b200.tpch import tpch_plan
     db = _db()
@@ -65,7 +65,7 @@ def test_tpch_cold_path_gpu_only():
     from paper_conf_sigmod_bressft16_b200.tpch import load_tpch, tpch_plan
     db = Database(cache_bytes=8 << 30, heap_bytes=4 << 30, placement=A.PLACE_GPU_ONLY)
     load_tpch(db, _data(), cache=False)
-    for q in ("tpch1", "tpch6", "tpch5", "tpch4"):
+    for q in ("tpch1", "tpch6", "tpch5", "tpch4", "tpch7"):
         r = db.run(tpch_plan(db, q))
         assert r.rows == _want(q) and r.host_ops == 0
     st = db.stats()
@@ -163,20 +163,22 @@ def test_dense_aggregate_int64_overflow_is_exact(n):
     assert [tuple(r) for r in got] == want
 
 
-def test_tpch4_cpu_only_host_operators():
-    """CPU-only placement: every operator of Q4 (incl. the FILTER_EQ with
-    CMP_LT and the lineitem-side semi-join build) runs in the host executor."""
+@pytest.mark.parametrize("q", ["tpch4", "tpch7"])
+def test_tpch_cpu_only_host_operators(q):
+    """CPU-only placement: every operator of Q4 / Q7 (incl. FILTER_EQ with CMP_LT /
+    CMP_NE, the lineitem-side semi-join build, the calendar fetch) runs in the
+    host executor."""
     from paper_conf_sigmod_bressft16_b200 import Database
     from paper_conf_sigmod_bressft16_b200 import _abi as A
     from paper_conf_sigmod_bressft16_b200.tpch import load_tpch, tpch_plan
     db = Database(cache_bytes=1 << 30, heap_bytes=1 << 30, placement=A.PLACE_CPU_ONLY)
-    load_tpch(db, _data(), cache=False, tables=["orders", "lineitem"])
-    r = db.run(tpch_plan(db, "tpch4"))
-    assert r.rows == _want("tpch4") and r.host_ops > 0
+    load_tpch(db, _data(), cache=False)
+    r = db.run(tpch_plan(db, q))
+    assert r.rows == _want(q) and r.host_ops > 0
     db.close()
 
 
-@pytest.mark.parametrize("cmp", ["eq", "lt"])
+@pytest.mark.parametrize("cmp", ["eq", "lt", "ne"])
 def test_filter_compare_vectors_at_tids(cmp):
     """FILTER_EQ over two gathered int32 vectors (CMP_EQ / CMP_LT, negative values,
     ragged tail) vs numpy: the kept TIDs and a count aggregate at them."""
@@ -198,10 +200,10 @@ def test_filter_compare_vectors_at_tids(cmp):
     t = P.select("t", [("s", 0, 6)])
     t = P.gather("t", "a", t)
     t = P.gather("t", "b", t)
-    t = P.filter_eq("t", t, 0, 1, A.CMP_LT if cmp == "lt" else A.CMP_EQ)
+    t = P.filter_eq("t", t, 0, 1, {"eq": A.CMP_EQ, "lt": A.CMP_LT, "ne": A.CMP_NE}[cmp])
     P.aggregate("t", t, keys=["g"], key_bits=[2], aggs=[(A.AGG_COUNT, []), (A.AGG_SUM, ["a"])],
                 order_by=[1], max_groups=4)
-    m = (s <= 6) & ((a < b) if cmp == "lt" else (a == b))
+    m = (s <= 6) & {"eq": a == b, "lt": a < b, "ne": a != b}[cmp]
     want = [(k, int((m & (g == k)).sum()), int(a[m & (g == k)].astype(np.int64).sum())) for k in range(4)]
     r = db.run(P)
     p = db.prepare(P)
