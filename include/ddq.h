@@ -368,6 +368,11 @@ typedef struct {
      l_commitdate < l_receiptdate), DDQ_CMP_NE keeps vec_a != vec_b (TPC-H Q7's
      pair of distinct nations).  Other values: DDQ_EINVAL. */
   int32_t eq_cmp;
+  /* HASH_BUILD: 1 = the build is a key SET for a semi-join (EXISTS / IN subquery,
+     TPC-H Q4): duplicate keys are allowed and collapse into one entry whose
+     payload is any one of their rows; 0 (default) = unique keys, a duplicate is
+     DDQ_EINVAL (reading O13). */
+  int32_t build_key_set;
 } ddq_op;
 
 #define DDQ_CMP_EQ 0

@@ -67,7 +67,8 @@ class Op(ctypes.Structure):
                 ("eq_vec", ctypes.c_int32 * 2), ("n_terms", ctypes.c_int32),
                 ("term_kind", ctypes.c_int32 * 4), ("term_build", ctypes.c_int32 * 4),
                 ("term_fk", ctypes.c_int32 * 4), ("term_emit", ctypes.c_int32 * 4),
-                ("fetch_build", ctypes.c_int32), ("eq_cmp", ctypes.c_int32)]
+                ("fetch_build", ctypes.c_int32), ("eq_cmp", ctypes.c_int32),
+                ("build_key_set", ctypes.c_int32)]
 
 
 class DevTerm(ctypes.Structure):

@@ -501,11 +501,16 @@ ddq_status run_host_op(ddq_db* db, const ddq_op& op, const std::vector<Inter>& I
         int32_t k = ((const int32_t*)kc->host)[r];
         int32_t v = pc ? ((const int32_t*)pc->host)[r] : r;
         uint32_t h = host_hash32(k, 32 - lg);
+        bool dup = false;
         while ((*t)[h] != kHostEmpty) {
-          if ((int32_t)((*t)[h] >> 32) == k) return set_error(DDQ_EINVAL, "duplicate build key");
+          if ((int32_t)((*t)[h] >> 32) == k) {
+            if (!op.build_key_set) return set_error(DDQ_EINVAL, "duplicate build key");
+            dup = true;  // key set (semi-join): the first row stays
+            break;
+          }
           h = (h + 1) & (uint32_t)(cap - 1);
         }
-        (*t)[h] = ((uint64_t)(uint32_t)k << 32) | (uint32_t)v;
+        if (!dup) (*t)[h] = ((uint64_t)(uint32_t)k << 32) | (uint32_t)v;
       }
       out.host_table = t;
       out.table_cap = (uint32_t)cap;

@@ -370,6 +370,7 @@ ddq_status run_gpu_op(GpuOpCtx& ctx, const ddq_op& op, Inter& out) {
       if (op.n_preds < 0 || op.n_preds > DDQ_MAX_PREDS) return set_error(DDQ_EINVAL, "build: bad n_preds");
       BuildPreds bp;
       bp.n = op.n_preds;
+      bp.key_set = op.build_key_set ? 1 : 0;
       for (int i = 0; i < op.n_preds; i++) {
         const ddq_pred& p = op.preds[i];
         const Column* c = col_of(db, p.column);

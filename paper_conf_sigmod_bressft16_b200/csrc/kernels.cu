@@ -76,8 +76,8 @@ __global__ void hash_build_kernel(const int32_t* __restrict__ keys, const int32_
       unsigned long long old = atomicCAS(reinterpret_cast<unsigned long long*>(table + h),
                                          (unsigned long long)HT_EMPTY, (unsigned long long)slot);
       if (old == HT_EMPTY) break;
-      if (ht_key(old) == k) {  // PKs must be unique (reading O13)
-        atomicMax(d_error, 1u);
+      if (ht_key(old) == k) {  // PKs must be unique (reading O13) unless a key set
+        if (!bp.key_set) atomicMax(d_error, 1u);
         break;
       }
       h = (h + 1) & mask;
@@ -208,7 +208,7 @@ __global__ void join_index_build_kernel(const int32_t* __restrict__ keys, const 
       continue;
     }
     const uint32_t old = atomicOr(bitmap + (o >> 5), 1u << (o & 31));
-    if (old & (1u << (o & 31))) atomicMax(d_error, 1u);  // PKs are unique (O13)
+    if ((old & (1u << (o & 31))) && !bp.key_set) atomicMax(d_error, 1u);  // PKs are unique (O13)
     if (coarse) {  // most coarse bits are set early: test before the atomic
       uint32_t* cw = coarse + ((o >> cg) >> 5);
       const uint32_t cb = 1u << ((o >> cg) & 31);

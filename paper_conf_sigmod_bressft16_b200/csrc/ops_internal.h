@@ -81,6 +81,7 @@ cudaError_t launch_ws(const FilterArgs& a, cudaStream_t st);
 // fail any predicate are not inserted -- the select -> build pair of a dimension
 // table in one kernel, without the intermediate TID list.
 struct BuildPreds {
+  int32_t key_set = 0;  // 1: duplicate build keys allowed (semi-join key set, ddq_op.build_key_set)
   int32_t n = 0;
   ddq_dev_pred p[DDQ_MAX_PREDS];
 };

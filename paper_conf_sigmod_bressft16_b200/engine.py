@@ -98,10 +98,13 @@ class PlanBuilder:
                     pr.in_vals[j] = int(v)
 
     def build(self, table: str, key: str, payload: str | None = None, input: int = -1,
-              where: list | None = None) -> int:
+              where: list | None = None, key_set: bool = False) -> int:
         """where: predicates evaluated on the input rows inside the build (a fused
-        selection: no intermediate TID list), same forms as select()."""
+        selection: no intermediate TID list), same forms as select().  key_set:
+        the build is the key set of a semi-join (EXISTS / IN): duplicate keys
+        allowed (reading O32)."""
         idx, op = self._op(A.OP_HASH_BUILD, table, input)
+        op.build_key_set = 1 if key_set else 0
         op.key_col = self.db.col(table, key)
         op.payload_col = self.db.col(table, payload) if payload else -1
         if where:

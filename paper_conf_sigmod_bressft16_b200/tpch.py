@@ -108,7 +108,7 @@ def tpch_plan(db: Database, q: str, limit: int = 0, dense: bool = True) -> PlanB
         t = P.gather(li, "l_commitdate", t)                              # vec0
         t = P.gather(li, "l_receiptdate", t)                             # vec1
         t = P.filter_lt(li, t, 0, 1)                                     # l_commitdate < l_receiptdate
-        hl = P.build(li, "l_orderkey", input=t)
+        hl = P.build(li, "l_orderkey", input=t, key_set=True)           # <= 4 lines per order
         o = P.probe("orders", "o_orderkey", hl, input=o)
         P.aggregate("orders", o, keys=["o_orderpriority"], aggs=[(A.AGG_COUNT, [])],
                     order_by=[1], max_groups=5, key_bits=[3])  # codes sorted == string order (O4)

@@ -212,3 +212,45 @@ def test_filter_compare_vectors_at_tids(cmp):
     p.close()
     db.close()
     assert [tuple(x) for x in got] == want and [tuple(x) for x in r.rows] == want
+
+
+@pytest.mark.parametrize("sparse", [False, True])
+def test_key_set_build_semi_join(sparse):
+    """HASH_BUILD with key_set (reading O32): duplicate keys collapse; a probe is the
+    semi-join `exists`.  Dense keys take the direct-mapped index, sparse keys
+    (range > 16x rows) the open-addressing table; a plain build of the same
+    duplicates is rejected."""
+    import numpy as np
+    from paper_conf_sigmod_bressft16_b200 import Database
+    from paper_conf_sigmod_bressft16_b200 import _abi as A
+    rng = np.random.default_rng(11)
+    n, m = 200_003, 50_021
+    mult = 30_011 if sparse else 1  # sparse: keys up to 1.8e9, range >> 16 x rows
+    bk = (rng.integers(1, 40_000, size=n) * mult).astype(np.int32)   # many duplicates
+    f = rng.integers(0, 3, size=n).astype(np.int32)
+    pk = (rng.integers(1, 60_000, size=m) * mult).astype(np.int32)
+    g = rng.integers(0, 4, size=m).astype(np.int32)
+    db = Database(cache_bytes=1 << 30, heap_bytes=1 << 28)
+    db.create_table("b", n)
+    db.create_table("p", m)
+    for t, name, col in (("b", "k", bk), ("b", "f", f), ("p", "k", pk), ("p", "g", g)):
+        db.load_column(t, name, col)
+        db.cache(t, name)
+    P = db.plan()
+    s = P.select("b", [("f", 0, 1)])
+    h = P.build("b", "k", input=s, key_set=True)
+    t = P.probe("p", "k", h)
+    P.aggregate("p", t, keys=["g"], key_bits=[2], aggs=[(A.AGG_COUNT, [])], order_by=[1], max_groups=4)
+    keys = set(bk[f <= 1].tolist())
+    hit = np.array([k in keys for k in pk.tolist()])
+    want = [(k, int((hit & (g == k)).sum())) for k in range(4)]
+    p = db.prepare(P)
+    p.launch()
+    got = [tuple(x) for x in p.fetch().rows]
+    p.close()
+    assert got == want and [tuple(x) for x in db.run(P).rows] == want
+    P2 = db.plan()
+    P2.probe("p", "k", P2.build("b", "k"))
+    with pytest.raises(A.DDQError):
+        db.run(P2)
+    db.close()
