@@ -1,4 +1,4 @@
-"""BASELINE config 4: TPC-H Q1/Q3/Q5/Q6 at SF30, hot and cold cache.
+"""BASELINE config 4: TPC-H Q1/Q3/Q5/Q6 at SF30 (plus Q4/Q7, S8(f) N2), hot and cold cache.
 
 hot : prepared plans (CUDA graphs) over resident columns, CUDA-event timed,
       lineitem rows/s per query;
