@@ -298,8 +298,10 @@ enum {
   DDQ_OP_HASH_PROBE = 3, /* semi-join input TIDs of `table` via fk_col against op `build` */
   DDQ_OP_GATHER = 4,     /* append vector col[tid] to the input's aligned vectors */
   DDQ_OP_AGGREGATE = 5,  /* group-by at input TIDs; root; finalised on the host */
-  DDQ_OP_FILTER_EQ = 6,  /* keep input rows whose two aligned vectors are equal (TPC-H Q5's
-                            c_nationkey = s_nationkey); vectors carried */
+  DDQ_OP_FILTER_EQ = 6,  /* keep input rows whose two aligned vectors compare true under
+                            eq_cmp: equal (TPC-H Q5's c_nationkey = s_nationkey), less
+                            (Q4's l_commitdate < l_receiptdate) or not equal (Q7's
+                            n1 <> n2); vectors carried */
   DDQ_OP_STAR = 7        /* conjunction of predicates and probes over all rows of a fact
                             table in one pass (all term columns streamed once); output as
                             a chain of SELECT/HASH_PROBE ops would produce it */
