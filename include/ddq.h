@@ -197,7 +197,11 @@ enum {
   DDQ_AGG_SUM_MUL = 3,        /* a * b */
   DDQ_AGG_SUM_SUB = 4,        /* a - b */
   DDQ_AGG_SUM_MUL_100M = 5,   /* a * (100 - b)            (TPC-H scale-2 decimals) */
-  DDQ_AGG_SUM_MUL_100M_100P = 6 /* a * (100 - b) * (100 + c) */
+  DDQ_AGG_SUM_MUL_100M_100P = 6, /* a * (100 - b) * (100 + c) */
+  DDQ_AGG_MIN = 7             /* min(a) (S8(a6); TPC-H Q2's min(ps_supplycost)): the group's
+                                 smallest int64 value, returned sign-extended in the
+                                 int128 cell; aggregations carrying a MIN run the
+                                 generic one-row-per-thread kernel on the global table */
 };
 #define DDQ_MAX_AGGS 8
 #define DDQ_MAX_KEYS 3

@@ -704,7 +704,7 @@ static bool dense_plan(int64_t n_rows, const BuildPreds* preds, const int32_t* c
   for (int k = 0; k < n_keys; k++)
     if ((p->kcol[k] = col_id(key_col[k], 4)) < 0) return false;
   for (int a = 0; a < n_aggs; a++) {
-    const int need = aggs[a].kind == DDQ_AGG_COUNT ? 0 : aggs[a].kind == DDQ_AGG_SUM ? 1
+    const int need = aggs[a].kind == DDQ_AGG_COUNT ? 0 : (aggs[a].kind == DDQ_AGG_SUM || aggs[a].kind == DDQ_AGG_MIN) ? 1
                    : aggs[a].kind == DDQ_AGG_SUM_MUL_100M_100P ? 3 : 2;
     for (int j = 0; j < 3; j++) {
       p->acol[a][j] = 0;
@@ -727,6 +727,8 @@ static bool dense_plan(int64_t n_rows, const BuildPreds* preds, const int32_t* c
 
 bool agg_dense_supported(int64_t n_rows, const BuildPreds* preds, const int32_t* const* key_col, int n_keys,
                          const int32_t* key_bits, const ddq_dev_agg* aggs, int n_aggs) {
+  for (int a = 0; a < n_aggs; a++)
+    if (aggs[a].kind == DDQ_AGG_MIN) return false;  // MIN: generic kernel (launch_groupby)
   DenseAggParams p{};
   return dense_plan(n_rows, preds, key_col, n_keys, key_bits, aggs, n_aggs, &p);
 }

@@ -78,7 +78,7 @@ static std::vector<int> op_columns(const ddq_op& op) {
       for (int k = 0; k < op.n_keys; k++)
         if (op.key_src[k] < -1) c.push_back(-2 - op.key_src[k]);
       for (int a = 0; a < op.n_aggs; a++) {
-        int need = op.agg_kind[a] == DDQ_AGG_COUNT ? 0 : op.agg_kind[a] == DDQ_AGG_SUM ? 1
+        int need = op.agg_kind[a] == DDQ_AGG_COUNT ? 0 : (op.agg_kind[a] == DDQ_AGG_SUM || op.agg_kind[a] == DDQ_AGG_MIN) ? 1
                  : op.agg_kind[a] == DDQ_AGG_SUM_MUL_100M_100P ? 3 : 2;
         for (int j = 0; j < need; j++) c.push_back(op.agg_col[a][j]);
       }
@@ -601,9 +601,15 @@ ddq_status run_host_op(ddq_db* db, const ddq_op& op, const std::vector<Inter>& I
           key |= (int64_t)(uint32_t)c << kshift[k];
         }
         auto& acc = g[key];
-        if (acc.empty()) acc.assign((size_t)na, 0);
+        const bool fresh = acc.empty();
+        if (fresh) acc.assign((size_t)na, 0);
         for (int a = 0; a < na; a++) {
           int kind = op.agg_kind[a];
+          if (kind == DDQ_AGG_MIN) {
+            const __int128 x = hcol(ac[(size_t)a][0], r);
+            if (fresh || x < acc[(size_t)a]) acc[(size_t)a] = x;
+            continue;
+          }
           __int128 v = 1;
           if (kind != DDQ_AGG_COUNT) {
             __int128 x = hcol(ac[(size_t)a][0], r);

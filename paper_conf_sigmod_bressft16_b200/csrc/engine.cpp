@@ -470,9 +470,13 @@ ddq_status run_gpu_op(GpuOpCtx& ctx, const ddq_op& op, Inter& out) {
       }
       ddq_dev_agg ag[DDQ_MAX_AGGS];
       std::memset(ag, 0, sizeof(ag));
+      bool has_min = false;  // MIN: the generic global-table kernel (launch_groupby)
       for (int a = 0; a < op.n_aggs; a++) {
         ag[a].kind = op.agg_kind[a];
-        int need = op.agg_kind[a] == DDQ_AGG_COUNT ? 0 : op.agg_kind[a] == DDQ_AGG_SUM ? 1
+        if (op.agg_kind[a] < DDQ_AGG_COUNT || op.agg_kind[a] > DDQ_AGG_MIN)
+          return set_error(DDQ_EINVAL, "aggregate: bad aggregate kind");
+        has_min |= op.agg_kind[a] == DDQ_AGG_MIN;
+        int need = op.agg_kind[a] == DDQ_AGG_COUNT ? 0 : (op.agg_kind[a] == DDQ_AGG_SUM || op.agg_kind[a] == DDQ_AGG_MIN) ? 1
                  : op.agg_kind[a] == DDQ_AGG_SUM_MUL_100M_100P ? 3 : 2;
         for (int j = 0; j < need; j++) {
           const Column* c = col_of(db, op.agg_col[a][j]);
@@ -518,7 +522,7 @@ ddq_status run_gpu_op(GpuOpCtx& ctx, const ddq_op& op, Inter& out) {
         d.n_in = p.n_in;
         for (int j = 0; j < DDQ_MAX_IN; j++) d.in_vals[j] = p.in_vals[j];
       }
-      if (!in && agg_dense_supported(in_cap, &bp, kc, op.n_keys, op.key_bits, ag, op.n_aggs)) {
+      if (!in && !has_min && agg_dense_supported(in_cap, &bp, kc, op.n_keys, op.key_bits, ag, op.n_aggs)) {
         out.d_rows = (uint32_t*)A.get(64);
         if (A.failed) return DDQ_ENOMEM_DEVICE;
         init_fill(out.d_rows, 4, 0, st);
@@ -541,7 +545,7 @@ ddq_status run_gpu_op(GpuOpCtx& ctx, const ddq_op& op, Inter& out) {
         g_tids = ft;
         g_count = fc;
       }
-      if (op.n_preds > 0 && (!in || !agg_ws_supported(in->tids, kv, op.n_keys, op.n_aggs, out.gb_cap))) {
+      if (op.n_preds > 0 && (has_min || !in || !agg_ws_supported(in->tids, kv, op.n_keys, op.n_aggs, out.gb_cap))) {
         // no fused kernel for this shape: a selection into a temporary TID list
         // (carrying the key vectors) feeds the aggregation
         int32_t* ft = (int32_t*)A.get((uint64_t)std::max<int64_t>(in_cap, 1) * 4);
@@ -1302,7 +1306,7 @@ void count_accesses(ddq_db* db, const ddq_op& op) {
       for (int k = 0; k < op.n_keys; k++)
         if (op.key_src[k] < -1) touch(-2 - op.key_src[k]);
       for (int a = 0; a < op.n_aggs; a++) {
-        int need = op.agg_kind[a] == DDQ_AGG_COUNT ? 0 : op.agg_kind[a] == DDQ_AGG_SUM ? 1
+        int need = op.agg_kind[a] == DDQ_AGG_COUNT ? 0 : (op.agg_kind[a] == DDQ_AGG_SUM || op.agg_kind[a] == DDQ_AGG_MIN) ? 1
                  : op.agg_kind[a] == DDQ_AGG_SUM_MUL_100M_100P ? 3 : 2;
         for (int j = 0; j < need; j++) touch(op.agg_col[a][j]);
       }
@@ -1582,7 +1586,7 @@ int32_t ddq_prepared_profile(ddq_prepared* p, void* stream, int32_t max_ops, flo
           for (int j = 0; j < 3; j++) {
             int c = op.agg_col[a][j];
             if (c < 0 || std::find(seen.begin(), seen.end(), c) != seen.end()) continue;
-            int need = op.agg_kind[a] == DDQ_AGG_COUNT ? 0 : op.agg_kind[a] == DDQ_AGG_SUM ? 1
+            int need = op.agg_kind[a] == DDQ_AGG_COUNT ? 0 : (op.agg_kind[a] == DDQ_AGG_SUM || op.agg_kind[a] == DDQ_AGG_MIN) ? 1
                      : op.agg_kind[a] == DDQ_AGG_SUM_MUL_100M_100P ? 3 : 2;
             if (j >= need) continue;
             seen.push_back(c);

@@ -603,6 +603,49 @@ __global__ void __launch_bounds__(GBS_THREADS) groupby_small_kernel(const __grid
   }
 }
 
+// Aggregations carrying a MIN (DDQ_AGG_MIN, S8(a6)): one row per thread straight
+// into the global table.  SUM kinds add exactly into the int128 cell; MIN takes
+// atomicMin of the cell's int64 lo word, which groupby_min_init_kernel set to
+// INT64_MAX and groupby_min_fix_kernel sign-extends into hi before compaction.
+__global__ void groupby_generic_kernel(const __grid_constant__ GroupbyParams P) {
+  const uint32_t n = P.d_count ? ld_relaxed_u32(P.d_count) : P.n_static;
+  const size_t cap = (size_t)P.cap_mask + 1;
+  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
+    const int32_t r = P.tids[i];
+    long long key = 0;
+    for (int k = 0; k < P.n_keys; k++) {
+      const int32_t c = P.key_vec[k] ? P.key_vec[k][i] : ldg_gather(P.key_col[k] + r);
+      key |= (long long)(uint32_t)c << P.key_shift[k];
+    }
+    const int64_t slot = table_slot(P.g_keys, P.cap_mask, gb_hash(key, P.shift), key);
+    if (slot < 0) {
+      atomicMax(P.d_error, 2u);
+      continue;
+    }
+    for (int a = 0; a < P.n_aggs; a++) {
+      unsigned long long* cell = &P.g_accs[((size_t)a * cap + slot) * 2];
+      if (P.kind[a] == DDQ_AGG_MIN) {
+        atomicMin(reinterpret_cast<long long*>(cell), col_at(P.arg[a][0], P.width[a][0], r));
+      } else {
+        const long long v = agg_value(P, a, r);
+        atomic_add_i128_pair(cell, cell + 1, (unsigned long long)v, v < 0 ? -1 : 0);
+      }
+    }
+  }
+}
+
+__global__ void groupby_min_init_kernel(unsigned long long* accs, uint32_t capacity, int n_aggs, uint32_t min_mask) {
+  for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < (size_t)capacity * n_aggs;
+       i += (size_t)gridDim.x * blockDim.x)
+    if ((min_mask >> (i / capacity)) & 1u) accs[i * 2] = (unsigned long long)LLONG_MAX;
+}
+
+__global__ void groupby_min_fix_kernel(unsigned long long* accs, uint32_t capacity, int n_aggs, uint32_t min_mask) {
+  for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < (size_t)capacity * n_aggs;
+       i += (size_t)gridDim.x * blockDim.x)
+    if ((min_mask >> (i / capacity)) & 1u) accs[i * 2 + 1] = (long long)accs[i * 2] < 0 ? ~0ull : 0ull;
+}
+
 size_t groupby_table_bytes(uint32_t capacity, int n_aggs) {
   return (size_t)capacity * 8 + (size_t)capacity * n_aggs * 16;
 }
@@ -628,7 +671,10 @@ cudaError_t launch_groupby(const int32_t* tids, const uint32_t* d_count, int64_t
                            const int32_t* key_bits,
                            const ddq_dev_agg* aggs, int n_aggs, void* table, uint32_t capacity,
                            uint32_t* d_error, cudaStream_t st) {
-  if (agg_ws_supported(tids, key_vec, n_keys, n_aggs, capacity) && d_count) {
+  uint32_t min_mask = 0;
+  for (int a = 0; a < n_aggs; a++)
+    if (aggs[a].kind == DDQ_AGG_MIN) min_mask |= 1u << a;
+  if (!min_mask && agg_ws_supported(tids, key_vec, n_keys, n_aggs, capacity) && d_count) {
     static const char* env = getenv("DDQ_AGG_WS");  // "0": the warp-match kernels below
     if (!env || env[0] != '0')
       return launch_agg_ws(tids, d_count, n_cap, key_vec, key_col, n_keys, key_bits, aggs, n_aggs, table, capacity,
@@ -662,6 +708,16 @@ cudaError_t launch_groupby(const int32_t* tids, const uint32_t* d_count, int64_t
   while ((1u << lg) < capacity) lg++;
   p.shift = 64 - lg;
   p.d_error = d_error;
+  if (min_mask) {  // MIN: the generic kernel on the global table (init / fix the MIN cells)
+    const int64_t cells = (int64_t)capacity * n_aggs;
+    const int gi = (int)std::min<int64_t>((cells + 255) / 256, (int64_t)num_sms() * 8);
+    groupby_min_init_kernel<<<gi, 256, 0, st>>>(p.g_accs, capacity, n_aggs, min_mask);
+    const int64_t g = (n_cap + 255) / 256;
+    const int grid = (int)(g < 1 ? 1 : (g > (int64_t)num_sms() * 8 ? (int64_t)num_sms() * 8 : g));
+    groupby_generic_kernel<<<grid, 256, 0, st>>>(p);
+    groupby_min_fix_kernel<<<gi, 256, 0, st>>>(p.g_accs, capacity, n_aggs, min_mask);
+    return cudaGetLastError();
+  }
   // small key domain: every key dictionary-coded (key_bits), D * n_aggs <= 64
   int total_bits = 0;
   bool coded = n_keys == 0 || key_bits != nullptr;
@@ -674,7 +730,7 @@ cudaError_t launch_groupby(const int32_t* tids, const uint32_t* d_count, int64_t
   for (int a = 0; a < n_aggs; a++)
     for (int j = 0; j < 3; j++) {
       p.uidx[a][j] = -1;
-      const int need = aggs[a].kind == DDQ_AGG_COUNT ? 0 : aggs[a].kind == DDQ_AGG_SUM ? 1
+      const int need = aggs[a].kind == DDQ_AGG_COUNT ? 0 : (aggs[a].kind == DDQ_AGG_SUM || aggs[a].kind == DDQ_AGG_MIN) ? 1
                      : aggs[a].kind == DDQ_AGG_SUM_MUL_100M_100P ? 3 : 2;
       if (j >= need) continue;
       int c = 0;

@@ -219,9 +219,9 @@ ddq_status ddq_op_groupby(const int32_t* tids, const uint32_t* d_count, int64_t 
   for (int k = 0; k < n_keys; k++)
     if (!((key_vec && key_vec[k]) || (key_col && key_col[k]))) return set_error(DDQ_EINVAL, "groupby: null key");
   for (int a = 0; a < n_aggs; a++) {
-    int need = aggs[a].kind == DDQ_AGG_COUNT ? 0 : aggs[a].kind == DDQ_AGG_SUM ? 1
+    int need = aggs[a].kind == DDQ_AGG_COUNT ? 0 : (aggs[a].kind == DDQ_AGG_SUM || aggs[a].kind == DDQ_AGG_MIN) ? 1
              : aggs[a].kind == DDQ_AGG_SUM_MUL_100M_100P ? 3 : 2;
-    if (aggs[a].kind < DDQ_AGG_COUNT || aggs[a].kind > DDQ_AGG_SUM_MUL_100M_100P)
+    if (aggs[a].kind < DDQ_AGG_COUNT || aggs[a].kind > DDQ_AGG_MIN)
       return set_error(DDQ_EINVAL, "groupby: bad aggregate kind");
     for (int j = 0; j < need; j++)
       if (!aggs[a].arg[j] || (aggs[a].width[j] != 4 && aggs[a].width[j] != 8))

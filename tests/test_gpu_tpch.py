@@ -254,3 +254,51 @@ def test_key_set_build_semi_join(sparse):
     with pytest.raises(A.DDQError):
         db.run(P2)
     db.close()
+
+
+@pytest.mark.parametrize("shape", ["tids_vec_keys", "dense_col_keys", "fused_pred", "cpu_only"])
+def test_aggregate_min(shape):
+    """AGG_MIN (S8(a6)) next to SUM / COUNT: group minima of int64 values of both
+    signs (and int32 arguments) vs numpy, at a TID list with vector keys, over all
+    rows with column keys, with a fused selection, and in the host executor."""
+    import numpy as np
+    from paper_conf_sigmod_bressft16_b200 import Database
+    from paper_conf_sigmod_bressft16_b200 import _abi as A
+    rng = np.random.default_rng(5)
+    n = 250_007
+    g = rng.integers(0, 37, size=n).astype(np.int32)
+    x = rng.integers(-(1 << 60), 1 << 60, size=n, dtype=np.int64)
+    y = rng.integers(-1000, 1000, size=n).astype(np.int32)
+    s = rng.integers(0, 10, size=n).astype(np.int32)
+    kw = {"placement": A.PLACE_CPU_ONLY} if shape == "cpu_only" else {}
+    db = Database(cache_bytes=1 << 30, heap_bytes=1 << 28, **kw)
+    db.create_table("t", n)
+    for name, col in (("g", g), ("x", x), ("y", y), ("s", s)):
+        db.load_column("t", name, col)
+        if shape != "cpu_only":
+            db.cache("t", name)
+    P = db.plan()
+    aggs = [(A.AGG_MIN, ["x"]), (A.AGG_SUM, ["y"]), (A.AGG_MIN, ["y"]), (A.AGG_COUNT, [])]
+    m = s <= 6
+    if shape in ("tids_vec_keys", "cpu_only"):
+        t = P.select("t", [("s", 0, 6)])
+        t = P.gather("t", "g", t)
+        P.aggregate("t", t, keys=[0], key_bits=[6], aggs=aggs, order_by=[1], max_groups=64)
+    elif shape == "dense_col_keys":
+        m = np.ones(n, dtype=bool)
+        P.aggregate("t", -1, keys=["g"], key_bits=[6], aggs=aggs, order_by=[1], max_groups=64)
+    else:
+        P.aggregate("t", -1, keys=["g"], key_bits=[6], aggs=aggs, where=[("s", 0, 6)], order_by=[1],
+                    max_groups=64)
+    want = []
+    for k in sorted(set(g[m].tolist())):
+        mk = m & (g == k)
+        want.append((k, int(x[mk].min()), int(y[mk].astype(np.int64).sum()), int(y[mk].min()), int(mk.sum())))
+    r = db.run(P)
+    assert [tuple(v) for v in r.rows] == want
+    if shape != "cpu_only":
+        p = db.prepare(P)
+        p.launch()
+        assert [tuple(v) for v in p.fetch().rows] == want
+        p.close()
+    db.close()
