@@ -216,6 +216,7 @@ __global__ void join_index_build_kernel(const int32_t* __restrict__ keys, const 
     }
     // only the row that set the bit writes the payload: a key set's duplicates
     // (O32; ~3 of 4 late lineitems of TPC-H Q4) skip their random 4-byte store
+    // (measured neutral on B200: Q4's key-set build stays at 100 us, atomic-bound)
     if (!(old & (1u << (o & 31)))) payarr[o] = payload ? payload[r] : r;
   }
 }
