@@ -45,7 +45,9 @@ int main(void) {
   P(ddq_dev_pred) P(ddq_dev_agg) P(ddq_config) P(ddq_pred) P(ddq_op) P(ddq_plan) P(ddq_result) P(ddq_stats)
   O(ddq_op, preds) O(ddq_op, key_col) O(ddq_op, agg_col) O(ddq_op, max_groups) O(ddq_op, order_by)
   O(ddq_op, limit) O(ddq_config, cache_bytes) O(ddq_config, fault_alloc_every) O(ddq_result, exec_ms)
-  O(ddq_dev_pred, in_vals) O(ddq_dev_agg, arg)
+  O(ddq_dev_pred, in_vals) O(ddq_dev_agg, arg) O(ddq_op, eq_cmp) O(ddq_op, build_key_set)
+  printf("DDQ_CMP_EQ %d\nDDQ_CMP_LT %d\nDDQ_CMP_NE %d\nDDQ_AGG_MIN %d\nDDQ_AGG_COUNT %d\n",
+         DDQ_CMP_EQ, DDQ_CMP_LT, DDQ_CMP_NE, (int)DDQ_AGG_MIN, (int)DDQ_AGG_COUNT);
   return 0;
 }
 """
@@ -60,8 +62,12 @@ def test_struct_layouts_match_c(tmp_path):
     got = dict(line.split() for line in subprocess.check_output([str(exe)], text=True).splitlines())
     py = {"ddq_dev_pred": A.DevPred, "ddq_dev_agg": A.DevAgg, "ddq_config": A.Config, "ddq_pred": A.Pred,
           "ddq_op": A.Op, "ddq_plan": A.Plan, "ddq_result": A.Result, "ddq_stats": A.Stats}
+    consts = {"DDQ_CMP_EQ": A.CMP_EQ, "DDQ_CMP_LT": A.CMP_LT, "DDQ_CMP_NE": A.CMP_NE,
+              "DDQ_AGG_MIN": A.AGG_MIN, "DDQ_AGG_COUNT": A.AGG_COUNT}
     for k, v in got.items():
-        if "." in k:
+        if k in consts:
+            assert consts[k] == int(v), k
+        elif "." in k:
             t, f = k.split(".")
             assert getattr(py[t], f).offset == int(v), k
         else:
