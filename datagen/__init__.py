@@ -158,7 +158,7 @@ class SSB:
 
 # --------------------------------------------------------------- TPC-H schema
 TPCH_TABLES = {"nation": 11, "region": 12, "customer": 13, "supplier": 14, "part": 15,
-               "orders": 16, "lineitem": 17}
+               "orders": 16, "lineitem": 17, "calendar": 18}
 TPCH_COLUMNS = {
     "nation": ["n_nationkey", "n_name", "n_regionkey"],
     "region": ["r_regionkey", "r_name"],
@@ -169,6 +169,8 @@ TPCH_COLUMNS = {
     "lineitem": ["l_orderkey", "l_partkey", "l_suppkey", "l_linenumber", "l_quantity",
                  "l_extendedprice", "l_discount", "l_tax", "l_returnflag", "l_linestatus",
                  "l_shipdate", "l_commitdate", "l_receiptdate"],
+    # the date dimension over TPC-H's date domain, 1992-01-01 .. 1998-12-31 (reading O34)
+    "calendar": ["d_datekey", "d_year"],
 }
 TPCH_STRING_COLUMNS = {"n_name": "nation", "r_name": "region", "c_mktsegment": "mktsegment",
                        "l_returnflag": "returnflag", "l_linestatus": "linestatus",

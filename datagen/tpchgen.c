@@ -16,7 +16,12 @@ int32_t ddqgen_datekey_of_index(int64_t idx);
 int ddqgen_dict_size(int dict);
 
 enum { TH_NATION = 11, TH_REGION = 12, TH_CUSTOMER = 13, TH_SUPPLIER = 14, TH_PART = 15,
-       TH_ORDERS = 16, TH_LINEITEM = 17 };
+       TH_ORDERS = 16, TH_LINEITEM = 17, TH_CALENDAR = 18 };
+/* TH_CALENDAR: the date dimension of TPC-H's date domain (one row per day
+ * 1992-01-01 .. 1998-12-31, as SSB's date table): d_datekey yyyymmdd, d_year.
+ * Q7's extract(year from l_shipdate) joins it (reading O34). */
+enum { CAL_DATEKEY = 0, CAL_YEAR };
+#define N_CALENDAR 2557
 enum { N_NATIONKEY = 0, N_NAME, N_REGIONKEY };
 enum { R_REGIONKEY = 0, R_NAME };
 enum { HC_CUSTKEY = 0, HC_NATIONKEY, HC_MKTSEGMENT };
@@ -54,6 +59,7 @@ int64_t ddqgen_tpch_rows(int table, double sf) {
     case TH_PART: return scaled_h(sf, 200000.0);
     case TH_ORDERS: return scaled_h(sf, 1500000.0);
     case TH_LINEITEM: return 4 * scaled_h(sf, 1500000.0);
+    case TH_CALENDAR: return N_CALENDAR;
   }
   return -1;
 }
@@ -68,6 +74,7 @@ int ddqgen_tpch_width(int table, int col) {
     case TH_LINEITEM:
       if (col < 0 || col >= L_NCOLS) return 0;
       return (col >= L_QUANTITY && col <= L_TAX) ? 8 : 4;
+    case TH_CALENDAR: return (col == CAL_DATEKEY || col == CAL_YEAR) ? 4 : 0;
   }
   return 0;
 }
@@ -86,6 +93,10 @@ static void gen_rows_h(uint64_t seed, double sf, int table, int col, int64_t b, 
         o32[k] = col == N_NATIONKEY ? (int32_t)i : col == N_NAME ? NATION_CODE[i] : NATION_REGION_H[i];
         break;
       case TH_REGION: o32[k] = (int32_t)i; break; /* region dict sorted == regionkey order */
+      case TH_CALENDAR: {
+        const int32_t dk = ddqgen_datekey_of_index(i);
+        o32[k] = col == CAL_DATEKEY ? dk : dk / 10000;
+      } break;
       case TH_CUSTOMER:
         if (col == HC_CUSTKEY) o32[k] = (int32_t)(i + 1);
         else if (col == HC_NATIONKEY) o32[k] = (int32_t)(ddqgen_hash(seed, table, DRH_NATION, (uint64_t)i) % 25u);

@@ -69,7 +69,11 @@ const char* ddq_version(void);
 /* Predicate kinds (S8(a1)-(a2)).  RANGE covers =, <, <=, >, >=, BETWEEN on integer
  * columns (constants folded into an inclusive [lo, hi]); IN holds up to 8 values
  * (string IN/= become dictionary-code sets, reading O4). */
-enum { DDQ_PRED_RANGE = 1, DDQ_PRED_IN = 2 };
+enum { DDQ_PRED_RANGE = 1, DDQ_PRED_IN = 2, DDQ_PRED_BITSET = 3 };
+/* DDQ_PRED_BITSET: a dictionary-code set too large for IN (e.g. TPC-H Q2's
+ * p_type LIKE '%BRASS', 30 of 150 codes; reading O35): v holds iff
+ * 0 <= v - lo < 512 and bit (v - lo) of the 512-bit mask in_vals[0..7] is set
+ * (bit b of word b / 64).  hi and n_in are ignored.  ddq_dictionary_like builds one. */
 #define DDQ_MAX_IN 8
 #define DDQ_MAX_PREDS 4
 #define DDQ_MAX_CARRY 4
@@ -274,6 +278,7 @@ ddq_status ddq_create_table(ddq_db* db, const char* name, int64_t n_rows, int64_
 ddq_status ddq_load_column(ddq_db* db, ddq_table t, const char* name, ddq_type type,
                            const void* host_data, int64_t n_rows, ddq_column* out);
 ddq_status ddq_find_column(ddq_db* db, const char* table, const char* name, ddq_column* out);
+
 /* Storage adviser: pin a column into the device cache (H2D copy on the
  * library's copy stream, counted in stats) / evict it (freed once no running
  * operator references it).  Fails with DDQ_ENOMEM_DEVICE if it does not
@@ -379,6 +384,14 @@ typedef struct {
      payload is any one of their rows; 0 (default) = unique keys, a duplicate is
      DDQ_EINVAL (reading O13). */
   int32_t build_key_set;
+  /* AGGREGATE finalisation (S8(a7), reading O10): n_avg derived double columns,
+     avg k = (double)acc[avg_sum[k]] / (double)acc[avg_count] / 10^avg_scale[k] (SQL AVG
+     of a scale-s decimal; TPC-H Q1's avg_qty / avg_price / avg_disc).  NULL when the
+     count is 0.  Computed on the host after the exact int128 merge. */
+  int32_t n_avg;
+  int32_t avg_sum[4];
+  int32_t avg_count;
+  int32_t avg_scale[4];
 } ddq_op;
 
 #define DDQ_CMP_EQ 0
@@ -391,6 +404,23 @@ typedef struct {
   ddq_op ops[DDQ_MAX_OPS];
 } ddq_plan;
 
+/* Order-preserving dictionary of a string column (reading O4; S8(b)): the column's
+ * int32 values are codes = ranks in `sorted_strings` (n distinct strings, strictly
+ * ascending in bytewise (C-locale) order; DDQ_EINVAL otherwise).  The strings are
+ * copied; the library decodes result keys through them (ddq_result.key_str) and
+ * folds string predicates into code predicates (below).  Plan-time host work only. */
+ddq_status ddq_set_dictionary(ddq_db* db, ddq_column c, const char* const* sorted_strings, int32_t n);
+/* Code range of a string constant: *lower = first code whose string >= s, *upper =
+ * first code whose string > s (so s is present iff lower < upper; BETWEEN a AND b
+ * is [lower(a), upper(b)) ).  DDQ_ENOTFOUND if the column has no dictionary. */
+ddq_status ddq_dictionary_range(ddq_db* db, ddq_column c, const char* s, int32_t* lower, int32_t* upper);
+/* SQL LIKE over the dictionary (TPC-H Q2's p_type like '%BRASS'; reading O35):
+ * fills *out with a predicate on column c that holds exactly for the codes whose
+ * string matches `pattern` ('%' = any run, '_' = any one byte, no escapes):
+ * DDQ_PRED_IN when <= 8 codes match, else DDQ_PRED_BITSET when they lie within
+ * 512 consecutive codes, else DDQ_EINVAL.  No match: an empty RANGE (lo > hi). */
+ddq_status ddq_dictionary_like(ddq_db* db, ddq_column c, const char* pattern, ddq_pred* out);
+
 /* Result of a query: rows of (n_keys int32-code keys, n_aggs int128 aggregates)
  * in ORDER BY order, or, for a select-* root, the TID list. Owned by the library. */
 typedef struct {
@@ -402,6 +432,21 @@ typedef struct {
   const int32_t* tids;
   int32_t gpu_ops, host_ops, aborts;
   double exec_ms;        /* submit -> root finished */
+  /* SQL NULLs (reading O7): agg_null[i * n_aggs + a] = 1 when aggregate a of row i
+     is NULL -- SUM / MIN over an empty input.  An AGGREGATE without keys always
+     returns exactly one row (count 0, SUMs NULL, when nothing qualified); grouped
+     queries return no row for an empty input. */
+  const uint8_t* agg_null;
+  /* root->n_avg finalisation doubles per row (avgs[i * n_avg + k]); NaN when NULL */
+  int32_t n_avg;
+  int32_t _pad;
+  const double* avgs;
+  /* decoded group keys: key_str[i * n_keys + k] = the dictionary string of key k of
+     row i when its source column has a dictionary (ddq_set_dictionary), else NULL.
+     The key source is the column behind the key: a key column, or the column an
+     aligned vector was gathered from / a build emitted as payload.  Strings are
+     owned by the database (valid until ddq_close); the pointer array by the result. */
+  const char* const* key_str;
 } ddq_result;
 
 /* Submit a plan (copied; thread-safe; many user threads may submit). */

@@ -62,6 +62,9 @@ def lib():
         L.oracle_result_naggs.argtypes = [ctypes.c_void_p]
         L.oracle_result_row.argtypes = [ctypes.c_void_p, ctypes.c_int64,
                                         ctypes.POINTER(ctypes.c_int64), ctypes.POINTER(ctypes.c_int64)]
+        L.oracle_result_nulls.argtypes = [ctypes.c_void_p, ctypes.c_int64]
+        L.oracle_result_navg.argtypes = [ctypes.c_void_p]
+        L.oracle_result_avgs.argtypes = [ctypes.c_void_p, ctypes.c_int64, ctypes.POINTER(ctypes.c_double)]
         L.oracle_result_ntids.restype = ctypes.c_int64
         L.oracle_result_ntids.argtypes = [ctypes.c_void_p]
         L.oracle_result_tids.argtypes = [ctypes.c_void_p, ctypes.c_void_p]
@@ -143,18 +146,24 @@ class OracleDB:
                 out = np.empty(n, dtype=np.int32)
                 L.oracle_result_tids(r, out.ctypes.data)
                 return out
-            nk, na = L.oracle_result_nkeys(r), L.oracle_result_naggs(r)
+            nk, na, nv = L.oracle_result_nkeys(r), L.oracle_result_naggs(r), L.oracle_result_navg(r)
             keys = (ctypes.c_int64 * 4)()
             aggs = (ctypes.c_int64 * 16)()
-            rows = []
+            av = (ctypes.c_double * 4)()
+            rows, avgs = [], []
             for i in range(L.oracle_result_rows(r)):
                 L.oracle_result_row(r, i, keys, aggs)
+                nulls = L.oracle_result_nulls(r, i)
                 vals = [int(keys[k]) for k in range(nk)]
                 for a in range(na):
                     lo = aggs[2 * a] & 0xFFFFFFFFFFFFFFFF
                     hi = aggs[2 * a + 1]
-                    vals.append((hi << 64) | lo)
+                    vals.append(None if (nulls >> a) & 1 else (hi << 64) | lo)  # SQL NULL (O7)
                 rows.append(tuple(vals))
+                if nv:
+                    L.oracle_result_avgs(r, i, av)
+                    avgs.append(tuple(float(av[k]) for k in range(nv)))
+            self.last_avgs = avgs
             return rows
         finally:
             L.oracle_result_free(r)
@@ -184,14 +193,23 @@ def ssb_db(db: "datagen.SSB", query: str, fact_rows: int | None = None) -> Oracl
 
 def run(db, query: str, fact_rows: int | None = None):
     """Evaluate `query` ("ssb1.1".."ssb4.3", "listing1".."listing8", "listing2b",
-    "tpch1", "tpch3", "tpch4", "tpch5", "tpch6", "tpch7") on a datagen database."""
+    "tpch1", "tpch3", "tpch4", "tpch5", "tpch6", "tpch7") on a datagen database.
+    Rows are (keys..., aggregates...) with None for a SQL NULL aggregate."""
+    return run_with_avgs(db, query, fact_rows)[0]
+
+
+def run_with_avgs(db, query: str, fact_rows: int | None = None):
+    """(rows, avgs): avgs[i] = the AVG columns of row i (TPC-H Q1: avg_qty,
+    avg_price, avg_disc as sum / count / 100 in long double, reading O10)."""
     if query.startswith("tpch"):
         odb = OracleDB()
         _set_dicts(odb)
         for (t, c) in TPCH_QUERY_COLUMNS[int(query[4:])]:
             odb.set_col(c, db.col(t, c))
-        return odb.query(query)
-    return ssb_db(db, query, fact_rows).query(query)
+    else:
+        odb = ssb_db(db, query, fact_rows)
+    rows = odb.query(query)
+    return rows, getattr(odb, "last_avgs", [])
 
 
 SSB_QUERIES = ["ssb1.1", "ssb1.2", "ssb1.3", "ssb2.1", "ssb2.2", "ssb2.3", "ssb3.1", "ssb3.2",

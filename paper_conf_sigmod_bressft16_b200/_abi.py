@@ -17,7 +17,7 @@ STATUS = {0: "DDQ_OK", -1: "DDQ_EINVAL", -2: "DDQ_ENOTFOUND", -3: "DDQ_ENOMEM_HO
           -4: "DDQ_ENOMEM_DEVICE", -5: "DDQ_ECUDA", -6: "DDQ_ENCCL", -7: "DDQ_ESTATE",
           -8: "DDQ_ETIMEOUT", -9: "DDQ_EOVERFLOW"}
 
-PRED_RANGE, PRED_IN = 1, 2
+PRED_RANGE, PRED_IN, PRED_BITSET = 1, 2, 3
 MAX_IN, MAX_PREDS, MAX_CARRY, MAX_AGGS, MAX_KEYS, MAX_OPS = 8, 4, 4, 8, 3, 32
 CMP_EQ, CMP_LT, CMP_NE = 0, 1, 2  # FILTER_EQ comparison (ddq_op.eq_cmp)
 OP_SELECT, OP_HASH_BUILD, OP_HASH_PROBE, OP_GATHER, OP_AGGREGATE, OP_FILTER_EQ, OP_STAR = 1, 2, 3, 4, 5, 6, 7
@@ -69,7 +69,9 @@ class Op(ctypes.Structure):
                 ("term_kind", ctypes.c_int32 * 4), ("term_build", ctypes.c_int32 * 4),
                 ("term_fk", ctypes.c_int32 * 4), ("term_emit", ctypes.c_int32 * 4),
                 ("fetch_build", ctypes.c_int32), ("eq_cmp", ctypes.c_int32),
-                ("build_key_set", ctypes.c_int32)]
+                ("build_key_set", ctypes.c_int32), ("n_avg", ctypes.c_int32),
+                ("avg_sum", ctypes.c_int32 * 4), ("avg_count", ctypes.c_int32),
+                ("avg_scale", ctypes.c_int32 * 4)]
 
 
 class DevTerm(ctypes.Structure):
@@ -89,7 +91,9 @@ class Result(ctypes.Structure):
                 ("keys", ctypes.POINTER(ctypes.c_int64)), ("aggs", ctypes.POINTER(ctypes.c_int64)),
                 ("n_tids", ctypes.c_int64), ("tids", ctypes.POINTER(ctypes.c_int32)),
                 ("gpu_ops", ctypes.c_int32), ("host_ops", ctypes.c_int32), ("aborts", ctypes.c_int32),
-                ("exec_ms", ctypes.c_double)]
+                ("exec_ms", ctypes.c_double), ("agg_null", ctypes.POINTER(ctypes.c_uint8)),
+                ("n_avg", ctypes.c_int32), ("_pad", ctypes.c_int32), ("avgs", ctypes.POINTER(ctypes.c_double)),
+                ("key_str", ctypes.POINTER(ctypes.c_char_p))]
 
 
 class Stats(ctypes.Structure):
@@ -129,6 +133,9 @@ SIGNATURES = {
     "ddq_create_table": (_i32, [_vp, ctypes.c_char_p, _i64, _i64, ctypes.POINTER(_i32)]),
     "ddq_load_column": (_i32, [_vp, _i32, ctypes.c_char_p, _i32, _vp, _i64, ctypes.POINTER(_i32)]),
     "ddq_find_column": (_i32, [_vp, ctypes.c_char_p, ctypes.c_char_p, ctypes.POINTER(_i32)]),
+    "ddq_set_dictionary": (_i32, [_vp, _i32, ctypes.POINTER(ctypes.c_char_p), _i32]),
+    "ddq_dictionary_range": (_i32, [_vp, _i32, ctypes.c_char_p, ctypes.POINTER(_i32), ctypes.POINTER(_i32)]),
+    "ddq_dictionary_like": (_i32, [_vp, _i32, ctypes.c_char_p, ctypes.POINTER(Pred)]),
     "ddq_cache_column": (_i32, [_vp, _i32]),
     "ddq_evict_column": (_i32, [_vp, _i32]),
     "ddq_column_is_cached": (_i32, [_vp, _i32]),

@@ -251,6 +251,9 @@ __global__ void __launch_bounds__(AG_NW * 32, 1) agg_ws_kernel(const __grid_cons
 #pragma unroll
         for (int j = 0; j < AG_ITEMS; j++) m |= ((uint64_t)(x[j] - pr.lo) <= pr.d64 ? 1u : 0u) << j;
         if (pr.empty) m = 0;
+      } else if (pr.kind == DDQ_PRED_BITSET) {
+#pragma unroll
+        for (int j = 0; j < AG_ITEMS; j++) m |= (bitset_hit(pr.in_vals, pr.lo, x[j]) ? 1u : 0u) << j;
       } else {
 #pragma unroll
         for (int j = 0; j < AG_ITEMS; j++) {
@@ -378,6 +381,7 @@ struct DenseAggParams {
 
 __device__ __forceinline__ bool pred_ok(const AggParams::Pred& p, long long v) {
   if (p.kind == DDQ_PRED_RANGE) return !p.empty && (uint64_t)(v - p.lo) <= p.d64;
+  if (p.kind == DDQ_PRED_BITSET) return bitset_hit(p.in_vals, p.lo, v);
   bool m = false;
 #pragma unroll
   for (int j = 0; j < 8; j++) m |= (j < p.n_in) && (v == p.in_vals[j]);

@@ -145,6 +145,7 @@ __device__ __forceinline__ void copy_out(const WsParams& P, const int32_t* ring,
 
 __device__ __forceinline__ bool pred_generic(const WsPred& p, int64_t v) {
   if (p.kind == DDQ_PRED_RANGE) return (uint64_t)(v - p.lo) <= p.d64 && !p.empty;
+  if (p.kind == DDQ_PRED_BITSET) return bitset_hit(p.in_vals, p.lo, v);
   bool m = false;
 #pragma unroll
   for (int j = 0; j < 8; j++) m |= (j < p.n_in) && (v == p.in_vals[j]);

@@ -16,6 +16,12 @@ __device__ __forceinline__ bool vec_cmp(int cmp, int32_t a, int32_t b) {
   return cmp == 1 ? a < b : cmp == 2 ? a != b : a == b;
 }
 
+// DDQ_PRED_BITSET membership (include/ddq.h): bit (v - lo) of a 512-bit mask
+__device__ __forceinline__ bool bitset_hit(const int64_t* words, int64_t lo, int64_t v) {
+  const uint64_t o = (uint64_t)(v - lo);
+  return o < 512 && ((uint64_t)words[o >> 6] >> (o & 63)) & 1;
+}
+
 __device__ __forceinline__ int4 ld_stream_i4(const void* p) {
   int4 r;
   asm volatile("ld.global.nc.L1::no_allocate.v4.s32 {%0,%1,%2,%3}, [%4];"

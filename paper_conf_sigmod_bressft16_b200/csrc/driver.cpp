@@ -272,6 +272,18 @@ static int host_threads(ddq_db* db) {
   return std::max(1, t);
 }
 
+// one predicate of the plan IR on a host value (RANGE, IN, BITSET; include/ddq.h)
+static inline bool host_pred(const ddq_pred& pr, int64_t v) {
+  if (pr.kind == DDQ_PRED_RANGE) return v >= pr.lo && v <= pr.hi;
+  if (pr.kind == DDQ_PRED_BITSET) {
+    const uint64_t o = (uint64_t)(v - pr.lo);
+    return o < 512 && (((uint64_t)pr.in_vals[o >> 6] >> (o & 63)) & 1);
+  }
+  bool m = false;
+  for (int j = 0; j < pr.n_in && j < DDQ_MAX_IN; j++) m |= v == pr.in_vals[j];
+  return m;
+}
+
 static inline int64_t hcol(const Column* c, int64_t r) {
   return c->width == 8 ? ((const int64_t*)c->host)[r] : (int64_t)((const int32_t*)c->host)[r];
 }
@@ -324,12 +336,7 @@ ddq_status run_host_op(ddq_db* db, const ddq_op& op, const std::vector<Inter>& I
             const int64_t v = hcol(ts[(size_t)j].col, r);
             if (op.term_kind[j] == DDQ_TERM_PRED) {
               const ddq_pred& pr = op.preds[j];
-              if (pr.kind == DDQ_PRED_RANGE) ok = v >= pr.lo && v <= pr.hi;
-              else {
-                bool m = false;
-                for (int x = 0; x < pr.n_in; x++) m |= v == pr.in_vals[x];
-                ok = m;
-              }
+              ok = host_pred(pr, v);
               continue;
             }
             const Inter& B = *ts[(size_t)j].b;
@@ -419,12 +426,7 @@ ddq_status run_host_op(ddq_db* db, const ddq_op& op, const std::vector<Inter>& I
             for (int p = 0; p < op.n_preds && ok; p++) {
               int64_t v = hcol(pc[(size_t)p], r);
               const ddq_pred& pr = op.preds[p];
-              if (pr.kind == DDQ_PRED_RANGE) ok = v >= pr.lo && v <= pr.hi;
-              else {
-                bool m = false;
-                for (int j = 0; j < pr.n_in; j++) m |= v == pr.in_vals[j];
-                ok = m;
-              }
+              ok = host_pred(pr, v);
             }
             if (ok) S.push_back(i);
           } else {
@@ -489,13 +491,7 @@ ddq_status run_host_op(ddq_db* db, const ddq_op& op, const std::vector<Inter>& I
         for (int p = 0; p < op.n_preds && ok; p++) {
           const int64_t v = hcol(bpc[(size_t)p], r);
           const ddq_pred& pr = op.preds[p];
-          if (pr.kind == DDQ_PRED_RANGE) {
-            ok = v >= pr.lo && v <= pr.hi;
-          } else {
-            bool m = false;
-            for (int j = 0; j < pr.n_in; j++) m |= v == pr.in_vals[j];
-            ok = m;
-          }
+          ok = host_pred(pr, v);
         }
         if (!ok) continue;
         int32_t k = ((const int32_t*)kc->host)[r];
@@ -585,13 +581,7 @@ ddq_status run_host_op(ddq_db* db, const ddq_op& op, const std::vector<Inter>& I
         for (int p = 0; p < op.n_preds && ok; p++) {
           const int64_t v = hcol(apc[(size_t)p], r);
           const ddq_pred& pr = op.preds[p];
-          if (pr.kind == DDQ_PRED_RANGE) {
-            ok = v >= pr.lo && v <= pr.hi;
-          } else {
-            bool m = false;
-            for (int j = 0; j < pr.n_in; j++) m |= v == pr.in_vals[j];
-            ok = m;
-          }
+          ok = host_pred(pr, v);
         }
         if (!ok) continue;
         int64_t key = 0;
@@ -762,6 +752,7 @@ static void finish_query(ddq_db* db, QueryState& q) {
       res->tids = t;
     }
   }
+  if (s == DDQ_OK && res) decode_result_keys(db, q.plan, res);
   for (auto& x : q.inters) release_inter(db, x);
   std::lock_guard<std::mutex> g(q.mu);
   q.status = s;

@@ -616,8 +616,9 @@ static inline __int128 acc128(const int64_t* accs, int64_t g, int n_aggs, int a)
 static ddq_status finalize_unique(const ddq_op& root, int64_t n_groups, const int64_t* keys, const int64_t* accs,
                                   ddq_result** out);
 
-// Merge equal packed keys (partials of several shards, S8(e)) by exact int128
-// addition, then finalise.
+// Merge equal packed keys (partials of several shards, S8(e)) per aggregate kind:
+// SUM / COUNT kinds by exact int128 addition, MIN by taking the smaller value (the
+// merge of per-shard minima is the minimum); then finalise.
 ddq_status finalize_result(const ddq_op& root, int64_t n_groups, const int64_t* keys, const int64_t* accs,
                            ddq_result** out) {
   const int na = root.n_aggs;
@@ -639,13 +640,11 @@ ddq_status finalize_result(const ddq_op& root, int64_t n_groups, const int64_t* 
     } else {
       const size_t m = mk.size() - 1;
       for (int a = 0; a < na; a++) {
-        unsigned __int128 x = ((unsigned __int128)(uint64_t)ma[(m * na + a) * 2 + 1] << 64) |
-                              (uint64_t)ma[(m * na + a) * 2];
-        unsigned __int128 y = ((unsigned __int128)(uint64_t)accs[(g * na + a) * 2 + 1] << 64) |
-                              (uint64_t)accs[(g * na + a) * 2];
-        x += y;
-        ma[(m * na + a) * 2] = (int64_t)(uint64_t)x;
-        ma[(m * na + a) * 2 + 1] = (int64_t)(uint64_t)(x >> 64);
+        __int128 x = acc128(ma.data(), (int64_t)m, na, a), y = acc128(accs, g, na, a);
+        if (root.agg_kind[a] == DDQ_AGG_MIN) x = std::min(x, y);
+        else x = (__int128)((unsigned __int128)x + (unsigned __int128)y);
+        ma[(m * na + a) * 2] = (int64_t)(uint64_t)(unsigned __int128)x;
+        ma[(m * na + a) * 2 + 1] = (int64_t)(uint64_t)((unsigned __int128)x >> 64);
       }
     }
   }
@@ -655,6 +654,23 @@ ddq_status finalize_result(const ddq_op& root, int64_t n_groups, const int64_t* 
 static ddq_status finalize_unique(const ddq_op& root, int64_t n_groups, const int64_t* keys, const int64_t* accs,
                                   ddq_result** out) {
   const int nk = root.n_keys, na = root.n_aggs;
+  if (root.n_avg < 0 || root.n_avg > 4) return set_error(DDQ_EINVAL, "finalize: n_avg must be 0..4");
+  for (int k = 0; k < root.n_avg; k++)
+    if (root.avg_sum[k] < 0 || root.avg_sum[k] >= na || root.avg_count < 0 || root.avg_count >= na ||
+        root.agg_kind[root.avg_count] != DDQ_AGG_COUNT || root.avg_scale[k] < 0 || root.avg_scale[k] > 18)
+      return set_error(DDQ_EINVAL, "finalize: bad AVG operands (sum aggregate, COUNT aggregate, scale 0..18)");
+  // an aggregate without GROUP BY has exactly one row, also over an empty input
+  // (reading O7: its SUMs / MINs are then SQL NULL, its COUNTs 0)
+  std::vector<int64_t> zero_acc;
+  bool empty_ungrouped = false;
+  if (nk == 0 && n_groups == 0) {
+    static const int64_t zero_key = 0;
+    zero_acc.assign((size_t)std::max(na, 1) * 2, 0);
+    keys = &zero_key;
+    accs = zero_acc.data();
+    n_groups = 1;
+    empty_ungrouped = true;
+  }
   std::vector<int64_t> idx((size_t)n_groups);
   std::iota(idx.begin(), idx.end(), 0);
   int shift[DDQ_MAX_KEYS], bits[DDQ_MAX_KEYS];
@@ -688,12 +704,21 @@ static ddq_status finalize_unique(const ddq_op& root, int64_t n_groups, const in
   std::memset(r, 0, sizeof(*r));
   int64_t* k = new int64_t[(size_t)std::max<int64_t>(1, n * nk)];
   int64_t* a = new int64_t[(size_t)std::max<int64_t>(1, n * na * 2)];
+  uint8_t* nul = new uint8_t[(size_t)std::max<int64_t>(1, n * na)];
+  double* av = root.n_avg > 0 ? new double[(size_t)std::max<int64_t>(1, n * root.n_avg)] : nullptr;
   for (int64_t i = 0; i < n; i++) {
     int64_t g = idx[(size_t)i];
     for (int j = 0; j < nk; j++) k[i * nk + j] = keyk(g, j);
     for (int j = 0; j < na; j++) {
       a[(i * na + j) * 2] = accs[(g * na + j) * 2];
       a[(i * na + j) * 2 + 1] = accs[(g * na + j) * 2 + 1];
+      nul[i * na + j] = empty_ungrouped && root.agg_kind[j] != DDQ_AGG_COUNT ? 1 : 0;
+    }
+    // AVG = SUM / COUNT / 10^scale in double (reading O10): NULL (NaN) for no rows
+    for (int j = 0; j < root.n_avg; j++) {
+      const __int128 cnt = acc128(accs, g, na, root.avg_count);
+      const __int128 sum = acc128(accs, g, na, root.avg_sum[j]);
+      av[i * root.n_avg + j] = cnt == 0 ? std::nan("") : (double)sum / (double)cnt / std::pow(10.0, root.avg_scale[j]);
     }
   }
   r->n_rows = n;
@@ -701,8 +726,74 @@ static ddq_status finalize_unique(const ddq_op& root, int64_t n_groups, const in
   r->n_aggs = na;
   r->keys = k;
   r->aggs = a;
+  r->agg_null = nul;
+  r->n_avg = root.n_avg;
+  r->avgs = av;
   *out = r;
   return DDQ_OK;
+}
+
+// Aligned vectors of op i's output, mirroring run_gpu_op / run_host_op: carried
+// input vectors first (in order), then the vector the op appends -- a probe's
+// emitted payload, a GATHER's column (or a fetch's payload); a STAR emits its
+// probe terms' payloads in term order.
+static int vec_count(const ddq_plan& plan, int i) {
+  if (i < 0 || i >= plan.n_ops) return 0;
+  const ddq_op& op = plan.ops[i];
+  if (op.kind == DDQ_OP_STAR) {
+    int e = 0;
+    for (int j = 0; j < op.n_terms && j < 4; j++) e += op.term_kind[j] == DDQ_TERM_PROBE && op.term_emit[j];
+    return e;
+  }
+  if (op.kind == DDQ_OP_HASH_BUILD || op.kind == DDQ_OP_AGGREGATE) return 0;
+  const int base = op.input >= 0 && op.input < i ? vec_count(plan, op.input) : 0;
+  if ((op.kind == DDQ_OP_HASH_PROBE && op.emit_payload) || op.kind == DDQ_OP_GATHER) return base + 1;
+  return base;
+}
+
+// Column behind aligned vector v of op i's output (-1: a dimension row id or unknown).
+static int vec_column(const ddq_plan& plan, int i, int v) {
+  if (i < 0 || i >= plan.n_ops || v < 0) return -1;
+  const ddq_op& op = plan.ops[i];
+  auto payload_of = [&](int b) { return b >= 0 && b < i ? plan.ops[b].payload_col : -1; };
+  if (op.kind == DDQ_OP_STAR) {
+    for (int j = 0, e = 0; j < op.n_terms && j < 4; j++)
+      if (op.term_kind[j] == DDQ_TERM_PROBE && op.term_emit[j] && e++ == v) return payload_of(op.term_build[j]);
+    return -1;
+  }
+  const int base = op.input >= 0 && op.input < i ? vec_count(plan, op.input) : 0;
+  if (v < base) return vec_column(plan, op.input, v);
+  if (v == base && op.kind == DDQ_OP_HASH_PROBE && op.emit_payload) return payload_of(op.build);
+  if (v == base && op.kind == DDQ_OP_GATHER) return op.fetch_build > 0 ? payload_of(op.fetch_build - 1) : op.gather_col;
+  return -1;
+}
+
+void decode_result_keys(ddq_db* db, const ddq_plan& plan, ddq_result* r) {
+  if (!db || !r || plan.n_ops < 1 || r->n_keys <= 0 || r->key_str) return;
+  const ddq_op& root = plan.ops[plan.n_ops - 1];
+  if (root.kind != DDQ_OP_AGGREGATE) return;
+  const std::vector<std::string>* dict[DDQ_MAX_KEYS] = {nullptr, nullptr, nullptr};
+  bool any = false;
+  {
+    std::lock_guard<std::mutex> g(db->mu);
+    for (int k = 0; k < r->n_keys && k < DDQ_MAX_KEYS; k++) {
+      const int src = root.key_src[k];
+      const int c = src < -1 ? -2 - src : src >= 0 ? vec_column(plan, root.input, src) : -1;
+      if (c >= 0 && c < (int)db->cols.size() && !db->cols[(size_t)c]->dict.empty()) {
+        dict[k] = &db->cols[(size_t)c]->dict;  // set once before queries, never reallocated
+        any = true;
+      }
+    }
+  }
+  if (!any) return;
+  const char** ks = new const char*[(size_t)std::max<int64_t>(1, r->n_rows * r->n_keys)];
+  for (int64_t i = 0; i < r->n_rows; i++)
+    for (int k = 0; k < r->n_keys; k++) {
+      const int64_t code = r->keys[i * r->n_keys + k];
+      const std::vector<std::string>* d = k < DDQ_MAX_KEYS ? dict[k] : nullptr;
+      ks[i * r->n_keys + k] = d && code >= 0 && code < (int64_t)d->size() ? (*d)[(size_t)code].c_str() : nullptr;
+    }
+  r->key_str = ks;
 }
 
 }  // namespace ddq
@@ -870,6 +961,82 @@ ddq_status ddq_find_column(ddq_db* db, const char* table, const char* name, ddq_
       }
   }
   return set_error(DDQ_ENOTFOUND, std::string("column ") + table + "." + name);
+}
+
+ddq_status ddq_set_dictionary(ddq_db* db, ddq_column c, const char* const* sorted_strings, int32_t n) {
+  if (!db || n < 0 || (n > 0 && !sorted_strings)) return set_error(DDQ_EINVAL, "set_dictionary: null argument");
+  std::vector<std::string> d;
+  d.reserve((size_t)n);
+  for (int32_t i = 0; i < n; i++) {
+    if (!sorted_strings[i]) return set_error(DDQ_EINVAL, "set_dictionary: null string");
+    d.emplace_back(sorted_strings[i]);
+    if (i > 0 && !(d[(size_t)i - 1] < d[(size_t)i]))  // std::string compares bytewise (C locale)
+      return set_error(DDQ_EINVAL, "set_dictionary: strings not strictly ascending (bytewise)");
+  }
+  std::lock_guard<std::mutex> g(db->mu);
+  if (c < 0 || c >= (int)db->cols.size()) return set_error(DDQ_ENOTFOUND, "set_dictionary: bad column");
+  Column& col = *db->cols[(size_t)c];
+  if (col.width != 4) return set_error(DDQ_EINVAL, "set_dictionary: codes are int32");
+  if (col.n > 0 && (col.vmin < 0 || col.vmax >= (int64_t)n))
+    return set_error(DDQ_EINVAL, "set_dictionary: column holds codes outside the dictionary");
+  col.dict = std::move(d);
+  return DDQ_OK;
+}
+
+ddq_status ddq_dictionary_range(ddq_db* db, ddq_column c, const char* s, int32_t* lower, int32_t* upper) {
+  if (!db || !s || !lower || !upper) return set_error(DDQ_EINVAL, "dictionary_range: null argument");
+  std::lock_guard<std::mutex> g(db->mu);
+  if (c < 0 || c >= (int)db->cols.size()) return set_error(DDQ_ENOTFOUND, "dictionary_range: bad column");
+  const std::vector<std::string>& d = db->cols[(size_t)c]->dict;
+  if (d.empty()) return set_error(DDQ_ENOTFOUND, "dictionary_range: column has no dictionary");
+  *lower = (int32_t)(std::lower_bound(d.begin(), d.end(), std::string(s)) - d.begin());
+  *upper = (int32_t)(std::upper_bound(d.begin(), d.end(), std::string(s)) - d.begin());
+  return DDQ_OK;
+}
+
+// SQL LIKE: '%' matches any run of bytes, '_' exactly one byte (no escape character)
+static bool like_match(const char* s, const char* p) {
+  if (*p == 0) return *s == 0;
+  if (*p == '%') {
+    while (*p == '%') p++;
+    if (*p == 0) return true;
+    for (; *s; s++)
+      if (like_match(s, p)) return true;
+    return false;
+  }
+  if (*s == 0) return false;
+  return (*p == '_' || *p == *s) && like_match(s + 1, p + 1);
+}
+
+ddq_status ddq_dictionary_like(ddq_db* db, ddq_column c, const char* pattern, ddq_pred* out) {
+  if (!db || !pattern || !out) return set_error(DDQ_EINVAL, "dictionary_like: null argument");
+  std::lock_guard<std::mutex> g(db->mu);
+  if (c < 0 || c >= (int)db->cols.size()) return set_error(DDQ_ENOTFOUND, "dictionary_like: bad column");
+  const std::vector<std::string>& d = db->cols[(size_t)c]->dict;
+  if (d.empty()) return set_error(DDQ_ENOTFOUND, "dictionary_like: column has no dictionary");
+  std::vector<int64_t> hits;
+  for (size_t i = 0; i < d.size(); i++)
+    if (like_match(d[i].c_str(), pattern)) hits.push_back((int64_t)i);
+  std::memset(out, 0, sizeof(*out));
+  out->column = c;
+  if (hits.empty()) {  // matches nothing: an empty range
+    out->kind = DDQ_PRED_RANGE;
+    out->lo = 1;
+    out->hi = 0;
+    return DDQ_OK;
+  }
+  if (hits.size() <= DDQ_MAX_IN) {
+    out->kind = DDQ_PRED_IN;
+    out->n_in = (int32_t)hits.size();
+    for (size_t i = 0; i < hits.size(); i++) out->in_vals[i] = hits[i];
+    return DDQ_OK;
+  }
+  if (hits.back() - hits.front() >= 512) return set_error(DDQ_EINVAL, "dictionary_like: matches span > 512 codes");
+  out->kind = DDQ_PRED_BITSET;
+  out->lo = hits.front();
+  out->hi = hits.back();
+  for (int64_t h : hits) out->in_vals[(h - out->lo) >> 6] |= (int64_t)(1ull << ((h - out->lo) & 63));
+  return DDQ_OK;
 }
 
 }  // extern "C"
@@ -1101,6 +1268,9 @@ void ddq_result_free(ddq_result* r) {
   delete[] r->keys;
   delete[] r->aggs;
   delete[] r->tids;
+  delete[] r->agg_null;
+  delete[] r->avgs;
+  delete[] r->key_str;
   delete r;
 }
 
@@ -1153,6 +1323,15 @@ static ddq_status validate_plan(ddq_db* db, const ddq_plan* plan) {
       for (int k = 0; k < op.n_keys && k < DDQ_MAX_KEYS; k++) bits += op.key_bits[k] > 0 ? op.key_bits[k] : 21;
       if (bits > 63) return set_error(DDQ_EINVAL, "plan: packed group key wider than 63 bits");
     }
+    if (op.n_preds < 0 || op.n_preds > DDQ_MAX_PREDS) return set_error(DDQ_EINVAL, "plan: bad n_preds");
+    for (int k = 0; k < op.n_preds; k++) {
+      const ddq_pred& pr = op.preds[k];
+      if (pr.kind != DDQ_PRED_RANGE && pr.kind != DDQ_PRED_IN && pr.kind != DDQ_PRED_BITSET)
+        return set_error(DDQ_EINVAL, "plan: bad predicate kind");
+      if (pr.kind == DDQ_PRED_IN && (pr.n_in < 0 || pr.n_in > DDQ_MAX_IN))
+        return set_error(DDQ_EINVAL, "plan: IN list must hold 0..8 values");
+    }
+    if (op.kind == DDQ_OP_AGGREGATE && (op.n_avg < 0 || op.n_avg > 4)) return set_error(DDQ_EINVAL, "plan: n_avg 0..4");
     if (op.input >= i || op.input < -1) return set_error(DDQ_EINVAL, "plan: input must precede the op");
     if (op.kind == DDQ_OP_HASH_PROBE && (op.build < 0 || op.build >= i ||
                                          plan->ops[op.build].kind != DDQ_OP_HASH_BUILD))
@@ -1674,7 +1853,9 @@ ddq_status ddq_finalize_partials(const ddq_op* root, int64_t n, const int64_t* k
 ddq_status ddq_prepared_finalize(ddq_prepared* p, int64_t n_groups, const int64_t* h_keys, const int64_t* h_accs,
                                  ddq_result** out) {
   if (!p || !out) return set_error(DDQ_EINVAL, "prepared_finalize: null");
-  return finalize_result(p->plan.ops[p->plan.n_ops - 1], n_groups, h_keys, h_accs, out);
+  ddq_status s = finalize_result(p->plan.ops[p->plan.n_ops - 1], n_groups, h_keys, h_accs, out);
+  if (s == DDQ_OK) decode_result_keys(p->db, p->plan, *out);
+  return s;
 }
 
 ddq_status ddq_prepared_fetch(ddq_prepared* p, void* stream, ddq_result** out) {
@@ -1713,7 +1894,10 @@ ddq_status ddq_prepared_fetch(ddq_prepared* p, void* stream, ddq_result** out) {
   int64_t g = 0;
   if (ddq_status s = ddq_prepared_partials(p, stream, &g, keys.data(), accs.data(), r.gb_cap)) return s;
   ddq_status s = finalize_result(root, g, keys.data(), accs.data(), out);
-  if (s == DDQ_OK) (*out)->gpu_ops = p->plan.n_ops;
+  if (s == DDQ_OK) {
+    (*out)->gpu_ops = p->plan.n_ops;
+    decode_result_keys(p->db, p->plan, *out);
+  }
   return s;
 }
 

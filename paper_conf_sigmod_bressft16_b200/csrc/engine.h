@@ -61,6 +61,8 @@ struct Column {
   bool evict_pending = false;
   bool on_demand = false;   // cached by operator-driven placement (GPU-only arm)
   bool loading = false;     // H2D copy in flight (db->mu released; waiters use cache_cv)
+  // order-preserving dictionary (reading O4): code = index; set once, read-only after
+  std::vector<std::string> dict;
 };
 
 struct Table {
@@ -179,6 +181,8 @@ void release_inter(ddq_db* db, Inter& x);
 ddq_status inter_to_host(ddq_db* db, Inter& x, cudaStream_t st);
 ddq_status finalize_result(const ddq_op& root, int64_t n_groups, const int64_t* keys, const int64_t* accs,
                            ddq_result** out);
+// S8(a7) decode: attach the dictionary strings of the result's keys (key_str)
+void decode_result_keys(ddq_db* db, const ddq_plan& plan, ddq_result* r);
 int64_t pow2_at_least(int64_t x);
 const ddq::Column* col_of(ddq_db* db, int c);
 

@@ -74,6 +74,7 @@ struct FilterParams {
 
 __device__ __forceinline__ bool eval_pred(const DevPredK& p, int64_t v) {
   if (p.kind == 1) return v >= p.lo && v <= p.hi;
+  if (p.kind == DDQ_PRED_BITSET) return bitset_hit(p.in_vals, p.lo, v);
   bool m = false;
 #pragma unroll
   for (int j = 0; j < 8; j++) m |= (j < p.n_in) && (v == p.in_vals[j]);

@@ -40,6 +40,8 @@ __device__ __forceinline__ bool build_row_passes(const BuildPreds& bp, int32_t r
     bool m = false;
     if (p.kind == DDQ_PRED_RANGE) {
       m = v >= p.lo && v <= p.hi;
+    } else if (p.kind == DDQ_PRED_BITSET) {
+      m = bitset_hit(p.in_vals, p.lo, v);
     } else {
 #pragma unroll
       for (int j = 0; j < DDQ_MAX_IN; j++) m |= j < p.n_in && v == p.in_vals[j];

@@ -42,7 +42,7 @@ ddq_status ddq_op_select(const ddq_dev_pred* preds, int32_t n_preds, const int32
   for (int i = 0; i < n_preds; i++) {
     if ((n_cap > 0 && !preds[i].col) || (preds[i].width != 4 && preds[i].width != 8))
       return set_error(DDQ_EINVAL, "select: predicate column must be non-null int32/int64");
-    if (preds[i].kind != DDQ_PRED_RANGE && preds[i].kind != DDQ_PRED_IN)
+    if (preds[i].kind != DDQ_PRED_RANGE && preds[i].kind != DDQ_PRED_IN && preds[i].kind != DDQ_PRED_BITSET)
       return set_error(DDQ_EINVAL, "select: bad predicate kind");
     if (preds[i].kind == DDQ_PRED_IN && (preds[i].n_in < 0 || preds[i].n_in > DDQ_MAX_IN))
       return set_error(DDQ_EINVAL, "select: IN list too long");
@@ -123,7 +123,7 @@ ddq_status ddq_op_star(const ddq_dev_term* terms, int32_t n_terms, int64_t n_row
     if ((n_rows > 0 && !t.col) || ((uintptr_t)t.col & 15)) return set_error(DDQ_EINVAL, "star: column must be 16-byte aligned");
     if (t.width != 4 && t.width != 8) return set_error(DDQ_EINVAL, "star: bad width");
     if (t.kind == DDQ_TERM_PRED) {
-      if (t.pred_kind != DDQ_PRED_RANGE && t.pred_kind != DDQ_PRED_IN) return set_error(DDQ_EINVAL, "star: bad predicate");
+      if (t.pred_kind != DDQ_PRED_RANGE && t.pred_kind != DDQ_PRED_IN && t.pred_kind != DDQ_PRED_BITSET) return set_error(DDQ_EINVAL, "star: bad predicate");
       if (t.pred_kind == DDQ_PRED_IN && (t.n_in < 0 || t.n_in > DDQ_MAX_IN)) return set_error(DDQ_EINVAL, "star: IN list too long");
     } else {
       if (t.width != 4) return set_error(DDQ_EINVAL, "star: probe keys are int32");

@@ -134,6 +134,7 @@ __device__ __forceinline__ void issue_tile(const ScanParams& P, uint32_t n, uint
 
 __device__ __forceinline__ bool scan_pred(const ScanPred& p, int64_t v) {
   if (p.kind == DDQ_PRED_RANGE) return v >= p.lo && v <= p.hi;
+  if (p.kind == DDQ_PRED_BITSET) return bitset_hit(p.in_vals, p.lo, v);
   bool m = false;
 #pragma unroll
   for (int j = 0; j < 8; j++) m |= (j < p.n_in) && (v == p.in_vals[j]);

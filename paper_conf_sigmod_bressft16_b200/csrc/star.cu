@@ -94,6 +94,7 @@ __device__ __forceinline__ void st_issue(const StarParams& P, uint8_t* buf, uint
 
 __device__ __forceinline__ bool st_pred(const StarTerm& p, int64_t v) {
   if (p.pred_kind == DDQ_PRED_RANGE) return v >= p.lo && v <= p.hi;
+  if (p.pred_kind == DDQ_PRED_BITSET) return bitset_hit(p.in_vals, p.lo, v);
   bool m = false;
 #pragma unroll
   for (int j = 0; j < 8; j++) m |= (j < p.n_in) && (v == p.in_vals[j]);

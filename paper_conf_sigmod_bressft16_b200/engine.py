@@ -18,9 +18,13 @@ from ._abi import check, lib
 
 @dataclass
 class QueryResult:
-    """Rows (keys..., aggregates...) as Python ints, in ORDER BY order, or TIDs."""
+    """Rows (keys..., aggregates...) as Python ints (None = SQL NULL, reading O7), in
+    ORDER BY order, or TIDs.  avgs: per row the AVG columns (reading O10); decoded:
+    rows with dictionary-coded keys replaced by their strings (S8(a7))."""
     rows: list = field(default_factory=list)
     tids: np.ndarray | None = None
+    avgs: list = field(default_factory=list)
+    decoded: list = field(default_factory=list)
     n_keys: int = 0
     n_aggs: int = 0
     gpu_ops: int = 0
@@ -40,10 +44,19 @@ def _convert(res_ptr) -> QueryResult:
     for i in range(r.n_rows):
         vals = [int(r.keys[i * nk + k]) for k in range(nk)]
         for a in range(na):
+            if r.agg_null and r.agg_null[i * na + a]:
+                vals.append(None)
+                continue
             lo = r.aggs[(i * na + a) * 2] & 0xFFFFFFFFFFFFFFFF
             hi = r.aggs[(i * na + a) * 2 + 1]
             vals.append((hi << 64) | lo)
         out.rows.append(tuple(vals))
+        if r.n_avg > 0:
+            out.avgs.append(tuple(float(r.avgs[i * r.n_avg + k]) for k in range(r.n_avg)))
+        if r.key_str:
+            ks = [r.key_str[i * nk + k] for k in range(nk)]
+            out.decoded.append(tuple(ks[k].decode() if ks[k] is not None else vals[k] for k in range(nk))
+                               + tuple(vals[nk:]))
     lib().ddq_result_free(res_ptr)
     return out
 
@@ -86,6 +99,9 @@ class PlanBuilder:
         op.n_preds = len(preds)
         for i, p in enumerate(preds):
             pr = op.preds[i]
+            if isinstance(p, A.Pred):  # a predicate built by the library (Database.like)
+                ctypes.memmove(ctypes.byref(pr), ctypes.byref(p), ctypes.sizeof(A.Pred))
+                continue
             pr.column = self.db.col(table, p[0])
             if len(p) == 3:
                 pr.kind, pr.lo, pr.hi = A.PRED_RANGE, int(p[1]), int(p[2])
@@ -181,7 +197,7 @@ class PlanBuilder:
 
     def aggregate(self, table: str, input: int, keys: list, aggs: list, order_by: list | None = None,
                   max_groups: int = 0, limit: int = 0, key_bits: list | None = None,
-                  where: list | None = None) -> int:
+                  where: list | None = None, avg: list | None = None, avg_count: int = -1) -> int:
         """keys: int (aligned vector index) or str (column of `table`).
         aggs: (kind, [cols]).  order_by: ints per include/ddq.h (+/-(1+k), +/-(101+a)).
         key_bits: bits per key in the packed group key (default 21 each, sum <= 63).
@@ -206,6 +222,15 @@ class PlanBuilder:
             op.order_by[i] = o
         op.max_groups = max_groups
         op.limit = limit
+        # AVG columns computed at finalisation: (index of the SUM aggregate, decimal scale)
+        # over the COUNT aggregate avg_count (reading O10)
+        avg = avg or []
+        if len(avg) > 4:
+            raise ValueError("at most 4 AVG columns")
+        op.n_avg = len(avg)
+        op.avg_count = avg_count
+        for k, (a, scale) in enumerate(avg):
+            op.avg_sum[k], op.avg_scale[k] = a, scale
         return idx
 
 
@@ -371,6 +396,25 @@ class Database:
                                     data.size, ctypes.byref(c)))
         self._cols[(table, name)] = c.value
         return c.value
+
+    def set_dictionary(self, table: str, name: str, strings: list[str]) -> None:
+        """Order-preserving dictionary of a string column (codes = ranks, reading O4)."""
+        enc = [x.encode() for x in strings]
+        arr = (ctypes.c_char_p * max(len(enc), 1))(*enc)
+        check(lib().ddq_set_dictionary(self.h, self.col(table, name), arr, len(enc)))
+
+    def dictionary_range(self, table: str, name: str, s: str) -> tuple[int, int]:
+        """[lower, upper) codes of string s in the column's dictionary."""
+        lo, hi = ctypes.c_int32(), ctypes.c_int32()
+        check(lib().ddq_dictionary_range(self.h, self.col(table, name), s.encode(), ctypes.byref(lo),
+                                         ctypes.byref(hi)))
+        return lo.value, hi.value
+
+    def like(self, table: str, name: str, pattern: str) -> A.Pred:
+        """SQL `name LIKE pattern` folded over the dictionary into a code predicate."""
+        pr = A.Pred()
+        check(lib().ddq_dictionary_like(self.h, self.col(table, name), pattern.encode(), ctypes.byref(pr)))
+        return pr
 
     def table_id(self, table: str) -> int:
         return self._tables[table]

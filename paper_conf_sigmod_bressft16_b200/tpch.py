@@ -8,7 +8,6 @@ from . import _abi as A
 from .engine import Database, PlanBuilder
 from .ssb import code
 
-import numpy as np
 
 TPCH_QUERIES = ["tpch1", "tpch3", "tpch4", "tpch5", "tpch6", "tpch7"]
 
@@ -20,6 +19,7 @@ TABLE_COLUMNS = {
     "orders": ["o_orderkey", "o_custkey", "o_orderdate", "o_shippriority", "o_orderpriority"],
     "lineitem": ["l_orderkey", "l_suppkey", "l_quantity", "l_extendedprice", "l_discount", "l_tax",
                  "l_returnflag", "l_linestatus", "l_shipdate", "l_commitdate", "l_receiptdate"],
+    "calendar": ["d_datekey", "d_year"],  # datagen's date dimension (reading O34)
 }
 STRING_DICTS = {"n_name": "nation", "r_name": "region", "c_mktsegment": "mktsegment",
                 "l_returnflag": "returnflag", "l_linestatus": "linestatus",
@@ -31,22 +31,10 @@ QUERY_TABLES = {"tpch1": ["lineitem"], "tpch6": ["lineitem"],
                 "tpch5": ["region", "nation", "supplier", "customer", "orders", "lineitem"]}
 
 
-def calendar_table() -> dict:
-    """The date dimension (one row per day 1992-01-01 .. 1998-12-31, TPC-H's date
-    domain): d_datekey (int yyyymmdd, reading O11) and d_year.  extract(year from
-    l_shipdate) of Q7 is a join of l_shipdate with it (reading O36), as SSB's
-    lo_orderdate joins its date table."""
-    days = np.arange(np.datetime64("1992-01-01"), np.datetime64("1999-01-01"))
-    y = days.astype("datetime64[Y]").astype(np.int64) + 1970
-    m = days.astype("datetime64[M]").astype(np.int64) % 12 + 1
-    d = (days - days.astype("datetime64[M]")).astype(np.int64) + 1
-    return {"d_datekey": (y * 10000 + m * 100 + d).astype(np.int32), "d_year": y.astype(np.int32)}
-
-
 def load_tpch(db: Database, data, cache: bool = True, tables=None) -> None:
     """data: ``data.col(table, col)``, ``data.rows(table)``, ``data.dict_for(col)``."""
-    for t in (tables or list(TABLE_COLUMNS) + ["calendar"]):
-        cols = calendar_table() if t == "calendar" else {c: data.col(t, c) for c in TABLE_COLUMNS[t]}
+    for t in (tables or list(TABLE_COLUMNS)):
+        cols = {c: data.col(t, c) for c in TABLE_COLUMNS[t]}
         db.create_table(t, len(next(iter(cols.values()))))
         for c, v in cols.items():
             db.load_column(t, c, v)
@@ -54,6 +42,9 @@ def load_tpch(db: Database, data, cache: bool = True, tables=None) -> None:
                 db.cache(t, c)
     for c, d in STRING_DICTS.items():
         db.dicts[d] = data.dict_for(c)
+        t = next(t for t, cols in TABLE_COLUMNS.items() if c in cols)
+        if tables is None or t in tables:
+            db.set_dictionary(t, c, db.dicts[d])  # decode result keys (S8(a7))
 
 
 def tpch_plan(db: Database, q: str, limit: int = 0, dense: bool = True) -> PlanBuilder:
@@ -72,7 +63,9 @@ def tpch_plan(db: Database, q: str, limit: int = 0, dense: bool = True) -> PlanB
                           (A.AGG_SUM_MUL_100M_100P, ["l_extendedprice", "l_discount", "l_tax"]),
                           (A.AGG_SUM, ["l_discount"]), (A.AGG_COUNT, [])],
                     order_by=[1, 2], max_groups=6,
-                    key_bits=[2, 1])  # dictionary codes: returnflag A/N/R, linestatus F/O
+                    key_bits=[2, 1],  # dictionary codes: returnflag A/N/R, linestatus F/O
+                    # avg_qty, avg_price, avg_disc = sum / count / 10^2 at finalisation (O10)
+                    avg=[(0, 2), (1, 2), (4, 2)], avg_count=5)
         return P
     if q == "tpch6":
         # shipdate in 1994 (15 %) first; discount 0.05..0.07 and quantity < 24 at its TIDs

@@ -10,13 +10,15 @@
 --       date '1993-07-01' + interval '3' month = 19931001,
 --       extract(year from l_shipdate) = l_shipdate / 10000.
 --   avg(x) is reported as sum(x) and count(*) (O10: the average is a double
---   computed at finalisation).  Q1's avg_disc uses sum(l_discount).
+--   computed at finalisation).  Q1's avg_disc uses sum(l_discount).  Q1 also
+--   reports SQLite's own avg(x) of the scale-2 integers (the tests divide by 100),
+--   which pins the oracle's AVG columns.
 --   LIMIT 10 of Q3 is dropped here so the whole pre-LIMIT group set is compared (O9).
 -- Used by tests/test_oracle_sqlite.py (SQLite 3.45) to pin the oracle.
 -- @tpch1
 select l_returnflag, l_linestatus, sum(l_quantity), sum(l_extendedprice),
        sum(l_extendedprice*(100-l_discount)), sum(l_extendedprice*(100-l_discount)*(100+l_tax)),
-       sum(l_discount), count(*)
+       sum(l_discount), count(*), avg(l_quantity), avg(l_extendedprice), avg(l_discount)
   from lineitem where l_shipdate <= 19980902
  group by l_returnflag, l_linestatus order by l_returnflag, l_linestatus;
 -- @tpch3

@@ -46,8 +46,10 @@ int main(void) {
   O(ddq_op, preds) O(ddq_op, key_col) O(ddq_op, agg_col) O(ddq_op, max_groups) O(ddq_op, order_by)
   O(ddq_op, limit) O(ddq_config, cache_bytes) O(ddq_config, fault_alloc_every) O(ddq_result, exec_ms)
   O(ddq_dev_pred, in_vals) O(ddq_dev_agg, arg) O(ddq_op, eq_cmp) O(ddq_op, build_key_set)
+  O(ddq_op, n_avg) O(ddq_op, avg_scale) O(ddq_result, agg_null) O(ddq_result, avgs) O(ddq_result, key_str)
   printf("DDQ_CMP_EQ %d\nDDQ_CMP_LT %d\nDDQ_CMP_NE %d\nDDQ_AGG_MIN %d\nDDQ_AGG_COUNT %d\n",
          DDQ_CMP_EQ, DDQ_CMP_LT, DDQ_CMP_NE, (int)DDQ_AGG_MIN, (int)DDQ_AGG_COUNT);
+  printf("DDQ_PRED_BITSET %d\n", (int)DDQ_PRED_BITSET);
   return 0;
 }
 """
@@ -63,7 +65,7 @@ def test_struct_layouts_match_c(tmp_path):
     py = {"ddq_dev_pred": A.DevPred, "ddq_dev_agg": A.DevAgg, "ddq_config": A.Config, "ddq_pred": A.Pred,
           "ddq_op": A.Op, "ddq_plan": A.Plan, "ddq_result": A.Result, "ddq_stats": A.Stats}
     consts = {"DDQ_CMP_EQ": A.CMP_EQ, "DDQ_CMP_LT": A.CMP_LT, "DDQ_CMP_NE": A.CMP_NE,
-              "DDQ_AGG_MIN": A.AGG_MIN, "DDQ_AGG_COUNT": A.AGG_COUNT}
+              "DDQ_AGG_MIN": A.AGG_MIN, "DDQ_AGG_COUNT": A.AGG_COUNT, "DDQ_PRED_BITSET": A.PRED_BITSET}
     for k, v in got.items():
         if k in consts:
             assert consts[k] == int(v), k

@@ -1,0 +1,122 @@
+"""Host finalisation (S8(a7)) through the C ABI, no GPU needed: ddq_finalize_partials
+is the merge + ORDER BY / LIMIT step every query result passes through (P:256:
+"once the root operator ... finished, the query result is returned").
+
+Pins (closed forms, not a retyped formula):
+  * the merge of per-shard partial groups equals the single-shard result: SUM / COUNT
+    add, MIN takes the smaller (the merge used to add minima);
+  * reading O7: an aggregate without GROUP BY over no rows is ONE row, COUNT 0 and
+    SUM / MIN SQL NULL; a grouped aggregate over no rows is no row;
+  * reading O10: AVG = sum / count / 10^scale as a double, NULL (NaN) at count 0,
+    compared with exact rational arithmetic (fractions.Fraction) at rel 1e-15.
+"""
+import ctypes
+import math
+from fractions import Fraction
+
+import numpy as np
+import pytest
+
+
+def _root(kinds, n_keys=0, key_bits=(), order_by=(), limit=0, avg=(), avg_count=-1):
+    from paper_conf_sigmod_bressft16_b200 import _abi as A
+    op = A.Op()
+    ctypes.memset(ctypes.addressof(op), 0, ctypes.sizeof(op))
+    op.kind = A.OP_AGGREGATE
+    op.input = -1
+    op.n_keys = n_keys
+    for k, b in enumerate(key_bits):
+        op.key_bits[k] = b
+    op.n_aggs = len(kinds)
+    for a, k in enumerate(kinds):
+        op.agg_kind[a] = k
+    op.n_order = len(order_by)
+    for i, o in enumerate(order_by):
+        op.order_by[i] = o
+    op.limit = limit
+    op.n_avg = len(avg)
+    op.avg_count = avg_count
+    for k, (a, s) in enumerate(avg):
+        op.avg_sum[k], op.avg_scale[k] = a, s
+    return op
+
+
+def _accs(rows):
+    """rows: list of lists of Python ints (int128 each) -> int64 (lo, hi) words."""
+    out = []
+    for r in rows:
+        for v in r:
+            u = v & ((1 << 128) - 1)
+            lo, hi = u & ((1 << 64) - 1), u >> 64
+            out += [lo - (1 << 64) if lo >= 1 << 63 else lo, hi - (1 << 64) if hi >= 1 << 63 else hi]
+    return np.array(out, np.int64)
+
+
+def test_merge_per_aggregate_kind():
+    from paper_conf_sigmod_bressft16_b200 import _abi as A
+    from paper_conf_sigmod_bressft16_b200.engine import finalize_partials
+    root = _root([A.AGG_SUM, A.AGG_MIN, A.AGG_COUNT], n_keys=1, key_bits=[8], order_by=[1])
+    # group 3 appears in three shards, group 5 in one; values beyond int64 to exercise int128
+    keys = np.array([3, 5, 3, 3], np.int64)
+    big = 1 << 70
+    accs = _accs([[big, 40, 2], [7, -9, 1], [5, 12, 3], [-1, 17, 4]])
+    r = finalize_partials(root, keys, accs)
+    assert r.rows == [(3, big + 5 - 1, 12, 9), (5, 7, -9, 1)]
+
+
+def test_ungrouped_empty_is_one_null_row():
+    from paper_conf_sigmod_bressft16_b200 import _abi as A
+    from paper_conf_sigmod_bressft16_b200.engine import finalize_partials
+    root = _root([A.AGG_SUM_MUL, A.AGG_COUNT, A.AGG_MIN])
+    r = finalize_partials(root, np.zeros(0, np.int64), np.zeros(0, np.int64))
+    assert r.rows == [(None, 0, None)]
+    # non-empty: no NULLs
+    r = finalize_partials(root, np.zeros(1, np.int64), _accs([[42, 3, -5]]))
+    assert r.rows == [(42, 3, -5)]
+
+
+def test_grouped_empty_has_no_rows():
+    from paper_conf_sigmod_bressft16_b200 import _abi as A
+    from paper_conf_sigmod_bressft16_b200.engine import finalize_partials
+    root = _root([A.AGG_SUM], n_keys=2, key_bits=[4, 4], order_by=[1, 2])
+    r = finalize_partials(root, np.zeros(0, np.int64), np.zeros(0, np.int64))
+    assert r.rows == []
+
+
+def test_avg_columns():
+    from paper_conf_sigmod_bressft16_b200 import _abi as A
+    from paper_conf_sigmod_bressft16_b200.engine import finalize_partials
+    # TPC-H Q1 shape: sum_qty, sum_price, sum_disc, count; avg over scale-2 decimals
+    root = _root([A.AGG_SUM, A.AGG_SUM, A.AGG_SUM, A.AGG_COUNT], n_keys=1, key_bits=[2], order_by=[1],
+                 avg=[(0, 2), (1, 2), (2, 2)], avg_count=3)
+    rng = np.random.default_rng(7)
+    sums = [[int(rng.integers(1, 1 << 60)) * 1000 + 7, (1 << 66) + 12345, int(rng.integers(0, 1000)),
+             int(rng.integers(1, 1 << 40))] for _ in range(3)]
+    r = finalize_partials(root, np.arange(3, dtype=np.int64), _accs(sums))
+    assert len(r.avgs) == 3
+    for g, s in enumerate(sums):
+        for k, a in enumerate((0, 1, 2)):
+            exact = Fraction(s[a], s[3] * 100)
+            assert r.avgs[g][k] == pytest.approx(float(exact), rel=1e-15)
+    # count 0 -> NULL (NaN) for an ungrouped AVG
+    root = _root([A.AGG_SUM, A.AGG_COUNT], avg=[(0, 2)], avg_count=1)
+    r = finalize_partials(root, np.zeros(0, np.int64), np.zeros(0, np.int64))
+    assert r.rows == [(None, 0)] and math.isnan(r.avgs[0][0])
+
+
+def test_avg_operands_validated():
+    from paper_conf_sigmod_bressft16_b200 import _abi as A, DDQError
+    from paper_conf_sigmod_bressft16_b200.engine import finalize_partials
+    root = _root([A.AGG_SUM, A.AGG_SUM], avg=[(0, 2)], avg_count=1)  # avg_count must be a COUNT
+    with pytest.raises(DDQError):
+        finalize_partials(root, np.zeros(1, np.int64), _accs([[1, 2]]))
+
+
+def test_order_limit_with_ties():
+    from paper_conf_sigmod_bressft16_b200 import _abi as A
+    from paper_conf_sigmod_bressft16_b200.engine import finalize_partials
+    # ORDER BY agg desc, key asc; LIMIT 2 (TPC-H Q3 shape, reading O9)
+    root = _root([A.AGG_SUM], n_keys=1, key_bits=[10], order_by=[-101, 1], limit=2)
+    keys = np.array([9, 2, 7, 4], np.int64)
+    r = finalize_partials(root, keys, _accs([[5], [8], [8], [1]]))
+    assert r.rows == [(2, 8), (7, 8)]

@@ -15,13 +15,25 @@ pytestmark = [pytest.mark.gpu, pytest.mark.slow]
 
 
 def _norm(q, rows):
-    if q.startswith("ssb1") and rows == []:
-        return [(0, 0)]
     return [tuple(r) for r in rows]
 
 
+def _mem_available_gib() -> float:
+    try:
+        for line in open("/proc/meminfo"):
+            if line.startswith("MemAvailable:"):
+                return int(line.split()[1]) / (1 << 20)
+    except OSError:
+        pass
+    return 0.0
+
+
+# SF100 (north_star's headline parity target: 600 M lineorder rows) needs ~70 GB of
+# host RAM (numpy columns + the library's pinned copies); the B200 boxes have 196 GB.
+# It runs in ~90 s, exercising the O30 supplier-first join orders and the O31 coarse
+# bitmaps at the size that triggers them (customer 3 M keys).
 @pytest.mark.parametrize("sf", [20, pytest.param(100, marks=pytest.mark.skipif(
-    os.environ.get("DDQ_SF100") != "1", reason="SF100 (600 M rows, ~70 GB host RAM): set DDQ_SF100=1"))])
+    _mem_available_gib() < 90, reason="SF100 needs >= 90 GiB of available host RAM"))])
 def test_ssb_all_queries_equal_oracle(sf):
     from paper_conf_sigmod_bressft16_b200 import Database
     from paper_conf_sigmod_bressft16_b200.ssb import SSB_QUERIES, load_ssb, ssb_plan
