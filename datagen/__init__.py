@@ -21,6 +21,9 @@ _SO = os.path.join(_HERE, "libddqgen.so")
 _SRC = [os.path.join(_HERE, "ssbgen.c"), os.path.join(_HERE, "tpchgen.c")]
 
 DEFAULT_SEED = 0x5EED2016
+# primary-key encodings (ssbgen.c ddqgen_key_of): "dense" keys 1..n, or "sparse" keys
+# spread by a bijection over >= 16x the rows (the general open-addressing join path)
+KEY_MODES = {"dense": 0, "sparse": 1}
 
 
 def build(force: bool = False) -> str:
@@ -49,6 +52,10 @@ def lib():
         L.ddqgen_ssb_column.restype = ctypes.c_int
         L.ddqgen_ssb_column.argtypes = [ctypes.c_uint64, ctypes.c_double, ctypes.c_int, ctypes.c_int,
                                         ctypes.c_int64, ctypes.c_int64, ctypes.c_void_p, ctypes.c_int]
+        L.ddqgen_ssb_column_k.restype = ctypes.c_int
+        L.ddqgen_ssb_column_k.argtypes = L.ddqgen_ssb_column.argtypes + [ctypes.c_int]
+        L.ddqgen_key_of.restype = ctypes.c_int64
+        L.ddqgen_key_of.argtypes = [ctypes.c_int, ctypes.c_int64, ctypes.c_int64]
         L.ddqgen_dict_size.restype = ctypes.c_int
         L.ddqgen_dict_size.argtypes = [ctypes.c_int]
         L.ddqgen_dict_entry.restype = ctypes.c_char_p
@@ -65,6 +72,8 @@ def lib():
             L.ddqgen_tpch_column.restype = ctypes.c_int
             L.ddqgen_tpch_column.argtypes = [ctypes.c_uint64, ctypes.c_double, ctypes.c_int, ctypes.c_int,
                                              ctypes.c_int64, ctypes.c_int64, ctypes.c_void_p, ctypes.c_int]
+            L.ddqgen_tpch_column_k.restype = ctypes.c_int
+            L.ddqgen_tpch_column_k.argtypes = L.ddqgen_tpch_column.argtypes + [ctypes.c_int]
         _lib = L
     return _lib
 
@@ -113,7 +122,7 @@ def ssb_rows(table: str, sf: float) -> int:
 
 
 def ssb_column(col: str, sf: float, seed: int = DEFAULT_SEED, begin: int = 0, end: int | None = None,
-               nthreads: int | None = None, out: np.ndarray | None = None) -> np.ndarray:
+               nthreads: int | None = None, out: np.ndarray | None = None, keys: str = "dense") -> np.ndarray:
     """Rows [begin, end) of one SSB column as a numpy array (int32 or int64)."""
     L = lib()
     table = ssb_table_of(col)
@@ -127,18 +136,20 @@ def ssb_column(col: str, sf: float, seed: int = DEFAULT_SEED, begin: int = 0, en
         out = np.empty(end - begin, dtype=dt)
     assert out.dtype == dt and out.size == end - begin and out.flags.c_contiguous
     nthreads = nthreads or os.cpu_count() or 1
-    rc = L.ddqgen_ssb_column(seed, float(sf), t, c, begin, end, out.ctypes.data, nthreads)
+    rc = L.ddqgen_ssb_column_k(seed, float(sf), t, c, begin, end, out.ctypes.data, nthreads, KEY_MODES[keys])
     if rc != 0:
         raise ValueError(f"ddqgen_ssb_column({col}, sf={sf}, [{begin},{end})) failed")
     return out
 
 
 class SSB:
-    """Lazily generated SSB database at one scale factor (host numpy columns)."""
+    """Lazily generated SSB database at one scale factor (host numpy columns);
+    keys: "dense" (1..n) or "sparse" primary / foreign keys (KEY_MODES)."""
 
-    def __init__(self, sf: float, seed: int = DEFAULT_SEED):
+    def __init__(self, sf: float, seed: int = DEFAULT_SEED, keys: str = "dense"):
         self.sf = sf
         self.seed = seed
+        self.keys = keys
         self._cols: dict[str, np.ndarray] = {}
 
     def rows(self, table: str) -> int:
@@ -146,7 +157,7 @@ class SSB:
 
     def __getitem__(self, col: str) -> np.ndarray:
         if col not in self._cols:
-            self._cols[col] = ssb_column(col, self.sf, self.seed)
+            self._cols[col] = ssb_column(col, self.sf, self.seed, keys=self.keys)
         return self._cols[col]
 
     def dict_for(self, col: str) -> list[str]:
@@ -182,7 +193,7 @@ def tpch_rows(table: str, sf: float) -> int:
 
 
 def tpch_column(table: str, col: str, sf: float, seed: int = DEFAULT_SEED, begin: int = 0,
-                end: int | None = None, nthreads: int | None = None) -> np.ndarray:
+                end: int | None = None, nthreads: int | None = None, keys: str = "dense") -> np.ndarray:
     L = lib()
     t = TPCH_TABLES[table]
     c = TPCH_COLUMNS[table].index(col)
@@ -190,19 +201,21 @@ def tpch_column(table: str, col: str, sf: float, seed: int = DEFAULT_SEED, begin
     end = n if end is None else end
     w = L.ddqgen_tpch_width(t, c)
     out = np.empty(end - begin, dtype=np.int32 if w == 4 else np.int64)
-    rc = L.ddqgen_tpch_column(seed, float(sf), t, c, begin, end, out.ctypes.data,
-                              nthreads or os.cpu_count() or 1)
+    rc = L.ddqgen_tpch_column_k(seed, float(sf), t, c, begin, end, out.ctypes.data,
+                                nthreads or os.cpu_count() or 1, KEY_MODES[keys])
     if rc != 0:
         raise ValueError(f"ddqgen_tpch_column({table}.{col}) failed")
     return out
 
 
 class TPCH:
-    """Lazily generated TPC-H database; columns addressed as (table, column)."""
+    """Lazily generated TPC-H database; columns addressed as (table, column);
+    keys: "dense" or "sparse" (KEY_MODES)."""
 
-    def __init__(self, sf: float, seed: int = DEFAULT_SEED):
+    def __init__(self, sf: float, seed: int = DEFAULT_SEED, keys: str = "dense"):
         self.sf = sf
         self.seed = seed
+        self.keys = keys
         self._cols: dict[tuple[str, str], np.ndarray] = {}
 
     def rows(self, table: str) -> int:
@@ -210,7 +223,7 @@ class TPCH:
 
     def col(self, table: str, col: str) -> np.ndarray:
         if (table, col) not in self._cols:
-            self._cols[(table, col)] = tpch_column(table, col, self.sf, self.seed)
+            self._cols[(table, col)] = tpch_column(table, col, self.sf, self.seed, keys=self.keys)
         return self._cols[(table, col)]
 
     def dict_for(self, col: str) -> list[str]:

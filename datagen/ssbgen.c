@@ -221,6 +221,24 @@ int ddqgen_ssb_width(int table, int col) {
   return 0;
 }
 
+/* Primary-key encoding (SURVEY 8(c).2 "the kernels must not assume dense keys").
+ * key_mode 0 (default): dense keys 1..n.  key_mode 1 ("sparse"): row i of an
+ * n-row table gets key 1 + ((i * 0x9E3779B1) mod 2^b), b = min(30, max(22,
+ * ceil(log2 n) + 5)) -- a bijection on [0, 2^b), so keys stay unique, spread over
+ * >= 16x the row count and > 2^20 values: builds take the open-addressing hash
+ * table (reading O24), not the direct-mapped join index.  Foreign keys
+ * map through the same function; measures (prices) keep using the dense index,
+ * so every query result that does not output a key is identical in both modes. */
+int64_t ddqgen_key_of(int key_mode, int64_t n, int64_t i) {
+  if (key_mode == 0) return i + 1;
+  int b = 0;
+  while (b < 62 && (1ll << b) < n) b++;
+  b += 5;
+  if (b < 22) b = 22;
+  if (b > 30) b = 30;
+  return 1 + (int64_t)(((uint64_t)i * 0x9E3779B1ull) & ((1ull << b) - 1));
+}
+
 /* TPC-H part retail price in cents (the TPC-H formula), partkey >= 1 */
 static inline int64_t retailprice(int64_t k) {
   return 90000 + ((k / 10) % 20001) + 100 * (k % 1000);
@@ -242,7 +260,7 @@ static inline line_t lo_line(uint64_t seed, int64_t i, int64_t n_p) {
   return L;
 }
 
-static void gen_rows(uint64_t seed, double sf, int table, int col, int64_t b, int64_t e, void* out) {
+static void gen_rows(uint64_t seed, double sf, int table, int col, int64_t b, int64_t e, void* out, int km) {
   int32_t* o32 = (int32_t*)out; int64_t* o64 = (int64_t*)out; int64_t i;
   if (table == T_DATE) {
     for (i = b; i < e; i++) {
@@ -262,11 +280,12 @@ static void gen_rows(uint64_t seed, double sf, int table, int col, int64_t b, in
     return;
   }
   if (table == T_CUSTOMER || table == T_SUPPLIER) {
+    const int64_t n_t = ddqgen_ssb_rows(table, sf);
     for (i = b; i < e; i++) {
       int nat = (int)(H(seed, table, DR_NATION, (uint64_t)i) % 25u);
       int32_t v = 0;
       switch (col) {
-        case 0: v = (int32_t)(i + 1); break;
+        case 0: v = (int32_t)ddqgen_key_of(km, n_t, i); break;
         case 1: v = g_city_code[nat][H(seed, table, DR_CITY, (uint64_t)i) % 10u]; break;
         case 2: v = g_nation_code[nat]; break;
         case 3: v = NATION_REGION[nat]; break; /* region dict sorted == regionkey order */
@@ -277,12 +296,13 @@ static void gen_rows(uint64_t seed, double sf, int table, int col, int64_t b, in
     return;
   }
   if (table == T_PART) {
+    const int64_t n_t = ddqgen_ssb_rows(T_PART, sf);
     for (i = b; i < e; i++) {
       int m = (int)(H(seed, T_PART, DR_MFGR, (uint64_t)i) % 5u);
       int c = (int)(H(seed, T_PART, DR_CAT, (uint64_t)i) % 5u);
       int br = (int)(H(seed, T_PART, DR_BRAND, (uint64_t)i) % 40u);
       switch (col) {
-        case P_PARTKEY: o32[i - b] = (int32_t)(i + 1); break;
+        case P_PARTKEY: o32[i - b] = (int32_t)ddqgen_key_of(km, n_t, i); break;
         case P_MFGR: o32[i - b] = m; break;             /* "MFGR#1".."MFGR#5" sorted */
         case P_CATEGORY: o32[i - b] = m * 5 + c; break; /* "MFGR#11".."MFGR#55" sorted */
         case P_BRAND1: o32[i - b] = g_brand_code[m][c][br]; break;
@@ -299,9 +319,13 @@ static void gen_rows(uint64_t seed, double sf, int table, int col, int64_t b, in
       switch (col) {
         case LO_ORDERKEY: o32[i - b] = (int32_t)(o + 1); break;
         case LO_LINENUMBER: o32[i - b] = (int32_t)(i % 4 + 1); break;
-        case LO_CUSTKEY: o32[i - b] = (int32_t)(1 + H(seed, T_LINEORDER, DR_CUST, (uint64_t)o) % (uint64_t)n_c); break;
-        case LO_PARTKEY: o32[i - b] = (int32_t)lo_line(seed, i, n_p).pk; break;
-        case LO_SUPPKEY: o32[i - b] = (int32_t)(1 + H(seed, T_LINEORDER, DR_SUPP, (uint64_t)i) % (uint64_t)n_s); break;
+        case LO_CUSTKEY:
+          o32[i - b] = (int32_t)ddqgen_key_of(km, n_c, (int64_t)(H(seed, T_LINEORDER, DR_CUST, (uint64_t)o) % (uint64_t)n_c));
+          break;
+        case LO_PARTKEY: o32[i - b] = (int32_t)ddqgen_key_of(km, n_p, lo_line(seed, i, n_p).pk - 1); break;
+        case LO_SUPPKEY:
+          o32[i - b] = (int32_t)ddqgen_key_of(km, n_s, (int64_t)(H(seed, T_LINEORDER, DR_SUPP, (uint64_t)i) % (uint64_t)n_s));
+          break;
         case LO_ORDERDATE:
           o32[i - b] = datekey_of_index((int64_t)(H(seed, T_LINEORDER, DR_ODATE, (uint64_t)o) % N_ORDERDATES)); break;
         case LO_ORDERPRIORITY: o32[i - b] = (int32_t)(H(seed, T_LINEORDER, DR_OPRIO, (uint64_t)o) % 5u); break;
@@ -334,8 +358,8 @@ static void gen_rows(uint64_t seed, double sf, int table, int col, int64_t b, in
 /* Generate rows [row_begin, row_end) of one SSB column into out (width per
  * ddqgen_ssb_width).  Multi-threaded over row chunks; output is independent of
  * the thread count.  Returns 0 on success, -1 on bad arguments. */
-int ddqgen_ssb_column(uint64_t seed, double sf, int table, int col, int64_t row_begin,
-                      int64_t row_end, void* out, int nthreads) {
+int ddqgen_ssb_column_k(uint64_t seed, double sf, int table, int col, int64_t row_begin,
+                        int64_t row_end, void* out, int nthreads, int key_mode) {
   init_dicts();
   int w = ddqgen_ssb_width(table, col);
   int64_t n = ddqgen_ssb_rows(table, sf);
@@ -347,7 +371,11 @@ int ddqgen_ssb_column(uint64_t seed, double sf, int table, int col, int64_t row_
 #pragma omp parallel for schedule(dynamic, 4) num_threads(nthreads)
   for (c = 0; c < nchunks; c++) {
     int64_t b = row_begin + c * chunk, e = b + chunk < row_end ? b + chunk : row_end;
-    gen_rows(seed, sf, table, col, b, e, (char*)out + (b - row_begin) * w);
+    gen_rows(seed, sf, table, col, b, e, (char*)out + (b - row_begin) * w, key_mode);
   }
   return 0;
+}
+int ddqgen_ssb_column(uint64_t seed, double sf, int table, int col, int64_t row_begin,
+                      int64_t row_end, void* out, int nthreads) {
+  return ddqgen_ssb_column_k(seed, sf, table, col, row_begin, row_end, out, nthreads, 0);
 }

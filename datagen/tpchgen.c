@@ -14,6 +14,7 @@
 uint64_t ddqgen_hash(uint64_t seed, uint32_t table, uint32_t draw, uint64_t i);
 int32_t ddqgen_datekey_of_index(int64_t idx);
 int ddqgen_dict_size(int dict);
+int64_t ddqgen_key_of(int key_mode, int64_t n, int64_t i); /* ssbgen.c: dense / sparse keys */
 
 enum { TH_NATION = 11, TH_REGION = 12, TH_CUSTOMER = 13, TH_SUPPLIER = 14, TH_PART = 15,
        TH_ORDERS = 16, TH_LINEITEM = 17, TH_CALENDAR = 18 };
@@ -82,10 +83,10 @@ static inline int64_t retailprice_h(int64_t k) {
   return 90000 + ((k / 10) % 20001) + 100 * (k % 1000);
 }
 
-static void gen_rows_h(uint64_t seed, double sf, int table, int col, int64_t b, int64_t e, void* out) {
+static void gen_rows_h(uint64_t seed, double sf, int table, int col, int64_t b, int64_t e, void* out, int km) {
   int32_t* o32 = (int32_t*)out; int64_t* o64 = (int64_t*)out; int64_t i;
   int64_t n_c = ddqgen_tpch_rows(TH_CUSTOMER, sf), n_s = ddqgen_tpch_rows(TH_SUPPLIER, sf);
-  int64_t n_p = ddqgen_tpch_rows(TH_PART, sf);
+  int64_t n_p = ddqgen_tpch_rows(TH_PART, sf), n_o = ddqgen_tpch_rows(TH_ORDERS, sf);
   for (i = b; i < e; i++) {
     int64_t k = i - b;
     switch (table) {
@@ -98,20 +99,21 @@ static void gen_rows_h(uint64_t seed, double sf, int table, int col, int64_t b, 
         o32[k] = col == CAL_DATEKEY ? dk : dk / 10000;
       } break;
       case TH_CUSTOMER:
-        if (col == HC_CUSTKEY) o32[k] = (int32_t)(i + 1);
+        if (col == HC_CUSTKEY) o32[k] = (int32_t)ddqgen_key_of(km, n_c, i);
         else if (col == HC_NATIONKEY) o32[k] = (int32_t)(ddqgen_hash(seed, table, DRH_NATION, (uint64_t)i) % 25u);
         else o32[k] = (int32_t)(ddqgen_hash(seed, table, DRH_SEGMENT, (uint64_t)i) % 5u);
         break;
       case TH_SUPPLIER:
-        if (col == HS_SUPPKEY) o32[k] = (int32_t)(i + 1);
+        if (col == HS_SUPPKEY) o32[k] = (int32_t)ddqgen_key_of(km, n_s, i);
         else o32[k] = (int32_t)(ddqgen_hash(seed, table, DRH_NATION, (uint64_t)i) % 25u);
         break;
       case TH_PART:
-        if (col == HP_PARTKEY) o32[k] = (int32_t)(i + 1); else o64[k] = retailprice_h(i + 1);
+        if (col == HP_PARTKEY) o32[k] = (int32_t)ddqgen_key_of(km, n_p, i); else o64[k] = retailprice_h(i + 1);
         break;
       case TH_ORDERS:
-        if (col == O_ORDERKEY) o32[k] = (int32_t)(i + 1);
-        else if (col == O_CUSTKEY) o32[k] = (int32_t)(1 + ddqgen_hash(seed, TH_ORDERS, DRH_CUST, (uint64_t)i) % (uint64_t)n_c);
+        if (col == O_ORDERKEY) o32[k] = (int32_t)ddqgen_key_of(km, n_o, i);
+        else if (col == O_CUSTKEY)
+          o32[k] = (int32_t)ddqgen_key_of(km, n_c, (int64_t)(ddqgen_hash(seed, TH_ORDERS, DRH_CUST, (uint64_t)i) % (uint64_t)n_c));
         else if (col == O_ORDERDATE)
           o32[k] = ddqgen_datekey_of_index((int64_t)(ddqgen_hash(seed, TH_ORDERS, DRH_ODATE, (uint64_t)i) % N_ORDERDATES));
         else if (col == O_ORDERPRIORITY) /* dict "1-URGENT".."5-LOW" (sorted == priority) */
@@ -126,9 +128,11 @@ static void gen_rows_h(uint64_t seed, double sf, int table, int col, int64_t b, 
         int64_t pk = 1 + (int64_t)(ddqgen_hash(seed, TH_LINEITEM, DRH_PART, (uint64_t)i) % (uint64_t)n_p);
         int64_t qty = 100 * (1 + (int64_t)(ddqgen_hash(seed, TH_LINEITEM, DRH_QTY, (uint64_t)i) % 50u));
         switch (col) {
-          case L_ORDERKEY: o32[k] = (int32_t)(o + 1); break;
-          case L_PARTKEY: o32[k] = (int32_t)pk; break;
-          case L_SUPPKEY: o32[k] = (int32_t)(1 + ddqgen_hash(seed, TH_LINEITEM, DRH_SUPP, (uint64_t)i) % (uint64_t)n_s); break;
+          case L_ORDERKEY: o32[k] = (int32_t)ddqgen_key_of(km, n_o, o); break;
+          case L_PARTKEY: o32[k] = (int32_t)ddqgen_key_of(km, n_p, pk - 1); break;
+          case L_SUPPKEY:
+            o32[k] = (int32_t)ddqgen_key_of(km, n_s, (int64_t)(ddqgen_hash(seed, TH_LINEITEM, DRH_SUPP, (uint64_t)i) % (uint64_t)n_s));
+            break;
           case L_LINENUMBER: o32[k] = (int32_t)(i % 4 + 1); break;
           case L_QUANTITY: o64[k] = qty; break;
           case L_EXTENDEDPRICE: o64[k] = (qty / 100) * retailprice_h(pk); break;
@@ -152,8 +156,8 @@ static void gen_rows_h(uint64_t seed, double sf, int table, int col, int64_t b, 
   }
 }
 
-int ddqgen_tpch_column(uint64_t seed, double sf, int table, int col, int64_t row_begin,
-                       int64_t row_end, void* out, int nthreads) {
+int ddqgen_tpch_column_k(uint64_t seed, double sf, int table, int col, int64_t row_begin,
+                         int64_t row_end, void* out, int nthreads, int key_mode) {
   (void)ddqgen_dict_size(0); /* make sure dictionaries are initialised */
   int w = ddqgen_tpch_width(table, col);
   int64_t n = ddqgen_tpch_rows(table, sf);
@@ -165,7 +169,11 @@ int ddqgen_tpch_column(uint64_t seed, double sf, int table, int col, int64_t row
 #pragma omp parallel for schedule(dynamic, 4) num_threads(nthreads)
   for (c = 0; c < nchunks; c++) {
     int64_t b = row_begin + c * chunk, e = b + chunk < row_end ? b + chunk : row_end;
-    gen_rows_h(seed, sf, table, col, b, e, (char*)out + (b - row_begin) * w);
+    gen_rows_h(seed, sf, table, col, b, e, (char*)out + (b - row_begin) * w, key_mode);
   }
   return 0;
+}
+int ddqgen_tpch_column(uint64_t seed, double sf, int table, int col, int64_t row_begin,
+                       int64_t row_end, void* out, int nthreads) {
+  return ddqgen_tpch_column_k(seed, sf, table, col, row_begin, row_end, out, nthreads, 0);
 }

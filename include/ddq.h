@@ -278,6 +278,10 @@ ddq_status ddq_create_table(ddq_db* db, const char* name, int64_t n_rows, int64_
 ddq_status ddq_load_column(ddq_db* db, ddq_table t, const char* name, ddq_type type,
                            const void* host_data, int64_t n_rows, ddq_column* out);
 ddq_status ddq_find_column(ddq_db* db, const char* table, const char* name, ddq_column* out);
+/* Column statistics recorded at load (the strategic optimiser's input):
+ * row count and value range [vmin, vmax] (vmin > vmax for an empty column).  Plans
+ * size packed group keys from them (e.g. bits of a key column = bit length of vmax). */
+ddq_status ddq_column_stats(ddq_db* db, ddq_column c, int64_t* n, int64_t* vmin, int64_t* vmax);
 
 /* Storage adviser: pin a column into the device cache (H2D copy on the
  * library's copy stream, counted in stats) / evict it (freed once no running

@@ -133,6 +133,7 @@ SIGNATURES = {
     "ddq_create_table": (_i32, [_vp, ctypes.c_char_p, _i64, _i64, ctypes.POINTER(_i32)]),
     "ddq_load_column": (_i32, [_vp, _i32, ctypes.c_char_p, _i32, _vp, _i64, ctypes.POINTER(_i32)]),
     "ddq_find_column": (_i32, [_vp, ctypes.c_char_p, ctypes.c_char_p, ctypes.POINTER(_i32)]),
+    "ddq_column_stats": (_i32, [_vp, _i32, ctypes.POINTER(_i64), ctypes.POINTER(_i64), ctypes.POINTER(_i64)]),
     "ddq_set_dictionary": (_i32, [_vp, _i32, ctypes.POINTER(ctypes.c_char_p), _i32]),
     "ddq_dictionary_range": (_i32, [_vp, _i32, ctypes.c_char_p, ctypes.POINTER(_i32), ctypes.POINTER(_i32)]),
     "ddq_dictionary_like": (_i32, [_vp, _i32, ctypes.c_char_p, ctypes.POINTER(Pred)]),

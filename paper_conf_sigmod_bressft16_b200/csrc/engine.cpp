@@ -963,6 +963,17 @@ ddq_status ddq_find_column(ddq_db* db, const char* table, const char* name, ddq_
   return set_error(DDQ_ENOTFOUND, std::string("column ") + table + "." + name);
 }
 
+ddq_status ddq_column_stats(ddq_db* db, ddq_column c, int64_t* n, int64_t* vmin, int64_t* vmax) {
+  if (!db || !n || !vmin || !vmax) return set_error(DDQ_EINVAL, "column_stats: null argument");
+  std::lock_guard<std::mutex> g(db->mu);
+  if (c < 0 || c >= (int)db->cols.size()) return set_error(DDQ_ENOTFOUND, "column_stats: bad column");
+  const Column& col = *db->cols[(size_t)c];
+  *n = col.n;
+  *vmin = col.n > 0 ? col.vmin : 1;
+  *vmax = col.n > 0 ? col.vmax : 0;
+  return DDQ_OK;
+}
+
 ddq_status ddq_set_dictionary(ddq_db* db, ddq_column c, const char* const* sorted_strings, int32_t n) {
   if (!db || n < 0 || (n > 0 && !sorted_strings)) return set_error(DDQ_EINVAL, "set_dictionary: null argument");
   std::vector<std::string> d;

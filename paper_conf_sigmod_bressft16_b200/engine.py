@@ -397,6 +397,13 @@ class Database:
         self._cols[(table, name)] = c.value
         return c.value
 
+    def column_stats(self, table: str, name: str) -> tuple[int, int, int]:
+        """(rows, min, max) of a loaded column (recorded by the library at load)."""
+        n, lo, hi = ctypes.c_int64(), ctypes.c_int64(), ctypes.c_int64()
+        check(lib().ddq_column_stats(self.h, self.col(table, name), ctypes.byref(n), ctypes.byref(lo),
+                                     ctypes.byref(hi)))
+        return n.value, lo.value, hi.value
+
     def set_dictionary(self, table: str, name: str, strings: list[str]) -> None:
         """Order-preserving dictionary of a string column (codes = ranks, reading O4)."""
         enc = [x.encode() for x in strings]

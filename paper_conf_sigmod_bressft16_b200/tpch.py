@@ -31,6 +31,17 @@ QUERY_TABLES = {"tpch1": ["lineitem"], "tpch6": ["lineitem"],
                 "tpch5": ["region", "nation", "supplier", "customer", "orders", "lineitem"]}
 
 
+def _bits(db, table: str, col: str) -> int:
+    """Bits of a non-negative key column in a packed group key (from the column's
+    load-time statistics: dense and sparse key encodings need different widths)."""
+    if not hasattr(db, "column_stats"):  # host-only catalogue (finalisation tests)
+        return 21
+    n, lo, hi = db.column_stats(table, col)
+    if lo < 0:
+        raise ValueError(f"{table}.{col}: negative group key")
+    return max(1, int(hi).bit_length())
+
+
 def load_tpch(db: Database, data, cache: bool = True, tables=None) -> None:
     """data: ``data.col(table, col)``, ``data.rows(table)``, ``data.dict_for(col)``."""
     for t in (tables or list(TABLE_COLUMNS)):
@@ -87,7 +98,9 @@ def tpch_plan(db: Database, q: str, limit: int = 0, dense: bool = True) -> PlanB
         t = P.probe(li, "l_orderkey", hos, input=t, emit=True)            # vec1 = o_shippriority
         # group by l_orderkey, o_orderdate, o_shippriority; order by revenue desc,
         # o_orderdate, then l_orderkey (O9)
-        P.aggregate(li, t, keys=["l_orderkey", 0, 1], key_bits=[28, 25, 10],
+        P.aggregate(li, t, keys=["l_orderkey", 0, 1],
+                    key_bits=[_bits(db, li, "l_orderkey"), _bits(db, "orders", "o_orderdate"),
+                              _bits(db, "orders", "o_shippriority")],
                     aggs=[(A.AGG_SUM_MUL_100M, ["l_extendedprice", "l_discount"])],
                     order_by=[-101, 2, 1], max_groups=1 << 22, limit=limit)
         return P

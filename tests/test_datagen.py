@@ -126,3 +126,39 @@ def test_tpch_domains():
     nat = datagen.dictionary("nation")
     names = np.array(nat)[db.col("nation", "n_name")]
     assert names[24] == "UNITED STATES" and names[18] == "CHINA" and names[0] == "ALGERIA"
+
+
+# ---- sparse key encoding ("the kernels must not assume dense keys")
+SSB_KEYS = [("c_custkey", "lo_custkey"), ("s_suppkey", "lo_suppkey"), ("p_partkey", "lo_partkey")]
+TPCH_KEYS = [(("customer", "c_custkey"), ("orders", "o_custkey")), (("orders", "o_orderkey"), ("lineitem", "l_orderkey")),
+             (("supplier", "s_suppkey"), ("lineitem", "l_suppkey")), (("part", "p_partkey"), ("lineitem", "l_partkey"))]
+
+
+def _takes_hash_path(keys: np.ndarray) -> bool:
+    """DESIGN.md reading O24: a build key column gets the direct-mapped join index iff
+    its range is <= 2^20 values or <= 16x the rows; sparse keys must exceed both."""
+    rng = int(keys.max()) - int(keys.min()) + 1
+    return rng > (1 << 20) and rng > 16 * keys.size
+
+
+@pytest.mark.parametrize("sf", [0.01, 1.0])
+def test_sparse_ssb_keys(sf):
+    sp, de = datagen.SSB(sf, keys="sparse"), datagen.SSB(sf)
+    for pk, fk in SSB_KEYS:
+        k = sp[pk]
+        assert np.unique(k).size == k.size and k.min() >= 1 and k.max() < 2**31
+        assert _takes_hash_path(k), pk
+        # the FK maps through the same bijection as the PK: row r of the dense FK
+        # (a key 1..n) becomes the sparse key of dimension row r - 1
+        assert np.array_equal(sp[fk], k[de[fk] - 1])
+    for c in ("lo_revenue", "lo_extendedprice", "lo_supplycost", "lo_orderdate", "c_nation", "p_brand1"):
+        assert np.array_equal(sp[c], de[c]), c  # measures and attributes unchanged
+
+
+def test_sparse_tpch_keys():
+    sp, de = datagen.TPCH(0.1, keys="sparse"), datagen.TPCH(0.1)
+    for (pt, pk), (ft, fk) in TPCH_KEYS:
+        k = sp.col(pt, pk)
+        assert np.unique(k).size == k.size and _takes_hash_path(k), pk
+        assert np.array_equal(sp.col(ft, fk), k[de.col(ft, fk) - 1]), fk
+    assert np.array_equal(sp.col("lineitem", "l_extendedprice"), de.col("lineitem", "l_extendedprice"))

@@ -32,12 +32,14 @@ def _mem_available_gib() -> float:
 # host RAM (numpy columns + the library's pinned copies); the B200 boxes have 196 GB.
 # It runs in ~90 s, exercising the O30 supplier-first join orders and the O31 coarse
 # bitmaps at the size that triggers them (customer 3 M keys).
-@pytest.mark.parametrize("sf", [20, pytest.param(100, marks=pytest.mark.skipif(
+@pytest.mark.parametrize("sf,keys", [(20, "dense"), (20, "sparse"), pytest.param(100, "dense", marks=pytest.mark.skipif(
     _mem_available_gib() < 90, reason="SF100 needs >= 90 GiB of available host RAM"))])
-def test_ssb_all_queries_equal_oracle(sf):
+def test_ssb_all_queries_equal_oracle(sf, keys):
+    """keys="sparse": every dimension build but date's is an open-addressing hash
+    table (reading O24), probed at full size."""
     from paper_conf_sigmod_bressft16_b200 import Database
     from paper_conf_sigmod_bressft16_b200.ssb import SSB_QUERIES, load_ssb, ssb_plan
-    data = datagen.SSB(sf)
+    data = datagen.SSB(sf, keys=keys)
     db = Database(cache_bytes=64 << 30, heap_bytes=(24 << 30) * sf // 20)
     load_ssb(db, data)
     import torch
@@ -62,10 +64,11 @@ def test_ssb_all_queries_equal_oracle(sf):
         assert _norm(q, got[q]) == _norm(q, want[q]), q
 
 
-def test_tpch_sf30_all_queries_equal_oracle():
+@pytest.mark.parametrize("keys", ["dense", "sparse"])
+def test_tpch_sf30_all_queries_equal_oracle(keys):
     from paper_conf_sigmod_bressft16_b200 import Database
     from paper_conf_sigmod_bressft16_b200.tpch import load_tpch, tpch_plan
-    data = datagen.TPCH(30)
+    data = datagen.TPCH(30, keys=keys)
     db = Database(cache_bytes=64 << 30, heap_bytes=24 << 30)
     load_tpch(db, data)
     qs = ("tpch1", "tpch3", "tpch4", "tpch5", "tpch6", "tpch7")

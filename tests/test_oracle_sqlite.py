@@ -63,15 +63,15 @@ def nkeys_of(q):
 
 
 @functools.lru_cache(maxsize=None)
-def _ssb(sf):
-    db = datagen.SSB(sf)
+def _ssb(sf, keys="dense"):
+    db = datagen.SSB(sf, keys=keys)
     return db, ssb_sqlite(db)
 
 
-@pytest.mark.parametrize("sf", [0.01, 0.05])
+@pytest.mark.parametrize("sf,keys", [(0.01, "dense"), (0.05, "dense"), (0.01, "sparse")])
 @pytest.mark.parametrize("q", oracle.SSB_QUERIES)
-def test_ssb_oracle_equals_sqlite(sf, q):
-    db, con = _ssb(sf)
+def test_ssb_oracle_equals_sqlite(sf, keys, q):
+    db, con = _ssb(sf, keys)
     sql = load_sql("ssb_queries.sql")[q]
     want = [tuple(r) for r in con.execute(sql).fetchall()]
     got = to_sql_rows(q, oracle.run(db, q), nkeys_of(q))
@@ -115,8 +115,8 @@ def test_ungrouped_sum_over_no_rows_is_null(q):
 
 
 @functools.lru_cache(maxsize=None)
-def _tpch(sf):
-    db = datagen.TPCH(sf)
+def _tpch(sf, keys="dense"):
+    db = datagen.TPCH(sf, keys=keys)
     return db, tpch_sqlite(db)
 
 
@@ -138,9 +138,10 @@ def tpch_to_sql(q, rows):
     return [tuple(r) for r in rows]
 
 
+@pytest.mark.parametrize("keys", ["dense", "sparse"])
 @pytest.mark.parametrize("q", ["tpch1", "tpch3", "tpch4", "tpch5", "tpch6", "tpch7"])
-def test_tpch_oracle_equals_sqlite(q):
-    db, con = _tpch(0.01)
+def test_tpch_oracle_equals_sqlite(q, keys):
+    db, con = _tpch(0.01, keys)
     want = [tuple(r) for r in con.execute(load_sql("tpch_queries.sql")[q]).fetchall()]
     got = tpch_to_sql(q, oracle.run(db, q))
     if q == "tpch1":
