@@ -94,7 +94,7 @@ SSB_COLUMNS = {
 # string columns -> dictionary id
 DICTS = {"nation": 0, "region": 1, "city": 2, "mfgr": 3, "category": 4, "brand1": 5,
          "yearmonth": 6, "mktsegment": 7, "orderpriority": 8, "shipmode": 9,
-         "returnflag": 10, "linestatus": 11}
+         "returnflag": 10, "linestatus": 11, "type": 12, "tpch_mfgr": 13}
 SSB_STRING_COLUMNS = {
     "d_yearmonth": "yearmonth", "c_city": "city", "c_nation": "nation", "c_region": "region",
     "c_mktsegment": "mktsegment", "s_city": "city", "s_nation": "nation", "s_region": "region",
@@ -169,23 +169,25 @@ class SSB:
 
 # --------------------------------------------------------------- TPC-H schema
 TPCH_TABLES = {"nation": 11, "region": 12, "customer": 13, "supplier": 14, "part": 15,
-               "orders": 16, "lineitem": 17, "calendar": 18}
+               "orders": 16, "lineitem": 17, "calendar": 18, "partsupp": 19}
 TPCH_COLUMNS = {
     "nation": ["n_nationkey", "n_name", "n_regionkey"],
     "region": ["r_regionkey", "r_name"],
     "customer": ["c_custkey", "c_nationkey", "c_mktsegment"],
-    "supplier": ["s_suppkey", "s_nationkey"],
-    "part": ["p_partkey", "p_retailprice"],
+    "supplier": ["s_suppkey", "s_nationkey", "s_acctbal"],
+    "part": ["p_partkey", "p_retailprice", "p_mfgr", "p_type", "p_size"],
     "orders": ["o_orderkey", "o_custkey", "o_orderdate", "o_shippriority", "o_orderpriority"],
     "lineitem": ["l_orderkey", "l_partkey", "l_suppkey", "l_linenumber", "l_quantity",
                  "l_extendedprice", "l_discount", "l_tax", "l_returnflag", "l_linestatus",
                  "l_shipdate", "l_commitdate", "l_receiptdate"],
     # the date dimension over TPC-H's date domain, 1992-01-01 .. 1998-12-31 (reading O34)
     "calendar": ["d_datekey", "d_year"],
+    # TPC-H Q2: 4 suppliers per part (the TPC-H supplier rule), supplycost scale 2
+    "partsupp": ["ps_partkey", "ps_suppkey", "ps_supplycost"],
 }
 TPCH_STRING_COLUMNS = {"n_name": "nation", "r_name": "region", "c_mktsegment": "mktsegment",
                        "l_returnflag": "returnflag", "l_linestatus": "linestatus",
-                       "o_orderpriority": "orderpriority"}
+                       "o_orderpriority": "orderpriority", "p_type": "type", "p_mfgr": "tpch_mfgr"}
 
 
 def tpch_rows(table: str, sf: float) -> int:

@@ -42,7 +42,7 @@ uint64_t ddqgen_hash(uint64_t seed, uint32_t table, uint32_t draw, uint64_t i) {
 enum {
   DICT_NATION = 0, DICT_REGION, DICT_CITY, DICT_MFGR, DICT_CATEGORY, DICT_BRAND1,
   DICT_YEARMONTH, DICT_MKTSEGMENT, DICT_ORDERPRIORITY, DICT_SHIPMODE,
-  DICT_RETURNFLAG, DICT_LINESTATUS, DICT_N
+  DICT_RETURNFLAG, DICT_LINESTATUS, DICT_TYPE, DICT_TPCH_MFGR, DICT_N
 };
 
 /* TPC-H nations in nationkey order, with their regionkey. */
@@ -61,6 +61,11 @@ static const char* MONTHS[12] = {"Jan", "Feb", "Mar", "Apr", "May", "Jun",
                                  "Jul", "Aug", "Sep", "Oct", "Nov", "Dec"};
 static const char* RETURNFLAGS[3] = {"A", "N", "R"};
 static const char* LINESTATUS[2] = {"F", "O"};
+/* TPC-H p_type = one syllable of each list (150 types), p_mfgr = Manufacturer#1..5 */
+static const char* TYPE_S1[6] = {"STANDARD", "SMALL", "MEDIUM", "LARGE", "ECONOMY", "PROMO"};
+static const char* TYPE_S2[5] = {"ANODIZED", "BURNISHED", "PLATED", "POLISHED", "BRUSHED"};
+static const char* TYPE_S3[5] = {"TIN", "NICKEL", "BRASS", "STEEL", "COPPER"};
+static int g_type_code[6][5][5];    /* (s1, s2, s3) -> code in DICT_TYPE */
 
 typedef struct { int n; char** s; } dict_t;
 static dict_t g_dict[DICT_N];
@@ -130,6 +135,17 @@ static void init_dicts(void) {
   dict_build(&g_dict[DICT_RETURNFLAG], tmp, 3);
   for (i = 0; i < 2; i++) tmp[i] = xstrdup(LINESTATUS[i]);
   dict_build(&g_dict[DICT_LINESTATUS], tmp, 2);
+  n = 0;
+  for (i = 0; i < 6; i++) for (j = 0; j < 5; j++) for (k = 0; k < 5; k++) {
+    sprintf(buf, "%s %s %s", TYPE_S1[i], TYPE_S2[j], TYPE_S3[k]); tmp[n++] = xstrdup(buf);
+  }
+  dict_build(&g_dict[DICT_TYPE], tmp, n);
+  for (i = 0; i < 6; i++) for (j = 0; j < 5; j++) for (k = 0; k < 5; k++) {
+    sprintf(buf, "%s %s %s", TYPE_S1[i], TYPE_S2[j], TYPE_S3[k]);
+    g_type_code[i][j][k] = dict_rank(&g_dict[DICT_TYPE], buf);
+  }
+  for (i = 0; i < 5; i++) { sprintf(buf, "Manufacturer#%d", i + 1); tmp[i] = xstrdup(buf); }
+  dict_build(&g_dict[DICT_TPCH_MFGR], tmp, 5);
 
   for (i = 0; i < 25; i++) g_nation_code[i] = dict_rank(&g_dict[DICT_NATION], NATION_NAMES[i]);
   for (i = 0; i < 25; i++) for (j = 0; j < 10; j++) {
@@ -175,6 +191,8 @@ static int day_of_year(int y, int m, int d) {
   return cum[m - 1] + d + (m > 2 && is_leap(y));
 }
 int32_t ddqgen_datekey_of_index(int64_t idx) { return datekey_of_index(idx); }
+/* TPC-H p_type code of syllables (s1, s2, s3) (tpchgen.c) */
+int ddqgen_type_code(int s1, int s2, int s3) { init_dicts(); return g_type_code[s1][s2][s3]; }
 
 /* ------------------------------------------------------------------- sizes */
 enum { T_DATE = 1, T_CUSTOMER = 2, T_SUPPLIER = 3, T_PART = 4, T_LINEORDER = 5 };

@@ -15,9 +15,14 @@ uint64_t ddqgen_hash(uint64_t seed, uint32_t table, uint32_t draw, uint64_t i);
 int32_t ddqgen_datekey_of_index(int64_t idx);
 int ddqgen_dict_size(int dict);
 int64_t ddqgen_key_of(int key_mode, int64_t n, int64_t i); /* ssbgen.c: dense / sparse keys */
+int ddqgen_type_code(int s1, int s2, int s3);               /* ssbgen.c: p_type dictionary */
 
 enum { TH_NATION = 11, TH_REGION = 12, TH_CUSTOMER = 13, TH_SUPPLIER = 14, TH_PART = 15,
-       TH_ORDERS = 16, TH_LINEITEM = 17, TH_CALENDAR = 18 };
+       TH_ORDERS = 16, TH_LINEITEM = 17, TH_CALENDAR = 18, TH_PARTSUPP = 19 };
+/* TH_PARTSUPP (TPC-H Q2): 4 rows per part; row j = (part j / 4, the (j % 4)-th supplier
+ * of the TPC-H rule ps_suppkey = (ps_partkey + i * (S/4 + (ps_partkey - 1) / S)) % S + 1
+ * on dense keys), ps_supplycost uniform 1.00 .. 1000.00 (scale 2). */
+enum { PS_PARTKEY = 0, PS_SUPPKEY, PS_SUPPLYCOST };
 /* TH_CALENDAR: the date dimension of TPC-H's date domain (one row per day
  * 1992-01-01 .. 1998-12-31, as SSB's date table): d_datekey yyyymmdd, d_year.
  * Q7's extract(year from l_shipdate) joins it (reading O34). */
@@ -26,15 +31,16 @@ enum { CAL_DATEKEY = 0, CAL_YEAR };
 enum { N_NATIONKEY = 0, N_NAME, N_REGIONKEY };
 enum { R_REGIONKEY = 0, R_NAME };
 enum { HC_CUSTKEY = 0, HC_NATIONKEY, HC_MKTSEGMENT };
-enum { HS_SUPPKEY = 0, HS_NATIONKEY };
-enum { HP_PARTKEY = 0, HP_RETAILPRICE };
+enum { HS_SUPPKEY = 0, HS_NATIONKEY, HS_ACCTBAL };            /* s_acctbal -999.99 .. 9999.99 */
+enum { HP_PARTKEY = 0, HP_RETAILPRICE, HP_MFGR, HP_TYPE, HP_SIZE }; /* TPC-H part attributes */
 enum { O_ORDERKEY = 0, O_CUSTKEY, O_ORDERDATE, O_SHIPPRIORITY, O_ORDERPRIORITY };
 enum { L_ORDERKEY = 0, L_PARTKEY, L_SUPPKEY, L_LINENUMBER, L_QUANTITY, L_EXTENDEDPRICE,
        L_DISCOUNT, L_TAX, L_RETURNFLAG, L_LINESTATUS, L_SHIPDATE, L_COMMITDATE, L_RECEIPTDATE,
        L_NCOLS };
 enum { DRH_NATION = 1, DRH_SEGMENT = 2, DRH_CUST = 10, DRH_ODATE = 11, DRH_PART = 12, DRH_SUPP = 13,
        DRH_QTY = 14, DRH_DISC = 15, DRH_TAX = 16, DRH_SHIP = 17, DRH_RECEIPT = 18, DRH_COMMIT = 19,
-       DRH_RFLAG = 20, DRH_OPRIO = 21 };
+       DRH_RFLAG = 20, DRH_OPRIO = 21, DRH_MFGR = 22, DRH_TYPE = 23, DRH_SIZE = 24, DRH_ACCTBAL = 25,
+       DRH_PSCOST = 26 };
 
 #define N_ORDERDATES 2406
 #define CUTOFF_19950617 19950617
@@ -61,6 +67,7 @@ int64_t ddqgen_tpch_rows(int table, double sf) {
     case TH_ORDERS: return scaled_h(sf, 1500000.0);
     case TH_LINEITEM: return 4 * scaled_h(sf, 1500000.0);
     case TH_CALENDAR: return N_CALENDAR;
+    case TH_PARTSUPP: return 4 * scaled_h(sf, 200000.0);
   }
   return -1;
 }
@@ -69,8 +76,9 @@ int ddqgen_tpch_width(int table, int col) {
     case TH_NATION: return (col >= 0 && col <= N_REGIONKEY) ? 4 : 0;
     case TH_REGION: return (col >= 0 && col <= R_NAME) ? 4 : 0;
     case TH_CUSTOMER: return (col >= 0 && col <= HC_MKTSEGMENT) ? 4 : 0;
-    case TH_SUPPLIER: return (col >= 0 && col <= HS_NATIONKEY) ? 4 : 0;
-    case TH_PART: return col == HP_RETAILPRICE ? 8 : col == HP_PARTKEY ? 4 : 0;
+    case TH_SUPPLIER: return col == HS_ACCTBAL ? 8 : (col >= 0 && col <= HS_NATIONKEY) ? 4 : 0;
+    case TH_PART: return col == HP_RETAILPRICE ? 8 : (col >= 0 && col <= HP_SIZE) ? 4 : 0;
+    case TH_PARTSUPP: return col == PS_SUPPLYCOST ? 8 : (col == PS_PARTKEY || col == PS_SUPPKEY) ? 4 : 0;
     case TH_ORDERS: return (col >= 0 && col <= O_ORDERPRIORITY) ? 4 : 0;
     case TH_LINEITEM:
       if (col < 0 || col >= L_NCOLS) return 0;
@@ -105,11 +113,26 @@ static void gen_rows_h(uint64_t seed, double sf, int table, int col, int64_t b, 
         break;
       case TH_SUPPLIER:
         if (col == HS_SUPPKEY) o32[k] = (int32_t)ddqgen_key_of(km, n_s, i);
+        else if (col == HS_ACCTBAL) o64[k] = -99999 + (int64_t)(ddqgen_hash(seed, table, DRH_ACCTBAL, (uint64_t)i) % 1099999u);
         else o32[k] = (int32_t)(ddqgen_hash(seed, table, DRH_NATION, (uint64_t)i) % 25u);
         break;
       case TH_PART:
-        if (col == HP_PARTKEY) o32[k] = (int32_t)ddqgen_key_of(km, n_p, i); else o64[k] = retailprice_h(i + 1);
+        if (col == HP_PARTKEY) o32[k] = (int32_t)ddqgen_key_of(km, n_p, i);
+        else if (col == HP_RETAILPRICE) o64[k] = retailprice_h(i + 1);
+        else if (col == HP_MFGR) o32[k] = (int32_t)(ddqgen_hash(seed, table, DRH_MFGR, (uint64_t)i) % 5u); /* sorted */
+        else if (col == HP_SIZE) o32[k] = 1 + (int32_t)(ddqgen_hash(seed, table, DRH_SIZE, (uint64_t)i) % 50u);
+        else {
+          const uint64_t h = ddqgen_hash(seed, table, DRH_TYPE, (uint64_t)i) % 150u;
+          o32[k] = ddqgen_type_code((int)(h / 25), (int)(h / 5 % 5), (int)(h % 5));
+        }
         break;
+      case TH_PARTSUPP: {
+        const int64_t p = i / 4, pk = p + 1, j = i % 4;
+        const int64_t sd = (pk + j * (n_s / 4 + (pk - 1) / n_s)) % n_s; /* 0-based supplier index */
+        if (col == PS_PARTKEY) o32[k] = (int32_t)ddqgen_key_of(km, n_p, p);
+        else if (col == PS_SUPPKEY) o32[k] = (int32_t)ddqgen_key_of(km, n_s, sd);
+        else o64[k] = 100 + (int64_t)(ddqgen_hash(seed, table, DRH_PSCOST, (uint64_t)i) % 99901u);
+      } break;
       case TH_ORDERS:
         if (col == O_ORDERKEY) o32[k] = (int32_t)ddqgen_key_of(km, n_o, i);
         else if (col == O_CUSTKEY)

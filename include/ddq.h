@@ -346,7 +346,10 @@ typedef struct {
   int32_t emit_payload;    /* append matched payload as an aligned vector */
   /* GATHER */
   ddq_column gather_col;
-  /* AGGREGATE: keys are aligned vectors (index >= 0) or columns (-2 - column id) */
+  /* AGGREGATE: keys are aligned vectors (index >= 0) or columns (-2 - column id).
+     agg_col[a][j] is a column id (>= 0), -1 = none, or, for DDQ_AGG_MIN only, an
+     aligned int32 vector v of the input encoded as -2 - v (a functionally dependent
+     dimension attribute fetched through a join, TPC-H Q2); not with fused predicates. */
   int32_t n_keys;
   int32_t key_src[DDQ_MAX_KEYS];
   int32_t n_aggs;
@@ -385,8 +388,12 @@ typedef struct {
   int32_t eq_cmp;
   /* HASH_BUILD: 1 = the build is a key SET for a semi-join (EXISTS / IN subquery,
      TPC-H Q4): duplicate keys are allowed and collapse into one entry whose
-     payload is any one of their rows; 0 (default) = unique keys, a duplicate is
-     DDQ_EINVAL (reading O13). */
+     payload is any one of their rows; 2 = a MIN-aggregating build (a decorrelated
+     scalar subquery `= (select min(x) ... where key = outer.key)`, TPC-H Q2, reading
+     O35): duplicate keys collapse into one entry whose payload is the SMALLEST payload
+     value among them; 0 (default) = unique keys, a duplicate is DDQ_EINVAL (reading
+     O13).  Any build's payload column may be int64 when its load-time range fits
+     int32 (it is narrowed exactly; else DDQ_EINVAL). */
   int32_t build_key_set;
   /* AGGREGATE finalisation (S8(a7), reading O10): n_avg derived double columns,
      avg k = (double)acc[avg_sum[k]] / (double)acc[avg_count] / 10^avg_scale[k] (SQL AVG
@@ -396,6 +403,10 @@ typedef struct {
   int32_t avg_sum[4];
   int32_t avg_count;
   int32_t avg_scale[4];
+  /* GATHER: 1 = gather an int64 column into an int32 vector (exact: allowed only when
+     the column's load-time range fits int32, else DDQ_EINVAL), so it can be compared
+     with FILTER_EQ or carried (TPC-H Q2's ps_supplycost = min cost) */
+  int32_t gather_narrow;
 } ddq_op;
 
 #define DDQ_CMP_EQ 0

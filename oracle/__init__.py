@@ -14,7 +14,8 @@ Parity status per function:
                      on planted tables, group-count / sum-conservation invariants
   listing1..8        pinned: closed form (empty by the SSB value domains), brute force
   listing2b          pinned: numpy.flatnonzero of the predicate, binomial bounds
-  tpch1,3,4,5,6,7    pinned: SQLite 3.45 on decoded tables (tpch4: EXISTS subquery)
+  tpch1-7            pinned: SQLite 3.45 on decoded tables (tpch4: EXISTS subquery;
+                     tpch2: the correlated MIN subquery, LIKE '%BRASS')
 """
 from __future__ import annotations
 
@@ -86,6 +87,11 @@ SSB_QUERY_COLUMNS = {
 LISTING_COLUMNS = {1: "lo_quantity", 2: "lo_discount", 3: "lo_shippriority", 4: "lo_extendedprice",
                    5: "lo_ordtotalprice", 6: "lo_revenue", 7: "lo_supplycost", 8: "lo_tax"}
 TPCH_QUERY_COLUMNS = {
+    2: [("region", "r_regionkey"), ("region", "r_name"), ("nation", "n_nationkey"), ("nation", "n_name"),
+        ("nation", "n_regionkey"), ("supplier", "s_suppkey"), ("supplier", "s_nationkey"),
+        ("supplier", "s_acctbal"), ("part", "p_partkey"), ("part", "p_size"), ("part", "p_type"),
+        ("part", "p_mfgr"), ("partsupp", "ps_partkey"), ("partsupp", "ps_suppkey"),
+        ("partsupp", "ps_supplycost")],
     1: [("lineitem", c) for c in ["l_shipdate", "l_returnflag", "l_linestatus", "l_quantity",
                                   "l_extendedprice", "l_discount", "l_tax"]],
     3: [("customer", "c_custkey"), ("customer", "c_mktsegment"), ("orders", "o_orderkey"),

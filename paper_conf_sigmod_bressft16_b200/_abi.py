@@ -71,7 +71,7 @@ class Op(ctypes.Structure):
                 ("fetch_build", ctypes.c_int32), ("eq_cmp", ctypes.c_int32),
                 ("build_key_set", ctypes.c_int32), ("n_avg", ctypes.c_int32),
                 ("avg_sum", ctypes.c_int32 * 4), ("avg_count", ctypes.c_int32),
-                ("avg_scale", ctypes.c_int32 * 4)]
+                ("avg_scale", ctypes.c_int32 * 4), ("gather_narrow", ctypes.c_int32)]
 
 
 class DevTerm(ctypes.Structure):

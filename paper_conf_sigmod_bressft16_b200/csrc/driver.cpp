@@ -80,7 +80,8 @@ static std::vector<int> op_columns(const ddq_op& op) {
       for (int a = 0; a < op.n_aggs; a++) {
         int need = op.agg_kind[a] == DDQ_AGG_COUNT ? 0 : (op.agg_kind[a] == DDQ_AGG_SUM || op.agg_kind[a] == DDQ_AGG_MIN) ? 1
                  : op.agg_kind[a] == DDQ_AGG_SUM_MUL_100M_100P ? 3 : 2;
-        for (int j = 0; j < need; j++) c.push_back(op.agg_col[a][j]);
+        for (int j = 0; j < need; j++)
+          if (op.agg_col[a][j] >= 0) c.push_back(op.agg_col[a][j]);  // <= -2: an aligned vector
       }
       break;
   }
@@ -479,6 +480,7 @@ ddq_status run_host_op(ddq_db* db, const ddq_op& op, const std::vector<Inter>& I
     case DDQ_OP_HASH_BUILD: {
       const Column* kc = col_of(db, op.key_col);
       const Column* pc = op.payload_col >= 0 ? col_of(db, op.payload_col) : nullptr;
+      if (pc && !fits_int32(*pc)) return set_error(DDQ_EINVAL, "build: payload values do not fit int32");
       int64_t cap = pow2_at_least(std::max<int64_t>(16, 2 * n));
       int lg = 0;
       while ((1ll << lg) < cap) lg++;
@@ -495,13 +497,15 @@ ddq_status run_host_op(ddq_db* db, const ddq_op& op, const std::vector<Inter>& I
         }
         if (!ok) continue;
         int32_t k = ((const int32_t*)kc->host)[r];
-        int32_t v = pc ? ((const int32_t*)pc->host)[r] : r;
+        int32_t v = pc ? (int32_t)hcol(pc, r) : r;  // an int64 payload fits int32 (checked below)
         uint32_t h = host_hash32(k, 32 - lg);
         bool dup = false;
         while ((*t)[h] != kHostEmpty) {
           if ((int32_t)((*t)[h] >> 32) == k) {
             if (!op.build_key_set) return set_error(DDQ_EINVAL, "duplicate build key");
             dup = true;  // key set (semi-join): the first row stays
+            if (op.build_key_set == 2 && v < (int32_t)(uint32_t)(*t)[h])  // MIN build: keep the smallest
+              (*t)[h] = ((uint64_t)(uint32_t)k << 32) | (uint32_t)v;
             break;
           }
           h = (h + 1) & (uint32_t)(cap - 1);
@@ -551,12 +555,15 @@ ddq_status run_host_op(ddq_db* db, const ddq_op& op, const std::vector<Inter>& I
         out.vecs.push_back(Vec{dst, 4, true});
         return DDQ_OK;
       }
-      void* dst = host_alloc(out, (size_t)n * c->width);
+      if (op.gather_narrow && (c->width != 8 || !fits_int32(*c)))
+        return set_error(DDQ_EINVAL, "gather: narrowing needs an int64 column whose values fit int32");
+      const int w = op.gather_narrow ? 4 : c->width;
+      void* dst = host_alloc(out, (size_t)n * w);
       for (int64_t i = 0; i < n; i++) {
-        if (c->width == 8) ((int64_t*)dst)[i] = ((const int64_t*)c->host)[in->tids[i]];
-        else ((int32_t*)dst)[i] = ((const int32_t*)c->host)[in->tids[i]];
+        if (w == 8) ((int64_t*)dst)[i] = ((const int64_t*)c->host)[in->tids[i]];
+        else ((int32_t*)dst)[i] = (int32_t)hcol(c, in->tids[i]);
       }
-      out.vecs.push_back(Vec{dst, c->width, true});
+      out.vecs.push_back(Vec{dst, w, true});
       return DDQ_OK;
     }
     case DDQ_OP_AGGREGATE: {
@@ -595,8 +602,12 @@ ddq_status run_host_op(ddq_db* db, const ddq_op& op, const std::vector<Inter>& I
         if (fresh) acc.assign((size_t)na, 0);
         for (int a = 0; a < na; a++) {
           int kind = op.agg_kind[a];
-          if (kind == DDQ_AGG_MIN) {
-            const __int128 x = hcol(ac[(size_t)a][0], r);
+          if (kind == DDQ_AGG_MIN) {  // operand: a column, or an aligned vector (agg_col <= -2)
+            const int vs = -2 - op.agg_col[a][0];
+            const __int128 x = op.agg_col[a][0] <= -2
+                                   ? (in->vecs[(size_t)vs].width == 8 ? ((const int64_t*)in->vecs[(size_t)vs].ptr)[i]
+                                                                      : ((const int32_t*)in->vecs[(size_t)vs].ptr)[i])
+                                   : (__int128)hcol(ac[(size_t)a][0], r);
             if (fresh || x < acc[(size_t)a]) acc[(size_t)a] = x;
             continue;
           }

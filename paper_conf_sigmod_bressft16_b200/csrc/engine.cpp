@@ -109,6 +109,11 @@ bool use_join_index(const Column& kc, int64_t n_rows) {
   return r <= (1ll << 28) && (r <= (1ll << 20) || r <= 16 * std::max<int64_t>(n_rows, 1));
 }
 
+// An int64 column whose load-time range fits int32 (exact narrowing) or an int32 column.
+bool fits_int32(const Column& c) {
+  return c.width == 4 || c.n == 0 || (c.vmin >= INT32_MIN && c.vmax <= INT32_MAX);
+}
+
 // ----------------------------------------------------------- GPU operator runner
 struct Alloc {
   ddq_db* db;
@@ -358,19 +363,24 @@ ddq_status run_gpu_op(GpuOpCtx& ctx, const ddq_op& op, Inter& out) {
       if (!kc || kc->table != op.table || kc->width != 4) return set_error(DDQ_EINVAL, "build: bad key column");
       const int32_t* keys = (const int32_t*)need_col(op.key_col);
       const int32_t* payload = nullptr;
+      const long long* payload64 = nullptr;
       if (op.payload_col >= 0) {
         const Column* pc = col_of(db, op.payload_col);
-        if (!pc || pc->table != op.table || pc->width != 4) return set_error(DDQ_EINVAL, "build: bad payload column");
-        payload = (const int32_t*)need_col(op.payload_col);
-        if (!payload) return set_error(DDQ_ESTATE, "build: payload column not cached on the GPU");
+        if (!pc || pc->table != op.table || !fits_int32(*pc)) return set_error(DDQ_EINVAL, "build: bad payload column");
+        const void* pp = need_col(op.payload_col);
+        if (!pp) return set_error(DDQ_ESTATE, "build: payload column not cached on the GPU");
+        if (pc->width == 8) payload64 = (const long long*)pp;
+        else payload = (const int32_t*)pp;
       }
+      if (op.build_key_set < 0 || op.build_key_set > 2) return set_error(DDQ_EINVAL, "build: bad build_key_set");
       if (!keys) return set_error(DDQ_ESTATE, "build: key column not cached on the GPU");
       // fused selection (BUILD op with predicates): evaluated per input row in the
       // build kernel
       if (op.n_preds < 0 || op.n_preds > DDQ_MAX_PREDS) return set_error(DDQ_EINVAL, "build: bad n_preds");
       BuildPreds bp;
       bp.n = op.n_preds;
-      bp.key_set = op.build_key_set ? 1 : 0;
+      bp.key_set = op.build_key_set;
+      bp.payload64 = payload64;
       for (int i = 0; i < op.n_preds; i++) {
         const ddq_pred& p = op.preds[i];
         const Column* c = col_of(db, p.column);
@@ -395,6 +405,8 @@ ddq_status run_gpu_op(GpuOpCtx& ctx, const ddq_op& op, Inter& out) {
         if (A.failed) return DDQ_ENOMEM_DEVICE;
         init_fill(out.d_error, 4, 0, st);
         cudaError_t e = join_index_init(out.jidx, out.jrange, st);
+        if (e == cudaSuccess && op.build_key_set == 2)  // MIN build: payloads start at INT32_MAX
+          e = init_fill(join_index_payload(out.jidx, out.jrange), (size_t)out.jrange * 4, 0x7FFFFFFF7FFFFFFFull, st);
         if (e == cudaSuccess)
           e = launch_join_index_build(keys, payload, in_tids, in_cnt, in_cap, out.jmin, out.jrange, out.jidx,
                                       out.d_error, st, &bp);
@@ -443,10 +455,14 @@ ddq_status run_gpu_op(GpuOpCtx& ctx, const ddq_op& op, Inter& out) {
                                         B.table_ptr, B.table_cap, dst, st),
                            "fetch");
       }
-      void* dst = A.get((uint64_t)std::max<int64_t>(in->cap, 1) * c->width);
+      if (op.gather_narrow && (c->width != 8 || !fits_int32(*c)))
+        return set_error(DDQ_EINVAL, "gather: narrowing needs an int64 column whose values fit int32");
+      const int w = op.gather_narrow ? 4 : c->width;
+      void* dst = A.get((uint64_t)std::max<int64_t>(in->cap, 1) * w);
       if (A.failed) return DDQ_ENOMEM_DEVICE;
-      out.vecs.push_back(Vec{dst, c->width, false});
-      return cuda_status(launch_gather(src, c->width, in->tids, in->d_count, in->cap, dst, st), "gather");
+      out.vecs.push_back(Vec{dst, w, false});
+      return cuda_status(launch_gather(src, op.gather_narrow ? -8 : c->width, in->tids, in->d_count, in->cap, dst, st),
+                         "gather");
     }
     case DDQ_OP_AGGREGATE: {
       // no input: every row of op.table (a dense aggregation, e.g. TPC-H Q1 with
@@ -479,6 +495,14 @@ ddq_status run_gpu_op(GpuOpCtx& ctx, const ddq_op& op, Inter& out) {
         int need = op.agg_kind[a] == DDQ_AGG_COUNT ? 0 : (op.agg_kind[a] == DDQ_AGG_SUM || op.agg_kind[a] == DDQ_AGG_MIN) ? 1
                  : op.agg_kind[a] == DDQ_AGG_SUM_MUL_100M_100P ? 3 : 2;
         for (int j = 0; j < need; j++) {
+          if (op.agg_col[a][j] <= -2) {  // MIN over an aligned vector: positional (negative width)
+            const int v = -2 - op.agg_col[a][j];
+            if (op.agg_kind[a] != DDQ_AGG_MIN || !in || op.n_preds > 0 || v >= (int)in->vecs.size())
+              return set_error(DDQ_EINVAL, "aggregate: a vector operand needs MIN, an input and no fused predicates");
+            ag[a].arg[j] = in->vecs[(size_t)v].ptr;
+            ag[a].width[j] = -in->vecs[(size_t)v].width;
+            continue;
+          }
           const Column* c = col_of(db, op.agg_col[a][j]);
           if (!c || c->table != op.table) return set_error(DDQ_EINVAL, "aggregate: bad argument column");
           ag[a].arg[j] = need_col(op.agg_col[a][j]);
@@ -1343,6 +1367,8 @@ static ddq_status validate_plan(ddq_db* db, const ddq_plan* plan) {
         return set_error(DDQ_EINVAL, "plan: IN list must hold 0..8 values");
     }
     if (op.kind == DDQ_OP_AGGREGATE && (op.n_avg < 0 || op.n_avg > 4)) return set_error(DDQ_EINVAL, "plan: n_avg 0..4");
+    if (op.kind == DDQ_OP_HASH_BUILD && (op.build_key_set < 0 || op.build_key_set > 2))
+      return set_error(DDQ_EINVAL, "plan: build_key_set must be 0, 1 or 2");
     if (op.input >= i || op.input < -1) return set_error(DDQ_EINVAL, "plan: input must precede the op");
     if (op.kind == DDQ_OP_HASH_PROBE && (op.build < 0 || op.build >= i ||
                                          plan->ops[op.build].kind != DDQ_OP_HASH_BUILD))

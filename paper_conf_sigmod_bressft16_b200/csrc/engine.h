@@ -185,5 +185,6 @@ ddq_status finalize_result(const ddq_op& root, int64_t n_groups, const int64_t* 
 void decode_result_keys(ddq_db* db, const ddq_plan& plan, ddq_result* r);
 int64_t pow2_at_least(int64_t x);
 const ddq::Column* col_of(ddq_db* db, int c);
+bool fits_int32(const ddq::Column& c);
 
 }  // namespace ddq

@@ -66,7 +66,7 @@ __global__ void hash_build_kernel(const int32_t* __restrict__ keys, const int32_
     const int32_t r = in_tids ? in_tids[i] : (int32_t)i;
     if (bp.n && !build_row_passes(bp, r)) continue;
     const int32_t k = keys[r];
-    const int32_t v = payload ? payload[r] : r;
+    const int32_t v = bp.payload64 ? (int32_t)bp.payload64[r] : payload ? payload[r] : r;
     if (k == INT32_MIN) {
       atomicMax(d_error, 3u);
       continue;
@@ -80,6 +80,13 @@ __global__ void hash_build_kernel(const int32_t* __restrict__ keys, const int32_
       if (old == HT_EMPTY) break;
       if (ht_key(old) == k) {  // PKs must be unique (reading O13) unless a key set
         if (!bp.key_set) atomicMax(d_error, 1u);
+        // MIN build: lower the slot's payload until it holds the smallest value
+        while (bp.key_set == 2 && v < ht_val(old)) {
+          const unsigned long long seen = atomicCAS(reinterpret_cast<unsigned long long*>(table + h), old,
+                                                    (unsigned long long)slot);
+          if (seen == old) break;
+          old = seen;
+        }
         break;
       }
       h = (h + 1) & mask;
@@ -211,6 +218,16 @@ __global__ void join_index_build_kernel(const int32_t* __restrict__ keys, const 
     }
     const uint32_t old = atomicOr(bitmap + (o >> 5), 1u << (o & 31));
     if ((old & (1u << (o & 31))) && !bp.key_set) atomicMax(d_error, 1u);  // PKs are unique (O13)
+    const int32_t v = bp.payload64 ? (int32_t)bp.payload64[r] : payload ? payload[r] : r;
+    if (bp.key_set == 2) {  // MIN build: payload array pre-filled with INT32_MAX
+      atomicMin(payarr + o, v);
+      if (coarse) {
+        uint32_t* cw = coarse + ((o >> cg) >> 5);
+        const uint32_t cb = 1u << ((o >> cg) & 31);
+        if (!(*reinterpret_cast<volatile uint32_t*>(cw) & cb)) atomicOr(cw, cb);
+      }
+      continue;
+    }
     if (coarse) {  // most coarse bits are set early: test before the atomic
       uint32_t* cw = coarse + ((o >> cg) >> 5);
       const uint32_t cb = 1u << ((o >> cg) & 31);
@@ -219,7 +236,7 @@ __global__ void join_index_build_kernel(const int32_t* __restrict__ keys, const 
     // only the row that set the bit writes the payload: a key set's duplicates
     // (O32; ~3 of 4 late lineitems of TPC-H Q4) skip their random 4-byte store
     // (measured neutral on B200: Q4's key-set build stays at 100 us, atomic-bound)
-    if (!(old & (1u << (o & 31)))) payarr[o] = payload ? payload[r] : r;
+    if (!(old & (1u << (o & 31)))) payarr[o] = v;
   }
 }
 
@@ -236,6 +253,8 @@ cudaError_t launch_join_index_build(const int32_t* keys, const int32_t* payload,
 }
 
 // --------------------------------------------------------------------- gather
+// W = 8 / 4: copy; W = -8: an int64 column narrowed to an int32 vector (the caller
+// checked from the column's load-time range that every value fits)
 template <int W>
 __global__ void gather_kernel(const void* __restrict__ col, const int32_t* __restrict__ tids,
                               const uint32_t* d_count, uint32_t n_static, void* __restrict__ out) {
@@ -244,6 +263,8 @@ __global__ void gather_kernel(const void* __restrict__ col, const int32_t* __res
     const int32_t r = tids[i];
     if (W == 8)
       reinterpret_cast<long long*>(out)[i] = ldg_gather(reinterpret_cast<const long long*>(col) + r);
+    else if (W == -8)
+      reinterpret_cast<int*>(out)[i] = (int)ldg_gather(reinterpret_cast<const long long*>(col) + r);
     else
       reinterpret_cast<int*>(out)[i] = ldg_gather(reinterpret_cast<const int32_t*>(col) + r);
   }
@@ -310,6 +331,8 @@ cudaError_t launch_gather(const void* col, int width, const int32_t* tids, const
   int grid = (int)(g > num_sms() * 16 ? num_sms() * 16 : (g < 1 ? 1 : g));
   if (width == 8)
     gather_kernel<8><<<grid, 256, 0, st>>>(col, tids, d_count, (uint32_t)n_cap, out);
+  else if (width == -8)
+    gather_kernel<-8><<<grid, 256, 0, st>>>(col, tids, d_count, (uint32_t)n_cap, out);
   else
     gather_kernel<4><<<grid, 256, 0, st>>>(col, tids, d_count, (uint32_t)n_cap, out);
   return cudaGetLastError();
@@ -629,8 +652,9 @@ __global__ void groupby_generic_kernel(const __grid_constant__ GroupbyParams P) 
     }
     for (int a = 0; a < P.n_aggs; a++) {
       unsigned long long* cell = &P.g_accs[((size_t)a * cap + slot) * 2];
-      if (P.kind[a] == DDQ_AGG_MIN) {
-        atomicMin(reinterpret_cast<long long*>(cell), col_at(P.arg[a][0], P.width[a][0], r));
+      if (P.kind[a] == DDQ_AGG_MIN) {  // width < 0: an aligned vector, indexed by position
+        const int w = P.width[a][0];
+        atomicMin(reinterpret_cast<long long*>(cell), w < 0 ? col_at(P.arg[a][0], -w, i) : col_at(P.arg[a][0], w, r));
       } else {
         const long long v = agg_value(P, a, r);
         atomic_add_i128_pair(cell, cell + 1, (unsigned long long)v, v < 0 ? -1 : 0);

@@ -81,9 +81,13 @@ cudaError_t launch_ws(const FilterArgs& a, cudaStream_t st);
 // fail any predicate are not inserted -- the select -> build pair of a dimension
 // table in one kernel, without the intermediate TID list.
 struct BuildPreds {
-  int32_t key_set = 0;  // 1: duplicate build keys allowed (semi-join key set, ddq_op.build_key_set)
+  int32_t key_set = 0;  // 1: duplicate build keys allowed (semi-join key set, ddq_op.build_key_set);
+                        // 2: duplicates allowed, the payload is their MINIMUM (a MIN-aggregating
+                        //    build: TPC-H Q2's decorrelated min(ps_supplycost) per part)
   int32_t n = 0;
   ddq_dev_pred p[DDQ_MAX_PREDS];
+  const long long* payload64 = nullptr;  // int64 payload column whose values fit int32 (checked
+                                         // from the column's load-time range), narrowed exactly
 };
 
 cudaError_t launch_hash_init(uint64_t* table, uint32_t capacity, cudaStream_t st);

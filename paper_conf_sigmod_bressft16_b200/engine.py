@@ -114,13 +114,14 @@ class PlanBuilder:
                     pr.in_vals[j] = int(v)
 
     def build(self, table: str, key: str, payload: str | None = None, input: int = -1,
-              where: list | None = None, key_set: bool = False) -> int:
+              where: list | None = None, key_set: bool | str = False) -> int:
         """where: predicates evaluated on the input rows inside the build (a fused
         selection: no intermediate TID list), same forms as select().  key_set:
-        the build is the key set of a semi-join (EXISTS / IN): duplicate keys
-        allowed (reading O32)."""
+        True = the key set of a semi-join (EXISTS / IN), duplicate keys allowed
+        (reading O32); "min" = duplicate keys keep the smallest payload (a
+        decorrelated MIN subquery, reading O35)."""
         idx, op = self._op(A.OP_HASH_BUILD, table, input)
-        op.build_key_set = 1 if key_set else 0
+        op.build_key_set = 2 if key_set == "min" else 1 if key_set else 0
         op.key_col = self.db.col(table, key)
         op.payload_col = self.db.col(table, payload) if payload else -1
         if where:
@@ -181,9 +182,11 @@ class PlanBuilder:
         comparison, e.g. TPC-H Q4's l_commitdate < l_receiptdate)."""
         return self.filter_eq(table, input, vec_a, vec_b, A.CMP_LT)
 
-    def gather(self, table: str, col: str, input: int) -> int:
+    def gather(self, table: str, col: str, input: int, narrow: bool = False) -> int:
+        """narrow: an int64 column whose values fit int32 becomes an int32 vector."""
         idx, op = self._op(A.OP_GATHER, table, input)
         op.gather_col = self.db.col(table, col)
+        op.gather_narrow = 1 if narrow else 0
         return idx
 
     def fetch(self, table: str, fk: str, build: int, input: int) -> int:
@@ -214,8 +217,9 @@ class PlanBuilder:
         op.n_aggs = len(aggs)
         for a, (kind, cols) in enumerate(aggs):
             op.agg_kind[a] = kind
-            for j in range(3):
-                op.agg_col[a][j] = self.db.col(table, cols[j]) if j < len(cols) else -1
+            for j in range(3):  # an int operand = aligned vector index (MIN only): -2 - v
+                c = cols[j] if j < len(cols) else None
+                op.agg_col[a][j] = -1 if c is None else (-2 - c if isinstance(c, int) else self.db.col(table, c))
         order_by = order_by or []
         op.n_order = len(order_by)
         for i, o in enumerate(order_by):

@@ -9,13 +9,15 @@ from .engine import Database, PlanBuilder
 from .ssb import code
 
 
-TPCH_QUERIES = ["tpch1", "tpch3", "tpch4", "tpch5", "tpch6", "tpch7"]
+TPCH_QUERIES = ["tpch1", "tpch2", "tpch3", "tpch4", "tpch5", "tpch6", "tpch7"]
 
 TABLE_COLUMNS = {
     "nation": ["n_nationkey", "n_name", "n_regionkey"],
     "region": ["r_regionkey", "r_name"],
     "customer": ["c_custkey", "c_nationkey", "c_mktsegment"],
-    "supplier": ["s_suppkey", "s_nationkey"],
+    "supplier": ["s_suppkey", "s_nationkey", "s_acctbal"],
+    "part": ["p_partkey", "p_mfgr", "p_type", "p_size"],
+    "partsupp": ["ps_partkey", "ps_suppkey", "ps_supplycost"],
     "orders": ["o_orderkey", "o_custkey", "o_orderdate", "o_shippriority", "o_orderpriority"],
     "lineitem": ["l_orderkey", "l_suppkey", "l_quantity", "l_extendedprice", "l_discount", "l_tax",
                  "l_returnflag", "l_linestatus", "l_shipdate", "l_commitdate", "l_receiptdate"],
@@ -23,8 +25,9 @@ TABLE_COLUMNS = {
 }
 STRING_DICTS = {"n_name": "nation", "r_name": "region", "c_mktsegment": "mktsegment",
                 "l_returnflag": "returnflag", "l_linestatus": "linestatus",
-                "o_orderpriority": "orderpriority"}
+                "o_orderpriority": "orderpriority", "p_type": "type", "p_mfgr": "tpch_mfgr"}
 QUERY_TABLES = {"tpch1": ["lineitem"], "tpch6": ["lineitem"],
+                "tpch2": ["region", "nation", "supplier", "part", "partsupp"],
                 "tpch3": ["customer", "orders", "lineitem"],
                 "tpch4": ["orders", "lineitem"],
                 "tpch7": ["nation", "supplier", "customer", "orders", "lineitem", "calendar"],
@@ -40,6 +43,10 @@ def _bits(db, table: str, col: str) -> int:
     if lo < 0:
         raise ValueError(f"{table}.{col}: negative group key")
     return max(1, int(hi).bit_length())
+
+
+def _rows(db, table: str) -> int:
+    return db.table_rows(table) if hasattr(db, "table_rows") else 1 << 20
 
 
 def load_tpch(db: Database, data, cache: bool = True, tables=None) -> None:
@@ -85,6 +92,38 @@ def tpch_plan(db: Database, q: str, limit: int = 0, dense: bool = True) -> PlanB
         t = P.select(li, [("l_quantity", -2**62, 2399)], input=t)
         P.aggregate(li, t, keys=[], aggs=[(A.AGG_SUM_MUL, ["l_extendedprice", "l_discount"]),
                                           (A.AGG_COUNT, [])], max_groups=1)
+        return P
+    if q == "tpch2":
+        # The correlated scalar subquery ps_supplycost = (select min(ps_supplycost) ..
+        # where p_partkey = ps_partkey ..) decorrelated (reading O35): the European
+        # partsupp rows of the qualifying parts build a MIN-aggregating index
+        # ps_partkey -> min cost, and the same rows keep those whose cost equals it.
+        eu = code(db, "region", "EUROPE")
+        r = P.select("region", [("r_name", [eu])])
+        hr = P.build("region", "r_regionkey", input=r)
+        n = P.probe("nation", "n_regionkey", hr)                          # nations of EUROPE
+        hn = P.build("nation", "n_nationkey", "n_name", input=n)
+        s = P.probe("supplier", "s_nationkey", hn)                        # European suppliers
+        hsn = P.build("supplier", "s_suppkey", "s_nationkey", input=s)
+        hsa = P.build("supplier", "s_suppkey", "s_acctbal", input=s)      # int64 payload, fits int32
+        # p_size = 15 and p_type like '%BRASS' (a dictionary code set, ddq_dictionary_like)
+        hp = P.build("part", "p_partkey", "p_mfgr", where=[("p_size", 15, 15), db.like("part", "p_type", "%BRASS")])
+        ps = "partsupp"
+        t = P.probe(ps, "ps_partkey", hp, emit=True)                      # vec0 = p_mfgr
+        t = P.probe(ps, "ps_suppkey", hsn, input=t, emit=True)            # vec1 = s_nationkey
+        hm = P.build(ps, "ps_partkey", "ps_supplycost", input=t, key_set="min")
+        t = P.probe(ps, "ps_partkey", hm, input=t, emit=True)             # vec2 = the part's min cost
+        t = P.gather(ps, "ps_supplycost", t, narrow=True)                 # vec3 = ps_supplycost
+        t = P.filter_eq(ps, t, 2, 3)                                      # ps_supplycost = min
+        t = P.probe(ps, 1, hn, input=t, emit=True)                        # vec4 = n_name
+        t = P.fetch(ps, "ps_suppkey", hsa, t)                             # vec5 = s_acctbal
+        # one row per (part, supplier): the select list's supplier / nation / part
+        # attributes are functionally dependent -> MIN; order by s_acctbal desc,
+        # n_name, s_name (= s_suppkey), p_partkey
+        P.aggregate(ps, t, keys=["ps_partkey", "ps_suppkey"],
+                    key_bits=[_bits(db, ps, "ps_partkey"), _bits(db, ps, "ps_suppkey")],
+                    aggs=[(A.AGG_MIN, [5]), (A.AGG_MIN, [4]), (A.AGG_MIN, [0])],
+                    order_by=[-101, 102, 2, 1], max_groups=max(1024, _rows(db, ps)), limit=limit)
         return P
     if q == "tpch3":
         c = P.select("customer", [("c_mktsegment", [code(db, "mktsegment", "BUILDING")])])

@@ -21,6 +21,21 @@ select l_returnflag, l_linestatus, sum(l_quantity), sum(l_extendedprice),
        sum(l_discount), count(*), avg(l_quantity), avg(l_extendedprice), avg(l_discount)
   from lineitem where l_shipdate <= 19980902
  group by l_returnflag, l_linestatus order by l_returnflag, l_linestatus;
+-- @tpch2
+-- Q2 (SIZE 15, TYPE BRASS, REGION EUROPE).  Reading O35: s_name is reported as
+-- s_suppkey (TPC-H's s_name = 'Supplier#' || lpad(s_suppkey, 9, '0') sorts the same),
+-- the free-text columns s_address, s_phone, s_comment are not generated, and LIMIT
+-- 100 is dropped so the whole ordered set is compared.
+select s_acctbal, s_suppkey, n_name, p_partkey, p_mfgr
+  from part, supplier, partsupp, nation, region
+ where p_partkey = ps_partkey and s_suppkey = ps_suppkey and p_size = 15
+   and p_type like '%BRASS' and s_nationkey = n_nationkey and n_regionkey = r_regionkey
+   and r_name = 'EUROPE'
+   and ps_supplycost = (select min(ps_supplycost) from partsupp, supplier, nation, region
+                         where p_partkey = ps_partkey and s_suppkey = ps_suppkey
+                           and s_nationkey = n_nationkey and n_regionkey = r_regionkey
+                           and r_name = 'EUROPE')
+ order by s_acctbal desc, n_name, s_suppkey, p_partkey;
 -- @tpch3
 select l_orderkey, o_orderdate, o_shippriority, sum(l_extendedprice*(100-l_discount)) as revenue
   from customer, orders, lineitem

@@ -71,7 +71,7 @@ def test_tpch_sf30_all_queries_equal_oracle(keys):
     data = datagen.TPCH(30, keys=keys)
     db = Database(cache_bytes=64 << 30, heap_bytes=24 << 30)
     load_tpch(db, data)
-    qs = ("tpch1", "tpch3", "tpch4", "tpch5", "tpch6", "tpch7")
+    qs = ("tpch1", "tpch2", "tpch3", "tpch4", "tpch5", "tpch6", "tpch7")
     got = {}
     for q in qs:
         p = db.prepare(tpch_plan(db, q))

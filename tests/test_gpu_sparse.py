@@ -21,7 +21,7 @@ pytestmark = pytest.mark.gpu
 
 VARIANTS = {"chain": dict(star=False), "star": dict(star=True), "chain_eager": dict(star=False, late=False),
             "chain_unfused": dict(star=False, fused_build=False, late=False, fused_agg=False)}
-TPCH = ["tpch1", "tpch3", "tpch4", "tpch5", "tpch6", "tpch7"]
+TPCH = ["tpch1", "tpch2", "tpch3", "tpch4", "tpch5", "tpch6", "tpch7"]
 
 
 @functools.lru_cache(maxsize=None)

@@ -33,7 +33,7 @@ def _want(q):
     return [tuple(r) for r in oracle.run(_data(), q)]
 
 
-@pytest.mark.parametrize("q", ["tpch1", "tpch3", "tpch4", "tpch5", "tpch6", "tpch7"])
+@pytest.mark.parametrize("q", ["tpch1", "tpch2", "tpch3", "tpch4", "tpch5", "tpch6", "tpch7"])
 def test_tpch_prepared_equals_oracle(q):
     from paper_conf_sigmod_bressft16_b200.tpch import tpch_plan
     db = _db()
@@ -44,7 +44,7 @@ def test_tpch_prepared_equals_oracle(q):
     assert got and got == _want(q)
 
 
-@pytest.mark.parametrize("q", ["tpch1", "tpch3", "tpch4", "tpch5", "tpch6", "tpch7"])
+@pytest.mark.parametrize("q", ["tpch1", "tpch2", "tpch3", "tpch4", "tpch5", "tpch6", "tpch7"])
 def test_tpch_submit_equals_oracle(q):
     from paper_conf_sigmod_bressft16_b200.tpch import tpch_plan
     db = _db()
@@ -301,4 +301,113 @@ def test_aggregate_min(shape):
         p.launch()
         assert [tuple(v) for v in p.fetch().rows] == want
         p.close()
+    db.close()
+
+
+class _Ties:
+    """TPC-H data with every ps_supplycost equal: each qualifying part's minimum is
+    reached by ALL its European suppliers, so Q2 must return every such row (SQL
+    `=` against the subquery's MIN, not an arg-min)."""
+
+    def __init__(self, d):
+        import numpy as np
+        self.d = d
+        self.cost = np.full(d.rows("partsupp"), 50000, np.int64)
+
+    def col(self, t, c):
+        return self.cost if (t, c) == ("partsupp", "ps_supplycost") else self.d.col(t, c)
+
+    def rows(self, t):
+        return self.d.rows(t)
+
+    def dict_for(self, c):
+        return self.d.dict_for(c)
+
+
+@pytest.mark.parametrize("path", ["prepared", "submit", "host"])
+def test_tpch2_min_ties(path):
+    from paper_conf_sigmod_bressft16_b200 import Database
+    from paper_conf_sigmod_bressft16_b200 import _abi as A
+    from paper_conf_sigmod_bressft16_b200.tpch import load_tpch, tpch_plan
+    data = _Ties(_data())
+    want = [tuple(r) for r in oracle.run(data, "tpch2")]
+    assert len({r[0] for r in want}) < len(want)  # several suppliers per part tie
+    db = Database(cache_bytes=4 << 30, heap_bytes=2 << 30,
+                  **(dict(placement=A.PLACE_CPU_ONLY) if path == "host" else {}))
+    load_tpch(db, data, tables=["region", "nation", "supplier", "part", "partsupp"])
+    if path == "prepared":
+        p = db.prepare(tpch_plan(db, "tpch2"))
+        p.launch()
+        got = p.fetch().rows
+        p.close()
+    else:
+        got = db.run(tpch_plan(db, "tpch2")).rows
+    db.close()
+    assert got == want
+
+
+def test_tpch2_limit100():
+    from paper_conf_sigmod_bressft16_b200 import Database
+    from paper_conf_sigmod_bressft16_b200.tpch import load_tpch, tpch_plan
+    data = datagen.TPCH(1)
+    want = [tuple(r) for r in oracle.run(data, "tpch2")]
+    assert len(want) > 100
+    db = Database(cache_bytes=4 << 30, heap_bytes=2 << 30)
+    load_tpch(db, data, tables=["region", "nation", "supplier", "part", "partsupp"])
+    assert db.run(tpch_plan(db, "tpch2", limit=100)).rows == want[:100]
+    db.close()
+
+
+@pytest.mark.parametrize("index", ["join_index", "hash"])
+def test_min_build_and_narrow_gather(index):
+    """A MIN-aggregating build (build_key_set = 2) over duplicate keys, read back by a
+    fetch at every row, equals numpy's per-key minimum; an int64 payload is narrowed
+    exactly; a narrowing GATHER of a column whose values do not fit int32 is refused."""
+    import numpy as np
+    from paper_conf_sigmod_bressft16_b200 import Database, DDQError
+    from paper_conf_sigmod_bressft16_b200 import _abi as A
+    rng = np.random.default_rng(11)
+    n = 100_003
+    nk = 997
+    keys = rng.integers(0, nk, n).astype(np.int32)
+    if index == "hash":  # a sparse key range: open addressing (reading O24)
+        keys = (keys.astype(np.int64) * 1_000_003 + 7).astype(np.int32)
+    vals = rng.integers(-2**31, 2**31 - 1, n).astype(np.int64)
+    big = vals.copy()
+    big[5] = 2**40
+    db = Database(cache_bytes=1 << 30, heap_bytes=1 << 30)
+    db.create_table("t", n)
+    for c, v in (("k", keys), ("v", vals), ("big", big)):
+        db.load_column("t", c, v)
+        db.cache("t", c)
+    P = db.plan()
+    hm = P.build("t", "k", "v", key_set="min")
+    t = P.select("t", [("k", -2**31, 2**31 - 1)])
+    t = P.fetch("t", "k", hm, t)                      # vec0 = min of the row's key
+    t = P.gather("t", "v", t, narrow=True)            # vec1 = own value
+    t = P.filter_eq("t", t, 0, 1)                     # rows holding their key's minimum
+    P.aggregate("t", t, keys=["k"], key_bits=[32], aggs=[(A.AGG_COUNT, []), (A.AGG_MIN, [1])], max_groups=4096)
+    mins = {}
+    for k, v in zip(keys.tolist(), vals.tolist()):
+        mins[k] = min(mins.get(k, v), v)
+    cnt = {}
+    for k, v in zip(keys.tolist(), vals.tolist()):
+        if v == mins[k]:
+            cnt[k] = cnt.get(k, 0) + 1
+    want = sorted((k & 0xFFFFFFFF, cnt[k], mins[k]) for k in cnt)
+    for path in ("prepared", "submit"):
+        if path == "prepared":
+            p = db.prepare(P)
+            p.launch()
+            got = p.fetch().rows
+            p.close()
+        else:
+            got = db.run(P).rows
+        assert sorted(got) == want, path
+    Q = db.plan()
+    t = Q.select("t", [("k", -2**31, 2**31 - 1)])
+    t = Q.gather("t", "big", t, narrow=True)
+    Q.aggregate("t", t, keys=[], aggs=[(A.AGG_COUNT, [])], max_groups=1)
+    with pytest.raises(DDQError):
+        db.prepare(Q)
     db.close()
