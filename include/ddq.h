@@ -264,6 +264,9 @@ typedef struct {
                                     cold cache load copies that and widens it on the device
                                     (fewer bytes over PCIe);
                                     0: copy the raw column */
+  uint32_t fault_op_mask;        /* fault injection: the GPU attempt of plan op i (i < 32) aborts as if
+                                    its heap allocation failed when bit i is set (deterministic
+                                    abort -> host restart traces, Fig. 8); 0 = off */
 } ddq_config;
 
 void ddq_config_default(ddq_config* cfg);
@@ -462,7 +465,14 @@ typedef struct {
      aligned vector was gathered from / a build emitted as payload.  Strings are
      owned by the database (valid until ddq_close); the pointer array by the result. */
   const char* const* key_str;
+  /* placement trace (driver results only; prepared plans: NULL): op_place[i] for plan
+     op i = DDQ_RAN_GPU, DDQ_RAN_HOST, or DDQ_RAN_ABORTED (started on the GPU, aborted
+     on allocation failure, restarted on the host) */
+  int32_t n_ops;
+  int32_t _pad2;
+  const uint8_t* op_place;
 } ddq_result;
+enum { DDQ_RAN_GPU = 1, DDQ_RAN_HOST = 2, DDQ_RAN_ABORTED = 3 };
 
 /* Submit a plan (copied; thread-safe; many user threads may submit). */
 ddq_status ddq_submit(ddq_db* db, const ddq_plan* plan, ddq_query* out);

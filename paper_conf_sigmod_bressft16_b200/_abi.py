@@ -26,6 +26,7 @@ AGG_COUNT, AGG_SUM, AGG_SUM_MUL, AGG_SUM_SUB, AGG_SUM_MUL_100M, AGG_SUM_MUL_100M
 AGG_MIN = 7  # min(a): S8(a6); generic global-table kernel
 I32, I64 = 1, 2
 PLACE_DATA_DRIVEN, PLACE_GPU_ONLY, PLACE_CPU_ONLY = 0, 1, 2
+RAN_GPU, RAN_HOST, RAN_ABORTED = 1, 2, 3  # ddq_result.op_place
 
 
 class DevPred(ctypes.Structure):
@@ -44,7 +45,7 @@ class Config(ctypes.Structure):
                 ("gpu_workers", ctypes.c_int32), ("host_workers", ctypes.c_int32),
                 ("placement", ctypes.c_int32), ("chopping", ctypes.c_int32),
                 ("cache_policy", ctypes.c_int32), ("fault_alloc_every", ctypes.c_uint32),
-                ("transfer_packing", ctypes.c_int32)]
+                ("transfer_packing", ctypes.c_int32), ("fault_op_mask", ctypes.c_uint32)]
 
 
 class Pred(ctypes.Structure):
@@ -93,7 +94,8 @@ class Result(ctypes.Structure):
                 ("gpu_ops", ctypes.c_int32), ("host_ops", ctypes.c_int32), ("aborts", ctypes.c_int32),
                 ("exec_ms", ctypes.c_double), ("agg_null", ctypes.POINTER(ctypes.c_uint8)),
                 ("n_avg", ctypes.c_int32), ("_pad", ctypes.c_int32), ("avgs", ctypes.POINTER(ctypes.c_double)),
-                ("key_str", ctypes.POINTER(ctypes.c_char_p))]
+                ("key_str", ctypes.POINTER(ctypes.c_char_p)), ("n_ops", ctypes.c_int32), ("_pad2", ctypes.c_int32),
+                ("op_place", ctypes.POINTER(ctypes.c_uint8))]
 
 
 class Stats(ctypes.Structure):

@@ -666,12 +666,12 @@ cudaError_t launch_agg_ws(const int32_t* tids, const uint32_t* d_count, int64_t 
   p.s_slots = S;
   p.s_shift = 32 - slg;
   const size_t smem = (size_t)S * (8 + 16 * (size_t)n_aggs);
-  static bool attr = false;
-  if (!attr) {
+  static const bool attr = [] {  // thread-safe one-time opt-in
     cudaFuncSetAttribute(agg_ws_kernel<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, AG_MAX_SLOTS * (8 + 16));
     cudaFuncSetAttribute(agg_ws_kernel<2>, cudaFuncAttributeMaxDynamicSharedMemorySize, AG_MAX_SLOTS * (8 + 32));
-    attr = true;
-  }
+    return true;
+  }();
+  (void)attr;
   const int64_t ntiles = (n_cap + AG_TILE - 1) / AG_TILE;  // upper bound
   int64_t grid = num_sms();
   const int64_t need = (ntiles + AG_NW - 1) / AG_NW;
@@ -772,8 +772,7 @@ cudaError_t launch_agg_dense(int64_t n_rows, const int32_t* const* key_col, int 
   p.shift = 64 - lg;
   p.d_error = d_error;
   const size_t smem = (size_t)p.n_stages * p.stage_bytes + ((size_t)p.D * n_aggs) * (DS_T * 8 + 16);
-  static bool attr = false;
-  if (!attr) {
+  static const bool attr = [] {  // thread-safe one-time opt-in
     const int mx = (int)DS_SMEM_MAX;
     cudaFuncSetAttribute(agg_dense_small_kernel<6, DS_Q1>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx);
     cudaFuncSetAttribute(agg_dense_small_kernel<1, DS_RUNTIME>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx);
@@ -784,8 +783,9 @@ cudaError_t launch_agg_dense(int64_t n_rows, const int32_t* const* key_col, int 
     cudaFuncSetAttribute(agg_dense_small_kernel<6, DS_RUNTIME>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx);
     cudaFuncSetAttribute(agg_dense_small_kernel<7, DS_RUNTIME>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx);
     cudaFuncSetAttribute(agg_dense_small_kernel<8, DS_RUNTIME>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx);
-    attr = true;
-  }
+    return true;
+  }();
+  (void)attr;
   if (n_rows == 0) return cudaSuccess;
   const int64_t nch = (n_rows + DS_SR - 1) / DS_SR;
   int64_t grid = num_sms();

@@ -633,7 +633,9 @@ bool ws_supported(const FilterArgs& a) {
 static bool stage_pays(int64_t n_cap, size_t tab) { return n_cap >= (int64_t)(tab * 4); }
 
 cudaError_t launch_ws(const FilterArgs& a, cudaStream_t st) {
-  if (!g_optin) {
+  // one-time opt-in of every variant's dynamic shared memory; a function-local static
+  // initialiser, so concurrent GPU workers wait for it (no launch before the attributes)
+  static const bool ws_ready = [] {
     int dev = 0, v = 0;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&v, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
@@ -646,7 +648,9 @@ cudaError_t launch_ws(const FilterArgs& a, cudaStream_t st) {
     ws_attr_kind<WK_SEL_GENERIC>();
     ws_attr_kind<WK_EQ>();
     ws_attr_kind<WK_BM_COARSE>();
-  }
+    return true;
+  }();
+  (void)ws_ready;
   const int in = a.in_bits ? 2 : (a.in_tids ? 1 : 0);
   WsParams p{};
   p.n = (uint32_t)a.n_cap;

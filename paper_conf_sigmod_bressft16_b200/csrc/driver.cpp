@@ -42,18 +42,22 @@ struct QueryState {
   std::vector<int> place;                   // compile-time placement (chopping=0)
   std::vector<int> consumers_left;          // for freeing intermediates early
   int ops_left = 0;
+  int inflight = 0;          // operators of this query a worker is running right now
+  bool failed = false;       // an operator failed: remaining ops are dropped
+  bool released = false;     // intermediates of a failed query freed (once, at inflight == 0)
   bool done = false;
   ddq_status status = DDQ_OK;
   std::string error;
   ddq_result* result = nullptr;
   uint64_t t_submit = 0, t_done = 0;
   int gpu_ops = 0, host_ops = 0, aborts = 0;
+  std::vector<uint8_t> trace;               // per op: DDQ_RAN_GPU / _HOST / _ABORTED
   std::mutex mu;
   std::condition_variable cv;
 };
 
 // ------------------------------------------------------------ column helpers
-static std::vector<int> op_columns(const ddq_op& op) {
+std::vector<int> op_columns(const ddq_op& op) {
   std::vector<int> c;
   switch (op.kind) {
     case DDQ_OP_SELECT:
@@ -772,6 +776,10 @@ static void finish_query(ddq_db* db, QueryState& q) {
     res->gpu_ops = q.gpu_ops;
     res->host_ops = q.host_ops;
     res->aborts = q.aborts;
+    uint8_t* tr = new uint8_t[std::max<size_t>(q.trace.size(), 1)];
+    std::copy(q.trace.begin(), q.trace.end(), tr);
+    res->n_ops = (int32_t)q.trace.size();
+    res->op_place = tr;
   }
   q.t_done = now_ns();
   if (res) res->exec_ms = (double)(q.t_done - q.t_submit) / 1e6;
@@ -781,13 +789,17 @@ static void finish_query(ddq_db* db, QueryState& q) {
   q.cv.notify_all();
 }
 
+// A failed operator fails its query: waiters are woken at once, but the query's
+// intermediates are released only when no operator of it is still running (the
+// caller is itself in flight; worker_loop releases when the count drains).
 static void fail_query(ddq_db* db, QueryState& q, ddq_status s) {
+  (void)db;
   std::string msg = ddq_last_error();
-  for (auto& x : q.inters) release_inter(db, x);
   std::lock_guard<std::mutex> g(q.mu);
   if (q.done) return;
   q.status = s;
   q.error = msg;
+  q.failed = true;
   q.done = true;
   q.cv.notify_all();
 }
@@ -848,6 +860,7 @@ static void run_on_host(ddq_db* db, std::shared_ptr<QueryState> q, int i, cudaSt
   }
   q->inters[(size_t)i] = std::move(out);
   q->host_ops++;
+  if (q->trace[(size_t)i] != DDQ_RAN_ABORTED) q->trace[(size_t)i] = DDQ_RAN_HOST;
   db->stats.host_ops++;
   op_finished(db, q, i);
 }
@@ -857,7 +870,7 @@ static void run_on_gpu(ddq_db* db, std::shared_ptr<QueryState> q, int i, cudaStr
   const uint64_t t0 = now_ns();
   ddq_status s = DDQ_OK;
   if (db->cfg.placement == DDQ_PLACE_GPU_ONLY || !db->cfg.chopping) s = ensure_cached_lru(db, op);
-  bool abort = s == DDQ_ENOMEM_DEVICE;
+  bool abort = s == DDQ_ENOMEM_DEVICE || (i < 32 && ((db->cfg.fault_op_mask >> i) & 1u));
   if (s != DDQ_OK && !abort) {
     fail_query(db, *q, s);
     return;
@@ -896,6 +909,18 @@ static void run_on_gpu(ddq_db* db, std::shared_ptr<QueryState> q, int i, cudaStr
       cudaMemcpy(&e2, out.d_error, 4, cudaMemcpyDeviceToHost);
       if (e2) s = set_error(e2 == 2 ? DDQ_EOVERFLOW : DDQ_EINVAL, "hash build failed (duplicate key or overflow)");
     }
+    static const bool dbg = getenv("DDQ_DEBUG_ERRORS") != nullptr;
+    if (dbg && s == DDQ_OK && out.d_error) {
+      uint32_t e2 = 0;
+      cudaMemcpy(&e2, out.d_error, 4, cudaMemcpyDeviceToHost);
+      fprintf(stderr, "ddq: query %lld op %d kind %d error cell %u count %lld\n", (long long)q->id, i, op.kind, e2,
+              (long long)out.count);
+    }
+    if (s == DDQ_OK && op.kind == DDQ_OP_AGGREGATE && out.d_error) {  // group table overflow (max_groups)
+      uint32_t e2 = 0;
+      cudaMemcpy(&e2, out.d_error, 4, cudaMemcpyDeviceToHost);
+      if (e2) s = set_error(DDQ_EOVERFLOW, "aggregate: more groups than the plan's max_groups allows");
+    }
     if (s == DDQ_ENOMEM_DEVICE) {
       abort = true;
       release_inter(db, out);
@@ -906,6 +931,7 @@ static void run_on_gpu(ddq_db* db, std::shared_ptr<QueryState> q, int i, cudaStr
     }
   }
   if (abort) {  // abort immediately, restart on the host
+    q->trace[(size_t)i] = DDQ_RAN_ABORTED;
     q->aborts++;
     db->stats.aborts++;
     db->stats.wasted_ns += now_ns() - t0;
@@ -914,6 +940,7 @@ static void run_on_gpu(ddq_db* db, std::shared_ptr<QueryState> q, int i, cudaStr
   }
   if (op.kind == DDQ_OP_GATHER) out.count = q->inters[(size_t)op.input].count;
   q->inters[(size_t)i] = std::move(out);
+  q->trace[(size_t)i] = DDQ_RAN_GPU;
   q->gpu_ops++;
   db->stats.gpu_ops++;
   op_finished(db, q, i);
@@ -938,9 +965,15 @@ static void worker_loop(ddq_db* db, bool gpu) {
     {
       std::lock_guard<std::mutex> g(q->mu);
       if (q->done) continue;  // failed query: drop remaining ops
+      q->inflight++;
     }
     if (gpu) run_on_gpu(db, q, i, st);
     else run_on_host(db, q, i, st);
+    std::lock_guard<std::mutex> g(q->mu);
+    if (--q->inflight == 0 && q->failed && !q->released) {  // last running op of a failed query
+      q->released = true;
+      for (auto& x : q->inters) release_inter(db, x);
+    }
   }
   cudaStreamDestroy(st);
 }
@@ -986,6 +1019,7 @@ ddq_status ddq_submit(ddq_db* db, const ddq_plan* plan, ddq_query* out) {
   q->parents.assign((size_t)n, {});
   q->consumers_left.assign((size_t)n, 0);
   q->place.assign((size_t)n, P_NONE);
+  q->trace.assign((size_t)n, 0);
   q->ops_left = n;
   q->t_submit = now_ns();
   for (int i = 0; i < n; i++)
@@ -1048,12 +1082,18 @@ ddq_status ddq_fetch(ddq_db* db, ddq_query id, ddq_result** out) {
   }
   std::unique_lock<std::mutex> g(q->mu);
   q->cv.wait(g, [&] { return q->done; });
-  if (q->status != DDQ_OK) return set_error(q->status, q->error);
-  *out = q->result;
+  const ddq_status s = q->status;
+  const std::string err = q->error;
+  *out = s == DDQ_OK ? q->result : nullptr;
   q->result = nullptr;
   g.unlock();
-  std::lock_guard<std::mutex> g2(db->qmu);
-  db->queries.erase(id);
+  {  // a fetched query -- failed or not -- leaves the table (its intermediates are
+     // released by the workers: at the root for a result, at the last in-flight op
+     // of a failed query)
+    std::lock_guard<std::mutex> g2(db->qmu);
+    db->queries.erase(id);
+  }
+  if (s != DDQ_OK) return set_error(s, err);
   return DDQ_OK;
 }
 

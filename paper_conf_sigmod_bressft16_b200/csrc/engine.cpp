@@ -295,7 +295,11 @@ ddq_status run_gpu_op(GpuOpCtx& ctx, const ddq_op& op, Inter& out) {
       fa.d_overflow = ctx.forced_cap >= 0 && in && in->d_error ? in->d_error : nullptr;
       fa.scratch = scratch;
       // error cell propagates down the chain so a prepared plan can detect overflow
-      out.d_error = in ? in->d_error : nullptr;
+      // (its intermediates all live until ddq_prepared_free); in the chopping driver
+      // an op's inputs are released as soon as their consumers are done, so every op
+      // owns its cell there (a shared cell in a freed block was overwritten by a later
+      // allocation: TPC-H Q2 on sparse keys)
+      out.d_error = in && ctx.forced_cap >= 0 ? in->d_error : nullptr;
       if (!out.d_error) {
         out.d_error = (uint32_t*)A.get(64);
         if (A.failed) return DDQ_ENOMEM_DEVICE;
@@ -520,7 +524,7 @@ ddq_status run_gpu_op(GpuOpCtx& ctx, const ddq_op& op, Inter& out) {
       out.gb_keys = (int64_t*)A.get((uint64_t)cap * 8);
       out.gb_accs = (int64_t*)A.get((uint64_t)cap * op.n_aggs * 16);
       out.gb_groups = (uint32_t*)A.get(64);
-      out.d_error = in ? in->d_error : nullptr;
+      out.d_error = in && ctx.forced_cap >= 0 ? in->d_error : nullptr;  // see the probe case
       if (!out.d_error) {
         out.d_error = (uint32_t*)A.get(64);
         if (!A.failed) init_fill(out.d_error, 4, 0, st);
@@ -1170,6 +1174,16 @@ ddq_status cache_column_locked(ddq_db* db, int c, bool on_demand, std::unique_lo
 // Evict (deferred while running operators hold references).  Prepared
 // plans launched asynchronously may still read the column: wait for the device
 // (cudaFree's implicit synchronisation), then return the block to the pool.
+// Drop cache references (one per entry of cols); a column whose eviction was
+// deferred is evicted when its last reference goes.
+void release_column_refs(ddq_db* db, const std::vector<int>& cols) {
+  std::lock_guard<std::mutex> g(db->mu);
+  for (int c : cols) {
+    Column& col = *db->cols[(size_t)c];
+    if (--col.refs == 0 && col.evict_pending) evict_column_locked(db, c);
+  }
+}
+
 void evict_column_locked(ddq_db* db, int c) {
   Column& col = *db->cols[(size_t)c];
   if (!col.dev) return;
@@ -1248,6 +1262,8 @@ ddq_status ddq_update_placement(ddq_db* db) {
   }
   for (size_t c = 0; c < db->cols.size(); c++)  // evict(C_old \ C_new)
     if (!keep[c] && db->cols[c]->dev) evict_column_locked(db, (int)c);
+  for (size_t c = 0; c < db->cols.size(); c++)  // a kept column no longer pending eviction
+    if (keep[c] && db->cols[c]->dev) db->cols[c]->evict_pending = false;
   for (size_t c = 0; c < db->cols.size(); c++)  // cache(C_new \ C_old)
     if (keep[c] && !db->cols[c]->dev) {
       ddq_status s = cache_column_locked(db, (int)c, false, lk);
@@ -1306,6 +1322,7 @@ void ddq_result_free(ddq_result* r) {
   delete[] r->agg_null;
   delete[] r->avgs;
   delete[] r->key_str;
+  delete[] r->op_place;
   delete r;
 }
 
@@ -1314,6 +1331,10 @@ void ddq_result_free(ddq_result* r) {
 // ============================================================ prepared plans
 struct ddq_prepared {
   ddq_db* db = nullptr;
+  // cache references on every column the plan reads: an eviction (explicit,
+  // Algorithm 1 or the GPU-only LRU) is deferred until ddq_prepared_free, so the
+  // graph never reads a freed or reused column block
+  std::vector<int> held;
   ddq_plan plan{};
   std::vector<ddq::Inter> inters;
   std::vector<int64_t> forced;  // per-op output capacity (exact count + slack)
@@ -1546,14 +1567,30 @@ ddq_status ddq_prepare(ddq_db* db, const ddq_plan* plan, int32_t use_graph, ddq_
   P->db = db;
   P->plan = *plan;
   P->use_graph = use_graph != 0;
+  {  // data-driven placement: every input column resident; pin them
+    std::vector<int> cols;
+    for (int i = 0; i < plan->n_ops; i++)
+      for (int c : op_columns(plan->ops[i])) cols.push_back(c);
+    std::lock_guard<std::mutex> g(db->mu);
+    for (int c : cols) {
+      const Column* col = col_of(db, c);
+      if (!col || !col->dev || col->evict_pending)
+        return set_error(DDQ_ESTATE, "prepare: an input column is not cached on the GPU (data-driven placement)");
+    }
+    for (int c : cols) db->cols[(size_t)c]->refs++;
+    P->held = std::move(cols);
+  }
   cudaStream_t st;
-  if (cudaStreamCreateWithFlags(&st, cudaStreamNonBlocking) != cudaSuccess)
+  if (cudaStreamCreateWithFlags(&st, cudaStreamNonBlocking) != cudaSuccess) {
+    release_column_refs(db, P->held);
     return set_error(DDQ_ECUDA, "prepare: stream");
+  }
   P->cap_stream = st;
   auto fail = [&](ddq_status s) {
     free_inters(db, P->inters);
     cudaStreamDestroy(st);
     P->cap_stream = nullptr;
+    release_column_refs(db, P->held);
     return s;
   };
   // 1. calibration run (worst-case capacities) -> exact counts
@@ -1944,6 +1981,7 @@ void ddq_prepared_free(ddq_prepared* p) {
   if (p->exec) cudaGraphExecDestroy(p->exec);
   if (p->graph) cudaGraphDestroy(p->graph);
   free_inters(p->db, p->inters);
+  release_column_refs(p->db, p->held);
   if (p->cap_stream) cudaStreamDestroy(p->cap_stream);
   for (cudaStream_t s2 : p->side) cudaStreamDestroy(s2);
   for (cudaEvent_t e : p->ev) cudaEventDestroy(e);

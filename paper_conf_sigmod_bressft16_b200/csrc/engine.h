@@ -186,5 +186,9 @@ void decode_result_keys(ddq_db* db, const ddq_plan& plan, ddq_result* r);
 int64_t pow2_at_least(int64_t x);
 const ddq::Column* col_of(ddq_db* db, int c);
 bool fits_int32(const ddq::Column& c);
+// columns an operator reads (driver.cpp): placement checks and cache references
+std::vector<int> op_columns(const ddq_op& op);
+void evict_column_locked(ddq_db* db, int c);
+void release_column_refs(ddq_db* db, const std::vector<int>& cols);
 
 }  // namespace ddq

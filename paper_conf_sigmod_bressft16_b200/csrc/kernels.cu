@@ -20,13 +20,12 @@
 namespace ddq {
 
 int num_sms() {
-  static int sms = 0;
-  if (!sms) {
-    int dev = 0;
+  static const int sms = [] {
+    int dev = 0, v = 0;
     cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    if (sms <= 0) sms = 1;
-  }
+    cudaDeviceGetAttribute(&v, cudaDevAttrMultiProcessorCount, dev);
+    return v <= 0 ? 1 : v;
+  }();
   return sms;
 }
 
@@ -778,14 +777,14 @@ cudaError_t launch_groupby(const int32_t* tids, const uint32_t* d_count, int64_t
   if (ucols_ok && coded && total_bits <= 6 && (n_aggs << total_bits) <= GBS_MAX_DA && p.tids != nullptr) {
     const uint32_t D = 1u << total_bits;
     const size_t smem = (size_t)D * n_aggs * (GBS_THREADS * 8 + 16) + 16;
-    static int occs = 0;
-    if (!occs) {
+    static const int occs = [] {  // thread-safe one-time opt-in
+      int o = 0;
       cudaFuncSetAttribute(groupby_small_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
                            GBS_MAX_DA * (GBS_THREADS * 8 + 16) + 16);
-      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occs, groupby_small_kernel, GBS_THREADS,
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, groupby_small_kernel, GBS_THREADS,
                                                     GBS_MAX_DA * (GBS_THREADS * 8 + 16) + 16);
-      if (occs < 1) occs = 1;
-    }
+      return o < 1 ? 1 : o;
+    }();
     const int64_t want = (n_cap + GBS_THREADS * GBS_ROWS - 1) / (GBS_THREADS * GBS_ROWS);
     const int64_t maxb = (int64_t)num_sms() * occs;
     const int grid = (int)(want < 1 ? 1 : (want > maxb ? maxb : want));
@@ -801,12 +800,12 @@ cudaError_t launch_groupby(const int32_t* tids, const uint32_t* d_count, int64_t
   p.s_slots = S;
   p.s_shift = 64 - slg;
   const size_t smem = (size_t)S * (8 + 16 * (size_t)n_aggs);
-  static int occ = 0;
-  if (!occ) {
+  static const int occ = [] {  // thread-safe one-time opt-in
+    int o = 0;
     cudaFuncSetAttribute(groupby_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 160 * 1024);
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, groupby_kernel, GB_THREADS, GB_SMEM_BUDGET);
-    if (occ < 1) occ = 1;
-  }
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, groupby_kernel, GB_THREADS, GB_SMEM_BUDGET);
+    return o < 1 ? 1 : o;
+  }();
   int64_t want = (n_cap + GB_THREADS - 1) / GB_THREADS;
   int64_t maxb = (int64_t)num_sms() * occ;
   int grid = (int)(want < 1 ? 1 : (want > maxb ? maxb : want));

@@ -561,7 +561,7 @@ static void launch_m(int mode, int64_t grid, size_t smem, cudaStream_t st, const
 }
 
 cudaError_t launch_scan(const FilterArgs& a, cudaStream_t st) {
-  if (!g_smem_optin) {
+  static const bool scan_ready = [] {  // thread-safe one-time opt-in
     int dev = 0;
     cudaGetDevice(&dev);
     int v = 0;
@@ -573,7 +573,9 @@ cudaError_t launch_scan(const FilterArgs& a, cudaStream_t st) {
     set_attrs_g<1, true>(v);
     set_attrs_g<2, true>(v);
     g_smem_optin = v;
-  }
+    return true;
+  }();
+  (void)scan_ready;
   const bool tids = a.in_tids != nullptr;
   ScanParams p{};
   p.n = (uint32_t)a.n_cap;

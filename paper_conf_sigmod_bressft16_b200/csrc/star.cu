@@ -327,14 +327,16 @@ static void star_launch_g(int G, int64_t grid, size_t smem, cudaStream_t st, con
 
 cudaError_t launch_star(const ddq_dev_term* terms, int n_terms, int64_t n_rows, int32_t* out_tids,
                         uint32_t* d_out_count, int64_t out_cap, uint32_t* d_overflow, cudaStream_t st) {
-  if (!g_star_optin) {
+  static const bool star_ready = [] {  // thread-safe one-time opt-in
     int dev = 0, v = 0;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&v, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
     star_attrs<4>(v);
     star_attrs<8>(v);
     g_star_optin = v;
-  }
+    return true;
+  }();
+  (void)star_ready;
   StarParams p{};
   p.n = (uint32_t)n_rows;
   p.n_terms = n_terms;

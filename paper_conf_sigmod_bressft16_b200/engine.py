@@ -8,6 +8,7 @@ data-driven placement, query chopping, Algorithm 1 (P:146-15
 from __future__ import annotations
 
 import ctypes
+import weakref
 from dataclasses import dataclass, field
 
 import numpy as np
@@ -25,6 +26,7 @@ class QueryResult:
     tids: np.ndarray | None = None
     avgs: list = field(default_factory=list)
     decoded: list = field(default_factory=list)
+    placement: list = field(default_factory=list)  # per plan op: A.RAN_GPU / RAN_HOST / RAN_ABORTED
     n_keys: int = 0
     n_aggs: int = 0
     gpu_ops: int = 0
@@ -41,6 +43,8 @@ def _convert(res_ptr) -> QueryResult:
         out.tids = np.ctypeslib.as_array(r.tids, shape=(r.n_tids,)).copy() if r.n_tids else \
             np.empty(0, np.int32)
     nk, na = r.n_keys, r.n_aggs
+    if r.op_place:
+        out.placement = [int(r.op_place[i]) for i in range(r.n_ops)]
     for i in range(r.n_rows):
         vals = [int(r.keys[i * nk + k]) for k in range(nk)]
         for a in range(na):
@@ -278,10 +282,12 @@ class Prepared:
 
     def __init__(self, db: "Database", plan: A.Plan, use_graph: bool = True):
         self.db = db
+        self.h = None
         h = ctypes.c_void_p()
         check(lib().ddq_prepare(db.h, ctypes.byref(plan), 1 if use_graph else 0, ctypes.byref(h)))
         self.h = h
         self.kernels = lib().ddq_prepared_kernel_count(h)
+        db._prepared.add(self)
 
     def launch(self, stream: int = 0) -> None:
         check(lib().ddq_prepared_launch(self.h, ctypes.c_void_p(stream)))
@@ -329,9 +335,10 @@ class Prepared:
         return _convert(p)
 
     def close(self) -> None:
-        if self.h:
+        # a prepared plan belongs to its database: freed before it (Database.close)
+        if self.h and self.db.h:
             lib().ddq_prepared_free(self.h)
-            self.h = None
+        self.h = None
 
     def __del__(self):
         try:
@@ -346,7 +353,7 @@ class Database:
     def __init__(self, device: int = 0, cache_bytes: int = 64 << 30, heap_bytes: int = 32 << 30,
                  gpu_workers: int = 4, host_workers: int = 4, placement: int = A.PLACE_DATA_DRIVEN,
                  chopping: bool = True, cache_policy: int = 0, fault_alloc_every: int = 0,
-                 rank: int = 0, world: int = 1, transfer_packing: bool = True):
+                 rank: int = 0, world: int = 1, transfer_packing: bool = True, fault_op_mask: int = 0):
         cfg = A.Config()
         lib().ddq_config_default(ctypes.byref(cfg))
         cfg.device, cfg.rank, cfg.world = device, rank, world
@@ -355,6 +362,7 @@ class Database:
         cfg.placement, cfg.chopping = placement, 1 if chopping else 0
         cfg.cache_policy, cfg.fault_alloc_every = cache_policy, fault_alloc_every
         cfg.transfer_packing = 1 if transfer_packing else 0
+        cfg.fault_op_mask = fault_op_mask
         h = ctypes.c_void_p()
         check(lib().ddq_open(ctypes.byref(cfg), ctypes.byref(h)))
         self.h = h
@@ -363,9 +371,12 @@ class Database:
         self._cols: dict[tuple[str, str], int] = {}
         self.dicts: dict[str, list[str]] = {}
         self._root_aggs: dict = {}
+        self._prepared = weakref.WeakSet()
 
     def close(self) -> None:
         if self.h:
+            for p in list(self._prepared):  # prepared plans hold cache references and heap blocks
+                p.close()
             lib().ddq_close(self.h)
             self.h = None
 
