@@ -160,7 +160,7 @@ ddq_status ddq_op_join_index_probe(const void* index, int32_t key_min, uint32_t 
  * Columns must be 16-byte aligned and readable up to the next 16-byte boundary.
  * *d_out_count uses 2 words (count, CTA counter); overflow of out_cap sets
  * *d_overflow = 4 (if non-NULL). */
-enum { DDQ_TERM_PRED = 1, DDQ_TERM_PROBE = 2 };
+enum { DDQ_TERM_PRED = 1, DDQ_TERM_PROBE = 2, DDQ_TERM_FETCH = 3 /* AGGREGATE terms only, see ddq_op */ };
 typedef struct {
   int32_t kind;          /* DDQ_TERM_PRED | DDQ_TERM_PROBE */
   int32_t width;         /* column width (4 or 8; probes: 4) */
@@ -372,7 +372,14 @@ typedef struct {
   int32_t eq_vec[2];       /* FILTER_EQ: 1 + indexes of the two aligned vectors compared */
   /* STAR (n-ary semi-join over all rows of `table`, evaluated in one pass): term j is
      a predicate (preds[j]) or a probe of fk column term_fk[j] against HASH_BUILD op
-     term_build[j], emitting its payload as the next aligned vector if term_emit[j]. */
+     term_build[j], emitting its payload as the next aligned vector if term_emit[j].
+     AGGREGATE (reading O37, the fused late-materialised tail): terms evaluated at the
+     input TIDs after the fused predicates, in order -- DDQ_TERM_PROBE (a semi-join:
+     rows whose fk misses the build are dropped; payload emitted if term_emit[j]) or
+     DDQ_TERM_FETCH (the build's payload of fk, INT32_MIN on a miss, the row kept, as
+     a GATHER with fetch_build); emitted payloads are appended, in term order, after
+     the input's aligned vectors, so key_src may name them.  GPU: <= 2 aggregates, no
+     MIN, group table <= 2048 slots (the warp-autonomous aggregation), else EINVAL. */
   int32_t n_terms;
   int32_t term_kind[4];    /* DDQ_TERM_PRED | DDQ_TERM_PROBE */
   int32_t term_build[4];

@@ -66,6 +66,21 @@ struct AggParams {
     int64_t in_vals[8];
   } preds[4];
   uint32_t* d_rows;
+  // fused probe / fetch terms (reading O37), evaluated after the predicates
+  int32_t n_terms;
+  struct Term {
+    int32_t kind, emit;
+    const int32_t* fk;
+    const uint32_t* bitmap;
+    const int32_t* payarr;
+    int32_t key_min;
+    uint32_t range;
+    const uint64_t* table;
+    uint32_t cap_mask;
+    int32_t shift;
+    int32_t key_shift;  // the payload is group key bits at this shift (-1: not a key)
+  } terms[4];
+  int32_t key_pay[3];  // key k from payload slot key_pay[k] (>= 0): packed by its term
 };
 
 __device__ __forceinline__ int64_t find_or_insert(long long* keys, uint32_t mask, uint32_t h, long long key) {
@@ -265,11 +280,59 @@ __global__ void __launch_bounds__(AG_NW * 32, 1) agg_ws_kernel(const __grid_cons
       }
       valid &= m;
     }
-    if (P.d_rows) rows += __popc(valid);
+    // fused probe / fetch terms (O37): gather the fk at the live rows, look it up; an
+    // emitted payload that is a group key is packed into the key right away
     long long key[AG_ITEMS];
 #pragma unroll
     for (int j = 0; j < AG_ITEMS; j++) key[j] = 0;
+    for (int t = 0; t < P.n_terms; t++) {
+      const AggParams::Term& T = P.terms[t];
+      int32_t fk[AG_ITEMS];
+#pragma unroll
+      for (int j = 0; j < AG_ITEMS; j++) fk[j] = ((valid >> j) & 1u) ? ldg_gather(T.fk + (uint32_t)tid[j]) : 0;
+      uint32_t hit = 0;
+      int32_t v[AG_ITEMS];
+      if (T.bitmap) {  // join index: the bits first (independent loads), payloads of the hits
+        uint32_t w[AG_ITEMS];
+#pragma unroll
+        for (int j = 0; j < AG_ITEMS; j++) {
+          const uint32_t o = (uint32_t)(fk[j] - T.key_min);
+          w[j] = ((valid >> j) & 1u) && o < T.range ? __ldg(T.bitmap + (o >> 5)) : 0u;
+        }
+#pragma unroll
+        for (int j = 0; j < AG_ITEMS; j++)
+          hit |= ((w[j] >> ((uint32_t)(fk[j] - T.key_min) & 31u)) & 1u) << j;
+        if (T.emit >= 0) {
+#pragma unroll
+          for (int j = 0; j < AG_ITEMS; j++)
+            v[j] = ((hit >> j) & 1u) ? __ldg(T.payarr + (uint32_t)(fk[j] - T.key_min)) : INT32_MIN;
+        }
+      } else {  // open addressing
+#pragma unroll
+        for (int j = 0; j < AG_ITEMS; j++) {
+          v[j] = INT32_MIN;
+          if (!((valid >> j) & 1u)) continue;
+          uint32_t h = ht_hash(fk[j], T.shift);
+          uint64_t sl = __ldg(T.table + h);
+          while (sl != HT_EMPTY && ht_key(sl) != fk[j]) {
+            h = (h + 1) & T.cap_mask;
+            sl = __ldg(T.table + h);
+          }
+          if (sl != HT_EMPTY) {
+            hit |= 1u << j;
+            v[j] = ht_val(sl);
+          }
+        }
+      }
+      if (T.kind == DDQ_TERM_PROBE) valid &= hit;
+      if (T.key_shift >= 0) {
+#pragma unroll
+        for (int j = 0; j < AG_ITEMS; j++) key[j] |= (long long)(uint32_t)v[j] << T.key_shift;
+      }
+    }
+    if (P.d_rows) rows += __popc(valid);
     for (int k = 0; k < P.n_keys; k++) {
+      if (P.key_pay[k] >= 0) continue;  // packed by its term
       int32_t c[AG_ITEMS];
       if (P.key_vec[k]) {
         int4 r[2];
@@ -617,9 +680,31 @@ cudaError_t launch_agg_ws(const int32_t* tids, const uint32_t* d_count, int64_t 
                           const int32_t* const* key_vec, const int32_t* const* key_col, int n_keys,
                           const int32_t* key_bits, const ddq_dev_agg* aggs, int n_aggs, void* table,
                           uint32_t capacity, uint32_t* d_error, cudaStream_t st, const BuildPreds* preds,
-                          uint32_t* d_rows) {
+                          uint32_t* d_rows, const AggTerms* terms) {
   AggParams p{};
   p.d_rows = d_rows;
+  p.key_pay[0] = p.key_pay[1] = p.key_pay[2] = -1;
+  if (terms) {
+    p.n_terms = terms->n;
+    for (int t = 0; t < terms->n && t < 4; t++) {
+      const AggTerm& a = terms->t[t];
+      AggParams::Term& q = p.terms[t];
+      q.kind = a.kind;
+      q.emit = a.emit;
+      q.fk = a.fk;
+      q.bitmap = a.bitmap;
+      q.payarr = a.payarr;
+      q.key_min = a.key_min;
+      q.range = a.range;
+      q.table = a.table;
+      q.cap_mask = a.capacity ? a.capacity - 1 : 0;
+      int lg = 0;
+      while (a.capacity && (1u << lg) < a.capacity) lg++;
+      q.shift = 32 - lg;
+      q.key_shift = -1;
+    }
+    for (int k = 0; k < 3; k++) p.key_pay[k] = terms->key_pay[k];
+  }
   if (preds) {
     p.n_preds = preds->n;
     for (int i = 0; i < preds->n && i < 4; i++) {
@@ -642,6 +727,9 @@ cudaError_t launch_agg_ws(const int32_t* tids, const uint32_t* d_count, int64_t 
     p.key_shift[k] = sh;
     sh += (key_bits && key_bits[k] > 0) ? key_bits[k] : 21;
   }
+  for (int k = 0; k < n_keys && k < 3; k++)  // a term's payload used as key k
+    for (int t = 0; t < p.n_terms; t++)
+      if (p.key_pay[k] >= 0 && p.terms[t].emit == p.key_pay[k]) p.terms[t].key_shift = p.key_shift[k];
   for (int k = 0; k < n_keys; k++) {
     p.key_vec[k] = key_vec ? key_vec[k] : nullptr;
     p.key_col[k] = key_col ? key_col[k] : nullptr;

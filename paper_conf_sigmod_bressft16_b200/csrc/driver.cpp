@@ -79,6 +79,7 @@ std::vector<int> op_columns(const ddq_op& op) {
     case DDQ_OP_GATHER: c.push_back(op.gather_col); break;
     case DDQ_OP_AGGREGATE:
       for (int i = 0; i < op.n_preds; i++) c.push_back(op.preds[i].column);  // fused selection
+      for (int j = 0; j < op.n_terms && j < 4; j++) c.push_back(op.term_fk[j]);  // fused probe terms (O37)
       for (int k = 0; k < op.n_keys; k++)
         if (op.key_src[k] < -1) c.push_back(-2 - op.key_src[k]);
       for (int a = 0; a < op.n_aggs; a++) {
@@ -98,9 +99,10 @@ static std::vector<int> op_children(const ddq_op& op) {
   if (op.kind == DDQ_OP_HASH_PROBE && op.build >= 0 && op.build != op.input) ch.push_back(op.build);
   if (op.kind == DDQ_OP_GATHER && op.fetch_build > 0 && op.fetch_build - 1 != op.input)
     ch.push_back(op.fetch_build - 1);
-  if (op.kind == DDQ_OP_STAR)
+  if (op.kind == DDQ_OP_STAR || op.kind == DDQ_OP_AGGREGATE)
     for (int j = 0; j < op.n_terms && j < 4; j++)
-      if (op.term_kind[j] == DDQ_TERM_PROBE && std::find(ch.begin(), ch.end(), op.term_build[j]) == ch.end())
+      if ((op.term_kind[j] == DDQ_TERM_PROBE || op.term_kind[j] == DDQ_TERM_FETCH) &&
+          std::find(ch.begin(), ch.end(), op.term_build[j]) == ch.end())
         ch.push_back(op.term_build[j]);
   return ch;
 }
@@ -287,6 +289,30 @@ static inline bool host_pred(const ddq_pred& pr, int64_t v) {
   bool m = false;
   for (int j = 0; j < pr.n_in && j < DDQ_MAX_IN; j++) m |= v == pr.in_vals[j];
   return m;
+}
+
+// Look key k up in a host-resident build (hash table or join index copy).
+static bool host_lookup(const Inter& B, int32_t k, int32_t* v) {
+  if (B.h_bitmap) {
+    const uint32_t o = (uint32_t)(k - B.jmin);
+    if (o < B.jrange && (((*B.h_bitmap)[o >> 5] >> (o & 31)) & 1u)) {
+      *v = (*B.h_payarr)[o];
+      return true;
+    }
+    return false;
+  }
+  int lg = 0;
+  while ((1u << lg) < B.table_cap) lg++;
+  uint32_t h = ((uint32_t)k * 0x9E3779B1u) >> (32 - lg);
+  while (true) {
+    const uint64_t sl = (*B.host_table)[h];
+    if (sl == 0x8000000000000000ull) return false;
+    if ((int32_t)(sl >> 32) == k) {
+      *v = (int32_t)(uint32_t)sl;
+      return true;
+    }
+    h = (h + 1) & (B.table_cap - 1);
+  }
 }
 
 static inline int64_t hcol(const Column* c, int64_t r) {
@@ -583,6 +609,16 @@ ddq_status run_host_op(ddq_db* db, const ddq_op& op, const std::vector<Inter>& I
         kshift[k] = sh;
         sh += op.key_bits[k] > 0 ? op.key_bits[k] : 21;
       }
+      // fused probe / fetch terms (reading O37): builds on the host, emitted payloads
+      // numbered after the input's vectors
+      std::vector<const Inter*> tb;
+      std::vector<const Column*> tfk;
+      for (int j = 0; j < op.n_terms && j < 4; j++) {
+        tb.push_back(&I[(size_t)op.term_build[j]]);
+        tfk.push_back(col_of(db, op.term_fk[j]));
+        if (!tb.back()->host_table && !tb.back()->h_bitmap) return set_error(DDQ_ESTATE, "host aggregate: term build not on the host");
+      }
+      const int n_in_vecs = in ? (int)in->vecs.size() : 0;
       std::unordered_map<int64_t, std::vector<__int128>> g;
       std::vector<const Column*> apc;  // fused selection (AGGREGATE op with predicates)
       for (int p = 0; p < op.n_preds; p++) apc.push_back(col_of(db, op.preds[p].column));
@@ -595,10 +631,21 @@ ddq_status run_host_op(ddq_db* db, const ddq_op& op, const std::vector<Inter>& I
           ok = host_pred(pr, v);
         }
         if (!ok) continue;
+        int32_t tpay[4];
+        int ne = 0;
+        for (size_t j = 0; j < tb.size() && ok; j++) {
+          int32_t v = INT32_MIN;
+          const bool hit = host_lookup(*tb[j], ((const int32_t*)tfk[j]->host)[r], &v);
+          if (op.term_kind[j] == DDQ_TERM_PROBE && !hit) ok = false;
+          if (op.term_kind[j] == DDQ_TERM_FETCH || op.term_emit[j]) tpay[ne++] = v;
+        }
+        if (!ok) continue;
         int64_t key = 0;
         for (int k = 0; k < op.n_keys; k++) {
-          int32_t c = op.key_src[k] >= 0 ? ((const int32_t*)in->vecs[(size_t)op.key_src[k]].ptr)[i]
-                                         : ((const int32_t*)kc[(size_t)k]->host)[r];
+          const int src = op.key_src[k];
+          int32_t c = src >= n_in_vecs && !tb.empty() ? tpay[src - n_in_vecs]
+                      : src >= 0 ? ((const int32_t*)in->vecs[(size_t)src].ptr)[i]
+                                 : ((const int32_t*)kc[(size_t)k]->host)[r];
           key |= (int64_t)(uint32_t)c << kshift[k];
         }
         auto& acc = g[key];

@@ -109,6 +109,14 @@ bool use_join_index(const Column& kc, int64_t n_rows) {
   return r <= (1ll << 28) && (r <= (1ll << 20) || r <= 16 * std::max<int64_t>(n_rows, 1));
 }
 
+// Input rows up to which an AGGREGATE evaluates its probe terms row by row (reading
+// O37); about two waves of the warp-autonomous aggregation (148 SMs x 16 warps x
+// 256-row tiles x 2 = 1.2 M rows on B200).  Longer inputs evaluate them term by term.
+int64_t fused_tail_max_rows() {
+  if (const char* e = getenv("DDQ_FUSED_TAIL_MAX")) return (int64_t)strtoll(e, nullptr, 10);  // tests / A-B
+  return (int64_t)num_sms() * 16 * 256 * 2;
+}
+
 // An int64 column whose load-time range fits int32 (exact narrowing) or an int32 column.
 bool fits_int32(const Column& c) {
   return c.width == 4 || c.n == 0 || (c.vmin >= INT32_MIN && c.vmax <= INT32_MAX);
@@ -475,8 +483,50 @@ ddq_status run_gpu_op(GpuOpCtx& ctx, const ddq_op& op, Inter& out) {
         return set_error(DDQ_EINVAL, "aggregate: bad key/agg counts");
       const int32_t* kv[3] = {nullptr, nullptr, nullptr};
       const int32_t* kc[3] = {nullptr, nullptr, nullptr};
+      // fused probe / fetch terms (reading O37): their emitted payloads follow the
+      // input's vectors; a key naming one reads payload slot key_pay
+      AggTerms terms;
+      const int n_in_vecs = in ? (int)in->vecs.size() : 0;
+      if (op.n_terms > 0) {
+        if (!in) return set_error(DDQ_EINVAL, "aggregate: terms need an input TID list");
+        terms.n = op.n_terms;
+        int slot = 0;
+        for (int j = 0; j < op.n_terms; j++) {
+          const int b = op.term_build[j];
+          if (b < 0 || b >= (int)I.size()) return set_error(DDQ_EINVAL, "aggregate: bad term build");
+          const Inter& B = I[(size_t)b];
+          if (!B.table_ptr && !B.jidx) return set_error(DDQ_ESTATE, "aggregate: term build is not on the device");
+          const Column* c = col_of(db, op.term_fk[j]);
+          if (!c || c->table != op.table || c->width != 4) return set_error(DDQ_EINVAL, "aggregate: bad term fk column");
+          AggTerm& t = terms.t[j];
+          t.kind = op.term_kind[j];
+          t.fk = (const int32_t*)need_col(op.term_fk[j]);
+          if (!t.fk) return set_error(DDQ_ESTATE, "aggregate: term fk column not cached on the GPU");
+          const bool emits = op.term_kind[j] == DDQ_TERM_FETCH || op.term_emit[j];
+          if (emits && slot >= 3) return set_error(DDQ_EINVAL, "aggregate: at most 3 emitting terms");
+          t.emit = emits ? slot++ : -1;
+          if (B.jidx) {
+            t.bitmap = join_index_bitmap(B.jidx);
+            t.payarr = join_index_payload(B.jidx, B.jrange);
+            t.key_min = B.jmin;
+            t.range = B.jrange;
+          } else {
+            t.table = B.table_ptr;
+            t.capacity = B.table_cap;
+          }
+        }
+      }
       for (int k = 0; k < op.n_keys; k++) {
         int src = op.key_src[k];
+        if (src >= n_in_vecs && op.n_terms > 0) {  // an emitted payload of a term
+          int e = src - n_in_vecs, slot = -1;
+          for (int j = 0; j < op.n_terms; j++)
+            if (terms.t[j].emit >= 0 && e-- == 0) slot = terms.t[j].emit;
+          if (slot < 0) return set_error(DDQ_EINVAL, "aggregate: key names a term that emits nothing");
+          terms.key_pay[k] = slot;
+          kv[k] = nullptr;
+          continue;
+        }
         if (src >= 0) {
           if (!in || src >= (int)in->vecs.size() || in->vecs[(size_t)src].width != 4)
             return set_error(DDQ_EINVAL, "aggregate: bad key vector");
@@ -549,6 +599,97 @@ ddq_status run_gpu_op(GpuOpCtx& ctx, const ddq_op& op, Inter& out) {
         d.hi = p.hi;
         d.n_in = p.n_in;
         for (int j = 0; j < DDQ_MAX_IN; j++) d.in_vals[j] = p.in_vals[j];
+      }
+      if (op.n_terms > 0) {  // the fused tail (O37): the warp-autonomous aggregation only
+        bool aligned = ((uintptr_t)in->tids & 15) == 0;
+        for (int k = 0; k < op.n_keys; k++) aligned = aligned && (!kv[k] || ((uintptr_t)kv[k] & 15) == 0);
+        if (has_min || op.n_aggs > 2 || out.gb_cap > 2048 || !aligned || !in->d_count)
+          return set_error(DDQ_EINVAL, "aggregate: fused terms need <= 2 SUM/COUNT aggregates and <= 1024 groups");
+        const int32_t* a_tids = in->tids;
+        const uint32_t* a_count = in->d_count;
+        const AggTerms* a_terms = &terms;
+        if (in_cap > fused_tail_max_rows()) {
+          // A long input: row-by-row terms would pay every term's gather latency for
+          // every input tile while most rows are already dead.  The same operator
+          // then evaluates its terms as the chain does -- one compacting probe (or
+          // fetch) pass per term, survivors and payloads materialised -- and
+          // aggregates the final rows (a physical algorithm choice).
+          std::vector<const int32_t*> cv;
+          for (const Vec& v : in->vecs) {
+            if (v.width != 4) return set_error(DDQ_EINVAL, "aggregate: only int32 vectors can be carried");
+            cv.push_back((const int32_t*)v.ptr);
+          }
+          const int64_t cap = in_cap;
+          for (int j = 0; j < op.n_terms; j++) {
+            const AggTerm& t = terms.t[j];
+            if (t.kind == DDQ_TERM_FETCH) {
+              int32_t* dst = (int32_t*)A.get((uint64_t)std::max<int64_t>(cap, 1) * 4);
+              if (A.failed) return DDQ_ENOMEM_DEVICE;
+              cudaError_t e0 = launch_fetch(a_tids, a_count, cap, t.fk, t.bitmap, t.payarr, t.key_min, t.range, t.table,
+                                            t.capacity, dst, st);
+              if (e0 != cudaSuccess) return cuda_status(e0, "aggregate: term fetch");
+              cv.push_back(dst);
+              continue;
+            }
+            if (cv.size() > DDQ_MAX_CARRY) return set_error(DDQ_EINVAL, "aggregate: too many aligned vectors");
+            std::vector<int32_t*> co;
+            int32_t* nt = (int32_t*)A.get((uint64_t)std::max<int64_t>(cap, 1) * 4);
+            uint32_t* nc = (uint32_t*)A.get(64);
+            for (size_t c = 0; c < cv.size(); c++) co.push_back((int32_t*)A.get((uint64_t)std::max<int64_t>(cap, 1) * 4));
+            int32_t* pay = t.emit >= 0 ? (int32_t*)A.get((uint64_t)std::max<int64_t>(cap, 1) * 4) : nullptr;
+            void* scr = A.get(filter_scratch_bytes(cap));
+            if (A.failed) return DDQ_ENOMEM_DEVICE;
+            FilterArgs fa;
+            fa.probe = true;
+            fa.table = t.table;
+            fa.capacity = t.capacity;
+            if (t.bitmap) {
+              const Inter& B = I[(size_t)op.term_build[j]];
+              fa.bitmap = t.bitmap;
+              fa.payarr = t.payarr;
+              fa.coarse = join_index_coarse(B.jidx, B.jrange);
+              fa.key_min = t.key_min;
+              fa.range = t.range;
+            }
+            fa.fk = t.fk;
+            fa.out_payload = pay;
+            fa.in_tids = a_tids;
+            fa.d_in_count = a_count;
+            fa.n_cap = cap;
+            fa.carry_in = cv.data();
+            fa.carry_out = co.data();
+            fa.n_carry = (int)cv.size();
+            fa.out_tids = nt;
+            fa.d_out_count = nc;
+            fa.out_cap = cap;
+            fa.d_overflow = out.d_error;
+            fa.scratch = scr;
+            cudaError_t e0 = launch_filter(fa, st);
+            if (e0 != cudaSuccess) return cuda_status(e0, "aggregate: term probe");
+            a_tids = nt;
+            a_count = nc;
+            cv.assign(co.begin(), co.end());
+            if (pay) cv.push_back(pay);
+          }
+          for (int k = 0; k < op.n_keys; k++) {  // keys: every vector is materialised now
+            const int src = op.key_src[k];
+            if (src >= 0) {
+              if (src >= (int)cv.size()) return set_error(DDQ_EINVAL, "aggregate: bad key vector");
+              kv[k] = cv[(size_t)src];
+            }
+          }
+          a_terms = nullptr;
+        }
+        out.d_rows = (uint32_t*)A.get(64);
+        if (A.failed) return DDQ_ENOMEM_DEVICE;
+        init_fill(out.d_rows, 4, 0, st);
+        cudaError_t e = launch_groupby_init(out.gb_table, out.gb_cap, op.n_aggs, st);
+        if (e == cudaSuccess)
+          e = launch_agg_ws(a_tids, a_count, in_cap, kv, kc, op.n_keys, op.key_bits, ag, op.n_aggs, out.gb_table,
+                            out.gb_cap, out.d_error, st, &bp, out.d_rows, a_terms);
+        if (e == cudaSuccess)
+          e = launch_groupby_compact(out.gb_table, out.gb_cap, op.n_aggs, out.gb_keys, out.gb_accs, out.gb_groups, st);
+        return cuda_status(e, "aggregate (fused terms)");
       }
       if (!in && !has_min && agg_dense_supported(in_cap, &bp, kc, op.n_keys, op.key_bits, ag, op.n_aggs)) {
         out.d_rows = (uint32_t*)A.get(64);
@@ -806,7 +947,16 @@ void decode_result_keys(ddq_db* db, const ddq_plan& plan, ddq_result* r) {
     std::lock_guard<std::mutex> g(db->mu);
     for (int k = 0; k < r->n_keys && k < DDQ_MAX_KEYS; k++) {
       const int src = root.key_src[k];
-      const int c = src < -1 ? -2 - src : src >= 0 ? vec_column(plan, root.input, src) : -1;
+      const int nv = vec_count(plan, root.input);
+      int c = src < -1 ? -2 - src : src >= 0 && src < nv ? vec_column(plan, root.input, src) : -1;
+      if (src >= nv && root.n_terms > 0) {  // a fused term's emitted payload (O37)
+        int e = src - nv;
+        for (int j = 0; j < root.n_terms && j < 4; j++)
+          if ((root.term_kind[j] == DDQ_TERM_FETCH || root.term_emit[j]) && e-- == 0) {
+            const int b = root.term_build[j];
+            c = b >= 0 && b < plan.n_ops ? plan.ops[b].payload_col : -1;
+          }
+      }
       if (c >= 0 && c < (int)db->cols.size() && !db->cols[(size_t)c]->dict.empty()) {
         dict[k] = &db->cols[(size_t)c]->dict;  // set once before queries, never reallocated
         any = true;
@@ -1365,6 +1515,14 @@ static ddq_status validate_plan(ddq_db* db, const ddq_plan* plan) {
             (op.term_build[j] < 0 || op.term_build[j] >= i || plan->ops[op.term_build[j]].kind != DDQ_OP_HASH_BUILD))
           return set_error(DDQ_EINVAL, "plan: STAR probe must reference an earlier HASH_BUILD");
     }
+    if (op.kind == DDQ_OP_AGGREGATE && op.n_terms != 0) {  // fused probe / fetch terms (O37)
+      if (op.input < 0) return set_error(DDQ_EINVAL, "plan: aggregate terms need an input TID list");
+      if (op.n_terms < 0 || op.n_terms > 4) return set_error(DDQ_EINVAL, "plan: aggregate needs 0..4 terms");
+      for (int j = 0; j < op.n_terms; j++)
+        if ((op.term_kind[j] != DDQ_TERM_PROBE && op.term_kind[j] != DDQ_TERM_FETCH) || op.term_build[j] < 0 ||
+            op.term_build[j] >= i || plan->ops[op.term_build[j]].kind != DDQ_OP_HASH_BUILD)
+          return set_error(DDQ_EINVAL, "plan: an aggregate term probes / fetches an earlier HASH_BUILD");
+    }
     if (op.kind == DDQ_OP_FILTER_EQ && op.input < 0) return set_error(DDQ_EINVAL, "plan: filter_eq needs an input");
     if (op.fetch_build != 0 && (op.kind != DDQ_OP_GATHER || op.fetch_build - 1 < 0 || op.fetch_build - 1 >= i ||
                                 plan->ops[op.fetch_build - 1].kind != DDQ_OP_HASH_BUILD))
@@ -1455,9 +1613,9 @@ static std::vector<int> op_deps(const ddq_op& op, int i) {
   add(op.input);
   if (op.kind == DDQ_OP_HASH_PROBE) add(op.build);
   if (op.kind == DDQ_OP_GATHER && op.fetch_build > 0) add(op.fetch_build - 1);
-  if (op.kind == DDQ_OP_STAR)
+  if (op.kind == DDQ_OP_STAR || op.kind == DDQ_OP_AGGREGATE)
     for (int j = 0; j < op.n_terms && j < 4; j++)
-      if (op.term_kind[j] == DDQ_TERM_PROBE) add(op.term_build[j]);
+      if (op.term_kind[j] == DDQ_TERM_PROBE || op.term_kind[j] == DDQ_TERM_FETCH) add(op.term_build[j]);
   return d;
 }
 
@@ -1540,6 +1698,7 @@ void count_accesses(ddq_db* db, const ddq_op& op) {
       break;
     case DDQ_OP_AGGREGATE:
       for (int i = 0; i < op.n_preds; i++) touch(op.preds[i].column);  // fused selection
+      for (int j = 0; j < op.n_terms && j < 4; j++) touch(op.term_fk[j]);  // fused probe terms
       for (int k = 0; k < op.n_keys; k++)
         if (op.key_src[k] < -1) touch(-2 - op.key_src[k]);
       for (int a = 0; a < op.n_aggs; a++) {
@@ -1827,11 +1986,15 @@ int32_t ddq_prepared_profile(ddq_prepared* p, void* stream, int32_t max_ops, flo
         // fused selection: first predicate column at every input TID, the rest
         // and everything below at the rows that passed (d_rows)
         double mr = m;
-        if (op.n_preds > 0 && o.d_rows) {
+        if ((op.n_preds > 0 || op.n_terms > 0) && o.d_rows) {
           uint32_t r = 0;
           cudaMemcpy(&r, o.d_rows, 4, cudaMemcpyDeviceToHost);
           mr = r;
           for (int k = 0; k < op.n_preds; k++) bytes += sector_bytes(N, k == 0 ? m : mr, width(op.preds[k].column));
+          // fused probe / fetch terms (O37): the first term's fk at every input row that
+          // passed the predicates, later ones at least at the final rows (a lower bound)
+          for (int j = 0; j < op.n_terms && j < 4; j++)
+            bytes += sector_bytes(N, j == 0 && op.n_preds == 0 ? m : mr, 4);
         }
         for (int k = 0; k < op.n_keys; k++) bytes += op.key_src[k] >= 0 ? m * 4 : sector_bytes(N, mr, 4);
         std::vector<int> seen;

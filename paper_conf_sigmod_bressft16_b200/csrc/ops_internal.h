@@ -165,13 +165,35 @@ cudaError_t launch_agg_dense(int64_t n_rows, const int32_t* const* key_col, int 
                              const ddq_dev_agg* aggs, int n_aggs, void* table, uint32_t capacity, uint32_t* d_error,
                              cudaStream_t st, const struct BuildPreds* preds, uint32_t* d_rows);
 cudaError_t launch_iota(int32_t* out, int64_t n, uint32_t* d_count, cudaStream_t st);
+// A probe / fetch term fused into the aggregation at TIDs (reading O37):
+// the fk column is gathered at the row, looked up in a join index (bitmap +
+// payload array) or an open-addressing hash table; a PROBE drops rows whose key
+// misses, a FETCH keeps them with payload INT32_MIN; `emit` >= 0 stores the payload
+// in slot `emit` (0..2) for use as a group key (AggKeys::pay).
+struct AggTerm {
+  int32_t kind = 0;  // DDQ_TERM_PROBE | DDQ_TERM_FETCH
+  int32_t emit = -1;
+  const int32_t* fk = nullptr;
+  const uint32_t* bitmap = nullptr;  // join index (or null: hash table)
+  const int32_t* payarr = nullptr;
+  int32_t key_min = 0;
+  uint32_t range = 0;
+  const uint64_t* table = nullptr;
+  uint32_t capacity = 0;
+};
+struct AggTerms {
+  int32_t n = 0;
+  AggTerm t[4];
+  int32_t key_pay[3] = {-1, -1, -1};  // key k = payload slot key_pay[k] (>= 0) instead of a vector / column
+};
 bool agg_ws_supported(const int32_t* tids, const int32_t* const* key_vec, int n_keys, int n_aggs,
                       uint32_t capacity);
 cudaError_t launch_agg_ws(const int32_t* tids, const uint32_t* d_count, int64_t n_cap,
                           const int32_t* const* key_vec, const int32_t* const* key_col, int n_keys,
                           const int32_t* key_bits, const ddq_dev_agg* aggs, int n_aggs, void* table,
                           uint32_t capacity, uint32_t* d_error, cudaStream_t st,
-                          const BuildPreds* preds = nullptr, uint32_t* d_rows = nullptr);
+                          const BuildPreds* preds = nullptr, uint32_t* d_rows = nullptr,
+                          const AggTerms* terms = nullptr);
 cudaError_t launch_groupby_compact(const void* table, uint32_t capacity, int n_aggs, int64_t* out_keys,
                                    int64_t* out_accs, uint32_t* d_out_groups, cudaStream_t st);
 

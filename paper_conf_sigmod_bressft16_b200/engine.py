@@ -204,15 +204,28 @@ class PlanBuilder:
 
     def aggregate(self, table: str, input: int, keys: list, aggs: list, order_by: list | None = None,
                   max_groups: int = 0, limit: int = 0, key_bits: list | None = None,
-                  where: list | None = None, avg: list | None = None, avg_count: int = -1) -> int:
+                  where: list | None = None, avg: list | None = None, avg_count: int = -1,
+                  terms: list | None = None) -> int:
         """keys: int (aligned vector index) or str (column of `table`).
         aggs: (kind, [cols]).  order_by: ints per include/ddq.h (+/-(1+k), +/-(101+a)).
         key_bits: bits per key in the packed group key (default 21 each, sum <= 63).
         where: predicates on the input rows evaluated inside the aggregation (a fused
-        selection, reading O26), same forms as select()."""
+        selection, reading O26), same forms as select().
+        terms: fused probe / fetch terms evaluated at the input rows after `where`
+        (reading O37): ("probe", fk_col, build_op, emit) | ("fetch", fk_col, build_op);
+        emitted payloads are numbered after the input's aligned vectors."""
         idx, op = self._op(A.OP_AGGREGATE, table, input)
         if where:
             self._preds(op, table, where)
+        terms = terms or []
+        if len(terms) > 4:
+            raise ValueError("at most 4 aggregate terms")
+        op.n_terms = len(terms)
+        for j, t in enumerate(terms):
+            op.term_kind[j] = A.TERM_FETCH if t[0] == "fetch" else A.TERM_PROBE
+            op.term_fk[j] = self.db.col(table, t[1])
+            op.term_build[j] = t[2]
+            op.term_emit[j] = 1 if (t[0] == "fetch" or t[3]) else 0
         for k, b in enumerate(key_bits or []):
             op.key_bits[k] = b
         op.n_keys = len(keys)

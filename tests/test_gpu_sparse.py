@@ -19,7 +19,7 @@ import oracle
 
 pytestmark = pytest.mark.gpu
 
-VARIANTS = {"chain": dict(star=False), "star": dict(star=True), "chain_eager": dict(star=False, late=False),
+VARIANTS = {"chain": dict(star=False), "chain_fused": dict(star=False, fuse_tail=True), "star": dict(star=True), "chain_eager": dict(star=False, late=False),
             "chain_unfused": dict(star=False, fused_build=False, late=False, fused_agg=False)}
 TPCH = ["tpch1", "tpch2", "tpch3", "tpch4", "tpch5", "tpch6", "tpch7"]
 

@@ -49,7 +49,7 @@ def _oracle(kind, q):
     return norm(q, oracle.run(_data(kind), q))
 
 
-VARIANTS = {"star": dict(star=True), "chain": dict(star=False),
+VARIANTS = {"star": dict(star=True), "chain": dict(star=False), "chain_fused": dict(star=False, fuse_tail=True),
             "chain_eager": dict(star=False, late=False),
             "chain_unfused": dict(star=False, fused_build=False, late=False, fused_agg=False)}
 
@@ -199,3 +199,21 @@ def test_o30_supplier_first_orders_equal_oracle(monkeypatch):
                 p.close()
                 assert norm(q, got) == _oracle(kind, q), (kind, q, variant)
             assert norm(q, db.run(S.ssb_plan(db, q)).rows) == _oracle(kind, q), (kind, q)
+
+
+@pytest.mark.parametrize("mode", ["row_by_row", "term_by_term"])
+def test_fused_tail_both_algorithms(mode, monkeypatch):
+    """Reading O37: an AGGREGATE carrying probe / fetch terms evaluates them row by row
+    inside the aggregation (short inputs) or term by term with compaction (long
+    inputs); DDQ_FUSED_TAIL_MAX forces either.  Both equal the oracle, prepared and
+    through the chopping driver, on SF1 and the planted database."""
+    from paper_conf_sigmod_bressft16_b200.ssb import ssb_plan
+    monkeypatch.setenv("DDQ_FUSED_TAIL_MAX", "1000000000" if mode == "row_by_row" else "0")
+    for kind in ("1", "planted"):
+        db = _db(kind)
+        for q in oracle.SSB_QUERIES:
+            p = db.prepare(ssb_plan(db, q, fuse_tail=True))
+            p.launch()
+            assert p.fetch().rows == _oracle(kind, q), (kind, q)
+            p.close()
+            assert db.run(ssb_plan(db, q, fuse_tail=True)).rows == _oracle(kind, q), (kind, q)
