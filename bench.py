@@ -124,9 +124,48 @@ def dist_env():
     return ws, rank, local
 
 
-def cpu_baseline(sf: float, sample_rows: int) -> dict:
+def host_facts() -> dict:
+    """The host the CPU baseline runs on: online cores, CPU model, memory (S8(d))."""
+    facts = {"nproc": os.cpu_count()}
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                facts["cpu"] = line.split(":", 1)[1].strip()
+                break
+        for line in open("/proc/meminfo"):
+            if line.startswith("MemTotal:"):
+                facts["mem_gib"] = round(int(line.split()[1]) / (1 << 20), 1)
+                break
+    except OSError:
+        pass
+    return facts
+
+
+class pinned_core:
+    """Pin this process to one core (taskset -c 0 equivalent) while the
+    single-threaded oracle is timed; the previous affinity is restored after."""
+
+    def __init__(self, core: int = 0):
+        self.core = core
+        self.old = None
+
+    def __enter__(self):
+        try:
+            self.old = os.sched_getaffinity(0)
+            os.sched_setaffinity(0, {self.core if self.core in self.old else min(self.old)})
+        except (AttributeError, OSError):
+            self.old = None
+        return self
+
+    def __exit__(self, *exc):
+        if self.old is not None:
+            os.sched_setaffinity(0, self.old)
+
+
+def cpu_baseline(sf: float, sample_rows: int, repeats: int = 3) -> dict:
     """The oracle as it stands (single-threaded C++), on the first `sample_rows`
-    lineorder rows of the same SF database, all 13 queries."""
+    lineorder rows of the same SF database, all 13 queries; pinned to one core, the
+    median of `repeats` runs (S8(d) oracle timing)."""
     import datagen
     import oracle
     data = datagen.SSB(sf)
@@ -148,13 +187,19 @@ def cpu_baseline(sf: float, sample_rows: int) -> dict:
     for q in oracle.SSB_QUERIES:  # generate inputs outside the timed region
         for c in oracle.SSB_QUERY_COLUMNS[int(q[3])]:
             v[c]
-    t0 = time.perf_counter()
-    for q in oracle.SSB_QUERIES:
-        oracle.run(v, q)
-    dt = time.perf_counter() - t0
+    runs = []
+    with pinned_core(0):
+        for _ in range(repeats):
+            t0 = time.perf_counter()
+            for q in oracle.SSB_QUERIES:
+                oracle.run(v, q)
+            runs.append(time.perf_counter() - t0)
+    dt = sorted(runs)[len(runs) // 2]
     return {"value": 13 * sample_rows / dt, "unit": UNIT, "cores": 1, "kind": "oracle",
             "sample": f"all 13 SSB queries over the first {sample_rows} lineorder rows of SF{sf:g} "
-                      f"(full dimension tables), single-threaded, {dt:.2f} s"}
+                      f"(full dimension tables), single-threaded, pinned to core 0, median of {repeats} runs "
+                      f"({', '.join(f'{x:.2f}' for x in runs)} s)",
+            "host": host_facts()}
 
 
 def run_reference(args):
@@ -166,10 +211,10 @@ def run_reference(args):
     sf = args.sf * max(args.gpus, ws, 1)  # our arm's workload at N GPUs: SF 20 x N (weak scaling)
     vals = []
     for _ in range(args.warmup):
-        cpu_baseline(sf, sample)
+        cpu_baseline(sf, sample, repeats=1)
     t_total = 0.0
     for _ in range(args.steps):
-        r = cpu_baseline(sf, sample)
+        r = cpu_baseline(sf, sample, repeats=1)
         vals.append(r["value"])
         t_total += 13 * sample / r["value"]
     value = 13 * sample * args.steps / t_total
@@ -180,7 +225,8 @@ def run_reference(args):
             "config": {"workload": f"SSB SF{sf:g}, all 13 queries (bounded sample: first {sample} lineorder "
                                    f"rows per step)", "queries": 13},
             "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle",
-                             "sample": f"first {sample} lineorder rows of SF{sf:g} per step"},
+                             "sample": f"first {sample} lineorder rows of SF{sf:g} per step, pinned to core 0",
+                             "host": host_facts()},
             "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
 
@@ -195,6 +241,7 @@ def main():
     from paper_conf_sigmod_bressft16_b200 import Database
     from paper_conf_sigmod_bressft16_b200 import _abi as A
     from paper_conf_sigmod_bressft16_b200.ssb import SSB_QUERIES, load_ssb, ssb_plan, QUERY_COLUMNS
+    QUERY_COLUMNS_ALL = sorted(set(sum(QUERY_COLUMNS.values(), [])))
 
     ws, rank, local = dist_env()
     assert ws == args.gpus or ws == 1, "launch N>1 with torchrun --nproc-per-node N"
@@ -361,6 +408,8 @@ def main():
         ms = float(t.item())
         dist.barrier()
     ms_per_step = ms / args.steps
+    fact_gb = sum(shard[c].nbytes for c in QUERY_COLUMNS_ALL) / 1e9
+    l2_mb = torch.cuda.get_device_properties(local).L2_cache_size / 2**20
     total_rows = 13 * n_lo * ws // dws  # all ranks together (emulation: this shard only)
     value = total_rows * args.steps / (ms / 1e3)
     # the same K steps with the 13 plans back to back on one stream (per-query latency view)
@@ -470,7 +519,8 @@ def main():
                            "query_streams": max(args.streams, 1),
                            "serial_ms_per_step": round(serial_ms / args.steps, 4) if serial_ms else None,
                            "serial_value": total_rows * args.steps / (serial_ms / 1e3) if serial_ms else None,
-                           "l2": "inputs (6.7 GB/GPU) larger than L2; no flush"},
+                           "l2": f"inputs ({fact_gb:.1f} GB of lineorder columns per GPU) larger than L2 "
+                                 f"({l2_mb:.0f} MB); no flush"},
                 "queries_per_s": 13 * args.steps / (ms / 1e3),
                 "gpu_launches": kernels_per_step * args.steps,
                 "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks,

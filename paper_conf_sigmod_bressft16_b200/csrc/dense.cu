@@ -496,6 +496,13 @@ __global__ void __launch_bounds__(ws_nw(kIn == 1) * 32, 1) ws_kernel(const __gri
       __threadfence_block();
     }
     flush = __shfl_sync(FULL, flush, 0);
+    // ring hand-off between warps is flag-synchronised, not barrier-synchronised:
+    // writers fence (CTA) before their s_filled atomics, the flushing warp's lane 0
+    // fences after its atomic, and this warp barrier orders that for all its lanes
+    // before they read the block; the block is recycled through s_gen the same way.
+    // (compute-sanitizer racecheck models only barriers and reports these hand-offs,
+    // profiles/r2_sanitize_summary.txt)
+    __syncwarp();
     while (flush) {
       const uint32_t b = (flush & 1u) ? pos0 / BLK : (pos0 + tot - 1) / BLK;
       flush &= flush - 1;
