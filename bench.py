@@ -9,10 +9,13 @@ value = 13 * lineorder_rows * steps / device time (CUDA events), max over ranks.
 Inputs (6.7 GB of lineorder columns) are larger than L2 (126 MB), so no L2 flush
 is needed between steps.
 
-N > 1 (torchrun): lineorder of SF 20*N is range-sharded by row (P:407 horizontal
-partitioning), each rank holding 120M rows (weak scaling); per step every rank runs
-the 13 plans on its shard and the partial group tables are exchanged with one NCCL
-all_gather per query; rank 0 merges them (host finalisation, S8(a7)).
+N > 1 (torchrun): lineorder is range-sharded by row (P:407 horizontal partitioning):
+weak scaling by default (SF 20*N, 120 M rows per rank), strong scaling with
+--sf-total 100 (S8(d) M3: 600 M rows split over the ranks).  libddq owns the
+multi-GPU path (include/ddq.h "multi-GPU"): an NCCL communicator per database
+(unique id bootstrapped through torch.distributed), dimension indexes built once on
+rank 0 and broadcast inside each plan's CUDA graph, and per step one ncclAllGather of
+the 13 packed partial group tables, merged exactly by ddq_dist_result on rank 0.
 
 --impl reference: the oracle (oracle/, single-threaded C++) on a bounded sample
 of the same workload, on the host's cores.
@@ -41,7 +44,11 @@ def parse():
     ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--sf", type=float, default=SF_PER_GPU, help="scale factor per GPU")
+    ap.add_argument("--sf", type=float, default=SF_PER_GPU, help="scale factor per GPU (weak scaling)")
+    ap.add_argument("--sf-total", type=float, default=0,
+                    help="strong scaling (S8(d) M3): one database of this SF, lineorder row-sharded over the ranks")
+    ap.add_argument("--no-build-once", action="store_true",
+                    help="N>1: every rank builds its dimension indexes (default: rank 0 builds, NCCL broadcasts)")
     ap.add_argument("--e2e-steps", type=int, default=5)
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--dump-results", default="",
@@ -258,7 +265,8 @@ def main():
         else:
             dist.init_process_group(backend)
     dws = args.emulate_world if (args.emulate_world and ws == 1) else ws  # ranks the data is sized for
-    sf_total = args.sf * dws
+    strong = args.sf_total > 0  # M3: one SF (e.g. 100) split over the ranks
+    sf_total = args.sf_total if strong else args.sf * dws
     data = datagen.SSB(sf_total)
     n_lo = data.rows("lineorder")
     b, e = rank * n_lo // dws, (rank + 1) * n_lo // dws
@@ -285,8 +293,24 @@ def main():
     # heap: intermediates scale with the shard (24 GiB at SF20's 120 M rows)
     heap = min(110 << 30, max(24 << 30, int((24 << 30) * shard_rows / 120_000_000)))
     db = Database(device=local, cache_bytes=64 << 30, heap_bytes=heap, rank=rank, world=ws)
+    if ws > 1:  # the library's multi-GPU exchange (S8(e)) before any plan is prepared
+        import torch.distributed as dist
+        if backend == "nccl":
+            from paper_conf_sigmod_bressft16_b200.engine import nccl_unique_id
+            box = [nccl_unique_id() if rank == 0 else None]
+            dist.broadcast_object_list(box, src=0)
+            db.dist_init_nccl(box[0], rank, ws, build_once=not args.no_build_once)
+        else:  # test hook: a host all-gather over the gloo process group
+            def host_allgather(buf: bytes) -> bytes:
+                t = torch.frombuffer(bytearray(buf), dtype=torch.uint8)
+                out = [torch.empty_like(t) for _ in range(ws)]
+                dist.all_gather(out, t)
+                return b"".join(bytes(o.numpy()) for o in out)
+            db.dist_init_host(rank, ws, host_allgather)
 
     load_ssb(db, shard, row_begin=b, row_end=e, presliced=True)
+    if ws > 1:
+        db.set_partitioned("lineorder")
     preps = [db.prepare(ssb_plan(db, q), use_graph=True) for q in SSB_QUERIES]
     setup_s = time.perf_counter() - t_setup
     stream = torch.cuda.Stream()
@@ -332,48 +356,17 @@ def main():
         args.streams = min(trial, key=trial.get)
         side = all_side[:args.streams - 1]
 
-    # N>1: the 13 compacted partial group tables of a step are packed on the device
-    # ([n, keys[cap], accs[cap*n_aggs*2]] per query) and exchanged with ONE NCCL
-    # all_gather; rank 0 merges them at finalisation (dist.py, S8(e)).
-    from paper_conf_sigmod_bressft16_b200 import dist as D
-
-    class _Dev:  # zero-copy torch view of a library-owned device buffer
-        def __init__(self, ptr, n, typestr):
-            self.__cuda_array_interface__ = {"data": (ptr, False), "shape": (n,), "typestr": typestr,
-                                             "version": 3}
-    views, offs, total = [], [], 0
-    if ws > 1:
-        for p in preps:
-            kp, ap, cp, cap = p.partials_device()
-            na = db._root_aggs[id(p)]
-            views.append((torch.as_tensor(_Dev(cp, 1, "<u4"), device="cuda"),
-                          torch.as_tensor(_Dev(kp, cap, "<i8"), device="cuda"),
-                          torch.as_tensor(_Dev(ap, cap * na * 2, "<i8"), device="cuda"), cap, na))
-            offs.append(total)
-            total += D.packed_words(cap, na)
-    packed = torch.zeros(max(total, 1), dtype=torch.int64, device="cuda")
-    gathered = torch.zeros(max(total, 1) * ws, dtype=torch.int64, device="cuda")
-
+    # N>1: after the 13 launches, libddq packs the compacted partial group tables on the
+    # device and all-gathers them (ncclAllGather over NVLink; the gloo test hook: a host
+    # all-gather), and merges them exactly at finalisation (ddq_dist_exchange /
+    # ddq_dist_result, S8(e)).
     def exchange():
-        if ws == 1:
-            return
-        import torch.distributed as dist
-        with torch.cuda.stream(stream):
-            for (cnt, keys, accs, cap, na), o in zip(views, offs):
-                packed[o:o + 1].copy_(cnt.to(torch.int64))
-                packed[o + 1:o + 1 + cap].copy_(keys)
-                packed[o + 1 + cap:o + 1 + cap + cap * na * 2].copy_(accs)
-            dist.all_gather_into_tensor(gathered, packed)
+        if ws > 1:
+            db.dist_exchange(preps, sptr)
 
     def merged_results():
-        """rank 0: unpack every rank's partials per query and finalise (exact merge)."""
-        g = gathered.view(ws, -1).cpu().numpy()
-        res = {}
-        for q, p, (cnt, keys, accs, cap, na), o in zip(SSB_QUERIES, preps, views, offs):
-            flat = g[:, o:o + D.packed_words(cap, na)].reshape(-1)
-            k, a = D.unpack_gathered(flat, ws, cap, na)
-            res[q] = p.finalize(k, a).rows
-        return res
+        """rank 0: every query's result over all ranks' rows."""
+        return {q: db.dist_result(i).rows for i, q in enumerate(SSB_QUERIES)}
 
     if args.profile_only:
         for _ in range(2):
@@ -512,8 +505,12 @@ def main():
     if rank == 0:
         line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": ws, "steps": args.steps,
                 "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
-                "scaling": "weak", "vs_baseline": None, "dtype": "int64", "data": "synthetic (datagen, seed 0x5EED2016)",
-                "config": {"workload": f"SSB SF{sf_total:g}, all 13 queries, hot cache (BASELINE configs[1])",
+                "scaling": "strong" if strong else "weak", "vs_baseline": None, "dtype": "int64",
+                "data": "synthetic (datagen, seed 0x5EED2016)",
+                "config": {"workload": f"SSB SF{sf_total:g}, all 13 queries, hot cache " +
+                                       ("(BASELINE configs[2]: lineorder row-sharded)" if ws > 1 else
+                                        "(BASELINE configs[1])"),
+                           "build_once": ws > 1 and backend == "nccl" and not args.no_build_once,
                            "lineorder_rows": n_lo, "rows_per_gpu": shard_rows, "queries": 13,
                            "parallelism": f"row-sharded x{ws}" if ws > 1 else "1 GPU",
                            "query_streams": max(args.streams, 1),

@@ -532,6 +532,43 @@ ddq_status ddq_prepared_finalize(ddq_prepared* p, int64_t n_groups, const int64_
                                  const int64_t* h_accs, ddq_result** out);
 void ddq_prepared_free(ddq_prepared* p);
 
+/* ---- multi-GPU: row-sharded fact table, one process per GPU (S8(e); Sec. 6.3
+ * "Our Data-Driven strategy can support multiple co-processors by performing
+ * horizontal partitioning").  Each rank loads its row range of the partitioned table
+ * (ddq_create_table's shard_row_begin = global row id of its first row) and the whole
+ * replicated (dimension) tables.
+ *
+ * ddq_dist_nccl_unique_id: 128 bytes for ncclCommInitRank (rank 0 creates it; the
+ * caller's bootstrap -- e.g. a torch.distributed process group -- sends it to the
+ * other ranks).  ddq_dist_init_nccl: the NCCL communicator of this database (NCCL is
+ * loaded at run time: DDQ_ENCCL if libnccl.so.2 is missing); build_once = 1: a
+ * prepared plan's HASH_BUILD over a replicated table runs on rank 0 only and its
+ * index is broadcast (ncclBroadcast on the plan's stream, inside its CUDA graph,
+ * which is then captured serially so every rank issues its collectives in one order;
+ * every rank must prepare the same plans in the same order).  ddq_dist_init_host:
+ * the same exchange through a caller-provided host all-gather (fn gathers `bytes` of
+ * `send` from every rank into `recv`, rank-major, returns 0 on success) -- e.g. a
+ * gloo process group; no build broadcast.
+ *
+ * ddq_table_set_partitioned: mark the row-sharded table (builds over it are never
+ * broadcast; its rows differ per rank).
+ *
+ * ddq_dist_exchange: after the plans' launches on `stream`, pack each plan's compacted
+ * partial group table ([count, keys[cap], accs[cap * n_aggs * 2]] int64 words) into a
+ * library-owned device buffer and all-gather it across the ranks (ncclAllGather on
+ * `stream`, asynchronous; host transport: synchronous).  Every rank calls it with the
+ * same plans in the same order.  ddq_dist_result(i): the result of plans[i] over ALL
+ * ranks' rows -- partial groups merged exactly (SUM / COUNT by int128 addition, MIN
+ * by minimum; the same result as one GPU) and finalised (S8(a7)); synchronises
+ * the exchange stream.  Owned by the caller (ddq_result_free). */
+typedef int32_t (*ddq_allgather_fn)(const void* send, void* recv, size_t bytes, void* user);
+ddq_status ddq_dist_nccl_unique_id(void* out128);
+ddq_status ddq_dist_init_nccl(ddq_db* db, const void* id128, int32_t rank, int32_t world, int32_t build_once);
+ddq_status ddq_dist_init_host(ddq_db* db, int32_t rank, int32_t world, ddq_allgather_fn fn, void* user);
+ddq_status ddq_table_set_partitioned(ddq_db* db, ddq_table t, int32_t partitioned);
+ddq_status ddq_dist_exchange(ddq_db* db, ddq_prepared* const* plans, int32_t n, void* stream);
+ddq_status ddq_dist_result(ddq_db* db, int32_t i, ddq_result** out);
+
 /* ---- statistics (paper's counters, D10: P:330) ---- */
 typedef struct {
   uint64_t h2d_bytes, d2h_bytes;

@@ -105,6 +105,9 @@ class Stats(ctypes.Structure):
                  "cache_misses", "queries_done")]
 
 
+# host all-gather callback of ddq_dist_init_host: (send, recv, bytes, user) -> 0 on success
+ALLGATHER_FN = ctypes.CFUNCTYPE(ctypes.c_int32, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_size_t, ctypes.c_void_p)
+
 # name -> (restype, argtypes)
 _vp, _i32, _i64, _u32, _u64, _sz = (ctypes.c_void_p, ctypes.c_int32, ctypes.c_int64, ctypes.c_uint32,
                                     ctypes.c_uint64, ctypes.c_size_t)
@@ -163,6 +166,12 @@ SIGNATURES = {
     "ddq_finalize_partials": (_i32, [ctypes.POINTER(Op), _i64, _vp, _vp, ctypes.POINTER(ctypes.POINTER(Result))]),
     "ddq_prepared_finalize": (_i32, [_vp, _i64, _vp, _vp, ctypes.POINTER(ctypes.POINTER(Result))]),
     "ddq_prepared_free": (None, [_vp]),
+    "ddq_dist_nccl_unique_id": (_i32, [_vp]),
+    "ddq_dist_init_nccl": (_i32, [_vp, _vp, _i32, _i32, _i32]),
+    "ddq_dist_init_host": (_i32, [_vp, _i32, _i32, _vp, _vp]),
+    "ddq_table_set_partitioned": (_i32, [_vp, _i32, _i32]),
+    "ddq_dist_exchange": (_i32, [_vp, ctypes.POINTER(_vp), _i32, _vp]),
+    "ddq_dist_result": (_i32, [_vp, _i32, ctypes.POINTER(ctypes.POINTER(Result))]),
     "ddq_get_stats": (_i32, [_vp, ctypes.POINTER(Stats)]),
     "ddq_reset_stats": (_i32, [_vp]),
     "ddq_heap_try_alloc": (_vp, [_vp, _u64]),

@@ -8,7 +8,8 @@ import sys
 HERE = os.path.dirname(os.path.abspath(__file__))
 CSRC = os.path.join(HERE, "csrc")
 SO = os.path.join(HERE, "libddq.so")
-SOURCES = ["transfer.cu", "filter.cu", "dense.cu", "agg.cu", "scan.cu", "star.cu", "kernels.cu", "ops.cu", "engine.cpp", "driver.cpp"]
+SOURCES = ["transfer.cu", "filter.cu", "dense.cu", "agg.cu", "scan.cu", "star.cu", "kernels.cu", "ops.cu", "engine.cpp",
+           "driver.cpp", "dist.cpp"]
 HEADERS = ["device_common.cuh", "ops_internal.h", "engine.h"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
@@ -44,7 +45,7 @@ def build(force: bool = False, verbose: bool = False) -> str:
                    os.path.join(CSRC, src), "-o", obj]
         subprocess.check_call(cmd)
     tmp = SO + ".tmp"
-    subprocess.check_call([NVCC, *ARCH, "-shared", "-o", tmp, *objs, "-lpthread", "-Xlinker", "--no-undefined"])
+    subprocess.check_call([NVCC, *ARCH, "-shared", "-o", tmp, *objs, "-lpthread", "-ldl", "-Xlinker", "--no-undefined"])
     os.replace(tmp, SO)
     return SO
 

@@ -416,12 +416,15 @@ ddq_status run_gpu_op(GpuOpCtx& ctx, const ddq_op& op, Inter& out) {
         out.cap = 0;
         if (A.failed) return DDQ_ENOMEM_DEVICE;
         init_fill(out.d_error, 4, 0, st);
-        cudaError_t e = join_index_init(out.jidx, out.jrange, st);
-        if (e == cudaSuccess && op.build_key_set == 2)  // MIN build: payloads start at INT32_MAX
+        const bool recv = ctx.dist && dist_build_receives(db, op);  // built once, on rank 0 (S8(e))
+        cudaError_t e = recv ? cudaSuccess : join_index_init(out.jidx, out.jrange, st);
+        if (e == cudaSuccess && op.build_key_set == 2 && !recv)  // MIN build: payloads start at INT32_MAX
           e = init_fill(join_index_payload(out.jidx, out.jrange), (size_t)out.jrange * 4, 0x7FFFFFFF7FFFFFFFull, st);
-        if (e == cudaSuccess)
+        if (e == cudaSuccess && !recv)
           e = launch_join_index_build(keys, payload, in_tids, in_cnt, in_cap, out.jmin, out.jrange, out.jidx,
                                       out.d_error, st, &bp);
+        if (e == cudaSuccess && ctx.dist)
+          return dist_build_broadcast(db, op, out.jidx, join_index_bytes(out.jrange), st);
         return cuda_status(e, "join_index_build");
       }
       // sparse keys: open addressing; small tables (shared-memory resident) get load <= 0.25
@@ -434,10 +437,13 @@ ddq_status run_gpu_op(GpuOpCtx& ctx, const ddq_op& op, Inter& out) {
       out.cap = 0;
       if (A.failed) return DDQ_ENOMEM_DEVICE;
       init_fill(out.d_error, 4, 0, st);
-      cudaError_t e = launch_hash_init(out.table_ptr, out.table_cap, st);
-      if (e == cudaSuccess)
+      const bool recv = ctx.dist && dist_build_receives(db, op);  // built once, on rank 0 (S8(e))
+      cudaError_t e = recv ? cudaSuccess : launch_hash_init(out.table_ptr, out.table_cap, st);
+      if (e == cudaSuccess && !recv)
         e = launch_hash_build(keys, payload, in_tids, in_cnt, in_cap, out.table_ptr, out.table_cap, out.d_error, st,
                               &bp);
+      if (e == cudaSuccess && ctx.dist)
+        return dist_build_broadcast(db, op, out.table_ptr, (size_t)out.table_cap * 8, st);
       return cuda_status(e, "hash_build");
     }
     case DDQ_OP_GATHER: {
@@ -1048,6 +1054,7 @@ ddq_status ddq_open(const ddq_config* cfg, ddq_db** out) {
 void ddq_close(ddq_db* db) {
   if (!db) return;
   ddq::driver_stop(db);
+  ddq::dist_free(db);
   cudaSetDevice(db->device);
   cudaDeviceSynchronize();
   for (auto& c : db->cols) {
@@ -1594,6 +1601,7 @@ static ddq_status replay_op(ddq_prepared* P, int i, cudaStream_t st) {
   ctx.count_column_access = false;
   ctx.reuse = &blocks;
   ctx.bits_out = P->bits_out[(size_t)i] != 0;
+  ctx.dist = true;
   return run_gpu_op(ctx, P->plan.ops[i], P->inters[(size_t)i]);
 }
 static ddq_status replay(ddq_prepared* P, cudaStream_t st) {
@@ -1830,6 +1838,7 @@ ddq_status ddq_prepare(ddq_db* db, const ddq_plan* plan, int32_t use_graph, ddq_
     ctx.forced_cap = P->forced[(size_t)i];
     ctx.count_column_access = false;
     ctx.bits_out = P->bits_out[(size_t)i] != 0;
+    ctx.dist = true;
     ddq_status s = run_gpu_op(ctx, plan->ops[i], P->inters[(size_t)i]);
     if (s != DDQ_OK) {
       fill_hoist().rec = nullptr;
@@ -1845,7 +1854,8 @@ ddq_status ddq_prepare(ddq_db* db, const ddq_plan* plan, int32_t use_graph, ddq_
     e = cudaStreamBeginCapture(st, cudaStreamCaptureModeThreadLocal);
     if (e != cudaSuccess) return fail(cuda_status(e, "prepare: begin capture"));
     static const char* env = getenv("DDQ_GRAPH_BRANCHES");  // "0": one serial chain
-    const bool branches = !env || env[0] != '0';
+    // multi-GPU build broadcasts: one collective order on every rank -> serial capture
+    const bool branches = (!env || env[0] != '0') && !dist_serial_capture(db);
     // all buffer initialisations as ONE fill kernel at the graph root; the
     // operators' own fills are skipped while capturing
     ddq_status s = DDQ_OK;
@@ -1903,6 +1913,7 @@ int32_t ddq_prepared_profile(ddq_prepared* p, void* stream, int32_t max_ops, flo
     ctx.count_column_access = false;
     ctx.reuse = &blocks;
     ctx.bits_out = p->bits_out[(size_t)i] != 0;
+    ctx.dist = true;
     ddq_status s = run_gpu_op(ctx, p->plan.ops[i], p->inters[(size_t)i]);
     if (s != DDQ_OK) {
       for (auto& e : ev) cudaEventDestroy(e);
@@ -2066,6 +2077,16 @@ ddq_status ddq_prepared_partials(ddq_prepared* p, void* stream, int64_t* h_n_gro
   return DDQ_OK;
 }
 
+ddq_status ddq_prepared_partials_device(ddq_prepared* p, int64_t** keys, int64_t** accs, uint32_t** count,
+                                        int64_t* cap);
+}  // extern "C"
+namespace ddq {
+const ddq_plan& prepared_plan(const ddq_prepared* p) { return p->plan; }
+ddq_status prepared_partials_device(ddq_prepared* p, int64_t** keys, int64_t** accs, uint32_t** count, int64_t* cap) {
+  return ddq_prepared_partials_device(p, keys, accs, count, cap);
+}
+}  // namespace ddq
+extern "C" {
 ddq_status ddq_prepared_partials_device(ddq_prepared* p, int64_t** keys, int64_t** accs, uint32_t** count,
                                         int64_t* cap) {
   if (!p || !keys || !accs || !count || !cap) return set_error(DDQ_EINVAL, "prepared_partials_device: null");

@@ -69,6 +69,7 @@ struct Table {
   std::string name;
   int64_t n_rows = 0;
   int64_t row_begin = 0;
+  bool partitioned = false;  // row-sharded across ranks (ddq_table_set_partitioned)
   std::vector<int> cols;
 };
 
@@ -153,6 +154,7 @@ struct ddq_db {
   bool stopping = false;
   std::vector<std::thread> workers;
   int busy_gpu = 0;
+  void* dist = nullptr;  // multi-GPU state (dist.cpp), or null
 };
 
 namespace ddq {
@@ -170,7 +172,15 @@ struct GpuOpCtx {
   // a dense semi-join probe writes its survivors as a row bitmap (1 bit per row)
   // instead of a TID list: set by ddq_prepare when every consumer reads bitmaps
   bool bits_out = false;
+  // prepared plans on a multi-GPU database: builds over replicated tables run once and
+  // are broadcast (dist.cpp); off for calibration runs and the chopping driver
+  bool dist = false;
 };
+// dist.cpp
+void dist_free(ddq_db* db);
+bool dist_build_receives(ddq_db* db, const ddq_op& op);
+ddq_status dist_build_broadcast(ddq_db* db, const ddq_op& op, void* buf, size_t bytes, cudaStream_t st);
+bool dist_serial_capture(ddq_db* db);
 void count_accesses(ddq_db* db, const ddq_op& op);
 void driver_start(ddq_db* db);
 void driver_stop(ddq_db* db);

@@ -255,6 +255,13 @@ class PlanBuilder:
         return idx
 
 
+def nccl_unique_id() -> bytes:
+    """128-byte NCCL unique id (rank 0 creates it; the bootstrap sends it to the others)."""
+    buf = ctypes.create_string_buffer(128)
+    check(lib().ddq_dist_nccl_unique_id(buf))
+    return buf.raw
+
+
 def finalize_partials(root: A.Op, keys: np.ndarray, accs: np.ndarray) -> QueryResult:
     """Host finalisation of (possibly duplicated) partial groups: exact merge of equal
     packed keys, ORDER BY / LIMIT of the root AGGREGATE (no GPU needed)."""
@@ -481,6 +488,38 @@ class Database:
 
     def reset_access_counts(self) -> None:
         check(lib().ddq_reset_access_counts(self.h))
+
+    # ---- multi-GPU (include/ddq.h "multi-GPU"; S8(e)) -----------------------
+    def set_partitioned(self, table: str, partitioned: bool = True) -> None:
+        check(lib().ddq_table_set_partitioned(self.h, self._tables[table], 1 if partitioned else 0))
+
+    def dist_init_nccl(self, unique_id: bytes, rank: int, world: int, build_once: bool = True) -> None:
+        """NCCL communicator of this database (unique_id from nccl_unique_id() on rank 0)."""
+        buf = ctypes.create_string_buffer(bytes(unique_id), 128)
+        check(lib().ddq_dist_init_nccl(self.h, buf, rank, world, 1 if build_once else 0))
+
+    def dist_init_host(self, rank: int, world: int, allgather) -> None:
+        """Exchange through a host all-gather: allgather(send: bytes) -> bytes (rank-major)."""
+        def cb(send, recv, nbytes, user):
+            try:
+                out = allgather(ctypes.string_at(send, nbytes))
+                ctypes.memmove(recv, out, len(out))
+                return 0
+            except Exception:  # an exception must not cross the C ABI
+                return -1
+        self._allgather_cb = A.ALLGATHER_FN(cb)  # kept alive with the database
+        check(lib().ddq_dist_init_host(self.h, rank, world, ctypes.cast(self._allgather_cb, ctypes.c_void_p), None))
+
+    def dist_exchange(self, preps: list, stream: int = 0) -> None:
+        """All-gather the partial group tables of the prepared plans (after their launches)."""
+        arr = (ctypes.c_void_p * len(preps))(*[p.h.value if hasattr(p.h, "value") else p.h for p in preps])
+        check(lib().ddq_dist_exchange(self.h, arr, len(preps), ctypes.c_void_p(stream)))
+
+    def dist_result(self, i: int) -> QueryResult:
+        """The result of plan i of the last exchange over every rank's rows."""
+        p = ctypes.POINTER(A.Result)()
+        check(lib().ddq_dist_result(self.h, i, ctypes.byref(p)))
+        return _convert(p)
 
     # ---- plans -----------------------------------------------------------------
     def plan(self) -> PlanBuilder:
