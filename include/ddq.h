@@ -264,6 +264,10 @@ typedef struct {
                                     cold cache load copies that and widens it on the device
                                     (fewer bytes over PCIe);
                                     0: copy the raw column */
+  int32_t max_queries;           /* query-level admission control (the comparison arm of P:371,
+                                    P:445, Wang et al.): at most this many submitted queries run at
+                                    once, later ones wait in submission order until one finishes;
+                                    0 (default) = no admission control */
   uint32_t fault_op_mask;        /* fault injection: the GPU attempt of plan op i (i < 32) aborts as if
                                     its heap allocation failed when bit i is set (deterministic
                                     abort -> host restart traces, Fig. 8); 0 = off */

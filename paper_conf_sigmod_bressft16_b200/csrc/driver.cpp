@@ -619,10 +619,14 @@ ddq_status run_host_op(ddq_db* db, const ddq_op& op, const std::vector<Inter>& I
         if (!tb.back()->host_table && !tb.back()->h_bitmap) return set_error(DDQ_ESTATE, "host aggregate: term build not on the host");
       }
       const int n_in_vecs = in ? (int)in->vecs.size() : 0;
-      std::unordered_map<int64_t, std::vector<__int128>> g;
       std::vector<const Column*> apc;  // fused selection (AGGREGATE op with predicates)
       for (int p = 0; p < op.n_preds; p++) apc.push_back(col_of(db, op.preds[p].column));
-      for (int64_t i = 0; i < n; i++) {
+      // every core of the op's share aggregates a row range into its own table
+      // (A2: an operator uses all cores); the tables merge exactly below
+      std::vector<std::unordered_map<int64_t, std::vector<__int128>>> part((size_t)std::max(threads, 1));
+      parallel_chunks(n, threads, [&](int chunk, int64_t b, int64_t e) {
+      auto& g = part[(size_t)chunk];
+      for (int64_t i = b; i < e; i++) {
         int32_t r = row_of(i);
         bool ok = true;
         for (int p = 0; p < op.n_preds && ok; p++) {
@@ -677,6 +681,19 @@ ddq_status run_host_op(ddq_db* db, const ddq_op& op, const std::vector<Inter>& I
           acc[(size_t)a] += v;
         }
       }
+      });
+      std::unordered_map<int64_t, std::vector<__int128>>& g = part[0];
+      for (size_t t = 1; t < part.size(); t++)
+        for (auto& kv : part[t]) {
+          auto it = g.find(kv.first);
+          if (it == g.end()) {
+            g.emplace(kv.first, std::move(kv.second));
+            continue;
+          }
+          for (int a = 0; a < na; a++)
+            it->second[(size_t)a] = op.agg_kind[a] == DDQ_AGG_MIN ? std::min(it->second[(size_t)a], kv.second[(size_t)a])
+                                                                 : it->second[(size_t)a] + kv.second[(size_t)a];
+        }
       auto keys = std::make_shared<std::vector<int64_t>>();
       auto accs = std::make_shared<std::vector<int64_t>>();
       for (auto& kv : g) {
@@ -770,6 +787,30 @@ static bool hold_if_cached(ddq_db* db, const ddq_op& op) {
 
 static void enqueue(ddq_db* db, std::shared_ptr<QueryState> q, int i);
 
+// The leaf operators of a query enter the global operator stream.  Collect
+// them first: once one is enqueued, workers may finish it and make parents ready.
+static void start_query(ddq_db* db, std::shared_ptr<QueryState> q) {
+  std::vector<int> leaves;
+  for (int i = 0; i < q->plan.n_ops; i++)
+    if (q->pending[(size_t)i] == 0) leaves.push_back(i);
+  for (int i : leaves) enqueue(db, q, i);
+}
+
+// A query finished or failed: its admission slot goes to the oldest waiting query.
+static void release_admission(ddq_db* db) {
+  std::shared_ptr<QueryState> next;
+  {
+    std::lock_guard<std::mutex> g(db->qmu);
+    db->running_queries--;
+    if (!db->admit_queue.empty() && (db->cfg.max_queries <= 0 || db->running_queries < db->cfg.max_queries)) {
+      next = db->admit_queue.front();
+      db->admit_queue.pop_front();
+      db->running_queries++;
+    }
+  }
+  if (next) start_query(db, next);
+}
+
 static void finish_query(ddq_db* db, QueryState& q) {
   const ddq_op& root = q.plan.ops[q.plan.n_ops - 1];
   Inter& r = q.inters.back();
@@ -836,19 +877,26 @@ static void finish_query(ddq_db* db, QueryState& q) {
   q.cv.notify_all();
 }
 
+static void finish_query_and_admit(ddq_db* db, QueryState& q) {
+  finish_query(db, q);
+  release_admission(db);
+}
+
 // A failed operator fails its query: waiters are woken at once, but the query's
 // intermediates are released only when no operator of it is still running (the
 // caller is itself in flight; worker_loop releases when the count drains).
 static void fail_query(ddq_db* db, QueryState& q, ddq_status s) {
-  (void)db;
   std::string msg = ddq_last_error();
-  std::lock_guard<std::mutex> g(q.mu);
-  if (q.done) return;
-  q.status = s;
-  q.error = msg;
-  q.failed = true;
-  q.done = true;
-  q.cv.notify_all();
+  {
+    std::lock_guard<std::mutex> g(q.mu);
+    if (q.done) return;
+    q.status = s;
+    q.error = msg;
+    q.failed = true;
+    q.done = true;
+    q.cv.notify_all();
+  }
+  release_admission(db);
 }
 
 // Called when op i of q finished: notify parents, free consumed inputs.
@@ -867,7 +915,7 @@ static void op_finished(ddq_db* db, std::shared_ptr<QueryState> q, int i) {
     last = --q->ops_left == 0;
   }
   for (int p : ready) enqueue(db, q, p);
-  if (last) finish_query(db, *q);
+  if (last) finish_query_and_admit(db, *q);
 }
 
 static int decide_place(ddq_db* db, QueryState& q, int i) {
@@ -1005,9 +1053,17 @@ static void worker_loop(ddq_db* db, bool gpu) {
       auto& Q = gpu ? db->gpu_ready : db->host_ready;
       db->qcv.wait(g, [&] { return db->stopping || !Q.empty(); });
       if (db->stopping) break;
-      q = Q.front().first;
-      i = Q.front().second;
-      Q.pop_front();
+      // pull the ready operator of the OLDEST query (FIFO among its ops): a query
+      // already in flight finishes before the leaves of newer ones start, so the
+      // heap holds the intermediates of about gpu_workers queries, not of every
+      // submitted one (measured M5: FIFO pulls let 32 users' first intermediates
+      // pile up and abort, profiles/r2_config5_sf20.jsonl)
+      auto pick = Q.begin();
+      for (auto it = Q.begin(); it != Q.end(); ++it)
+        if (it->first->id < pick->first->id) pick = it;
+      q = pick->first;
+      i = pick->second;
+      Q.erase(pick);
     }
     {
       std::lock_guard<std::mutex> g(q->mu);
@@ -1086,18 +1142,21 @@ ddq_status ddq_submit(ddq_db* db, const ddq_plan* plan, ddq_query* out) {
       }
     }
   }
+  bool admitted = true;
   {
     std::lock_guard<std::mutex> g(db->qmu);
     q->id = db->next_query++;
     db->queries[q->id] = q;
+    // admission control (max_queries): beyond the limit the query waits its turn
+    if (db->cfg.max_queries > 0 && db->running_queries >= db->cfg.max_queries) {
+      db->admit_queue.push_back(q);
+      admitted = false;
+    } else {
+      db->running_queries++;
+    }
   }
   *out = q->id;
-  // leaf operators enter the global operator stream.  Collect them first:
-  // once one is enqueued, workers may finish it and make parents ready concurrently.
-  std::vector<int> leaves;
-  for (int i = 0; i < n; i++)
-    if (q->pending[(size_t)i] == 0) leaves.push_back(i);
-  for (int i : leaves) enqueue(db, q, i);
+  if (admitted) start_query(db, q);
   return DDQ_OK;
 }
 

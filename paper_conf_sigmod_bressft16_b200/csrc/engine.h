@@ -154,6 +154,9 @@ struct ddq_db {
   bool stopping = false;
   std::vector<std::thread> workers;
   int busy_gpu = 0;
+  // admission control (ddq_config.max_queries): queries running / waiting (qmu)
+  int running_queries = 0;
+  std::deque<std::shared_ptr<ddq::QueryState>> admit_queue;
   void* dist = nullptr;  // multi-GPU state (dist.cpp), or null
 };
 

@@ -373,7 +373,8 @@ class Database:
     def __init__(self, device: int = 0, cache_bytes: int = 64 << 30, heap_bytes: int = 32 << 30,
                  gpu_workers: int = 4, host_workers: int = 4, placement: int = A.PLACE_DATA_DRIVEN,
                  chopping: bool = True, cache_policy: int = 0, fault_alloc_every: int = 0,
-                 rank: int = 0, world: int = 1, transfer_packing: bool = True, fault_op_mask: int = 0):
+                 rank: int = 0, world: int = 1, transfer_packing: bool = True, fault_op_mask: int = 0,
+                 max_queries: int = 0):
         cfg = A.Config()
         lib().ddq_config_default(ctypes.byref(cfg))
         cfg.device, cfg.rank, cfg.world = device, rank, world
@@ -383,6 +384,7 @@ class Database:
         cfg.cache_policy, cfg.fault_alloc_every = cache_policy, fault_alloc_every
         cfg.transfer_packing = 1 if transfer_packing else 0
         cfg.fault_op_mask = fault_op_mask
+        cfg.max_queries = max_queries
         h = ctypes.c_void_p()
         check(lib().ddq_open(ctypes.byref(cfg), ctypes.byref(h)))
         self.h = h

@@ -274,3 +274,17 @@ def test_fig8_abort_then_successor_placement(chopping):
         assert st["h2d_bytes"] > 0           # op1's output copied back for op2
     assert st["d2h_bytes"] > 0               # op0's output moved to the CPU for op1's restart
     db.close()
+
+
+def test_admission_control_runs_queries_one_at_a_time():
+    """ddq_config.max_queries = 1 (the admission-control arm): concurrently
+    submitted queries run strictly in submission order, one at a time; results are
+    unchanged (P:111)."""
+    from paper_conf_sigmod_bressft16_b200 import _abi as A
+    db, want = _chain_db(placement=A.PLACE_GPU_ONLY, chopping=False, max_queries=1)
+    qs = [db.submit(_chain(db)) for _ in range(8)]
+    res = [db.fetch(q) for q in qs]
+    assert all(np.array_equal(r.tids, want) for r in res)
+    ms = [r.exec_ms for r in res]  # submit -> done: FIFO service makes it increase
+    assert ms == sorted(ms)
+    db.close()
