@@ -51,6 +51,7 @@ def parse():
                     help="N>1: every rank builds its dimension indexes (default: rank 0 builds, NCCL broadcasts)")
     ap.add_argument("--e2e-steps", type=int, default=5)
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-prefetch", action="store_true", help="e2e: copy columns on demand instead of streaming")
     ap.add_argument("--dump-results", default="",
                     help="rank 0 writes the 13 (merged) query results of the timed plans as JSON (tests)")
     ap.add_argument("--emulate-world", type=int, default=0,
@@ -468,7 +469,8 @@ def main():
     #      H2D from pinned host memory inside the timed region (GPU-only placement)
     e2e = None
     if not args.no_e2e and ws == 1:
-        cold = Database(device=local, cache_bytes=64 << 30, heap_bytes=heap, placement=A.PLACE_GPU_ONLY)
+        cold = Database(device=local, cache_bytes=64 << 30, heap_bytes=heap, placement=A.PLACE_GPU_ONLY,
+                        prefetch=not args.no_prefetch)
         load_ssb(cold, shard, row_begin=b, row_end=e, cache=False, presliced=True)
         plans = [ssb_plan(cold, q) for q in SSB_QUERIES]
         all_cols = [(t, c) for (t, c) in cold._cols]
@@ -495,7 +497,9 @@ def main():
                "d2h_bytes_per_step": st["d2h_bytes"] // args.e2e_steps,
                "h2d_gbs": round(st["h2d_bytes"] / dt / 1e9, 2), "step_ms": step_ms,
                "path": "ddq_submit (13 queries at once) / ddq_fetch, GPU-only placement, empty cache; "
-                       "columns copied on demand from pinned host memory (cold cache, P:32)"}
+                       "columns copied from pinned host memory (cold cache, P:32)" +
+                       ("; streamed cold path: the plans' columns stream in from submit while earlier "
+                        "operators compute (prefetch, N1)" if not args.no_prefetch else "; on demand")}
         cold.close()
 
     cpu = None

@@ -264,6 +264,14 @@ typedef struct {
                                     cold cache load copies that and widens it on the device
                                     (fewer bytes over PCIe);
                                     0: copy the raw column */
+  int32_t prefetch;              /* 1: streamed cold path (S8(f) N1, "overlap data transfer and
+                                    computation"): at submit, every column the plan reads that is not
+                                    resident is queued for an asynchronous H2D copy in plan order on
+                                    the copy stream (a background copy thread), so operator k computes
+                                    while the columns of operators k+1.. stream in; GPU workers pull
+                                    ready operators whose columns are resident first (cached-first
+                                    schedule).  0 (default): columns are copied when an operator
+                                    needs them (the paper's operator-driven placement) */
   int32_t max_queries;           /* query-level admission control (the comparison arm of P:371,
                                     P:445, Wang et al.): at most this many submitted queries run at
                                     once, later ones wait in submission order until one finishes;
@@ -482,6 +490,8 @@ typedef struct {
   int32_t n_ops;
   int32_t _pad2;
   const uint8_t* op_place;
+  const float* op_ms;    /* driver results: per op, host wall time from its pull by a worker to its
+                            completion (incl. transfers and synchronisation), ms; else NULL */
 } ddq_result;
 enum { DDQ_RAN_GPU = 1, DDQ_RAN_HOST = 2, DDQ_RAN_ABORTED = 3 };
 

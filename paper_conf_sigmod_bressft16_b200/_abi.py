@@ -45,7 +45,7 @@ class Config(ctypes.Structure):
                 ("gpu_workers", ctypes.c_int32), ("host_workers", ctypes.c_int32),
                 ("placement", ctypes.c_int32), ("chopping", ctypes.c_int32),
                 ("cache_policy", ctypes.c_int32), ("fault_alloc_every", ctypes.c_uint32),
-                ("transfer_packing", ctypes.c_int32), ("max_queries", ctypes.c_int32),
+                ("transfer_packing", ctypes.c_int32), ("prefetch", ctypes.c_int32), ("max_queries", ctypes.c_int32),
                 ("fault_op_mask", ctypes.c_uint32)]
 
 
@@ -96,7 +96,7 @@ class Result(ctypes.Structure):
                 ("exec_ms", ctypes.c_double), ("agg_null", ctypes.POINTER(ctypes.c_uint8)),
                 ("n_avg", ctypes.c_int32), ("_pad", ctypes.c_int32), ("avgs", ctypes.POINTER(ctypes.c_double)),
                 ("key_str", ctypes.POINTER(ctypes.c_char_p)), ("n_ops", ctypes.c_int32), ("_pad2", ctypes.c_int32),
-                ("op_place", ctypes.POINTER(ctypes.c_uint8))]
+                ("op_place", ctypes.POINTER(ctypes.c_uint8)), ("op_ms", ctypes.POINTER(ctypes.c_float))]
 
 
 class Stats(ctypes.Structure):

@@ -52,6 +52,8 @@ struct QueryState {
   uint64_t t_submit = 0, t_done = 0;
   int gpu_ops = 0, host_ops = 0, aborts = 0;
   std::vector<uint8_t> trace;               // per op: DDQ_RAN_GPU / _HOST / _ABORTED
+  std::vector<float> op_ms;                 // per op: wall time from pull to completion
+  std::vector<uint64_t> op_t0;
   std::mutex mu;
   std::condition_variable cv;
 };
@@ -868,6 +870,9 @@ static void finish_query(ddq_db* db, QueryState& q) {
     std::copy(q.trace.begin(), q.trace.end(), tr);
     res->n_ops = (int32_t)q.trace.size();
     res->op_place = tr;
+    float* om = new float[std::max<size_t>(q.op_ms.size(), 1)];
+    std::copy(q.op_ms.begin(), q.op_ms.end(), om);
+    res->op_ms = om;
   }
   q.t_done = now_ns();
   if (res) res->exec_ms = (double)(q.t_done - q.t_submit) / 1e6;
@@ -954,6 +959,7 @@ static void run_on_host(ddq_db* db, std::shared_ptr<QueryState> q, int i, cudaSt
     return;
   }
   q->inters[(size_t)i] = std::move(out);
+  q->op_ms[(size_t)i] = (float)((now_ns() - q->op_t0[(size_t)i]) / 1e6);
   q->host_ops++;
   if (q->trace[(size_t)i] != DDQ_RAN_ABORTED) q->trace[(size_t)i] = DDQ_RAN_HOST;
   db->stats.host_ops++;
@@ -1035,10 +1041,45 @@ static void run_on_gpu(ddq_db* db, std::shared_ptr<QueryState> q, int i, cudaStr
   }
   if (op.kind == DDQ_OP_GATHER) out.count = q->inters[(size_t)op.input].count;
   q->inters[(size_t)i] = std::move(out);
+  q->op_ms[(size_t)i] = (float)((now_ns() - q->op_t0[(size_t)i]) / 1e6);
   q->trace[(size_t)i] = DDQ_RAN_GPU;
   q->gpu_ops++;
   db->stats.gpu_ops++;
   op_finished(db, q, i);
+}
+
+// Streamed cold path (N1): copy the queued columns in order on the copy stream
+// while the operators of earlier-arriving data compute.  A column that no longer
+// fits the cache budget is skipped (the operator copies it on demand, LRU).
+static void prefetch_loop(ddq_db* db) {
+  cudaSetDevice(db->device);
+  while (true) {
+    int c = -1;
+    {
+      std::unique_lock<std::mutex> g(db->qmu);
+      db->qcv.wait(g, [&] { return db->stopping || !db->prefetch_queue.empty(); });
+      if (db->stopping) break;
+      c = db->prefetch_queue.front();
+      db->prefetch_queue.pop_front();
+    }
+    std::unique_lock<std::mutex> lk(db->mu);
+    if (c < 0 || c >= (int)db->cols.size()) continue;
+    Column& col = *db->cols[(size_t)c];
+    if (col.dev || col.loading) continue;
+    const uint64_t bytes = (uint64_t)std::max<int64_t>(col.n, 1) * col.width;
+    if (db->cache_used + bytes > db->cfg.cache_bytes) continue;
+    (void)cache_column_locked(db, c, true, lk);  // failures: the operator fetches on demand
+  }
+}
+
+// every input column of op resident on the GPU (the cached-first pull order)
+static bool op_resident(ddq_db* db, const ddq_op& op) {
+  std::lock_guard<std::mutex> g(db->mu);
+  for (int c : op_columns(op)) {
+    const Column* col = col_of(db, c);
+    if (!col || !col->dev || col->loading) return false;
+  }
+  return true;
 }
 
 static void worker_loop(ddq_db* db, bool gpu) {
@@ -1061,6 +1102,11 @@ static void worker_loop(ddq_db* db, bool gpu) {
       auto pick = Q.begin();
       for (auto it = Q.begin(); it != Q.end(); ++it)
         if (it->first->id < pick->first->id) pick = it;
+      if (gpu && db->cfg.prefetch && !op_resident(db, pick->first->plan.ops[pick->second]))
+        for (auto it = Q.begin(); it != Q.end(); ++it)  // cached-first: an op whose data is here
+          if (op_resident(db, it->first->plan.ops[it->second]) &&
+              (!op_resident(db, pick->first->plan.ops[pick->second]) || it->first->id < pick->first->id))
+            pick = it;
       q = pick->first;
       i = pick->second;
       Q.erase(pick);
@@ -1070,6 +1116,7 @@ static void worker_loop(ddq_db* db, bool gpu) {
       if (q->done) continue;  // failed query: drop remaining ops
       q->inflight++;
     }
+    q->op_t0[(size_t)i] = now_ns();  // op_ms: pull -> completion (recorded before op_finished)
     if (gpu) run_on_gpu(db, q, i, st);
     else run_on_host(db, q, i, st);
     std::lock_guard<std::mutex> g(q->mu);
@@ -1088,6 +1135,7 @@ void driver_start(ddq_db* db) {
   int h = db->cfg.chopping ? db->cfg.host_workers : std::max(db->cfg.host_workers, 16);
   for (int i = 0; i < g; i++) db->workers.emplace_back(worker_loop, db, true);
   for (int i = 0; i < h; i++) db->workers.emplace_back(worker_loop, db, false);
+  if (db->cfg.prefetch && db->cfg.placement != DDQ_PLACE_CPU_ONLY) db->prefetcher = std::thread(prefetch_loop, db);
 }
 
 void driver_stop(ddq_db* db) {
@@ -1098,6 +1146,7 @@ void driver_stop(ddq_db* db) {
   }
   for (auto& t : db->workers) t.join();
   db->workers.clear();
+  if (db->prefetcher.joinable()) db->prefetcher.join();
   for (auto& kv : db->queries) {
     for (auto& x : kv.second->inters) release_inter(db, x);
     if (kv.second->result) ddq_result_free(kv.second->result);
@@ -1123,6 +1172,8 @@ ddq_status ddq_submit(ddq_db* db, const ddq_plan* plan, ddq_query* out) {
   q->consumers_left.assign((size_t)n, 0);
   q->place.assign((size_t)n, P_NONE);
   q->trace.assign((size_t)n, 0);
+  q->op_ms.assign((size_t)n, 0.f);
+  q->op_t0.assign((size_t)n, 0);
   q->ops_left = n;
   q->t_submit = now_ns();
   for (int i = 0; i < n; i++)
@@ -1156,6 +1207,15 @@ ddq_status ddq_submit(ddq_db* db, const ddq_plan* plan, ddq_query* out) {
     }
   }
   *out = q->id;
+  if (db->cfg.prefetch && db->cfg.placement != DDQ_PLACE_CPU_ONLY) {  // N1: stream the plan's columns in
+    std::vector<int> cols;
+    for (int i = 0; i < n; i++)
+      for (int c : op_columns(plan->ops[i]))
+        if (std::find(cols.begin(), cols.end(), c) == cols.end()) cols.push_back(c);
+    std::lock_guard<std::mutex> g(db->qmu);
+    for (int c : cols) db->prefetch_queue.push_back(c);
+    db->qcv.notify_all();
+  }
   if (admitted) start_query(db, q);
   return DDQ_OK;
 }

@@ -157,6 +157,9 @@ struct ddq_db {
   // admission control (ddq_config.max_queries): queries running / waiting (qmu)
   int running_queries = 0;
   std::deque<std::shared_ptr<ddq::QueryState>> admit_queue;
+  // streamed cold path (ddq_config.prefetch): columns queued for H2D (qmu), copy thread
+  std::deque<int> prefetch_queue;
+  std::thread prefetcher;
   void* dist = nullptr;  // multi-GPU state (dist.cpp), or null
 };
 

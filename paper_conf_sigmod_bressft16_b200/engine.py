@@ -27,6 +27,7 @@ class QueryResult:
     avgs: list = field(default_factory=list)
     decoded: list = field(default_factory=list)
     placement: list = field(default_factory=list)  # per plan op: A.RAN_GPU / RAN_HOST / RAN_ABORTED
+    op_ms: list = field(default_factory=list)      # per plan op: wall ms (driver results)
     n_keys: int = 0
     n_aggs: int = 0
     gpu_ops: int = 0
@@ -45,6 +46,8 @@ def _convert(res_ptr) -> QueryResult:
     nk, na = r.n_keys, r.n_aggs
     if r.op_place:
         out.placement = [int(r.op_place[i]) for i in range(r.n_ops)]
+    if r.op_ms:
+        out.op_ms = [float(r.op_ms[i]) for i in range(r.n_ops)]
     for i in range(r.n_rows):
         vals = [int(r.keys[i * nk + k]) for k in range(nk)]
         for a in range(na):
@@ -374,7 +377,7 @@ class Database:
                  gpu_workers: int = 4, host_workers: int = 4, placement: int = A.PLACE_DATA_DRIVEN,
                  chopping: bool = True, cache_policy: int = 0, fault_alloc_every: int = 0,
                  rank: int = 0, world: int = 1, transfer_packing: bool = True, fault_op_mask: int = 0,
-                 max_queries: int = 0):
+                 max_queries: int = 0, prefetch: bool = False):
         cfg = A.Config()
         lib().ddq_config_default(ctypes.byref(cfg))
         cfg.device, cfg.rank, cfg.world = device, rank, world
@@ -385,6 +388,7 @@ class Database:
         cfg.transfer_packing = 1 if transfer_packing else 0
         cfg.fault_op_mask = fault_op_mask
         cfg.max_queries = max_queries
+        cfg.prefetch = 1 if prefetch else 0
         h = ctypes.c_void_p()
         check(lib().ddq_open(ctypes.byref(cfg), ctypes.byref(h)))
         self.h = h

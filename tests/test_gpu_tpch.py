@@ -59,15 +59,24 @@ def test_tpch3_limit10():
     assert r.rows == _want("tpch3")[:10]
 
 
-def test_tpch_cold_path_gpu_only():
+@pytest.mark.parametrize("prefetch", [False, True])
+def test_tpch_cold_path_gpu_only(prefetch):
+    """Cold cache, GPU-only: columns copied on demand, or streamed from submit on the
+    copy thread while earlier operators compute (prefetch, S8(f) N1) -- also with
+    every query submitted at once (concurrent users, cached-first pulls)."""
     from paper_conf_sigmod_bressft16_b200 import Database
     from paper_conf_sigmod_bressft16_b200 import _abi as A
     from paper_conf_sigmod_bressft16_b200.tpch import load_tpch, tpch_plan
-    db = Database(cache_bytes=8 << 30, heap_bytes=4 << 30, placement=A.PLACE_GPU_ONLY)
+    db = Database(cache_bytes=8 << 30, heap_bytes=4 << 30, placement=A.PLACE_GPU_ONLY, prefetch=prefetch)
     load_tpch(db, _data(), cache=False)
     for q in ("tpch1", "tpch6", "tpch5", "tpch4", "tpch7"):
         r = db.run(tpch_plan(db, q))
         assert r.rows == _want(q) and r.host_ops == 0
+    for (t, c) in list(db._cols):
+        db.evict(t, c)
+    qs = {q: db.submit(tpch_plan(db, q)) for q in ("tpch1", "tpch2", "tpch3", "tpch4", "tpch5", "tpch6", "tpch7")}
+    for q, h in qs.items():
+        assert db.fetch(h).rows == _want(q), q
     st = db.stats()
     assert st["h2d_bytes"] > 0 and st["cache_misses"] > 0
     db.close()
