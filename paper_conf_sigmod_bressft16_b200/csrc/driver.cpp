@@ -820,7 +820,7 @@ static void finish_query(ddq_db* db, QueryState& q) {
   ddq_status s = DDQ_OK;
   if (root.kind == DDQ_OP_AGGREGATE) {
     if (r.on_host) {
-      s = finalize_result(root, r.h_groups, r.h_keys->data(), r.h_accs->data(), &res);
+      s = finalize_result(root, r.h_groups, r.h_keys->data(), r.h_accs->data(), &res, true);
     } else {
       cudaStream_t st;
       cudaSetDevice(db->device);
@@ -838,7 +838,7 @@ static void finish_query(ddq_db* db, QueryState& q) {
       cudaStreamDestroy(st);
       db->stats.d2h_bytes += 4 + (uint64_t)g * (8 + 16 * root.n_aggs);
       db->stats.d2h_ns += now_ns() - t0;
-      s = e == cudaSuccess ? finalize_result(root, g, keys.data(), accs.data(), &res) : cuda_status(e, "fetch");
+      s = e == cudaSuccess ? finalize_result(root, g, keys.data(), accs.data(), &res, true) : cuda_status(e, "fetch");
     }
   } else {
     cudaStream_t st;

@@ -796,10 +796,10 @@ static ddq_status finalize_unique(const ddq_op& root, int64_t n_groups, const in
 // SUM / COUNT kinds by exact int128 addition, MIN by taking the smaller value (the
 // merge of per-shard minima is the minimum); then finalise.
 ddq_status finalize_result(const ddq_op& root, int64_t n_groups, const int64_t* keys, const int64_t* accs,
-                           ddq_result** out) {
+                           ddq_result** out, bool unique_keys) {
   const int na = root.n_aggs;
   bool dup = false;  // one device group table has unique keys; shards' partials may repeat them
-  {
+  if (!unique_keys) {
     std::unordered_set<int64_t> seen;
     seen.reserve((size_t)n_groups * 2);
     for (int64_t i = 0; i < n_groups && !dup; i++) dup = !seen.insert(keys[i]).second;
@@ -2160,7 +2160,7 @@ ddq_status ddq_prepared_fetch(ddq_prepared* p, void* stream, ddq_result** out) {
   std::vector<int64_t> keys(r.gb_cap), accs((size_t)r.gb_cap * na * 2);
   int64_t g = 0;
   if (ddq_status s = ddq_prepared_partials(p, stream, &g, keys.data(), accs.data(), r.gb_cap)) return s;
-  ddq_status s = finalize_result(root, g, keys.data(), accs.data(), out);
+  ddq_status s = finalize_result(root, g, keys.data(), accs.data(), out, true);
   if (s == DDQ_OK) {
     (*out)->gpu_ops = p->plan.n_ops;
     decode_result_keys(p->db, p->plan, *out);

@@ -195,8 +195,10 @@ ddq_status run_gpu_op(GpuOpCtx& ctx, const ddq_op& op, Inter& out);
 ddq_status run_host_op(ddq_db* db, const ddq_op& op, const std::vector<Inter>& inters, Inter& out);
 void release_inter(ddq_db* db, Inter& x);
 ddq_status inter_to_host(ddq_db* db, Inter& x, cudaStream_t st);
+// unique_keys: the groups come from ONE group table (a prepared plan, a driver
+// query), so equal packed keys cannot occur and the merge step is skipped
 ddq_status finalize_result(const ddq_op& root, int64_t n_groups, const int64_t* keys, const int64_t* accs,
-                           ddq_result** out);
+                           ddq_result** out, bool unique_keys = false);
 // S8(a7) decode: attach the dictionary strings of the result's keys (key_str)
 void decode_result_keys(ddq_db* db, const ddq_plan& plan, ddq_result* r);
 int64_t pow2_at_least(int64_t x);
