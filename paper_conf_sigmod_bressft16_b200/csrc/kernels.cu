@@ -275,7 +275,7 @@ __global__ void gather_kernel(const void* __restrict__ col, const int32_t* __res
 // resident -- no compaction: a late-materialisation fetch after a semi-join of the
 // same build passes every row, so a probe's ring, reservation and TID copy would be
 // wasted work (opprofile SF20 Q3.1: 119 us as an emitting probe).
-constexpr int FT_PER = 4;  // items per thread (independent gathers in flight)
+constexpr int FT_PER = 8;  // items per thread (independent gathers in flight)
 __global__ void __launch_bounds__(256) fetch_kernel(const int32_t* __restrict__ tids, const uint32_t* d_count,
                                                     const int32_t* __restrict__ fk, const uint32_t* __restrict__ bitmap,
                                                     const int32_t* __restrict__ payarr, int32_t key_min, uint32_t range,
@@ -290,15 +290,32 @@ __global__ void __launch_bounds__(256) fetch_kernel(const int32_t* __restrict__ 
       const uint32_t i = i0 + u * stride;
       k[u] = i < n ? ldg_gather(fk + (uint32_t)tids[i]) : 0;
     }
+    if (bitmap) {  // join index: every item's bitmap word, then the payloads of the hits
+      // (two rounds of independent L2 loads instead of FT_PER dependent pairs: ncu
+      // showed the fetch stalled on long scoreboard 167 cycles per issue)
+      uint32_t w[FT_PER];
+#pragma unroll
+      for (int u = 0; u < FT_PER; u++) {
+        const uint32_t o = (uint32_t)(k[u] - key_min);
+        w[u] = (i0 + u * stride < n && o < range) ? __ldg(bitmap + (o >> 5)) : 0u;
+      }
+      int32_t v[FT_PER];
+#pragma unroll
+      for (int u = 0; u < FT_PER; u++) {
+        const uint32_t o = (uint32_t)(k[u] - key_min);
+        v[u] = ((w[u] >> (o & 31)) & 1u) ? __ldg(payarr + o) : INT32_MIN;
+      }
+#pragma unroll
+      for (int u = 0; u < FT_PER; u++)
+        if (i0 + u * stride < n) out[i0 + u * stride] = v[u];
+      continue;
+    }
 #pragma unroll
     for (int u = 0; u < FT_PER; u++) {
       const uint32_t i = i0 + u * stride;
       if (i >= n) continue;
       int32_t v = INT32_MIN;
-      if (bitmap) {
-        const uint32_t o = (uint32_t)(k[u] - key_min);
-        if (o < range && ((__ldg(bitmap + (o >> 5)) >> (o & 31)) & 1u)) v = __ldg(payarr + o);
-      } else {
+      {
         uint32_t h = ht_hash(k[u], shift);
         uint64_t sl = __ldg(table + h);
         while (sl != HT_EMPTY && ht_key(sl) != k[u]) {
