@@ -583,6 +583,26 @@ ddq_status ddq_table_set_partitioned(ddq_db* db, ddq_table t, int32_t partitione
 ddq_status ddq_dist_exchange(ddq_db* db, ddq_prepared* const* plans, int32_t n, void* stream);
 ddq_status ddq_dist_result(ddq_db* db, int32_t i, ddq_result** out);
 
+/* ---- multi-GPU data-driven placement (Sec. 6.3) ---------
+ * A cluster is one database per GPU (ddq_cluster_open: cfg copied, device taken from
+ * devices[i]); the caller loads the SAME tables and columns, in the same order, into
+ * every member (ddq_cluster_db), so column ids agree.  Each member's cache is filled by
+ * Algorithm 1 over the access counts of the queries it ran (ddq_cluster_update_
+ * placement runs ddq_update_placement on every member).  ddq_cluster_submit is
+ * data-driven placement of the query: the member whose cache holds the most of the
+ * plan's input bytes (ties: fewest queries in flight, then round robin); inside the
+ * member every operator is placed as in ddq_submit.  *member receives the member;
+ * fetch with ddq_cluster_fetch(member, query).  A single process drives all members
+ * (devices may repeat: several members on one GPU are valid, e.g. for tests). */
+typedef struct ddq_cluster ddq_cluster;
+ddq_status ddq_cluster_open(const ddq_config* cfg, const int32_t* devices, int32_t n, ddq_cluster** out);
+void ddq_cluster_close(ddq_cluster* c);
+int32_t ddq_cluster_size(ddq_cluster* c);
+ddq_db* ddq_cluster_db(ddq_cluster* c, int32_t i);
+ddq_status ddq_cluster_submit(ddq_cluster* c, const ddq_plan* plan, int32_t* member, ddq_query* out);
+ddq_status ddq_cluster_fetch(ddq_cluster* c, int32_t member, ddq_query q, ddq_result** out);
+ddq_status ddq_cluster_update_placement(ddq_cluster* c);
+
 /* ---- statistics (paper's counters, D10: P:330) ---- */
 typedef struct {
   uint64_t h2d_bytes, d2h_bytes;

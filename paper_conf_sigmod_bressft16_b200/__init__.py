@@ -5,6 +5,6 @@ behind the C ABI of include/ddq.h, driven by the paper's data-driven placement a
 query chopping.  This package is argument marshalling over libddq.so only.
 """
 from ._abi import DDQError, lib  # noqa: F401
-from .engine import Database, PlanBuilder, Prepared, QueryResult  # noqa: F401
+from .engine import Cluster, Database, PlanBuilder, Prepared, QueryResult  # noqa: F401
 
-__all__ = ["Database", "PlanBuilder", "Prepared", "QueryResult", "DDQError", "lib"]
+__all__ = ["Cluster", "Database", "PlanBuilder", "Prepared", "QueryResult", "DDQError", "lib"]

@@ -173,6 +173,13 @@ SIGNATURES = {
     "ddq_table_set_partitioned": (_i32, [_vp, _i32, _i32]),
     "ddq_dist_exchange": (_i32, [_vp, ctypes.POINTER(_vp), _i32, _vp]),
     "ddq_dist_result": (_i32, [_vp, _i32, ctypes.POINTER(ctypes.POINTER(Result))]),
+    "ddq_cluster_open": (_i32, [ctypes.POINTER(Config), ctypes.POINTER(_i32), _i32, ctypes.POINTER(_vp)]),
+    "ddq_cluster_close": (None, [_vp]),
+    "ddq_cluster_size": (_i32, [_vp]),
+    "ddq_cluster_db": (_vp, [_vp, _i32]),
+    "ddq_cluster_submit": (_i32, [_vp, ctypes.POINTER(Plan), ctypes.POINTER(_i32), ctypes.POINTER(_i64)]),
+    "ddq_cluster_fetch": (_i32, [_vp, _i32, _i64, ctypes.POINTER(ctypes.POINTER(Result))]),
+    "ddq_cluster_update_placement": (_i32, [_vp]),
     "ddq_get_stats": (_i32, [_vp, ctypes.POINTER(Stats)]),
     "ddq_reset_stats": (_i32, [_vp]),
     "ddq_heap_try_alloc": (_vp, [_vp, _u64]),

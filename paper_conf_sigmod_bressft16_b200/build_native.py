@@ -9,7 +9,7 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 CSRC = os.path.join(HERE, "csrc")
 SO = os.path.join(HERE, "libddq.so")
 SOURCES = ["transfer.cu", "filter.cu", "dense.cu", "agg.cu", "scan.cu", "star.cu", "kernels.cu", "ops.cu", "engine.cpp",
-           "driver.cpp", "dist.cpp"]
+           "driver.cpp", "dist.cpp", "cluster.cpp"]
 HEADERS = ["device_common.cuh", "ops_internal.h", "engine.h"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]

@@ -377,7 +377,7 @@ class Database:
                  gpu_workers: int = 4, host_workers: int = 4, placement: int = A.PLACE_DATA_DRIVEN,
                  chopping: bool = True, cache_policy: int = 0, fault_alloc_every: int = 0,
                  rank: int = 0, world: int = 1, transfer_packing: bool = True, fault_op_mask: int = 0,
-                 max_queries: int = 0, prefetch: bool = False):
+                 max_queries: int = 0, prefetch: bool = False, _handle: int | None = None):
         cfg = A.Config()
         lib().ddq_config_default(ctypes.byref(cfg))
         cfg.device, cfg.rank, cfg.world = device, rank, world
@@ -389,8 +389,12 @@ class Database:
         cfg.fault_op_mask = fault_op_mask
         cfg.max_queries = max_queries
         cfg.prefetch = 1 if prefetch else 0
-        h = ctypes.c_void_p()
-        check(lib().ddq_open(ctypes.byref(cfg), ctypes.byref(h)))
+        self._owner = _handle is None
+        if _handle is None:
+            h = ctypes.c_void_p()
+            check(lib().ddq_open(ctypes.byref(cfg), ctypes.byref(h)))
+        else:  # a member of a Cluster (owned by the cluster)
+            h = ctypes.c_void_p(_handle)
         self.h = h
         self._tables: dict[str, int] = {}
         self._rows: dict[str, int] = {}
@@ -403,7 +407,8 @@ class Database:
         if self.h:
             for p in list(self._prepared):  # prepared plans hold cache references and heap blocks
                 p.close()
-            lib().ddq_close(self.h)
+            if self._owner:
+                lib().ddq_close(self.h)
             self.h = None
 
     def __del__(self):
@@ -562,3 +567,47 @@ class Database:
 
     def reset_stats(self) -> None:
         check(lib().ddq_reset_stats(self.h))
+
+
+class Cluster:
+    """Multi-GPU data-driven placement (include/ddq.h "cluster"): one
+    database per device; load the same tables into every member (`members`), then
+    submit: each query goes to the member whose cache holds most of its input bytes."""
+
+    def __init__(self, devices: list[int], **kw):
+        cfg = A.Config()
+        lib().ddq_config_default(ctypes.byref(cfg))
+        for k, v in {"cache_bytes": 64 << 30, "heap_bytes": 32 << 30, **kw}.items():
+            setattr(cfg, k, int(v))
+        devs = (ctypes.c_int32 * len(devices))(*devices)
+        h = ctypes.c_void_p()
+        check(lib().ddq_cluster_open(ctypes.byref(cfg), devs, len(devices), ctypes.byref(h)))
+        self.h = h
+        self.members = [Database(_handle=lib().ddq_cluster_db(h, i)) for i in range(len(devices))]
+
+    def submit(self, plan) -> tuple[int, int]:
+        p = plan.plan if isinstance(plan, PlanBuilder) else plan
+        m, q = ctypes.c_int32(), ctypes.c_int64()
+        check(lib().ddq_cluster_submit(self.h, ctypes.byref(p), ctypes.byref(m), ctypes.byref(q)))
+        return m.value, q.value
+
+    def fetch(self, member: int, q: int) -> QueryResult:
+        p = ctypes.POINTER(A.Result)()
+        check(lib().ddq_cluster_fetch(self.h, member, q, ctypes.byref(p)))
+        return _convert(p)
+
+    def update_placement(self) -> None:
+        check(lib().ddq_cluster_update_placement(self.h))
+
+    def close(self) -> None:
+        if self.h:
+            for m in self.members:
+                m.close()
+            lib().ddq_cluster_close(self.h)
+            self.h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
