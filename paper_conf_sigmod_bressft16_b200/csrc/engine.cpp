@@ -1114,25 +1114,46 @@ ddq_status ddq_load_column(ddq_db* db, ddq_table t, const char* name, ddq_type t
     if (i == 0 || v < c->vmin) c->vmin = v;
     if (i == 0 || v > c->vmax) c->vmax = v;
   }
-  // transfer encoding: value - vmin in the fewest whole bytes (<= 4, < width)
+  // transfer encoding: value - vmin in the bit length of the range (1..32 bits, fewer
+  // than the column's width), a little-endian bit stream (transfer.cu)
   if (db->cfg.transfer_packing && n_rows > 0) {
     const uint64_t range = (uint64_t)c->vmax - (uint64_t)c->vmin;
-    int tw = range < (1ull << 8) ? 1 : range < (1ull << 16) ? 2 : range < (1ull << 24) ? 3 : range < (1ull << 32) ? 4 : 0;
-    if (tw && tw < c->width &&
-        cudaHostAlloc(&c->host_packed, packed_bytes(n_rows, tw), cudaHostAllocPortable) == cudaSuccess) {
-      uint8_t* dst = (uint8_t*)c->host_packed;
-      std::memset(dst + (size_t)n_rows * tw, 0, packed_bytes(n_rows, tw) - (size_t)n_rows * tw);
-      for (int64_t i = 0; i < n_rows; i++) {
-        const int64_t v = c->width == 4 ? ((const int32_t*)host_data)[i] : ((const int64_t*)host_data)[i];
-        const uint32_t d = (uint32_t)((uint64_t)v - (uint64_t)c->vmin);
-        switch (tw) {
-          case 1: dst[i] = (uint8_t)d; break;
-          case 2: ((uint16_t*)dst)[i] = (uint16_t)d; break;
-          case 4: ((uint32_t*)dst)[i] = d; break;
-          default: std::memcpy(dst + (size_t)i * 3, &d, 3); break;  // little endian
+    int bits = 1;
+    while (bits < 64 && (range >> bits) != 0) bits++;
+    if (bits <= 32 && bits < 8 * c->width &&
+        cudaHostAlloc(&c->host_packed, packed_bytes(n_rows, bits), cudaHostAllocPortable) == cudaSuccess) {
+      uint32_t* dst = (uint32_t*)c->host_packed;
+      std::memset(dst, 0, packed_bytes(n_rows, bits));
+      // 32 values fill exactly `bits` words, so chunks of 32k values pack in parallel
+      const int64_t per = 32 * 65536;
+      const int64_t chunks = (n_rows + per - 1) / per;
+      const int nt = (int)std::max<int64_t>(1, std::min<int64_t>(chunks, std::thread::hardware_concurrency()));
+      const int64_t vmin = c->vmin;
+      const int width = c->width;
+      auto pack = [&](int t) {
+        for (int64_t ch = t; ch < chunks; ch += nt) {
+          const int64_t b = ch * per, e = std::min<int64_t>(n_rows, b + per);
+          uint64_t acc = 0;  // bits not yet flushed, low first
+          int have = 0;
+          size_t w = (size_t)(b / 32) * (size_t)bits;
+          for (int64_t i = b; i < e; i++) {
+            const int64_t v = width == 4 ? ((const int32_t*)host_data)[i] : ((const int64_t*)host_data)[i];
+            acc |= ((uint64_t)v - (uint64_t)vmin) << have;
+            have += bits;
+            if (have >= 32) {
+              dst[w++] = (uint32_t)acc;
+              acc >>= 32;
+              have -= 32;
+            }
+          }
+          if (have > 0) dst[w] = (uint32_t)acc;
         }
-      }
-      c->tw = tw;
+      };
+      std::vector<std::thread> th;
+      for (int t = 1; t < nt; t++) th.emplace_back(pack, t);
+      pack(0);
+      for (auto& x : th) x.join();
+      c->tw = bits;
     }
   }
   db->cols.push_back(std::move(c));

@@ -52,8 +52,8 @@ struct Column {
   int64_t n = 0;
   int64_t vmin = 0, vmax = -1;  // value range (computed at load; sizes join indexes)
   void* host = nullptr;   // pinned host copy
-  void* host_packed = nullptr;  // frame-of-reference byte-packed pinned copy (transfer.cu)
-  int tw = 0;                   // its bytes per value (1..4); 0 = none, the raw copy is sent
+  void* host_packed = nullptr;  // frame-of-reference bit-packed pinned copy (transfer.cu)
+  int tw = 0;                   // its bits per value (1..32); 0 = none, the raw copy is sent
   void* dev = nullptr;    // device cache copy or nullptr
   std::atomic<uint64_t> access{0};
   std::atomic<uint64_t> last_access{0};

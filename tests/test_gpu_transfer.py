@@ -1,7 +1,8 @@
 """Cold-path transfer encoding (transfer.cu): a column cached
-from its frame-of-reference byte-packed pinned copy is bit-identical to the raw
-column, for every packed width (1..4 bytes), negative bases, widths 4 and 8,
-ragged lengths, and columns that stay raw (range >= 2^32)."""
+from its frame-of-reference bit-packed pinned copy is bit-identical to the raw
+column, for bit lengths 1..32 (every byte boundary and odd lengths), negative bases,
+widths 4 and 8, ragged lengths, and columns that stay raw (range >= 2^32); the bytes
+sent are the packed stream's."""
 import numpy as np
 import pytest
 
@@ -32,9 +33,10 @@ def _roundtrip(values: np.ndarray, packing: bool = True):
 
 @pytest.mark.parametrize("n", [1, 2, 3, 4, 5, 7, 8, 9, 1023, 4097, 1_000_003])
 @pytest.mark.parametrize("span,base,dtype", [
-    (1, 0, np.int32), (255, -7, np.int32), (256, 19920101, np.int32), (65535, -(1 << 31), np.int32),
-    (65536, 5, np.int64), ((1 << 24) - 1, -3, np.int64), (1 << 24, 1 << 40, np.int64),
-    ((1 << 32) - 1, -(1 << 62), np.int64), (1 << 32, 0, np.int64)])
+    (1, 0, np.int32), (10, 0, np.int32), (49, 1, np.int64), (255, -7, np.int32), (256, 19920101, np.int32),
+    (60701, 19920101, np.int32), (65535, -(1 << 31), np.int32), (65536, 5, np.int64),
+    (599_999, 1, np.int32), ((1 << 24) - 1, -3, np.int64), (1 << 24, 1 << 40, np.int64),
+    ((1 << 31) + 12345, 7, np.int64), ((1 << 32) - 1, -(1 << 62), np.int64), (1 << 32, 0, np.int64)])
 def test_packed_cache_roundtrip(n, span, base, dtype):
     rng = np.random.default_rng(n * 7919 + span)
     v = (base + rng.integers(0, span + 1, size=n, dtype=np.int64)).astype(dtype)
@@ -43,9 +45,9 @@ def test_packed_cache_roundtrip(n, span, base, dtype):
     got, moved = _roundtrip(v)
     assert got.dtype == v.dtype and np.array_equal(got, v)
     width = v.dtype.itemsize
-    tw = next((b for b in (1, 2, 3, 4) if int(v.max()) - int(v.min()) < (1 << (8 * b))), None)
-    if tw is not None and tw < width:
-        assert moved < n * width or n < 16  # packed bytes (+ padding) went over the link
+    bits = max(1, (int(v.max()) - int(v.min())).bit_length())
+    if bits <= 32 and bits < 8 * width:  # the packed stream (+ <= 63 bytes of padding) went over the link
+        assert moved == (n * bits + 7) // 8 // 16 * 16 + 48
     else:
         assert moved == n * width
 
