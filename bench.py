@@ -13,9 +13,10 @@ N > 1 (torchrun): lineorder is range-sharded by row (P:407 horizontal partitioni
 weak scaling by default (SF 20*N, 120 M rows per rank), strong scaling with
 --sf-total 100 (S8(d) M3: 600 M rows split over the ranks).  libddq owns the
 multi-GPU path (include/ddq.h "multi-GPU"): an NCCL communicator per database
-(unique id bootstrapped through torch.distributed), dimension indexes built once on
-rank 0 and broadcast inside each plan's CUDA graph, and per step one ncclAllGather of
-the 13 packed partial group tables, merged exactly by ddq_dist_result on rank 0.
+(unique id bootstrapped through torch.distributed), per step one ncclAllGather of the
+13 packed partial group tables, merged exactly by ddq_dist_result on rank 0; with
+--build-once the dimension indexes are built on rank 0 and broadcast inside each
+plan's CUDA graph (then one query stream: NCCL needs one collective order).
 
 --impl reference: the oracle (oracle/, single-threaded C++) on a bounded sample
 of the same workload, on the host's cores.
@@ -47,8 +48,9 @@ def parse():
     ap.add_argument("--sf", type=float, default=SF_PER_GPU, help="scale factor per GPU (weak scaling)")
     ap.add_argument("--sf-total", type=float, default=0,
                     help="strong scaling (S8(d) M3): one database of this SF, lineorder row-sharded over the ranks")
-    ap.add_argument("--no-build-once", action="store_true",
-                    help="N>1: every rank builds its dimension indexes (default: rank 0 builds, NCCL broadcasts)")
+    ap.add_argument("--build-once", action="store_true",
+                    help="N>1: rank 0 builds the dimension indexes and NCCL broadcasts them inside the plan "
+                         "graphs (one collective order: forces 1 query stream); default: every rank builds")
     ap.add_argument("--e2e-steps", type=int, default=5)
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-prefetch", action="store_true", help="e2e: copy columns on demand instead of streaming")
@@ -300,7 +302,7 @@ def main():
             from paper_conf_sigmod_bressft16_b200.engine import nccl_unique_id
             box = [nccl_unique_id() if rank == 0 else None]
             dist.broadcast_object_list(box, src=0)
-            db.dist_init_nccl(box[0], rank, ws, build_once=not args.no_build_once)
+            db.dist_init_nccl(box[0], rank, ws, build_once=args.build_once)
         else:  # test hook: a host all-gather over the gloo process group
             def host_allgather(buf: bytes) -> bytes:
                 t = torch.frombuffer(bytearray(buf), dtype=torch.uint8)
@@ -321,6 +323,14 @@ def main():
     all_side = [torch.cuda.Stream() for _ in range(max(args.streams, 4) - 1)]
     side = all_side[:max(args.streams, 1) - 1]
 
+    # the 13 plans are dealt round robin over the K streams in query order, which pairs
+    # heavy and light plans on each stream (tried: longest-processing-time-first dealing
+    # balanced the streams' solo times but started the four heaviest plans together and
+    # measured slower, 2.66 -> 2.70 ms)
+    def deal(k: int) -> list:
+        return [i % k for i in range(len(preps))]
+    lane_of = deal(1)
+
     def step(serial: bool = False):
         if serial or not side:
             for p in preps:
@@ -330,7 +340,7 @@ def main():
         for s2 in side:
             s2.wait_stream(stream)
         for i, p in enumerate(preps):
-            p.launch(lanes[i % len(lanes)].cuda_stream)
+            p.launch(lanes[lane_of[i]].cuda_stream)
         for s2 in side:
             stream.wait_stream(s2)
 
@@ -340,6 +350,7 @@ def main():
         trial = {}
         for k in (1, 2, 4):
             side = all_side[:k - 1]
+            lane_of = deal(k)
             step()
             ta, tb = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             torch.cuda.synchronize()
@@ -355,7 +366,10 @@ def main():
             dist.all_reduce(t, op=dist.ReduceOp.MAX)
             trial = dict(zip((1, 2, 4), t.tolist()))
         args.streams = min(trial, key=trial.get)
-        side = all_side[:args.streams - 1]
+    if args.build_once and ws > 1:  # NCCL broadcasts inside the graphs: one collective order
+        args.streams = 1
+    side = all_side[:max(args.streams, 1) - 1]
+    lane_of = deal(max(args.streams, 1))
 
     # N>1: after the 13 launches, libddq packs the compacted partial group tables on the
     # device and all-gathers them (ncclAllGather over NVLink; the gloo test hook: a host
@@ -514,7 +528,7 @@ def main():
                 "config": {"workload": f"SSB SF{sf_total:g}, all 13 queries, hot cache " +
                                        ("(BASELINE configs[2]: lineorder row-sharded)" if ws > 1 else
                                         "(BASELINE configs[1])"),
-                           "build_once": ws > 1 and backend == "nccl" and not args.no_build_once,
+                           "build_once": ws > 1 and backend == "nccl" and args.build_once,
                            "lineorder_rows": n_lo, "rows_per_gpu": shard_rows, "queries": 13,
                            "parallelism": f"row-sharded x{ws}" if ws > 1 else "1 GPU",
                            "query_streams": max(args.streams, 1),
