@@ -525,9 +525,9 @@ def main():
                 "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
                 "scaling": "strong" if strong else "weak", "vs_baseline": None, "dtype": "int64",
                 "data": "synthetic (datagen, seed 0x5EED2016)",
-                "config": {"workload": f"SSB SF{sf_total:g}, all 13 queries, hot cache " +
-                                       ("(BASELINE configs[2]: lineorder row-sharded)" if ws > 1 else
-                                        "(BASELINE configs[1])"),
+                "config": {"workload": f"SSB SF{sf_total:g}, all 13 queries, hot cache" +
+                                       (" (BASELINE configs[2]: lineorder row-sharded)" if ws > 1 else
+                                        " (BASELINE configs[1])" if sf_total == 20 else ""),
                            "build_once": ws > 1 and backend == "nccl" and args.build_once,
                            "lineorder_rows": n_lo, "rows_per_gpu": shard_rows, "queries": 13,
                            "parallelism": f"row-sharded x{ws}" if ws > 1 else "1 GPU",
