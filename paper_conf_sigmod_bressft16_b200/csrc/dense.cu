@@ -31,6 +31,7 @@
 //     reservation: the output has no holes.
 // Output order: unspecified (reading O14': a TID list is a multiset; every consumer
 // is order-free); each input item is emitted at most once.
+#include <algorithm>
 #include <cstdint>
 #include <cstdlib>
 #include <cuda_runtime.h>
@@ -742,7 +743,13 @@ cudaError_t launch_ws(const FilterArgs& a, cudaStream_t st) {
   // live: 16 blocks made the date probe's d_year lookups miss (74 -> 141 us) and
   // 8 blocks slowed the late fetch itself (119 -> 195 us)
   const size_t tab_smem = (kind == WK_BM_SMEM || kind == WK_HT_SMEM || kind == WK_BM_COARSE) ? tab : 0;
-  const int logr = 2;
+  int logr = 2;
+  // (Tried: 8-16 blocks for a dense semi-join probe with a dense known output --
+  // ncu, SSB Q3.1 at 20 % survivors: 3.6 M spin loads on busy blocks next to 3.75 M
+  // bitmap lookups.  Q3.1 / Q4.2's probes 147 / 151 -> 137 / 137 us alone, but the
+  // 4-stream step 2.67 -> 3.03 ms: a 200 KB CTA leaves no room for the other
+  // streams' kernels on its SM.)  DDQ_WS_RING_LOGR: A/B override.
+  if (const char* e = getenv("DDQ_WS_RING_LOGR")) logr = std::max(2, std::min(4, atoi(e)));
   const size_t ring = obits ? 0 : ring1 << logr;
   p.ring_logr = logr;
   p.tab_off = (int32_t)ring;
