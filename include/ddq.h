@@ -249,7 +249,9 @@ typedef enum {
 
 typedef struct {
   int32_t device;                /* CUDA device ordinal (one process per GPU) */
-  int32_t rank, world;           /* for row-sharded multi-GPU runs */
+  int32_t rank, world;           /* this process's rank / the ranks of a row-sharded multi-GPU run
+                                    (P:407); informational until ddq_dist_init_nccl / _host,
+                                    which set them and create the exchange (multi-GPU, below) */
   uint64_t cache_bytes;          /* device column cache budget */
   uint64_t heap_bytes;           /* device heap for intermediates */
   int32_t gpu_workers;           /* chopping bound: GPU worker threads, O17 */
@@ -272,6 +274,10 @@ typedef struct {
                                     ready operators whose columns are resident first (cached-first
                                     schedule).  0 (default): columns are copied when an operator
                                     needs them (the paper's operator-driven placement) */
+  int32_t placement_period_ms;   /* > 0: a background job runs Algorithm 1 (ddq_update_placement)
+                                    every this many ms while the database is open -- the paper's
+                                    periodic data placement; 0 (default): only when
+                                    the caller invokes ddq_update_placement */
   int32_t max_queries;           /* query-level admission control (the comparison arm of P:371,
                                     P:445, Wang et al.): at most this many submitted queries run at
                                     once, later ones wait in submission order until one finishes;

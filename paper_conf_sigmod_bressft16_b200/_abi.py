@@ -45,7 +45,8 @@ class Config(ctypes.Structure):
                 ("gpu_workers", ctypes.c_int32), ("host_workers", ctypes.c_int32),
                 ("placement", ctypes.c_int32), ("chopping", ctypes.c_int32),
                 ("cache_policy", ctypes.c_int32), ("fault_alloc_every", ctypes.c_uint32),
-                ("transfer_packing", ctypes.c_int32), ("prefetch", ctypes.c_int32), ("max_queries", ctypes.c_int32),
+                ("transfer_packing", ctypes.c_int32), ("prefetch", ctypes.c_int32),
+                ("placement_period_ms", ctypes.c_int32), ("max_queries", ctypes.c_int32),
                 ("fault_op_mask", ctypes.c_uint32)]
 
 

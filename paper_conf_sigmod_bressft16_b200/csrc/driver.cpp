@@ -1072,6 +1072,21 @@ static void prefetch_loop(ddq_db* db) {
   }
 }
 
+// The paper's background data-placement job: Algorithm 1 every
+// placement_period_ms; running queries keep going (evictions are deferred while
+// referenced).
+static void placement_loop(ddq_db* db) {
+  cudaSetDevice(db->device);
+  std::unique_lock<std::mutex> g(db->qmu);
+  while (!db->stopping) {
+    db->qcv.wait_for(g, std::chrono::milliseconds(db->cfg.placement_period_ms), [&] { return db->stopping; });
+    if (db->stopping) break;
+    g.unlock();
+    (void)ddq_update_placement(db);
+    g.lock();
+  }
+}
+
 // every input column of op resident on the GPU (the cached-first pull order)
 static bool op_resident(ddq_db* db, const ddq_op& op) {
   std::lock_guard<std::mutex> g(db->mu);
@@ -1136,6 +1151,7 @@ void driver_start(ddq_db* db) {
   for (int i = 0; i < g; i++) db->workers.emplace_back(worker_loop, db, true);
   for (int i = 0; i < h; i++) db->workers.emplace_back(worker_loop, db, false);
   if (db->cfg.prefetch && db->cfg.placement != DDQ_PLACE_CPU_ONLY) db->prefetcher = std::thread(prefetch_loop, db);
+  if (db->cfg.placement_period_ms > 0) db->placer = std::thread(placement_loop, db);
 }
 
 void driver_stop(ddq_db* db) {
@@ -1147,6 +1163,7 @@ void driver_stop(ddq_db* db) {
   for (auto& t : db->workers) t.join();
   db->workers.clear();
   if (db->prefetcher.joinable()) db->prefetcher.join();
+  if (db->placer.joinable()) db->placer.join();
   for (auto& kv : db->queries) {
     for (auto& x : kv.second->inters) release_inter(db, x);
     if (kv.second->result) ddq_result_free(kv.second->result);

@@ -160,6 +160,7 @@ struct ddq_db {
   // streamed cold path (ddq_config.prefetch): columns queued for H2D (qmu), copy thread
   std::deque<int> prefetch_queue;
   std::thread prefetcher;
+  std::thread placer;  // periodic Algorithm 1 (ddq_config.placement_period_ms)
   void* dist = nullptr;  // multi-GPU state (dist.cpp), or null
 };
 

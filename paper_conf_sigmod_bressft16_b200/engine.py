@@ -377,7 +377,8 @@ class Database:
                  gpu_workers: int = 4, host_workers: int = 4, placement: int = A.PLACE_DATA_DRIVEN,
                  chopping: bool = True, cache_policy: int = 0, fault_alloc_every: int = 0,
                  rank: int = 0, world: int = 1, transfer_packing: bool = True, fault_op_mask: int = 0,
-                 max_queries: int = 0, prefetch: bool = False, _handle: int | None = None):
+                 max_queries: int = 0, prefetch: bool = False, placement_period_ms: int = 0,
+                 _handle: int | None = None):
         cfg = A.Config()
         lib().ddq_config_default(ctypes.byref(cfg))
         cfg.device, cfg.rank, cfg.world = device, rank, world
@@ -389,6 +390,7 @@ class Database:
         cfg.fault_op_mask = fault_op_mask
         cfg.max_queries = max_queries
         cfg.prefetch = 1 if prefetch else 0
+        cfg.placement_period_ms = placement_period_ms
         self._owner = _handle is None
         if _handle is None:
             h = ctypes.c_void_p()

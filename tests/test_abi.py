@@ -48,6 +48,7 @@ int main(void) {
   O(ddq_dev_pred, in_vals) O(ddq_dev_agg, arg) O(ddq_op, eq_cmp) O(ddq_op, build_key_set)
   O(ddq_op, n_avg) O(ddq_op, avg_scale) O(ddq_result, agg_null) O(ddq_result, avgs) O(ddq_result, key_str)
   O(ddq_op, gather_narrow) O(ddq_result, op_place) O(ddq_config, fault_op_mask) O(ddq_result, op_ms) O(ddq_config, prefetch)
+  O(ddq_config, placement_period_ms) O(ddq_config, max_queries)
   printf("DDQ_CMP_EQ %d\nDDQ_CMP_LT %d\nDDQ_CMP_NE %d\nDDQ_AGG_MIN %d\nDDQ_AGG_COUNT %d\n",
          DDQ_CMP_EQ, DDQ_CMP_LT, DDQ_CMP_NE, (int)DDQ_AGG_MIN, (int)DDQ_AGG_COUNT);
   printf("DDQ_PRED_BITSET %d\n", (int)DDQ_PRED_BITSET);

@@ -288,3 +288,23 @@ def test_admission_control_runs_queries_one_at_a_time():
     ms = [r.exec_ms for r in res]  # submit -> done: FIFO service makes it increase
     assert ms == sorted(ms)
     db.close()
+
+
+def test_periodic_placement_job():
+    """placement_period_ms: the background job runs Algorithm 1 periodically:
+    columns the workload touched become resident without a call, and the next run of
+    the same query is placed on the GPU (data-driven)."""
+    import time
+    from paper_conf_sigmod_bressft16_b200 import _abi as A
+    db = _db(1 << 30, placement_period_ms=20)
+    P = db.plan()
+    P.select("t2", [("c", 0, 49)])
+    r = db.run(P)
+    assert r.placement == [A.RAN_HOST]  # nothing cached yet
+    deadline = time.time() + 5
+    while not db.is_cached("t2", "c") and time.time() < deadline:
+        time.sleep(0.02)
+    assert db.is_cached("t2", "c")
+    r = db.run(P)
+    assert r.placement == [A.RAN_GPU] and np.array_equal(r.tids, np.flatnonzero(db_col(db, 2) <= 49))
+    db.close()
