@@ -120,3 +120,41 @@ def test_order_limit_with_ties():
     keys = np.array([9, 2, 7, 4], np.int64)
     r = finalize_partials(root, keys, _accs([[5], [8], [8], [1]]))
     assert r.rows == [(2, 8), (7, 8)]
+
+
+def test_merge_is_partition_invariant():
+    """Property (S8(e): sharding never changes results): for random groups split into
+    random shards, merging the shards' partial tables equals finalising the unsplit
+    table -- SUM / COUNT by exact int128 addition, MIN by minimum, any key order."""
+    from hypothesis import given, settings, strategies as st
+    from paper_conf_sigmod_bressft16_b200 import _abi as A
+    from paper_conf_sigmod_bressft16_b200.engine import finalize_partials
+
+    root = _root([A.AGG_SUM, A.AGG_MIN, A.AGG_COUNT], n_keys=2, key_bits=[5, 6], order_by=[-101, 1, 2])
+    big = st.integers(-(1 << 100), 1 << 100)
+
+    @settings(max_examples=60, deadline=None)
+    @given(st.lists(st.tuples(st.integers(0, 31), st.integers(0, 63), big, st.integers(-(1 << 62), 1 << 62)),
+                    min_size=0, max_size=40),
+           st.integers(1, 5), st.randoms())
+    def check(rows, shards, rnd):
+        exact = {}
+        for k0, k1, v, m in rows:
+            s, mn, c = exact.get((k0, k1), (0, None, 0))
+            exact[(k0, k1)] = (s + v, m if mn is None else min(mn, m), c + 1)
+        # the reference result: one row per group, ORDER BY SUM desc, keys asc
+        want = sorted(((k0, k1, s, mn, c) for (k0, k1), (s, mn, c) in exact.items()),
+                      key=lambda r: (-r[2], r[0], r[1]))
+        # split every group's rows over random shards, each shard a partial table
+        parts = {}
+        for k0, k1, v, m in rows:
+            sh = rnd.randrange(shards)
+            s, mn, c = parts.get((sh, k0, k1), (0, None, 0))
+            parts[(sh, k0, k1)] = (s + v, m if mn is None else min(mn, m), c + 1)
+        items = list(parts.items())
+        rnd.shuffle(items)
+        keys = np.array([k0 | (k1 << 5) for (_, k0, k1), _ in items], np.int64)
+        accs = _accs([[s, mn, c] for _, (s, mn, c) in items]) if items else np.zeros(0, np.int64)
+        got = finalize_partials(root, keys, accs).rows
+        assert got == want
+    check()
