@@ -1851,10 +1851,11 @@ ddq_status ddq_prepare(ddq_db* db, const ddq_plan* plan, int32_t use_graph, ddq_
         const ddq_op& c = plan->ops[j];
         if (c.input != i) continue;
         consumers++;
-        // semi-join consumers only: a consumer that emits payloads does the full
-        // probe + compaction work for every row (opprofile SF20: Q3.1's s_nation
-        // probe 105 us over a TID list, 155 us over a bitmap)
-        ok = ok && c.kind == DDQ_OP_HASH_PROBE && c.fk_vec <= 0 && !c.emit_payload;
+        // consumers that emit payloads too: over the bitmap they do the probe work for
+        // every row (opprofile SF20: Q3.1's s_nation probe 109 -> 160 us), but the
+        // producer no longer compacts 24 M TIDs through its ring (152 -> 84 us), and the
+        // 4-stream step drops 2.67 -> 2.60 ms (Q3.1, Q4.2)
+        ok = ok && c.kind == DDQ_OP_HASH_PROBE && c.fk_vec <= 0;
       }
       const int64_t rows = db->tables[(size_t)op.table].n_rows;
       const bool dense_enough = counts[(size_t)i] >= 0 && counts[(size_t)i] * 8 >= rows;

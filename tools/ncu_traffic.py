@@ -2,7 +2,11 @@
 command (ncu --metrics dram__bytes_read.sum,dram__bytes_write.sum,gpu__time_duration.sum
 --csv --log-file X python bench.py --profile-only).
 
-usage: python tools/ncu_traffic.py LAUNCHES.csv [OUT.json]
+usage: python tools/ncu_traffic.py LAUNCHES.csv [OUT.json [MODEL.json]]
+MODEL.json (tools/opprofile.py --json): the S8(d) algorithmic bytes per launch of each
+class; with it every class also gets algorithmic_bytes_per_launch and
+dram_over_algorithmic (> 1: bytes the model does not count -- 64-byte DRAM granules of
+random gathers, L2 write-backs; < 1: reuse through L2).
 Writes {class: {"launches", "dram_bytes_per_launch", "us_per_launch", "share"}}; bench.py
 reads profiles/r1_traffic.json to fill roofline.traffic for its dominant class.
 Classes follow bench.py / ddq_prepared_profile: dense (ws_kernel, every row),
@@ -29,7 +33,7 @@ def klass(name: str) -> str:
     return "other"
 
 
-def main(path: str, out: str | None):
+def main(path: str, out: str | None, model: str | None = None):
     rows = list(csv.reader(open(path)))
     h = None
     per = {}
@@ -57,10 +61,17 @@ def main(path: str, out: str | None):
     res = {c: {"launches": x["launches"], "dram_bytes_per_launch": round(x["bytes"] / x["launches"]),
                "us_per_launch": round(x["us"] / x["launches"], 2), "share": round(x["us"] / tot, 3)}
            for c, x in sorted(cls.items(), key=lambda t: -t[1]["us"])}
+    if model:
+        mc = json.load(open(model))["per_step"]
+        for c, x in res.items():
+            if c in mc:
+                alg = mc[c]["algorithmic_bytes_per_launch"]
+                x["algorithmic_bytes_per_launch"] = alg
+                x["dram_over_algorithmic"] = round(x["dram_bytes_per_launch"] / alg, 3) if alg else None
     print(json.dumps(res, indent=1))
     if out:
-        json.dump({"source": path, "classes": res}, open(out, "w"), indent=1)
+        json.dump({"source": path, "model": model, "classes": res}, open(out, "w"), indent=1)
 
 
 if __name__ == "__main__":
-    main(sys.argv[1], sys.argv[2] if len(sys.argv) > 2 else None)
+    main(sys.argv[1], sys.argv[2] if len(sys.argv) > 2 else None, sys.argv[3] if len(sys.argv) > 3 else None)

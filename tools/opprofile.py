@@ -1,7 +1,9 @@
 """Per-operator profile of the 13 SSB plans (event-timed replay + byte model).
 
-usage: python tools/opprofile.py [--sf 20] [--queries ssb1.1,ssb3.1] [--launch N]
+usage: python tools/opprofile.py [--sf 20] [--queries ssb1.1,ssb3.1] [--launch N] [--json OUT]
   --launch N: only launch each prepared plan N times (for ncu), no table.
+  --json OUT: also write per-class launches / algorithmic bytes per launch / event
+  time per launch (tools/ncu_traffic.py joins it with the ncu DRAM bytes).
 """
 import argparse
 import os
@@ -15,6 +17,7 @@ def main():
     ap.add_argument("--sf", type=float, default=20)
     ap.add_argument("--queries", default="")
     ap.add_argument("--launch", type=int, default=0)
+    ap.add_argument("--json", default="")
     ap.add_argument("--star", action="store_true", help="n-ary STAR operator instead of binary-operator chains")
     ap.add_argument("--world", type=int, default=1,
                     help="dimensions of SF sf*W, lineorder = rank 0's shard of W (a weak-scaling rank)")
@@ -77,12 +80,18 @@ def main():
         line = []
         for i, (ms, by, cl) in enumerate(prof):
             line.append(f"{names[cl]}:{ms*1e3:.0f}us/{by/1e6:.0f}MB/{by/ms/1e6 if ms else 0:.0f}GB/s")
-            t = tot.setdefault(names[cl], [0.0, 0.0])
+            t = tot.setdefault(names[cl], [0.0, 0.0, 0])
             t[0] += ms
             t[1] += by
+            t[2] += 1
         print(q, f"total {sum(x[0] for x in prof)*1e3:.0f}us", " | ".join(line))
-    for k, (ms, by) in tot.items():
+    for k, (ms, by, n) in tot.items():
         print(f"{k:8s} {ms*1e3:9.0f} us {by/1e9:8.3f} GB {by/ms/1e6:8.0f} GB/s")
+    if a.json:
+        import json
+        json.dump({"sf": a.sf, "queries": qs, "per_step": {
+            k: {"launches": n, "algorithmic_bytes_per_launch": round(by / n), "event_us_per_launch": round(ms * 1e3 / n, 2)}
+            for k, (ms, by, n) in tot.items()}}, open(a.json, "w"), indent=1)
 
 
 if __name__ == "__main__":
