@@ -122,6 +122,10 @@ __device__ __forceinline__ uint32_t ld_volatile_smem(const uint32_t* p) {
 // Copy `cnt` ring entries starting at ring offset `r0` (no wrap) of every field
 // (field f lives at ring + f * ring_n) to its output at [g, g + cnt), clamped to
 // out_cap.  Called by a whole warp (tid = lane, nthr = 32) or by the whole CTA.
+// kXlate: field 1 holds the hits' KEYS and is written as their join-index payloads
+// (payarr[key - key_min]) -- the lookups are done here, for dense survivors with every
+// lane active, instead of per item (mostly dead) in the probe loop.
+template <bool kXlate>
 __device__ __forceinline__ void copy_out(const WsParams& P, const int32_t* ring, uint32_t ring_n, uint32_t r0,
                                          uint32_t cnt, uint32_t g, uint32_t tid, uint32_t nthr) {
   uint32_t lim = cnt;
@@ -129,18 +133,36 @@ __device__ __forceinline__ void copy_out(const WsParams& P, const int32_t* ring,
     lim = P.out_cap > g ? P.out_cap - g : 0u;
     if (tid == 0 && P.d_overflow) atomicMax(P.d_overflow, 4u);
   }
+  const int32_t* pa = P.payarr;
+  const uint32_t kmin = (uint32_t)P.key_min;
   if ((g & 3u) == 0 && lim == cnt && (cnt & 3u) == 0) {  // 16-byte copies
     for (int f = 0; f < P.n_fields; f++) {
       const int4* src = reinterpret_cast<const int4*>(ring + (size_t)f * ring_n + r0);
       int4* dst = reinterpret_cast<int4*>(P.field_out[f] + g);
-      for (uint32_t i = tid; i < cnt / 4; i += nthr) dst[i] = src[i];
+      if (kXlate && f == 1) {
+#pragma unroll 4
+        for (uint32_t i = tid; i < cnt / 4; i += nthr) {
+          int4 k = src[i];
+          k.x = __ldg(pa + ((uint32_t)k.x - kmin));
+          k.y = __ldg(pa + ((uint32_t)k.y - kmin));
+          k.z = __ldg(pa + ((uint32_t)k.z - kmin));
+          k.w = __ldg(pa + ((uint32_t)k.w - kmin));
+          dst[i] = k;
+        }
+      } else {
+        for (uint32_t i = tid; i < cnt / 4; i += nthr) dst[i] = src[i];
+      }
     }
     return;
   }
   for (int f = 0; f < P.n_fields; f++) {
     const int32_t* src = ring + (size_t)f * ring_n + r0;
     int32_t* dst = P.field_out[f] + g;
-    for (uint32_t i = tid; i < lim; i += nthr) dst[i] = src[i];
+    if (kXlate && f == 1) {
+      for (uint32_t i = tid; i < lim; i += nthr) dst[i] = __ldg(pa + ((uint32_t)src[i] - kmin));
+    } else {
+      for (uint32_t i = tid; i < lim; i += nthr) dst[i] = src[i];
+    }
   }
 }
 
@@ -197,6 +219,9 @@ __global__ void __launch_bounds__(ws_nw(kIn == 1) * 32, 1) ws_kernel(const __gri
   int32_t* ring = reinterpret_cast<int32_t*>(smem);  // fields [tid | payload | carried...] x RING
   constexpr bool kProbe = kKind <= WK_HT_GLOBAL || kKind == WK_BM_COARSE;
   constexpr bool kHash = kKind == WK_HT_SMEM || kKind == WK_HT_GLOBAL;
+  // bitmap-masked join-index probe with payloads: most items are dead rows, so the
+  // payload lookups wait for the flush (copy_out<true>), where the survivors are dense
+  constexpr bool kXlate = kPay && kIn == 2 && !kHash;
   uint32_t* s_bm = reinterpret_cast<uint32_t*>(smem + P.tab_off);
   uint64_t* s_ht = reinterpret_cast<uint64_t*>(smem + P.tab_off);
 
@@ -273,7 +298,10 @@ __global__ void __launch_bounds__(ws_nw(kIn == 1) * 32, 1) ws_kernel(const __gri
         for (int j = 0; j < WS_ITEMS; j++) {
           uint32_t hit;
           if (kKind == WK_BM_SMEM) {
-            const uint32_t oo = min((uint32_t)(key[j] - P.key_min), P.range);
+            uint32_t oo = min((uint32_t)(key[j] - P.key_min), P.range);
+            // a row outside the input bitmap reads the clamp word like every other
+            // dead lane (one broadcast address: fewer bank conflicts, no branch)
+            if (kIn == 2) oo = ((flags >> j) & 1u) ? oo : P.range;
             hit = (s_bm[oo >> 5] >> (oo & 31)) & 1u;
           } else if (kKind == WK_BM_COARSE) {  // coarse filter here, exact bit below
             const uint32_t oo = min((uint32_t)(key[j] - P.key_min), P.range);
@@ -301,7 +329,7 @@ __global__ void __launch_bounds__(ws_nw(kIn == 1) * 32, 1) ws_kernel(const __gri
           m = m2;
         }
         flags &= m;
-        if (kPay) {
+        if (kPay && !kXlate) {
           const uint32_t any = __reduce_or_sync(FULL, flags);
 #pragma unroll
           for (int j = 0; j < WS_ITEMS; j++) {
@@ -309,6 +337,10 @@ __global__ void __launch_bounds__(ws_nw(kIn == 1) * 32, 1) ws_kernel(const __gri
             if ((any >> j) & 1u)
               if ((flags >> j) & 1u) pay[j] = __ldg(P.payarr + (uint32_t)(key[j] - P.key_min));
           }
+        }
+        if (kXlate) {  // the key goes into the ring, translated at the flush
+#pragma unroll
+          for (int j = 0; j < WS_ITEMS; j++) pay[j] = key[j];
         }
       } else {
 #pragma unroll
@@ -511,7 +543,7 @@ __global__ void __launch_bounds__(ws_nw(kIn == 1) * 32, 1) ws_kernel(const __gri
       uint32_t g = 0;
       if (lane == 0) g = atomicAdd(P.d_out_count, BLK);
       g = __shfl_sync(FULL, g, 0);
-      copy_out(P, ring, RING, slot * BLK, BLK, g, lane, 32);
+      copy_out<kXlate>(P, ring, RING, slot * BLK, BLK, g, lane, 32);
       __threadfence_block();
       __syncwarp();
       if (lane == 0) {
@@ -535,7 +567,7 @@ __global__ void __launch_bounds__(ws_nw(kIn == 1) * 32, 1) ws_kernel(const __gri
   if (rem) {
     if (threadIdx.x == 0) s_base = atomicAdd(P.d_out_count, rem);
     __syncthreads();
-    copy_out(P, ring, RING, ((total / BLK) & RM) * BLK, rem, s_base, threadIdx.x, blockDim.x);
+    copy_out<kXlate>(P, ring, RING, ((total / BLK) & RM) * BLK, rem, s_base, threadIdx.x, blockDim.x);
   }
   // the last CTA to finish clamps the count to the output capacity
   __syncthreads();
