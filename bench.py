@@ -463,13 +463,13 @@ def main():
     achieved = cls_bytes[dom] / (cls_ms[dom] / 1e3) / 1e9
     step_bytes = sum(cls_bytes.values())
     # measured DRAM traffic per launch of this kernel class: ncu launch list of the
-    # bench command (tools/ncu_traffic.py -> profiles/r1_traffic.json)
+    # bench command (tools/ncu_traffic.py -> profiles/r2_traffic.json)
     traffic = None
     try:
-        tr = json.load(open(os.path.join(ROOT, "profiles", "r1_traffic.json")))["classes"][tclass[dom]]
+        tr = json.load(open(os.path.join(ROOT, "profiles", "r2_traffic.json")))["classes"][tclass[dom]]
         traffic = {"dram_bytes_per_launch": tr["dram_bytes_per_launch"],
                    "algorithmic_bytes_per_launch": round(cls_bytes[dom] / cls_n[dom]),
-                   "source": "ncu dram__bytes_read.sum + dram__bytes_write.sum, profiles/r1_traffic.json"}
+                   "source": "ncu dram__bytes_read.sum + dram__bytes_write.sum, profiles/r2_traffic.json"}
     except Exception:
         pass
     roofline = {"bound": "hbm", "kernel": names[dom], "achieved": round(achieved, 1),
@@ -477,7 +477,13 @@ def main():
                 "launches_per_step": cls_n[dom], "share_of_step": round(cls_ms[dom] / sum(cls_ms.values()), 3),
                 "peak_source": "MEASURED_PEAKS.json hbm_gbs (measured)" if "hbm_gbs" in pk else "fallback 6.65 TB/s",
                 "step_model_gb": round(step_bytes / 1e9, 3),
-                "step_gbs": round(step_bytes / (ms_per_step / 1e3) / 1e9 * ws, 1)}
+                "step_gbs": round(step_bytes / (ms_per_step / 1e3) / 1e9 * ws, 1),
+                # every kernel class of the step, same event-timed replay and byte model
+                "classes": {tclass[c]: {"launches_per_step": cls_n[c], "us_per_step": round(cls_ms[c] * 1e3, 1),
+                                        "achieved_gbs": round(cls_bytes[c] / (cls_ms[c] / 1e3) / 1e9, 1),
+                                        "frac": round(cls_bytes[c] / (cls_ms[c] / 1e3) / 1e9 / hbm_peak, 4),
+                                        "share_of_step": round(cls_ms[c] / sum(cls_ms.values()), 3)}
+                            for c in sorted(cls_ms, key=lambda c: -cls_ms[c]) if cls_ms[c] > 0}}
 
     # ---- e2e through the public API with host buffers: cold cache, every column
     #      H2D from pinned host memory inside the timed region (GPU-only placement)

@@ -1936,6 +1936,9 @@ int32_t ddq_prepared_profile(ddq_prepared* p, void* stream, int32_t max_ops, flo
   const int n = p->plan.n_ops;
   std::vector<cudaEvent_t> ev((size_t)n + 1);
   for (auto& e : ev) cudaEventCreate(&e);
+  // the operators are enqueued behind a device-side delay (longer than their host
+  // set-up and launches take), so each event pair brackets device time only
+  launch_delay((uint64_t)(500 + 100 * n) * 1000, st);
   cudaEventRecord(ev[0], st);
   for (int i = 0; i < n; i++) {
     std::vector<void*> blocks = p->inters[(size_t)i].heap_blocks;

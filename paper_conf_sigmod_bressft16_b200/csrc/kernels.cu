@@ -138,6 +138,23 @@ cudaError_t launch_multi_fill(const std::vector<FillRec>& recs, cudaStream_t st)
   return cudaSuccess;
 }
 
+// One thread that holds the stream for `ns` nanoseconds (%globaltimer): a profiling
+// replay enqueues its operators behind it, so their event-to-event times are device
+// time, not the host's launch and set-up latency between small operators.
+__global__ void delay_kernel(uint64_t ns) {
+  uint64_t t0, t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t0));
+  do {
+    __nanosleep(1000);
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  } while (t - t0 < ns);
+}
+
+cudaError_t launch_delay(uint64_t ns, cudaStream_t st) {
+  delay_kernel<<<1, 1, 0, st>>>(ns);
+  return cudaGetLastError();
+}
+
 cudaError_t init_fill(void* ptr, size_t bytes, uint64_t pattern, cudaStream_t st) {
   if (bytes == 0) return cudaSuccess;
   FillHoist& h = fill_hoist();

@@ -30,6 +30,8 @@ def klass(name: str) -> str:
         return "agg"
     if "build" in name:
         return "build"
+    if "unpack" in name:  # load-time widening of packed columns (setup, not the step)
+        return "load"
     return "other"
 
 
