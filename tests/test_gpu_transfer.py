@@ -73,8 +73,6 @@ def test_ssb_cold_packed_equals_raw_equals_oracle():
         for q in SSB_QUERIES:
             r = db.run(ssb_plan(db, q))
             want = [tuple(x) for x in oracle.run(data, q)]
-            if q.startswith("ssb1") and not r.rows:
-                want = [w for w in want if w != (0, 0)]
             assert r.rows == want and r.host_ops == 0, (q, packing)
         moved[packing] = db.stats()["h2d_bytes"]
         db.close()
