@@ -413,6 +413,7 @@ constexpr int DS_R = 4;               // rows per thread per stage
 constexpr int DS_SR = DS_T * DS_R;    // rows per ring stage
 constexpr int DS_MAXC = 12;           // distinct columns streamed
 constexpr int DS_MAX_DA = 64;
+constexpr int DS_SMAX = 8;            // ring stages at most
 static_assert(4 /*DS_R*/ * 8 <= 32, "overflow mask: DS_R x A bits");
 constexpr size_t DS_SMEM_MAX = 227 * 1024 - 1024;
 
@@ -463,9 +464,9 @@ constexpr uint32_t DS_Q1 = ds_kinds(DDQ_AGG_SUM, DDQ_AGG_SUM, DDQ_AGG_SUM_MUL_10
                                     DDQ_AGG_SUM, DDQ_AGG_COUNT);
 
 template <int NA, uint32_t KINDS>
-__global__ void __launch_bounds__(DS_T, 1) agg_dense_small_kernel(const __grid_constant__ DenseAggParams P) {
+__global__ void __launch_bounds__(DS_T + 32, 1) agg_dense_small_kernel(const __grid_constant__ DenseAggParams P) {
   extern __shared__ __align__(128) uint8_t ds_smem[];
-  __shared__ __align__(8) uint64_t full[8];
+  __shared__ __align__(8) uint64_t full[DS_SMAX], empty[DS_SMAX];
   __shared__ uint32_t s_present, s_rows;
   constexpr int A = NA;
   const uint32_t DA = P.D * (uint32_t)A;
@@ -490,18 +491,29 @@ __global__ void __launch_bounds__(DS_T, 1) agg_dense_small_kernel(const __grid_c
                   (rows * P.width[c] + 15) & ~15u, &full[k % S]);
   };
   if (tid == 0) {
-    for (int s = 0; s < S; s++) mbar_init(&full[s], 1);
+    for (int s = 0; s < S; s++) {
+      mbar_init(&full[s], 1);
+      mbar_init(&empty[s], DS_T / 32);  // one arrival per consumer warp
+    }
     fence_mbar_init();
     s_present = 0;
     s_rows = 0;
   }
-  for (uint32_t e = 0; e < DA; e++) part[(size_t)e * DS_T + tid] = 0;
-  for (uint32_t i = tid; i < DA * 2; i += DS_T) spill[i] = 0;
+  if (tid < DS_T) {
+    for (uint32_t e = 0; e < DA; e++) part[(size_t)e * DS_T + tid] = 0;
+    for (uint32_t i = tid; i < DA * 2; i += DS_T) spill[i] = 0;
+  }
   __syncthreads();
-  if (tid == 0)
-    for (int s = 0; s < S && blockIdx.x + (uint32_t)s * gridDim.x < nch; s++) issue((uint32_t)s);
-
   uint32_t pm = 0, nrows = 0;
+  if (tid >= DS_T) {
+    // the producer warp: refills a slot as soon as every consumer warp released it
+    // (no CTA-wide barrier per stage: consumer warps drift up to S stages apart)
+    if (tid == DS_T)
+      for (uint32_t k = 0; blockIdx.x + k * gridDim.x < nch; k++) {
+        if (k >= (uint32_t)S) mbar_wait(&empty[k % S], (k / S - 1) & 1u);
+        issue(k);
+      }
+  } else
   for (uint32_t k = 0; blockIdx.x + k * gridDim.x < nch; k++) {
     const uint32_t row0 = (blockIdx.x + k * gridDim.x) * DS_SR;
     const uint8_t* stage = ring + (size_t)(k % S) * P.stage_bytes;
@@ -611,8 +623,8 @@ __global__ void __launch_bounds__(DS_T, 1) agg_dense_small_kernel(const __grid_c
             add_i128(sp, sp + 1, 0ull, v[a][j] > 0 ? 1 : -1);
           }
     }
-    __syncthreads();  // every thread is done with this slot: refill it
-    if (tid == 0 && blockIdx.x + (k + S) * gridDim.x < nch) issue(k + S);
+    __syncwarp();  // this warp is done with the slot
+    if ((tid & 31) == 0) mbar_arrive(&empty[k % S]);
   }
   pm = __reduce_or_sync(FULL, pm);
   nrows = __reduce_add_sync(FULL, nrows);
@@ -624,6 +636,7 @@ __global__ void __launch_bounds__(DS_T, 1) agg_dense_small_kernel(const __grid_c
   if (tid == 0 && P.d_rows && s_rows) atomicAdd(P.d_rows, s_rows);
   const int lane = tid & 31, warp = tid >> 5;
   const uint32_t pres = s_present;
+  if (tid < DS_T)
   for (uint32_t e = warp; e < DA; e += DS_T / 32) {
     const uint32_t g = e / A;
     const int a = (int)(e % A);
@@ -810,7 +823,7 @@ static bool dense_plan(int64_t n_rows, const BuildPreds* preds, const int32_t* c
   }
   p->stage_bytes = sb < 16 ? 16 : sb;
   const size_t fixed = ((size_t)p->D * n_aggs) * (DS_T * 8 + 16);
-  int S = 4;
+  int S = DS_SMAX;
   while (S > 2 && fixed + (size_t)S * p->stage_bytes > DS_SMEM_MAX) S--;
   if (fixed + (size_t)S * p->stage_bytes > DS_SMEM_MAX) return false;
   p->n_stages = S;
@@ -880,16 +893,16 @@ cudaError_t launch_agg_dense(int64_t n_rows, const int32_t* const* key_col, int 
   if (grid > nch) grid = nch;
   uint32_t kinds = 0;
   for (int a = 0; a < n_aggs; a++) kinds |= (uint32_t)aggs[a].kind << (3 * a);
-  if (n_aggs == 6 && kinds == DS_Q1) agg_dense_small_kernel<6, DS_Q1><<<(int)grid, DS_T, smem, st>>>(p);
+  if (n_aggs == 6 && kinds == DS_Q1) agg_dense_small_kernel<6, DS_Q1><<<(int)grid, DS_T + 32, smem, st>>>(p);
   else switch (n_aggs) {
-      case 1: agg_dense_small_kernel<1, DS_RUNTIME><<<(int)grid, DS_T, smem, st>>>(p); break;
-      case 2: agg_dense_small_kernel<2, DS_RUNTIME><<<(int)grid, DS_T, smem, st>>>(p); break;
-      case 3: agg_dense_small_kernel<3, DS_RUNTIME><<<(int)grid, DS_T, smem, st>>>(p); break;
-      case 4: agg_dense_small_kernel<4, DS_RUNTIME><<<(int)grid, DS_T, smem, st>>>(p); break;
-      case 5: agg_dense_small_kernel<5, DS_RUNTIME><<<(int)grid, DS_T, smem, st>>>(p); break;
-      case 6: agg_dense_small_kernel<6, DS_RUNTIME><<<(int)grid, DS_T, smem, st>>>(p); break;
-      case 7: agg_dense_small_kernel<7, DS_RUNTIME><<<(int)grid, DS_T, smem, st>>>(p); break;
-      default: agg_dense_small_kernel<8, DS_RUNTIME><<<(int)grid, DS_T, smem, st>>>(p); break;
+      case 1: agg_dense_small_kernel<1, DS_RUNTIME><<<(int)grid, DS_T + 32, smem, st>>>(p); break;
+      case 2: agg_dense_small_kernel<2, DS_RUNTIME><<<(int)grid, DS_T + 32, smem, st>>>(p); break;
+      case 3: agg_dense_small_kernel<3, DS_RUNTIME><<<(int)grid, DS_T + 32, smem, st>>>(p); break;
+      case 4: agg_dense_small_kernel<4, DS_RUNTIME><<<(int)grid, DS_T + 32, smem, st>>>(p); break;
+      case 5: agg_dense_small_kernel<5, DS_RUNTIME><<<(int)grid, DS_T + 32, smem, st>>>(p); break;
+      case 6: agg_dense_small_kernel<6, DS_RUNTIME><<<(int)grid, DS_T + 32, smem, st>>>(p); break;
+      case 7: agg_dense_small_kernel<7, DS_RUNTIME><<<(int)grid, DS_T + 32, smem, st>>>(p); break;
+      default: agg_dense_small_kernel<8, DS_RUNTIME><<<(int)grid, DS_T + 32, smem, st>>>(p); break;
     }
   return cudaGetLastError();
 }
