@@ -463,7 +463,10 @@ constexpr uint32_t ds_kinds(int k0, int k1 = 0, int k2 = 0, int k3 = 0, int k4 =
 constexpr uint32_t DS_Q1 = ds_kinds(DDQ_AGG_SUM, DDQ_AGG_SUM, DDQ_AGG_SUM_MUL_100M, DDQ_AGG_SUM_MUL_100M_100P,
                                     DDQ_AGG_SUM, DDQ_AGG_COUNT);
 
-template <int NA, uint32_t KINDS>
+// kOvf: test every partial add for signed overflow (wrap-and-count).  The host drops
+// the test when the columns' value ranges prove that no thread partial can reach
+// 2^62 (|row value| x rows per thread), which holds for TPC-H / SSB measures.
+template <int NA, uint32_t KINDS, bool kOvf>
 __global__ void __launch_bounds__(DS_T + 32, 1) agg_dense_small_kernel(const __grid_constant__ DenseAggParams P) {
   extern __shared__ __align__(128) uint8_t ds_smem[];
   __shared__ __align__(8) uint64_t full[DS_SMAX], empty[DS_SMAX];
@@ -610,7 +613,7 @@ __global__ void __launch_bounds__(DS_T + 32, 1) agg_dense_small_kernel(const __g
       for (int a = 0; a < A; a++) {
         const long long sum = (long long)((unsigned long long)old[a] + (unsigned long long)v[a][j]);
         row[a * DS_T] = sum;
-        omask |= (((old[a] ^ sum) & (v[a][j] ^ sum)) < 0 ? 1u : 0u) << (j * A + a);
+        if (kOvf) omask |= (((old[a] ^ sum) & (v[a][j] ^ sum)) < 0 ? 1u : 0u) << (j * A + a);
       }
     }
     if (__builtin_expect(omask != 0, 0)) {
@@ -840,7 +843,7 @@ bool agg_dense_supported(int64_t n_rows, const BuildPreds* preds, const int32_t*
 
 cudaError_t launch_agg_dense(int64_t n_rows, const int32_t* const* key_col, int n_keys, const int32_t* key_bits,
                              const ddq_dev_agg* aggs, int n_aggs, void* table, uint32_t capacity, uint32_t* d_error,
-                             cudaStream_t st, const BuildPreds* preds, uint32_t* d_rows) {
+                             cudaStream_t st, const BuildPreds* preds, uint32_t* d_rows, double max_row_abs) {
   DenseAggParams p{};
   if (!dense_plan(n_rows, preds, key_col, n_keys, key_bits, aggs, n_aggs, &p)) return cudaErrorInvalidValue;
   p.n = (uint32_t)n_rows;
@@ -875,15 +878,16 @@ cudaError_t launch_agg_dense(int64_t n_rows, const int32_t* const* key_col, int 
   const size_t smem = (size_t)p.n_stages * p.stage_bytes + ((size_t)p.D * n_aggs) * (DS_T * 8 + 16);
   static const bool attr = [] {  // thread-safe one-time opt-in
     const int mx = (int)DS_SMEM_MAX;
-    cudaFuncSetAttribute(agg_dense_small_kernel<6, DS_Q1>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx);
-    cudaFuncSetAttribute(agg_dense_small_kernel<1, DS_RUNTIME>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx);
-    cudaFuncSetAttribute(agg_dense_small_kernel<2, DS_RUNTIME>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx);
-    cudaFuncSetAttribute(agg_dense_small_kernel<3, DS_RUNTIME>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx);
-    cudaFuncSetAttribute(agg_dense_small_kernel<4, DS_RUNTIME>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx);
-    cudaFuncSetAttribute(agg_dense_small_kernel<5, DS_RUNTIME>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx);
-    cudaFuncSetAttribute(agg_dense_small_kernel<6, DS_RUNTIME>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx);
-    cudaFuncSetAttribute(agg_dense_small_kernel<7, DS_RUNTIME>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx);
-    cudaFuncSetAttribute(agg_dense_small_kernel<8, DS_RUNTIME>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx);
+    cudaFuncSetAttribute(agg_dense_small_kernel<6, DS_Q1, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx);
+    cudaFuncSetAttribute(agg_dense_small_kernel<6, DS_Q1, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx);
+    cudaFuncSetAttribute(agg_dense_small_kernel<1, DS_RUNTIME, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx);
+    cudaFuncSetAttribute(agg_dense_small_kernel<2, DS_RUNTIME, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx);
+    cudaFuncSetAttribute(agg_dense_small_kernel<3, DS_RUNTIME, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx);
+    cudaFuncSetAttribute(agg_dense_small_kernel<4, DS_RUNTIME, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx);
+    cudaFuncSetAttribute(agg_dense_small_kernel<5, DS_RUNTIME, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx);
+    cudaFuncSetAttribute(agg_dense_small_kernel<6, DS_RUNTIME, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx);
+    cudaFuncSetAttribute(agg_dense_small_kernel<7, DS_RUNTIME, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx);
+    cudaFuncSetAttribute(agg_dense_small_kernel<8, DS_RUNTIME, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx);
     return true;
   }();
   (void)attr;
@@ -893,16 +897,22 @@ cudaError_t launch_agg_dense(int64_t n_rows, const int32_t* const* key_col, int 
   if (grid > nch) grid = nch;
   uint32_t kinds = 0;
   for (int a = 0; a < n_aggs; a++) kinds |= (uint32_t)aggs[a].kind << (3 * a);
-  if (n_aggs == 6 && kinds == DS_Q1) agg_dense_small_kernel<6, DS_Q1><<<(int)grid, DS_T + 32, smem, st>>>(p);
-  else switch (n_aggs) {
-      case 1: agg_dense_small_kernel<1, DS_RUNTIME><<<(int)grid, DS_T + 32, smem, st>>>(p); break;
-      case 2: agg_dense_small_kernel<2, DS_RUNTIME><<<(int)grid, DS_T + 32, smem, st>>>(p); break;
-      case 3: agg_dense_small_kernel<3, DS_RUNTIME><<<(int)grid, DS_T + 32, smem, st>>>(p); break;
-      case 4: agg_dense_small_kernel<4, DS_RUNTIME><<<(int)grid, DS_T + 32, smem, st>>>(p); break;
-      case 5: agg_dense_small_kernel<5, DS_RUNTIME><<<(int)grid, DS_T + 32, smem, st>>>(p); break;
-      case 6: agg_dense_small_kernel<6, DS_RUNTIME><<<(int)grid, DS_T + 32, smem, st>>>(p); break;
-      case 7: agg_dense_small_kernel<7, DS_RUNTIME><<<(int)grid, DS_T + 32, smem, st>>>(p); break;
-      default: agg_dense_small_kernel<8, DS_RUNTIME><<<(int)grid, DS_T + 32, smem, st>>>(p); break;
+  // rows one thread adds into one partial at most: its CTA's stages x DS_R
+  const double rows_per_thread = (double)((nch + grid - 1) / grid) * DS_R;
+  const bool ovf = !(max_row_abs >= 0 && max_row_abs * rows_per_thread < 4.6e18);  // < 2^62
+  const dim3 blk(DS_T + 32);
+  if (n_aggs == 6 && kinds == DS_Q1) {
+    if (ovf) agg_dense_small_kernel<6, DS_Q1, true><<<(int)grid, blk, smem, st>>>(p);
+    else agg_dense_small_kernel<6, DS_Q1, false><<<(int)grid, blk, smem, st>>>(p);
+  } else switch (n_aggs) {
+      case 1: agg_dense_small_kernel<1, DS_RUNTIME, true><<<(int)grid, blk, smem, st>>>(p); break;
+      case 2: agg_dense_small_kernel<2, DS_RUNTIME, true><<<(int)grid, blk, smem, st>>>(p); break;
+      case 3: agg_dense_small_kernel<3, DS_RUNTIME, true><<<(int)grid, blk, smem, st>>>(p); break;
+      case 4: agg_dense_small_kernel<4, DS_RUNTIME, true><<<(int)grid, blk, smem, st>>>(p); break;
+      case 5: agg_dense_small_kernel<5, DS_RUNTIME, true><<<(int)grid, blk, smem, st>>>(p); break;
+      case 6: agg_dense_small_kernel<6, DS_RUNTIME, true><<<(int)grid, blk, smem, st>>>(p); break;
+      case 7: agg_dense_small_kernel<7, DS_RUNTIME, true><<<(int)grid, blk, smem, st>>>(p); break;
+      default: agg_dense_small_kernel<8, DS_RUNTIME, true><<<(int)grid, blk, smem, st>>>(p); break;
     }
   return cudaGetLastError();
 }

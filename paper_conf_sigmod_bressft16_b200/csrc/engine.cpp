@@ -113,6 +113,46 @@ bool use_join_index(const Column& kc, int64_t n_rows) {
 // Input rows up to which an AGGREGATE evaluates its probe terms row by row (reading
 // O37); about two waves of the warp-autonomous aggregation (148 SMs x 16 warps x
 // 256-row tiles x 2 = 1.2 M rows on B200).  Longer inputs evaluate them term by term.
+// The largest |value| one row can add to an aggregate of op, from the argument
+// columns' load-time value ranges (include/ddq.h's expression set); -1 if unknown.
+double max_row_abs(ddq_db* db, const ddq_op& op) {
+  auto mx = [&](int c, long double off, long double sgn, long double* out) {
+    const Column* col = col_of(db, c);
+    if (!col || col->n <= 0 || col->vmax < col->vmin) return false;
+    const long double a = fabsl(off + sgn * (long double)col->vmin), b = fabsl(off + sgn * (long double)col->vmax);
+    *out = a > b ? a : b;
+    return true;
+  };
+  long double best = 0;
+  for (int a = 0; a < op.n_aggs; a++) {
+    long double x = 1, y = 1, z = 1;
+    switch (op.agg_kind[a]) {
+      case DDQ_AGG_COUNT: break;
+      case DDQ_AGG_SUM: if (!mx(op.agg_col[a][0], 0, 1, &x)) return -1; break;
+      case DDQ_AGG_SUM_MUL:
+        if (!mx(op.agg_col[a][0], 0, 1, &x) || !mx(op.agg_col[a][1], 0, 1, &y)) return -1;
+        break;
+      case DDQ_AGG_SUM_SUB:
+        if (!mx(op.agg_col[a][0], 0, 1, &x) || !mx(op.agg_col[a][1], 0, 1, &y)) return -1;
+        x += y;
+        y = 1;
+        break;
+      case DDQ_AGG_SUM_MUL_100M:
+        if (!mx(op.agg_col[a][0], 0, 1, &x) || !mx(op.agg_col[a][1], 100, -1, &y)) return -1;
+        break;
+      case DDQ_AGG_SUM_MUL_100M_100P:
+        if (!mx(op.agg_col[a][0], 0, 1, &x) || !mx(op.agg_col[a][1], 100, -1, &y) ||
+            !mx(op.agg_col[a][2], 100, 1, &z))
+          return -1;
+        break;
+      default: return -1;
+    }
+    const long double v = x * y * z;
+    if (v > best) best = v;
+  }
+  return (double)best;
+}
+
 int64_t fused_tail_max_rows() {
   if (const char* e = getenv("DDQ_FUSED_TAIL_MAX")) return (int64_t)strtoll(e, nullptr, 10);  // tests / A-B
   return (int64_t)num_sms() * 16 * 256 * 2;
@@ -705,7 +745,7 @@ ddq_status run_gpu_op(GpuOpCtx& ctx, const ddq_op& op, Inter& out) {
         cudaError_t e = launch_groupby_init(out.gb_table, out.gb_cap, op.n_aggs, st);
         if (e == cudaSuccess)
           e = launch_agg_dense(in_cap, kc, op.n_keys, op.key_bits, ag, op.n_aggs, out.gb_table, out.gb_cap,
-                               out.d_error, st, &bp, out.d_rows);
+                               out.d_error, st, &bp, out.d_rows, max_row_abs(db, op));
         if (e == cudaSuccess)
           e = launch_groupby_compact(out.gb_table, out.gb_cap, op.n_aggs, out.gb_keys, out.gb_accs, out.gb_groups, st);
         return cuda_status(e, "aggregate (dense)");

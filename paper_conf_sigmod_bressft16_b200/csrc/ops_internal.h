@@ -164,7 +164,7 @@ bool agg_dense_supported(int64_t n_rows, const struct BuildPreds* preds, const i
                          const int32_t* key_bits, const ddq_dev_agg* aggs, int n_aggs);
 cudaError_t launch_agg_dense(int64_t n_rows, const int32_t* const* key_col, int n_keys, const int32_t* key_bits,
                              const ddq_dev_agg* aggs, int n_aggs, void* table, uint32_t capacity, uint32_t* d_error,
-                             cudaStream_t st, const struct BuildPreds* preds, uint32_t* d_rows);
+                             cudaStream_t st, const struct BuildPreds* preds, uint32_t* d_rows, double max_row_abs = -1);
 cudaError_t launch_iota(int32_t* out, int64_t n, uint32_t* d_count, cudaStream_t st);
 // A probe / fetch term fused into the aggregation at TIDs (reading O37):
 // the fk column is gathered at the row, looked up in a join index (bitmap +
