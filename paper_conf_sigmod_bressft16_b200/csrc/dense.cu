@@ -672,6 +672,23 @@ bool ws_supported(const FilterArgs& a) {
 // for a 75 KB bitmap per SM).
 static bool stage_pays(int64_t n_cap, size_t tab) { return n_cap >= (int64_t)(tab * 4); }
 
+// Whether launch_ws stages a probe's join-index bitmap (join index over `range`
+// keys) or hash table (`capacity` slots) in shared memory for a bitmap-masked probe
+// of n_rows rows (the WK_BM_SMEM / WK_HT_SMEM choice below).  ddq_prepare hands a
+// row bitmap only to such consumers: with the table in L2 (customer at SF >= 60)
+// the masked probe issues its L2 lookups at every row slot, live or dead
+// (SF100 Q3.1: 1.26 ms against a TID list's fraction of that).
+bool ws_masked_probe_smem(bool join_index, uint32_t range_or_capacity, int64_t n_rows, bool pay) {
+  int dev = 0, v = 0;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&v, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
+  const size_t budget = (size_t)v - kWsCtl;
+  const size_t ring1 = (size_t)ws_blk(false) * 4 * (pay ? 2 : 1);
+  const size_t tab = join_index ? ((size_t)((range_or_capacity + 31) / 32) * 4 + 15) / 16 * 16 + 16
+                                : (size_t)range_or_capacity * 8;
+  return 4 * ring1 + tab <= budget && stage_pays(n_rows, tab);
+}
+
 cudaError_t launch_ws(const FilterArgs& a, cudaStream_t st) {
   // one-time opt-in of every variant's dynamic shared memory; a function-local static
   // initialiser, so concurrent GPU workers wait for it (no launch before the attributes)

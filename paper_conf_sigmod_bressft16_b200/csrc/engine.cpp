@@ -1832,6 +1832,8 @@ ddq_status ddq_prepare(ddq_db* db, const ddq_plan* plan, int32_t use_graph, ddq_
   };
   // 1. calibration run (worst-case capacities) -> exact counts
   std::vector<int64_t> counts((size_t)plan->n_ops, -1);
+  // per build op: its join index's key range (>= 0) or hash table capacity (-2 - cap)
+  std::vector<int64_t> build_tab((size_t)plan->n_ops, -1);
   {
     std::vector<Inter> cal((size_t)plan->n_ops);
     GpuOpCtx ctx{db, st, &cal};
@@ -1843,6 +1845,9 @@ ddq_status ddq_prepare(ddq_db* db, const ddq_plan* plan, int32_t use_graph, ddq_
         free_inters(db, cal);
         return fail(s == DDQ_ENOMEM_DEVICE ? set_error(s, "prepare: device heap exhausted (calibration)") : s);
       }
+      if (plan->ops[i].kind == DDQ_OP_HASH_BUILD)
+        build_tab[(size_t)i] = cal[(size_t)i].jidx ? (int64_t)cal[(size_t)i].jrange
+                                                   : -2 - (int64_t)cal[(size_t)i].table_cap;
       if (cal[(size_t)i].d_count && plan->ops[i].kind != DDQ_OP_GATHER) {
         uint32_t c = 0;
         cudaMemcpyAsync(&c, cal[(size_t)i].d_count, 4, cudaMemcpyDeviceToHost, st);
@@ -1896,6 +1901,13 @@ ddq_status ddq_prepare(ddq_db* db, const ddq_plan* plan, int32_t use_graph, ddq_
         // producer no longer compacts 24 M TIDs through its ring (152 -> 84 us), and the
         // 4-stream step drops 2.67 -> 2.60 ms (Q3.1, Q4.2)
         ok = ok && c.kind == DDQ_OP_HASH_PROBE && c.fk_vec <= 0;
+        // ... whose table the masked probe keeps in shared memory (else TID lists)
+        if (ok && c.build >= 0 && c.build < plan->n_ops) {
+          const int64_t bt = build_tab[(size_t)c.build];
+          const int64_t rows_c = db->tables[(size_t)c.table].n_rows;
+          ok = bt >= 0 ? ws_masked_probe_smem(true, (uint32_t)bt, rows_c, c.emit_payload != 0)
+                       : (bt <= -2 && ws_masked_probe_smem(false, (uint32_t)(-2 - bt), rows_c, c.emit_payload != 0));
+        }
       }
       const int64_t rows = db->tables[(size_t)op.table].n_rows;
       const bool dense_enough = counts[(size_t)i] >= 0 && counts[(size_t)i] * 8 >= rows;

@@ -30,6 +30,7 @@ size_t packed_bytes(int64_t n, int tw);
 cudaError_t launch_unpack(const void* packed, int tw, int64_t base, void* out, int width, int64_t n, cudaStream_t st);
 cudaError_t init_fill(void* ptr, size_t bytes, uint64_t pattern, cudaStream_t st);
 cudaError_t launch_delay(uint64_t ns, cudaStream_t st);  // profiling: hold the stream
+bool ws_masked_probe_smem(bool join_index, uint32_t range_or_capacity, int64_t n_rows, bool pay);
 cudaError_t launch_multi_fill(const std::vector<FillRec>& recs, cudaStream_t st);
 
 struct FilterArgs {
