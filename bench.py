@@ -454,9 +454,10 @@ def main():
             cls_bytes[cl] = cls_bytes.get(cl, 0.0) + by
             cls_n[cl] = cls_n.get(cl, 0) + 1
     names = {0: "ws_kernel (csrc/dense.cu): dense probe over all rows", 1: "ws_kernel (csrc/dense.cu): "
-             "select/probe over a TID list or row bitmap", 2: "join_index_build_kernel (csrc/kernels.cu): build",
-             3: "gather_kernel (csrc/kernels.cu)", 4: "agg_ws_kernel (csrc/agg.cu): group-by aggregate"}
-    tclass = {0: "dense", 1: "at-tids", 2: "build", 3: "other", 4: "agg"}
+             "select/probe/fetch over a TID list", 2: "join_index_build_kernel (csrc/kernels.cu): build",
+             3: "gather_kernel (csrc/kernels.cu)", 4: "agg_ws_kernel (csrc/agg.cu): group-by aggregate",
+             5: "ws_kernel (csrc/dense.cu): probe of a key column masked by a row bitmap (every row streamed)"}
+    tclass = {0: "dense", 1: "at-tids", 2: "build", 3: "other", 4: "agg", 5: "masked"}
     dom = max(cls_ms, key=lambda c: cls_ms[c])
     pk = peaks()
     hbm_peak = pk.get("hbm_gbs", 6650.0)

@@ -531,8 +531,9 @@ int32_t ddq_prepared_kernel_count(ddq_prepared* p);
  * 8(d) model computed from the actual cardinalities (columns read once; TID-driven
  * reads at 32-byte-sector granularity: N*w*(1-(1-m/N)^(32/w)); TID / vector /
  * payload reads and writes; hash tables 0 bytes except their build writes),
- * op_class = 0 dense scan (select/probe over all rows), 1 select/probe at TIDs,
- * 2 hash build, 3 gather, 4 aggregate.  Returns the number of operators. */
+ * op_class = 0 dense scan (select/probe over all rows), 1 select/probe/fetch at
+ * TIDs, 2 hash build, 3 gather, 4 aggregate, 5 probe masked by a row bitmap (the
+ * key column streamed for every row).  Returns the number of operators. */
 int32_t ddq_prepared_profile(ddq_prepared* p, void* stream, int32_t max_ops, float* op_ms, double* op_bytes,
                              int32_t* op_class);
 /* Device views of the compacted partial group table of the last launch (for an

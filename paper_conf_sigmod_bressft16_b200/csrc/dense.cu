@@ -257,11 +257,11 @@ __global__ void __launch_bounds__(ws_nw(kIn == 1) * 32, 1) ws_kernel(const __gri
   };
   if (tile < ntiles) fetch(tile);
   uint32_t bits_cnt = 0;  // kOutBits: survivors of this lane
-  // kDefer (a dense semi-join: survivors are positions only): a tile's hit flags
+  // kDefer (a dense or bitmap-masked semi-join: survivors are positions only): a tile's hit flags
   // wait for the warp's next tile and both are compacted with ONE scan / claim /
   // ring accounting (the per-tile compaction was ~60 instructions and three
   // dependent shared-memory atomics for a handful of survivors)
-  constexpr bool kDefer = kIn == 0 && !kPay && !kCarry && !kOutBits;
+  constexpr bool kDefer = kIn != 1 && !kPay && !kCarry && !kOutBits;
   uint32_t pend = 0, pend_base = 0;
   bool have_pend = false;  // warp-uniform
 
@@ -272,7 +272,8 @@ __global__ void __launch_bounds__(ws_nw(kIn == 1) * 32, 1) ws_kernel(const __gri
     const uint32_t base = tile * WS_TILE + lofs;  // position of the lane's item 0
     if (tile + W < ntiles) fetch(tile + W);
     if (kIn == 2) {
-      if (__all_sync(FULL, flags == 0)) continue;  // an empty 512-row tile
+      // an empty 512-row tile (unless it is the warp's last and a held tile waits)
+      if (__all_sync(FULL, flags == 0) && (!kDefer || !have_pend || tile + W < ntiles)) continue;
     } else if (tile * WS_TILE + WS_TILE > n) {
       flags = 0;
 #pragma unroll

@@ -2045,7 +2045,8 @@ int32_t ddq_prepared_profile(ddq_prepared* p, void* stream, int32_t max_ops, flo
           cls = 0;
           for (int c : cols) bytes += N * width(c);
         } else {
-          cls = 1;
+          // a row-bitmap input streams the whole key column (class 5), a TID list gathers
+          cls = in_bits ? 5 : 1;
           bytes += in_bits ? N / 8 : m * 4;  // the input: a row bitmap or a TID list
           // a conjunction reads its first column at every input TID and the
           // others only at rows still alive (counted at the final survivors: a

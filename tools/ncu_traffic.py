@@ -10,7 +10,8 @@ random gathers, L2 write-backs; < 1: reuse through L2).
 Writes {class: {"launches", "dram_bytes_per_launch", "us_per_launch", "share"}}; bench.py
 reads profiles/r1_traffic.json to fill roofline.traffic for its dominant class.
 Classes follow bench.py / ddq_prepared_profile: dense (ws_kernel, every row),
-at-tids (ws_kernel over a TID list or row bitmap), agg, build, other.
+masked (ws_kernel over every row masked by a row bitmap), at-tids (ws_kernel over a
+TID list, fetch_kernel), agg, build, other.
 """
 import csv
 import json
@@ -21,7 +22,7 @@ import sys
 def klass(name: str) -> str:
     m = re.search(r"ws_kernel<\s*(?:\(int\))?\s*\d+,\s*(?:\(int\))?\s*(\d+)", name)
     if m:
-        return "dense" if m.group(1) == "0" else "at-tids"
+        return {"0": "dense", "2": "masked"}.get(m.group(1), "at-tids")
     if "scan_kernel" in name or "star_kernel" in name or "filter_kernel" in name:
         return "dense" if re.search(r"scan_kernel<\d+, (?:\(bool\))?(?:0|false)", name) else "at-tids"
     if "fetch_kernel" in name:  # late payload fetch through a join index: an at-TIDs lookup

@@ -53,7 +53,7 @@ def main():
                 p.launch()
         torch.cuda.synchronize()
         return
-    names = {0: "dense", 1: "at-tids", 2: "build", 3: "gather", 4: "agg"}
+    names = {0: "dense", 1: "at-tids", 2: "build", 3: "gather", 4: "agg", 5: "masked"}
     tot = {}
     # whole-graph time per query (the plan's CUDA graph, branches overlapped)
     stream = torch.cuda.Stream()

@@ -47,7 +47,7 @@ def main():
         prof = p.profile(st.cuda_stream)
         byt = sum(b for _, b, _ in prof)
         if a.ops:
-            names = {0: "dense", 1: "at-tids", 2: "build", 3: "gather", 4: "agg"}
+            names = {0: "dense", 1: "at-tids", 2: "build", 3: "gather", 4: "agg", 5: "masked"}
             print(q, " | ".join(f"{names.get(c, c)}:{m * 1e3:.0f}us/{b / 1e6:.0f}MB" for m, b, c in prof),
                   file=sys.stderr, flush=True)
         print(json.dumps({"config": "M4", "mode": "hot", "query": q, "sf": a.sf, "lineitem_rows": n,
