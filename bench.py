@@ -464,13 +464,13 @@ def main():
     achieved = cls_bytes[dom] / (cls_ms[dom] / 1e3) / 1e9
     step_bytes = sum(cls_bytes.values())
     # measured DRAM traffic per launch of this kernel class: ncu launch list of the
-    # bench command (tools/ncu_traffic.py -> profiles/r2_traffic.json)
+    # bench command (tools/ncu_traffic.py -> profiles/r2z_traffic.json)
     traffic = None
     try:
-        tr = json.load(open(os.path.join(ROOT, "profiles", "r2_traffic.json")))["classes"][tclass[dom]]
+        tr = json.load(open(os.path.join(ROOT, "profiles", "r2z_traffic.json")))["classes"][tclass[dom]]
         traffic = {"dram_bytes_per_launch": tr["dram_bytes_per_launch"],
                    "algorithmic_bytes_per_launch": round(cls_bytes[dom] / cls_n[dom]),
-                   "source": "ncu dram__bytes_read.sum + dram__bytes_write.sum, profiles/r2_traffic.json"}
+                   "source": "ncu dram__bytes_read.sum + dram__bytes_write.sum, profiles/r2z_traffic.json"}
     except Exception:
         pass
     roofline = {"bound": "hbm", "kernel": names[dom], "achieved": round(achieved, 1),

@@ -8,7 +8,7 @@ class; with it every class also gets algorithmic_bytes_per_launch and
 dram_over_algorithmic (> 1: bytes the model does not count -- 64-byte DRAM granules of
 random gathers, L2 write-backs; < 1: reuse through L2).
 Writes {class: {"launches", "dram_bytes_per_launch", "us_per_launch", "share"}}; bench.py
-reads profiles/r1_traffic.json to fill roofline.traffic for its dominant class.
+reads profiles/r2z_traffic.json to fill roofline.traffic for its dominant class.
 Classes follow bench.py / ddq_prepared_profile: dense (ws_kernel, every row),
 masked (ws_kernel over every row masked by a row bitmap), at-tids (ws_kernel over a
 TID list, fetch_kernel), agg, build, other.
