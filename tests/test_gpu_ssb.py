@@ -217,3 +217,30 @@ def test_fused_tail_both_algorithms(mode, monkeypatch):
             assert p.fetch().rows == _oracle(kind, q), (kind, q)
             p.close()
             assert db.run(ssb_plan(db, q, fuse_tail=True)).rows == _oracle(kind, q), (kind, q)
+
+
+def test_prepared_profile_classes_and_bytes():
+    """ddq_prepared_profile (the bench's roofline source): one entry per operator,
+    classes as include/ddq.h states -- builds 2, the dense first probe 0, Q3.1's
+    supplier probe masked by the customer probe's row bitmap 5 (O27: 20 % of the rows
+    survive), later probes / the fetch at TIDs 1, the aggregate 4 -- and the S8(d)
+    model bytes of a dense probe = one 4-byte key per row plus its output."""
+    from paper_conf_sigmod_bressft16_b200.ssb import ssb_plan
+    db = _db("1")
+    plan = ssb_plan(db, "ssb3.1")
+    p = db.prepare(plan, use_graph=True)
+    try:
+        p.launch()
+        want = [tuple(r) for r in p.fetch().rows]
+        prof = p.profile()
+        assert [tuple(r) for r in p.fetch().rows] == want  # the replay recomputes the same result
+    finally:
+        p.close()
+    assert want == _oracle("1", "ssb3.1")
+    classes = [c for _, _, c in prof]
+    assert classes[:3] == [2, 2, 2] and classes[3] == 0 and classes[4] == 5 and classes[-1] == 4
+    assert set(classes[5:-1]) == {1}
+    rows = _data("1").rows("lineorder")
+    ms0, by0, _ = prof[3]
+    assert ms0 > 0 and by0 >= rows * 4 and by0 <= rows * 4 * 1.25
+    assert all(ms > 0 and by > 0 for ms, by, c in prof if c != 2)
