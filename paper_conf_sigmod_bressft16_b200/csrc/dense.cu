@@ -308,9 +308,10 @@ __global__ void __launch_bounds__(ws_nw(kIn == 1) * 32, 1) ws_kernel(const __gri
             const uint32_t oo = min((uint32_t)(key[j] - P.key_min), P.range);
             const uint32_t cb = oo >> P.cg;
             hit = (s_bm[cb >> 5] >> (cb & 31)) & (oo < P.range ? 1u : 0u);
-          } else {
+          } else {  // bitmap in L2: a masked probe looks up its live rows only
             const uint32_t o = (uint32_t)(key[j] - P.key_min);
-            hit = o < P.range ? (__ldg(P.bitmap + (o >> 5)) >> (o & 31)) & 1u : 0u;
+            const bool look = o < P.range && (kIn != 2 || ((flags >> j) & 1u));
+            hit = look ? (__ldg(P.bitmap + (o >> 5)) >> (o & 31)) & 1u : 0u;
           }
           m |= hit << j;
         }

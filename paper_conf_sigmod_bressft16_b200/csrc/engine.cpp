@@ -1901,8 +1901,15 @@ ddq_status ddq_prepare(ddq_db* db, const ddq_plan* plan, int32_t use_graph, ddq_
         // producer no longer compacts 24 M TIDs through its ring (152 -> 84 us), and the
         // 4-stream step drops 2.67 -> 2.60 ms (Q3.1, Q4.2)
         ok = ok && c.kind == DDQ_OP_HASH_PROBE && c.fk_vec <= 0;
-        // ... whose table the masked probe keeps in shared memory (else TID lists)
-        if (ok && c.build >= 0 && c.build < plan->n_ops) {
+        // ... (round 2, final session) wherever its table lives: a masked probe of a
+        // join index in L2 looks up its live rows only (dense.cu), so the producer
+        // writes its bitmap at the kOutBits rate instead of compacting >= 1/8 of the
+        // rows into a TID list.  DDQ_MASKED_GLOBAL=0: only consumers whose table the
+        // masked probe stages in shared memory (the earlier rule; SF80-SF160 dims and
+        // SF100: customer's join index no longer fits one SM)
+        static const char* mg_env = getenv("DDQ_MASKED_GLOBAL");
+        const bool masked_global = !(mg_env && mg_env[0] == '0');
+        if (ok && !masked_global && c.build >= 0 && c.build < plan->n_ops) {
           const int64_t bt = build_tab[(size_t)c.build];
           const int64_t rows_c = db->tables[(size_t)c.table].n_rows;
           ok = bt >= 0 ? ws_masked_probe_smem(true, (uint32_t)bt, rows_c, c.emit_payload != 0)
