@@ -1109,6 +1109,7 @@ void ddq_close(ddq_db* db) {
     if (c->dev) cudaFreeAsync(c->dev, db->copy_stream);
     if (c->host) cudaFreeHost(c->host);
     if (c->host_packed) cudaFreeHost(c->host_packed);
+    if (c->host_tdict) cudaFreeHost(c->host_tdict);
   }
   for (auto& kv : db->cache_free) cudaFreeAsync(kv.second, db->copy_stream);
   db->cache_free.clear();
@@ -1160,6 +1161,57 @@ ddq_status ddq_load_column(ddq_db* db, ddq_table t, const char* name, ddq_type t
     const uint64_t range = (uint64_t)c->vmax - (uint64_t)c->vmin;
     int bits = 1;
     while (bits < 64 && (range >> bits) != 0) bits++;
+    // dictionary transfer code (ranks of the distinct values) when its packed stream
+    // plus the 8-byte dictionary is smaller: value ranges < 2^24 only (a presence
+    // bitmap and a rank table over the range)
+    std::vector<uint32_t> rank;
+    std::vector<int64_t> dict;
+    static const char* dict_env = getenv("DDQ_TRANSFER_DICT");  // "0": range code only (A/B)
+    if (bits <= 32 && bits < 8 * c->width && range < (1u << 24) && !(dict_env && dict_env[0] == '0')) {
+      const size_t pw = (size_t)(range >> 6) + 1;
+      const int np = (int)std::max<int64_t>(1, std::min<int64_t>(std::thread::hardware_concurrency(),
+                                                                  n_rows / (1 << 20)));
+      std::vector<std::vector<uint64_t>> part((size_t)np, std::vector<uint64_t>(pw, 0));
+      auto mark = [&](int t) {  // presence bitmap of rows [t*n/np, (t+1)*n/np)
+        uint64_t* pr = part[(size_t)t].data();
+        const int64_t b = n_rows * t / np, e = n_rows * (t + 1) / np;
+        for (int64_t i = b; i < e; i++) {
+          const int64_t v = c->width == 4 ? ((const int32_t*)host_data)[i] : ((const int64_t*)host_data)[i];
+          const uint64_t o = (uint64_t)(v - c->vmin);
+          pr[(size_t)(o >> 6)] |= 1ull << (o & 63);
+        }
+      };
+      {
+        std::vector<std::thread> th;
+        for (int t = 1; t < np; t++) th.emplace_back(mark, t);
+        mark(0);
+        for (auto& x : th) x.join();
+      }
+      std::vector<uint64_t>& present = part[0];
+      for (int t = 1; t < np; t++)
+        for (size_t w = 0; w < pw; w++) present[w] |= part[(size_t)t][w];
+      int64_t d = 0;
+      for (uint64_t w : present) d += __builtin_popcountll(w);
+      int dbits = 1;
+      while (dbits < 32 && ((uint64_t)(d - 1) >> dbits) != 0) dbits++;
+      if (packed_bytes(n_rows, dbits) + (size_t)d * 8 < packed_bytes(n_rows, bits)) {
+        rank.assign((size_t)range + 1, 0);
+        dict.reserve((size_t)d);
+        for (size_t w = 0; w < present.size(); w++)
+          for (uint64_t m = present[w]; m; m &= m - 1) {
+            const uint64_t o = (uint64_t)w * 64 + (uint64_t)__builtin_ctzll(m);
+            rank[(size_t)o] = (uint32_t)dict.size();
+            dict.push_back(c->vmin + (int64_t)o);
+          }
+        bits = dbits;
+      }
+    }
+    if (!dict.empty() && cudaHostAlloc((void**)&c->host_tdict, dict.size() * 8, cudaHostAllocPortable) != cudaSuccess)
+      dict.clear(), rank.clear(), bits = 64;  // no pinned room for the dictionary: raw copy
+    if (!dict.empty()) {
+      std::memcpy(c->host_tdict, dict.data(), dict.size() * 8);
+      c->tdict_n = (int64_t)dict.size();
+    }
     if (bits <= 32 && bits < 8 * c->width &&
         cudaHostAlloc(&c->host_packed, packed_bytes(n_rows, bits), cudaHostAllocPortable) == cudaSuccess) {
       uint32_t* dst = (uint32_t*)c->host_packed;
@@ -1170,6 +1222,7 @@ ddq_status ddq_load_column(ddq_db* db, ddq_table t, const char* name, ddq_type t
       const int nt = (int)std::max<int64_t>(1, std::min<int64_t>(chunks, std::thread::hardware_concurrency()));
       const int64_t vmin = c->vmin;
       const int width = c->width;
+      const uint32_t* rk = rank.empty() ? nullptr : rank.data();
       auto pack = [&](int t) {
         for (int64_t ch = t; ch < chunks; ch += nt) {
           const int64_t b = ch * per, e = std::min<int64_t>(n_rows, b + per);
@@ -1178,7 +1231,8 @@ ddq_status ddq_load_column(ddq_db* db, ddq_table t, const char* name, ddq_type t
           size_t w = (size_t)(b / 32) * (size_t)bits;
           for (int64_t i = b; i < e; i++) {
             const int64_t v = width == 4 ? ((const int32_t*)host_data)[i] : ((const int64_t*)host_data)[i];
-            acc |= ((uint64_t)v - (uint64_t)vmin) << have;
+            const uint64_t x = (uint64_t)v - (uint64_t)vmin;
+            acc |= (rk ? (uint64_t)rk[x] : x) << have;
             have += bits;
             if (have >= 32) {
               dst[w++] = (uint32_t)acc;
@@ -1194,6 +1248,10 @@ ddq_status ddq_load_column(ddq_db* db, ddq_table t, const char* name, ddq_type t
       pack(0);
       for (auto& x : th) x.join();
       c->tw = bits;
+    } else if (c->host_tdict) {  // no packed copy after all: the raw column goes
+      cudaFreeHost(c->host_tdict);
+      c->host_tdict = nullptr;
+      c->tdict_n = 0;
     }
   }
   db->cols.push_back(std::move(c));
@@ -1363,14 +1421,19 @@ ddq_status cache_column_locked(ddq_db* db, int c, bool on_demand, std::unique_lo
   col.loading = true;
   // packed transfer: stage the packed bytes in a pool block, widen into the column
   void* stage = nullptr;
-  const size_t pbytes = col.tw ? packed_bytes(col.n, col.tw) : 0;
+  const size_t sbytes = col.tw ? packed_bytes(col.n, col.tw) : 0;  // the stream, 16-byte multiple
+  const size_t dict_bytes = (size_t)col.tdict_n * 8;
+  const size_t pbytes = sbytes + dict_bytes;  // the dictionary travels behind the stream
   if (col.tw) stage = cache_block(db, pbytes);  // null: no room, send the raw column
   lk.unlock();
   uint64_t t0 = now_ns();
   uint64_t moved = 0;
   if (stage) {
-    e = cudaMemcpyAsync(stage, col.host_packed, pbytes, cudaMemcpyHostToDevice, db->copy_stream);
-    if (e == cudaSuccess) e = launch_unpack(stage, col.tw, col.vmin, p, col.width, col.n, db->copy_stream);
+    e = cudaMemcpyAsync(stage, col.host_packed, sbytes, cudaMemcpyHostToDevice, db->copy_stream);
+    void* ddict = dict_bytes ? (void*)((char*)stage + sbytes) : nullptr;
+    if (e == cudaSuccess && ddict)
+      e = cudaMemcpyAsync(ddict, col.host_tdict, dict_bytes, cudaMemcpyHostToDevice, db->copy_stream);
+    if (e == cudaSuccess) e = launch_unpack(stage, col.tw, col.vmin, p, col.width, col.n, db->copy_stream, ddict);
     moved = pbytes;
   } else {
     e = cudaMemcpyAsync(p, col.host, (size_t)col.n * col.width, cudaMemcpyHostToDevice, db->copy_stream);

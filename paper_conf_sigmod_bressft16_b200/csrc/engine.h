@@ -54,6 +54,11 @@ struct Column {
   void* host = nullptr;   // pinned host copy
   void* host_packed = nullptr;  // frame-of-reference bit-packed pinned copy (transfer.cu)
   int tw = 0;                   // its bits per value (1..32); 0 = none, the raw copy is sent
+  // dictionary transfer code: the packed values are ranks into this sorted pinned
+  // int64 array of the column's distinct values (sent with them), instead of
+  // value - vmin, when that is fewer bytes (e.g. yyyymmdd dates: 12 bits, not 17)
+  int64_t* host_tdict = nullptr;
+  int64_t tdict_n = 0;
   void* dev = nullptr;    // device cache copy or nullptr
   std::atomic<uint64_t> access{0};
   std::atomic<uint64_t> last_access{0};

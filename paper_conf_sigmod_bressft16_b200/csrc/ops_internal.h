@@ -27,7 +27,10 @@ FillHoist& fill_hoist();  // per host thread
 // bytes are rounded up to a multiple of 8 (every target allocation is padded)
 // cold-path transfer encoding (transfer.cu): frame-of-reference byte packing
 size_t packed_bytes(int64_t n, int tw);
-cudaError_t launch_unpack(const void* packed, int tw, int64_t base, void* out, int width, int64_t n, cudaStream_t st);
+// dict: null = frame of reference (value = base + code), else the sorted distinct
+// values (int64, device) the codes rank into
+cudaError_t launch_unpack(const void* packed, int tw, int64_t base, void* out, int width, int64_t n, cudaStream_t st,
+                          const void* dict = nullptr);
 cudaError_t init_fill(void* ptr, size_t bytes, uint64_t pattern, cudaStream_t st);
 cudaError_t launch_delay(uint64_t ns, cudaStream_t st);  // profiling: hold the stream
 bool ws_masked_probe_smem(bool join_index, uint32_t range_or_capacity, int64_t n_rows, bool pay);

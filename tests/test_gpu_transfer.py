@@ -2,7 +2,8 @@
 from its frame-of-reference bit-packed pinned copy is bit-identical to the raw
 column, for bit lengths 1..32 (every byte boundary and odd lengths), negative bases,
 widths 4 and 8, ragged lengths, and columns that stay raw (range >= 2^32); the bytes
-sent are the packed stream's."""
+sent are the packed stream's; columns with few distinct values in a wide range go
+as ranks into a sorted dictionary when that is smaller (dates)."""
 import numpy as np
 import pytest
 
@@ -44,12 +45,51 @@ def test_packed_cache_roundtrip(n, span, base, dtype):
         v[0], v[-1] = base, base + span
     got, moved = _roundtrip(v)
     assert got.dtype == v.dtype and np.array_equal(got, v)
-    width = v.dtype.itemsize
-    bits = max(1, (int(v.max()) - int(v.min())).bit_length())
-    if bits <= 32 and bits < 8 * width:  # the packed stream (+ <= 63 bytes of padding) went over the link
-        assert moved == (n * bits + 7) // 8 // 16 * 16 + 48
-    else:
-        assert moved == n * width
+    assert moved == _expected_moved(v)
+
+
+def _packed(n, bits):  # the packed stream's bytes (+ <= 63 bytes of padding)
+    return (n * bits + 7) // 8 // 16 * 16 + 48
+
+
+def _expected_moved(v):
+    """Bytes over the link: the raw column, the range code (value - vmin in the
+    range's bit length), or -- when smaller -- the dictionary code (ranks of the
+    distinct values in their bit length, plus the 8-byte sorted dictionary; value
+    ranges < 2^24)."""
+    n, width = len(v), v.dtype.itemsize
+    span = int(v.max()) - int(v.min())
+    bits = max(1, span.bit_length())
+    if not (bits <= 32 and bits < 8 * width):
+        return n * width
+    best = _packed(n, bits)
+    if span < (1 << 24):
+        d = len(np.unique(v))
+        dbits = max(1, (d - 1).bit_length())
+        if _packed(n, dbits) + 8 * d < best:
+            best = _packed(n, dbits) + 8 * d
+    return best
+
+
+@pytest.mark.parametrize("dtype", [np.int32, np.int64])
+@pytest.mark.parametrize("n", [5000, 1_000_003])
+def test_dictionary_transfer_code(n, dtype):
+    """yyyymmdd dates (2556 distinct days over a 69 129-wide range): 12-bit ranks into
+    a sorted dictionary instead of a 17-bit range code, bit-identical after the cache;
+    and a sparse domain (every 1000th value of 10^7) likewise."""
+    import datetime
+    days = np.array([int((datetime.date(1992, 1, 1) + datetime.timedelta(d)).strftime("%Y%m%d"))
+                     for d in range(2556)], dtype=np.int64)
+    rng = np.random.default_rng(n)
+    for dom in (days, np.arange(0, 10_000_000, 1000, dtype=np.int64)):
+        v = dom[rng.integers(0, len(dom), size=n)].astype(dtype)
+        v[0], v[-1] = dom[0], dom[-1]
+        got, moved = _roundtrip(v)
+        assert np.array_equal(got, v)
+        d = len(np.unique(v))
+        if n > 100_000:  # large enough that the dictionary pays
+            assert moved == _packed(n, max(1, (d - 1).bit_length())) + 8 * d
+        assert moved == _expected_moved(v)
 
 
 def test_packing_off_sends_raw():
