@@ -466,8 +466,12 @@ def main():
     # measured DRAM traffic per launch of this kernel class: ncu launch list of the
     # bench command (tools/ncu_traffic.py -> profiles/r2z_traffic.json)
     traffic = None
+    try:  # per class: ncu DRAM bytes / ncu device time of the same kernels (64-byte gather granules included)
+        trc = json.load(open(os.path.join(ROOT, "profiles", "r2z_traffic.json")))["classes"]
+    except Exception:
+        trc = {}
     try:
-        tr = json.load(open(os.path.join(ROOT, "profiles", "r2z_traffic.json")))["classes"][tclass[dom]]
+        tr = trc[tclass[dom]]
         traffic = {"dram_bytes_per_launch": tr["dram_bytes_per_launch"],
                    "algorithmic_bytes_per_launch": round(cls_bytes[dom] / cls_n[dom]),
                    "source": "ncu dram__bytes_read.sum + dram__bytes_write.sum, profiles/r2z_traffic.json"}
@@ -480,10 +484,16 @@ def main():
                 "step_model_gb": round(step_bytes / 1e9, 3),
                 "step_gbs": round(step_bytes / (ms_per_step / 1e3) / 1e9 * ws, 1),
                 # every kernel class of the step, same event-timed replay and byte model
-                "classes": {tclass[c]: {"launches_per_step": cls_n[c], "us_per_step": round(cls_ms[c] * 1e3, 1),
-                                        "achieved_gbs": round(cls_bytes[c] / (cls_ms[c] / 1e3) / 1e9, 1),
-                                        "frac": round(cls_bytes[c] / (cls_ms[c] / 1e3) / 1e9 / hbm_peak, 4),
-                                        "share_of_step": round(cls_ms[c] / sum(cls_ms.values()), 3)}
+                "classes": {tclass[c]: dict({"launches_per_step": cls_n[c], "us_per_step": round(cls_ms[c] * 1e3, 1),
+                                             "achieved_gbs": round(cls_bytes[c] / (cls_ms[c] / 1e3) / 1e9, 1),
+                                             "frac": round(cls_bytes[c] / (cls_ms[c] / 1e3) / 1e9 / hbm_peak, 4),
+                                             "share_of_step": round(cls_ms[c] / sum(cls_ms.values()), 3)},
+                                            **({"ncu_dram_gbs": round(trc[tclass[c]]["dram_bytes_per_launch"]
+                                                                      / trc[tclass[c]]["us_per_launch"] / 1e3, 1),
+                                                "ncu_dram_frac": round(trc[tclass[c]]["dram_bytes_per_launch"]
+                                                                       / trc[tclass[c]]["us_per_launch"] / 1e3
+                                                                       / hbm_peak, 3)}
+                                               if tclass[c] in trc else {}))
                             for c in sorted(cls_ms, key=lambda c: -cls_ms[c]) if cls_ms[c] > 0}}
 
     # ---- e2e through the public API with host buffers: cold cache, every column
