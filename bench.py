@@ -499,39 +499,67 @@ def main():
     # ---- e2e through the public API with host buffers: cold cache, every column
     #      H2D from pinned host memory inside the timed region (GPU-only placement)
     e2e = None
-    if not args.no_e2e and ws == 1:
+    e2e_results = None
+    if not args.no_e2e:
         cold = Database(device=local, cache_bytes=64 << 30, heap_bytes=heap, placement=A.PLACE_GPU_ONLY,
                         prefetch=not args.no_prefetch)
         load_ssb(cold, shard, row_begin=b, row_end=e, cache=False, presliced=True)
         plans = [ssb_plan(cold, q) for q in SSB_QUERIES]
         all_cols = [(t, c) for (t, c) in cold._cols]
 
+        from paper_conf_sigmod_bressft16_b200.dist import merge_finalized
+        roots = [pl.plan.ops[pl.n - 1] for pl in plans]
+
         def e2e_step():  # the 13 queries submitted at once (the paper's parallel users)
             qs = [cold.submit(pl) for pl in plans]
-            for q in qs:
-                cold.fetch(q)
+            res = [cold.fetch(q) for q in qs]
             for (t, c) in all_cols:
                 cold.evict(t, c)
+            if ws == 1:
+                return {q: r.rows for q, r in zip(SSB_QUERIES, res)}
+            # N > 1: every rank's finalised results to rank 0, merged exactly there
+            import torch.distributed as dist
+            gathered = [None] * ws
+            dist.all_gather_object(gathered, [r.rows for r in res])
+            if rank != 0:
+                return None
+            return {q: merge_finalized(roots[i], [g[i] for g in gathered]).rows for i, q in enumerate(SSB_QUERIES)}
         for _ in range(2):  # first cold steps pay one-time driver / allocator set-up
             e2e_step()
         cold.reset_stats()
+        if ws > 1:
+            import torch.distributed as dist
+            dist.barrier()
         t0 = time.perf_counter()
         step_ms = []
         for _ in range(args.e2e_steps):
             ts = time.perf_counter()
-            e2e_step()
+            e2e_results = e2e_step()
             step_ms.append(round(1e3 * (time.perf_counter() - ts), 1))
         dt = time.perf_counter() - t0
         st = cold.stats()
+        h2d, d2h = st["h2d_bytes"], st["d2h_bytes"]
+        if ws > 1:  # the whole job: the slowest rank's time, every rank's bytes
+            import torch.distributed as dist
+            mx = torch.tensor([dt], dtype=torch.float64, device="cuda")
+            sm = torch.tensor([float(h2d), float(d2h)], dtype=torch.float64, device="cuda")
+            dist.all_reduce(mx, op=dist.ReduceOp.MAX)
+            dist.all_reduce(sm, op=dist.ReduceOp.SUM)
+            dt, h2d, d2h = float(mx[0]), int(sm[0]), int(sm[1])
         e2e = {"value": total_rows * args.e2e_steps / dt, "unit": UNIT,
-               "h2d_bytes_per_step": st["h2d_bytes"] // args.e2e_steps,
-               "d2h_bytes_per_step": st["d2h_bytes"] // args.e2e_steps,
-               "h2d_gbs": round(st["h2d_bytes"] / dt / 1e9, 2), "step_ms": step_ms,
+               "h2d_bytes_per_step": h2d // args.e2e_steps,
+               "d2h_bytes_per_step": d2h // args.e2e_steps,
+               "h2d_gbs": round(h2d / dt / 1e9, 2), "step_ms": step_ms,
                "path": "ddq_submit (13 queries at once) / ddq_fetch, GPU-only placement, empty cache; "
                        "columns copied from pinned host memory (cold cache, P:32)" +
                        ("; streamed cold path: the plans' columns stream in from submit while earlier "
-                        "operators compute (prefetch, N1)" if not args.no_prefetch else "; on demand")}
+                        "operators compute (prefetch, N1)" if not args.no_prefetch else "; on demand") +
+                       ("; N > 1: every rank its own rows, finalised results all-gathered to rank 0 and "
+                        "merged exactly (dist.merge_finalized); time = slowest rank" if ws > 1 else "")}
         cold.close()
+        if args.dump_results and rank == 0 and e2e_results is not None:
+            with open(args.dump_results + ".e2e.json", "w") as f:
+                json.dump({q: [list(r) for r in rows] for q, rows in e2e_results.items()}, f)
 
     cpu = None
     if rank == 0 and not args.no_cpu_baseline:

@@ -54,3 +54,38 @@ def all_gather_packed(packed, world: int):
     out = torch.empty(world * packed.numel(), dtype=packed.dtype, device=packed.device)
     dist.all_gather_into_tensor(out, packed)
     return out
+
+
+def merge_finalized(root, rows_per_rank) -> "object":
+    """Exact merge of one query's FINALISED results from several shards (the N > 1
+    end-to-end path, where every rank runs ``ddq_submit`` / ``ddq_fetch`` on its own
+    rows): each row's group keys are re-packed into the root AGGREGATE's key layout
+    (key k at the sum of the earlier keys' bit lengths; 21 bits where the plan gives
+    none, as libddq packs them), its integer aggregates split into int128 words, and
+    libddq's host finalisation merges equal keys (SUM / COUNT add, MIN takes the
+    minimum) and applies ORDER BY / LIMIT.  A shard's SQL-NULL row (an ungrouped
+    aggregate over no rows, reading O7) contributes nothing.  Valid for aggregates
+    that merge (SUM / COUNT / MIN) without AVG columns -- every SSB query."""
+    from .engine import finalize_partials
+    nk, na = int(root.n_keys), int(root.n_aggs)
+    bits = [int(root.key_bits[k]) if int(root.key_bits[k]) > 0 else 21 for k in range(nk)]
+    keys, lo, hi = [], [], []
+    for rows in rows_per_rank:
+        for r in rows:
+            vals = r[nk:nk + na]
+            if any(v is None for v in vals):
+                continue
+            p, sh = 0, 0
+            for k in range(nk):
+                p |= int(r[k]) << sh
+                sh += bits[k]
+            keys.append(p)
+            for v in vals:
+                v = int(v)
+                lo.append(v & 0xFFFFFFFFFFFFFFFF)
+                hi.append(v >> 64)
+    accs = np.empty(2 * len(lo), np.int64)
+    if lo:
+        accs[0::2] = np.array(lo, np.uint64).view(np.int64)
+        accs[1::2] = np.array(hi, np.int64)
+    return finalize_partials(root, np.array(keys, np.int64), accs)

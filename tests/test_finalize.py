@@ -158,3 +158,22 @@ def test_merge_is_partition_invariant():
         got = finalize_partials(root, keys, accs).rows
         assert got == want
     check()
+
+
+def test_merge_finalized_shard_results():
+    """dist.merge_finalized (bench.py's N > 1 end-to-end merge of ddq_fetch results):
+    shard rows with unpacked keys re-pack into the root's key layout (here 2 keys of
+    5 and 21 default bits) and merge exactly -- equal keys add (beyond int64), the
+    ORDER BY of the root holds (key 1 asc, then SUM desc), and a shard's SQL-NULL
+    row of an empty ungrouped aggregate is dropped (O7)."""
+    from paper_conf_sigmod_bressft16_b200 import _abi as A
+    from paper_conf_sigmod_bressft16_b200.dist import merge_finalized
+    root = _root([A.AGG_SUM, A.AGG_COUNT], n_keys=2, key_bits=[5, 0], order_by=[1, -101])
+    big = 1 << 70
+    shard0 = [(3, 1_000_000, big, 2), (1, 7, -5, 1)]
+    shard1 = [(3, 1_000_000, big + 1, 3), (3, 9, 4, 1), (1, 7, 6, 2)]
+    got = merge_finalized(root, [shard0, shard1]).rows
+    assert got == [(1, 7, 1, 3), (3, 1_000_000, 2 * big + 1, 5), (3, 9, 4, 1)]
+    ungrouped = _root([A.AGG_SUM, A.AGG_COUNT])
+    assert merge_finalized(ungrouped, [[(None, 0)], [(10, 2)]]).rows == [(10, 2)]
+    assert merge_finalized(ungrouped, [[(None, 0)], [(None, 0)]]).rows == [(None, 0)]
