@@ -498,6 +498,13 @@ def main():
 
     # ---- e2e through the public API with host buffers: cold cache, every column
     #      H2D from pinned host memory inside the timed region (GPU-only placement)
+    # the hot database is done: free its cache and heap before the cold one opens
+    # (at SF100 both would not fit one GPU)
+    for p in preps:
+        p.close()
+    db.close()
+    torch.cuda.synchronize()
+
     e2e = None
     e2e_results = None
     if not args.no_e2e:
@@ -587,9 +594,6 @@ def main():
                 "setup_s": round(setup_s, 1),
                 "checks": {q: len(r) for q, r in results.items()}}
         print(json.dumps(line), flush=True)
-    for p in preps:
-        p.close()
-    db.close()
     if ws > 1:
         import torch.distributed as dist
         dist.destroy_process_group()
