@@ -371,6 +371,18 @@ __global__ void __launch_bounds__(ws_nw(kIn == 1) * 32, 1) ws_kernel(const __gri
 #pragma unroll
       for (int j = 0; j < WS_ITEMS; j++) m |= (vec_cmp(P.eq_cmp, a[j], b[j]) ? 1u : 0u) << j;
       flags &= m;
+    } else if (kIn == 0) {  // dense selection (row bitmap output): the one int32 column streamed
+      const WsPred& pr = P.preds[0];
+      uint32_t m = 0;
+      if (kKind == WK_SEL_RANGE) {
+#pragma unroll
+        for (int j = 0; j < WS_ITEMS; j++) m |= ((uint64_t)((int64_t)sv[j] - pr.lo) <= pr.d64 ? 1u : 0u) << j;
+        if (pr.empty) m = 0;
+      } else {
+#pragma unroll
+        for (int j = 0; j < WS_ITEMS; j++) m |= (pred_generic(pr, (int64_t)sv[j]) ? 1u : 0u) << j;
+      }
+      flags &= m;
     } else {  // selection at TIDs: later columns gathered for the remaining rows only
       for (int p = 0; p < P.n_preds; p++) {
         const WsPred& pr = P.preds[p];
@@ -598,6 +610,8 @@ void ws_attr_kind() {
     ws_attr<K, 0, true, false, false>();
     ws_attr<K, 0, false, false, true>();
   }
+  if constexpr (K == WK_SEL_RANGE || K == WK_SEL_GENERIC)  // dense selection -> row bitmap
+    ws_attr<K, 0, false, false, true>();
   ws_attr<K, 1, false, false, false>();
   ws_attr<K, 1, false, true, false>();
   if constexpr (kProbe) {
@@ -631,6 +645,12 @@ void launch_k(int in, bool pay, bool carry, bool obits, int grid, size_t smem, c
       return;
     }
   }
+  if constexpr (K == WK_SEL_RANGE || K == WK_SEL_GENERIC) {
+    if (in == 0) {  // a dense selection writes a row bitmap (ws_supported)
+      ws_kernel<K, 0, false, false, true><<<grid, dim3(ws_nw(false) * 32), smem, st>>>(p);
+      return;
+    }
+  }
   const dim3 blk(ws_nw(true) * 32);
   if constexpr (kProbe) {
     if (pay) {
@@ -648,13 +668,19 @@ void launch_k(int in, bool pay, bool carry, bool obits, int grid, size_t smem, c
 bool ws_supported(const FilterArgs& a) {
   const bool tids = a.in_tids != nullptr;
   if (a.n_carry > 4 || a.n_cap > (int64_t)0x7FFFFFFF) return false;
-  if (a.out_bits && (a.in_tids || a.in_bits || !a.probe || a.out_payload)) return false;
+  if (a.out_bits && (a.in_tids || a.in_bits || a.out_payload)) return false;
   if (a.in_bits) {  // row bitmap input: probes of a key column (streamed), no vectors
     if (!a.probe || a.fk_by_pos || a.eq_a || a.n_carry || ((uintptr_t)a.in_bits & 15) != 0) return false;
     if (((uintptr_t)a.fk & 15) != 0) return false;
-  } else if (!tids) {  // dense: probes only (dense selections stream several columns: scan.cu)
-    if (!a.probe || a.fk_by_pos || a.eq_a || a.n_carry) return false;
-    if (((uintptr_t)a.fk & 15) != 0) return false;
+  } else if (!tids) {  // dense: probes, or ONE int32 predicate column into a row bitmap (O27);
+                       // other dense selections stream several columns: scan.cu
+    if (!a.probe) {
+      if (!a.out_bits || a.n_preds != 1 || a.preds[0].width != 4 || a.eq_a || a.n_carry) return false;
+      if (((uintptr_t)a.preds[0].col & 15) != 0) return false;
+    } else {
+      if (a.fk_by_pos || a.eq_a || a.n_carry) return false;
+      if (((uintptr_t)a.fk & 15) != 0) return false;
+    }
   } else {
     if (((uintptr_t)a.in_tids & 15) != 0) return false;
     if (a.probe && a.fk_by_pos && ((uintptr_t)a.fk & 15) != 0) return false;
@@ -787,6 +813,7 @@ cudaError_t launch_ws(const FilterArgs& a, cudaStream_t st) {
       all_range = all_range && d.kind == DDQ_PRED_RANGE;
     }
     kind = all_range ? WK_SEL_RANGE : WK_SEL_GENERIC;
+    if (in == 0) p.fk = reinterpret_cast<const int32_t*>(a.preds[0].col);  // dense: the column streamed
   }
   // ring: 4 blocks.  More blocks would put more flushes in flight (ncu: a quarter
   // of a 100 %-pass late-fetch probe's instructions spin on a free slot), but

@@ -286,7 +286,9 @@ ddq_status run_gpu_op(GpuOpCtx& ctx, const ddq_op& op, Inter& out) {
           cin.push_back((const int32_t*)v.ptr);
         }
       }
-      const bool obits = ctx.bits_out && !in && probe && !op.emit_payload;
+      // a row-bitmap output (O27): a dense semi-join probe, or a dense selection on one
+      // int32 column (ws_kernel streams it; ddq_prepare decides, see bits_out)
+      const bool obits = ctx.bits_out && !in && ((probe && !op.emit_payload) || (!probe && op.n_preds == 1));
       out.cap = obits ? T.n_rows : out_cap;
       if (obits) out.bits = (uint32_t*)A.get(row_bitmap_bytes(T.n_rows));
       else out.tids = (int32_t*)A.get((uint64_t)std::max<int64_t>(out_cap, 1) * 4);
@@ -1952,7 +1954,11 @@ ddq_status ddq_prepare(ddq_db* db, const ddq_plan* plan, int32_t use_graph, ddq_
     const bool allow = !env || env[0] != '0';
     for (int i = 0; i < plan->n_ops && allow; i++) {
       const ddq_op& op = plan->ops[i];
-      if (op.kind != DDQ_OP_HASH_PROBE || op.input >= 0 || op.emit_payload || op.fk_vec > 0) continue;
+      const bool sel1 = op.kind == DDQ_OP_SELECT && op.input < 0 && op.n_preds == 1 && [&] {
+        const Column* c = col_of(db, op.preds[0].column);
+        return c && c->width == 4;
+      }();  // a dense selection on one int32 column (TPC-H Q3's l_shipdate)
+      if (!sel1 && (op.kind != DDQ_OP_HASH_PROBE || op.input >= 0 || op.emit_payload || op.fk_vec > 0)) continue;
       int consumers = 0;
       bool ok = true;
       for (int j = i + 1; j < plan->n_ops; j++) {
