@@ -65,10 +65,13 @@ def load_tpch(db: Database, data, cache: bool = True, tables=None) -> None:
             db.set_dictionary(t, c, db.dicts[d])  # decode result keys (S8(a7))
 
 
-def tpch_plan(db: Database, q: str, limit: int = 0, dense: bool = True) -> PlanBuilder:
+def tpch_plan(db: Database, q: str, limit: int = 0, dense: bool = True, fused_agg: bool = True) -> PlanBuilder:
     """dense (Q1): one AGGREGATE over every lineitem row with the shipdate predicate
     fused (agg_dense_small_kernel, reading O26); False: select -> TID list ->
-    aggregate at the TIDs (the paper's operator granularity, kept under test)."""
+    aggregate at the TIDs (the paper's operator granularity, kept under test).
+    fused_agg (Q6): the discount / quantity predicates evaluated inside the
+    aggregation at the shipdate selection's TIDs (reading O26, as SSB flight 1:
+    SF30 0.50 -> see DESIGN.md); False: two selections at TIDs feed it."""
     P = db.plan()
     li = "lineitem"
     if q == "tpch1":
@@ -88,10 +91,14 @@ def tpch_plan(db: Database, q: str, limit: int = 0, dense: bool = True) -> PlanB
     if q == "tpch6":
         # shipdate in 1994 (15 %) first; discount 0.05..0.07 and quantity < 24 at its TIDs
         t = P.select(li, [("l_shipdate", 19940101, 19941231)])
-        t = P.select(li, [("l_discount", 5, 7)], input=t)
-        t = P.select(li, [("l_quantity", -2**62, 2399)], input=t)
-        P.aggregate(li, t, keys=[], aggs=[(A.AGG_SUM_MUL, ["l_extendedprice", "l_discount"]),
-                                          (A.AGG_COUNT, [])], max_groups=1)
+        rest = [("l_discount", 5, 7), ("l_quantity", -2**62, 2399)]
+        aggs = [(A.AGG_SUM_MUL, ["l_extendedprice", "l_discount"]), (A.AGG_COUNT, [])]
+        if fused_agg:  # fused into the aggregate (O26, as SSB flight 1)
+            P.aggregate(li, t, keys=[], aggs=aggs, max_groups=1, where=rest)
+            return P
+        t = P.select(li, rest[:1], input=t)
+        t = P.select(li, rest[1:], input=t)
+        P.aggregate(li, t, keys=[], aggs=aggs, max_groups=1)
         return P
     if q == "tpch2":
         # The correlated scalar subquery ps_supplycost = (select min(ps_supplycost) ..
