@@ -69,9 +69,10 @@ def tpch_plan(db: Database, q: str, limit: int = 0, dense: bool = True, fused_ag
     """dense (Q1): one AGGREGATE over every lineitem row with the shipdate predicate
     fused (agg_dense_small_kernel, reading O26); False: select -> TID list ->
     aggregate at the TIDs (the paper's operator granularity, kept under test).
-    fused_agg (Q6): the discount / quantity predicates evaluated inside the
-    aggregation at the shipdate selection's TIDs (reading O26, as SSB flight 1:
-    SF30 0.50 -> see DESIGN.md); False: two selections at TIDs feed it."""
+    fused_agg: Q6's discount / quantity predicates evaluated inside the aggregation
+    at the shipdate selection's TIDs (reading O26, as SSB flight 1), and Q5's supplier
+    semi-join first with s_nationkey fetched late; False: the chains kept under test
+    (two selections at TIDs; orders first)."""
     P = db.plan()
     li = "lineitem"
     if q == "tpch1":
@@ -175,8 +176,16 @@ def tpch_plan(db: Database, q: str, limit: int = 0, dense: bool = True, fused_ag
         hc = P.build("customer", "c_custkey", "c_nationkey")
         o = P.select("orders", [("o_orderdate", 19940101, 19941231)])
         ho = P.build("orders", "o_orderkey", "o_custkey", input=o)
-        t = P.probe(li, "l_orderkey", ho, emit=True)                     # vec0 = o_custkey
-        t = P.probe(li, "l_suppkey", hs, input=t, emit=True)             # vec1 = s_nationkey
+        if fused_agg:
+            # the ASIA suppliers' semi-join first (20 % of lineitem: a row bitmap, O27),
+            # the 1994 orders probed masked by it, s_nationkey fetched late at the
+            # survivors (join order and late materialisation, O23)
+            t = P.probe(li, "l_suppkey", hs)                                 # semi-join
+            t = P.probe(li, "l_orderkey", ho, input=t, emit=True)            # vec0 = o_custkey
+            t = P.fetch(li, "l_suppkey", hs, input=t)                        # vec1 = s_nationkey
+        else:
+            t = P.probe(li, "l_orderkey", ho, emit=True)                     # vec0 = o_custkey
+            t = P.probe(li, "l_suppkey", hs, input=t, emit=True)             # vec1 = s_nationkey
         t = P.probe(li, 0, hc, input=t, emit=True)                       # vec2 = c_nationkey
         t = P.filter_eq(li, t, 1, 2)                                     # c_nationkey = s_nationkey
         t = P.probe(li, 1, hn, input=t, emit=True)                       # vec3 = n_name

@@ -44,18 +44,21 @@ def test_tpch_prepared_equals_oracle(q):
     assert got and got == _want(q)
 
 
+@pytest.mark.parametrize("q", ["tpch5", "tpch6"])
 @pytest.mark.parametrize("fused", [True, False])
-def test_tpch6_fused_and_chained_selection_equal_oracle(fused):
-    """Q6's discount / quantity predicates inside the aggregation (O26) or as two
-    selections at TIDs: same result, prepared and through the driver."""
+def test_tpch_plan_forms_equal_oracle(q, fused):
+    """Both plan forms = oracle, prepared and through the driver: Q6's discount /
+    quantity predicates inside the aggregation (O26) or as two selections at TIDs;
+    Q5's supplier semi-join first (a row bitmap) with s_nationkey fetched late, or
+    orders first."""
     from paper_conf_sigmod_bressft16_b200.tpch import tpch_plan
     db = _db()
-    p = db.prepare(tpch_plan(db, "tpch6", fused_agg=fused))
+    p = db.prepare(tpch_plan(db, q, fused_agg=fused))
     p.launch()
     got = p.fetch().rows
     p.close()
-    assert got == _want("tpch6")
-    assert db.run(tpch_plan(db, "tpch6", fused_agg=fused)).rows == _want("tpch6")
+    assert got == _want(q)
+    assert db.run(tpch_plan(db, q, fused_agg=fused)).rows == _want(q)
 
 
 @pytest.mark.parametrize("q", ["tpch1", "tpch2", "tpch3", "tpch4", "tpch5", "tpch6", "tpch7"])
